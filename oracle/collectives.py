@@ -1,0 +1,171 @@
+"""Collective semantics under a strategy and a ready mask -- TEST INFRASTRUCTURE ONLY.
+
+Ranks are simulated: ``xs[r]`` is rank r's 1-D send tensor (numpy), ``None``
+allowed for a non-ready rank (its tensor is never read, reading Q11).
+dtypes: 'f32' (np.float32), 'bf16' (np.uint16 bit patterns, see oracle.bf16),
+'i32' (np.int32).
+
+AllReduce has two definitions here:
+  * ``allreduce`` replays the strategy's reduction order exactly (DESIGN.md
+    §3 c-2): per tree, bottom-up behaviour tuples, every kernel
+    node folds its own tensor (if ready) then its children's flows in
+    ascending rank order, in the working precision (fp32 adds; bf16 widened to
+    fp32 and rounded once per kernel node with RNE, Q6; int32 wraps, Q15); the
+    root's result is broadcast to ALL ranks, relays included (Q4,
+    "execute Broadcast reversely" P:L165).
+  * ``allreduce_exact`` is the plain definition y = sum_{r in R} x_r in fp64
+    ("aggregated tensor"), used to bound the replay's rounding.
+AllGather ("one Broadcast on each GPU") and AlltoAll (P:L169,
+P:L209-211) move bytes only; their oracle is the plain index definition and
+the strategy can only be validated, not change the result (Q12 for masks).
+"""
+
+import numpy as np
+
+from . import bf16 as _bf
+from .strategy import parse, partition, ESIZE
+from .tuples import behavior
+
+_NP = {"f32": np.float32, "bf16": np.uint16, "i32": np.int32}
+
+
+def _fold(terms, dtype):
+    """Left-to-right fold of >= 2 equal-length arrays in the working precision."""
+    if dtype == "f32":
+        acc = terms[0].astype(np.float32, copy=True)
+        for t in terms[1:]:
+            acc = acc + t                     # one IEEE fp32 RNE add per element
+        return acc
+    if dtype == "bf16":
+        acc = _bf.to_f32(terms[0])
+        for t in terms[1:]:
+            acc = acc + _bf.to_f32(t)         # fp32 accumulation
+        return _bf.from_f32_rne(acc)          # one rounding per kernel node
+    if dtype == "i32":
+        acc = terms[0].astype(np.int64)
+        for t in terms[1:]:
+            acc = (acc + t.astype(np.int64)) & 0xFFFFFFFF   # mod 2^32
+        return acc.astype(np.uint32).view(np.int32)
+    raise ValueError(dtype)
+
+
+def _accumulate(prev, res, dtype):
+    """recvbuf += result with one rounding (flag ACCUMULATE, phase 2)."""
+    return _fold([prev, res], dtype)
+
+
+def _zero(k, dtype):
+    return np.zeros(k, dtype=_NP[dtype])       # +0 bits for every dtype (Q7)
+
+
+def allreduce(xs, strategy_text, ready, dtype, accumulate=False, y_prev=None):
+    """Replay AllReduce along the strategy; returns a list of n arrays.
+
+    xs           : list of n arrays (None for non-ready ranks) of equal length.
+    ready        : iterable of ready ranks R.
+    accumulate   : y_g <- y_prev_g + result (phase 2); y_prev required.
+    """
+    st = parse(strategy_text)
+    if st.collective != "allreduce":
+        raise ValueError("strategy is not an allreduce strategy")
+    n = st.nranks
+    ready = set(ready)
+    lens = {len(x) for x in xs if x is not None}
+    if y_prev is not None:
+        lens |= {len(y) for y in y_prev}
+    assert len(lens) == 1, "all tensors must have the same length"
+    count = lens.pop()
+    if accumulate:
+        ys = [np.array(y_prev[g], dtype=_NP[dtype], copy=True) for g in range(n)]
+    else:
+        ys = [np.empty(count, dtype=_NP[dtype]) for _ in range(n)]
+    bounds = partition(count, ESIZE[dtype], [s.weight for s in st.subs])
+    for m, sub in enumerate(st.subs):
+        lo, hi = bounds[m], bounds[m + 1]
+        if lo == hi:
+            continue
+        tup, flows = behavior(sub.parent, ready, sub.noagg)
+        agg_val = {}
+
+        def value(f):
+            kind, r = f
+            return xs[r][lo:hi] if kind == "in" else agg_val[r]
+
+        # post-order evaluation of the kernel nodes
+        order = []
+
+        def visit(g):
+            for c in sub.children(g):
+                visit(c)
+            order.append(g)
+
+        visit(sub.root)
+        for g in order:
+            if tup[g][2]:
+                terms = [xs[g][lo:hi]] if tup[g][0] else []
+                for c in sub.children(g):
+                    if tup[c][3]:
+                        terms += [value(f) for f in flows[c]]
+                agg_val[g] = _fold(terms, dtype)
+        root = sub.root
+        if tup[root][2]:
+            res = agg_val[root]
+        else:
+            fl = flows[root]
+            assert len(fl) <= 1, "a non-kernel root emits at most one flow"
+            res = np.array(value(fl[0]), copy=True) if fl else None
+        for g in range(n):
+            if accumulate:
+                if res is not None:
+                    ys[g][lo:hi] = _accumulate(ys[g][lo:hi], res, dtype)
+            else:
+                ys[g][lo:hi] = res if res is not None else _zero(hi - lo, dtype)
+    return ys
+
+
+def allreduce_exact(xs, ready, dtype, count=None):
+    """Plain definition: sum over ready ranks, fp64 for floats, mod 2^32 for int32.
+
+    Returns float64 (f32/bf16) or int32 (i32) array.
+    """
+    ready = sorted(set(ready))
+    if not ready:
+        return np.zeros(count, dtype=np.float64 if dtype != "i32" else np.int32)
+    if dtype == "i32":
+        tot = np.zeros(len(xs[ready[0]]), dtype=np.int64)   # |sum| < 64 * 2^31: exact
+        for r in ready:
+            tot = tot + xs[r].astype(np.int64)
+        return (tot & 0xFFFFFFFF).astype(np.uint32).view(np.int32)
+    vals = [(_bf.to_f32(xs[r]) if dtype == "bf16" else xs[r]).astype(np.float64)
+            for r in ready]
+    return np.sum(np.stack(vals), axis=0)
+
+
+def allgather(xs, strategy_text, ready, dtype, y_prev):
+    """y_g[s*cnt:(s+1)*cnt] = x_s for every g and every ready s; other slots
+    untouched (Q12).  y_prev: list of n arrays of n*cnt elements."""
+    st = parse(strategy_text)
+    if st.collective != "allgather":
+        raise ValueError("strategy is not an allgather strategy")
+    n = st.nranks
+    ys = [np.array(y_prev[g], copy=True) for g in range(n)]
+    for s in sorted(set(ready)):
+        cnt = len(xs[s])
+        for g in range(n):
+            ys[g][s * cnt:(s + 1) * cnt] = xs[s]
+    return ys
+
+
+def alltoall(xs, strategy_text, ready, dtype, y_prev):
+    """y_d[s*cnt:(s+1)*cnt] = x_s[d*cnt:(d+1)*cnt] for every d and ready s
+    (including s == d); blocks from non-ready sources untouched (Q12)."""
+    st = parse(strategy_text)
+    if st.collective != "alltoall":
+        raise ValueError("strategy is not an alltoall strategy")
+    n = st.nranks
+    ys = [np.array(y_prev[g], copy=True) for g in range(n)]
+    for s in sorted(set(ready)):
+        cnt = len(xs[s]) // n
+        for d in range(n):
+            ys[d][s * cnt:(s + 1) * cnt] = xs[s][d * cnt:(d + 1) * cnt]
+    return ys

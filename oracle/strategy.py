@@ -1,0 +1,246 @@
+"""Strategy text v1: parser, validator, ring expansion, partition, chunking.
+
+TEST INFRASTRUCTURE ONLY (see oracle/__init__.py).  Independent of the C++
+loader in paper_conf_icdcs_zhaozw24_b200/csrc/strategy.cpp; both follow the
+format specification in DESIGN.md §2.
+
+The paper's strategy is "M parallel sub-collectives", each with its own
+communication graph, a data partition S_m with sum S_m = S and a chunk size
+C_m (§IV-D, Fig. 8); aggregation flags a_{m,g}
+(P:L184); the paper serialises strategies as XML whose schema it does not give
+(P:L233), so the text format here is our own.
+
+Format (one directive per line, '#' starts a comment):
+
+    adapcc-strategy 1
+    nranks <n>                                  1 <= n <= 64
+    collective allreduce|allgather|alltoall
+    tree  weight=<w> chunk=<C> parent=<p_0,..,p_{n-1}> [noagg=<g,..>]   (allreduce)
+    ring  weight=<w> chunk=<C> order=<r_0,..,r_{n-1}>                     (allreduce)
+    bcast src=<s> weight=<w> chunk=<C> parent=<p_0,..,p_{n-1}>           (allgather)
+    a2a   weight=<w> chunk=<C>                                            (alltoall)
+
+Readings: Q9 partition, Q10 chunk, Q13 ring expansion.
+"""
+
+from dataclasses import dataclass, field
+
+MAX_RANKS = 64
+MAX_SUBS = 128
+MAX_WEIGHT = 1 << 24
+MAX_CHUNK = 1 << 31
+ESIZE = {"f32": 4, "bf16": 2, "i32": 4}
+
+
+class StrategyError(ValueError):
+    """Malformed or invalid strategy text."""
+
+
+@dataclass
+class Sub:
+    """One sub-collective m after ring expansion."""
+    kind: str                 # 'tree' (allreduce), 'bcast' (allgather), 'a2a'
+    weight: int               # effective integer weight (see expand_weights)
+    chunk: int                # C_m in bytes
+    parent: list = None       # parent[g], -1 at the root (tree / bcast)
+    noagg: frozenset = frozenset()   # ranks g with a_{m,g} = 0
+    src: int = -1             # bcast source (== root)
+
+    @property
+    def root(self):
+        return self.parent.index(-1)
+
+    def children(self, g):
+        """Children of g in ascending rank order (reading Q5)."""
+        return [c for c in range(len(self.parent)) if self.parent[c] == g]
+
+
+@dataclass
+class Strategy:
+    nranks: int
+    collective: str
+    subs: list = field(default_factory=list)
+
+
+def _int(tok, what):
+    try:
+        v = int(tok, 10)
+    except ValueError:
+        raise StrategyError(f"bad integer for {what}: {tok!r}")
+    return v
+
+
+def _intlist(tok, what):
+    if tok == "":
+        return []
+    return [_int(t, what) for t in tok.split(",")]
+
+
+def _check_tree(parent, n, what):
+    if len(parent) != n:
+        raise StrategyError(f"{what}: parent has {len(parent)} entries, nranks={n}")
+    roots = [g for g in range(n) if parent[g] == -1]
+    if len(roots) != 1:
+        raise StrategyError(f"{what}: need exactly one root, found {len(roots)}")
+    for g, p in enumerate(parent):
+        if p == -1:
+            continue
+        if not (0 <= p < n):
+            raise StrategyError(f"{what}: parent[{g}]={p} out of range")
+        if p == g:
+            raise StrategyError(f"{what}: self loop at {g}")
+    # every node must reach the root: walk at most n steps
+    for g in range(n):
+        x, steps = g, 0
+        while parent[x] != -1:
+            x = parent[x]
+            steps += 1
+            if steps > n:
+                raise StrategyError(f"{what}: cycle through rank {g}")
+
+
+def parse(text):
+    """Parse and validate strategy text; returns Strategy with rings expanded.
+
+    Ring expansion (reading Q13): ``ring order=r_0..r_{n-1}`` becomes n chain
+    trees; tree m has root r_m, leaf r_{m+1}, and parent[r_{m+j}] = r_{m+j+1}
+    for j = 1..n-1 (indices mod n).  A ring of weight w contributes w/n per
+    chain; to keep integers every tree/bcast/a2a weight is multiplied by n and
+    each chain gets weight w (only weight ratios enter the partition, Q9).
+    """
+    lines = []
+    for raw in text.splitlines():
+        s = raw.split("#", 1)[0].strip()
+        if s:
+            lines.append(s)
+    if not lines or lines[0].split() != ["adapcc-strategy", "1"]:
+        raise StrategyError("first line must be 'adapcc-strategy 1'")
+    n = None
+    coll = None
+    raw_subs = []
+    for s in lines[1:]:
+        toks = s.split()
+        head = toks[0]
+        if head == "nranks":
+            if n is not None or len(toks) != 2:
+                raise StrategyError("bad or repeated nranks line")
+            n = _int(toks[1], "nranks")
+            if not (1 <= n <= MAX_RANKS):
+                raise StrategyError(f"nranks {n} out of range")
+            continue
+        if head == "collective":
+            if coll is not None or len(toks) != 2:
+                raise StrategyError("bad or repeated collective line")
+            coll = toks[1]
+            if coll not in ("allreduce", "allgather", "alltoall"):
+                raise StrategyError(f"unknown collective {coll!r}")
+            continue
+        if head not in ("tree", "ring", "bcast", "a2a"):
+            raise StrategyError(f"unknown directive {head!r}")
+        kv = {}
+        for t in toks[1:]:
+            if "=" not in t:
+                raise StrategyError(f"expected key=value, got {t!r}")
+            k, v = t.split("=", 1)
+            if k in kv:
+                raise StrategyError(f"repeated key {k!r}")
+            kv[k] = v
+        raw_subs.append((head, kv))
+    if n is None or coll is None:
+        raise StrategyError("missing nranks or collective line")
+    allowed = {"allreduce": ("tree", "ring"), "allgather": ("bcast",),
+               "alltoall": ("a2a",)}[coll]
+    keys = {"tree": {"weight", "chunk", "parent"}, "ring": {"weight", "chunk", "order"},
+            "bcast": {"src", "weight", "chunk", "parent"}, "a2a": {"weight", "chunk"}}
+    optional = {"tree": {"noagg"}, "ring": set(), "bcast": set(), "a2a": set()}
+    if not raw_subs:
+        raise StrategyError("no sub-collective lines")
+    st = Strategy(nranks=n, collective=coll)
+    for head, kv in raw_subs:
+        if head not in allowed:
+            raise StrategyError(f"directive {head!r} not valid for {coll}")
+        missing = keys[head] - set(kv)
+        extra = set(kv) - keys[head] - optional[head]
+        if missing or extra:
+            raise StrategyError(f"{head}: missing {sorted(missing)} extra {sorted(extra)}")
+        w = _int(kv["weight"], "weight")
+        c = _int(kv["chunk"], "chunk")
+        if not (0 <= w <= MAX_WEIGHT):
+            raise StrategyError(f"weight {w} out of range")
+        if c < 16 or c % 16 != 0 or c > MAX_CHUNK:
+            raise StrategyError(f"chunk {c} must be a positive multiple of 16 <= 2^31")
+        if head == "tree":
+            parent = _intlist(kv["parent"], "parent")
+            _check_tree(parent, n, "tree")
+            noagg = _intlist(kv.get("noagg", ""), "noagg")
+            if len(set(noagg)) != len(noagg):
+                raise StrategyError("duplicate rank in noagg")
+            for g in noagg:
+                if not (0 <= g < n):
+                    raise StrategyError(f"noagg rank {g} out of range")
+                if parent[g] == -1:
+                    raise StrategyError("noagg may not contain the root")
+            st.subs.append(Sub("tree", w * n, c, parent, frozenset(noagg)))
+        elif head == "ring":
+            order = _intlist(kv["order"], "order")
+            if sorted(order) != list(range(n)):
+                raise StrategyError("ring order must be a permutation of 0..n-1")
+            for m in range(n):
+                parent = [None] * n
+                parent[order[m]] = -1
+                for j in range(1, n):
+                    parent[order[(m + j) % n]] = order[(m + j + 1) % n]
+                st.subs.append(Sub("tree", w, c, parent, frozenset()))
+        elif head == "bcast":
+            src = _int(kv["src"], "src")
+            if not (0 <= src < n):
+                raise StrategyError(f"bcast src {src} out of range")
+            parent = _intlist(kv["parent"], "parent")
+            _check_tree(parent, n, "bcast")
+            if parent[src] != -1:
+                raise StrategyError("bcast root must be its src")
+            st.subs.append(Sub("bcast", w * n, c, parent, frozenset(), src))
+        else:
+            st.subs.append(Sub("a2a", w * n, c))
+    if len(st.subs) > MAX_SUBS:
+        raise StrategyError(f"{len(st.subs)} sub-collectives > {MAX_SUBS}")
+    if coll == "allgather":
+        for s in range(n):
+            ws = [sb.weight for sb in st.subs if sb.src == s]
+            if not ws or sum(ws) == 0:
+                raise StrategyError(f"allgather source {s} has no positive-weight bcast")
+    else:
+        if sum(sb.weight for sb in st.subs) == 0:
+            raise StrategyError("total weight must be > 0")
+    return st
+
+
+def partition(count, esize, weights):
+    """Split ``count`` elements into len(weights) contiguous ranges (reading Q9).
+
+    P:L167 only says sum_m S_m = S.  Rule: unit u = 16/esize elements,
+    U = floor(count/u), W = sum(w); b_m = floor(U * sum_{j<m} w_j / W) * u for
+    m < M, b_M = count (the last range also takes the ragged tail).
+    Returns the M+1 bounds.  Python integers: exact.
+    """
+    u = 16 // esize
+    U = count // u
+    W = sum(weights)
+    bounds = []
+    acc = 0
+    for w in weights:
+        bounds.append((U * acc // W) * u)
+        acc += w
+    bounds.append(count)
+    return bounds
+
+
+def chunks(lo, hi, chunk_bytes, esize):
+    """Chunks of C_m bytes over [lo, hi) (reading Q10); last may be short."""
+    ce = chunk_bytes // esize
+    out = []
+    a = lo
+    while a < hi:
+        out.append((a, min(hi, a + ce)))
+        a += ce
+    return out
