@@ -1,0 +1,219 @@
+/*
+ * adapcc.h -- C ABI of the B200-native AdapCC hot path.
+ *
+ * What it computes: collective communication executed along an AdapCC
+ * *strategy* -- M parallel sub-collectives, each a weighted spanning tree over
+ * the ranks with its own data partition S_m and chunk size C_m (PAPER.md
+ * §IV-D) -- under a ready-rank mask: only ready ranks contribute,
+ * non-ready ranks act as relays and still receive the result (§IV-C,
+ * P:L127-159).  Semantics are defined by the CPU oracle (oracle/, DESIGN.md
+ * §3); the strategy text format is DESIGN.md §2.
+ *
+ * Conventions for every entry point:
+ *   - Returns adapcc_result_t; 0 == ADAPCC_SUCCESS.  Never throws, never exits.
+ *   - Pointers named *buf / *bufs are DEVICE pointers on the communicator's
+ *     device, 16-byte aligned; otherwise ADAPCC_ERR_INVALID_ARGUMENT.
+ *   - Synchronous errors (bad argument, bad strategy) are detected before
+ *     anything is enqueued; they are deterministic given identical arguments,
+ *     so all ranks fail together.
+ *   - Device-side errors (watchdog timeout) are latched; read them with
+ *     adapcc_get_async_error(), after which the communicator must be finalized.
+ *   - Collective calls (allreduce/allgather/alltoall/set_strategy) must be
+ *     issued in the same order with the same arguments (except buffers) on
+ *     every rank; they are asynchronous and stream-ordered (the paper's Work
+ *     Queue / Result Queue, become the CUDA stream).  Calls on one
+ *     communicator must be ordered (one stream, or streams joined by events).
+ *   - Ownership: the library owns its scratch arena, IPC mappings, plan tables
+ *     and a host-mapped error word; the caller owns every buffer and stream.
+ */
+#ifndef ADAPCC_H
+#define ADAPCC_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#if defined(__GNUC__)
+#define ADAPCC_API __attribute__((visibility("default")))
+#else
+#define ADAPCC_API
+#endif
+
+#define ADAPCC_VERSION 1
+#define ADAPCC_MAX_RANKS 64
+
+typedef struct adapcc_comm_s* adapcc_comm_t;
+typedef void* adapcc_stream_t; /* a cudaStream_t; NULL = legacy default stream */
+
+typedef enum {
+  ADAPCC_SUCCESS = 0,
+  ADAPCC_ERR_INVALID_ARGUMENT = 1,
+  ADAPCC_ERR_INVALID_STRATEGY = 2,
+  ADAPCC_ERR_UNSUPPORTED = 3,
+  ADAPCC_ERR_CUDA = 4,
+  ADAPCC_ERR_BOOTSTRAP = 5,
+  ADAPCC_ERR_OOM = 6,
+  ADAPCC_ERR_TIMEOUT = 7,
+  ADAPCC_ERR_MISMATCH = 8
+} adapcc_result_t;
+
+typedef enum { ADAPCC_FLOAT32 = 0, ADAPCC_BFLOAT16 = 1, ADAPCC_INT32 = 2 } adapcc_dtype_t;
+typedef enum { ADAPCC_ALLREDUCE = 0, ADAPCC_ALLGATHER = 1, ADAPCC_ALLTOALL = 2 } adapcc_coll_t;
+
+/* Transport modes.  DIRECT: every rank's send/recv buffer is addressable by
+ * the engine (loopback: one process owns all virtual ranks), so data moves
+ * once from source to destination.  STAGED: a rank only touches its own
+ * buffers plus the peers' IPC-mapped scratch arenas (landing and broadcast
+ * slots with per-chunk flags) -- the multi-process protocol. */
+typedef enum { ADAPCC_MODE_DIRECT = 0, ADAPCC_MODE_STAGED = 1 } adapcc_mode_t;
+
+/* ACCUMULATE: recvbuf += result (one rounding), the paper's phase 2 in which
+ * the late ranks' data is combined with the phase-1 result. */
+#define ADAPCC_FLAG_ACCUMULATE 0x1u
+
+/* Bootstrap all-gather the caller implements (Python: torch.distributed
+ * all_gather on the process group).  Gathers bytes_per_rank from every rank
+ * into recv in rank order.  Returns 0 on success.  Used once in adapcc_init
+ * to exchange CUDA IPC handles (the paper's "AllGather communication" of
+ * IPC handles into a memory pointer table, §V-A, Fig. 10). */
+typedef int (*adapcc_bootstrap_allgather_fn)(const void* send, void* recv,
+                                             size_t bytes_per_rank, void* ctx);
+
+/* ---------------------------------------------------------------- setup --- */
+
+/* Multi-process communicator: one process per GPU (§V-A).
+ * Allocates a scratch arena of scratch_bytes (0 = default 1 GiB) on
+ * cuda_device, exports it with cudaIpcGetMemHandle, all-gathers the handles
+ * through ag(), and maps every peer's arena.  Blocking; every rank must call
+ * it.  Mode is STAGED.  Installs the default strategies. */
+ADAPCC_API adapcc_result_t adapcc_init(adapcc_comm_t* comm, int rank, int nranks, int cuda_device,
+                            size_t scratch_bytes, adapcc_bootstrap_allgather_fn ag,
+                            void* ag_ctx);
+
+/* Loopback communicator: nranks VIRTUAL ranks hosted by this process on one
+ * device; one kernel launch executes every virtual rank's part of the
+ * collective with the same engine and flag protocol (mode STAGED), or the
+ * single-copy DIRECT plan.  scratch_bytes is per virtual rank. */
+ADAPCC_API adapcc_result_t adapcc_init_loopback(adapcc_comm_t* comm, int nranks, int cuda_device,
+                                     size_t scratch_bytes, adapcc_mode_t mode);
+
+/* Replace the strategy of one collective (§IV-B/§VI-E graph reconstruction
+ * without restart).  strategy_text: NUL-terminated,
+ * format DESIGN.md §2; nranks in the text must equal the communicator's.
+ * Takes effect for every later call in issue order; calls already enqueued
+ * keep the strategy they were issued with (their plan tables stay alive).
+ * stream is accepted for API symmetry; the swap itself needs no device work.
+ * Errors: INVALID_STRATEGY (parse/validate), INVALID_ARGUMENT (coll). */
+ADAPCC_API adapcc_result_t adapcc_set_strategy(adapcc_comm_t comm, adapcc_coll_t coll,
+                                    const char* strategy_text, adapcc_stream_t stream);
+
+/* ---------------------------------------------- collectives (multi-process) --- */
+
+/* AllReduce (SUM) of count elements: every rank, relays included, receives
+ * sum_{r ready} sendbuf_r in recvbuf.
+ * ready_mask bit r = rank r is ready; bits >= nranks must be 0.
+ * A non-ready rank's sendbuf is never read and may be NULL.
+ * In place allowed (sendbuf == recvbuf).  flags: ADAPCC_FLAG_ACCUMULATE. */
+ADAPCC_API adapcc_result_t adapcc_allreduce(adapcc_comm_t comm, const void* sendbuf, void* recvbuf,
+                                 size_t count, adapcc_dtype_t dtype, uint64_t ready_mask,
+                                 unsigned flags, adapcc_stream_t stream);
+
+/* AllGather = one Broadcast per source: recvbuf holds nranks slots of
+ * sendcount elements; slot s receives sendbuf_s for every ready s; slots of
+ * non-ready sources are left untouched.  In place allowed when
+ * sendbuf == recvbuf + rank*sendcount*esize. */
+ADAPCC_API adapcc_result_t adapcc_allgather(adapcc_comm_t comm, const void* sendbuf, void* recvbuf,
+                                 size_t sendcount, adapcc_dtype_t dtype, uint64_t ready_mask,
+                                 adapcc_stream_t stream);
+
+/* AlltoAll: sendbuf and recvbuf hold nranks
+ * blocks of count_per_peer elements; block d of rank s lands in block s of
+ * rank d, for every ready s.  Aliasing sendbuf/recvbuf is an error. */
+ADAPCC_API adapcc_result_t adapcc_alltoall(adapcc_comm_t comm, const void* sendbuf, void* recvbuf,
+                                size_t count_per_peer, adapcc_dtype_t dtype,
+                                uint64_t ready_mask, adapcc_stream_t stream);
+
+/* ---------------------------------------------------- collectives (loopback) --- */
+/* Same semantics; sendbufs/recvbufs are HOST arrays of nranks device pointers,
+ * one per virtual rank.  Non-ready entries of sendbufs may be NULL. */
+ADAPCC_API adapcc_result_t adapcc_allreduce_lb(adapcc_comm_t comm, const void* const* sendbufs,
+                                    void* const* recvbufs, size_t count, adapcc_dtype_t dtype,
+                                    uint64_t ready_mask, unsigned flags, adapcc_stream_t stream);
+ADAPCC_API adapcc_result_t adapcc_allgather_lb(adapcc_comm_t comm, const void* const* sendbufs,
+                                    void* const* recvbufs, size_t sendcount,
+                                    adapcc_dtype_t dtype, uint64_t ready_mask,
+                                    adapcc_stream_t stream);
+ADAPCC_API adapcc_result_t adapcc_alltoall_lb(adapcc_comm_t comm, const void* const* sendbufs,
+                                   void* const* recvbufs, size_t count_per_peer,
+                                   adapcc_dtype_t dtype, uint64_t ready_mask,
+                                   adapcc_stream_t stream);
+
+/* ------------------------------------------------------------- lifecycle --- */
+
+/* Latched device error (TIMEOUT) or SUCCESS.  Does not synchronize. */
+ADAPCC_API adapcc_result_t adapcc_get_async_error(adapcc_comm_t comm);
+/* Synchronizes the device, unmaps peers, frees everything.  comm may be NULL. */
+ADAPCC_API adapcc_result_t adapcc_finalize(adapcc_comm_t comm);
+ADAPCC_API const char* adapcc_strerror(adapcc_result_t r);
+
+/* Runtime knobs.  key: "timeout_ms" (watchdog, default 10000; env
+ * ADAPCC_TIMEOUT_MS), "max_ctas" (grid cap, 0 = #SMs x occupancy; env
+ * ADAPCC_NCTAS), "debug_drop_rank" (loopback test hook: virtual rank r posts
+ * nothing, so its consumers hit the watchdog; -1 = off). */
+ADAPCC_API adapcc_result_t adapcc_config(adapcc_comm_t comm, const char* key, int64_t value);
+
+/* Number of engine kernel launches this communicator has issued. */
+ADAPCC_API adapcc_result_t adapcc_launch_count(adapcc_comm_t comm, uint64_t* count);
+
+/* ------------------------------------------------- host-only inspection ---
+ * No GPU needed.  Used by the CPU tests to cross-check the C++ loader and
+ * planner against the oracle (they share no code). */
+
+/* Parse + validate.  On success fills nranks, coll, nsubs (after ring
+ * expansion); on INVALID_STRATEGY writes a message into err (may be NULL). */
+ADAPCC_API adapcc_result_t adapcc_strategy_check(const char* strategy_text, int* nranks, int* coll,
+                                      int* nsubs, char* err, size_t err_len);
+
+/* Behaviour tuples of sub-collective `sub` under ready_mask:
+ * tuples[4*g + {0,1,2,3}] = isActive, hasRecv, hasKernel, hasSend of rank g;
+ * nflows[g] = number of flows rank g emits upward (Fig. 8(b)). */
+ADAPCC_API adapcc_result_t adapcc_strategy_tuples(const char* strategy_text, int sub, uint64_t ready_mask,
+                                       uint8_t* tuples, int32_t* nflows);
+
+/* Effective integer weight, chunk bytes, parent array and bcast source of
+ * sub-collective `sub` (parent: nranks entries, -1 at the root). */
+ADAPCC_API adapcc_result_t adapcc_strategy_sub(const char* strategy_text, int sub, int64_t* weight,
+                                    int64_t* chunk_bytes, int32_t* parent, int32_t* src);
+
+/* Partition (DESIGN.md §3 Q9): bounds[0..nsubs] of `count` elements over all
+ * sub-collectives (allreduce/alltoall), or over the bcast lines of source
+ * `src` (allgather; bounds has (#lines of src)+1 entries). */
+ADAPCC_API adapcc_result_t adapcc_strategy_partition(const char* strategy_text, uint64_t count,
+                                          adapcc_dtype_t dtype, int src, uint64_t* bounds,
+                                          int* nbounds);
+
+/* Plan statistics for one rank (-1 = all virtual ranks) of a call. */
+typedef struct {
+  uint64_t tasks;         /* fold/copy tasks */
+  uint64_t items;         /* (task, chunk) work items */
+  uint64_t levels;        /* dependency depth + 1 */
+  uint64_t segments;      /* launches the call is split into */
+  uint64_t bytes_read;    /* payload bytes loaded by the engine */
+  uint64_t bytes_written; /* payload bytes stored by the engine */
+  uint64_t remote_bytes;  /* of which cross a rank boundary (loads+stores) */
+  uint64_t arena_bytes;   /* scratch bytes used per rank (max over ranks) */
+} adapcc_plan_stats_t;
+
+ADAPCC_API adapcc_result_t adapcc_plan_stats(const char* strategy_text, uint64_t count,
+                                  adapcc_dtype_t dtype, uint64_t ready_mask, unsigned flags,
+                                  adapcc_mode_t mode, int rank, size_t scratch_bytes,
+                                  adapcc_plan_stats_t* stats);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* ADAPCC_H */

@@ -84,36 +84,7 @@ def allreduce(xs, strategy_text, ready, dtype, accumulate=False, y_prev=None):
         lo, hi = bounds[m], bounds[m + 1]
         if lo == hi:
             continue
-        tup, flows = behavior(sub.parent, ready, sub.noagg)
-        agg_val = {}
-
-        def value(f):
-            kind, r = f
-            return xs[r][lo:hi] if kind == "in" else agg_val[r]
-
-        # post-order evaluation of the kernel nodes
-        order = []
-
-        def visit(g):
-            for c in sub.children(g):
-                visit(c)
-            order.append(g)
-
-        visit(sub.root)
-        for g in order:
-            if tup[g][2]:
-                terms = [xs[g][lo:hi]] if tup[g][0] else []
-                for c in sub.children(g):
-                    if tup[c][3]:
-                        terms += [value(f) for f in flows[c]]
-                agg_val[g] = _fold(terms, dtype)
-        root = sub.root
-        if tup[root][2]:
-            res = agg_val[root]
-        else:
-            fl = flows[root]
-            assert len(fl) <= 1, "a non-kernel root emits at most one flow"
-            res = np.array(value(fl[0]), copy=True) if fl else None
+        res = _tree_result([x[lo:hi] if x is not None else None for x in xs], sub, ready, dtype)
         for g in range(n):
             if accumulate:
                 if res is not None:
@@ -121,6 +92,62 @@ def allreduce(xs, strategy_text, ready, dtype, accumulate=False, y_prev=None):
             else:
                 ys[g][lo:hi] = res if res is not None else _zero(hi - lo, dtype)
     return ys
+
+
+def _tree_result(vals, sub, ready, dtype):
+    """Result of one reduce tree over the elements in ``vals`` (vals[r]: rank r's
+    values, None if not ready): bottom-up tuples, fold at every
+    kernel node (own first, then sending children ascending, Q5), the root's
+    aggregate or its single flow; None when no ready rank is in the tree."""
+    tup, flows = behavior(sub.parent, ready, sub.noagg)
+    agg_val = {}
+
+    def value(f):
+        kind, r = f
+        return vals[r] if kind == "in" else agg_val[r]
+
+    order = []
+
+    def visit(g):
+        for c in sub.children(g):
+            visit(c)
+        order.append(g)
+
+    visit(sub.root)
+    for g in order:
+        if tup[g][2]:
+            terms = [vals[g]] if tup[g][0] else []
+            for c in sub.children(g):
+                if tup[c][3]:
+                    terms += [value(f) for f in flows[c]]
+            agg_val[g] = _fold(terms, dtype)
+    root = sub.root
+    if tup[root][2]:
+        return agg_val[root]
+    fl = flows[root]
+    assert len(fl) <= 1, "a non-kernel root emits at most one flow"
+    return np.array(value(fl[0]), copy=True) if fl else None
+
+
+def allreduce_elements(vals, idx, count, strategy_text, ready, dtype):
+    """AllReduce result at selected element indices only (for sampled parity at
+    full size): vals[r] holds rank r's inputs AT ``idx``; each element is
+    reduced by the tree whose partition contains it (Q9), exactly as in
+    ``allreduce``.  Returns the (broadcast-identical) result at idx; +0 where
+    no rank is ready."""
+    st = parse(strategy_text)
+    ready = set(ready)
+    idx = np.asarray(idx, dtype=np.int64)
+    bounds = partition(count, ESIZE[dtype], [s.weight for s in st.subs])
+    out = _zero(len(idx), dtype)
+    for m, sub in enumerate(st.subs):
+        sel = np.nonzero((idx >= bounds[m]) & (idx < bounds[m + 1]))[0]
+        if len(sel) == 0:
+            continue
+        res = _tree_result([v[sel] if v is not None else None for v in vals], sub, ready, dtype)
+        if res is not None:
+            out[sel] = res
+    return out
 
 
 def allreduce_exact(xs, ready, dtype, count=None):

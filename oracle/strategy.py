@@ -23,6 +23,7 @@ Format (one directive per line, '#' starts a comment):
 Readings: Q9 partition, Q10 chunk, Q13 ring expansion.
 """
 
+import re
 from dataclasses import dataclass, field
 
 MAX_RANKS = 64
@@ -62,12 +63,14 @@ class Strategy:
     subs: list = field(default_factory=list)
 
 
+_INT_RE = re.compile(r"-?[0-9]+")
+
+
 def _int(tok, what):
-    try:
-        v = int(tok, 10)
-    except ValueError:
+    """Integers are ``-?[0-9]+``; no '+', '_' or whitespace."""
+    if not _INT_RE.fullmatch(tok):
         raise StrategyError(f"bad integer for {what}: {tok!r}")
-    return v
+    return int(tok, 10)
 
 
 def _intlist(tok, what):

@@ -1,0 +1,320 @@
+"""Thin Python binding of libadapcc.so (include/adapcc.h): argument marshalling only.
+
+Every step of the collective runs in the CUDA engine behind the C ABI; there
+is no Python or CPU fallback -- if the library is missing or a call fails,
+this module raises.  torch is used only for tensors, the current stream and
+the process group used to bootstrap IPC handles (the paper's set-up
+AllGather), as the north star requires.
+
+API (mirrors the paper's ``adapcc.init()/setup()/allreduce()``):
+    comm = Communicator.init(group)                 # one process per GPU
+    comm = Communicator.loopback(n, mode="direct")  # n virtual ranks, 1 GPU
+    comm.set_strategy("allreduce", text)
+    comm.allreduce(x, out, ready={...}, accumulate=False)
+    comm.allgather(x, out, ready) ; comm.alltoall(x, out, ready)
+    comm.allreduce_lb([x_r], [y_r], ready, accumulate)  # loopback
+Host-only helpers (no GPU): strategy_check, strategy_tuples, strategy_sub,
+strategy_partition, plan_stats.
+"""
+
+import ctypes
+import os
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+_LIB_PATH = os.path.join(_PKG, "libadapcc.so")
+
+SUCCESS, INVALID_ARGUMENT, INVALID_STRATEGY, UNSUPPORTED, CUDA, BOOTSTRAP, OOM, TIMEOUT, MISMATCH = range(9)
+COLL = {"allreduce": 0, "allgather": 1, "alltoall": 2}
+MODE = {"direct": 0, "staged": 1}
+FLAG_ACCUMULATE = 0x1
+DTYPE_CODE = {"f32": 0, "bf16": 1, "i32": 2}
+
+_lib = None
+
+
+class AdapccError(RuntimeError):
+    def __init__(self, code, where=""):
+        self.code = code
+        msg = _load().adapcc_strerror(code).decode() if code >= 0 else "error"
+        super().__init__(f"{where}: adapcc error {code} ({msg})")
+
+
+class PlanStats(ctypes.Structure):
+    _fields_ = [(k, ctypes.c_uint64) for k in (
+        "tasks", "items", "levels", "segments", "bytes_read", "bytes_written",
+        "remote_bytes", "arena_bytes")]
+
+    def as_dict(self):
+        return {k: getattr(self, k) for k, _ in self._fields_}
+
+
+AG_FN = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_size_t,
+                         ctypes.c_void_p)
+
+
+def _load():
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(_LIB_PATH):
+        raise ImportError(f"{_LIB_PATH} is missing: build it with "
+                          "`python -m paper_conf_icdcs_zhaozw24_b200._build` (there is no fallback)")
+    L = ctypes.CDLL(_LIB_PATH)
+    vp, sz, u64, i32, i64 = ctypes.c_void_p, ctypes.c_size_t, ctypes.c_uint64, ctypes.c_int, ctypes.c_int64
+    pp = ctypes.POINTER(ctypes.c_void_p)
+    sig = {
+        "adapcc_init": [ctypes.POINTER(vp), i32, i32, i32, sz, AG_FN, vp],
+        "adapcc_init_loopback": [ctypes.POINTER(vp), i32, i32, sz, i32],
+        "adapcc_set_strategy": [vp, i32, ctypes.c_char_p, vp],
+        "adapcc_allreduce": [vp, vp, vp, sz, i32, u64, ctypes.c_uint, vp],
+        "adapcc_allgather": [vp, vp, vp, sz, i32, u64, vp],
+        "adapcc_alltoall": [vp, vp, vp, sz, i32, u64, vp],
+        "adapcc_allreduce_lb": [vp, pp, pp, sz, i32, u64, ctypes.c_uint, vp],
+        "adapcc_allgather_lb": [vp, pp, pp, sz, i32, u64, vp],
+        "adapcc_alltoall_lb": [vp, pp, pp, sz, i32, u64, vp],
+        "adapcc_get_async_error": [vp],
+        "adapcc_finalize": [vp],
+        "adapcc_config": [vp, ctypes.c_char_p, i64],
+        "adapcc_launch_count": [vp, ctypes.POINTER(u64)],
+        "adapcc_strategy_check": [ctypes.c_char_p, ctypes.POINTER(i32), ctypes.POINTER(i32),
+                                  ctypes.POINTER(i32), ctypes.c_char_p, sz],
+        "adapcc_strategy_tuples": [ctypes.c_char_p, i32, u64, ctypes.POINTER(ctypes.c_uint8),
+                                   ctypes.POINTER(ctypes.c_int32)],
+        "adapcc_strategy_sub": [ctypes.c_char_p, i32, ctypes.POINTER(i64), ctypes.POINTER(i64),
+                                ctypes.POINTER(ctypes.c_int32), ctypes.POINTER(ctypes.c_int32)],
+        "adapcc_strategy_partition": [ctypes.c_char_p, u64, i32, i32, ctypes.POINTER(u64),
+                                      ctypes.POINTER(i32)],
+        "adapcc_plan_stats": [ctypes.c_char_p, u64, i32, u64, ctypes.c_uint, i32, i32, sz,
+                              ctypes.POINTER(PlanStats)],
+    }
+    for name, args in sig.items():
+        f = getattr(L, name)
+        f.argtypes = args
+        f.restype = ctypes.c_int
+    L.adapcc_strerror.argtypes = [ctypes.c_int]
+    L.adapcc_strerror.restype = ctypes.c_char_p
+    _lib = L
+    return L
+
+
+def lib_path():
+    return _LIB_PATH
+
+
+def _check(code, where):
+    if code != SUCCESS:
+        raise AdapccError(code, where)
+
+
+def _mask(ready, n):
+    if ready is None:
+        return (1 << n) - 1
+    if isinstance(ready, int):
+        return ready
+    m = 0
+    for r in ready:
+        m |= 1 << int(r)
+    return m
+
+
+def _dtype_code(t):
+    import torch
+    codes = {torch.float32: 0, torch.bfloat16: 1, torch.int32: 2}
+    if t.dtype not in codes:
+        raise TypeError(f"unsupported dtype {t.dtype}")
+    return codes[t.dtype]
+
+
+def _stream(stream):
+    import torch
+    s = stream if stream is not None else torch.cuda.current_stream()
+    return ctypes.c_void_p(s.cuda_stream)
+
+
+def _ptr(t):
+    return ctypes.c_void_p(t.data_ptr()) if t is not None else ctypes.c_void_p(0)
+
+
+# ------------------------------------------------------------ host-only helpers
+def strategy_check(text):
+    L = _load()
+    n, c, m = ctypes.c_int(), ctypes.c_int(), ctypes.c_int()
+    err = ctypes.create_string_buffer(256)
+    code = L.adapcc_strategy_check(text.encode(), ctypes.byref(n), ctypes.byref(c),
+                                   ctypes.byref(m), err, 256)
+    if code != SUCCESS:
+        raise AdapccError(code, "strategy_check: " + err.value.decode())
+    return n.value, c.value, m.value
+
+
+def strategy_tuples(text, sub, mask):
+    L = _load()
+    n, _, _ = strategy_check(text)
+    tup = (ctypes.c_uint8 * (4 * n))()
+    nfl = (ctypes.c_int32 * n)()
+    _check(L.adapcc_strategy_tuples(text.encode(), sub, mask, tup, nfl), "strategy_tuples")
+    return [tuple(bool(tup[4 * g + i]) for i in range(4)) for g in range(n)], list(nfl)
+
+
+def strategy_sub(text, sub):
+    L = _load()
+    n, _, _ = strategy_check(text)
+    w, c = ctypes.c_int64(), ctypes.c_int64()
+    par = (ctypes.c_int32 * n)()
+    src = ctypes.c_int32()
+    _check(L.adapcc_strategy_sub(text.encode(), sub, ctypes.byref(w), ctypes.byref(c), par,
+                                 ctypes.byref(src)), "strategy_sub")
+    return w.value, c.value, list(par), src.value
+
+
+def strategy_partition(text, count, dtype, src=-1):
+    L = _load()
+    _, _, m = strategy_check(text)
+    b = (ctypes.c_uint64 * (m + 1))()
+    nb = ctypes.c_int()
+    _check(L.adapcc_strategy_partition(text.encode(), count, DTYPE_CODE[dtype], src, b,
+                                       ctypes.byref(nb)), "strategy_partition")
+    return list(b[:nb.value])
+
+
+def plan_stats(text, count, dtype, mask, accumulate=False, mode="direct", rank=-1, scratch_bytes=0):
+    L = _load()
+    st = PlanStats()
+    _check(L.adapcc_plan_stats(text.encode(), count, DTYPE_CODE[dtype], mask,
+                               FLAG_ACCUMULATE if accumulate else 0, MODE[mode], rank,
+                               scratch_bytes, ctypes.byref(st)), "plan_stats")
+    return st.as_dict()
+
+
+# --------------------------------------------------------------- communicator
+class Communicator:
+    """A communicator (the paper's transmission contexts)."""
+
+    def __init__(self, handle, nranks, rank, device, loopback, keep=None):
+        self._h = handle
+        self.nranks = nranks
+        self.rank = rank
+        self.device = device
+        self.loopback = loopback
+        self._keep = keep
+
+    # ---- construction
+    @classmethod
+    def loopback(cls, nranks, device=0, scratch_bytes=0, mode="direct"):
+        L = _load()
+        h = ctypes.c_void_p()
+        _check(L.adapcc_init_loopback(ctypes.byref(h), nranks, device, scratch_bytes, MODE[mode]),
+               "init_loopback")
+        return cls(h, nranks, 0, device, True)
+
+    @classmethod
+    def init(cls, group=None, scratch_bytes=0, device=None):
+        """Multi-process communicator over a torch.distributed process group."""
+        import torch
+        import torch.distributed as dist
+        L = _load()
+        rank = dist.get_rank(group)
+        n = dist.get_world_size(group)
+        dev = torch.cuda.current_device() if device is None else device
+        backend = dist.get_backend(group)
+        tdev = torch.device("cuda", dev) if backend == "nccl" else torch.device("cpu")
+
+        def ag(send, recv, nbytes, _ctx):
+            try:
+                mine = torch.frombuffer(bytearray(ctypes.string_at(send, nbytes)), dtype=torch.uint8)
+                outs = [torch.empty(nbytes, dtype=torch.uint8, device=tdev) for _ in range(n)]
+                dist.all_gather(outs, mine.to(tdev), group=group)
+                blob = b"".join(o.cpu().numpy().tobytes() for o in outs)
+                ctypes.memmove(recv, blob, len(blob))
+                return 0
+            except Exception:  # noqa: BLE001 -- reported as ADAPCC_ERR_BOOTSTRAP
+                return 1
+
+        cb = AG_FN(ag)
+        h = ctypes.c_void_p()
+        _check(L.adapcc_init(ctypes.byref(h), rank, n, dev, scratch_bytes, cb, None), "init")
+        return cls(h, n, rank, dev, False, keep=cb)
+
+    # ---- control
+    def set_strategy(self, coll, text, stream=None):
+        s = ctypes.c_void_p(0) if stream is None else _stream(stream)
+        _check(_load().adapcc_set_strategy(self._h, COLL[coll], text.encode(), s), "set_strategy")
+
+    def config(self, key, value):
+        _check(_load().adapcc_config(self._h, key.encode(), int(value)), "config")
+
+    def get_async_error(self):
+        return _load().adapcc_get_async_error(self._h)
+
+    def launch_count(self):
+        v = ctypes.c_uint64()
+        _check(_load().adapcc_launch_count(self._h, ctypes.byref(v)), "launch_count")
+        return v.value
+
+    def finalize(self):
+        if self._h:
+            _load().adapcc_finalize(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.finalize()
+        except Exception:  # noqa: BLE001
+            pass
+
+    # ---- multi-process collectives
+    def allreduce(self, x, out=None, ready=None, accumulate=False, stream=None):
+        out = x if out is None else out
+        m = _mask(ready, self.nranks)
+        send = x if (m >> self.rank) & 1 else None
+        _check(_load().adapcc_allreduce(self._h, _ptr(send), _ptr(out), out.numel(),
+                                        _dtype_code(out), m,
+                                        FLAG_ACCUMULATE if accumulate else 0, _stream(stream)),
+               "allreduce")
+        return out
+
+    def allgather(self, x, out, ready=None, stream=None):
+        m = _mask(ready, self.nranks)
+        send = x if (m >> self.rank) & 1 else None
+        cnt = out.numel() // self.nranks
+        _check(_load().adapcc_allgather(self._h, _ptr(send), _ptr(out), cnt, _dtype_code(out), m,
+                                        _stream(stream)), "allgather")
+        return out
+
+    def alltoall(self, x, out, ready=None, stream=None):
+        m = _mask(ready, self.nranks)
+        send = x if (m >> self.rank) & 1 else None
+        cnt = out.numel() // self.nranks
+        _check(_load().adapcc_alltoall(self._h, _ptr(send), _ptr(out), cnt, _dtype_code(out), m,
+                                       _stream(stream)), "alltoall")
+        return out
+
+    # ---- loopback collectives (lists of per-virtual-rank tensors)
+    def _arrays(self, xs, outs, m):
+        n = self.nranks
+        S = (ctypes.c_void_p * n)(*[(xs[r].data_ptr() if ((m >> r) & 1 and xs[r] is not None) else 0)
+                                    for r in range(n)])
+        D = (ctypes.c_void_p * n)(*[outs[r].data_ptr() for r in range(n)])
+        return S, D
+
+    def allreduce_lb(self, xs, outs, ready=None, accumulate=False, stream=None):
+        m = _mask(ready, self.nranks)
+        S, D = self._arrays(xs, outs, m)
+        _check(_load().adapcc_allreduce_lb(self._h, S, D, outs[0].numel(), _dtype_code(outs[0]), m,
+                                           FLAG_ACCUMULATE if accumulate else 0, _stream(stream)),
+               "allreduce_lb")
+        return outs
+
+    def allgather_lb(self, xs, outs, ready=None, stream=None):
+        m = _mask(ready, self.nranks)
+        S, D = self._arrays(xs, outs, m)
+        _check(_load().adapcc_allgather_lb(self._h, S, D, outs[0].numel() // self.nranks,
+                                           _dtype_code(outs[0]), m, _stream(stream)), "allgather_lb")
+        return outs
+
+    def alltoall_lb(self, xs, outs, ready=None, stream=None):
+        m = _mask(ready, self.nranks)
+        S, D = self._arrays(xs, outs, m)
+        _check(_load().adapcc_alltoall_lb(self._h, S, D, outs[0].numel() // self.nranks,
+                                          _dtype_code(outs[0]), m, _stream(stream)), "alltoall_lb")
+        return outs

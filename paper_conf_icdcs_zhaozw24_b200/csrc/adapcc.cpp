@@ -1,0 +1,626 @@
+// C ABI of the AdapCC B200 hot path (include/adapcc.h).
+//
+// Communicator = the paper's set of transmission contexts: a
+// registered scratch arena per rank (landing + broadcast slots + per-chunk
+// flags, the paper's receive/result buffers P:L243), IPC-mapped by every peer
+// after one bootstrap all-gather of handles (Fig. 10), plus the
+// strategy per collective and a cache of compiled plans.  Every collective
+// call is one engine launch per segment on the caller's stream.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdlib>
+#include <cstring>
+#include <list>
+#include <map>
+#include <memory>
+#include <mutex>
+#include <string>
+#include <tuple>
+#include <vector>
+
+#include "../../include/adapcc.h"
+#include "launch.hpp"
+#include "plan.hpp"
+#include "strategy.hpp"
+
+using namespace adapcc;
+
+namespace {
+
+constexpr size_t kDefaultScratch = size_t(1) << 30;
+constexpr int kPlanCacheCap = 64;
+
+struct DevSegment {
+  Task* tasks = nullptr;
+  BufRef* refs = nullptr;
+  FlagRef* flags = nullptr;
+  Item* items = nullptr;
+  uint32_t nitems = 0;
+};
+
+struct DevPlan {
+  std::vector<DevSegment> segs;
+  cudaEvent_t last_use = nullptr;
+  ~DevPlan() {
+    if (last_use) {
+      cudaEventSynchronize(last_use);
+      cudaEventDestroy(last_use);
+    }
+    for (auto& s : segs) {
+      cudaFree(s.tasks);
+      cudaFree(s.refs);
+      cudaFree(s.flags);
+      cudaFree(s.items);
+    }
+  }
+};
+
+using PlanKey = std::tuple<int, uint64_t, uint64_t, int, uint64_t, unsigned>;
+
+int esize_of(adapcc_dtype_t d) { return d == ADAPCC_BFLOAT16 ? 2 : 4; }
+
+std::string default_strategy(Coll c, int n) {
+  std::string s = "adapcc-strategy 1\nnranks " + std::to_string(n) + "\ncollective ";
+  if (c == kAllReduce) {
+    s += "allreduce\n";
+    for (int m = 0; m < n; ++m) {  // n star trees, equal weights
+      s += "tree weight=1 chunk=262144 parent=";
+      for (int g = 0; g < n; ++g) s += (g ? "," : "") + std::to_string(g == m ? -1 : m);
+      s += "\n";
+    }
+  } else if (c == kAllGather) {
+    s += "allgather\n";
+    for (int src = 0; src < n; ++src) {
+      s += "bcast src=" + std::to_string(src) + " weight=1 chunk=262144 parent=";
+      for (int g = 0; g < n; ++g) s += (g ? "," : "") + std::to_string(g == src ? -1 : src);
+      s += "\n";
+    }
+  } else {
+    s += "alltoall\na2a weight=1 chunk=1048576\n";
+  }
+  return s;
+}
+
+int64_t env_int(const char* name, int64_t dflt) {
+  const char* v = std::getenv(name);
+  return v && *v ? std::strtoll(v, nullptr, 10) : dflt;
+}
+
+}  // namespace
+
+struct adapcc_comm_s {
+  int rank = 0;
+  int nranks = 0;
+  int device = 0;
+  bool loopback = false;
+  Mode mode = kStaged;
+  uint64_t arena_bytes = 0;  // header + 2 halves
+  uint64_t half_bytes = 0;
+  char* own_arena = nullptr;               // loopback: all virtual ranks' arenas
+  std::vector<char*> arena;                // per rank base (peer-mapped in IPC mode)
+  unsigned* counters = nullptr;
+  int* h_err = nullptr;
+  int* d_err = nullptr;
+  uint64_t epoch = 0;
+  Strategy strat[3];
+  uint64_t strat_version[3] = {0, 0, 0};
+  std::map<PlanKey, std::shared_ptr<DevPlan>> plans;
+  std::list<PlanKey> lru;
+  int64_t timeout_ms = 10000;
+  int64_t max_ctas = 0;
+  int64_t drop_rank = -1;
+  uint64_t launches = 0;
+  int num_sms = 148;
+  int occ[3] = {1, 1, 1};
+  std::mutex mu;
+};
+
+namespace {
+
+adapcc_result_t cuda_fail(cudaError_t e) {
+  (void)e;
+  return ADAPCC_ERR_CUDA;
+}
+
+#define CK(expr)                                   \
+  do {                                             \
+    cudaError_t _e = (expr);                       \
+    if (_e != cudaSuccess) return cuda_fail(_e);   \
+  } while (0)
+
+adapcc_result_t common_init(adapcc_comm_s* c, size_t scratch) {
+  if (scratch == 0) scratch = kDefaultScratch;
+  if (scratch < (size_t)kArenaHeader + 2 * (4096 + 65536)) return ADAPCC_ERR_INVALID_ARGUMENT;
+  c->half_bytes = ((scratch - kArenaHeader) / 2) / 256 * 256;
+  c->arena_bytes = kArenaHeader + 2 * c->half_bytes;
+  c->timeout_ms = env_int("ADAPCC_TIMEOUT_MS", 10000);
+  c->max_ctas = env_int("ADAPCC_NCTAS", 0);
+  CK(cudaSetDevice(c->device));
+  CK(cudaDeviceGetAttribute(&c->num_sms, cudaDevAttrMultiProcessorCount, c->device));
+  for (int d = 0; d < 3; ++d) {
+    CK(engine_occupancy(d, &c->occ[d]));
+    if (c->occ[d] < 1) c->occ[d] = 1;
+  }
+  CK(cudaMalloc(&c->counters, 4 * sizeof(unsigned)));
+  CK(cudaMemset(c->counters, 0, 4 * sizeof(unsigned)));
+  CK(cudaHostAlloc(&c->h_err, sizeof(int), cudaHostAllocMapped));
+  *c->h_err = 0;
+  CK(cudaHostGetDevicePointer(&c->d_err, c->h_err, 0));
+  for (int k = 0; k < 3; ++k) {
+    std::string err;
+    if (!parse_strategy(default_strategy((Coll)k, c->nranks).c_str(), &c->strat[k], &err))
+      return ADAPCC_ERR_INVALID_STRATEGY;
+  }
+  return ADAPCC_SUCCESS;
+}
+
+void release(adapcc_comm_s* c) {
+  if (!c) return;
+  cudaSetDevice(c->device);
+  cudaDeviceSynchronize();
+  c->plans.clear();
+  if (c->loopback) {
+    cudaFree(c->own_arena);
+  } else {
+    for (int r = 0; r < (int)c->arena.size(); ++r) {
+      if (r == c->rank) cudaFree(c->arena[r]);
+      else if (c->arena[r]) cudaIpcCloseMemHandle(c->arena[r]);
+    }
+  }
+  cudaFree(c->counters);
+  cudaFreeHost(c->h_err);
+  delete c;
+}
+
+// Validate arguments common to every collective.
+adapcc_result_t check_common(adapcc_comm_t c, adapcc_dtype_t dtype, uint64_t mask) {
+  if (!c) return ADAPCC_ERR_INVALID_ARGUMENT;
+  if (dtype != ADAPCC_FLOAT32 && dtype != ADAPCC_BFLOAT16 && dtype != ADAPCC_INT32)
+    return ADAPCC_ERR_INVALID_ARGUMENT;
+  if (c->nranks < 64 && (mask >> c->nranks) != 0) return ADAPCC_ERR_INVALID_ARGUMENT;
+  if (*reinterpret_cast<volatile int*>(c->h_err)) return (adapcc_result_t)*c->h_err;
+  return ADAPCC_SUCCESS;
+}
+
+bool misaligned(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15) != 0; }
+
+bool overlap(const void* a, size_t an, const void* b, size_t bn) {
+  auto x = reinterpret_cast<uintptr_t>(a), y = reinterpret_cast<uintptr_t>(b);
+  return x < y + bn && y < x + an;
+}
+
+adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, uint64_t count, adapcc_dtype_t dtype,
+                         uint64_t mask, unsigned flags, std::shared_ptr<DevPlan>* out) {
+  PlanKey key{(int)coll, c->strat_version[coll], count, (int)dtype, mask, flags};
+  auto it = c->plans.find(key);
+  if (it != c->plans.end()) {
+    c->lru.remove(key);
+    c->lru.push_front(key);
+    *out = it->second;
+    return ADAPCC_SUCCESS;
+  }
+  PlanRequest rq;
+  rq.st = &c->strat[coll];
+  rq.count = count;
+  rq.esize = esize_of(dtype);
+  rq.ready_mask = mask;
+  rq.accumulate = flags & ADAPCC_FLAG_ACCUMULATE;
+  rq.mode = c->mode;
+  rq.half_bytes = c->half_bytes;
+  std::vector<SegmentPlan> segs;
+  std::string err;
+  if (!build_plan(rq, &segs, &err)) return ADAPCC_ERR_OOM;
+  auto plan = std::make_shared<DevPlan>();
+  CK(cudaEventCreateWithFlags(&plan->last_use, cudaEventDisableTiming));
+  for (auto& sp : segs) {
+    DevSegment d;
+    std::vector<Item> items = order_items(sp, c->loopback ? -1 : c->rank);
+    d.nitems = (uint32_t)items.size();
+    auto up = [](auto** dst, const auto& v) -> cudaError_t {
+      using T = typename std::decay_t<decltype(v)>::value_type;
+      size_t bytes = std::max<size_t>(1, v.size()) * sizeof(T);
+      cudaError_t e = cudaMalloc((void**)dst, bytes);
+      if (e != cudaSuccess) return e;
+      return v.empty() ? cudaSuccess : cudaMemcpy(*dst, v.data(), v.size() * sizeof(T), cudaMemcpyHostToDevice);
+    };
+    CK(up(&d.tasks, sp.tasks));
+    CK(up(&d.refs, sp.refs));
+    CK(up(&d.flags, sp.flags));
+    CK(up(&d.items, items));
+    plan->segs.push_back(d);
+  }
+  // in loopback an empty call launches nothing; in multi-process mode every
+  // rank launches every segment so that epochs stay aligned across ranks
+  if (c->plans.size() >= (size_t)kPlanCacheCap) {
+    PlanKey victim = c->lru.back();
+    c->lru.pop_back();
+    c->plans.erase(victim);  // DevPlan dtor waits for its last launch
+  }
+  c->plans[key] = plan;
+  c->lru.push_front(key);
+  *out = plan;
+  return ADAPCC_SUCCESS;
+}
+
+adapcc_result_t run(adapcc_comm_s* c, Coll coll, const void* const* send, void* const* recv,
+                    uint64_t count, adapcc_dtype_t dtype, uint64_t mask, unsigned flags,
+                    adapcc_stream_t stream) {
+  std::lock_guard<std::mutex> lock(c->mu);
+  CK(cudaSetDevice(c->device));
+  std::shared_ptr<DevPlan> plan;
+  adapcc_result_t r = get_plan(c, coll, count, dtype, mask, flags, &plan);
+  if (r != ADAPCC_SUCCESS) return r;
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  for (const DevSegment& seg : plan->segs) {
+    if (c->loopback && seg.nitems == 0) continue;
+    LaunchParams P{};
+    P.tasks = seg.tasks;
+    P.refs = seg.refs;
+    P.flags = seg.flags;
+    P.items = seg.items;
+    P.nitems = seg.nitems;
+    P.dtype = (int)dtype;
+    P.nranks = c->nranks;
+    P.my_rank = c->loopback ? -1 : c->rank;
+    P.ipc = c->loopback ? 0 : 1;
+    P.drop_rank = (int)c->drop_rank;
+    P.epoch = ++c->epoch;
+    P.timeout_ns = (uint64_t)std::max<int64_t>(1, c->timeout_ms) * 1000000ull;
+    P.counters = c->counters;
+    P.err = c->d_err;
+    const uint64_t parity = P.epoch & 1;
+    for (int q = 0; q < c->nranks; ++q) {
+      if (c->loopback || q == c->rank) {
+        const int i = c->loopback ? q : 0;
+        P.send[q] = const_cast<char*>(static_cast<const char*>(send[i]));
+        P.recv[q] = static_cast<char*>(recv[i]);
+      }
+      P.hdr[q] = c->arena[q];
+      P.arena[q] = c->arena[q] + kArenaHeader + parity * c->half_bytes;
+    }
+    int grid = c->num_sms * c->occ[(int)dtype];
+    if (c->max_ctas > 0) grid = (int)std::min<int64_t>(grid, c->max_ctas);
+    grid = std::max(1, std::min<int>(grid, (int)std::max<uint32_t>(1, seg.nitems)));
+    CK(engine_launch(P, grid, s));
+    ++c->launches;
+  }
+  CK(cudaEventRecord(plan->last_use, s));
+  return ADAPCC_SUCCESS;
+}
+
+}  // namespace
+
+extern "C" {
+
+const char* adapcc_strerror(adapcc_result_t r) {
+  switch (r) {
+    case ADAPCC_SUCCESS: return "success";
+    case ADAPCC_ERR_INVALID_ARGUMENT: return "invalid argument";
+    case ADAPCC_ERR_INVALID_STRATEGY: return "invalid strategy";
+    case ADAPCC_ERR_UNSUPPORTED: return "unsupported";
+    case ADAPCC_ERR_CUDA: return "CUDA error";
+    case ADAPCC_ERR_BOOTSTRAP: return "bootstrap failed";
+    case ADAPCC_ERR_OOM: return "out of memory / scratch too small";
+    case ADAPCC_ERR_TIMEOUT: return "watchdog timeout (a peer never posted)";
+    case ADAPCC_ERR_MISMATCH: return "mismatched collective call";
+  }
+  return "unknown error";
+}
+
+adapcc_result_t adapcc_init_loopback(adapcc_comm_t* comm, int nranks, int cuda_device,
+                                     size_t scratch_bytes, adapcc_mode_t mode) {
+  if (!comm || nranks < 1 || nranks > ADAPCC_MAX_RANKS) return ADAPCC_ERR_INVALID_ARGUMENT;
+  if (mode != ADAPCC_MODE_DIRECT && mode != ADAPCC_MODE_STAGED) return ADAPCC_ERR_INVALID_ARGUMENT;
+  *comm = nullptr;
+  auto* c = new adapcc_comm_s();
+  c->nranks = nranks;
+  c->rank = 0;
+  c->device = cuda_device;
+  c->loopback = true;
+  c->mode = (Mode)mode;
+  adapcc_result_t r = common_init(c, scratch_bytes == 0 ? (size_t(64) << 20) : scratch_bytes);
+  if (r != ADAPCC_SUCCESS) { release(c); return r; }
+  if (cudaMalloc(&c->own_arena, c->arena_bytes * nranks) != cudaSuccess) { release(c); return ADAPCC_ERR_OOM; }
+  if (cudaMemset(c->own_arena, 0, c->arena_bytes * nranks) != cudaSuccess ||
+      cudaDeviceSynchronize() != cudaSuccess) { release(c); return ADAPCC_ERR_CUDA; }
+  for (int q = 0; q < nranks; ++q) c->arena.push_back(c->own_arena + q * c->arena_bytes);
+  *comm = c;
+  return ADAPCC_SUCCESS;
+}
+
+adapcc_result_t adapcc_init(adapcc_comm_t* comm, int rank, int nranks, int cuda_device,
+                            size_t scratch_bytes, adapcc_bootstrap_allgather_fn ag, void* ag_ctx) {
+  if (!comm || !ag || nranks < 1 || nranks > ADAPCC_MAX_RANKS || rank < 0 || rank >= nranks)
+    return ADAPCC_ERR_INVALID_ARGUMENT;
+  *comm = nullptr;
+  auto* c = new adapcc_comm_s();
+  c->nranks = nranks;
+  c->rank = rank;
+  c->device = cuda_device;
+  c->loopback = false;
+  c->mode = kStaged;
+  adapcc_result_t r = common_init(c, scratch_bytes);
+  if (r != ADAPCC_SUCCESS) { release(c); return r; }
+  c->arena.assign(nranks, nullptr);
+  char* mine = nullptr;
+  if (cudaMalloc(&mine, c->arena_bytes) != cudaSuccess) { release(c); return ADAPCC_ERR_OOM; }
+  c->arena[rank] = mine;
+  if (cudaMemset(mine, 0, c->arena_bytes) != cudaSuccess || cudaDeviceSynchronize() != cudaSuccess) {
+    release(c);
+    return ADAPCC_ERR_CUDA;
+  }
+  // handle exchange: the paper's set-up AllGather of IPC handles
+  struct Blob { cudaIpcMemHandle_t h; uint64_t arena_bytes; int32_t nranks, rank; };
+  Blob me{};
+  if (cudaIpcGetMemHandle(&me.h, mine) != cudaSuccess) { release(c); return ADAPCC_ERR_CUDA; }
+  me.arena_bytes = c->arena_bytes;
+  me.nranks = nranks;
+  me.rank = rank;
+  std::vector<Blob> all(nranks);
+  if (ag(&me, all.data(), sizeof(Blob), ag_ctx) != 0) { release(c); return ADAPCC_ERR_BOOTSTRAP; }
+  for (int q = 0; q < nranks; ++q) {
+    if (all[q].nranks != nranks || all[q].rank != q || all[q].arena_bytes != c->arena_bytes) {
+      release(c);
+      return ADAPCC_ERR_MISMATCH;
+    }
+  }
+  for (int q = 0; q < nranks; ++q) {
+    if (q == rank) continue;
+    void* p = nullptr;
+    if (cudaIpcOpenMemHandle(&p, all[q].h, cudaIpcMemLazyEnablePeerAccess) != cudaSuccess) {
+      release(c);
+      return ADAPCC_ERR_CUDA;
+    }
+    c->arena[q] = static_cast<char*>(p);
+  }
+  // second exchange doubles as a barrier: every peer has mapped every arena
+  int ok = 1;
+  std::vector<int> oks(nranks);
+  if (ag(&ok, oks.data(), sizeof(int), ag_ctx) != 0) { release(c); return ADAPCC_ERR_BOOTSTRAP; }
+  *comm = c;
+  return ADAPCC_SUCCESS;
+}
+
+adapcc_result_t adapcc_set_strategy(adapcc_comm_t c, adapcc_coll_t coll, const char* text,
+                                    adapcc_stream_t stream) {
+  (void)stream;
+  if (!c || coll < ADAPCC_ALLREDUCE || coll > ADAPCC_ALLTOALL) return ADAPCC_ERR_INVALID_ARGUMENT;
+  Strategy st;
+  std::string err;
+  if (!parse_strategy(text, &st, &err)) return ADAPCC_ERR_INVALID_STRATEGY;
+  if (st.nranks != c->nranks || (int)st.coll != (int)coll) return ADAPCC_ERR_INVALID_STRATEGY;
+  std::lock_guard<std::mutex> lock(c->mu);
+  c->strat[coll] = std::move(st);
+  c->strat_version[coll] += 1;
+  return ADAPCC_SUCCESS;
+}
+
+adapcc_result_t adapcc_allreduce(adapcc_comm_t c, const void* sendbuf, void* recvbuf, size_t count,
+                                 adapcc_dtype_t dtype, uint64_t mask, unsigned flags,
+                                 adapcc_stream_t stream) {
+  adapcc_result_t r = check_common(c, dtype, mask);
+  if (r != ADAPCC_SUCCESS) return r;
+  if (c->loopback || (flags & ~ADAPCC_FLAG_ACCUMULATE)) return ADAPCC_ERR_INVALID_ARGUMENT;
+  const size_t bytes = count * esize_of(dtype);
+  if (count && !recvbuf) return ADAPCC_ERR_INVALID_ARGUMENT;
+  const bool ready = (mask >> c->rank) & 1;
+  if (count && ready && !sendbuf) return ADAPCC_ERR_INVALID_ARGUMENT;
+  if (misaligned(recvbuf) || (ready && misaligned(sendbuf))) return ADAPCC_ERR_INVALID_ARGUMENT;
+  if (ready && sendbuf != recvbuf && overlap(sendbuf, bytes, recvbuf, bytes)) return ADAPCC_ERR_INVALID_ARGUMENT;
+  const void* s[1] = {ready ? sendbuf : recvbuf};
+  void* d[1] = {recvbuf};
+  return run(c, kAllReduce, s, d, count, dtype, mask, flags, stream);
+}
+
+adapcc_result_t adapcc_allgather(adapcc_comm_t c, const void* sendbuf, void* recvbuf,
+                                 size_t sendcount, adapcc_dtype_t dtype, uint64_t mask,
+                                 adapcc_stream_t stream) {
+  adapcc_result_t r = check_common(c, dtype, mask);
+  if (r != ADAPCC_SUCCESS) return r;
+  if (c->loopback) return ADAPCC_ERR_INVALID_ARGUMENT;
+  const size_t es = esize_of(dtype), bytes = sendcount * es;
+  const bool ready = (mask >> c->rank) & 1;
+  if (sendcount && (!recvbuf || (ready && !sendbuf))) return ADAPCC_ERR_INVALID_ARGUMENT;
+  if (misaligned(recvbuf) || (ready && misaligned(sendbuf))) return ADAPCC_ERR_INVALID_ARGUMENT;
+  if (ready && overlap(sendbuf, bytes, recvbuf, bytes * c->nranks) &&
+      sendbuf != static_cast<char*>(recvbuf) + c->rank * bytes)
+    return ADAPCC_ERR_INVALID_ARGUMENT;
+  const void* s[1] = {ready ? sendbuf : recvbuf};
+  void* d[1] = {recvbuf};
+  return run(c, kAllGather, s, d, sendcount, dtype, mask, 0, stream);
+}
+
+adapcc_result_t adapcc_alltoall(adapcc_comm_t c, const void* sendbuf, void* recvbuf,
+                                size_t count_per_peer, adapcc_dtype_t dtype, uint64_t mask,
+                                adapcc_stream_t stream) {
+  adapcc_result_t r = check_common(c, dtype, mask);
+  if (r != ADAPCC_SUCCESS) return r;
+  if (c->loopback) return ADAPCC_ERR_INVALID_ARGUMENT;
+  const size_t bytes = count_per_peer * esize_of(dtype) * c->nranks;
+  const bool ready = (mask >> c->rank) & 1;
+  if (count_per_peer && (!recvbuf || (ready && !sendbuf))) return ADAPCC_ERR_INVALID_ARGUMENT;
+  if (misaligned(recvbuf) || (ready && misaligned(sendbuf))) return ADAPCC_ERR_INVALID_ARGUMENT;
+  if (ready && bytes && overlap(sendbuf, bytes, recvbuf, bytes)) return ADAPCC_ERR_INVALID_ARGUMENT;
+  const void* s[1] = {ready ? sendbuf : recvbuf};
+  void* d[1] = {recvbuf};
+  return run(c, kAllToAll, s, d, count_per_peer, dtype, mask, 0, stream);
+}
+
+static adapcc_result_t check_lb(adapcc_comm_t c, const void* const* s, void* const* d, size_t sbytes,
+                                size_t rbytes, uint64_t mask, int kind) {
+  if (!c->loopback || !s || !d) return ADAPCC_ERR_INVALID_ARGUMENT;
+  for (int q = 0; q < c->nranks; ++q) {
+    const bool ready = (mask >> q) & 1;
+    if (rbytes && !d[q]) return ADAPCC_ERR_INVALID_ARGUMENT;
+    if (misaligned(d[q])) return ADAPCC_ERR_INVALID_ARGUMENT;
+    if (!ready) continue;
+    if (sbytes && !s[q]) return ADAPCC_ERR_INVALID_ARGUMENT;
+    if (misaligned(s[q])) return ADAPCC_ERR_INVALID_ARGUMENT;
+    if (!sbytes) continue;
+    const bool in_place_ok = (kind == 0 && s[q] == d[q]) ||
+                             (kind == 1 && s[q] == static_cast<const char*>(d[q]) + q * sbytes);
+    if (!in_place_ok && overlap(s[q], sbytes, d[q], rbytes)) return ADAPCC_ERR_INVALID_ARGUMENT;
+  }
+  return ADAPCC_SUCCESS;
+}
+
+adapcc_result_t adapcc_allreduce_lb(adapcc_comm_t c, const void* const* sendbufs,
+                                    void* const* recvbufs, size_t count, adapcc_dtype_t dtype,
+                                    uint64_t mask, unsigned flags, adapcc_stream_t stream) {
+  adapcc_result_t r = check_common(c, dtype, mask);
+  if (r != ADAPCC_SUCCESS) return r;
+  if (flags & ~ADAPCC_FLAG_ACCUMULATE) return ADAPCC_ERR_INVALID_ARGUMENT;
+  const size_t bytes = count * esize_of(dtype);
+  r = check_lb(c, sendbufs, recvbufs, bytes, bytes, mask, 0);
+  if (r != ADAPCC_SUCCESS) return r;
+  return run(c, kAllReduce, sendbufs, recvbufs, count, dtype, mask, flags, stream);
+}
+
+adapcc_result_t adapcc_allgather_lb(adapcc_comm_t c, const void* const* sendbufs,
+                                    void* const* recvbufs, size_t sendcount, adapcc_dtype_t dtype,
+                                    uint64_t mask, adapcc_stream_t stream) {
+  adapcc_result_t r = check_common(c, dtype, mask);
+  if (r != ADAPCC_SUCCESS) return r;
+  const size_t bytes = sendcount * esize_of(dtype);
+  r = check_lb(c, sendbufs, recvbufs, bytes, bytes * c->nranks, mask, 1);
+  if (r != ADAPCC_SUCCESS) return r;
+  return run(c, kAllGather, sendbufs, recvbufs, sendcount, dtype, mask, 0, stream);
+}
+
+adapcc_result_t adapcc_alltoall_lb(adapcc_comm_t c, const void* const* sendbufs,
+                                   void* const* recvbufs, size_t count_per_peer,
+                                   adapcc_dtype_t dtype, uint64_t mask, adapcc_stream_t stream) {
+  adapcc_result_t r = check_common(c, dtype, mask);
+  if (r != ADAPCC_SUCCESS) return r;
+  const size_t bytes = count_per_peer * esize_of(dtype) * c->nranks;
+  r = check_lb(c, sendbufs, recvbufs, bytes, bytes, mask, 2);
+  if (r != ADAPCC_SUCCESS) return r;
+  return run(c, kAllToAll, sendbufs, recvbufs, count_per_peer, dtype, mask, 0, stream);
+}
+
+adapcc_result_t adapcc_get_async_error(adapcc_comm_t c) {
+  if (!c) return ADAPCC_ERR_INVALID_ARGUMENT;
+  return (adapcc_result_t) * reinterpret_cast<volatile int*>(c->h_err);
+}
+
+adapcc_result_t adapcc_finalize(adapcc_comm_t c) {
+  release(c);
+  return ADAPCC_SUCCESS;
+}
+
+adapcc_result_t adapcc_config(adapcc_comm_t c, const char* key, int64_t value) {
+  if (!c || !key) return ADAPCC_ERR_INVALID_ARGUMENT;
+  std::lock_guard<std::mutex> lock(c->mu);
+  if (!std::strcmp(key, "timeout_ms")) { if (value < 1) return ADAPCC_ERR_INVALID_ARGUMENT; c->timeout_ms = value; }
+  else if (!std::strcmp(key, "max_ctas")) { if (value < 0) return ADAPCC_ERR_INVALID_ARGUMENT; c->max_ctas = value; }
+  else if (!std::strcmp(key, "debug_drop_rank")) {
+    if (!c->loopback || value < -1 || value >= c->nranks) return ADAPCC_ERR_INVALID_ARGUMENT;
+    c->drop_rank = value;
+  } else return ADAPCC_ERR_INVALID_ARGUMENT;
+  return ADAPCC_SUCCESS;
+}
+
+adapcc_result_t adapcc_launch_count(adapcc_comm_t c, uint64_t* count) {
+  if (!c || !count) return ADAPCC_ERR_INVALID_ARGUMENT;
+  *count = c->launches;
+  return ADAPCC_SUCCESS;
+}
+
+// ----------------------------------------------------------- host-only inspection
+adapcc_result_t adapcc_strategy_check(const char* text, int* nranks, int* coll, int* nsubs,
+                                      char* err, size_t err_len) {
+  Strategy st;
+  std::string e;
+  if (!parse_strategy(text, &st, &e)) {
+    if (err && err_len) {
+      std::strncpy(err, e.c_str(), err_len - 1);
+      err[err_len - 1] = 0;
+    }
+    return ADAPCC_ERR_INVALID_STRATEGY;
+  }
+  if (nranks) *nranks = st.nranks;
+  if (coll) *coll = (int)st.coll;
+  if (nsubs) *nsubs = (int)st.subs.size();
+  return ADAPCC_SUCCESS;
+}
+
+adapcc_result_t adapcc_strategy_tuples(const char* text, int sub, uint64_t mask, uint8_t* tuples,
+                                       int32_t* nflows) {
+  Strategy st;
+  if (!parse_strategy(text, &st, nullptr)) return ADAPCC_ERR_INVALID_STRATEGY;
+  if (sub < 0 || sub >= (int)st.subs.size() || st.subs[sub].kind != kTree || !tuples)
+    return ADAPCC_ERR_INVALID_ARGUMENT;
+  TreeBehavior b = tree_behavior(st.subs[sub], mask);
+  for (int g = 0; g < st.nranks; ++g) {
+    tuples[4 * g + 0] = b.tup[g].act;
+    tuples[4 * g + 1] = b.tup[g].recv;
+    tuples[4 * g + 2] = b.tup[g].kern;
+    tuples[4 * g + 3] = b.tup[g].send;
+    if (nflows) nflows[g] = (int32_t)b.flows[g].size();
+  }
+  return ADAPCC_SUCCESS;
+}
+
+adapcc_result_t adapcc_strategy_sub(const char* text, int sub, int64_t* weight, int64_t* chunk,
+                                    int32_t* parent, int32_t* src) {
+  Strategy st;
+  if (!parse_strategy(text, &st, nullptr)) return ADAPCC_ERR_INVALID_STRATEGY;
+  if (sub < 0 || sub >= (int)st.subs.size()) return ADAPCC_ERR_INVALID_ARGUMENT;
+  const SubColl& s = st.subs[sub];
+  if (weight) *weight = s.weight;
+  if (chunk) *chunk = s.chunk;
+  if (src) *src = s.src;
+  if (parent)
+    for (int g = 0; g < st.nranks; ++g) parent[g] = s.parent.empty() ? -2 : s.parent[g];
+  return ADAPCC_SUCCESS;
+}
+
+adapcc_result_t adapcc_strategy_partition(const char* text, uint64_t count, adapcc_dtype_t dtype,
+                                          int src, uint64_t* bounds, int* nbounds) {
+  Strategy st;
+  if (!parse_strategy(text, &st, nullptr)) return ADAPCC_ERR_INVALID_STRATEGY;
+  if (!bounds || !nbounds) return ADAPCC_ERR_INVALID_ARGUMENT;
+  std::vector<int64_t> w;
+  for (auto& s : st.subs)
+    if (st.coll != kAllGather || s.src == src) w.push_back(s.weight);
+  if (w.empty()) return ADAPCC_ERR_INVALID_ARGUMENT;
+  auto b = partition(count, esize_of(dtype), w);
+  for (size_t i = 0; i < b.size(); ++i) bounds[i] = b[i];
+  *nbounds = (int)b.size();
+  return ADAPCC_SUCCESS;
+}
+
+adapcc_result_t adapcc_plan_stats(const char* text, uint64_t count, adapcc_dtype_t dtype,
+                                  uint64_t mask, unsigned flags, adapcc_mode_t mode, int rank,
+                                  size_t scratch_bytes, adapcc_plan_stats_t* out) {
+  Strategy st;
+  if (!parse_strategy(text, &st, nullptr)) return ADAPCC_ERR_INVALID_STRATEGY;
+  if (!out || rank < -1 || rank >= st.nranks) return ADAPCC_ERR_INVALID_ARGUMENT;
+  PlanRequest rq;
+  rq.st = &st;
+  rq.count = count;
+  rq.esize = esize_of(dtype);
+  rq.ready_mask = mask;
+  rq.accumulate = flags & ADAPCC_FLAG_ACCUMULATE;
+  rq.mode = (Mode)mode;
+  const size_t scratch = scratch_bytes ? scratch_bytes : kDefaultScratch;
+  if (scratch < (size_t)kArenaHeader + 2 * (4096 + 65536)) return ADAPCC_ERR_INVALID_ARGUMENT;
+  rq.half_bytes = ((scratch - kArenaHeader) / 2) / 256 * 256;
+  std::vector<SegmentPlan> segs;
+  if (!build_plan(rq, &segs, nullptr)) return ADAPCC_ERR_OOM;
+  PlanStats s;
+  for (auto& p : segs) accumulate_stats(p, rank, rq.esize, &s);
+  s.segments = segs.size();
+  out->tasks = s.tasks;
+  out->items = s.items;
+  out->levels = s.levels;
+  out->segments = s.segments;
+  out->bytes_read = s.bytes_read;
+  out->bytes_written = s.bytes_written;
+  out->remote_bytes = s.remote_bytes;
+  out->arena_bytes = s.arena_bytes;
+  return ADAPCC_SUCCESS;
+}
+
+}  // extern "C"

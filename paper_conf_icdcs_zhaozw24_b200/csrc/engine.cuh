@@ -1,0 +1,63 @@
+// Device-visible plan tables of the AdapCC transfer engine.
+//
+// A call is compiled on the host (plan.cpp) into FOLD tasks: "wait for these
+// per-chunk flags, fold K source streams left to right, write the result to D
+// destination streams (some accumulating), post these per-chunk flags".  Every
+// step of the paper's executor maps onto one task kind:
+//   - aggregation kernel at a node with hasKernel: K >= 2
+//   - chunk send / relay forward: K = 1
+//   - root hand-off + broadcast "reversely": K = 1, D >= 1
+// A work item is one (task, chunk); items are ordered by (chunk + level,
+// level, task) so that every wait targets an item earlier in the order, which
+// makes the dynamic fetch deadlock-free.
+#pragma once
+
+#include <cstdint>
+
+namespace adapcc {
+
+constexpr int kMaxFold = 64;   // max sources of one fold (<= ranks)
+constexpr int kMaxDst = 65;    // max destinations of one task (<= ranks + 1)
+constexpr int kArenaHeader = 4096;  // per-rank arena header (done epoch)
+
+enum BufKind : uint8_t { kBufSend = 0, kBufRecv = 1, kBufArena = 2 };
+enum DType : int { kF32 = 0, kBF16 = 1, kI32 = 2 };
+enum TaskOp : uint16_t { kOpFold = 0, kOpZero = 1 };
+
+// address(e) = base(kind, rank) + bias + e * esize, e = element index in the
+// task's coordinate system.
+struct BufRef {
+  int64_t bias;
+  uint8_t kind;
+  uint8_t rank;
+  uint8_t accum;   // destination: recv += value (ACCUMULATE)
+  uint8_t pad[5];
+};
+static_assert(sizeof(BufRef) == 16, "BufRef layout");
+
+// per-chunk flag word: arena(rank) + off + 8 * chunk (inside the parity half)
+struct FlagRef {
+  uint64_t off;
+  uint32_t rank;
+  uint32_t pad;
+};
+static_assert(sizeof(FlagRef) == 16, "FlagRef layout");
+
+struct Task {
+  uint64_t lo, hi;          // element range covered by the task
+  uint32_t chunk_elems;     // C_m / esize
+  uint32_t nchunks;
+  uint16_t nsrc, ndst, nwait, npost;
+  uint32_t ref0;            // refs[ref0 .. ref0+nsrc) sources, then ndst destinations
+  uint32_t flag0;           // flags[flag0 .. +nwait) waits, then npost posts
+  uint32_t level;
+  uint16_t op;
+  uint16_t owner;           // executing rank
+};
+
+struct Item {
+  uint32_t task;
+  uint32_t chunk;
+};
+
+}  // namespace adapcc

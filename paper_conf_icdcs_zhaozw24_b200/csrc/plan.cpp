@@ -1,0 +1,440 @@
+// Plan compiler (see plan.hpp).  Data movement per collective and mode:
+//
+// AllReduce, tree m over [lo,hi) ("generate strategies for Reduce and
+// execute Broadcast reversely"):
+//   DIRECT  kernel node k (non-root): fold(sources(k)) -> slot_k, post flag_k
+//           root: fold(sources(root)) (or its single flow / zero) -> every
+//           rank's recvbuf (the broadcast collapses to one write per rank
+//           because every recvbuf is addressable).
+//   STAGED  every flow is pushed by its producer into a landing slot in the
+//           arena of its consumer (the kernel node that folds it, P:L263
+//           "send one chunk ... an event is then recorded"); the root folds
+//           into its own recvbuf and its broadcast slot; every other rank
+//           pulls the result from its tree parent's broadcast slot into its
+//           recvbuf and, if it has children, into its own broadcast slot
+//           (the reversed tree, pipelined per chunk).
+//   Pure relays forward by reference: their single incoming flow is
+//   pushed straight to their consumer, because on a uniform NVSwitch a
+//   store-and-forward hop adds bytes on the relay's ports without adding link
+//   capacity.  Relays still receive the result (Q4).
+// AllGather: one broadcast tree per source.
+// AlltoAll: direct routes; block d of s lands in block s of d.
+#include "plan.hpp"
+
+#include <algorithm>
+#include <map>
+#include <tuple>
+
+namespace adapcc {
+namespace {
+
+constexpr uint64_t kAlign = 256;
+
+uint64_t align_up(uint64_t v, uint64_t a) { return (v + a - 1) / a * a; }
+
+struct Stream {
+  BufRef ref{};
+  bool wait = false;
+  FlagRef flag{};
+};
+
+BufRef make_ref(uint8_t kind, int rank, int64_t bias, bool accum = false) {
+  BufRef r{};
+  r.bias = bias;
+  r.kind = kind;
+  r.rank = (uint8_t)rank;
+  r.accum = accum ? 1 : 0;
+  return r;
+}
+
+class Builder {
+ public:
+  Builder(int n, int esize, uint64_t half)
+      : n_(n), esize_(esize), half_(half), flag_cap_(flag_region_bytes(half)),
+        used_(n, 0), flags_used_(n, 0) {}
+
+  // Each parity half of a rank's arena = [flag region | data region].  Flag
+  // words only ever hold epochs (monotonic), so a later plan with a different
+  // layout can never mistake an old data byte for a posted flag.
+  uint64_t alloc(int r, uint64_t bytes) {
+    uint64_t off = flag_cap_ + used_[r];
+    used_[r] = align_up(used_[r] + bytes, kAlign);
+    return off;
+  }
+  FlagRef alloc_flags(int r, uint32_t nchunks) {
+    FlagRef f{};
+    f.off = flags_used_[r];
+    flags_used_[r] = align_up(flags_used_[r] + 8ull * nchunks, 128);
+    f.rank = (uint32_t)r;
+    return f;
+  }
+  bool fits() const {
+    for (int r = 0; r < n_; ++r)
+      if (flags_used_[r] > flag_cap_ || flag_cap_ + used_[r] > half_) return false;
+    return true;
+  }
+
+  // Slot holding elements [lo,hi) of a stream at rank r: address(e) = base + off + (e-lo)*esize
+  Stream slot_stream(int r, uint64_t off, uint64_t lo, const FlagRef* f) {
+    Stream s;
+    s.ref = make_ref(kBufArena, r, (int64_t)off - (int64_t)(lo * esize_));
+    if (f) { s.wait = true; s.flag = *f; }
+    return s;
+  }
+
+  int add(int owner, uint64_t lo, uint64_t hi, uint32_t ce, uint16_t op,
+          const std::vector<Stream>& srcs, const std::vector<BufRef>& dsts,
+          const std::vector<FlagRef>& posts) {
+    Task t{};
+    t.lo = lo;
+    t.hi = hi;
+    t.chunk_elems = ce;
+    t.nchunks = (uint32_t)((hi - lo + ce - 1) / ce);
+    t.nsrc = (uint16_t)srcs.size();
+    t.ndst = (uint16_t)dsts.size();
+    t.op = op;
+    t.owner = (uint16_t)owner;
+    t.ref0 = (uint32_t)p_.refs.size();
+    for (auto& s : srcs) p_.refs.push_back(s.ref);
+    for (auto& d : dsts) p_.refs.push_back(d);
+    t.flag0 = (uint32_t)p_.flags.size();
+    uint32_t level = 0;
+    uint16_t nwait = 0;
+    for (auto& s : srcs) {
+      if (!s.wait) continue;
+      p_.flags.push_back(s.flag);
+      ++nwait;
+      auto it = producer_.find({s.flag.rank, s.flag.off});
+      if (it != producer_.end()) level = std::max(level, p_.tasks[it->second].level + 1);
+    }
+    t.nwait = nwait;
+    for (auto& f : posts) p_.flags.push_back(f);
+    t.npost = (uint16_t)posts.size();
+    t.level = level;
+    const int idx = (int)p_.tasks.size();
+    for (auto& f : posts) producer_[{f.rank, f.off}] = idx;
+    p_.tasks.push_back(t);
+    p_.max_level = std::max(p_.max_level, level);
+    return idx;
+  }
+
+  SegmentPlan finish() {
+    p_.fits = fits();
+    p_.arena_used.resize(n_);
+    for (int r = 0; r < n_; ++r) p_.arena_used[r] = flag_cap_ + used_[r];
+    return std::move(p_);
+  }
+
+  int n_, esize_;
+  uint64_t half_, flag_cap_;
+  std::vector<uint64_t> used_, flags_used_;
+  SegmentPlan p_;
+  std::map<std::pair<uint32_t, uint64_t>, int> producer_;
+};
+
+std::vector<int> bfs_order(const SubColl& s) {
+  std::vector<int> q = {s.root};
+  for (size_t i = 0; i < q.size(); ++i)
+    for (int c : s.children[q[i]]) q.push_back(c);
+  return q;
+}
+
+// ------------------------------------------------------------- AllReduce
+void plan_allreduce_tree(Builder& B, const SubColl& s, uint64_t lo, uint64_t hi, uint64_t mask,
+                         bool accumulate, Mode mode) {
+  const int n = B.n_;
+  const int es = B.esize_;
+  const uint32_t ce = (uint32_t)(s.chunk / es);
+  const uint32_t nch = (uint32_t)((hi - lo + ce - 1) / ce);
+  const uint64_t len = (hi - lo) * es;
+  const TreeBehavior b = tree_behavior(s, mask);
+  const int root = s.root;
+
+  // sources folded at the root (kernel) or its single flow (no kernel)
+  std::vector<Flow> root_src =
+      b.tup[root].kern ? kernel_sources(s, b, root) : b.flows[root];
+  const bool zero = root_src.empty();
+  if (zero && accumulate) return;  // recvbuf untouched (reading Q7)
+
+  std::vector<BufRef> recv_all;
+  for (int g = 0; g < n; ++g) recv_all.push_back(make_ref(kBufRecv, g, 0, accumulate));
+
+  if (mode == kDirect) {
+    std::map<int, std::pair<uint64_t, FlagRef>> agg_slot;  // kernel node -> slot
+    auto stream_of = [&](const Flow& f) {
+      if (f.kind == Flow::kIn) { Stream st; st.ref = make_ref(kBufSend, f.rank, 0); return st; }
+      auto& as = agg_slot.at(f.rank);
+      return B.slot_stream(f.rank, as.first, lo, &as.second);
+    };
+    for (int k : b.postorder) {
+      if (!b.tup[k].kern || k == root) continue;
+      uint64_t off = B.alloc(k, len);
+      FlagRef fl = B.alloc_flags(k, nch);
+      agg_slot[k] = {off, fl};
+      std::vector<Stream> srcs;
+      for (auto& f : kernel_sources(s, b, k)) srcs.push_back(stream_of(f));
+      B.add(k, lo, hi, ce, kOpFold, srcs,
+            {make_ref(kBufArena, k, (int64_t)off - (int64_t)(lo * es))}, {fl});
+    }
+    std::vector<Stream> srcs;
+    for (auto& f : root_src) srcs.push_back(stream_of(f));
+    B.add(root, lo, hi, ce, zero ? kOpZero : kOpFold, srcs, recv_all, {});
+    return;
+  }
+
+  // STAGED: consumers and their landing slots
+  struct Dest { int rank; uint64_t off; FlagRef flag; };
+  std::map<std::pair<int, int>, Dest> dest_of;  // (flow kind, rank) -> landing at consumer
+  std::map<int, std::vector<Stream>> consumer_srcs;
+  std::vector<int> consumers;
+  for (int k : b.postorder)
+    if (b.tup[k].kern && k != root) consumers.push_back(k);
+  consumers.push_back(root);
+  for (int c : consumers) {
+    const std::vector<Flow> L = (c == root) ? root_src : kernel_sources(s, b, c);
+    std::vector<Stream> srcs;
+    for (const Flow& f : L) {
+      if (f.kind == Flow::kIn && f.rank == c) {
+        Stream st;
+        st.ref = make_ref(kBufSend, c, 0);
+        srcs.push_back(st);
+        continue;
+      }
+      uint64_t off = B.alloc(c, len);
+      FlagRef fl = B.alloc_flags(c, nch);
+      dest_of[{(int)f.kind, f.rank}] = {c, off, fl};
+      srcs.push_back(B.slot_stream(c, off, lo, &fl));
+    }
+    consumer_srcs[c] = std::move(srcs);
+  }
+  // pushes of ready ranks' own tensors (leaves, a=0 nodes, relayed flows)
+  for (auto& kv : dest_of) {
+    if (kv.first.first != Flow::kIn) continue;
+    const int r = kv.first.second;
+    const Dest& d = kv.second;
+    Stream src;
+    src.ref = make_ref(kBufSend, r, 0);
+    B.add(r, lo, hi, ce, kOpFold, {src},
+          {make_ref(kBufArena, d.rank, (int64_t)d.off - (int64_t)(lo * es))}, {d.flag});
+  }
+  // aggregation kernels (post-order: producers first)
+  for (int k : consumers) {
+    if (k == root) continue;
+    const Dest& d = dest_of.at({(int)Flow::kAgg, k});
+    B.add(k, lo, hi, ce, kOpFold, consumer_srcs[k],
+          {make_ref(kBufArena, d.rank, (int64_t)d.off - (int64_t)(lo * es))}, {d.flag});
+  }
+  // root hand-off: own recvbuf + broadcast slot
+  std::map<int, std::pair<uint64_t, FlagRef>> down;
+  auto add_down_dst = [&](int g, std::vector<BufRef>* dsts, std::vector<FlagRef>* posts) {
+    if (s.children[g].empty()) return;
+    uint64_t off = B.alloc(g, len);
+    FlagRef fl = B.alloc_flags(g, nch);
+    down[g] = {off, fl};
+    dsts->push_back(make_ref(kBufArena, g, (int64_t)off - (int64_t)(lo * es)));
+    posts->push_back(fl);
+  };
+  {
+    std::vector<BufRef> dsts = {make_ref(kBufRecv, root, 0, accumulate)};
+    std::vector<FlagRef> posts;
+    add_down_dst(root, &dsts, &posts);
+    B.add(root, lo, hi, ce, zero ? kOpZero : kOpFold, consumer_srcs[root], dsts, posts);
+  }
+  // broadcast down the reversed tree, parents before children
+  for (int g : bfs_order(s)) {
+    if (g == root) continue;
+    const int p = s.parent[g];
+    auto& pd = down.at(p);
+    std::vector<Stream> srcs = {B.slot_stream(p, pd.first, lo, &pd.second)};
+    std::vector<BufRef> dsts = {make_ref(kBufRecv, g, 0, accumulate)};
+    std::vector<FlagRef> posts;
+    add_down_dst(g, &dsts, &posts);
+    B.add(g, lo, hi, ce, kOpFold, srcs, dsts, posts);
+  }
+}
+
+// ------------------------------------------------------------- AllGather
+void plan_allgather_tree(Builder& B, const SubColl& s, uint64_t lo, uint64_t hi, uint64_t cnt,
+                         uint64_t mask, Mode mode) {
+  const int n = B.n_;
+  const int es = B.esize_;
+  const int src = s.src;
+  if (!((mask >> src) & 1)) return;  // non-ready source: slots untouched (Q12)
+  const uint32_t ce = (uint32_t)(s.chunk / es);
+  const uint32_t nch = (uint32_t)((hi - lo + ce - 1) / ce);
+  const uint64_t len = (hi - lo) * es;
+  const int64_t slot_bias = (int64_t)(src * cnt * es);
+  Stream in;
+  in.ref = make_ref(kBufSend, src, 0);
+  if (mode == kDirect) {
+    std::vector<BufRef> dsts;
+    for (int g = 0; g < n; ++g) dsts.push_back(make_ref(kBufRecv, g, slot_bias));
+    B.add(src, lo, hi, ce, kOpFold, {in}, dsts, {});
+    return;
+  }
+  std::map<int, std::pair<uint64_t, FlagRef>> down;
+  for (int g : bfs_order(s)) {
+    std::vector<Stream> srcs;
+    if (g == src) {
+      srcs.push_back(in);
+    } else {
+      auto& pd = down.at(s.parent[g]);
+      srcs.push_back(B.slot_stream(s.parent[g], pd.first, lo, &pd.second));
+    }
+    std::vector<BufRef> dsts = {make_ref(kBufRecv, g, slot_bias)};
+    std::vector<FlagRef> posts;
+    if (!s.children[g].empty()) {
+      uint64_t off = B.alloc(g, len);
+      FlagRef fl = B.alloc_flags(g, nch);
+      down[g] = {off, fl};
+      dsts.push_back(make_ref(kBufArena, g, (int64_t)off - (int64_t)(lo * es)));
+      posts.push_back(fl);
+    }
+    B.add(g, lo, hi, ce, kOpFold, srcs, dsts, posts);
+  }
+}
+
+// -------------------------------------------------------------- AlltoAll
+void plan_alltoall_line(Builder& B, const SubColl& s, uint64_t lo, uint64_t hi, uint64_t cnt,
+                        uint64_t mask, Mode mode) {
+  const int n = B.n_;
+  const int es = B.esize_;
+  const uint32_t ce = (uint32_t)(s.chunk / es);
+  const uint32_t nch = (uint32_t)((hi - lo + ce - 1) / ce);
+  const uint64_t len = (hi - lo) * es;
+  for (int src = 0; src < n; ++src) {
+    if (!((mask >> src) & 1)) continue;
+    for (int d = 0; d < n; ++d) {
+      Stream in;
+      in.ref = make_ref(kBufSend, src, (int64_t)(d * cnt * es));
+      BufRef out = make_ref(kBufRecv, d, (int64_t)(src * cnt * es));
+      if (mode == kDirect || d == src) {
+        B.add(src, lo, hi, ce, kOpFold, {in}, {out}, {});
+        continue;
+      }
+      uint64_t off = B.alloc(d, len);
+      FlagRef fl = B.alloc_flags(d, nch);
+      B.add(src, lo, hi, ce, kOpFold, {in},
+            {make_ref(kBufArena, d, (int64_t)off - (int64_t)(lo * es))}, {fl});
+      B.add(d, lo, hi, ce, kOpFold, {B.slot_stream(d, off, lo, &fl)}, {out}, {});
+    }
+  }
+}
+
+SegmentPlan build_segment(const PlanRequest& rq,
+                          const std::vector<std::pair<uint64_t, uint64_t>>& ranges) {
+  const Strategy& st = *rq.st;
+  Builder B(st.nranks, rq.esize, rq.half_bytes);
+  for (size_t m = 0; m < st.subs.size(); ++m) {
+    const uint64_t lo = ranges[m].first, hi = ranges[m].second;
+    if (lo >= hi) continue;
+    const SubColl& s = st.subs[m];
+    if (st.coll == kAllReduce)
+      plan_allreduce_tree(B, s, lo, hi, rq.ready_mask, rq.accumulate, rq.mode);
+    else if (st.coll == kAllGather)
+      plan_allgather_tree(B, s, lo, hi, rq.count, rq.ready_mask, rq.mode);
+    else
+      plan_alltoall_line(B, s, lo, hi, rq.count, rq.ready_mask, rq.mode);
+  }
+  return B.finish();
+}
+
+}  // namespace
+
+uint64_t flag_region_bytes(uint64_t half) {
+  uint64_t f = half / 32 / 256 * 256;
+  return std::min<uint64_t>(std::max<uint64_t>(f, 4096), uint64_t(32) << 20);
+}
+
+std::vector<std::pair<uint64_t, uint64_t>> sub_ranges(const Strategy& st, uint64_t count,
+                                                      int esize) {
+  std::vector<std::pair<uint64_t, uint64_t>> r(st.subs.size());
+  if (st.coll == kAllGather) {
+    for (int src = 0; src < st.nranks; ++src) {
+      std::vector<int64_t> w;
+      std::vector<size_t> idx;
+      for (size_t m = 0; m < st.subs.size(); ++m)
+        if (st.subs[m].src == src) { w.push_back(st.subs[m].weight); idx.push_back(m); }
+      auto b = partition(count, esize, w);
+      for (size_t i = 0; i < idx.size(); ++i) r[idx[i]] = {b[i], b[i + 1]};
+    }
+    return r;
+  }
+  std::vector<int64_t> w;
+  for (auto& s : st.subs) w.push_back(s.weight);
+  auto b = partition(count, esize, w);
+  for (size_t m = 0; m < st.subs.size(); ++m) r[m] = {b[m], b[m + 1]};
+  return r;
+}
+
+bool build_plan(const PlanRequest& rq, std::vector<SegmentPlan>* segs, std::string* err) {
+  segs->clear();
+  const auto full = sub_ranges(*rq.st, rq.count, rq.esize);
+  const uint64_t unit = 16 / rq.esize;
+  for (uint64_t nseg = 1;; nseg *= 2) {
+    std::vector<SegmentPlan> out;
+    bool fits = true;
+    uint64_t max_step = 0;
+    for (uint64_t k = 0; k < nseg && fits; ++k) {
+      std::vector<std::pair<uint64_t, uint64_t>> rr(full.size());
+      for (size_t m = 0; m < full.size(); ++m) {
+        const uint64_t lo = full[m].first, hi = full[m].second;
+        const uint64_t step = align_up((hi - lo + nseg - 1) / nseg, unit);
+        max_step = std::max(max_step, step);
+        const uint64_t a = std::min(hi, lo + k * step), b = std::min(hi, lo + (k + 1) * step);
+        rr[m] = {a, b};
+      }
+      SegmentPlan p = build_segment(rq, rr);
+      fits = fits && p.fits;
+      if (!p.tasks.empty()) out.push_back(std::move(p));
+    }
+    if (fits) {
+      *segs = std::move(out);
+      return true;
+    }
+    if (max_step <= unit) {  // cannot split further
+      if (err) *err = "scratch arena too small for this strategy";
+      return false;
+    }
+  }
+}
+
+std::vector<Item> order_items(const SegmentPlan& p, int rank) {
+  struct Key { uint64_t a; uint32_t level, task, chunk; };
+  std::vector<Key> keys;
+  for (uint32_t t = 0; t < p.tasks.size(); ++t) {
+    const Task& T = p.tasks[t];
+    if (rank >= 0 && T.owner != rank) continue;
+    for (uint32_t c = 0; c < T.nchunks; ++c) keys.push_back({(uint64_t)c + T.level, T.level, t, c});
+  }
+  std::sort(keys.begin(), keys.end(), [](const Key& x, const Key& y) {
+    return std::tie(x.a, x.level, x.task, x.chunk) < std::tie(y.a, y.level, y.task, y.chunk);
+  });
+  std::vector<Item> items(keys.size());
+  for (size_t i = 0; i < keys.size(); ++i) items[i] = {keys[i].task, keys[i].chunk};
+  return items;
+}
+
+void accumulate_stats(const SegmentPlan& p, int rank, int esize, PlanStats* s) {
+  for (const Task& t : p.tasks) {
+    if (rank >= 0 && t.owner != rank) continue;
+    const uint64_t bytes = (t.hi - t.lo) * esize;
+    s->tasks += 1;
+    s->items += t.nchunks;
+    s->levels = std::max<uint64_t>(s->levels, t.level + 1);
+    for (int i = 0; i < t.nsrc; ++i) {
+      const BufRef& r = p.refs[t.ref0 + i];
+      s->bytes_read += bytes;
+      if (r.rank != t.owner) s->remote_bytes += bytes;
+    }
+    for (int i = 0; i < t.ndst; ++i) {
+      const BufRef& r = p.refs[t.ref0 + t.nsrc + i];
+      s->bytes_written += bytes;
+      if (r.accum) s->bytes_read += bytes;
+      if (r.rank != t.owner) s->remote_bytes += bytes * (r.accum ? 2 : 1);
+    }
+  }
+  for (uint64_t u : p.arena_used) s->arena_bytes = std::max(s->arena_bytes, u);
+}
+
+}  // namespace adapcc

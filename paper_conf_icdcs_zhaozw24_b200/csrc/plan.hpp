@@ -1,0 +1,67 @@
+// Plan compiler: (strategy, ready mask, count, dtype, flags, mode) -> FOLD
+// tasks + per-chunk flags + ordered work items (engine.cuh).
+//
+// This is the B200 replacement of the paper's Executor, which "parses
+// communication strategies ... together with the information of relay workers
+// to generate respective CUDA codes": instead of generating
+// code per behaviour tuple we compile the tuples into a task table that one
+// persistent, parameterised kernel executes.
+#pragma once
+
+#include <cstdint>
+#include <string>
+#include <vector>
+
+#include "engine.cuh"
+#include "strategy.hpp"
+
+namespace adapcc {
+
+enum Mode : int { kDirect = 0, kStaged = 1 };
+
+struct PlanStats {
+  uint64_t tasks = 0, items = 0, levels = 0, segments = 0;
+  uint64_t bytes_read = 0, bytes_written = 0, remote_bytes = 0, arena_bytes = 0;
+};
+
+// One launch worth of work.
+struct SegmentPlan {
+  std::vector<Task> tasks;
+  std::vector<BufRef> refs;
+  std::vector<FlagRef> flags;
+  std::vector<uint64_t> arena_used;  // per rank, bytes inside one parity half
+  uint32_t max_level = 0;
+  bool fits = true;                  // flags and data fit their regions
+};
+
+struct PlanRequest {
+  const Strategy* st = nullptr;
+  uint64_t count = 0;       // allreduce: count; allgather: sendcount; alltoall: per peer
+  int esize = 4;
+  uint64_t ready_mask = 0;
+  bool accumulate = false;
+  Mode mode = kDirect;
+  uint64_t half_bytes = 0;  // arena bytes available per rank per parity half
+};
+
+// Bytes at the start of each parity half reserved for per-chunk flag words.
+uint64_t flag_region_bytes(uint64_t half);
+
+// Builds the segment plans of one call (one per launch; more than one only
+// when the staging slots exceed half_bytes).  Returns false + *err when the
+// call cannot be planned (e.g. arena too small even for 1 unit per segment).
+bool build_plan(const PlanRequest& rq, std::vector<SegmentPlan>* segs, std::string* err);
+
+// Work items of `rank` (-1: all ranks) in deadlock-free order.
+std::vector<Item> order_items(const SegmentPlan& p, int rank);
+
+// Byte accounting for adapcc_plan_stats.
+void accumulate_stats(const SegmentPlan& p, int rank, int esize, PlanStats* s);
+
+// Sub-collective ranges (before segmentation) in the collective's element
+// coordinates: allreduce/alltoall use partition() over all subs; allgather
+// partitions each source's shard over that source's bcast lines.
+std::vector<std::pair<uint64_t, uint64_t>> sub_ranges(const Strategy& st, uint64_t count,
+                                                      int esize);
+
+}  // namespace adapcc

@@ -1,0 +1,189 @@
+"""Strategy generator: emits strategy text v1.
+
+Stand-in for the paper's Synthesizer (§IV-D).  The MILP solved
+with Gurobi is out of scope (NP-hard, licensed solver); the strategy
+is an INPUT of the hot path.  This module produces the families the bench and
+tests use -- star trees, complementary binary trees, rings (chains), per-source
+broadcast trees, direct AlltoAll -- and link-bandwidth / ready-mask weighted
+star trees from the paper's own link-load model applied to one NVSwitch:
+
+  Reduce with aggregation at the root: one flow per (ready sender, tree)
+  (N_{ij} = 1); Broadcast: one flow per edge; the
+  profiled bandwidth of a link is shared by its flows (eq. 3).
+
+For star tree m with weight w_m (fraction of the tensor) under ready set R
+(k = |R|), the bytes each GPU g moves per byte of tensor are
+  egress_g  = [g in R] (1 - w_g) + (n - 1) w_g
+  ingress_g = (k - [g in R]) w_g + (1 - w_g)
+and the generator minimises max_g max(egress_g, ingress_g) / b_g (b_g: the
+GPU's NVLink bandwidth, uniform 900 GB/s by default) -- a small LP.
+"""
+
+DEFAULT_CHUNK = 262144
+
+
+def _header(n, coll):
+    return f"adapcc-strategy 1\nnranks {n}\ncollective {coll}\n"
+
+
+def _join(v):
+    return ",".join(str(int(x)) for x in v)
+
+
+def star_parent(n, root):
+    return [-1 if g == root else root for g in range(n)]
+
+
+def chain_parent(order):
+    """order[0] is the leaf, order[-1] the root."""
+    p = [None] * len(order)
+    for i, g in enumerate(order):
+        p[g] = order[i + 1] if i + 1 < len(order) else -1
+    return p
+
+
+def binary_tree_parent(order):
+    """Heap-shaped binary tree over `order` (order[0] is the root)."""
+    p = [None] * len(order)
+    for i, g in enumerate(order):
+        p[g] = -1 if i == 0 else order[(i - 1) // 2]
+    return p
+
+
+# ------------------------------------------------------------------- allreduce
+def allreduce_trees(parents, weights=None, chunk=DEFAULT_CHUNK, noaggs=None):
+    n = len(parents[0])
+    weights = weights if weights is not None else [1] * len(parents)
+    noaggs = noaggs or [()] * len(parents)
+    out = _header(n, "allreduce")
+    for p, w, na in zip(parents, weights, noaggs):
+        out += f"tree weight={int(w)} chunk={int(chunk)} parent={_join(p)}"
+        if na:
+            out += f" noagg={_join(na)}"
+        out += "\n"
+    return out
+
+
+def allreduce_stars(n, chunk=DEFAULT_CHUNK, roots=None, weights=None):
+    """M star trees rooted at `roots` (default: every rank) -- the B200 analogue
+    of M parallel sub-collectives (M sweep of Fig. 19(a))."""
+    roots = list(range(n)) if roots is None else list(roots)
+    return allreduce_trees([star_parent(n, r) for r in roots], weights, chunk)
+
+
+def allreduce_double_binary(n, chunk=DEFAULT_CHUNK):
+    """Two complementary heap trees (NCCL-style double binary tree)."""
+    a = list(range(n))
+    b = [(g + n // 2) % n for g in range(n)][::-1]
+    return allreduce_trees([binary_tree_parent(a), binary_tree_parent(b)], [1, 1], chunk)
+
+
+def allreduce_ring(n, chunk=DEFAULT_CHUNK, order=None, weight=1):
+    order = list(range(n)) if order is None else list(order)
+    return _header(n, "allreduce") + f"ring weight={int(weight)} chunk={int(chunk)} order={_join(order)}\n"
+
+
+def star_loads(n, ready, w, bw=None):
+    """Per-GPU (egress, ingress) bytes per tensor byte and the max time factor."""
+    ready = set(ready)
+    k = len(ready)
+    bw = bw or [1.0] * n
+    eg = [((g in ready) * (1 - w[g]) + (n - 1) * w[g]) for g in range(n)]
+    ig = [((k - (g in ready)) * w[g] + (1 - w[g])) for g in range(n)]
+    t = max(max(e, i) / b for e, i, b in zip(eg, ig, bw))
+    return eg, ig, t
+
+
+def mask_aware_star_weights(n, ready, bw=None, relays_as_roots=True, scale=1 << 16):
+    """Fractions w_m minimising the max per-GPU time under the load model above.
+
+    relays_as_roots=False forces w = 0 on non-ready roots (relays as leaves);
+    returns (integer weights, fractions, time factor)."""
+    ready = set(ready)
+    bw = bw or [1.0] * n
+    if not ready:
+        w = [1.0 / n] * n
+    else:
+        w = _solve_lp(n, ready, bw, relays_as_roots)
+    ints = [int(round(x * scale)) for x in w]
+    if sum(ints) == 0:
+        ints = [1] * n
+    return ints, w, star_loads(n, ready, w, bw)[2]
+
+
+def _solve_lp(n, ready, bw, relays_as_roots):
+    k = len(ready)
+    try:
+        from scipy.optimize import linprog
+    except ImportError:  # symmetric two-class search (uniform links only)
+        return _two_class(n, ready, relays_as_roots)
+    # variables: w_0..w_{n-1}, t ; minimise t
+    c = [0.0] * n + [1.0]
+    A, b = [], []
+    for g in range(n):
+        a = [0.0] * (n + 1)
+        # egress: [g in R](1 - w_g) + (n-1) w_g <= t b_g
+        a[g] = (n - 1) - (1 if g in ready else 0)
+        a[n] = -bw[g]
+        A.append(a)
+        b.append(-(1.0 if g in ready else 0.0))
+        a = [0.0] * (n + 1)
+        # ingress: (k - [g in R]) w_g + 1 - w_g <= t b_g
+        a[g] = (k - (1 if g in ready else 0)) - 1
+        a[n] = -bw[g]
+        A.append(a)
+        b.append(-1.0)
+    Aeq = [[1.0] * n + [0.0]]
+    bounds = [(0, None if (g in ready or relays_as_roots) else 0) for g in range(n)] + [(0, None)]
+    res = linprog(c, A_ub=A, b_ub=b, A_eq=Aeq, b_eq=[1.0], bounds=bounds, method="highs")
+    if not res.success:
+        return _two_class(n, ready, relays_as_roots)
+    return [max(0.0, float(x)) for x in res.x[:n]]
+
+
+def _two_class(n, ready, relays_as_roots):
+    k = len(ready)
+    best = None
+    steps = 20000
+    for i in range(steps + 1):
+        wa = i / steps / k
+        wr = (1 - k * wa) / (n - k) if n > k else 0.0
+        if n > k and not relays_as_roots:
+            if abs(1 - k * wa) > 1e-12:
+                continue
+            wr = 0.0
+        if wr < -1e-12:
+            continue
+        w = [wa if g in ready else wr for g in range(n)]
+        t = star_loads(n, ready, w)[2]
+        if best is None or t < best[0]:
+            best = (t, w)
+    return best[1]
+
+
+def allreduce_mask_aware_stars(n, ready, chunk=DEFAULT_CHUNK, bw=None, relays_as_roots=True):
+    ints, _, _ = mask_aware_star_weights(n, ready, bw, relays_as_roots)
+    return allreduce_stars(n, chunk, weights=ints)
+
+
+# ------------------------------------------------------------------- allgather
+def allgather_stars(n, chunk=DEFAULT_CHUNK):
+    """One Broadcast per source, each a star from the source."""
+    out = _header(n, "allgather")
+    for s in range(n):
+        out += f"bcast src={s} weight=1 chunk={int(chunk)} parent={_join(star_parent(n, s))}\n"
+    return out
+
+
+def allgather_chains(n, chunk=1 << 20):
+    out = _header(n, "allgather")
+    for s in range(n):
+        order = [(s + k) % n for k in range(n - 1, -1, -1)]
+        out += f"bcast src={s} weight=1 chunk={int(chunk)} parent={_join(chain_parent(order))}\n"
+    return out
+
+
+# -------------------------------------------------------------------- alltoall
+def alltoall_direct(n, chunk=1 << 20, lines=1):
+    return _header(n, "alltoall") + "".join(
+        f"a2a weight=1 chunk={int(chunk)}\n" for _ in range(lines))

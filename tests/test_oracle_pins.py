@@ -382,3 +382,15 @@ def test_alltoall_is_block_transpose_and_involution():
         for s in range(n):
             blk = part[d][s * cnt:(s + 1) * cnt]
             assert np.array_equal(blk, xs[2][d * cnt:(d + 1) * cnt] if s == 2 else prev[d][:cnt])
+
+
+def test_allreduce_elements_equals_full_replay_at_samples():
+    n, count = 5, 4099
+    xs = rank_tensors("bf16", count, n)
+    txt = S.allreduce_trees([S.chain([4, 2, 0, 1, 3]), S.star(n, 1), [1, 2, -1, 1, 2]],
+                            weights=[3, 1, 2], chunk=64, noaggs=[(), (), (0,)])
+    idx = np.array([0, 1, 7, 8, 1000, 2047, 2048, 3000, 4090, 4098])
+    for R in ({0, 1, 2, 3, 4}, {0, 3}, set()):
+        full = oc.allreduce(xs, txt, R, "bf16")[0]
+        got = oc.allreduce_elements([x[idx] for x in xs], idx, count, txt, R, "bf16")
+        assert np.array_equal(full[idx], got)
