@@ -1,0 +1,468 @@
+"""Benchmark of the AdapCC B200 hot path -- prints ONE JSON line.
+
+Metric (BASELINE.json): AllReduce busbw (GB/s) = algbw * 2(n-1)/n, algbw =
+bytes per rank / time per call (nccl-tests convention).
+
+  python bench.py                      # N=1: 8 virtual ranks on one B200 (loopback)
+  torchrun --nproc-per-node N bench.py --gpus N   # N>1: one process per GPU, CUDA IPC
+  python bench.py --impl reference     # the CPU oracle timed on the host (reference arm)
+
+N=1 workload: BASELINE config C2's multi-tree AllReduce at the paper's
+microbenchmark size ("float data of 256 MB"): 8 ranks x 256 MiB fp32,
+8 weighted star trees (one per rank, chunk 256 KiB), all ranks ready.  One B200
+hosts all 8 ranks (loopback DIRECT plan: every input read once, every output
+written once), so the kernel is HBM-bound and the roofline is HBM.
+N>1: the same call through CUDA IPC over NVLink (STAGED protocol), NCCL timed
+beside it on the same buffers.
+"""
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "AllReduce busbw GB/s vs size at 2/4/8 B200 (% of 900 GB/s) vs NCCL"
+UNIT = "GB/s"
+NVLINK_NOMINAL = 900.0
+
+
+def parse_args():
+    p = argparse.ArgumentParser()
+    p.add_argument("--gpus", type=int, default=1)
+    p.add_argument("--steps", type=int, default=100)
+    p.add_argument("--warmup", type=int, default=10)
+    p.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    p.add_argument("--vranks", type=int, default=8, help="virtual ranks at N=1")
+    p.add_argument("--size-mib", type=float, default=256.0, help="bytes per rank (MiB)")
+    p.add_argument("--dtype", choices=["f32", "bf16"], default="f32")
+    p.add_argument("--mode", choices=["direct", "staged"], default="direct")
+    p.add_argument("--chunk-kib", type=int, default=256)
+    p.add_argument("--e2e-steps", type=int, default=5)
+    p.add_argument("--no-cpu-baseline", action="store_true")
+    p.add_argument("--no-parity", action="store_true")
+    return p.parse_args()
+
+
+def dist_env():
+    r = int(os.environ.get("RANK", "0"))
+    w = int(os.environ.get("WORLD_SIZE", "1"))
+    lr = int(os.environ.get("LOCAL_RANK", "0"))
+    return r, w, lr
+
+
+def busbw(bytes_per_rank, seconds, n):
+    return bytes_per_rank / seconds / 1e9 * (2.0 * (n - 1) / n)
+
+
+def load_peaks():
+    path = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        with open(path) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, burst copy)"
+    except Exception:  # noqa: BLE001
+        return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+def profile_traffic(key):
+    """dram bytes per launch from the committed ncu --set full summary, if any."""
+    path = os.path.join(ROOT, "profiles", "ncu_summary.json")
+    try:
+        with open(path) as f:
+            d = json.load(f)
+        return d.get(key, {}).get("dram_bytes_per_launch")
+    except Exception:  # noqa: BLE001
+        return None
+
+
+class ClockSampler:
+    """NVML clocks + throttle reasons sampled DURING the timed region."""
+
+    def __init__(self, index):
+        self.index = index
+        self.samples = []
+        self.reasons = set()
+        self.max_mhz = None
+        self._stop = threading.Event()
+        self._t = None
+
+    def __enter__(self):
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            h = pynvml.nvmlDeviceGetHandleByIndex(self.index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(h, pynvml.NVML_CLOCK_SM)
+            names = {
+                getattr(pynvml, "nvmlClocksThrottleReasonHwSlowdown", 0x8): "hw_slowdown",
+                getattr(pynvml, "nvmlClocksThrottleReasonHwThermalSlowdown", 0x40): "hw_thermal_slowdown",
+                getattr(pynvml, "nvmlClocksThrottleReasonSwThermalSlowdown", 0x20): "sw_thermal_slowdown",
+                getattr(pynvml, "nvmlClocksThrottleReasonSwPowerCap", 0x4): "sw_power_cap",
+            }
+
+            def loop():
+                while not self._stop.is_set():
+                    try:
+                        self.samples.append(pynvml.nvmlDeviceGetClockInfo(h, pynvml.NVML_CLOCK_SM))
+                        bits = pynvml.nvmlDeviceGetCurrentClocksThrottleReasons(h)
+                        for b, nm in names.items():
+                            if bits & b:
+                                self.reasons.add(nm)
+                    except Exception:  # noqa: BLE001
+                        pass
+                    time.sleep(0.01)
+
+            self._t = threading.Thread(target=loop, daemon=True)
+            self._t.start()
+        except Exception:  # noqa: BLE001
+            self._t = None
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        if self._t:
+            self._t.join(timeout=2)
+
+    def summary(self):
+        s = sorted(self.samples)
+        med = s[len(s) // 2] if s else None
+        return {"sm_mhz": med, "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons),
+                "samples": len(s)}
+
+
+# ------------------------------------------------------------------ oracle leg
+def oracle_sample_busbw(n, dtype, count, reps=1):
+    """Time the CPU oracle (as it stands) on a bounded sample; 1 host core."""
+    import numpy as np  # noqa: F401
+
+    from oracle import collectives as oc
+    from paper_conf_icdcs_zhaozw24_b200 import generator as G
+    from synth import rank_tensors
+    try:
+        os.sched_setaffinity(0, {sorted(os.sched_getaffinity(0))[0]})
+    except Exception:  # noqa: BLE001
+        pass
+    xs = rank_tensors(dtype, count, n)
+    text = G.allreduce_stars(n, chunk=262144)
+    es = 4 if dtype == "f32" else 2
+    t0 = time.perf_counter()
+    for _ in range(reps):
+        oc.allreduce(xs, text, set(range(n)), dtype)
+    dt = (time.perf_counter() - t0) / reps
+    return busbw(count * es, dt, n), dt
+
+
+def cpu_baseline_block(n, dtype, target_s=15.0):
+    count = 1 << 20
+    v, dt = oracle_sample_busbw(n, dtype, count)
+    reps = max(1, min(200, int(target_s / max(dt, 1e-6))))
+    v, dt = oracle_sample_busbw(n, dtype, count, reps=reps)
+    es = 4 if dtype == "f32" else 2
+    return {"value": round(v, 4), "unit": UNIT, "cores": 1, "kind": "oracle",
+            "sample": f"{n} simulated ranks x {count} {dtype} elements ({count * es >> 20} MiB/rank), "
+                      f"{reps} reps, numpy single thread pinned to 1 core of {os.cpu_count()}"}
+
+
+def run_reference(args):
+    r, w, _ = dist_env()
+    if r != 0:
+        return None
+    n = args.vranks if w == 1 else w
+    count = 1 << 20
+    es = 4 if args.dtype == "f32" else 2
+    for _ in range(args.warmup):
+        oracle_sample_busbw(n, args.dtype, count)
+    times = []
+    for _ in range(args.steps):
+        _, dt = oracle_sample_busbw(n, args.dtype, count)
+        times.append(dt)
+    t = sum(times) / len(times)
+    v = busbw(count * es, t, n)
+    sample = (f"{n} simulated ranks x {count} {args.dtype} elements per step "
+              f"({count * es >> 20} MiB/rank), numpy 1 core of {os.cpu_count()}")
+    return {
+        "impl": "reference", "metric": METRIC, "value": round(v, 4), "unit": UNIT,
+        "n_gpus": w, "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(t * 1e3, 3),
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": args.dtype,
+        "data": "synthetic", "config": workload_config(args, n, w),
+        "cpu_baseline": {"value": round(v, 4), "unit": UNIT, "cores": 1, "kind": "oracle",
+                         "sample": sample},
+        "e2e": {"value": round(v, 4), "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+
+
+def workload_config(args, n, world):
+    nbytes = int(args.size_mib * (1 << 20))
+    where = "loopback-vr" if world == 1 else "ipc-gpu"
+    return {
+        "workload": f"allreduce-{where}{n}-{args.dtype}-{nbytes >> 20}MiB-star{n}",
+        "ranks": n, "virtual_ranks": world == 1, "bytes_per_rank": nbytes,
+        "strategy": f"{n} star trees (one rooted at each rank), equal weights, chunk {args.chunk_kib} KiB",
+        "mode": args.mode if world == 1 else "staged", "ready_mask": "all",
+        "l2": f"inputs {n * nbytes >> 20} MiB per step > 126 MB L2 (no flush needed)",
+        "parallelism": f"{'virtual ' if world == 1 else ''}dp{n}",
+    }
+
+
+# ---------------------------------------------------------------- our arm, N=1
+def run_single(args):
+    import numpy as np
+    import torch
+
+    import paper_conf_icdcs_zhaozw24_b200 as pkg
+    from paper_conf_icdcs_zhaozw24_b200 import generator as G
+    from synth import rank_tensors
+
+    torch.cuda.set_device(0)
+    n = args.vranks
+    es = 4 if args.dtype == "f32" else 2
+    nbytes = int(args.size_mib * (1 << 20)) // 16 * 16
+    count = nbytes // es
+    tdt = torch.float32 if args.dtype == "f32" else torch.bfloat16
+    text = G.allreduce_stars(n, chunk=args.chunk_kib * 1024)
+
+    comm = pkg.Communicator.loopback(n, device=0, scratch_bytes=max(64 << 20, 2 * nbytes + (8 << 20))
+                                     if args.mode == "staged" else 64 << 20, mode=args.mode)
+    comm.set_strategy("allreduce", text)
+
+    host_in = []
+    for r in range(n):
+        x = rank_tensors(args.dtype, count, 1, base=1000 + r)[0]
+        t = torch.from_numpy(x)
+        if args.dtype == "bf16":
+            t = t.view(torch.int16)
+        host_in.append(t.pin_memory())
+    dx = [h.cuda().view(tdt) for h in host_in]
+    dy = [torch.empty(count, dtype=tdt, device="cuda") for _ in range(n)]
+    stream = torch.cuda.current_stream()
+
+    for _ in range(args.warmup):
+        comm.allreduce_lb(dx, dy)
+    torch.cuda.synchronize()
+    assert comm.get_async_error() == 0
+
+    starts = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+    ends = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
+    launches0 = comm.launch_count()
+    with ClockSampler(0) as clk:
+        torch.cuda.synchronize()
+        t_begin = torch.cuda.Event(enable_timing=True)
+        t_end = torch.cuda.Event(enable_timing=True)
+        t_begin.record(stream)
+        for i in range(args.steps):
+            starts[i].record(stream)
+            comm.allreduce_lb(dx, dy)
+            ends[i].record(stream)
+        t_end.record(stream)
+        torch.cuda.synchronize()
+    launches = comm.launch_count() - launches0
+    assert comm.get_async_error() == 0
+    total_ms = t_begin.elapsed_time(t_end)
+    per = [s.elapsed_time(e) for s, e in zip(starts, ends)]
+    ms = total_ms / args.steps
+    kern_ms = sum(per) / len(per)
+    value = busbw(nbytes, ms / 1e3, n)
+
+    # parity on sampled outputs at full size (oracle, one element at a time)
+    parity = None
+    if not args.no_parity:
+        parity = sampled_parity(dy, host_in, text, n, count, args.dtype)
+
+    # end to end: pinned host inputs -> device -> allreduce -> host, every step
+    host_out = [torch.empty(count, dtype=host_in[0].dtype).pin_memory() for _ in range(n)]
+    e2e_ms = []
+    for i in range(args.e2e_steps + 1):
+        a = torch.cuda.Event(enable_timing=True)
+        b = torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        for r in range(n):
+            dx[r].view(host_in[r].dtype).copy_(host_in[r], non_blocking=True)
+        comm.allreduce_lb(dx, dy)
+        for r in range(n):
+            host_out[r].copy_(dy[r].view(host_out[r].dtype), non_blocking=True)
+        b.record(stream)
+        torch.cuda.synchronize()
+        if i > 0:
+            e2e_ms.append(a.elapsed_time(b))
+    e2e_t = sum(e2e_ms) / len(e2e_ms)
+
+    peak, peak_src = load_peaks()
+    alg_bytes = 2 * n * nbytes   # every rank's input read once + output written once
+    achieved = alg_bytes / (kern_ms / 1e3) / 1e9
+    out = {
+        "metric": METRIC, "value": round(value, 3), "unit": UNIT, "n_gpus": 1,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms, 4),
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": args.dtype,
+        "data": "synthetic (seeded N(0,1), synth/inputs.py)",
+        "config": workload_config(args, n, 1),
+        "algbw": round(nbytes / (ms / 1e3) / 1e9, 3),
+        "pct_of_nvlink_900": None,
+        "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
+                     "frac": round(achieved / peak, 4), "traffic": profile_traffic("allreduce_loopback"),
+                     "algorithmic_bytes_per_launch": alg_bytes, "peak_source": peak_src,
+                     "kernel": "adapcc::engine_kernel<f32>", "kernel_ms": round(kern_ms, 4)},
+        "e2e": {"value": round(busbw(nbytes, e2e_t / 1e3, n), 3), "unit": UNIT,
+                "h2d_bytes_per_step": n * nbytes, "d2h_bytes_per_step": n * nbytes,
+                "ms_per_step": round(e2e_t, 3)},
+        "gpu_launches": launches,
+        "clocks": clk.summary(),
+        "parity": parity,
+        "nccl": None,
+    }
+    if not args.no_cpu_baseline:
+        out["cpu_baseline"] = cpu_baseline_block(n, args.dtype)
+    comm.finalize()
+    return out
+
+
+def sampled_parity(dy, host_in, text, n, count, dtype, k=4096):
+    import numpy as np
+    import torch
+
+    from oracle import collectives as oc
+    rng = np.random.default_rng(11)
+    idx = np.unique(np.concatenate([rng.integers(0, count, size=k), [0, count - 1]]))
+    ti = torch.from_numpy(idx).cuda()
+    vals = []
+    for h in host_in:
+        a = h.numpy()
+        vals.append(a[idx].view(np.uint16) if dtype == "bf16" else a[idx])
+    exp = oc.allreduce_elements(vals, idx, count, text, set(range(n)), dtype)
+    bad = 0
+    for y in dy:
+        g = y.index_select(0, ti)
+        g = g.view(torch.int16).cpu().numpy().view(np.uint16) if dtype == "bf16" else g.cpu().numpy()
+        ebits = exp.view(np.uint16) if dtype == "bf16" else exp.view(np.uint32)
+        gbits = g.view(np.uint16) if dtype == "bf16" else g.view(np.uint32)
+        bad += int(np.count_nonzero(ebits != gbits))
+    return {"samples_per_rank": int(len(idx)), "ranks": n, "mismatches": bad,
+            "reference": "oracle.allreduce_elements (strategy-order replay), bit-exact"}
+
+
+# ---------------------------------------------------------------- our arm, N>1
+def run_multi(args):
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_icdcs_zhaozw24_b200 as pkg
+    from paper_conf_icdcs_zhaozw24_b200 import generator as G
+    from synth import rank_tensors
+
+    rank, world, local = dist_env()
+    torch.cuda.set_device(local)
+    dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    es = 4 if args.dtype == "f32" else 2
+    nbytes = int(args.size_mib * (1 << 20)) // 16 * 16
+    count = nbytes // es
+    tdt = torch.float32 if args.dtype == "f32" else torch.bfloat16
+    text = G.allreduce_stars(world, chunk=args.chunk_kib * 1024)
+    comm = pkg.Communicator.init(scratch_bytes=max(1 << 30, 2 * nbytes + (64 << 20)), device=local)
+    comm.set_strategy("allreduce", text)
+    xh = torch.from_numpy(rank_tensors(args.dtype, count, 1, base=1000 + rank)[0])
+    if args.dtype == "bf16":
+        xh = xh.view(torch.int16)
+    xh = xh.pin_memory()
+    x = xh.cuda().view(tdt)
+    y = torch.empty_like(x)
+    stream = torch.cuda.current_stream()
+
+    def timed(fn, steps):
+        dist.barrier()
+        torch.cuda.synchronize()
+        a = torch.cuda.Event(enable_timing=True)
+        b = torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        for _ in range(steps):
+            fn()
+        b.record(stream)
+        torch.cuda.synchronize()
+        t = torch.tensor([a.elapsed_time(b) / steps], device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        dist.barrier()
+        return float(t.item())
+
+    def ours():
+        comm.allreduce(x, y)
+
+    z = x.clone()
+
+    def nccl():
+        dist.all_reduce(z)
+
+    for _ in range(args.warmup):
+        ours()
+        nccl()
+    torch.cuda.synchronize()
+    l0 = comm.launch_count()
+    with ClockSampler(local) as clk:
+        ms = timed(ours, args.steps)
+    launches = comm.launch_count() - l0
+    ms_nccl = timed(nccl, args.steps)
+    err = comm.get_async_error()
+
+    e2e = []
+    for i in range(args.e2e_steps + 1):
+        dist.barrier()
+        torch.cuda.synchronize()
+        a = torch.cuda.Event(enable_timing=True)
+        b = torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        x.view(xh.dtype).copy_(xh, non_blocking=True)
+        comm.allreduce(x, y)
+        out_h = y.view(xh.dtype).to("cpu", non_blocking=True)
+        b.record(stream)
+        torch.cuda.synchronize()
+        t = torch.tensor([a.elapsed_time(b)], device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        if i > 0:
+            e2e.append(float(t.item()))
+    del out_h
+    e2e_t = sum(e2e) / len(e2e)
+    value = busbw(nbytes, ms / 1e3, world)
+    res = None
+    if rank == 0:
+        res = {
+            "metric": METRIC, "value": round(value, 3), "unit": UNIT, "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms, 4),
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": args.dtype,
+            "data": "synthetic (seeded N(0,1), synth/inputs.py)",
+            "config": workload_config(args, world, world),
+            "algbw": round(nbytes / (ms / 1e3) / 1e9, 3),
+            "pct_of_nvlink_900": round(100 * value / NVLINK_NOMINAL, 2),
+            "roofline": {"bound": "nvlink", "achieved": round(value, 1), "peak": 770.0, "unit": "GB/s",
+                         "frac": round(value / 770.0, 4), "traffic": None,
+                         "peak_source": "B200_PROFILING.md measured peer copy 770 GB/s per direction",
+                         "algorithmic_bytes_per_launch": int(2 * (world - 1) * nbytes // world)},
+            "e2e": {"value": round(busbw(nbytes, e2e_t / 1e3, world), 3), "unit": UNIT,
+                    "h2d_bytes_per_step": nbytes, "d2h_bytes_per_step": nbytes,
+                    "ms_per_step": round(e2e_t, 3)},
+            "gpu_launches": launches, "clocks": clk.summary(), "async_error": err,
+            "nccl": {"value": round(busbw(nbytes, ms_nccl / 1e3, world), 3), "unit": UNIT,
+                     "ms_per_step": round(ms_nccl, 4), "version": ".".join(map(str, torch.cuda.nccl.version()))},
+        }
+    comm.finalize()
+    dist.destroy_process_group()
+    return res
+
+
+def main():
+    args = parse_args()
+    _, world, _ = dist_env()
+    if args.impl == "reference":
+        out = run_reference(args)
+    elif world > 1:
+        out = run_multi(args)
+    else:
+        out = run_single(args)
+    if out is not None:
+        print(json.dumps(out), flush=True)
+
+
+if __name__ == "__main__":
+    main()

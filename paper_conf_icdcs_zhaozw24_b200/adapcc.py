@@ -21,7 +21,8 @@ import ctypes
 import os
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-_LIB_PATH = os.path.join(_PKG, "libadapcc.so")
+# ADAPCC_LIB selects an alternative in-tree build (tuning sweeps only)
+_LIB_PATH = os.environ.get("ADAPCC_LIB") or os.path.join(_PKG, "libadapcc.so")
 
 SUCCESS, INVALID_ARGUMENT, INVALID_STRATEGY, UNSUPPORTED, CUDA, BOOTSTRAP, OOM, TIMEOUT, MISMATCH = range(9)
 COLL = {"allreduce": 0, "allgather": 1, "alltoall": 2}

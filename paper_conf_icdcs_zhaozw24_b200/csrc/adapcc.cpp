@@ -110,6 +110,7 @@ struct adapcc_comm_s {
   int64_t timeout_ms = 10000;
   int64_t max_ctas = 0;
   int64_t drop_rank = -1;
+  int64_t piece_kib = 0;  // 0 = automatic (total traffic / (8 * grid))
   uint64_t launches = 0;
   int num_sms = 148;
   int occ[3] = {1, 1, 1};
@@ -136,6 +137,7 @@ adapcc_result_t common_init(adapcc_comm_s* c, size_t scratch) {
   c->arena_bytes = kArenaHeader + 2 * c->half_bytes;
   c->timeout_ms = env_int("ADAPCC_TIMEOUT_MS", 10000);
   c->max_ctas = env_int("ADAPCC_NCTAS", 0);
+  c->piece_kib = env_int("ADAPCC_PIECE_KIB", 0);
   CK(cudaSetDevice(c->device));
   CK(cudaDeviceGetAttribute(&c->num_sms, cudaDevAttrMultiProcessorCount, c->device));
   for (int d = 0; d < 3; ++d) {
@@ -190,6 +192,12 @@ bool overlap(const void* a, size_t an, const void* b, size_t bn) {
   return x < y + bn && y < x + an;
 }
 
+int grid_size(const adapcc_comm_s* c, adapcc_dtype_t dtype) {
+  int grid = c->num_sms * c->occ[(int)dtype];
+  if (c->max_ctas > 0) grid = (int)std::min<int64_t>(grid, c->max_ctas);
+  return std::max(grid, 1);
+}
+
 adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, uint64_t count, adapcc_dtype_t dtype,
                          uint64_t mask, unsigned flags, std::shared_ptr<DevPlan>* out) {
   PlanKey key{(int)coll, c->strat_version[coll], count, (int)dtype, mask, flags};
@@ -215,7 +223,8 @@ adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, uint64_t count, adapcc_dty
   CK(cudaEventCreateWithFlags(&plan->last_use, cudaEventDisableTiming));
   for (auto& sp : segs) {
     DevSegment d;
-    std::vector<Item> items = order_items(sp, c->loopback ? -1 : c->rank);
+    std::vector<Item> items = order_items(sp, c->loopback ? -1 : c->rank, rq.esize, grid_size(c, dtype),
+                                          (uint64_t)c->piece_kib * 1024);
     d.nitems = (uint32_t)items.size();
     auto up = [](auto** dst, const auto& v) -> cudaError_t {
       using T = typename std::decay_t<decltype(v)>::value_type;
@@ -279,9 +288,7 @@ adapcc_result_t run(adapcc_comm_s* c, Coll coll, const void* const* send, void* 
       P.hdr[q] = c->arena[q];
       P.arena[q] = c->arena[q] + kArenaHeader + parity * c->half_bytes;
     }
-    int grid = c->num_sms * c->occ[(int)dtype];
-    if (c->max_ctas > 0) grid = (int)std::min<int64_t>(grid, c->max_ctas);
-    grid = std::max(1, std::min<int>(grid, (int)std::max<uint32_t>(1, seg.nitems)));
+    const int grid = std::max(1, std::min<int>(grid_size(c, dtype), (int)std::max<uint32_t>(1, seg.nitems)));
     CK(engine_launch(P, grid, s));
     ++c->launches;
   }

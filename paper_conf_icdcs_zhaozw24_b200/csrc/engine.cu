@@ -26,6 +26,12 @@ namespace adapcc {
 namespace {
 
 constexpr int kThreads = 256;
+#ifndef ADAPCC_UNROLL
+#define ADAPCC_UNROLL 8   // 128-bit vectors in flight per thread per source
+#endif
+#ifndef ADAPCC_MINB
+#define ADAPCC_MINB 2     // resident CTAs per SM the register budget is sized for
+#endif
 
 __device__ __forceinline__ uint64_t ld_acquire_sys(const uint64_t* p) {
   uint64_t v;
@@ -136,41 +142,48 @@ struct Shared {
 
 // ---------------------------------------------------------- vector fold
 // Sources are folded one at a time with U 128-bit loads in flight per thread
-// (U * 16 B * 256 threads * 2 CTAs = 32-64 KB in flight per SM, enough to
-// cover HBM / NVLink latency); the accumulator stays in registers.
+// (U=8: 8 x 16 B x 256 threads x 2 CTAs = 64 KB in flight per SM, enough to
+// cover HBM / NVLink latency); the accumulator stays in registers.  Vector
+// indices are 32-bit (a chunk is at most 2^31 bytes).
+template <int U>
+__device__ __forceinline__ void load_u(uint4 (&x)[U], const char* src, uint32_t base, uint32_t nvec,
+                                       bool full) {
+  if (full) {
+#pragma unroll
+    for (int u = 0; u < U; ++u) x[u] = ld16(src + (size_t)(base + u * kThreads) * 16);
+  } else {
+#pragma unroll
+    for (int u = 0; u < U; ++u)
+      if (base + u * kThreads < nvec) x[u] = ld16(src + (size_t)(base + u * kThreads) * 16);
+  }
+}
+
+template <int U>
+__device__ __forceinline__ void store_u(char* dst, const uint4 (&x)[U], uint32_t base, uint32_t nvec,
+                                        bool full) {
+  if (full) {
+#pragma unroll
+    for (int u = 0; u < U; ++u) st16(dst + (size_t)(base + u * kThreads) * 16, x[u]);
+  } else {
+#pragma unroll
+    for (int u = 0; u < U; ++u)
+      if (base + u * kThreads < nvec) st16(dst + (size_t)(base + u * kThreads) * 16, x[u]);
+  }
+}
+
 template <int DT, int U>
-__device__ __forceinline__ void fold_vec(const Shared& sh, int nsrc, int ndst, uint64_t nvec) {
+__device__ __forceinline__ void fold_vec(const Shared& sh, int nsrc, int ndst, uint32_t nvec) {
   using O = Ops<DT>;
-  const bool pure_copy = nsrc == 1 && !sh.any_acc;
-  for (uint64_t base = threadIdx.x; base < nvec; base += (uint64_t)U * kThreads) {
+  for (uint32_t base = threadIdx.x; base < nvec; base += U * kThreads) {
+    const bool full = base + (U - 1) * kThreads < nvec;
     uint4 x[U];
-#pragma unroll
-    for (int u = 0; u < U; ++u) {
-      const uint64_t v = base + (uint64_t)u * kThreads;
-      if (v < nvec) x[u] = ld16(sh.src[0] + v * 16);
-    }
-    if (pure_copy) {  // bytes unchanged (relay forward / broadcast)
-      for (int d = 0; d < ndst; ++d) {
-        char* dst = sh.dst[d];
-#pragma unroll
-        for (int u = 0; u < U; ++u) {
-          const uint64_t v = base + (uint64_t)u * kThreads;
-          if (v < nvec) st16(dst + v * 16, x[u]);
-        }
-      }
-      continue;
-    }
+    load_u<U>(x, sh.src[0], base, nvec, full);
     if (nsrc > 1) {
       typename O::Acc a[U];
 #pragma unroll
       for (int u = 0; u < U; ++u) a[u] = O::widen(x[u]);
       for (int k = 1; k < nsrc; ++k) {
-        const char* src = sh.src[k];
-#pragma unroll
-        for (int u = 0; u < U; ++u) {
-          const uint64_t v = base + (uint64_t)u * kThreads;
-          if (v < nvec) x[u] = ld16(src + v * 16);
-        }
+        load_u<U>(x, sh.src[k], base, nvec, full);
 #pragma unroll
         for (int u = 0; u < U; ++u) O::add(a[u], x[u]);
       }
@@ -179,28 +192,18 @@ __device__ __forceinline__ void fold_vec(const Shared& sh, int nsrc, int ndst, u
     }
     for (int d = 0; d < ndst; ++d) {
       char* dst = sh.dst[d];
-      if (sh.acc[d]) {
-        uint4 p[U];
+      if (sh.acc[d]) {  // recv += result (phase 2): one vector at a time
 #pragma unroll
         for (int u = 0; u < U; ++u) {
-          const uint64_t v = base + (uint64_t)u * kThreads;
-          if (v < nvec) p[u] = ld16(dst + v * 16);
-        }
-#pragma unroll
-        for (int u = 0; u < U; ++u) {
-          const uint64_t v = base + (uint64_t)u * kThreads;
+          const uint32_t v = base + u * kThreads;
           if (v < nvec) {
-            typename O::Acc q = O::widen(p[u]);
+            typename O::Acc q = O::widen(ld16(dst + (size_t)v * 16));
             O::add(q, x[u]);
-            st16(dst + v * 16, O::narrow(q));
+            st16(dst + (size_t)v * 16, O::narrow(q));
           }
         }
       } else {
-#pragma unroll
-        for (int u = 0; u < U; ++u) {
-          const uint64_t v = base + (uint64_t)u * kThreads;
-          if (v < nvec) st16(dst + v * 16, x[u]);
-        }
+        store_u<U>(dst, x, base, nvec, full);  // bytes unchanged when nsrc == 1
       }
     }
   }
@@ -251,7 +254,7 @@ __device__ void fold_chunk(const Shared& sh, int nsrc, int ndst, uint64_t n, int
   }
   constexpr int VE = 16 / O::kEsize;
   const uint64_t nvec = n / VE;
-  fold_vec<DT, 4>(sh, nsrc, ndst, nvec);
+  fold_vec<DT, ADAPCC_UNROLL>(sh, nsrc, ndst, (uint32_t)nvec);
   if (nvec * VE < n) fold_scalar<DT>(sh, nsrc, ndst, nvec * VE, n);
 }
 
@@ -278,7 +281,7 @@ __device__ __forceinline__ char* base_of(const LaunchParams& P, uint8_t kind, in
 }
 
 template <int DT>
-__global__ void __launch_bounds__(kThreads, 4) engine_kernel(const __grid_constant__ LaunchParams P) {
+__global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __grid_constant__ LaunchParams P) {
   __shared__ Shared sh;
   if (threadIdx.x == 0) sh.abort = 0;
   __syncthreads();
@@ -300,8 +303,8 @@ __global__ void __launch_bounds__(kThreads, 4) engine_kernel(const __grid_consta
     const Item item = P.items[it];
     const Task& t = P.tasks[item.task];
     const int nsrc = t.nsrc, ndst = t.ndst;
-    const uint64_t e0 = t.lo + (uint64_t)item.chunk * t.chunk_elems;
-    const uint64_t e1 = min(t.hi, e0 + t.chunk_elems);
+    const uint64_t e0 = t.lo + (uint64_t)item.chunk * t.chunk_elems + item.off;
+    const uint64_t e1 = e0 + item.len;
     const bool dropped = (int)t.owner == P.drop_rank;
     if (threadIdx.x == 0) { sh.bad_align = 0; sh.any_acc = 0; }
     __syncthreads();

@@ -55,9 +55,15 @@ struct Task {
   uint16_t owner;           // executing rank
 };
 
+// A work item covers elements [off, off+len) of chunk `chunk` of `task`.  A
+// task that posts flags is executed one whole chunk per item (the flag means
+// "the whole chunk is written"); a task without posts may be split into
+// several pieces per chunk so that CTAs get even work (grid balance).
 struct Item {
   uint32_t task;
   uint32_t chunk;
+  uint32_t off;   // elements from the chunk start
+  uint32_t len;   // elements
 };
 
 }  // namespace adapcc

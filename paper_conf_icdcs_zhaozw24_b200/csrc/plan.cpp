@@ -399,19 +399,47 @@ bool build_plan(const PlanRequest& rq, std::vector<SegmentPlan>* segs, std::stri
   }
 }
 
-std::vector<Item> order_items(const SegmentPlan& p, int rank) {
-  struct Key { uint64_t a; uint32_t level, task, chunk; };
+std::vector<Item> order_items(const SegmentPlan& p, int rank, int esize, int grid,
+                              uint64_t piece_bytes) {
+  // Work balance: tasks that post no flags are cut into pieces of roughly
+  // equal traffic so that the grid sees >= ~8 items per CTA.
+  uint64_t total = 0;
+  for (const Task& T : p.tasks)
+    if (rank < 0 || T.owner == rank) total += (T.hi - T.lo) * esize * (uint64_t)(T.nsrc + T.ndst);
+  // Measured on B200 (profiles/sweep_r01.json): ~512 KiB of traffic per item
+  // (32 KiB per stream for a 16-stream fold) is the sweet spot -- smaller
+  // items pay the per-item claim/sync overhead, larger ones lose bandwidth.
+  const uint64_t target =
+      piece_bytes ? piece_bytes
+                  : std::min<uint64_t>(std::max<uint64_t>(total / (4ull * std::max(grid, 1)), 64 * 1024),
+                                       512 * 1024);
+  const uint64_t align = 512;  // elements: keeps every piece 16-byte aligned
+  struct Key { uint64_t a; uint32_t level, task, chunk, off, len; };
   std::vector<Key> keys;
   for (uint32_t t = 0; t < p.tasks.size(); ++t) {
     const Task& T = p.tasks[t];
     if (rank >= 0 && T.owner != rank) continue;
-    for (uint32_t c = 0; c < T.nchunks; ++c) keys.push_back({(uint64_t)c + T.level, T.level, t, c});
+    uint64_t piece = T.chunk_elems;
+    if (T.npost == 0) {
+      const uint64_t streams = std::max<uint64_t>(1, T.nsrc + T.ndst);
+      piece = std::max<uint64_t>(align, target / (streams * esize) / align * align);
+      piece = std::min<uint64_t>(piece, T.chunk_elems);
+    }
+    for (uint32_t c = 0; c < T.nchunks; ++c) {
+      const uint64_t c0 = T.lo + (uint64_t)c * T.chunk_elems;
+      const uint64_t clen = std::min<uint64_t>(T.hi, c0 + T.chunk_elems) - c0;
+      for (uint64_t off = 0; off < clen; off += piece)
+        keys.push_back({(uint64_t)c + T.level, T.level, t, c, (uint32_t)off,
+                        (uint32_t)std::min<uint64_t>(piece, clen - off)});
+    }
   }
   std::sort(keys.begin(), keys.end(), [](const Key& x, const Key& y) {
-    return std::tie(x.a, x.level, x.task, x.chunk) < std::tie(y.a, y.level, y.task, y.chunk);
+    return std::tie(x.a, x.level, x.task, x.chunk, x.off) <
+           std::tie(y.a, y.level, y.task, y.chunk, y.off);
   });
   std::vector<Item> items(keys.size());
-  for (size_t i = 0; i < keys.size(); ++i) items[i] = {keys[i].task, keys[i].chunk};
+  for (size_t i = 0; i < keys.size(); ++i)
+    items[i] = {keys[i].task, keys[i].chunk, keys[i].off, keys[i].len};
   return items;
 }
 

@@ -52,8 +52,11 @@ uint64_t flag_region_bytes(uint64_t half);
 // call cannot be planned (e.g. arena too small even for 1 unit per segment).
 bool build_plan(const PlanRequest& rq, std::vector<SegmentPlan>* segs, std::string* err);
 
-// Work items of `rank` (-1: all ranks) in deadlock-free order.
-std::vector<Item> order_items(const SegmentPlan& p, int rank);
+// Work items of `rank` (-1: all ranks) in deadlock-free order; `grid` CTAs
+// will execute them (used to size the pieces of flag-free tasks).
+// piece_bytes: traffic per piece (all streams); 0 = total / (8 * grid).
+std::vector<Item> order_items(const SegmentPlan& p, int rank, int esize, int grid,
+                              uint64_t piece_bytes = 0);
 
 // Byte accounting for adapcc_plan_stats.
 void accumulate_stats(const SegmentPlan& p, int rank, int esize, PlanStats* s);
