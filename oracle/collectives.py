@@ -129,24 +129,26 @@ def _tree_result(vals, sub, ready, dtype):
     return np.array(value(fl[0]), copy=True) if fl else None
 
 
-def allreduce_elements(vals, idx, count, strategy_text, ready, dtype):
+def allreduce_elements(vals, idx, count, strategy_text, ready, dtype, accumulate=False,
+                       y_prev=None):
     """AllReduce result at selected element indices only (for sampled parity at
     full size): vals[r] holds rank r's inputs AT ``idx``; each element is
     reduced by the tree whose partition contains it (Q9), exactly as in
     ``allreduce``.  Returns the (broadcast-identical) result at idx; +0 where
-    no rank is ready."""
+    no rank is ready.  With ``accumulate``, y_prev (values at idx of one
+    rank's recvbuf) is combined as in ``allreduce``."""
     st = parse(strategy_text)
     ready = set(ready)
     idx = np.asarray(idx, dtype=np.int64)
     bounds = partition(count, ESIZE[dtype], [s.weight for s in st.subs])
-    out = _zero(len(idx), dtype)
+    out = np.array(y_prev, copy=True) if accumulate else _zero(len(idx), dtype)
     for m, sub in enumerate(st.subs):
         sel = np.nonzero((idx >= bounds[m]) & (idx < bounds[m + 1]))[0]
         if len(sel) == 0:
             continue
         res = _tree_result([v[sel] if v is not None else None for v in vals], sub, ready, dtype)
         if res is not None:
-            out[sel] = res
+            out[sel] = _accumulate(out[sel], res, dtype) if accumulate else res
     return out
 
 

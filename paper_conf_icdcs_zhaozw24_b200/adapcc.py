@@ -188,6 +188,31 @@ def plan_stats(text, count, dtype, mask, accumulate=False, mode="direct", rank=-
 
 
 # --------------------------------------------------------------- communicator
+def make_bootstrap_allgather(group=None, device=None):
+    """ctypes callback implementing adapcc_bootstrap_allgather_fn over a
+    torch.distributed group (gloo: CPU tensors; nccl: tensors on `device`).
+    The paper's set-up AllGather of IPC handles (Fig. 10)."""
+    import torch
+    import torch.distributed as dist
+    n = dist.get_world_size(group)
+    backend = dist.get_backend(group)
+    tdev = torch.device("cuda", device if device is not None else torch.cuda.current_device()) \
+        if backend == "nccl" else torch.device("cpu")
+
+    def ag(send, recv, nbytes, _ctx):
+        try:
+            mine = torch.frombuffer(bytearray(ctypes.string_at(send, nbytes)), dtype=torch.uint8)
+            outs = [torch.empty(nbytes, dtype=torch.uint8, device=tdev) for _ in range(n)]
+            dist.all_gather(outs, mine.to(tdev), group=group)
+            blob = b"".join(o.cpu().numpy().tobytes() for o in outs)
+            ctypes.memmove(recv, blob, len(blob))
+            return 0
+        except Exception:  # noqa: BLE001 -- reported as ADAPCC_ERR_BOOTSTRAP
+            return 1
+
+    return AG_FN(ag)
+
+
 class Communicator:
     """A communicator (the paper's transmission contexts)."""
 
@@ -217,21 +242,7 @@ class Communicator:
         rank = dist.get_rank(group)
         n = dist.get_world_size(group)
         dev = torch.cuda.current_device() if device is None else device
-        backend = dist.get_backend(group)
-        tdev = torch.device("cuda", dev) if backend == "nccl" else torch.device("cpu")
-
-        def ag(send, recv, nbytes, _ctx):
-            try:
-                mine = torch.frombuffer(bytearray(ctypes.string_at(send, nbytes)), dtype=torch.uint8)
-                outs = [torch.empty(nbytes, dtype=torch.uint8, device=tdev) for _ in range(n)]
-                dist.all_gather(outs, mine.to(tdev), group=group)
-                blob = b"".join(o.cpu().numpy().tobytes() for o in outs)
-                ctypes.memmove(recv, blob, len(blob))
-                return 0
-            except Exception:  # noqa: BLE001 -- reported as ADAPCC_ERR_BOOTSTRAP
-                return 1
-
-        cb = AG_FN(ag)
+        cb = make_bootstrap_allgather(group, dev)
         h = ctypes.c_void_p()
         _check(L.adapcc_init(ctypes.byref(h), rank, n, dev, scratch_bytes, cb, None), "init")
         return cls(h, n, rank, dev, False, keep=cb)

@@ -1,0 +1,143 @@
+"""Parity at BASELINE.json's full sizes, in the launch configuration bench.py times (-m gpu).
+
+Outputs are checked on sampled indices the oracle computes element by element
+(oracle.allreduce_elements replays each sampled element's tree), or completely
+where the definition is a pure index map (AlltoAll).
+"""
+
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+
+import paper_conf_icdcs_zhaozw24_b200 as pkg  # noqa: E402
+from oracle import collectives as oc  # noqa: E402
+from paper_conf_icdcs_zhaozw24_b200 import generator as G  # noqa: E402
+from synth import GPT2XL_LAYERS, rank_tensors  # noqa: E402
+from tests.gpu_util import bits, to_dev, to_host  # noqa: E402
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(autouse=True)
+def _need_gpu():
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+
+
+def _samples(count, k=4096, seed=11):
+    rng = np.random.default_rng(seed)
+    return np.unique(np.concatenate([rng.integers(0, count, size=k), [0, count - 1]]))
+
+
+def _gather(ts, idx, dtype):
+    ti = torch.from_numpy(idx).cuda()
+    return [to_host(t.index_select(0, ti), dtype) for t in ts]
+
+
+@pytest.mark.parametrize("mode,dtype", [("direct", "f32"), ("staged", "f32"), ("direct", "bf16")])
+def test_c2_bench_config_sampled(mode, dtype):
+    """C2 at the bench point: 8 ranks x 256 MiB, 8 star trees, chunk 256 KiB."""
+    n, nbytes = 8, 256 << 20
+    es = 4 if dtype == "f32" else 2
+    count = nbytes // es
+    text = G.allreduce_stars(n, chunk=262144)
+    comm = pkg.Communicator.loopback(n, scratch_bytes=(2 * nbytes + (8 << 20)) if mode == "staged"
+                                     else 64 << 20, mode=mode)
+    comm.set_strategy("allreduce", text)
+    xs = rank_tensors(dtype, count, n)
+    dx = [to_dev(x, dtype) for x in xs]
+    dy = [torch.empty_like(t) for t in dx]
+    comm.allreduce_lb(dx, dy)
+    torch.cuda.synchronize()
+    assert comm.get_async_error() == 0
+    idx = _samples(count)
+    exp = oc.allreduce_elements([x[idx] for x in xs], idx, count, text, set(range(n)), dtype)
+    for g in _gather(dy, idx, dtype):
+        assert np.array_equal(bits(g), bits(exp))
+    comm.finalize()
+
+
+@pytest.mark.parametrize("mib", [25, 100])
+def test_c3_partial_aggregation_sampled(mib):
+    """C3: 8 ranks, stragglers {3,6} relay in phase 1 (mask-aware weighted stars),
+    then join with ACCUMULATE in phase 2; STAGED protocol."""
+    n = 8
+    count = (mib << 20) // 4
+    R1, R2 = {0, 1, 2, 4, 5, 7}, {3, 6}
+    t1 = G.allreduce_mask_aware_stars(n, R1, chunk=262144)
+    t2 = G.allreduce_mask_aware_stars(n, R2, chunk=262144)
+    comm = pkg.Communicator.loopback(n, scratch_bytes=2 * (mib << 20) + (16 << 20), mode="staged")
+    xs = rank_tensors("f32", count, n)
+    dx = [to_dev(x, "f32") for x in xs]
+    dy = [torch.empty_like(t) for t in dx]
+    comm.set_strategy("allreduce", t1)
+    comm.allreduce_lb([x if r in R1 else None for r, x in enumerate(dx)], dy, ready=R1)
+    comm.set_strategy("allreduce", t2)
+    comm.allreduce_lb([x if r in R2 else None for r, x in enumerate(dx)], dy, ready=R2, accumulate=True)
+    torch.cuda.synchronize()
+    assert comm.get_async_error() == 0
+    idx = _samples(count)
+    vals = [x[idx] for x in xs]
+    p1 = oc.allreduce_elements([v if r in R1 else None for r, v in enumerate(vals)], idx, count, t1, R1, "f32")
+    p2 = oc.allreduce_elements([v if r in R2 else None for r, v in enumerate(vals)], idx, count, t2, R2, "f32",
+                               accumulate=True, y_prev=p1)
+    for g in _gather(dy, idx, "f32"):
+        assert np.array_equal(bits(g), bits(p2))
+    full = oc.allreduce_exact(vals, set(range(n)), "f32")
+    assert np.max(np.abs(p2.astype(np.float64) - full)) / np.max(np.abs(full)) < 1e-6
+    comm.finalize()
+
+
+@pytest.mark.parametrize("mode", ["direct", "staged"])
+def test_c4_alltoall_full(mode):
+    """C4: 8 ranks, [8 dest][512 tokens][4096] bf16 per rank, checked completely."""
+    n, cnt = 8, 512 * 4096
+    text = G.alltoall_direct(n, chunk=1 << 20)
+    comm = pkg.Communicator.loopback(n, scratch_bytes=(2 * n * cnt * 2 + (8 << 20)) if mode == "staged"
+                                     else 64 << 20, mode=mode)
+    comm.set_strategy("alltoall", text)
+    xs = rank_tensors("bf16", n * cnt, n, base=2000)
+    dx = [to_dev(x, "bf16") for x in xs]
+    dy = [torch.empty_like(t) for t in dx]
+    comm.alltoall_lb(dx, dy)
+    torch.cuda.synchronize()
+    prev = [np.zeros(n * cnt, np.uint16)] * n
+    exp = oc.alltoall(xs, text, set(range(n)), "bf16", prev)
+    for g in range(n):
+        assert np.array_equal(to_host(dy[g], "bf16"), exp[g])
+    comm.finalize()
+
+
+@pytest.mark.parametrize("n", [2, 8])
+def test_c5_allgather_gpt2xl_with_swap(n):
+    """C5: 192 AllGathers of GPT-2-XL row shards (48 layers x 4 weights), strategy
+    swapped at call 96 (star, 256 KiB -> chain, 1 MiB), all enqueued back to back."""
+    comm = pkg.Communicator.loopback(n, scratch_bytes=256 << 20, mode="staged")
+    t_a, t_b = G.allgather_stars(n, chunk=262144), G.allgather_chains(n, chunk=1 << 20)
+    comm.set_strategy("allgather", t_a)
+    cache = {}
+    calls = []
+    for layer in range(48):
+        for wi, (_, rows, cols) in enumerate(GPT2XL_LAYERS):
+            call = layer * 4 + wi
+            if call == 96:
+                comm.set_strategy("allgather", t_b)
+            key = (wi, layer % 3)
+            if key not in cache:
+                cnt = rows // n * cols
+                xs = rank_tensors("bf16", cnt, n, base=3000 + 10 * wi + layer % 3)
+                cache[key] = (xs, [to_dev(x, "bf16") for x in xs])
+            xs, dx = cache[key]
+            dy = [torch.empty(n * len(xs[0]), dtype=torch.bfloat16, device="cuda") for _ in range(n)]
+            comm.allgather_lb(dx, dy)
+            calls.append((xs, dy))
+    torch.cuda.synchronize()
+    assert comm.get_async_error() == 0
+    for call, (xs, dy) in enumerate(calls):
+        cnt = len(xs[0])
+        idx = _samples(n * cnt, k=512, seed=call)
+        exp = np.concatenate(xs)[idx]
+        for g in _gather(dy, idx, "bf16"):
+            assert np.array_equal(g, exp), call
+    comm.finalize()
