@@ -118,12 +118,18 @@ def _mask(ready, n):
     return m
 
 
+_TORCH_CODES = None
+
+
 def _dtype_code(t):
-    import torch
-    codes = {torch.float32: 0, torch.bfloat16: 1, torch.int32: 2}
-    if t.dtype not in codes:
+    global _TORCH_CODES
+    if _TORCH_CODES is None:
+        import torch
+        _TORCH_CODES = {torch.float32: 0, torch.bfloat16: 1, torch.int32: 2}
+    code = _TORCH_CODES.get(t.dtype)
+    if code is None:
         raise TypeError(f"unsupported dtype {t.dtype}")
-    return codes[t.dtype]
+    return code
 
 
 def _stream(stream):
@@ -304,9 +310,15 @@ class Communicator:
     # ---- loopback collectives (lists of per-virtual-rank tensors)
     def _arrays(self, xs, outs, m):
         n = self.nranks
-        S = (ctypes.c_void_p * n)(*[(xs[r].data_ptr() if ((m >> r) & 1 and xs[r] is not None) else 0)
-                                    for r in range(n)])
-        D = (ctypes.c_void_p * n)(*[outs[r].data_ptr() for r in range(n)])
+        skey = tuple((xs[r].data_ptr() if ((m >> r) & 1 and xs[r] is not None) else 0)
+                     for r in range(n))
+        dkey = tuple(o.data_ptr() for o in outs)
+        cached = getattr(self, "_arr_cache", None)
+        if cached is not None and cached[0] == skey and cached[1] == dkey:
+            return cached[2], cached[3]
+        S = (ctypes.c_void_p * n)(*skey)
+        D = (ctypes.c_void_p * n)(*dkey)
+        self._arr_cache = (skey, dkey, S, D)
         return S, D
 
     def allreduce_lb(self, xs, outs, ready=None, accumulate=False, stream=None):

@@ -42,6 +42,7 @@ struct DevSegment {
 struct DevPlan {
   std::vector<DevSegment> segs;
   cudaEvent_t last_use = nullptr;
+  uint64_t last_tick = 0;
   ~DevPlan() {
     if (last_use) {
       cudaEventSynchronize(last_use);
@@ -99,14 +100,13 @@ struct adapcc_comm_s {
   uint64_t half_bytes = 0;
   char* own_arena = nullptr;               // loopback: all virtual ranks' arenas
   std::vector<char*> arena;                // per rank base (peer-mapped in IPC mode)
-  unsigned* counters = nullptr;
+  DevState* state = nullptr;              // device epoch + work counters
   int* h_err = nullptr;
   int* d_err = nullptr;
-  uint64_t epoch = 0;
   Strategy strat[3];
   uint64_t strat_version[3] = {0, 0, 0};
   std::map<PlanKey, std::shared_ptr<DevPlan>> plans;
-  std::list<PlanKey> lru;
+  uint64_t tick = 0;  // plan-cache clock (least recently used plan is evicted)
   int64_t timeout_ms = 10000;
   int64_t max_ctas = 0;
   int64_t drop_rank = -1;
@@ -144,8 +144,8 @@ adapcc_result_t common_init(adapcc_comm_s* c, size_t scratch) {
     CK(engine_occupancy(d, &c->occ[d]));
     if (c->occ[d] < 1) c->occ[d] = 1;
   }
-  CK(cudaMalloc(&c->counters, 4 * sizeof(unsigned)));
-  CK(cudaMemset(c->counters, 0, 4 * sizeof(unsigned)));
+  CK(cudaMalloc(&c->state, sizeof(DevState)));
+  CK(cudaMemset(c->state, 0, sizeof(DevState)));
   CK(cudaHostAlloc(&c->h_err, sizeof(int), cudaHostAllocMapped));
   *c->h_err = 0;
   CK(cudaHostGetDevicePointer(&c->d_err, c->h_err, 0));
@@ -170,7 +170,7 @@ void release(adapcc_comm_s* c) {
       else if (c->arena[r]) cudaIpcCloseMemHandle(c->arena[r]);
     }
   }
-  cudaFree(c->counters);
+  cudaFree(c->state);
   cudaFreeHost(c->h_err);
   delete c;
 }
@@ -203,8 +203,7 @@ adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, uint64_t count, adapcc_dty
   PlanKey key{(int)coll, c->strat_version[coll], count, (int)dtype, mask, flags};
   auto it = c->plans.find(key);
   if (it != c->plans.end()) {
-    c->lru.remove(key);
-    c->lru.push_front(key);
+    it->second->last_tick = ++c->tick;
     *out = it->second;
     return ADAPCC_SUCCESS;
   }
@@ -242,12 +241,13 @@ adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, uint64_t count, adapcc_dty
   // in loopback an empty call launches nothing; in multi-process mode every
   // rank launches every segment so that epochs stay aligned across ranks
   if (c->plans.size() >= (size_t)kPlanCacheCap) {
-    PlanKey victim = c->lru.back();
-    c->lru.pop_back();
+    auto victim = c->plans.begin();
+    for (auto i = c->plans.begin(); i != c->plans.end(); ++i)
+      if (i->second->last_tick < victim->second->last_tick) victim = i;
     c->plans.erase(victim);  // DevPlan dtor waits for its last launch
   }
+  plan->last_tick = ++c->tick;
   c->plans[key] = plan;
-  c->lru.push_front(key);
   *out = plan;
   return ADAPCC_SUCCESS;
 }
@@ -274,11 +274,10 @@ adapcc_result_t run(adapcc_comm_s* c, Coll coll, const void* const* send, void* 
     P.my_rank = c->loopback ? -1 : c->rank;
     P.ipc = c->loopback ? 0 : 1;
     P.drop_rank = (int)c->drop_rank;
-    P.epoch = ++c->epoch;
+    P.half_bytes = c->half_bytes;
     P.timeout_ns = (uint64_t)std::max<int64_t>(1, c->timeout_ms) * 1000000ull;
-    P.counters = c->counters;
+    P.state = c->state;
     P.err = c->d_err;
-    const uint64_t parity = P.epoch & 1;
     for (int q = 0; q < c->nranks; ++q) {
       if (c->loopback || q == c->rank) {
         const int i = c->loopback ? q : 0;
@@ -286,7 +285,6 @@ adapcc_result_t run(adapcc_comm_s* c, Coll coll, const void* const* send, void* 
         P.recv[q] = static_cast<char*>(recv[i]);
       }
       P.hdr[q] = c->arena[q];
-      P.arena[q] = c->arena[q] + kArenaHeader + parity * c->half_bytes;
     }
     const int grid = std::max(1, std::min<int>(grid_size(c, dtype), (int)std::max<uint32_t>(1, seg.nitems)));
     CK(engine_launch(P, grid, s));

@@ -1,19 +1,24 @@
 // AdapCC transfer engine: one persistent sm_100a kernel per collective call.
 //
-// Each CTA repeatedly claims the next work item (task, chunk) from a per-rank
-// counter, waits for the chunk's input flags (system-scope acquire; the
-// paper's cudaStreamWaitEvent per chunk), folds its K source
-// streams left to right with 128-bit loads (the aggregation kernel, P:L154,
-// P:L265), writes the result to its D destinations -- local HBM, or a peer
-// GPU's IPC-mapped arena over NVLink -- and posts the chunk's output flags
-// (system-scope release; the paper's cudaEventRecord after
-// cudaMemcpyPeerAsync).  Reduce and broadcast stages of every tree
-// run in the same launch and pipeline chunk by chunk.
+// Each CTA repeatedly claims the next work item (task, chunk, piece) from a
+// per-rank counter, waits for the chunk's input flags (acquire; the paper's
+// cudaStreamWaitEvent per chunk), folds its K source streams left
+// to right with 128-bit loads (the aggregation kernel), writes
+// the result to its D destinations -- local HBM, or a peer GPU's IPC-mapped
+// arena over NVLink -- and posts the chunk's output flags (release; the
+// paper's cudaEventRecord after cudaMemcpyPeerAsync).  Reduce and
+// broadcast stages of every tree run in the same launch and pipeline chunk by
+// chunk.
 //
 // Arithmetic (DESIGN.md §3 Q6): fp32 adds in IEEE RNE (__fadd_rn, no FTZ, no
 // contraction); bf16 widened to fp32, folded, rounded ONCE per task with RNE;
 // int32 wraps.  A single-source task without accumulation copies bytes
 // unchanged (relay forwarding, broadcast).
+//
+// Epochs live on the device (DevState): every launch reads the epoch the
+// previous launch on this communicator published, so captured CUDA graphs can
+// be replayed any number of times.  Memory-model scope: .gpu in loopback (one
+// device), .sys across processes / GPUs.
 #include <cuda_bf16.h>
 #include <cuda_runtime.h>
 
@@ -26,20 +31,26 @@ namespace adapcc {
 namespace {
 
 constexpr int kThreads = 256;
-#ifndef ADAPCC_UNROLL
-#define ADAPCC_UNROLL 8   // 128-bit vectors in flight per thread per source
-#endif
 #ifndef ADAPCC_MINB
 #define ADAPCC_MINB 2     // resident CTAs per SM the register budget is sized for
 #endif
+#ifndef ADAPCC_COPY_UNROLL
+#define ADAPCC_COPY_UNROLL 4  // 128-bit vectors in flight per thread for 1-source tasks
+#endif
 
-__device__ __forceinline__ uint64_t ld_acquire_sys(const uint64_t* p) {
+__device__ __forceinline__ uint64_t ld_acquire(const uint64_t* p, bool sys) {
   uint64_t v;
-  asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  if (sys) asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  else asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
   return v;
 }
-__device__ __forceinline__ void st_release_sys(uint64_t* p, uint64_t v) {
-  asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+__device__ __forceinline__ void st_release(uint64_t* p, uint64_t v, bool sys) {
+  if (sys) asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+  else asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ void fence(bool sys) {
+  if (sys) __threadfence_system();
+  else __threadfence();
 }
 __device__ __forceinline__ uint64_t globaltimer() {
   uint64_t t;
@@ -130,89 +141,115 @@ template <> struct Ops<kI32> {
   __device__ static E n1(uint32_t a) { return a; }
 };
 
+struct Cur {  // header of the work item being executed (staged by thread 0)
+  uint64_t e0;
+  uint32_t ref0, flag0, chunk, len;
+  uint16_t nsrc, ndst, nwait, npost, op;
+  bool dropped;
+};
+
 struct Shared {
+  Cur cur;
   const char* src[kMaxFold];
   char* dst[kMaxDst];
   uint8_t acc[kMaxDst];
+  uint64_t epoch;
   uint32_t item;
   int bad_align;
   int abort;
   int any_acc;
 };
 
-// ---------------------------------------------------------- vector fold
-// Sources are folded one at a time with U 128-bit loads in flight per thread
-// (U=8: 8 x 16 B x 256 threads x 2 CTAs = 64 KB in flight per SM, enough to
-// cover HBM / NVLink latency); the accumulator stays in registers.  Vector
-// indices are 32-bit (a chunk is at most 2^31 bytes).
+// ---------------------------------------------------------------- vector fold
+// Thread t handles vectors base, base + 256, ..., base + (U-1)*256 of a
+// stride of U*256 vectors; addresses are one per-stream pointer plus
+// immediate offsets (keeps the register count low).
 template <int U>
-__device__ __forceinline__ void load_u(uint4 (&x)[U], const char* src, uint32_t base, uint32_t nvec,
+__device__ __forceinline__ void load_u(uint4 (&x)[U], const char* p, uint32_t base, uint32_t nvec,
                                        bool full) {
-  if (full) {
 #pragma unroll
-    for (int u = 0; u < U; ++u) x[u] = ld16(src + (size_t)(base + u * kThreads) * 16);
-  } else {
-#pragma unroll
-    for (int u = 0; u < U; ++u)
-      if (base + u * kThreads < nvec) x[u] = ld16(src + (size_t)(base + u * kThreads) * 16);
-  }
+  for (int u = 0; u < U; ++u)
+    if (full || base + u * kThreads < nvec) x[u] = ld16(p + u * kThreads * 16);
 }
 
 template <int U>
-__device__ __forceinline__ void store_u(char* dst, const uint4 (&x)[U], uint32_t base, uint32_t nvec,
+__device__ __forceinline__ void store_u(char* p, const uint4 (&x)[U], uint32_t base, uint32_t nvec,
                                         bool full) {
-  if (full) {
 #pragma unroll
-    for (int u = 0; u < U; ++u) st16(dst + (size_t)(base + u * kThreads) * 16, x[u]);
-  } else {
-#pragma unroll
-    for (int u = 0; u < U; ++u)
-      if (base + u * kThreads < nvec) st16(dst + (size_t)(base + u * kThreads) * 16, x[u]);
-  }
+  for (int u = 0; u < U; ++u)
+    if (full || base + u * kThreads < nvec) st16(p + u * kThreads * 16, x[u]);
 }
 
 template <int DT, int U>
+__device__ __forceinline__ void write_dsts(const Shared& sh, int ndst, const uint4 (&x)[U], uint32_t base,
+                                           uint32_t nvec, bool full) {
+  using O = Ops<DT>;
+  const size_t off = (size_t)base * 16;
+  for (int d = 0; d < ndst; ++d) {
+    char* p = sh.dst[d] + off;
+    if (sh.acc[d]) {  // recv += result (phase 2): one vector at a time
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        if (full || base + u * kThreads < nvec) {
+          typename O::Acc q = O::widen(ld16(p + u * kThreads * 16));
+          O::add(q, x[u]);
+          st16(p + u * kThreads * 16, O::narrow(q));
+        }
+      }
+    } else {
+      store_u<U>(p, x, base, nvec, full);
+    }
+  }
+}
+
+// One source: bytes unchanged (relay forwarding, broadcast, AllGather,
+// AlltoAll), U vectors in flight per thread.
+template <int DT, int U>
+__device__ __forceinline__ void copy_vec(const Shared& sh, int ndst, uint32_t nvec) {
+  for (uint32_t base = threadIdx.x; base < nvec; base += U * kThreads) {
+    const bool full = base + (U - 1) * kThreads < nvec;
+    uint4 x[U];
+    load_u<U>(x, sh.src[0] + (size_t)base * 16, base, nvec, full);
+    write_dsts<DT, U>(sh, ndst, x, base, nvec, full);
+  }
+}
+
+// K >= 2 sources: KB sources x U vectors of loads are issued before the first
+// add (KB*U = 8 loads in flight per thread; a small chunk costs one memory
+// round trip per KB sources instead of one per source).
+template <int DT, int U, int KB>
 __device__ __forceinline__ void fold_vec(const Shared& sh, int nsrc, int ndst, uint32_t nvec) {
   using O = Ops<DT>;
   for (uint32_t base = threadIdx.x; base < nvec; base += U * kThreads) {
     const bool full = base + (U - 1) * kThreads < nvec;
-    uint4 x[U];
-    load_u<U>(x, sh.src[0], base, nvec, full);
-    if (nsrc > 1) {
-      typename O::Acc a[U];
+    const size_t off = (size_t)base * 16;
+    typename O::Acc a[U];
+    for (int k0 = 0; k0 < nsrc; k0 += KB) {
+      uint4 x[KB][U];
 #pragma unroll
-      for (int u = 0; u < U; ++u) a[u] = O::widen(x[u]);
-      for (int k = 1; k < nsrc; ++k) {
-        load_u<U>(x, sh.src[k], base, nvec, full);
+      for (int j = 0; j < KB; ++j)
+        if (k0 + j < nsrc) load_u<U>(x[j], sh.src[k0 + j] + off, base, nvec, full);
 #pragma unroll
-        for (int u = 0; u < U; ++u) O::add(a[u], x[u]);
-      }
-#pragma unroll
-      for (int u = 0; u < U; ++u) x[u] = O::narrow(a[u]);  // one rounding per task
-    }
-    for (int d = 0; d < ndst; ++d) {
-      char* dst = sh.dst[d];
-      if (sh.acc[d]) {  // recv += result (phase 2): one vector at a time
+      for (int j = 0; j < KB; ++j) {
+        if (k0 + j >= nsrc) break;
 #pragma unroll
         for (int u = 0; u < U; ++u) {
-          const uint32_t v = base + u * kThreads;
-          if (v < nvec) {
-            typename O::Acc q = O::widen(ld16(dst + (size_t)v * 16));
-            O::add(q, x[u]);
-            st16(dst + (size_t)v * 16, O::narrow(q));
-          }
+          if (k0 + j == 0) a[u] = O::widen(x[0][u]);
+          else O::add(a[u], x[j][u]);
         }
-      } else {
-        store_u<U>(dst, x, base, nvec, full);  // bytes unchanged when nsrc == 1
       }
     }
+    uint4 r[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u) r[u] = O::narrow(a[u]);  // one rounding per task
+    write_dsts<DT, U>(sh, ndst, r, base, nvec, full);
   }
 }
 
-// element path: e in [e_begin, e_end) relative to the chunk start
+// element path (misaligned slots / ragged tail): e in [e_begin, e_end)
 template <int DT>
-__device__ __noinline__ void fold_scalar(const Shared& sh, int nsrc, int ndst, uint64_t e_begin,
-                                            uint64_t e_end) {
+__device__ __forceinline__ void fold_scalar(const Shared& sh, int nsrc, int ndst, uint64_t e_begin,
+                                         uint64_t e_end) {
   using O = Ops<DT>;
   using E = typename O::E;
   for (uint64_t e = e_begin + threadIdx.x; e < e_end; e += kThreads) {
@@ -253,21 +290,26 @@ __device__ void fold_chunk(const Shared& sh, int nsrc, int ndst, uint64_t n, int
     return;
   }
   constexpr int VE = 16 / O::kEsize;
-  const uint64_t nvec = n / VE;
-  fold_vec<DT, ADAPCC_UNROLL>(sh, nsrc, ndst, (uint32_t)nvec);
-  if (nvec * VE < n) fold_scalar<DT>(sh, nsrc, ndst, nvec * VE, n);
+  const uint32_t nvec = (uint32_t)(n / VE);
+  // bf16 accumulators are 8 floats per vector: fewer vectors per source
+  // keep the kernel within 128 registers (2 CTAs/SM) without spills
+  if (nsrc == 1) copy_vec<DT, ADAPCC_COPY_UNROLL>(sh, ndst, nvec);
+  else if (nsrc <= 4) fold_vec<DT, (DT == kBF16 ? 1 : 2), 4>(sh, nsrc, ndst, nvec);
+  else fold_vec<DT, 1, 8>(sh, nsrc, ndst, nvec);
+  if ((uint64_t)nvec * VE < n) fold_scalar<DT>(sh, nsrc, ndst, (uint64_t)nvec * VE, n);
 }
 
 // spin until *flag >= target; false on watchdog timeout or abort
 __device__ bool wait_flag(const uint64_t* flag, uint64_t target, const LaunchParams& P) {
-  if (ld_acquire_sys(flag) >= target) return true;
+  const bool sys = P.ipc;
+  if (ld_acquire(flag, sys) >= target) return true;
   const uint64_t t0 = globaltimer();
   for (uint32_t spin = 1;; ++spin) {
-    if (ld_acquire_sys(flag) >= target) return true;
+    if (ld_acquire(flag, sys) >= target) return true;
     if ((spin & 63) == 0) {
-      if (*reinterpret_cast<volatile unsigned*>(&P.counters[2])) return false;
+      if (*reinterpret_cast<volatile unsigned*>(&P.state->abort)) return false;
       if (globaltimer() - t0 > P.timeout_ns) {
-        atomicExch(&P.counters[2], 1u);
+        atomicExch(&P.state->abort, 1u);
         *reinterpret_cast<volatile int*>(P.err) = 7;  // ADAPCC_ERR_TIMEOUT
         __threadfence_system();
         return false;
@@ -276,49 +318,77 @@ __device__ bool wait_flag(const uint64_t* flag, uint64_t target, const LaunchPar
   }
 }
 
-__device__ __forceinline__ char* base_of(const LaunchParams& P, uint8_t kind, int rank) {
-  return kind == kBufSend ? P.send[rank] : kind == kBufRecv ? P.recv[rank] : P.arena[rank];
-}
-
 template <int DT>
 __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __grid_constant__ LaunchParams P) {
   __shared__ Shared sh;
-  if (threadIdx.x == 0) sh.abort = 0;
-  __syncthreads();
-  // multi-process: every peer must have finished the call that last used this
-  // parity half of the arenas (epoch - 2) before we write into any arena
-  if (P.ipc && P.epoch > 2) {
-    const int r = threadIdx.x;
-    if (r < P.nranks && r != P.my_rank) {
-      if (!wait_flag(reinterpret_cast<const uint64_t*>(P.hdr[r]), P.epoch - 2, P)) sh.abort = 1;
+  const bool sys = P.ipc;
+  if (threadIdx.x == 0) {
+    sh.abort = 0;
+    // this launch's epoch = the one the previous launch published + 1
+    const uint64_t e = *reinterpret_cast<volatile unsigned long long*>(&P.state->epoch) + 1;
+    sh.epoch = e;
+    if (blockIdx.x == 0) {  // re-arm the other parity's counters for the next launch
+      P.state->work[(e + 1) & 1] = 0;
+      P.state->done[(e + 1) & 1] = 0;
     }
   }
   __syncthreads();
+  const uint64_t epoch = sh.epoch;
+  const unsigned par = (unsigned)(epoch & 1);
+  const uint64_t half_off = kArenaHeader + par * P.half_bytes;
+  // multi-process: every peer must have finished the call that last used this
+  // parity half of the arenas (epoch - 2) before we write into any arena
+  if (P.ipc && epoch > 2) {
+    const int r = threadIdx.x;
+    if (r < P.nranks && r != P.my_rank) {
+      if (!wait_flag(reinterpret_cast<const uint64_t*>(P.hdr[r]), epoch - 2, P)) sh.abort = 1;
+    }
+    __syncthreads();
+  }
   constexpr int esize = Ops<DT>::kEsize;
   while (!sh.abort) {
-    if (threadIdx.x == 0) sh.item = atomicAdd(&P.counters[0], 1u);
+    if (threadIdx.x == 0) {
+      // claim the next item and stage its header in shared memory, so that no
+      // task field stays live in registers across the fold
+      const uint32_t it = atomicAdd(&P.state->work[par], 1u);
+      sh.item = it;
+      sh.bad_align = 0;
+      sh.any_acc = 0;
+      if (it < P.nitems) {
+        const Item item = P.items[it];
+        const Task& t = P.tasks[item.task];
+        Cur& c = sh.cur;
+        c.nsrc = t.nsrc;
+        c.ndst = t.ndst;
+        c.nwait = t.nwait;
+        c.npost = t.npost;
+        c.op = t.op;
+        c.dropped = (int)t.owner == P.drop_rank;
+        c.ref0 = t.ref0;
+        c.flag0 = t.flag0;
+        c.chunk = item.chunk;
+        c.len = item.len;
+        c.e0 = t.lo + (uint64_t)item.chunk * t.chunk_elems + item.off;
+      }
+    }
     __syncthreads();
-    const uint32_t it = sh.item;
-    if (it >= P.nitems) break;
-    const Item item = P.items[it];
-    const Task& t = P.tasks[item.task];
-    const int nsrc = t.nsrc, ndst = t.ndst;
-    const uint64_t e0 = t.lo + (uint64_t)item.chunk * t.chunk_elems + item.off;
-    const uint64_t e1 = e0 + item.len;
-    const bool dropped = (int)t.owner == P.drop_rank;
-    if (threadIdx.x == 0) { sh.bad_align = 0; sh.any_acc = 0; }
-    __syncthreads();
+    if (sh.item >= P.nitems) break;
+    const int nsrc = sh.cur.nsrc, ndst = sh.cur.ndst;
+    const bool dropped = sh.cur.dropped;
     if (!dropped) {
       // input flags, one waiter thread per flag
-      if (threadIdx.x < t.nwait) {
-        const FlagRef f = P.flags[t.flag0 + threadIdx.x];
-        const uint64_t* fl = reinterpret_cast<const uint64_t*>(P.arena[f.rank] + f.off) + item.chunk;
-        if (!wait_flag(fl, P.epoch, P)) sh.abort = 1;
+      if (threadIdx.x < sh.cur.nwait) {
+        const FlagRef f = P.flags[sh.cur.flag0 + threadIdx.x];
+        const uint64_t* fl =
+            reinterpret_cast<const uint64_t*>(P.hdr[f.rank] + half_off + f.off) + sh.cur.chunk;
+        if (!wait_flag(fl, epoch, P)) sh.abort = 1;
       }
-      // resolve stream pointers for this chunk
+      // resolve stream pointers for this piece
       if (threadIdx.x < nsrc + ndst) {
-        const BufRef r = P.refs[t.ref0 + threadIdx.x];
-        char* p = base_of(P, r.kind, r.rank) + r.bias + (int64_t)(e0 * esize);
+        const BufRef r = P.refs[sh.cur.ref0 + threadIdx.x];
+        char* base = r.kind == kBufSend ? P.send[r.rank]
+                   : r.kind == kBufRecv ? P.recv[r.rank] : P.hdr[r.rank] + half_off;
+        char* p = base + r.bias + (int64_t)(sh.cur.e0 * esize);
         if (reinterpret_cast<uintptr_t>(p) & 15) atomicOr(&sh.bad_align, 1);
         if (threadIdx.x < nsrc) {
           sh.src[threadIdx.x] = p;
@@ -332,29 +402,31 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
     __syncthreads();
     if (sh.abort) break;
     if (!dropped) {
-      fold_chunk<DT>(sh, nsrc, ndst, e1 - e0, t.op);
+      fold_chunk<DT>(sh, nsrc, ndst, sh.cur.len, sh.cur.op);
       __syncthreads();
-      if (threadIdx.x == 0 && t.npost) {
-        __threadfence_system();  // chunk bytes (incl. remote NVLink stores) before the flag
-        for (int i = 0; i < t.npost; ++i) {
-          const FlagRef f = P.flags[t.flag0 + t.nwait + i];
-          st_release_sys(reinterpret_cast<uint64_t*>(P.arena[f.rank] + f.off) + item.chunk, P.epoch);
+      if (threadIdx.x == 0 && sh.cur.npost) {
+        const uint64_t e = sh.epoch;
+        const char* const* hdr = P.hdr;
+        fence(sys);  // the chunk's bytes (incl. remote NVLink stores) before its flag
+        for (int i = 0; i < sh.cur.npost; ++i) {
+          const FlagRef f = P.flags[sh.cur.flag0 + sh.cur.nwait + i];
+          st_release(reinterpret_cast<uint64_t*>(const_cast<char*>(hdr[f.rank]) + half_off + f.off) +
+                         sh.cur.chunk, e, sys);
         }
       }
     }
   }
   __syncthreads();
   if (threadIdx.x == 0) {
-    __threadfence_system();
-    const unsigned done = atomicAdd(&P.counters[1], 1u);
+    fence(sys);
+    const unsigned done = atomicAdd(&P.state->done[par], 1u);
     if (done == gridDim.x - 1) {
-      // last CTA: re-arm the counters for the next launch on this stream and
-      // publish "this rank finished epoch" to the peers
-      P.counters[0] = 0;
-      P.counters[1] = 0;
+      // last CTA: publish the epoch for the next launch on this stream and,
+      // across processes, "this rank finished epoch" to the peers
+      *reinterpret_cast<volatile unsigned long long*>(&P.state->epoch) = epoch;
       if (P.ipc) {
         __threadfence_system();
-        st_release_sys(reinterpret_cast<uint64_t*>(P.hdr[P.my_rank]), P.epoch);
+        st_release(reinterpret_cast<uint64_t*>(P.hdr[P.my_rank]), epoch, true);
       }
     }
   }

@@ -11,6 +11,17 @@ namespace adapcc {
 
 constexpr int kMaxRanksDev = 64;
 
+// Per-communicator device state.  Counters are double-buffered by epoch
+// parity: launch e uses [e & 1] and block 0 re-arms [(e + 1) & 1] for the
+// next launch, so no host reset is needed between launches (CUDA graphs).
+struct DevState {
+  unsigned work[2];          // work-item cursor
+  unsigned done[2];          // finished CTAs
+  unsigned abort;            // watchdog fired
+  unsigned pad;
+  unsigned long long epoch;  // last completed launch
+};
+
 struct LaunchParams {
   const Task* tasks;
   const BufRef* refs;
@@ -19,17 +30,16 @@ struct LaunchParams {
   uint32_t nitems;
   int dtype;
   int nranks;
-  int my_rank;        // multi-process: this rank; loopback: -1
-  int ipc;            // 1: multi-process start check + done post
-  int drop_rank;      // test hook (loopback): tasks owned by this rank are skipped
-  uint64_t epoch;     // flag value of this launch (monotonic per communicator)
+  int my_rank;          // multi-process: this rank; loopback: -1
+  int ipc;              // 1: multi-process (.sys scope, start check, done publish)
+  int drop_rank;        // test hook (loopback): tasks owned by this rank are skipped
+  uint64_t half_bytes;  // bytes of one parity half of an arena
   uint64_t timeout_ns;
-  unsigned* counters; // device: [0] work cursor, [1] finished CTAs, [2] abort
-  int* err;           // host-mapped error word
+  DevState* state;
+  int* err;             // host-mapped error word
   char* send[kMaxRanksDev];
   char* recv[kMaxRanksDev];
-  char* arena[kMaxRanksDev];  // parity half of each rank's arena (peer-mapped)
-  char* hdr[kMaxRanksDev];    // arena header of each rank (done epoch at +0)
+  char* hdr[kMaxRanksDev];  // arena base of each rank (peer-mapped): [header | half 0 | half 1]
 };
 
 int engine_threads();

@@ -264,3 +264,30 @@ def test_argument_errors():
         comm.alltoall_lb(x, x)                                    # aliasing
     assert e.value.code == pkg.adapcc.INVALID_ARGUMENT
     comm.finalize()
+
+
+@pytest.mark.parametrize("mode", MODES)
+def test_cuda_graph_capture_and_replay(mode):
+    """Calls are capturable once their plan is cached (warm-up call first)."""
+    n, count = 4, 50_001
+    comm = _comm(n, mode)
+    text = G.allreduce_stars(n, chunk=16384)
+    comm.set_strategy("allreduce", text)
+    xs = rank_tensors("f32", count, n)
+    dx = [to_dev(x, "f32") for x in xs]
+    dy = [empty_dev(count, "f32") for _ in range(n)]
+    comm.allreduce_lb(dx, dy)          # warm-up builds and uploads the plan
+    torch.cuda.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g):
+        comm.allreduce_lb(dx, dy)
+        comm.allreduce_lb(dx, dy)
+    exp = oc.allreduce(xs, text, set(range(n)), "f32")
+    for rep in range(3):   # epochs advance on the device: replays never see stale flags
+        for t in dy:
+            t.zero_()
+        g.replay()
+        torch.cuda.synchronize()
+        assert comm.get_async_error() == 0
+        _assert_bits([to_host(t, "f32") for t in dy], exp, f"graph replay {rep}")
+    comm.finalize()
