@@ -158,6 +158,8 @@ ADAPCC_API adapcc_result_t adapcc_get_async_error(adapcc_comm_t comm);
 /* Synchronizes the device, unmaps peers, frees everything.  comm may be NULL. */
 ADAPCC_API adapcc_result_t adapcc_finalize(adapcc_comm_t comm);
 ADAPCC_API const char* adapcc_strerror(adapcc_result_t r);
+/* Text of the CUDA error behind the calling thread's last ADAPCC_ERR_CUDA. */
+ADAPCC_API const char* adapcc_last_cuda_error(void);
 
 /* Runtime knobs.  key: "timeout_ms" (watchdog, default 10000; env
  * ADAPCC_TIMEOUT_MS), "max_ctas" (grid cap, 0 = #SMs x occupancy; env

@@ -37,6 +37,8 @@ class AdapccError(RuntimeError):
     def __init__(self, code, where=""):
         self.code = code
         msg = _load().adapcc_strerror(code).decode() if code >= 0 else "error"
+        if code == CUDA:
+            msg += ": " + _load().adapcc_last_cuda_error().decode()
         super().__init__(f"{where}: adapcc error {code} ({msg})")
 
 
@@ -94,6 +96,8 @@ def _load():
         f.restype = ctypes.c_int
     L.adapcc_strerror.argtypes = [ctypes.c_int]
     L.adapcc_strerror.restype = ctypes.c_char_p
+    L.adapcc_last_cuda_error.argtypes = []
+    L.adapcc_last_cuda_error.restype = ctypes.c_char_p
     _lib = L
     return L
 

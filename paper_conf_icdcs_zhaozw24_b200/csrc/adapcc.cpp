@@ -9,6 +9,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <cstdio>
 #include <cstdlib>
 #include <cstring>
 #include <list>
@@ -43,6 +44,7 @@ struct DevPlan {
   std::vector<DevSegment> segs;
   cudaEvent_t last_use = nullptr;
   uint64_t last_tick = 0;
+  bool pinned = false;  // referenced by a captured CUDA graph: never evicted
   ~DevPlan() {
     if (last_use) {
       cudaEventSynchronize(last_use);
@@ -54,6 +56,7 @@ struct DevPlan {
       cudaFree(s.flags);
       cudaFree(s.items);
     }
+    cudaGetLastError();  // teardown errors must not leak into a later call's check
   }
 };
 
@@ -119,15 +122,20 @@ struct adapcc_comm_s {
 
 namespace {
 
-adapcc_result_t cuda_fail(cudaError_t e) {
-  (void)e;
+thread_local cudaError_t g_last_cuda_error = cudaSuccess;
+thread_local int g_last_cuda_line = 0;
+thread_local char g_last_cuda_msg[160];
+
+adapcc_result_t cuda_fail(cudaError_t e, int line) {
+  g_last_cuda_error = e;
+  g_last_cuda_line = line;
   return ADAPCC_ERR_CUDA;
 }
 
 #define CK(expr)                                   \
   do {                                             \
     cudaError_t _e = (expr);                       \
-    if (_e != cudaSuccess) return cuda_fail(_e);   \
+    if (_e != cudaSuccess) return cuda_fail(_e, __LINE__); \
   } while (0)
 
 adapcc_result_t common_init(adapcc_comm_s* c, size_t scratch) {
@@ -241,10 +249,11 @@ adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, uint64_t count, adapcc_dty
   // in loopback an empty call launches nothing; in multi-process mode every
   // rank launches every segment so that epochs stay aligned across ranks
   if (c->plans.size() >= (size_t)kPlanCacheCap) {
-    auto victim = c->plans.begin();
+    auto victim = c->plans.end();
     for (auto i = c->plans.begin(); i != c->plans.end(); ++i)
-      if (i->second->last_tick < victim->second->last_tick) victim = i;
-    c->plans.erase(victim);  // DevPlan dtor waits for its last launch
+      if (!i->second->pinned && (victim == c->plans.end() || i->second->last_tick < victim->second->last_tick))
+        victim = i;
+    if (victim != c->plans.end()) c->plans.erase(victim);  // DevPlan dtor waits for its last launch
   }
   plan->last_tick = ++c->tick;
   c->plans[key] = plan;
@@ -261,6 +270,10 @@ adapcc_result_t run(adapcc_comm_s* c, Coll coll, const void* const* send, void* 
   adapcc_result_t r = get_plan(c, coll, count, dtype, mask, flags, &plan);
   if (r != ADAPCC_SUCCESS) return r;
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  cudaStreamCaptureStatus cap = cudaStreamCaptureStatusNone;
+  CK(cudaStreamIsCapturing(s, &cap));
+  const bool capturing = cap != cudaStreamCaptureStatusNone;
+  if (capturing) plan->pinned = true;  // the graph keeps pointing at these tables
   for (const DevSegment& seg : plan->segs) {
     if (c->loopback && seg.nitems == 0) continue;
     LaunchParams P{};
@@ -290,7 +303,7 @@ adapcc_result_t run(adapcc_comm_s* c, Coll coll, const void* const* send, void* 
     CK(engine_launch(P, grid, s));
     ++c->launches;
   }
-  CK(cudaEventRecord(plan->last_use, s));
+  if (!capturing) CK(cudaEventRecord(plan->last_use, s));
   return ADAPCC_SUCCESS;
 }
 
@@ -502,6 +515,12 @@ adapcc_result_t adapcc_alltoall_lb(adapcc_comm_t c, const void* const* sendbufs,
   r = check_lb(c, sendbufs, recvbufs, bytes, bytes, mask, 2);
   if (r != ADAPCC_SUCCESS) return r;
   return run(c, kAllToAll, sendbufs, recvbufs, count_per_peer, dtype, mask, 0, stream);
+}
+
+const char* adapcc_last_cuda_error(void) {
+  std::snprintf(g_last_cuda_msg, sizeof(g_last_cuda_msg), "%s (adapcc.cpp:%d)",
+                cudaGetErrorString(g_last_cuda_error), g_last_cuda_line);
+  return g_last_cuda_msg;
 }
 
 adapcc_result_t adapcc_get_async_error(adapcc_comm_t c) {

@@ -445,6 +445,7 @@ cudaError_t engine_occupancy(int dtype, int* blocks_per_sm) {
 }
 
 cudaError_t engine_launch(const LaunchParams& p, int grid, cudaStream_t stream) {
+  cudaGetLastError();  // clear any stale error so the check below is about this launch
   switch (p.dtype) {
     case kF32: engine_kernel<kF32><<<grid, kThreads, 0, stream>>>(p); break;
     case kBF16: engine_kernel<kBF16><<<grid, kThreads, 0, stream>>>(p); break;
