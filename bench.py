@@ -226,7 +226,8 @@ def run_single(args):
     tdt = torch.float32 if args.dtype == "f32" else torch.bfloat16
     text = G.allreduce_stars(n, chunk=args.chunk_kib * 1024)
 
-    comm = pkg.Communicator.loopback(n, device=0, scratch_bytes=max(64 << 20, 2 * nbytes + (8 << 20))
+    # staged: each half needs ~S of slots + a flag region of half/32
+    comm = pkg.Communicator.loopback(n, device=0, scratch_bytes=max(64 << 20, 2 * nbytes + nbytes // 8 + (16 << 20))
                                      if args.mode == "staged" else 64 << 20, mode=args.mode)
     comm.set_strategy("allreduce", text)
 

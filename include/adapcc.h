@@ -163,8 +163,9 @@ ADAPCC_API const char* adapcc_last_cuda_error(void);
 
 /* Runtime knobs.  key: "timeout_ms" (watchdog, default 10000; env
  * ADAPCC_TIMEOUT_MS), "max_ctas" (grid cap, 0 = #SMs x occupancy; env
- * ADAPCC_NCTAS), "debug_drop_rank" (loopback test hook: virtual rank r posts
- * nothing, so its consumers hit the watchdog; -1 = off). */
+ * ADAPCC_NCTAS), "engine" (2 = auto by call size, default; 1 = TMA bulk-copy
+ * pipeline; 0 = 128-bit LDG/STG fold; env ADAPCC_ENGINE), "debug_drop_rank" (loopback test hook:
+ * virtual rank r posts nothing, so its consumers hit the watchdog; -1 = off). */
 ADAPCC_API adapcc_result_t adapcc_config(adapcc_comm_t comm, const char* key, int64_t value);
 
 /* Number of engine kernel launches this communicator has issued. */

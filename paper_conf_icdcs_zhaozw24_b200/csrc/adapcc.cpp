@@ -41,6 +41,7 @@ struct DevSegment {
 };
 
 struct DevPlan {
+  int engine = 0;      // kernel this plan's pieces were sized for
   std::vector<DevSegment> segs;
   cudaEvent_t last_use = nullptr;
   uint64_t last_tick = 0;
@@ -116,7 +117,8 @@ struct adapcc_comm_s {
   int64_t piece_kib = 0;  // 0 = automatic (total traffic / (8 * grid))
   uint64_t launches = 0;
   int num_sms = 148;
-  int occ[3] = {1, 1, 1};
+  int occ[2][3] = {{1, 1, 1}, {1, 1, 1}};  // [engine][dtype] resident CTAs per SM
+  int engine = 2;  // 0: LDG/STG fold, 1: TMA bulk pipeline, 2: auto by call size
   std::mutex mu;
 };
 
@@ -145,12 +147,15 @@ adapcc_result_t common_init(adapcc_comm_s* c, size_t scratch) {
   c->arena_bytes = kArenaHeader + 2 * c->half_bytes;
   c->timeout_ms = env_int("ADAPCC_TIMEOUT_MS", 10000);
   c->max_ctas = env_int("ADAPCC_NCTAS", 0);
+  c->engine = (int)std::min<int64_t>(2, std::max<int64_t>(0, env_int("ADAPCC_ENGINE", 2)));
   c->piece_kib = env_int("ADAPCC_PIECE_KIB", 0);
   CK(cudaSetDevice(c->device));
   CK(cudaDeviceGetAttribute(&c->num_sms, cudaDevAttrMultiProcessorCount, c->device));
   for (int d = 0; d < 3; ++d) {
-    CK(engine_occupancy(d, &c->occ[d]));
-    if (c->occ[d] < 1) c->occ[d] = 1;
+    CK(engine_occupancy(d, &c->occ[0][d]));
+    CK(engine_tma_occupancy(d, &c->occ[1][d]));
+    for (int k = 0; k < 2; ++k)
+      if (c->occ[k][d] < 1) c->occ[k][d] = 1;
   }
   CK(cudaMalloc(&c->state, sizeof(DevState)));
   CK(cudaMemset(c->state, 0, sizeof(DevState)));
@@ -200,8 +205,12 @@ bool overlap(const void* a, size_t an, const void* b, size_t bn) {
   return x < y + bn && y < x + an;
 }
 
-int grid_size(const adapcc_comm_s* c, adapcc_dtype_t dtype) {
-  int grid = c->num_sms * c->occ[(int)dtype];
+// Measured crossover (profiles/sizes_*_r01.json): below ~64 MiB of traffic per
+// launch the LDG kernel's lower fixed cost wins, above it the TMA pipeline.
+constexpr uint64_t kTmaMinTraffic = uint64_t(64) << 20;
+
+int grid_size(const adapcc_comm_s* c, adapcc_dtype_t dtype, int engine) {
+  int grid = c->num_sms * c->occ[engine][(int)dtype];
   if (c->max_ctas > 0) grid = (int)std::min<int64_t>(grid, c->max_ctas);
   return std::max(grid, 1);
 }
@@ -227,10 +236,16 @@ adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, uint64_t count, adapcc_dty
   std::string err;
   if (!build_plan(rq, &segs, &err)) return ADAPCC_ERR_OOM;
   auto plan = std::make_shared<DevPlan>();
+  {
+    PlanStats st;
+    for (auto& sp : segs) accumulate_stats(sp, c->loopback ? -1 : c->rank, rq.esize, &st);
+    const uint64_t traffic = st.bytes_read + st.bytes_written;
+    plan->engine = c->engine != 2 ? c->engine : (traffic / std::max<size_t>(1, segs.size()) >= kTmaMinTraffic ? 1 : 0);
+  }
   CK(cudaEventCreateWithFlags(&plan->last_use, cudaEventDisableTiming));
   for (auto& sp : segs) {
     DevSegment d;
-    std::vector<Item> items = order_items(sp, c->loopback ? -1 : c->rank, rq.esize, grid_size(c, dtype),
+    std::vector<Item> items = order_items(sp, c->loopback ? -1 : c->rank, rq.esize, grid_size(c, dtype, plan->engine),
                                           (uint64_t)c->piece_kib * 1024);
     d.nitems = (uint32_t)items.size();
     auto up = [](auto** dst, const auto& v) -> cudaError_t {
@@ -299,8 +314,8 @@ adapcc_result_t run(adapcc_comm_s* c, Coll coll, const void* const* send, void* 
       }
       P.hdr[q] = c->arena[q];
     }
-    const int grid = std::max(1, std::min<int>(grid_size(c, dtype), (int)std::max<uint32_t>(1, seg.nitems)));
-    CK(engine_launch(P, grid, s));
+    const int grid = std::max(1, std::min<int>(grid_size(c, dtype, plan->engine), (int)std::max<uint32_t>(1, seg.nitems)));
+    CK(plan->engine ? engine_tma_launch(P, grid, s) : engine_launch(P, grid, s));
     ++c->launches;
   }
   if (!capturing) CK(cudaEventRecord(plan->last_use, s));
@@ -538,6 +553,11 @@ adapcc_result_t adapcc_config(adapcc_comm_t c, const char* key, int64_t value) {
   std::lock_guard<std::mutex> lock(c->mu);
   if (!std::strcmp(key, "timeout_ms")) { if (value < 1) return ADAPCC_ERR_INVALID_ARGUMENT; c->timeout_ms = value; }
   else if (!std::strcmp(key, "max_ctas")) { if (value < 0) return ADAPCC_ERR_INVALID_ARGUMENT; c->max_ctas = value; }
+  else if (!std::strcmp(key, "engine")) {
+    if (value < 0 || value > 2) return ADAPCC_ERR_INVALID_ARGUMENT;
+    if (value != c->engine) c->plans.clear();  // pieces are sized for the engine's grid
+    c->engine = (int)value;
+  }
   else if (!std::strcmp(key, "debug_drop_rank")) {
     if (!c->loopback || value < -1 || value >= c->nranks) return ADAPCC_ERR_INVALID_ARGUMENT;
     c->drop_rank = value;

@@ -1,0 +1,141 @@
+// Device helpers shared by the transfer-engine kernels (engine.cu: 128-bit
+// LDG/STG fold; engine_tma.cu: TMA bulk-copy pipeline).  Internal header.
+#pragma once
+
+#include <cuda_bf16.h>
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+#include "engine.cuh"
+#include "launch.hpp"
+
+namespace adapcc {
+namespace dev {
+
+__device__ __forceinline__ uint64_t ld_acquire(const uint64_t* p, bool sys) {
+  uint64_t v;
+  if (sys) asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  else asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release(uint64_t* p, uint64_t v, bool sys) {
+  if (sys) asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+  else asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ void fence(bool sys) {
+  if (sys) __threadfence_system();
+  else __threadfence();
+}
+__device__ __forceinline__ uint64_t globaltimer() {
+  uint64_t t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+
+// 128-bit load/store; .cg keeps in-kernel-produced data out of L1
+__device__ __forceinline__ uint4 ld16(const char* p) { return __ldcg(reinterpret_cast<const uint4*>(p)); }
+__device__ __forceinline__ void st16(char* p, uint4 v) { __stcg(reinterpret_cast<uint4*>(p), v); }
+
+// ------------------------------------------------------------ dtype traits
+template <int DT> struct Ops;
+
+template <> struct Ops<kF32> {
+  static constexpr int kEsize = 4;
+  struct Acc { float v[4]; };
+  __device__ static Acc widen(uint4 x) {
+    return {{__uint_as_float(x.x), __uint_as_float(x.y), __uint_as_float(x.z), __uint_as_float(x.w)}};
+  }
+  __device__ static void add(Acc& a, uint4 x) {
+    a.v[0] = __fadd_rn(a.v[0], __uint_as_float(x.x));
+    a.v[1] = __fadd_rn(a.v[1], __uint_as_float(x.y));
+    a.v[2] = __fadd_rn(a.v[2], __uint_as_float(x.z));
+    a.v[3] = __fadd_rn(a.v[3], __uint_as_float(x.w));
+  }
+  __device__ static uint4 narrow(const Acc& a) {
+    return make_uint4(__float_as_uint(a.v[0]), __float_as_uint(a.v[1]), __float_as_uint(a.v[2]),
+                      __float_as_uint(a.v[3]));
+  }
+  // scalar element path (misaligned slots / ragged tail)
+  using E = uint32_t;
+  __device__ static float w1(E x) { return __uint_as_float(x); }
+  __device__ static float a1(float a, E x) { return __fadd_rn(a, __uint_as_float(x)); }
+  __device__ static E n1(float a) { return __float_as_uint(a); }
+};
+
+template <> struct Ops<kBF16> {
+  static constexpr int kEsize = 2;
+  struct Acc { float v[8]; };
+  __device__ static void w2(uint32_t p, float& lo, float& hi) {
+    lo = __uint_as_float(p << 16);
+    hi = __uint_as_float(p & 0xFFFF0000u);
+  }
+  __device__ static Acc widen(uint4 x) {
+    Acc a;
+    w2(x.x, a.v[0], a.v[1]);
+    w2(x.y, a.v[2], a.v[3]);
+    w2(x.z, a.v[4], a.v[5]);
+    w2(x.w, a.v[6], a.v[7]);
+    return a;
+  }
+  __device__ static void add(Acc& a, uint4 x) {
+    Acc b = widen(x);
+#pragma unroll
+    for (int i = 0; i < 8; ++i) a.v[i] = __fadd_rn(a.v[i], b.v[i]);
+  }
+  __device__ static uint32_t n2(float lo, float hi) {
+    __nv_bfloat162 h = __floats2bfloat162_rn(lo, hi);  // cvt.rn.bf16x2.f32: RNE
+    return *reinterpret_cast<uint32_t*>(&h);
+  }
+  __device__ static uint4 narrow(const Acc& a) {
+    return make_uint4(n2(a.v[0], a.v[1]), n2(a.v[2], a.v[3]), n2(a.v[4], a.v[5]), n2(a.v[6], a.v[7]));
+  }
+  using E = uint16_t;
+  __device__ static float w1(E x) { return __uint_as_float(uint32_t(x) << 16); }
+  __device__ static float a1(float a, E x) { return __fadd_rn(a, w1(x)); }
+  __device__ static E n1(float a) {
+    __nv_bfloat16 h = __float2bfloat16_rn(a);
+    return *reinterpret_cast<uint16_t*>(&h);
+  }
+};
+
+template <> struct Ops<kI32> {
+  static constexpr int kEsize = 4;
+  struct Acc { uint32_t v[4]; };
+  __device__ static Acc widen(uint4 x) { return {{x.x, x.y, x.z, x.w}}; }
+  __device__ static void add(Acc& a, uint4 x) {
+    a.v[0] += x.x;  // unsigned: wraps mod 2^32 (reading Q15)
+    a.v[1] += x.y;
+    a.v[2] += x.z;
+    a.v[3] += x.w;
+  }
+  __device__ static uint4 narrow(const Acc& a) { return make_uint4(a.v[0], a.v[1], a.v[2], a.v[3]); }
+  using E = uint32_t;
+  __device__ static uint32_t w1(E x) { return x; }
+  __device__ static uint32_t a1(uint32_t a, E x) { return a + x; }
+  __device__ static E n1(uint32_t a) { return a; }
+};
+
+
+// spin until *flag >= target; false on watchdog timeout or abort
+static __device__ __noinline__ bool wait_flag(const uint64_t* flag, uint64_t target, const LaunchParams& P) {
+  const bool sys = P.ipc;
+  if (ld_acquire(flag, sys) >= target) return true;
+  const uint64_t t0 = globaltimer();
+  for (uint32_t spin = 1;; ++spin) {
+    if (ld_acquire(flag, sys) >= target) return true;
+    if ((spin & 63) == 0) {
+      if (*reinterpret_cast<volatile unsigned*>(&P.state->abort)) return false;
+      if (globaltimer() - t0 > P.timeout_ns) {
+        atomicExch(&P.state->abort, 1u);
+        *reinterpret_cast<volatile int*>(P.err) = 7;  // ADAPCC_ERR_TIMEOUT
+        __threadfence_system();
+        return false;
+      }
+    }
+  }
+}
+
+
+}  // namespace dev
+}  // namespace adapcc

@@ -1,0 +1,438 @@
+// AdapCC transfer engine, TMA variant: warp-specialised persistent kernel in
+// which one producer warp moves every source tile with TMA bulk copies
+// (cp.async.bulk global -> shared, completion on an mbarrier) through a
+// 3-stage shared-memory ring, and 8 consumer warps fold the K tiles of a
+// stage from shared memory and store the result to the D destinations.
+//
+// Same work items, flags, epochs and deadlock-freedom argument as engine.cu
+// (DESIGN.md §6); what changes is the data path:
+//   - bytes in flight no longer cost registers: 2 CTAs x 3 stages x 32 KiB =
+//     192 KiB per SM, issued by ONE thread per CTA (the TMA engine does the
+//     addressing), also for peer (NVLink) sources;
+//   - the producer claims and waits for the next item while the consumers are
+//     still folding the current one (an item queue in shared memory), so the
+//     per-item claim / flag latency is hidden.
+// Paper mapping: the producer is the "receive" side of the chunk pipeline
+// (wait for the chunk, then aggregate), consumers are the
+// aggregation kernel + send.
+#include "engine_common.cuh"
+
+namespace adapcc {
+namespace {
+
+using namespace dev;
+
+constexpr int kConsumerWarps = 8;
+constexpr int kConsumers = kConsumerWarps * 32;
+constexpr int kTmaThreads = kConsumers + 32;  // + 1 producer warp
+constexpr int kStages = 3;
+constexpr uint32_t kStageBytes = 32768;
+constexpr int kMaxKS = 8;       // sources per stage
+constexpr int kQ = 2;           // item queue depth
+constexpr int kMaxPost = 4;
+
+struct ItemDesc {
+  const char* src[kMaxFold];
+  char* dst[kMaxDst];
+  uint64_t* post[kMaxPost];
+  uint64_t len;         // elements
+  uint32_t vec_bytes;   // bytes moved by tiles (multiple of 16)
+  uint32_t tile;        // bytes per source per stage
+  uint32_t ntiles;
+  uint16_t nsrc, ndst, op, npost, passes, ks;
+  uint8_t acc[kMaxDst];
+  uint8_t stop, dropped, scalar_only, any_acc;
+};
+
+struct Smem {
+  uint64_t full[kStages];
+  uint64_t empty[kStages];
+  uint64_t qfull[kQ];
+  uint64_t qempty[kQ];
+  uint64_t epoch;
+  int abort;
+  int pad;
+  ItemDesc q[kQ];
+};
+
+constexpr size_t kSmemHeader = (sizeof(Smem) + 127) / 128 * 128;
+constexpr size_t kSmemBytes = kSmemHeader + (size_t)kStages * kStageBytes;
+
+// ------------------------------------------------------------ PTX helpers
+__device__ __forceinline__ uint32_t su32(const void* p) {
+  return (uint32_t)__cvta_generic_to_shared(p);
+}
+__device__ __forceinline__ void mbar_init(uint64_t* b, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(su32(b)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* b, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(su32(b)), "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* b) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(su32(b)) : "memory");
+}
+__device__ __forceinline__ bool mbar_try(uint64_t* b, uint32_t parity) {
+  uint32_t ok;
+  asm volatile(
+      "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}\n"
+      : "=r"(ok)
+      : "r"(su32(b)), "r"(parity)
+      : "memory");
+  return ok != 0;
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* b, uint32_t parity) {
+  while (!mbar_try(b, parity)) {
+  }
+}
+// TMA bulk copy global -> shared, completes `bytes` on the mbarrier
+__device__ __forceinline__ void tma_load(void* sdst, const void* gsrc, uint32_t bytes, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          su32(sdst)),
+      "l"(gsrc), "r"(bytes), "r"(su32(bar))
+      : "memory");
+}
+__device__ __forceinline__ void fence_proxy_async() {
+  asm volatile("fence.proxy.async.global;" ::: "memory");
+}
+__device__ __forceinline__ void consumer_sync() {
+  asm volatile("bar.sync 1, %0;" ::"n"(kConsumers) : "memory");
+}
+__device__ __forceinline__ uint4 lds16(const char* p) { return *reinterpret_cast<const uint4*>(p); }
+
+// ------------------------------------------------------------ consumers
+template <int DT>
+__device__ __forceinline__ void store_result(const ItemDesc& d, size_t off, uint4 r) {
+  using O = Ops<DT>;
+  for (int k = 0; k < d.ndst; ++k) {
+    char* p = d.dst[k] + off;
+    if (d.acc[k]) {  // recv += result (phase 2)
+      typename O::Acc q = O::widen(ld16(p));
+      O::add(q, r);
+      st16(p, O::narrow(q));
+    } else {
+      st16(p, r);
+    }
+  }
+}
+
+// element path for misaligned streams and the sub-16-byte tail
+template <int DT>
+__device__ void scalar_range(const ItemDesc& d, uint64_t e_begin, uint64_t e_end, int tid) {
+  using O = Ops<DT>;
+  using E = typename O::E;
+  for (uint64_t e = e_begin + tid; e < e_end; e += kConsumers) {
+    E x0 = *reinterpret_cast<const volatile E*>(d.src[0] + e * sizeof(E));
+    E r;
+    if (d.nsrc == 1) {
+      r = x0;
+    } else {
+      auto a = O::w1(x0);
+      for (int k = 1; k < d.nsrc; ++k)
+        a = O::a1(a, *reinterpret_cast<const volatile E*>(d.src[k] + e * sizeof(E)));
+      r = O::n1(a);
+    }
+    for (int k = 0; k < d.ndst; ++k) {
+      E* p = reinterpret_cast<E*>(d.dst[k] + e * sizeof(E));
+      if (d.acc[k]) *p = O::n1(O::a1(O::w1(*reinterpret_cast<volatile E*>(p)), r));
+      else *p = r;
+    }
+  }
+}
+
+// Copy the tiles of a one-source item (bytes unchanged): VPT vectors per
+// thread per tile.
+template <int DT, int VPT>
+__device__ __forceinline__ void consume_copy(Smem& sm, char* stages, const ItemDesc& d, int tid,
+                                             uint32_t& stage, uint32_t& sphase) {
+  const bool warp_lane0 = (tid & 31) == 0;
+  for (uint32_t t = 0; t < d.ntiles; ++t) {
+    const uint32_t nv = min(d.tile, d.vec_bytes - t * d.tile) / 16;
+    uint4 raw[VPT];
+    mbar_wait(&sm.full[stage], sphase);
+    const char* sb = stages + (size_t)stage * kStageBytes;
+#pragma unroll
+    for (int j = 0; j < VPT; ++j) {
+      const uint32_t v = tid + j * kConsumers;
+      if (v < nv) raw[j] = lds16(sb + (size_t)v * 16);
+    }
+    __syncwarp();
+    if (warp_lane0) mbar_arrive(&sm.empty[stage]);
+    if (++stage == kStages) { stage = 0; sphase ^= 1; }
+#pragma unroll
+    for (int j = 0; j < VPT; ++j) {
+      const uint32_t v = tid + j * kConsumers;
+      if (v < nv) store_result<DT>(d, (size_t)t * d.tile + (size_t)v * 16, raw[j]);
+    }
+  }
+}
+
+// Fold the tiles of a K >= 2 item: every stage holds ks source tiles; a tile
+// of K > 8 sources spans several stages (passes) accumulated in registers.
+template <int DT, int VPT>
+__device__ __forceinline__ void consume_fold(Smem& sm, char* stages, const ItemDesc& d, int tid,
+                                             uint32_t& stage, uint32_t& sphase) {
+  using O = Ops<DT>;
+  const bool warp_lane0 = (tid & 31) == 0;
+  for (uint32_t t = 0; t < d.ntiles; ++t) {
+    const uint32_t nv = min(d.tile, d.vec_bytes - t * d.tile) / 16;
+    typename O::Acc a[VPT];
+    for (int p = 0; p < d.passes; ++p) {
+      const int ks = min((int)d.ks, (int)d.nsrc - p * (int)d.ks);
+      mbar_wait(&sm.full[stage], sphase);
+      const char* sb = stages + (size_t)stage * kStageBytes;
+#pragma unroll
+      for (int j = 0; j < VPT; ++j) {
+        const uint32_t v = tid + j * kConsumers;
+        if (v < nv) {
+          const char* pv = sb + (size_t)v * 16;
+          int k = 0;
+          if (p == 0) {
+            a[j] = O::widen(lds16(pv));
+            k = 1;
+          }
+          for (; k < ks; ++k) O::add(a[j], lds16(pv + (size_t)k * d.tile));
+        }
+      }
+      __syncwarp();
+      if (warp_lane0) mbar_arrive(&sm.empty[stage]);
+      if (++stage == kStages) { stage = 0; sphase ^= 1; }
+    }
+#pragma unroll
+    for (int j = 0; j < VPT; ++j) {
+      const uint32_t v = tid + j * kConsumers;
+      if (v < nv) store_result<DT>(d, (size_t)t * d.tile + (size_t)v * 16, O::narrow(a[j]));  // one rounding
+    }
+  }
+}
+
+// ------------------------------------------------------------- producer
+template <int DT>
+__device__ __forceinline__ void fill_desc(const LaunchParams& P, ItemDesc& d, const Item& item,
+                                          const Task& t, uint64_t half_off, int lane) {
+  constexpr int esize = Ops<DT>::kEsize;
+  const uint64_t e0 = t.lo + (uint64_t)item.chunk * t.chunk_elems + item.off;
+  int misaligned = 0;
+  for (int i = lane; i < t.nsrc + t.ndst; i += 32) {
+    const BufRef r = P.refs[t.ref0 + i];
+    char* base = r.kind == kBufSend ? P.send[r.rank] : r.kind == kBufRecv ? P.recv[r.rank]
+                                                                         : P.hdr[r.rank] + half_off;
+    char* p = base + r.bias + (int64_t)(e0 * esize);
+    misaligned |= (reinterpret_cast<uintptr_t>(p) & 15) != 0;
+    if (i < t.nsrc) {
+      d.src[i] = p;
+    } else {
+      d.dst[i - t.nsrc] = p;
+      d.acc[i - t.nsrc] = r.accum;
+    }
+  }
+  for (int i = lane; i < t.npost; i += 32) {
+    const FlagRef f = P.flags[t.flag0 + t.nwait + i];
+    d.post[i] = reinterpret_cast<uint64_t*>(P.hdr[f.rank] + half_off + f.off) + item.chunk;
+  }
+  misaligned = __any_sync(0xffffffffu, misaligned);
+  __syncwarp();
+  if (lane == 0) {
+    d.nsrc = t.nsrc;
+    d.ndst = t.ndst;
+    d.op = t.op;
+    d.npost = t.npost;
+    d.len = item.len;
+    d.dropped = (int)t.owner == P.drop_rank;
+    int any_acc = 0;
+    for (int k = 0; k < t.ndst; ++k) any_acc |= d.acc[k];
+    d.any_acc = any_acc;
+    const uint64_t bytes = (uint64_t)item.len * esize;
+    d.scalar_only = misaligned || t.op != kOpFold || bytes < 16;
+    d.vec_bytes = d.scalar_only ? 0 : (uint32_t)(bytes & ~uint64_t(15));
+    const int ks = t.nsrc < kMaxKS ? t.nsrc : kMaxKS;
+    d.ks = (uint16_t)ks;
+    d.passes = (uint16_t)((t.nsrc + kMaxKS - 1) / kMaxKS);
+    uint32_t tile = kStageBytes / (uint32_t)ks / 4096u * 4096u;
+    d.tile = tile;
+    d.ntiles = d.vec_bytes ? (d.vec_bytes + tile - 1) / tile : 0;
+  }
+}
+
+template <int DT>
+__global__ void __launch_bounds__(kTmaThreads, 2) engine_tma_kernel(const __grid_constant__ LaunchParams P) {
+  extern __shared__ __align__(128) unsigned char smem_raw[];
+  Smem& sm = *reinterpret_cast<Smem*>(smem_raw);
+  char* stages = reinterpret_cast<char*>(smem_raw) + kSmemHeader;
+  const int tid = threadIdx.x;
+  const int warp = tid >> 5, lane = tid & 31;
+  const bool sys = P.ipc;
+  if (tid == 0) {
+    for (int s = 0; s < kStages; ++s) {
+      mbar_init(&sm.full[s], 1);
+      mbar_init(&sm.empty[s], kConsumerWarps);
+    }
+    for (int s = 0; s < kQ; ++s) {
+      mbar_init(&sm.qfull[s], 1);
+      mbar_init(&sm.qempty[s], 1);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    sm.abort = 0;
+    const uint64_t e = *reinterpret_cast<volatile unsigned long long*>(&P.state->epoch) + 1;
+    sm.epoch = e;
+    if (blockIdx.x == 0) {
+      P.state->work[(e + 1) & 1] = 0;
+      P.state->done[(e + 1) & 1] = 0;
+    }
+  }
+  __syncthreads();
+  const uint64_t epoch = sm.epoch;
+  const unsigned par = (unsigned)(epoch & 1);
+  const uint64_t half_off = kArenaHeader + par * P.half_bytes;
+  if (P.ipc && epoch > 2) {  // peers done with the last user of this half
+    if (tid < P.nranks && tid != P.my_rank)
+      if (!wait_flag(reinterpret_cast<const uint64_t*>(P.hdr[tid]), epoch - 2, P)) sm.abort = 1;
+    __syncthreads();
+  }
+
+  if (warp == kConsumerWarps) {
+    // ================================================================ producer
+    uint32_t stage = 0, sphase = 0, qi = 0, qphase = 0;
+    for (;;) {
+      uint32_t it = 0;
+      int stop_i = 0;
+      if (lane == 0) {
+        it = atomicAdd(&P.state->work[par], 1u);
+        mbar_wait(&sm.qempty[qi], qphase ^ 1);  // queue slot free
+        stop_i = it >= P.nitems || *reinterpret_cast<volatile int*>(&sm.abort) != 0;
+      }
+      it = __shfl_sync(0xffffffffu, it, 0);
+      bool stop = __shfl_sync(0xffffffffu, stop_i, 0) != 0;
+      ItemDesc& d = sm.q[qi];
+      const Item item = stop ? Item{} : P.items[it];
+      const Task& t = P.tasks[item.task];
+      if (!stop) {
+        fill_desc<DT>(P, d, item, t, half_off, lane);
+        __syncwarp();
+        if (!d.dropped) {
+          int ok = 1;
+          for (int i = lane; i < t.nwait; i += 32) {
+            const FlagRef f = P.flags[t.flag0 + i];
+            const uint64_t* fl = reinterpret_cast<const uint64_t*>(P.hdr[f.rank] + half_off + f.off) + item.chunk;
+            ok &= wait_flag(fl, epoch, P);
+          }
+          if (!__all_sync(0xffffffffu, ok)) {
+            stop = true;
+            if (lane == 0) sm.abort = 1;
+          }
+        }
+      }
+      if (lane == 0) {
+        d.stop = stop;
+        fence_proxy_async();      // acquired peer/arena data -> async-proxy (TMA) reads
+        mbar_arrive(&sm.qfull[qi]);
+      }
+      __syncwarp();
+      if (stop) break;
+      if (!d.dropped && !d.scalar_only) {
+        for (uint32_t tt = 0; tt < d.ntiles; ++tt) {
+          const uint32_t tb = min(d.tile, d.vec_bytes - tt * d.tile);
+          for (int p = 0; p < d.passes; ++p) {
+            if (lane == 0) {
+              const int ks = min((int)d.ks, (int)d.nsrc - p * (int)d.ks);
+              mbar_wait(&sm.empty[stage], sphase ^ 1);
+              mbar_expect_tx(&sm.full[stage], (uint32_t)ks * tb);
+              char* sb = stages + (size_t)stage * kStageBytes;
+              for (int j = 0; j < ks; ++j)
+                tma_load(sb + (size_t)j * d.tile, d.src[p * d.ks + j] + (size_t)tt * d.tile, tb,
+                         &sm.full[stage]);
+            }
+            if (++stage == kStages) { stage = 0; sphase ^= 1; }
+          }
+        }
+      }
+      if (++qi == kQ) { qi = 0; qphase ^= 1; }
+    }
+  } else {
+    // =============================================================== consumers
+    uint32_t stage = 0, sphase = 0, qi = 0, qphase = 0;
+    for (;;) {
+      mbar_wait(&sm.qfull[qi], qphase);
+      const ItemDesc& d = sm.q[qi];
+      if (d.stop) break;
+      if (!d.dropped) {
+        if (d.op == kOpZero) {
+          using E = typename Ops<DT>::E;
+          for (int k = 0; k < d.ndst; ++k)
+            for (uint64_t e = tid; e < d.len; e += kConsumers) reinterpret_cast<E*>(d.dst[k])[e] = E(0);
+        } else {
+          if (!d.scalar_only) {
+            const uint32_t vpt = d.tile / (16u * kConsumers);  // 8 (K=1), 4, 2 or 1
+            if (d.nsrc == 1) consume_copy<DT, 8>(sm, stages, d, tid, stage, sphase);
+            else if (vpt >= 4) consume_fold<DT, 4>(sm, stages, d, tid, stage, sphase);
+            else if (vpt >= 2) consume_fold<DT, 2>(sm, stages, d, tid, stage, sphase);
+            else consume_fold<DT, 1>(sm, stages, d, tid, stage, sphase);
+          }
+          constexpr int esize = Ops<DT>::kEsize;
+          scalar_range<DT>(d, d.vec_bytes / esize, d.len, tid);
+        }
+        consumer_sync();  // every consumer's stores for this item are issued
+        if (tid == 0 && d.npost) {
+          fence(sys);      // the chunk's bytes (incl. remote NVLink stores) before its flag
+          for (int i = 0; i < d.npost; ++i) st_release(d.post[i], epoch, sys);
+        }
+      }
+      consumer_sync();    // all consumers are done reading the descriptor
+      if (tid == 0) mbar_arrive(&sm.qempty[qi]);
+      if (++qi == kQ) { qi = 0; qphase ^= 1; }
+    }
+  }
+  __syncthreads();
+  if (tid == 0) {
+    fence(sys);
+    const unsigned done = atomicAdd(&P.state->done[par], 1u);
+    if (done == gridDim.x - 1) {
+      *reinterpret_cast<volatile unsigned long long*>(&P.state->epoch) = epoch;
+      if (P.ipc) {
+        __threadfence_system();
+        st_release(reinterpret_cast<uint64_t*>(P.hdr[P.my_rank]), epoch, true);
+      }
+    }
+  }
+}
+
+template <int DT>
+cudaError_t prepare() {
+  static bool done = false;
+  if (done) return cudaSuccess;
+  cudaError_t e = cudaFuncSetAttribute(engine_tma_kernel<DT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       (int)kSmemBytes);
+  done = e == cudaSuccess;
+  return e;
+}
+
+}  // namespace
+
+int engine_tma_threads() { return kTmaThreads; }
+
+cudaError_t engine_tma_occupancy(int dtype, int* blocks_per_sm) {
+  switch (dtype) {
+    case kF32:
+      if (cudaError_t e = prepare<kF32>()) return e;
+      return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, engine_tma_kernel<kF32>, kTmaThreads, kSmemBytes);
+    case kBF16:
+      if (cudaError_t e = prepare<kBF16>()) return e;
+      return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, engine_tma_kernel<kBF16>, kTmaThreads, kSmemBytes);
+    default:
+      if (cudaError_t e = prepare<kI32>()) return e;
+      return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, engine_tma_kernel<kI32>, kTmaThreads, kSmemBytes);
+  }
+}
+
+cudaError_t engine_tma_launch(const LaunchParams& p, int grid, cudaStream_t stream) {
+  cudaGetLastError();
+  switch (p.dtype) {
+    case kF32: prepare<kF32>(); engine_tma_kernel<kF32><<<grid, kTmaThreads, kSmemBytes, stream>>>(p); break;
+    case kBF16: prepare<kBF16>(); engine_tma_kernel<kBF16><<<grid, kTmaThreads, kSmemBytes, stream>>>(p); break;
+    default: prepare<kI32>(); engine_tma_kernel<kI32><<<grid, kTmaThreads, kSmemBytes, stream>>>(p); break;
+  }
+  return cudaGetLastError();
+}
+
+}  // namespace adapcc

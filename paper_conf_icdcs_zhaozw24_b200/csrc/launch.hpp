@@ -42,8 +42,13 @@ struct LaunchParams {
   char* hdr[kMaxRanksDev];  // arena base of each rank (peer-mapped): [header | half 0 | half 1]
 };
 
+// engine.cu: 128-bit LDG/STG fold (256 threads, 2 CTAs/SM)
 int engine_threads();
 cudaError_t engine_occupancy(int dtype, int* blocks_per_sm);
 cudaError_t engine_launch(const LaunchParams& p, int grid, cudaStream_t stream);
+// engine_tma.cu: TMA bulk-copy pipeline (1 producer + 8 consumer warps, 2 CTAs/SM)
+int engine_tma_threads();
+cudaError_t engine_tma_occupancy(int dtype, int* blocks_per_sm);
+cudaError_t engine_tma_launch(const LaunchParams& p, int grid, cudaStream_t stream);
 
 }  // namespace adapcc

@@ -23,6 +23,7 @@ from tests.gpu_util import bits, empty_dev, to_dev, to_host  # noqa: E402
 pytestmark = pytest.mark.gpu
 
 MODES = ["direct", "staged"]
+ENGINES = [0, 1]   # 0: LDG/STG fold kernel, 1: TMA bulk-copy pipeline kernel
 
 
 @pytest.fixture(autouse=True)
@@ -31,9 +32,10 @@ def _need_gpu():
         pytest.skip("no GPU")
 
 
-def _comm(n, mode, scratch=64 << 20):
+def _comm(n, mode, scratch=64 << 20, engine=2):
     c = pkg.Communicator.loopback(n, device=0, scratch_bytes=scratch, mode=mode)
     c.config("timeout_ms", 20000)
+    c.config("engine", engine)
     return c
 
 
@@ -76,11 +78,12 @@ ALLREDUCE_STRATS = {
 @pytest.mark.parametrize("mode", MODES)
 @pytest.mark.parametrize("dtype", ["f32", "bf16", "i32"])
 @pytest.mark.parametrize("strat", list(ALLREDUCE_STRATS))
-def test_allreduce_parity(mode, dtype, strat):
+@pytest.mark.parametrize("engine", ENGINES)
+def test_allreduce_parity(mode, dtype, strat, engine):
     n = 8 if strat != "mixed_noagg" else 5
     count = 100_003  # ragged: not a multiple of any vector width
     text = ALLREDUCE_STRATS[strat](n)
-    comm = _comm(n, mode)
+    comm = _comm(n, mode, engine=engine)
     comm.set_strategy("allreduce", text)
     xs = rank_tensors(dtype, count, n)
     for mask in ((1 << n) - 1, 0b10110111 & ((1 << n) - 1), 0b1, 1 << (n - 1)):
@@ -100,11 +103,12 @@ def test_allreduce_parity(mode, dtype, strat):
 
 
 @pytest.mark.parametrize("mode", MODES)
-def test_c1_config_bit_exact(mode):
+@pytest.mark.parametrize("engine", ENGINES)
+def test_c1_config_bit_exact(mode, engine):
     """BASELINE config C1: fp32 1M elements, 2 ranks, single tree, chunk 256 KB."""
     n, count = 2, 1 << 20
     text = S.allreduce_trees([[-1, 0]], chunk=262144)
-    comm = _comm(n, mode)
+    comm = _comm(n, mode, engine=engine)
     comm.set_strategy("allreduce", text)
     for dtype, dist in (("f32", "normal"), ("i32", "int")):
         xs = rank_tensors(dtype, count, n, dist=dist)
@@ -115,14 +119,15 @@ def test_c1_config_bit_exact(mode):
 
 @pytest.mark.parametrize("mode", MODES)
 @pytest.mark.parametrize("dtype", ["f32", "bf16", "i32"])
-def test_phase1_phase2_accumulate(mode, dtype):
+@pytest.mark.parametrize("engine", ENGINES)
+def test_phase1_phase2_accumulate(mode, dtype, engine):
     """C3 shape (reduced): stragglers {3,6} relay in phase 1, join with ACCUMULATE."""
     n, count = 8, 65_537
     R1, R2 = {0, 1, 2, 4, 5, 7}, {3, 6}
     xs = rank_tensors(dtype, count, n)
     t1 = G.allreduce_mask_aware_stars(n, R1, chunk=8192)
     t2 = G.allreduce_mask_aware_stars(n, R2, chunk=8192)
-    comm = _comm(n, mode)
+    comm = _comm(n, mode, engine=engine)
     comm.set_strategy("allreduce", t1)
     y1 = _run_allreduce(comm, [x if r in R1 else None for r, x in enumerate(xs)], dtype, R1)
     e1 = oc.allreduce(xs, t1, R1, dtype)
@@ -135,9 +140,10 @@ def test_phase1_phase2_accumulate(mode, dtype):
 
 
 @pytest.mark.parametrize("mode", MODES)
-def test_empty_mask_and_in_place(mode):
+@pytest.mark.parametrize("engine", ENGINES)
+def test_empty_mask_and_in_place(mode, engine):
     n, count = 4, 3001
-    comm = _comm(n, mode)
+    comm = _comm(n, mode, engine=engine)
     xs = rank_tensors("f32", count, n)
     text = G.allreduce_stars(n, chunk=512)
     comm.set_strategy("allreduce", text)
@@ -154,11 +160,12 @@ def test_empty_mask_and_in_place(mode):
 @pytest.mark.parametrize("mode", MODES)
 @pytest.mark.parametrize("dtype", ["bf16", "f32"])
 @pytest.mark.parametrize("strat", ["stars", "chains"])
-def test_allgather_parity(mode, dtype, strat):
+@pytest.mark.parametrize("engine", ENGINES)
+def test_allgather_parity(mode, dtype, strat, engine):
     n, cnt = 6, 10_001
     text = (G.allgather_stars(n, chunk=4096) if strat == "stars"
             else G.allgather_chains(n, chunk=2048))
-    comm = _comm(n, mode)
+    comm = _comm(n, mode, engine=engine)
     comm.set_strategy("allgather", text)
     xs = rank_tensors(dtype, cnt, n)
     for R in (set(range(n)), {1, 4}):
@@ -174,10 +181,11 @@ def test_allgather_parity(mode, dtype, strat):
 
 @pytest.mark.parametrize("mode", MODES)
 @pytest.mark.parametrize("dtype", ["bf16", "i32"])
-def test_alltoall_parity(mode, dtype):
+@pytest.mark.parametrize("engine", ENGINES)
+def test_alltoall_parity(mode, dtype, engine):
     n, cnt = 8, 4099
     text = G.alltoall_direct(n, chunk=2048, lines=3)
-    comm = _comm(n, mode)
+    comm = _comm(n, mode, engine=engine)
     comm.set_strategy("alltoall", text)
     xs = rank_tensors(dtype, n * cnt, n)
     for R in (set(range(n)), {0, 5, 6}):
@@ -191,12 +199,13 @@ def test_alltoall_parity(mode, dtype):
     comm.finalize()
 
 
+@pytest.mark.parametrize("engine", ENGINES)
 @pytest.mark.parametrize("mode", MODES)
-def test_strategy_swap_mid_stream(mode):
+def test_strategy_swap_mid_stream(mode, engine):
     """C5 shape (reduced): AllGather stream with a strategy swap at call 6 of 12,
     all calls enqueued back to back on one stream."""
     n, cnt = 4, 6400
-    comm = _comm(n, mode)
+    comm = _comm(n, mode, engine=engine)
     t_a, t_b = G.allgather_stars(n, chunk=4096), G.allgather_chains(n, chunk=8192)
     comm.set_strategy("allgather", t_a)
     xs_all, outs = [], []
@@ -217,9 +226,10 @@ def test_strategy_swap_mid_stream(mode):
     comm.finalize()
 
 
-def test_segmented_call_when_arena_small():
+@pytest.mark.parametrize("engine", ENGINES)
+def test_segmented_call_when_arena_small(engine):
     n, count = 4, 1 << 20
-    comm = _comm(n, "staged", scratch=1 << 20)
+    comm = _comm(n, "staged", scratch=1 << 20, engine=engine)
     text = G.allreduce_stars(n, chunk=16384)
     comm.set_strategy("allreduce", text)
     xs = rank_tensors("f32", count, n)
@@ -230,9 +240,10 @@ def test_segmented_call_when_arena_small():
     comm.finalize()
 
 
-def test_watchdog_reports_timeout():
+@pytest.mark.parametrize("engine", ENGINES)
+def test_watchdog_reports_timeout(engine):
     n = 4
-    comm = _comm(n, "staged")
+    comm = _comm(n, "staged", engine=engine)
     comm.config("timeout_ms", 300)
     comm.config("debug_drop_rank", 2)
     xs = [to_dev(x, "f32") for x in rank_tensors("f32", 4096, n)]
@@ -267,10 +278,11 @@ def test_argument_errors():
 
 
 @pytest.mark.parametrize("mode", MODES)
-def test_cuda_graph_capture_and_replay(mode):
+@pytest.mark.parametrize("engine", ENGINES)
+def test_cuda_graph_capture_and_replay(mode, engine):
     """Calls are capturable once their plan is cached (warm-up call first)."""
     n, count = 4, 50_001
-    comm = _comm(n, mode)
+    comm = _comm(n, mode, engine=engine)
     text = G.allreduce_stars(n, chunk=16384)
     comm.set_strategy("allreduce", text)
     xs = rank_tensors("f32", count, n)
