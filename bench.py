@@ -30,6 +30,8 @@ sys.path.insert(0, ROOT)
 METRIC = "AllReduce busbw GB/s vs size at 2/4/8 B200 (% of 900 GB/s) vs NCCL"
 UNIT = "GB/s"
 NVLINK_NOMINAL = 900.0
+ENGINE_NAMES = {0: "adapcc::engine_kernel (128-bit LDG/STG fold)",
+                1: "adapcc::engine_tma_kernel (TMA bulk-copy pipeline)"}
 
 
 def parse_args():
@@ -79,6 +81,10 @@ def profile_traffic(key):
         return d.get(key, {}).get("dram_bytes_per_launch")
     except Exception:  # noqa: BLE001
         return None
+
+
+def traffic_key(engine, mode):
+    return f"allreduce_loopback_{mode}_{'tma' if engine == 1 else 'ldg'}"
 
 
 class ClockSampler:
@@ -304,9 +310,10 @@ def run_single(args):
         "algbw": round(nbytes / (ms / 1e3) / 1e9, 3),
         "pct_of_nvlink_900": None,
         "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
-                     "frac": round(achieved / peak, 4), "traffic": profile_traffic("allreduce_loopback"),
+                     "frac": round(achieved / peak, 4), "traffic": profile_traffic(traffic_key(comm.last_engine(), args.mode)),
                      "algorithmic_bytes_per_launch": alg_bytes, "peak_source": peak_src,
-                     "kernel": "adapcc::engine_kernel<f32>", "kernel_ms": round(kern_ms, 4)},
+                     "kernel": ENGINE_NAMES.get(comm.last_engine(), "?") + f"<{args.dtype}>",
+                     "kernel_ms": round(kern_ms, 4)},
         "e2e": {"value": round(busbw(nbytes, e2e_t / 1e3, n), 3), "unit": UNIT,
                 "h2d_bytes_per_step": n * nbytes, "d2h_bytes_per_step": n * nbytes,
                 "ms_per_step": round(e2e_t, 3)},

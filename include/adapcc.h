@@ -170,6 +170,8 @@ ADAPCC_API adapcc_result_t adapcc_config(adapcc_comm_t comm, const char* key, in
 
 /* Number of engine kernel launches this communicator has issued. */
 ADAPCC_API adapcc_result_t adapcc_launch_count(adapcc_comm_t comm, uint64_t* count);
+/* Kernel of the most recent launch: 0 = LDG/STG fold, 1 = TMA pipeline, -1 = none. */
+ADAPCC_API adapcc_result_t adapcc_last_engine(adapcc_comm_t comm, int* engine);
 
 /* ------------------------------------------------- host-only inspection ---
  * No GPU needed.  Used by the CPU tests to cross-check the C++ loader and

@@ -79,6 +79,7 @@ def _load():
         "adapcc_finalize": [vp],
         "adapcc_config": [vp, ctypes.c_char_p, i64],
         "adapcc_launch_count": [vp, ctypes.POINTER(u64)],
+        "adapcc_last_engine": [vp, ctypes.POINTER(i32)],
         "adapcc_strategy_check": [ctypes.c_char_p, ctypes.POINTER(i32), ctypes.POINTER(i32),
                                   ctypes.POINTER(i32), ctypes.c_char_p, sz],
         "adapcc_strategy_tuples": [ctypes.c_char_p, i32, u64, ctypes.POINTER(ctypes.c_uint8),
@@ -271,6 +272,12 @@ class Communicator:
     def launch_count(self):
         v = ctypes.c_uint64()
         _check(_load().adapcc_launch_count(self._h, ctypes.byref(v)), "launch_count")
+        return v.value
+
+    def last_engine(self):
+        """Kernel of the most recent launch: 0 LDG/STG fold, 1 TMA pipeline."""
+        v = ctypes.c_int()
+        _check(_load().adapcc_last_engine(self._h, ctypes.byref(v)), "last_engine")
         return v.value
 
     def finalize(self):

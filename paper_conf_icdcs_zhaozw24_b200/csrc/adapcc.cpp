@@ -119,6 +119,7 @@ struct adapcc_comm_s {
   int num_sms = 148;
   int occ[2][3] = {{1, 1, 1}, {1, 1, 1}};  // [engine][dtype] resident CTAs per SM
   int engine = 2;  // 0: LDG/STG fold, 1: TMA bulk pipeline, 2: auto by call size
+  int last_engine = -1;  // kernel used by the most recent launch
   std::mutex mu;
 };
 
@@ -316,6 +317,7 @@ adapcc_result_t run(adapcc_comm_s* c, Coll coll, const void* const* send, void* 
     }
     const int grid = std::max(1, std::min<int>(grid_size(c, dtype, plan->engine), (int)std::max<uint32_t>(1, seg.nitems)));
     CK(plan->engine ? engine_tma_launch(P, grid, s) : engine_launch(P, grid, s));
+    c->last_engine = plan->engine;
     ++c->launches;
   }
   if (!capturing) CK(cudaEventRecord(plan->last_use, s));
@@ -568,6 +570,12 @@ adapcc_result_t adapcc_config(adapcc_comm_t c, const char* key, int64_t value) {
 adapcc_result_t adapcc_launch_count(adapcc_comm_t c, uint64_t* count) {
   if (!c || !count) return ADAPCC_ERR_INVALID_ARGUMENT;
   *count = c->launches;
+  return ADAPCC_SUCCESS;
+}
+
+adapcc_result_t adapcc_last_engine(adapcc_comm_t c, int* engine) {
+  if (!c || !engine) return ADAPCC_ERR_INVALID_ARGUMENT;
+  *engine = c->last_engine;
   return ADAPCC_SUCCESS;
 }
 

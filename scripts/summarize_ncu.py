@@ -44,7 +44,8 @@ def raw(rep):
 def main():
     tag = sys.argv[1] if len(sys.argv) > 1 else "r01"
     res = {}
-    for name, key in (("direct", "allreduce_loopback"), ("staged", "allreduce_loopback_staged")):
+    for name in ("direct_tma", "direct_ldg", "staged_tma", "staged_ldg"):
+        key = "allreduce_loopback_" + name
         rep = os.path.join(ROOT, "gpurun_out", f"prof_{name}_{tag}.ncu-rep")
         if not os.path.exists(rep):
             continue
