@@ -108,6 +108,8 @@ struct adapcc_comm_s {
   int* h_err = nullptr;
   int* d_err = nullptr;
   Strategy strat[3];
+  // plan-cache identity of the active strategy: the hash of its normalised
+  // text, so swapping back to a strategy seen before reuses its cached plans
   uint64_t strat_version[3] = {0, 0, 0};
   std::map<PlanKey, std::shared_ptr<DevPlan>> plans;
   uint64_t tick = 0;  // plan-cache clock (least recently used plan is evicted)
@@ -167,6 +169,7 @@ adapcc_result_t common_init(adapcc_comm_s* c, size_t scratch) {
     std::string err;
     if (!parse_strategy(default_strategy((Coll)k, c->nranks).c_str(), &c->strat[k], &err))
       return ADAPCC_ERR_INVALID_STRATEGY;
+    c->strat_version[k] = c->strat[k].hash;
   }
   return ADAPCC_SUCCESS;
 }
@@ -427,7 +430,7 @@ adapcc_result_t adapcc_set_strategy(adapcc_comm_t c, adapcc_coll_t coll, const c
   if (st.nranks != c->nranks || (int)st.coll != (int)coll) return ADAPCC_ERR_INVALID_STRATEGY;
   std::lock_guard<std::mutex> lock(c->mu);
   c->strat[coll] = std::move(st);
-  c->strat_version[coll] += 1;
+  c->strat_version[coll] = c->strat[coll].hash;
   return ADAPCC_SUCCESS;
 }
 

@@ -1,0 +1,273 @@
+"""Measure every BASELINE.json config on one B200 (loopback virtual ranks).
+
+    python scripts/bench_configs.py [--out gpurun_out/configs.json]
+
+C1  AllReduce fp32 1 Mi elements, 2 ranks, single tree, chunk 256 KiB (DIRECT and STAGED)
+C2  AllReduce 8 ranks at 256 MiB: fp32 and bf16, M = 1/2/4/8 star trees, double binary, ring
+C3  partial AllReduce, 8 ranks, stragglers {3,6}: T_adapcc = end of phase 2 (phase 1 among the
+    ready ranks at t=0 with relays, phase 2 ACCUMULATE once the stragglers are ready) vs
+    T_wait = t_s + T_full, straggler lag t_s simulated by a 1-CTA spin kernel on a compute stream
+C4  AlltoAll 8 ranks, [8][512][4096] bf16 per rank
+C5  AllGather of GPT-2-XL row shards, 48 layers x 4 weights, strategy swap at call 96
+Timing: CUDA events on the launching stream, warm-up first; busbw factors as nccl-tests.
+Every config also checks parity on sampled outputs against the oracle.
+"""
+import argparse
+import json
+import os
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--out", default=os.path.join(ROOT, "gpurun_out", "configs.json"))
+    ap.add_argument("--only", default="C1,C2,C3,C4,C5")
+    a = ap.parse_args()
+
+    import numpy as np
+    import torch
+
+    import paper_conf_icdcs_zhaozw24_b200 as pkg
+    from oracle import collectives as oc
+    from paper_conf_icdcs_zhaozw24_b200 import generator as G
+    from synth import GPT2XL_LAYERS, rank_tensors
+
+    def dev(x, dtype):
+        t = torch.from_numpy(x)
+        return t.view(torch.int16).cuda().view(torch.bfloat16) if dtype == "bf16" else t.cuda()
+
+    def host_bits(t, dtype):
+        return t.view(torch.int16).cpu().numpy().view(np.uint16) if dtype == "bf16" else \
+            t.cpu().numpy().view(np.uint32)
+
+    def timeit(fn, iters=20, warm=3):
+        for _ in range(warm):
+            fn()
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        for _ in range(iters):
+            fn()
+        e1.record()
+        torch.cuda.synchronize()
+        return e0.elapsed_time(e1) / iters
+
+    def sampled_ok(ys, xs, text, R, count, dtype, k=2048):
+        idx = np.unique(np.random.default_rng(5).integers(0, count, size=k))
+        exp = oc.allreduce_elements([x[idx] if x is not None else None for x in xs], idx, count, text, R, dtype)
+        eb = exp.view(np.uint16) if dtype == "bf16" else exp.view(np.uint32)
+        ti = torch.from_numpy(idx).cuda()
+        return all(np.array_equal(host_bits(y.index_select(0, ti), dtype), eb) for y in ys)
+
+    out = {"gpu": torch.cuda.get_device_name(0), "when": time.strftime("%Y-%m-%dT%H:%M:%SZ", time.gmtime())}
+    only = set(a.only.split(","))
+
+    # ------------------------------------------------------------------ C1
+    if "C1" in only:
+        res = []
+        n, count = 2, 1 << 20
+        text = G.allreduce_trees([[-1, 0]], chunk=262144)
+        xs = rank_tensors("f32", count, n)
+        for mode in ("direct", "staged"):
+            comm = pkg.Communicator.loopback(n, mode=mode, scratch_bytes=64 << 20)
+            comm.set_strategy("allreduce", text)
+            dx = [dev(x, "f32") for x in xs]
+            dy = [torch.empty_like(t) for t in dx]
+            ms = timeit(lambda: comm.allreduce_lb(dx, dy), iters=200)
+            exp = oc.allreduce(xs, text, {0, 1}, "f32")
+            ok = all(np.array_equal(host_bits(dy[g], "f32"), exp[g].view(np.uint32)) for g in range(n))
+            res.append({"mode": mode, "us": round(ms * 1e3, 2), "busbw": round(count * 4 / ms / 1e6 * 1.0, 2),
+                        "parity_bit_exact": ok, "kernel": comm.last_engine()})
+            comm.finalize()
+        out["C1"] = res
+        print("C1", res, flush=True)
+
+    # ------------------------------------------------------------------ C2
+    if "C2" in only:
+        res = []
+        n, nbytes = 8, 256 << 20
+        comm = pkg.Communicator.loopback(n, mode="direct", scratch_bytes=512 << 20)
+        for dtype in ("f32", "bf16"):
+            es = 4 if dtype == "f32" else 2
+            count = nbytes // es
+            xs = rank_tensors(dtype, count, n)
+            dx = [dev(x, dtype) for x in xs]
+            dy = [torch.empty_like(t) for t in dx]
+            strategies = {f"star M={m}": G.allreduce_stars(n, roots=list(range(m))) for m in (1, 2, 4, 8)}
+            strategies["double binary"] = G.allreduce_double_binary(n)
+            strategies["ring"] = G.allreduce_ring(n)
+            for name, text in strategies.items():
+                if dtype == "bf16" and name not in ("star M=8",):
+                    continue
+                comm.set_strategy("allreduce", text)
+                ms = timeit(lambda: comm.allreduce_lb(dx, dy), iters=10)
+                bus = nbytes / ms / 1e6 * 2 * (n - 1) / n
+                ok = sampled_ok(dy, xs, text, set(range(n)), count, dtype)
+                res.append({"dtype": dtype, "strategy": name, "ms": round(ms, 4), "busbw": round(bus, 1),
+                            "hbm_frac": round(2 * n * nbytes / ms / 1e6 / 6545.6, 4), "parity": ok,
+                            "kernel": comm.last_engine()})
+                print("C2", res[-1], flush=True)
+            del dx, dy
+        comm.finalize()
+        out["C2"] = res
+
+    # ------------------------------------------------------------------ C3
+    if "C3" in only:
+        res = []
+        n = 8
+        R1, R2 = {0, 1, 2, 4, 5, 7}, {3, 6}
+        comm = pkg.Communicator.loopback(n, mode="staged", scratch_bytes=(2 * 100 << 20) + (64 << 20))
+        s_comm = torch.cuda.Stream()
+        s_comp = torch.cuda.Stream()
+        # cycles per ms of the spin kernel
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        torch.cuda._sleep(10_000_000)
+        e1.record()
+        torch.cuda.synchronize()
+        cyc_per_ms = 10_000_000 / e0.elapsed_time(e1)
+        for mib in (25, 50, 100):
+            count = (mib << 20) // 4
+            xs = rank_tensors("f32", count, n)
+            dx = [dev(x, "f32") for x in xs]
+            dy = [torch.empty_like(t) for t in dx]
+            t_full_txt = G.allreduce_stars(n)
+            variants = {
+                "relays as roots (mask-aware weights)": (G.allreduce_mask_aware_stars(n, R1),
+                                                         G.allreduce_mask_aware_stars(n, R2)),
+                "paper-faithful (unweighted stars, relays per tuples)": (G.allreduce_stars(n), G.allreduce_stars(n)),
+                "relays as leaves only": (G.allreduce_mask_aware_stars(n, R1, relays_as_roots=False),
+                                          G.allreduce_mask_aware_stars(n, R2, relays_as_roots=False)),
+            }
+            comm.set_strategy("allreduce", t_full_txt)
+            t_full = timeit(lambda: comm.allreduce_lb(dx, dy), iters=10)
+            point = {"mib": mib, "T_full_ms": round(t_full, 4), "variants": {}}
+            for vname, (t1, t2) in variants.items():
+                comm.set_strategy("allreduce", t1)
+                p1 = timeit(lambda: comm.allreduce_lb([x if r in R1 else None for r, x in enumerate(dx)], dy,
+                                                      ready=R1), iters=10)
+                comm.set_strategy("allreduce", t2)
+                p2 = timeit(lambda: comm.allreduce_lb([x if r in R2 else None for r, x in enumerate(dx)], dy,
+                                                      ready=R2, accumulate=True), iters=10)
+                lags = {}
+                for f in (0.0, 0.25, 0.5, 1.0, 2.0):
+                    ts = f * t_full
+                    # measured end-to-end: spin kernel (straggler compute) on s_comp, phase 1 on
+                    # s_comm at t=0, phase 2 on s_comm after the straggler's event
+                    torch.cuda.synchronize()
+                    a0 = torch.cuda.Event(enable_timing=True)
+                    a1 = torch.cuda.Event(enable_timing=True)
+                    ready_ev = torch.cuda.Event()
+                    a0.record(s_comm)
+                    s_comp.wait_event(a0)
+                    with torch.cuda.stream(s_comp):
+                        if ts > 0:
+                            torch.cuda._sleep(int(ts * cyc_per_ms))
+                        ready_ev.record(s_comp)
+                    with torch.cuda.stream(s_comm):
+                        comm.set_strategy("allreduce", t1)
+                        comm.allreduce_lb([x if r in R1 else None for r, x in enumerate(dx)], dy, ready=R1)
+                        s_comm.wait_event(ready_ev)
+                        comm.set_strategy("allreduce", t2)
+                        comm.allreduce_lb([x if r in R2 else None for r, x in enumerate(dx)], dy, ready=R2,
+                                          accumulate=True)
+                        a1.record(s_comm)
+                    torch.cuda.synchronize()
+                    t_adapcc = a0.elapsed_time(a1)
+                    t_wait = ts + t_full
+                    lags[str(f)] = {"t_s_ms": round(ts, 4), "T_adapcc_ms": round(t_adapcc, 4),
+                                    "T_wait_ms": round(t_wait, 4), "speedup": round(t_wait / t_adapcc, 3)}
+                full = oc.allreduce_exact([x[:4096] for x in xs], set(range(n)), "f32")
+                got = dy[0][:4096].cpu().numpy().astype(np.float64)
+                point["variants"][vname] = {"phase1_ms": round(p1, 4), "phase2_ms": round(p2, 4),
+                                            "lags": lags,
+                                            "rel_err_vs_full_sum": float(np.max(np.abs(got - full)) /
+                                                                         np.max(np.abs(full)))}
+            res.append(point)
+            print("C3", json.dumps(point)[:400], flush=True)
+            del dx, dy
+        comm.finalize()
+        out["C3"] = res
+
+    # ------------------------------------------------------------------ C4
+    if "C4" in only:
+        res = []
+        n, cnt = 8, 512 * 4096
+        text = G.alltoall_direct(n, chunk=1 << 20)
+        xs = rank_tensors("bf16", n * cnt, n, base=2000)
+        for mode in ("direct", "staged"):
+            comm = pkg.Communicator.loopback(n, mode=mode, scratch_bytes=(2 * n * cnt * 2 + (64 << 20)))
+            comm.set_strategy("alltoall", text)
+            dx = [dev(x, "bf16") for x in xs]
+            dy = [torch.empty_like(t) for t in dx]
+            ms = timeit(lambda: comm.alltoall_lb(dx, dy), iters=20)
+            nbytes = n * cnt * 2
+            exp = oc.alltoall(xs, text, set(range(n)), "bf16", [np.zeros(n * cnt, np.uint16)] * n)
+            ok = all(np.array_equal(host_bits(dy[d], "bf16"), exp[d]) for d in range(n))
+            res.append({"mode": mode, "ms": round(ms, 4),
+                        "busbw": round(nbytes / ms / 1e6 * (n - 1) / n, 1),
+                        "hbm_frac": round(2 * n * nbytes / ms / 1e6 / 6545.6, 4), "parity": ok,
+                        "kernel": comm.last_engine()})
+            print("C4", res[-1], flush=True)
+            comm.finalize()
+        out["C4"] = res
+
+    # ------------------------------------------------------------------ C5
+    if "C5" in only:
+        res = []
+        for n in (2, 4, 8):
+            comm = pkg.Communicator.loopback(n, mode="staged", scratch_bytes=256 << 20)
+            t_a, t_b = G.allgather_stars(n, chunk=262144), G.allgather_chains(n, chunk=1 << 20)
+            shards = {}
+            for wi, (name, rows, cols) in enumerate(GPT2XL_LAYERS):
+                cnt = rows // n * cols
+                xs = rank_tensors("bf16", cnt, n, base=3000 + wi)
+                shards[name] = ([dev(x, "bf16") for x in xs],
+                                [torch.empty(n * cnt, dtype=torch.bfloat16, device="cuda") for _ in range(n)],
+                                xs)
+            comm.set_strategy("allgather", t_a)
+            for name in shards:   # warm plans of strategy A
+                comm.allgather_lb(shards[name][0], shards[name][1])
+            torch.cuda.synchronize()
+            evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(192)]
+            swap_host_ms = None
+            for call in range(192):
+                name = GPT2XL_LAYERS[call % 4][0]
+                if call == 96:
+                    h0 = time.perf_counter()
+                    comm.set_strategy("allgather", t_b)
+                    swap_host_ms = (time.perf_counter() - h0) * 1e3
+                evs[call][0].record()
+                comm.allgather_lb(shards[name][0], shards[name][1])
+                evs[call][1].record()
+            torch.cuda.synchronize()
+            t = [s.elapsed_time(e) for s, e in evs]
+            bus = []
+            for call in range(192):
+                name = GPT2XL_LAYERS[call % 4][0]
+                out_bytes = shards[name][1][0].numel() * 2
+                bus.append(out_bytes / t[call] / 1e6 * (n - 1) / n)
+            ok = True
+            for name, (_, dy, xs) in shards.items():
+                cat = np.concatenate(xs)
+                ok &= all(np.array_equal(host_bits(y, "bf16"), cat) for y in dy)
+            res.append({"n": n, "busbw_median_A": round(float(np.median(bus[:96])), 1),
+                        "busbw_median_B": round(float(np.median(bus[97:])), 1),
+                        "call_ms_median_A": round(float(np.median(t[:96])), 4),
+                        "call_ms_median_B": round(float(np.median(t[97:])), 4),
+                        "first_call_after_swap_ms": round(t[96], 4),
+                        "set_strategy_host_ms": round(swap_host_ms, 4), "parity": bool(ok)})
+            print("C5", res[-1], flush=True)
+            comm.finalize()
+        out["C5"] = res
+
+    os.makedirs(os.path.dirname(a.out), exist_ok=True)
+    json.dump(out, open(a.out, "w"), indent=1)
+
+
+if __name__ == "__main__":
+    main()
