@@ -93,6 +93,23 @@ __device__ __forceinline__ void tma_load(void* sdst, const void* gsrc, uint32_t 
       "l"(gsrc), "r"(bytes), "r"(su32(bar))
       : "memory");
 }
+// TMA bulk copy shared -> global (bulk-group completion)
+__device__ __forceinline__ void tma_store(void* gdst, const void* ssrc, uint32_t bytes) {
+  asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(gdst), "r"(su32(ssrc)),
+               "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void tma_store_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void tma_store_wait_read() {  // all but N groups have read their smem
+  asm volatile("cp.async.bulk.wait_group.read %0;" ::"n"(N) : "memory");
+}
+__device__ __forceinline__ void tma_store_wait_all() {  // all bulk stores complete (writes performed)
+  asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_arrive_cnt(uint64_t* b, uint32_t count) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0], %1;" ::"r"(su32(b)), "r"(count) : "memory");
+}
 __device__ __forceinline__ void fence_proxy_async() {
   asm volatile("fence.proxy.async.global;" ::: "memory");
 }
@@ -165,6 +182,38 @@ __device__ __forceinline__ void consume_copy(Smem& sm, char* stages, const ItemD
       const uint32_t v = tid + j * kConsumers;
       if (v < nv) store_result<DT>(d, (size_t)t * d.tile + (size_t)v * 16, raw[j]);
     }
+  }
+}
+
+// Pure copy (one source, no accumulation) entirely on the TMA engines: one
+// thread waits for each loaded stage and issues the D bulk stores straight
+// from shared memory; a stage is released once its stores have read it.
+// Other consumer threads only advance their ring position.
+__device__ __forceinline__ void copy_tma(Smem& sm, char* stages, const ItemDesc& d, int tid,
+                                         uint32_t& stage, uint32_t& sphase) {
+  if (tid == 0) {
+    int prev = -1;
+    for (uint32_t t = 0; t < d.ntiles; ++t) {
+      const uint32_t tb = min(d.tile, d.vec_bytes - t * d.tile);
+      mbar_wait(&sm.full[stage], sphase);
+      const char* sb = stages + (size_t)stage * kStageBytes;
+      for (int k = 0; k < d.ndst; ++k) tma_store(d.dst[k] + (size_t)t * d.tile, sb, tb);
+      tma_store_commit();
+      if (prev >= 0) {
+        tma_store_wait_read<1>();
+        mbar_arrive_cnt(&sm.empty[prev], kConsumerWarps);
+      }
+      prev = (int)stage;
+      if (++stage == kStages) { stage = 0; sphase ^= 1; }
+    }
+    if (prev >= 0) {
+      tma_store_wait_read<0>();
+      mbar_arrive_cnt(&sm.empty[prev], kConsumerWarps);
+    }
+  } else {
+    const uint32_t total = stage + d.ntiles;
+    sphase ^= (total / kStages) & 1;
+    stage = total % kStages;
   }
 }
 
@@ -364,7 +413,8 @@ __global__ void __launch_bounds__(kTmaThreads, 2) engine_tma_kernel(const __grid
         } else {
           if (!d.scalar_only) {
             const uint32_t vpt = d.tile / (16u * kConsumers);  // 8 (K=1), 4, 2 or 1
-            if (d.nsrc == 1) consume_copy<DT, 8>(sm, stages, d, tid, stage, sphase);
+            if (d.nsrc == 1 && !d.any_acc) copy_tma(sm, stages, d, tid, stage, sphase);
+            else if (d.nsrc == 1) consume_copy<DT, 8>(sm, stages, d, tid, stage, sphase);
             else if (vpt >= 4) consume_fold<DT, 4>(sm, stages, d, tid, stage, sphase);
             else if (vpt >= 2) consume_fold<DT, 2>(sm, stages, d, tid, stage, sphase);
             else consume_fold<DT, 1>(sm, stages, d, tid, stage, sphase);
@@ -374,6 +424,8 @@ __global__ void __launch_bounds__(kTmaThreads, 2) engine_tma_kernel(const __grid
         }
         consumer_sync();  // every consumer's stores for this item are issued
         if (tid == 0 && d.npost) {
+          tma_store_wait_all();  // bulk (async-proxy) stores performed ...
+          fence_proxy_async();   // ... and ordered before generic-proxy accesses
           fence(sys);      // the chunk's bytes (incl. remote NVLink stores) before its flag
           for (int i = 0; i < d.npost; ++i) st_release(d.post[i], epoch, sys);
         }
@@ -385,6 +437,8 @@ __global__ void __launch_bounds__(kTmaThreads, 2) engine_tma_kernel(const __grid
   }
   __syncthreads();
   if (tid == 0) {
+    tma_store_wait_all();  // this CTA's bulk stores are complete before it counts as done
+    fence_proxy_async();
     fence(sys);
     const unsigned done = atomicAdd(&P.state->done[par], 1u);
     if (done == gridDim.x - 1) {
