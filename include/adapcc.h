@@ -61,7 +61,10 @@ typedef enum {
 } adapcc_result_t;
 
 typedef enum { ADAPCC_FLOAT32 = 0, ADAPCC_BFLOAT16 = 1, ADAPCC_INT32 = 2 } adapcc_dtype_t;
-typedef enum { ADAPCC_ALLREDUCE = 0, ADAPCC_ALLGATHER = 1, ADAPCC_ALLTOALL = 2 } adapcc_coll_t;
+typedef enum {
+  ADAPCC_ALLREDUCE = 0, ADAPCC_ALLGATHER = 1, ADAPCC_ALLTOALL = 2,
+  ADAPCC_REDUCE = 3, ADAPCC_BROADCAST = 4, ADAPCC_REDUCESCATTER = 5
+} adapcc_coll_t;
 
 /* Transport modes.  DIRECT: every rank's send/recv buffer is addressable by
  * the engine (loopback: one process owns all virtual ranks), so data moves
@@ -150,6 +153,41 @@ ADAPCC_API adapcc_result_t adapcc_alltoall_lb(adapcc_comm_t comm, const void* co
                                    void* const* recvbufs, size_t count_per_peer,
                                    adapcc_dtype_t dtype, uint64_t ready_mask,
                                    adapcc_stream_t stream);
+
+/* ------------------------------- more primitives on the same engine (NEXT-4) ---
+ * Reduce: the root receives sum_{r ready} sendbuf_r (the paper's Reduce, whose
+ * strategy AllReduce reverses; evaluated in Fig. 11).
+ * Every tree of a Reduce strategy is rooted at `root` (else INVALID_ARGUMENT);
+ * without a user strategy a star rooted at `root` is used.  Only the root's
+ * recvbuf is written (non-roots may pass NULL).  flags: ACCUMULATE.
+ * Broadcast: every rank's recvbuf receives the root's sendbuf;
+ * nothing is written when the root is not ready.  In place at the root allowed.
+ * ReduceScatter: rank b receives block b (recvcount elements) of
+ * sum_{r ready} sendbuf_r, reduced along the "rtree dst=b" lines of the
+ * strategy (default: a star rooted at b).  sendbuf holds nranks blocks; in
+ * place allowed when recvbuf == sendbuf + rank*recvcount*esize. */
+ADAPCC_API adapcc_result_t adapcc_reduce(adapcc_comm_t comm, const void* sendbuf, void* recvbuf,
+                                         size_t count, adapcc_dtype_t dtype, int root,
+                                         uint64_t ready_mask, unsigned flags, adapcc_stream_t stream);
+ADAPCC_API adapcc_result_t adapcc_broadcast(adapcc_comm_t comm, const void* sendbuf, void* recvbuf,
+                                            size_t count, adapcc_dtype_t dtype, int root,
+                                            uint64_t ready_mask, adapcc_stream_t stream);
+ADAPCC_API adapcc_result_t adapcc_reducescatter(adapcc_comm_t comm, const void* sendbuf, void* recvbuf,
+                                                size_t recvcount, adapcc_dtype_t dtype,
+                                                uint64_t ready_mask, unsigned flags,
+                                                adapcc_stream_t stream);
+ADAPCC_API adapcc_result_t adapcc_reduce_lb(adapcc_comm_t comm, const void* const* sendbufs,
+                                            void* const* recvbufs, size_t count, adapcc_dtype_t dtype,
+                                            int root, uint64_t ready_mask, unsigned flags,
+                                            adapcc_stream_t stream);
+ADAPCC_API adapcc_result_t adapcc_broadcast_lb(adapcc_comm_t comm, const void* const* sendbufs,
+                                               void* const* recvbufs, size_t count,
+                                               adapcc_dtype_t dtype, int root, uint64_t ready_mask,
+                                               adapcc_stream_t stream);
+ADAPCC_API adapcc_result_t adapcc_reducescatter_lb(adapcc_comm_t comm, const void* const* sendbufs,
+                                                   void* const* recvbufs, size_t recvcount,
+                                                   adapcc_dtype_t dtype, uint64_t ready_mask,
+                                                   unsigned flags, adapcc_stream_t stream);
 
 /* ------------------------------------------------------------- lifecycle --- */
 

@@ -198,3 +198,81 @@ def alltoall(xs, strategy_text, ready, dtype, y_prev):
         for d in range(n):
             ys[d][s * cnt:(s + 1) * cnt] = xs[s][d * cnt:(d + 1) * cnt]
     return ys
+
+
+# ---------------------------------------------------------------- NEXT-4 primitives
+def reduce(xs, strategy_text, ready, dtype, accumulate=False, y_prev=None):
+    """Reduce: the trees' common root r receives sum_{R} x replayed along the
+    trees (AdapCC "generate[s] strategies for Reduce"; the root GPU of
+    each sub-collective "aggregates gradients").  Every other
+    rank's recvbuf is untouched (returned as y_prev[g], or None)."""
+    st = parse(strategy_text)
+    if st.collective != "reduce":
+        raise ValueError("strategy is not a reduce strategy")
+    n = st.nranks
+    ready = set(ready)
+    root = st.subs[0].root
+    lens = {len(x) for x in xs if x is not None}
+    if y_prev is not None:
+        lens |= {len(y_prev[root])}
+    count = lens.pop()
+    ys = [None if y_prev is None else np.array(y_prev[g], copy=True) for g in range(n)]
+    y = np.array(y_prev[root], copy=True) if accumulate else np.empty(count, dtype=_NP[dtype])
+    bounds = partition(count, ESIZE[dtype], [s.weight for s in st.subs])
+    for m, sub in enumerate(st.subs):
+        lo, hi = bounds[m], bounds[m + 1]
+        if lo == hi:
+            continue
+        res = _tree_result([x[lo:hi] if x is not None else None for x in xs], sub, ready, dtype)
+        if accumulate:
+            if res is not None:
+                y[lo:hi] = _accumulate(y[lo:hi], res, dtype)
+        else:
+            y[lo:hi] = res if res is not None else _zero(hi - lo, dtype)
+    ys[root] = y
+    return ys
+
+
+def broadcast(xs, strategy_text, ready, dtype, y_prev):
+    """Broadcast from the common src s of the bcast lines: y_g = x_s for every
+    g when s is ready; otherwise every recvbuf is untouched (Q12)."""
+    st = parse(strategy_text)
+    if st.collective != "broadcast":
+        raise ValueError("strategy is not a broadcast strategy")
+    src = st.subs[0].src
+    ys = [np.array(y, copy=True) for y in y_prev]
+    if src in set(ready):
+        for g in range(st.nranks):
+            ys[g][:] = xs[src]
+    return ys
+
+
+def reducescatter(xs, strategy_text, ready, dtype, accumulate=False, y_prev=None):
+    """ReduceScatter: rank b receives block b (cnt = len(x)/n elements) of
+    sum_{R} x, replayed along the rtree lines of block b (rooted at b); the
+    block's elements are partitioned over its lines by weight (Q9)."""
+    st = parse(strategy_text)
+    if st.collective != "reducescatter":
+        raise ValueError("strategy is not a reducescatter strategy")
+    n = st.nranks
+    ready = set(ready)
+    total = {len(x) for x in xs if x is not None}
+    cnt = (total.pop() // n) if total else len(y_prev[0])
+    ys = []
+    for b in range(n):
+        y = np.array(y_prev[b], copy=True) if accumulate else np.empty(cnt, dtype=_NP[dtype])
+        lines = [sb for sb in st.subs if sb.src == b]
+        bounds = partition(cnt, ESIZE[dtype], [sb.weight for sb in lines])
+        for i, sub in enumerate(lines):
+            lo, hi = bounds[i], bounds[i + 1]
+            if lo == hi:
+                continue
+            res = _tree_result([x[b * cnt + lo:b * cnt + hi] if x is not None else None for x in xs],
+                               sub, ready, dtype)
+            if accumulate:
+                if res is not None:
+                    y[lo:hi] = _accumulate(y[lo:hi], res, dtype)
+            else:
+                y[lo:hi] = res if res is not None else _zero(hi - lo, dtype)
+        ys.append(y)
+    return ys

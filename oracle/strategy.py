@@ -17,8 +17,12 @@ Format (one directive per line, '#' starts a comment):
     collective allreduce|allgather|alltoall
     tree  weight=<w> chunk=<C> parent=<p_0,..,p_{n-1}> [noagg=<g,..>]   (allreduce)
     ring  weight=<w> chunk=<C> order=<r_0,..,r_{n-1}>                     (allreduce)
-    bcast src=<s> weight=<w> chunk=<C> parent=<p_0,..,p_{n-1}>           (allgather)
+    bcast src=<s> weight=<w> chunk=<C> parent=<p_0,..,p_{n-1}>           (allgather, broadcast)
     a2a   weight=<w> chunk=<C>                                            (alltoall)
+    rtree dst=<b> weight=<w> chunk=<C> parent=<...> [noagg=<g,..>]       (reducescatter)
+  collective reduce uses tree lines sharing one root; broadcast uses bcast
+  lines sharing one src (NEXT-4 primitives: Reduce / Broadcast, P:L165,
+  ReduceScatter, P:L154(1)).
 
 Readings: Q9 partition, Q10 chunk, Q13 ring expansion.
 """
@@ -45,7 +49,7 @@ class Sub:
     chunk: int                # C_m in bytes
     parent: list = None       # parent[g], -1 at the root (tree / bcast)
     noagg: frozenset = frozenset()   # ranks g with a_{m,g} = 0
-    src: int = -1             # bcast source (== root)
+    src: int = -1             # bcast: source (== root); rtree: destination block (== root)
 
     @property
     def root(self):
@@ -135,10 +139,11 @@ def parse(text):
             if coll is not None or len(toks) != 2:
                 raise StrategyError("bad or repeated collective line")
             coll = toks[1]
-            if coll not in ("allreduce", "allgather", "alltoall"):
+            if coll not in ("allreduce", "allgather", "alltoall", "reduce", "broadcast",
+                            "reducescatter"):
                 raise StrategyError(f"unknown collective {coll!r}")
             continue
-        if head not in ("tree", "ring", "bcast", "a2a"):
+        if head not in ("tree", "ring", "bcast", "a2a", "rtree"):
             raise StrategyError(f"unknown directive {head!r}")
         kv = {}
         for t in toks[1:]:
@@ -151,11 +156,12 @@ def parse(text):
         raw_subs.append((head, kv))
     if n is None or coll is None:
         raise StrategyError("missing nranks or collective line")
-    allowed = {"allreduce": ("tree", "ring"), "allgather": ("bcast",),
-               "alltoall": ("a2a",)}[coll]
+    allowed = {"allreduce": ("tree", "ring"), "allgather": ("bcast",), "alltoall": ("a2a",),
+               "reduce": ("tree",), "broadcast": ("bcast",), "reducescatter": ("rtree",)}[coll]
     keys = {"tree": {"weight", "chunk", "parent"}, "ring": {"weight", "chunk", "order"},
-            "bcast": {"src", "weight", "chunk", "parent"}, "a2a": {"weight", "chunk"}}
-    optional = {"tree": {"noagg"}, "ring": set(), "bcast": set(), "a2a": set()}
+            "bcast": {"src", "weight", "chunk", "parent"}, "a2a": {"weight", "chunk"},
+            "rtree": {"dst", "weight", "chunk", "parent"}}
+    optional = {"tree": {"noagg"}, "ring": set(), "bcast": set(), "a2a": set(), "rtree": {"noagg"}}
     if not raw_subs:
         raise StrategyError("no sub-collective lines")
     st = Strategy(nranks=n, collective=coll)
@@ -172,9 +178,9 @@ def parse(text):
             raise StrategyError(f"weight {w} out of range")
         if c < 16 or c % 16 != 0 or c > MAX_CHUNK:
             raise StrategyError(f"chunk {c} must be a positive multiple of 16 <= 2^31")
-        if head == "tree":
+        if head in ("tree", "rtree"):
             parent = _intlist(kv["parent"], "parent")
-            _check_tree(parent, n, "tree")
+            _check_tree(parent, n, head)
             noagg = _intlist(kv.get("noagg", ""), "noagg")
             if len(set(noagg)) != len(noagg):
                 raise StrategyError("duplicate rank in noagg")
@@ -183,7 +189,13 @@ def parse(text):
                     raise StrategyError(f"noagg rank {g} out of range")
                 if parent[g] == -1:
                     raise StrategyError("noagg may not contain the root")
-            st.subs.append(Sub("tree", w * n, c, parent, frozenset(noagg)))
+            if head == "rtree":
+                dst = _int(kv["dst"], "dst")
+                if not (0 <= dst < n) or parent[dst] != -1:
+                    raise StrategyError("rtree root must be its dst")
+                st.subs.append(Sub("rtree", w * n, c, parent, frozenset(noagg), dst))
+            else:
+                st.subs.append(Sub("tree", w * n, c, parent, frozenset(noagg)))
         elif head == "ring":
             order = _intlist(kv["order"], "order")
             if sorted(order) != list(range(n)):
@@ -207,12 +219,16 @@ def parse(text):
             st.subs.append(Sub("a2a", w * n, c))
     if len(st.subs) > MAX_SUBS:
         raise StrategyError(f"{len(st.subs)} sub-collectives > {MAX_SUBS}")
-    if coll == "allgather":
+    if coll in ("allgather", "reducescatter"):
         for s in range(n):
             ws = [sb.weight for sb in st.subs if sb.src == s]
             if not ws or sum(ws) == 0:
-                raise StrategyError(f"allgather source {s} has no positive-weight bcast")
+                raise StrategyError(f"{coll} block {s} has no positive-weight line")
     else:
+        if coll == "reduce" and len({sb.root for sb in st.subs}) != 1:
+            raise StrategyError("reduce trees must share one root")
+        if coll == "broadcast" and len({sb.src for sb in st.subs}) != 1:
+            raise StrategyError("broadcast lines must share one src")
         if sum(sb.weight for sb in st.subs) == 0:
             raise StrategyError("total weight must be > 0")
     return st

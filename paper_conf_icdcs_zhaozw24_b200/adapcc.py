@@ -25,7 +25,8 @@ _PKG = os.path.dirname(os.path.abspath(__file__))
 _LIB_PATH = os.environ.get("ADAPCC_LIB") or os.path.join(_PKG, "libadapcc.so")
 
 SUCCESS, INVALID_ARGUMENT, INVALID_STRATEGY, UNSUPPORTED, CUDA, BOOTSTRAP, OOM, TIMEOUT, MISMATCH = range(9)
-COLL = {"allreduce": 0, "allgather": 1, "alltoall": 2}
+COLL = {"allreduce": 0, "allgather": 1, "alltoall": 2, "reduce": 3, "broadcast": 4,
+        "reducescatter": 5}
 MODE = {"direct": 0, "staged": 1}
 FLAG_ACCUMULATE = 0x1
 DTYPE_CODE = {"f32": 0, "bf16": 1, "i32": 2}
@@ -75,6 +76,12 @@ def _load():
         "adapcc_allreduce_lb": [vp, pp, pp, sz, i32, u64, ctypes.c_uint, vp],
         "adapcc_allgather_lb": [vp, pp, pp, sz, i32, u64, vp],
         "adapcc_alltoall_lb": [vp, pp, pp, sz, i32, u64, vp],
+        "adapcc_reduce": [vp, vp, vp, sz, i32, i32, u64, ctypes.c_uint, vp],
+        "adapcc_broadcast": [vp, vp, vp, sz, i32, i32, u64, vp],
+        "adapcc_reducescatter": [vp, vp, vp, sz, i32, u64, ctypes.c_uint, vp],
+        "adapcc_reduce_lb": [vp, pp, pp, sz, i32, i32, u64, ctypes.c_uint, vp],
+        "adapcc_broadcast_lb": [vp, pp, pp, sz, i32, i32, u64, vp],
+        "adapcc_reducescatter_lb": [vp, pp, pp, sz, i32, u64, ctypes.c_uint, vp],
         "adapcc_get_async_error": [vp],
         "adapcc_finalize": [vp],
         "adapcc_config": [vp, ctypes.c_char_p, i64],
@@ -318,12 +325,37 @@ class Communicator:
                                        _stream(stream)), "alltoall")
         return out
 
+    def reduce(self, x, out, root, ready=None, accumulate=False, stream=None):
+        """Only the root's `out` is written (non-roots may pass None)."""
+        m = _mask(ready, self.nranks)
+        send = x if (m >> self.rank) & 1 else None
+        n_el = (out if out is not None else x).numel()
+        _check(_load().adapcc_reduce(self._h, _ptr(send), _ptr(out), n_el,
+                                     _dtype_code(out if out is not None else x), root, m,
+                                     FLAG_ACCUMULATE if accumulate else 0, _stream(stream)), "reduce")
+        return out
+
+    def broadcast(self, x, out, root, ready=None, stream=None):
+        m = _mask(ready, self.nranks)
+        send = x if (self.rank == root and (m >> root) & 1) else None
+        _check(_load().adapcc_broadcast(self._h, _ptr(send), _ptr(out), out.numel(), _dtype_code(out),
+                                        root, m, _stream(stream)), "broadcast")
+        return out
+
+    def reducescatter(self, x, out, ready=None, accumulate=False, stream=None):
+        m = _mask(ready, self.nranks)
+        send = x if (m >> self.rank) & 1 else None
+        _check(_load().adapcc_reducescatter(self._h, _ptr(send), _ptr(out), out.numel(),
+                                            _dtype_code(out), m, FLAG_ACCUMULATE if accumulate else 0,
+                                            _stream(stream)), "reducescatter")
+        return out
+
     # ---- loopback collectives (lists of per-virtual-rank tensors)
     def _arrays(self, xs, outs, m):
         n = self.nranks
         skey = tuple((xs[r].data_ptr() if ((m >> r) & 1 and xs[r] is not None) else 0)
                      for r in range(n))
-        dkey = tuple(o.data_ptr() for o in outs)
+        dkey = tuple((o.data_ptr() if o is not None else 0) for o in outs)
         cached = getattr(self, "_arr_cache", None)
         if cached is not None and cached[0] == skey and cached[1] == dkey:
             return cached[2], cached[3]
@@ -352,4 +384,27 @@ class Communicator:
         S, D = self._arrays(xs, outs, m)
         _check(_load().adapcc_alltoall_lb(self._h, S, D, outs[0].numel() // self.nranks,
                                           _dtype_code(outs[0]), m, _stream(stream)), "alltoall_lb")
+        return outs
+
+    def reduce_lb(self, xs, outs, root, ready=None, accumulate=False, stream=None):
+        m = _mask(ready, self.nranks)
+        S, D = self._arrays(xs, outs, m)
+        _check(_load().adapcc_reduce_lb(self._h, S, D, outs[root].numel(), _dtype_code(outs[root]), root,
+                                        m, FLAG_ACCUMULATE if accumulate else 0, _stream(stream)),
+               "reduce_lb")
+        return outs
+
+    def broadcast_lb(self, xs, outs, root, ready=None, stream=None):
+        m = _mask(ready, self.nranks)
+        S, D = self._arrays(xs, outs, m)
+        _check(_load().adapcc_broadcast_lb(self._h, S, D, outs[0].numel(), _dtype_code(outs[0]), root, m,
+                                           _stream(stream)), "broadcast_lb")
+        return outs
+
+    def reducescatter_lb(self, xs, outs, ready=None, accumulate=False, stream=None):
+        m = _mask(ready, self.nranks)
+        S, D = self._arrays(xs, outs, m)
+        _check(_load().adapcc_reducescatter_lb(self._h, S, D, outs[0].numel(), _dtype_code(outs[0]), m,
+                                               FLAG_ACCUMULATE if accumulate else 0, _stream(stream)),
+               "reducescatter_lb")
         return outs

@@ -65,8 +65,25 @@ using PlanKey = std::tuple<int, uint64_t, uint64_t, int, uint64_t, unsigned>;
 
 int esize_of(adapcc_dtype_t d) { return d == ADAPCC_BFLOAT16 ? 2 : 4; }
 
-std::string default_strategy(Coll c, int n) {
+std::string star(int n, int root) {
+  std::string p;
+  for (int g = 0; g < n; ++g) p += (g ? "," : "") + std::to_string(g == root ? -1 : root);
+  return p;
+}
+
+// Defaults; Reduce / Broadcast defaults are generated for the
+// call's root: one star tree (all trees of a Reduce share the root).
+std::string default_strategy(Coll c, int n, int root = 0) {
   std::string s = "adapcc-strategy 1\nnranks " + std::to_string(n) + "\ncollective ";
+  if (c == kReduce) return s + "reduce\ntree weight=1 chunk=262144 parent=" + star(n, root) + "\n";
+  if (c == kBroadcast)
+    return s + "broadcast\nbcast src=" + std::to_string(root) + " weight=1 chunk=262144 parent=" + star(n, root) + "\n";
+  if (c == kReduceScatter) {
+    s += "reducescatter\n";
+    for (int b = 0; b < n; ++b)
+      s += "rtree dst=" + std::to_string(b) + " weight=1 chunk=262144 parent=" + star(n, b) + "\n";
+    return s;
+  }
   if (c == kAllReduce) {
     s += "allreduce\n";
     for (int m = 0; m < n; ++m) {  // n star trees, equal weights
@@ -107,10 +124,9 @@ struct adapcc_comm_s {
   DevState* state = nullptr;              // device epoch + work counters
   int* h_err = nullptr;
   int* d_err = nullptr;
-  Strategy strat[3];
-  // plan-cache identity of the active strategy: the hash of its normalised
-  // text, so swapping back to a strategy seen before reuses its cached plans
-  uint64_t strat_version[3] = {0, 0, 0};
+  Strategy strat[kNumColl];
+  bool user_set[kNumColl] = {};          // set_strategy was called for this collective
+  std::map<int, Strategy> rooted[kNumColl];  // default Reduce/Broadcast strategies per root
   std::map<PlanKey, std::shared_ptr<DevPlan>> plans;
   uint64_t tick = 0;  // plan-cache clock (least recently used plan is evicted)
   int64_t timeout_ms = 10000;
@@ -165,11 +181,10 @@ adapcc_result_t common_init(adapcc_comm_s* c, size_t scratch) {
   CK(cudaHostAlloc(&c->h_err, sizeof(int), cudaHostAllocMapped));
   *c->h_err = 0;
   CK(cudaHostGetDevicePointer(&c->d_err, c->h_err, 0));
-  for (int k = 0; k < 3; ++k) {
+  for (int k = 0; k < kNumColl; ++k) {
     std::string err;
     if (!parse_strategy(default_strategy((Coll)k, c->nranks).c_str(), &c->strat[k], &err))
       return ADAPCC_ERR_INVALID_STRATEGY;
-    c->strat_version[k] = c->strat[k].hash;
   }
   return ADAPCC_SUCCESS;
 }
@@ -219,9 +234,37 @@ int grid_size(const adapcc_comm_s* c, adapcc_dtype_t dtype, int engine) {
   return std::max(grid, 1);
 }
 
-adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, uint64_t count, adapcc_dtype_t dtype,
-                         uint64_t mask, unsigned flags, std::shared_ptr<DevPlan>* out) {
-  PlanKey key{(int)coll, c->strat_version[coll], count, (int)dtype, mask, flags};
+// The strategy a call runs on: the user's, or (Reduce / Broadcast without a
+// user strategy) the default rooted at the call's root.  Plans are cached by
+// the strategy's hash, so swapping back to a strategy seen before reuses them.
+adapcc_result_t pick_strategy(adapcc_comm_s* c, Coll coll, int root, const Strategy** out) {
+  if (coll != kReduce && coll != kBroadcast) {
+    *out = &c->strat[coll];
+    return ADAPCC_SUCCESS;
+  }
+  if (root < 0 || root >= c->nranks) return ADAPCC_ERR_INVALID_ARGUMENT;
+  if (c->user_set[coll]) {
+    const Strategy& st = c->strat[coll];
+    const int sroot = coll == kReduce ? st.subs[0].root : st.subs[0].src;
+    if (sroot != root) return ADAPCC_ERR_INVALID_ARGUMENT;
+    *out = &st;
+    return ADAPCC_SUCCESS;
+  }
+  auto it = c->rooted[coll].find(root);
+  if (it == c->rooted[coll].end()) {
+    Strategy st;
+    if (!parse_strategy(default_strategy(coll, c->nranks, root).c_str(), &st, nullptr))
+      return ADAPCC_ERR_INVALID_STRATEGY;
+    it = c->rooted[coll].emplace(root, std::move(st)).first;
+  }
+  *out = &it->second;
+  return ADAPCC_SUCCESS;
+}
+
+adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, const Strategy* strat, uint64_t count,
+                         adapcc_dtype_t dtype, uint64_t mask, unsigned flags,
+                         std::shared_ptr<DevPlan>* out) {
+  PlanKey key{(int)coll, strat->hash, count, (int)dtype, mask, flags};
   auto it = c->plans.find(key);
   if (it != c->plans.end()) {
     it->second->last_tick = ++c->tick;
@@ -229,7 +272,7 @@ adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, uint64_t count, adapcc_dty
     return ADAPCC_SUCCESS;
   }
   PlanRequest rq;
-  rq.st = &c->strat[coll];
+  rq.st = strat;
   rq.count = count;
   rq.esize = esize_of(dtype);
   rq.ready_mask = mask;
@@ -282,11 +325,14 @@ adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, uint64_t count, adapcc_dty
 
 adapcc_result_t run(adapcc_comm_s* c, Coll coll, const void* const* send, void* const* recv,
                     uint64_t count, adapcc_dtype_t dtype, uint64_t mask, unsigned flags,
-                    adapcc_stream_t stream) {
+                    adapcc_stream_t stream, int root = 0) {
   std::lock_guard<std::mutex> lock(c->mu);
   CK(cudaSetDevice(c->device));
+  const Strategy* strat = nullptr;
+  adapcc_result_t r = pick_strategy(c, coll, root, &strat);
+  if (r != ADAPCC_SUCCESS) return r;
   std::shared_ptr<DevPlan> plan;
-  adapcc_result_t r = get_plan(c, coll, count, dtype, mask, flags, &plan);
+  r = get_plan(c, coll, strat, count, dtype, mask, flags, &plan);
   if (r != ADAPCC_SUCCESS) return r;
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
   cudaStreamCaptureStatus cap = cudaStreamCaptureStatusNone;
@@ -423,14 +469,14 @@ adapcc_result_t adapcc_init(adapcc_comm_t* comm, int rank, int nranks, int cuda_
 adapcc_result_t adapcc_set_strategy(adapcc_comm_t c, adapcc_coll_t coll, const char* text,
                                     adapcc_stream_t stream) {
   (void)stream;
-  if (!c || coll < ADAPCC_ALLREDUCE || coll > ADAPCC_ALLTOALL) return ADAPCC_ERR_INVALID_ARGUMENT;
+  if (!c || coll < ADAPCC_ALLREDUCE || coll > ADAPCC_REDUCESCATTER) return ADAPCC_ERR_INVALID_ARGUMENT;
   Strategy st;
   std::string err;
   if (!parse_strategy(text, &st, &err)) return ADAPCC_ERR_INVALID_STRATEGY;
   if (st.nranks != c->nranks || (int)st.coll != (int)coll) return ADAPCC_ERR_INVALID_STRATEGY;
   std::lock_guard<std::mutex> lock(c->mu);
   c->strat[coll] = std::move(st);
-  c->strat_version[coll] = c->strat[coll].hash;
+  c->user_set[coll] = true;
   return ADAPCC_SUCCESS;
 }
 
@@ -497,7 +543,8 @@ static adapcc_result_t check_lb(adapcc_comm_t c, const void* const* s, void* con
     if (misaligned(s[q])) return ADAPCC_ERR_INVALID_ARGUMENT;
     if (!sbytes) continue;
     const bool in_place_ok = (kind == 0 && s[q] == d[q]) ||
-                             (kind == 1 && s[q] == static_cast<const char*>(d[q]) + q * sbytes);
+                             (kind == 1 && s[q] == static_cast<const char*>(d[q]) + q * sbytes) ||
+                             (kind == 3 && d[q] == static_cast<const char*>(s[q]) + q * rbytes);
     if (!in_place_ok && overlap(s[q], sbytes, d[q], rbytes)) return ADAPCC_ERR_INVALID_ARGUMENT;
   }
   return ADAPCC_SUCCESS;
@@ -535,6 +582,107 @@ adapcc_result_t adapcc_alltoall_lb(adapcc_comm_t c, const void* const* sendbufs,
   r = check_lb(c, sendbufs, recvbufs, bytes, bytes, mask, 2);
   if (r != ADAPCC_SUCCESS) return r;
   return run(c, kAllToAll, sendbufs, recvbufs, count_per_peer, dtype, mask, 0, stream);
+}
+
+// ------------------------------------------------ NEXT-4: Reduce / Broadcast / ReduceScatter
+adapcc_result_t adapcc_reduce(adapcc_comm_t c, const void* sendbuf, void* recvbuf, size_t count,
+                              adapcc_dtype_t dtype, int root, uint64_t mask, unsigned flags,
+                              adapcc_stream_t stream) {
+  adapcc_result_t r = check_common(c, dtype, mask);
+  if (r != ADAPCC_SUCCESS) return r;
+  if (c->loopback || (flags & ~ADAPCC_FLAG_ACCUMULATE) || root < 0 || root >= c->nranks)
+    return ADAPCC_ERR_INVALID_ARGUMENT;
+  const size_t bytes = count * esize_of(dtype);
+  const bool ready = (mask >> c->rank) & 1, is_root = c->rank == root;
+  if (count && ((ready && !sendbuf) || (is_root && !recvbuf))) return ADAPCC_ERR_INVALID_ARGUMENT;
+  if ((ready && misaligned(sendbuf)) || (is_root && misaligned(recvbuf))) return ADAPCC_ERR_INVALID_ARGUMENT;
+  if (ready && is_root && sendbuf != recvbuf && overlap(sendbuf, bytes, recvbuf, bytes))
+    return ADAPCC_ERR_INVALID_ARGUMENT;
+  const void* s[1] = {ready ? sendbuf : nullptr};
+  void* d[1] = {recvbuf};
+  return run(c, kReduce, s, d, count, dtype, mask, flags, stream, root);
+}
+
+adapcc_result_t adapcc_broadcast(adapcc_comm_t c, const void* sendbuf, void* recvbuf, size_t count,
+                                 adapcc_dtype_t dtype, int root, uint64_t mask, adapcc_stream_t stream) {
+  adapcc_result_t r = check_common(c, dtype, mask);
+  if (r != ADAPCC_SUCCESS) return r;
+  if (c->loopback || root < 0 || root >= c->nranks) return ADAPCC_ERR_INVALID_ARGUMENT;
+  const size_t bytes = count * esize_of(dtype);
+  const bool src = c->rank == root && ((mask >> root) & 1);
+  if (count && (!recvbuf || (src && !sendbuf))) return ADAPCC_ERR_INVALID_ARGUMENT;
+  if (misaligned(recvbuf) || (src && misaligned(sendbuf))) return ADAPCC_ERR_INVALID_ARGUMENT;
+  if (src && sendbuf != recvbuf && overlap(sendbuf, bytes, recvbuf, bytes)) return ADAPCC_ERR_INVALID_ARGUMENT;
+  const void* s[1] = {src ? sendbuf : nullptr};
+  void* d[1] = {recvbuf};
+  return run(c, kBroadcast, s, d, count, dtype, mask, 0, stream, root);
+}
+
+adapcc_result_t adapcc_reducescatter(adapcc_comm_t c, const void* sendbuf, void* recvbuf,
+                                     size_t recvcount, adapcc_dtype_t dtype, uint64_t mask,
+                                     unsigned flags, adapcc_stream_t stream) {
+  adapcc_result_t r = check_common(c, dtype, mask);
+  if (r != ADAPCC_SUCCESS) return r;
+  if (c->loopback || (flags & ~ADAPCC_FLAG_ACCUMULATE)) return ADAPCC_ERR_INVALID_ARGUMENT;
+  const size_t rbytes = recvcount * esize_of(dtype);
+  const bool ready = (mask >> c->rank) & 1;
+  if (recvcount && (!recvbuf || (ready && !sendbuf))) return ADAPCC_ERR_INVALID_ARGUMENT;
+  if (misaligned(recvbuf) || (ready && misaligned(sendbuf))) return ADAPCC_ERR_INVALID_ARGUMENT;
+  if (ready && overlap(sendbuf, rbytes * c->nranks, recvbuf, rbytes) &&
+      recvbuf != static_cast<const char*>(sendbuf) + c->rank * rbytes)
+    return ADAPCC_ERR_INVALID_ARGUMENT;
+  const void* s[1] = {ready ? sendbuf : nullptr};
+  void* d[1] = {recvbuf};
+  return run(c, kReduceScatter, s, d, recvcount, dtype, mask, flags, stream);
+}
+
+adapcc_result_t adapcc_reduce_lb(adapcc_comm_t c, const void* const* sendbufs, void* const* recvbufs,
+                                 size_t count, adapcc_dtype_t dtype, int root, uint64_t mask,
+                                 unsigned flags, adapcc_stream_t stream) {
+  adapcc_result_t r = check_common(c, dtype, mask);
+  if (r != ADAPCC_SUCCESS) return r;
+  if (!c->loopback || !sendbufs || !recvbufs || (flags & ~ADAPCC_FLAG_ACCUMULATE) || root < 0 ||
+      root >= c->nranks)
+    return ADAPCC_ERR_INVALID_ARGUMENT;
+  const size_t bytes = count * esize_of(dtype);
+  for (int q = 0; q < c->nranks; ++q) {
+    if (((mask >> q) & 1) && ((count && !sendbufs[q]) || misaligned(sendbufs[q]))) return ADAPCC_ERR_INVALID_ARGUMENT;
+  }
+  if ((count && !recvbufs[root]) || misaligned(recvbufs[root])) return ADAPCC_ERR_INVALID_ARGUMENT;
+  if (((mask >> root) & 1) && sendbufs[root] != recvbufs[root] &&
+      overlap(sendbufs[root], bytes, recvbufs[root], bytes))
+    return ADAPCC_ERR_INVALID_ARGUMENT;
+  return run(c, kReduce, sendbufs, recvbufs, count, dtype, mask, flags, stream, root);
+}
+
+adapcc_result_t adapcc_broadcast_lb(adapcc_comm_t c, const void* const* sendbufs, void* const* recvbufs,
+                                    size_t count, adapcc_dtype_t dtype, int root, uint64_t mask,
+                                    adapcc_stream_t stream) {
+  adapcc_result_t r = check_common(c, dtype, mask);
+  if (r != ADAPCC_SUCCESS) return r;
+  if (!c->loopback || !sendbufs || !recvbufs || root < 0 || root >= c->nranks) return ADAPCC_ERR_INVALID_ARGUMENT;
+  const size_t bytes = count * esize_of(dtype);
+  for (int q = 0; q < c->nranks; ++q)
+    if ((count && !recvbufs[q]) || misaligned(recvbufs[q])) return ADAPCC_ERR_INVALID_ARGUMENT;
+  if ((mask >> root) & 1) {
+    if ((count && !sendbufs[root]) || misaligned(sendbufs[root])) return ADAPCC_ERR_INVALID_ARGUMENT;
+    for (int q = 0; q < c->nranks; ++q)
+      if (!(q == root && sendbufs[root] == recvbufs[q]) && overlap(sendbufs[root], bytes, recvbufs[q], bytes))
+        return ADAPCC_ERR_INVALID_ARGUMENT;
+  }
+  return run(c, kBroadcast, sendbufs, recvbufs, count, dtype, mask, 0, stream, root);
+}
+
+adapcc_result_t adapcc_reducescatter_lb(adapcc_comm_t c, const void* const* sendbufs,
+                                        void* const* recvbufs, size_t recvcount, adapcc_dtype_t dtype,
+                                        uint64_t mask, unsigned flags, adapcc_stream_t stream) {
+  adapcc_result_t r = check_common(c, dtype, mask);
+  if (r != ADAPCC_SUCCESS) return r;
+  if (flags & ~ADAPCC_FLAG_ACCUMULATE) return ADAPCC_ERR_INVALID_ARGUMENT;
+  const size_t rbytes = recvcount * esize_of(dtype);
+  r = check_lb(c, sendbufs, recvbufs, rbytes * c->nranks, rbytes, mask, 3);
+  if (r != ADAPCC_SUCCESS) return r;
+  return run(c, kReduceScatter, sendbufs, recvbufs, recvcount, dtype, mask, flags, stream);
 }
 
 const char* adapcc_last_cuda_error(void) {
@@ -638,7 +786,7 @@ adapcc_result_t adapcc_strategy_partition(const char* text, uint64_t count, adap
   if (!bounds || !nbounds) return ADAPCC_ERR_INVALID_ARGUMENT;
   std::vector<int64_t> w;
   for (auto& s : st.subs)
-    if (st.coll != kAllGather || s.src == src) w.push_back(s.weight);
+    if ((st.coll != kAllGather && st.coll != kReduceScatter) || s.src == src) w.push_back(s.weight);
   if (w.empty()) return ADAPCC_ERR_INVALID_ARGUMENT;
   auto b = partition(count, esize_of(dtype), w);
   for (size_t i = 0; i < b.size(); ++i) bounds[i] = b[i];

@@ -140,8 +140,11 @@ std::vector<int> bfs_order(const SubColl& s) {
 }
 
 // ------------------------------------------------------------- AllReduce
+// send_bias: byte offset of the tree's block inside every rank's sendbuf
+// (ReduceScatter block b); root_only: the result goes to the root's recvbuf
+// only (Reduce, ReduceScatter) instead of every rank (AllReduce).
 void plan_allreduce_tree(Builder& B, const SubColl& s, uint64_t lo, uint64_t hi, uint64_t mask,
-                         bool accumulate, Mode mode) {
+                         bool accumulate, Mode mode, int64_t send_bias = 0, bool root_only = false) {
   const int n = B.n_;
   const int es = B.esize_;
   const uint32_t ce = (uint32_t)(s.chunk / es);
@@ -157,12 +160,13 @@ void plan_allreduce_tree(Builder& B, const SubColl& s, uint64_t lo, uint64_t hi,
   if (zero && accumulate) return;  // recvbuf untouched (reading Q7)
 
   std::vector<BufRef> recv_all;
-  for (int g = 0; g < n; ++g) recv_all.push_back(make_ref(kBufRecv, g, 0, accumulate));
+  for (int g = 0; g < n; ++g)
+    if (!root_only || g == s.root) recv_all.push_back(make_ref(kBufRecv, g, 0, accumulate));
 
   if (mode == kDirect) {
     std::map<int, std::pair<uint64_t, FlagRef>> agg_slot;  // kernel node -> slot
     auto stream_of = [&](const Flow& f) {
-      if (f.kind == Flow::kIn) { Stream st; st.ref = make_ref(kBufSend, f.rank, 0); return st; }
+      if (f.kind == Flow::kIn) { Stream st; st.ref = make_ref(kBufSend, f.rank, send_bias); return st; }
       auto& as = agg_slot.at(f.rank);
       return B.slot_stream(f.rank, as.first, lo, &as.second);
     };
@@ -196,7 +200,7 @@ void plan_allreduce_tree(Builder& B, const SubColl& s, uint64_t lo, uint64_t hi,
     for (const Flow& f : L) {
       if (f.kind == Flow::kIn && f.rank == c) {
         Stream st;
-        st.ref = make_ref(kBufSend, c, 0);
+        st.ref = make_ref(kBufSend, c, send_bias);
         srcs.push_back(st);
         continue;
       }
@@ -213,7 +217,7 @@ void plan_allreduce_tree(Builder& B, const SubColl& s, uint64_t lo, uint64_t hi,
     const int r = kv.first.second;
     const Dest& d = kv.second;
     Stream src;
-    src.ref = make_ref(kBufSend, r, 0);
+    src.ref = make_ref(kBufSend, r, send_bias);
     B.add(r, lo, hi, ce, kOpFold, {src},
           {make_ref(kBufArena, d.rank, (int64_t)d.off - (int64_t)(lo * es))}, {d.flag});
   }
@@ -237,9 +241,10 @@ void plan_allreduce_tree(Builder& B, const SubColl& s, uint64_t lo, uint64_t hi,
   {
     std::vector<BufRef> dsts = {make_ref(kBufRecv, root, 0, accumulate)};
     std::vector<FlagRef> posts;
-    add_down_dst(root, &dsts, &posts);
+    if (!root_only) add_down_dst(root, &dsts, &posts);
     B.add(root, lo, hi, ce, zero ? kOpZero : kOpFold, consumer_srcs[root], dsts, posts);
   }
+  if (root_only) return;
   // broadcast down the reversed tree, parents before children
   for (int g : bfs_order(s)) {
     if (g == root) continue;
@@ -254,8 +259,10 @@ void plan_allreduce_tree(Builder& B, const SubColl& s, uint64_t lo, uint64_t hi,
 }
 
 // ------------------------------------------------------------- AllGather
+// slot_bias < 0: AllGather (source s lands in slot s of every recvbuf);
+// otherwise Broadcast (lands at that byte offset).
 void plan_allgather_tree(Builder& B, const SubColl& s, uint64_t lo, uint64_t hi, uint64_t cnt,
-                         uint64_t mask, Mode mode) {
+                         uint64_t mask, Mode mode, int64_t slot_bias_override = -1) {
   const int n = B.n_;
   const int es = B.esize_;
   const int src = s.src;
@@ -263,7 +270,7 @@ void plan_allgather_tree(Builder& B, const SubColl& s, uint64_t lo, uint64_t hi,
   const uint32_t ce = (uint32_t)(s.chunk / es);
   const uint32_t nch = (uint32_t)((hi - lo + ce - 1) / ce);
   const uint64_t len = (hi - lo) * es;
-  const int64_t slot_bias = (int64_t)(src * cnt * es);
+  const int64_t slot_bias = slot_bias_override >= 0 ? slot_bias_override : (int64_t)(src * cnt * es);
   Stream in;
   in.ref = make_ref(kBufSend, src, 0);
   if (mode == kDirect) {
@@ -329,12 +336,17 @@ SegmentPlan build_segment(const PlanRequest& rq,
     const uint64_t lo = ranges[m].first, hi = ranges[m].second;
     if (lo >= hi) continue;
     const SubColl& s = st.subs[m];
-    if (st.coll == kAllReduce)
-      plan_allreduce_tree(B, s, lo, hi, rq.ready_mask, rq.accumulate, rq.mode);
-    else if (st.coll == kAllGather)
-      plan_allgather_tree(B, s, lo, hi, rq.count, rq.ready_mask, rq.mode);
-    else
-      plan_alltoall_line(B, s, lo, hi, rq.count, rq.ready_mask, rq.mode);
+    switch (st.coll) {
+      case kAllReduce: plan_allreduce_tree(B, s, lo, hi, rq.ready_mask, rq.accumulate, rq.mode); break;
+      case kReduce: plan_allreduce_tree(B, s, lo, hi, rq.ready_mask, rq.accumulate, rq.mode, 0, true); break;
+      case kReduceScatter:
+        plan_allreduce_tree(B, s, lo, hi, rq.ready_mask, rq.accumulate, rq.mode,
+                            (int64_t)((uint64_t)s.src * rq.count * rq.esize), true);
+        break;
+      case kAllGather: plan_allgather_tree(B, s, lo, hi, rq.count, rq.ready_mask, rq.mode); break;
+      case kBroadcast: plan_allgather_tree(B, s, lo, hi, rq.count, rq.ready_mask, rq.mode, 0); break;
+      default: plan_alltoall_line(B, s, lo, hi, rq.count, rq.ready_mask, rq.mode); break;
+    }
   }
   return B.finish();
 }
@@ -349,7 +361,7 @@ uint64_t flag_region_bytes(uint64_t half) {
 std::vector<std::pair<uint64_t, uint64_t>> sub_ranges(const Strategy& st, uint64_t count,
                                                       int esize) {
   std::vector<std::pair<uint64_t, uint64_t>> r(st.subs.size());
-  if (st.coll == kAllGather) {
+  if (st.coll == kAllGather || st.coll == kReduceScatter) {
     for (int src = 0; src < st.nranks; ++src) {
       std::vector<int64_t> w;
       std::vector<size_t> idx;

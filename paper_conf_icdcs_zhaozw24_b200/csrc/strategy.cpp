@@ -146,10 +146,13 @@ bool parse_strategy(const char* text, Strategy* out, std::string* err) {
       if (t[1] == "allreduce") coll = kAllReduce;
       else if (t[1] == "allgather") coll = kAllGather;
       else if (t[1] == "alltoall") coll = kAllToAll;
+      else if (t[1] == "reduce") coll = kReduce;
+      else if (t[1] == "broadcast") coll = kBroadcast;
+      else if (t[1] == "reducescatter") coll = kReduceScatter;
       else return fail(err, "unknown collective");
       continue;
     }
-    if (t[0] != "tree" && t[0] != "ring" && t[0] != "bcast" && t[0] != "a2a")
+    if (t[0] != "tree" && t[0] != "ring" && t[0] != "bcast" && t[0] != "a2a" && t[0] != "rtree")
       return fail(err, "unknown directive " + t[0]);
     Raw r;
     r.head = t[0];
@@ -171,11 +174,15 @@ bool parse_strategy(const char* text, Strategy* out, std::string* err) {
   for (const Raw& r : raws) {
     const bool ok_kind = (coll == kAllReduce && (r.head == "tree" || r.head == "ring")) ||
                          (coll == kAllGather && r.head == "bcast") ||
-                         (coll == kAllToAll && r.head == "a2a");
+                         (coll == kAllToAll && r.head == "a2a") ||
+                         (coll == kReduce && r.head == "tree") ||
+                         (coll == kBroadcast && r.head == "bcast") ||
+                         (coll == kReduceScatter && r.head == "rtree");
     if (!ok_kind) return fail(err, "directive " + r.head + " not valid for this collective");
     std::vector<std::string> required = {"weight", "chunk"};
     std::vector<std::string> optional;
     if (r.head == "tree") { required.push_back("parent"); optional.push_back("noagg"); }
+    if (r.head == "rtree") { required.push_back("parent"); required.push_back("dst"); optional.push_back("noagg"); }
     if (r.head == "ring") required.push_back("order");
     if (r.head == "bcast") { required.push_back("parent"); required.push_back("src"); }
     for (auto& k : required)
@@ -227,8 +234,14 @@ bool parse_strategy(const char* text, Strategy* out, std::string* err) {
     if (!check_tree(parent, n, err)) return false;
     s.parent.assign(parent.begin(), parent.end());
     finish_tree(&s, n);
-    if (r.head == "tree") {
-      s.kind = kTree;
+    if (r.head == "tree" || r.head == "rtree") {
+      s.kind = r.head == "tree" ? kTree : kRTree;
+      if (s.kind == kRTree) {
+        int64_t dst;
+        if (!parse_int(r.kv.at("dst"), &dst) || dst < 0 || dst >= n) return fail(err, "bad rtree dst");
+        if (s.root != dst) return fail(err, "rtree root must be its dst");
+        s.src = (int)dst;
+      }
       if (r.kv.count("noagg")) {
         std::vector<int64_t> na;
         if (!parse_list(r.kv.at("noagg"), &na)) return fail(err, "bad noagg list");
@@ -249,15 +262,19 @@ bool parse_strategy(const char* text, Strategy* out, std::string* err) {
     st.subs.push_back(std::move(s));
   }
   if ((int)st.subs.size() > kMaxSubs) return fail(err, "too many sub-collectives");
-  if (coll == kAllGather) {
+  if (coll == kAllGather || coll == kReduceScatter) {
     for (int src = 0; src < n; ++src) {
       int64_t tot = 0;
       int lines_for_src = 0;
       for (auto& s : st.subs)
         if (s.src == src) { tot += s.weight; ++lines_for_src; }
-      if (lines_for_src == 0 || tot == 0) return fail(err, "allgather source without positive-weight bcast");
+      if (lines_for_src == 0 || tot == 0) return fail(err, "block without a positive-weight line");
     }
   } else {
+    for (auto& s : st.subs) {
+      if (coll == kReduce && s.root != st.subs[0].root) return fail(err, "reduce trees must share one root");
+      if (coll == kBroadcast && s.src != st.subs[0].src) return fail(err, "broadcast lines must share one src");
+    }
     int64_t tot = 0;
     for (auto& s : st.subs) tot += s.weight;
     if (tot == 0) return fail(err, "total weight must be > 0");

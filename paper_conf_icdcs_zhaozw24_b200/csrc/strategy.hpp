@@ -19,8 +19,12 @@ constexpr int kMaxSubs = 128;
 constexpr int64_t kMaxWeight = int64_t(1) << 24;
 constexpr int64_t kMaxChunk = int64_t(1) << 31;
 
-enum Coll : int { kAllReduce = 0, kAllGather = 1, kAllToAll = 2 };
-enum SubKind : int { kTree = 0, kBcast = 1, kA2A = 2 };
+enum Coll : int {
+  kAllReduce = 0, kAllGather = 1, kAllToAll = 2,
+  kReduce = 3, kBroadcast = 4, kReduceScatter = 5  // NEXT-4 primitives
+};
+constexpr int kNumColl = 6;
+enum SubKind : int { kTree = 0, kBcast = 1, kA2A = 2, kRTree = 3 };
 
 struct SubColl {
   SubKind kind = kTree;
@@ -28,7 +32,7 @@ struct SubColl {
   int64_t chunk = 0;           // C_m, bytes, multiple of 16
   std::vector<int> parent;     // tree / bcast; -1 at the root
   uint64_t noagg = 0;          // bit g: a_{m,g} = 0
-  int src = -1;                // bcast source
+  int src = -1;                // bcast: source; rtree: destination block (== root)
   int root = -1;
   std::vector<std::vector<int>> children;  // ascending rank order (reading Q5)
 };

@@ -187,3 +187,38 @@ def allgather_chains(n, chunk=1 << 20):
 def alltoall_direct(n, chunk=1 << 20, lines=1):
     return _header(n, "alltoall") + "".join(
         f"a2a weight=1 chunk={int(chunk)}\n" for _ in range(lines))
+
+
+# ----------------------------------------------------- NEXT-4 primitives
+def reduce_trees(parents, weights=None, chunk=DEFAULT_CHUNK, noaggs=None):
+    """Reduce: every tree must be rooted at the Reduce root."""
+    n = len(parents[0])
+    weights = weights if weights is not None else [1] * len(parents)
+    noaggs = noaggs or [()] * len(parents)
+    out = _header(n, "reduce")
+    for p, w, na in zip(parents, weights, noaggs):
+        out += f"tree weight={int(w)} chunk={int(chunk)} parent={_join(p)}"
+        if na:
+            out += f" noagg={_join(na)}"
+        out += "\n"
+    return out
+
+
+def broadcast_trees(root, parents, weights=None, chunk=DEFAULT_CHUNK):
+    n = len(parents[0])
+    weights = weights if weights is not None else [1] * len(parents)
+    return _header(n, "broadcast") + "".join(
+        f"bcast src={root} weight={int(w)} chunk={int(chunk)} parent={_join(p)}\n"
+        for p, w in zip(parents, weights))
+
+
+def reducescatter_stars(n, chunk=DEFAULT_CHUNK):
+    """One star per block b rooted at b (b's block is reduced at b)."""
+    return _header(n, "reducescatter") + "".join(
+        f"rtree dst={b} weight=1 chunk={int(chunk)} parent={_join(star_parent(n, b))}\n" for b in range(n))
+
+
+def reducescatter_trees(lines, n, chunk=DEFAULT_CHUNK):
+    """lines: list of (dst, parent, weight)."""
+    return _header(n, "reducescatter") + "".join(
+        f"rtree dst={d} weight={int(w)} chunk={int(chunk)} parent={_join(p)}\n" for d, p, w in lines)

@@ -117,7 +117,19 @@ BAD = [
     "adapcc-strategy 1\nnranks 0\ncollective allreduce\ntree weight=1 chunk=16 parent=-1\n",
     "adapcc-strategy 1\nnranks 65\ncollective allreduce\n",
     "adapcc-strategy 1\nnranks 2\ncollective allreduce\n",
-    "adapcc-strategy 1\nnranks 2\ncollective reduce\ntree weight=1 chunk=16 parent=-1,0\n",
+    "adapcc-strategy 1\nnranks 2\ncollective gather\ntree weight=1 chunk=16 parent=-1,0\n",
+    # reduce trees must share one root; broadcast lines one src; rtree root == dst;
+    # every reducescatter block needs a positive-weight line
+    "adapcc-strategy 1\nnranks 2\ncollective reduce\ntree weight=1 chunk=16 parent=-1,0\n"
+    "tree weight=1 chunk=16 parent=1,-1\n",
+    "adapcc-strategy 1\nnranks 2\ncollective reduce\nring weight=1 chunk=16 order=0,1\n",
+    "adapcc-strategy 1\nnranks 2\ncollective broadcast\nbcast src=0 weight=1 chunk=16 parent=-1,0\n"
+    "bcast src=1 weight=1 chunk=16 parent=1,-1\n",
+    "adapcc-strategy 1\nnranks 2\ncollective reducescatter\nrtree dst=0 weight=1 chunk=16 parent=1,-1\n"
+    "rtree dst=1 weight=1 chunk=16 parent=1,-1\n",
+    "adapcc-strategy 1\nnranks 2\ncollective reducescatter\nrtree dst=0 weight=1 chunk=16 parent=-1,0\n",
+    "adapcc-strategy 1\nnranks 2\ncollective reducescatter\nrtree dst=0 weight=1 chunk=16 parent=-1,0\n"
+    "rtree dst=1 weight=0 chunk=16 parent=1,-1\n",
     "adapcc-strategy 1\nnranks 2\ncollective allreduce\ntree weight=1 chunk=8 parent=-1,0\n",
     "adapcc-strategy 1\nnranks 2\ncollective allreduce\ntree weight=1 chunk=24 parent=-1,0\n",
     "adapcc-strategy 1\nnranks 2\ncollective allreduce\ntree weight=0 chunk=16 parent=-1,0\n",
@@ -394,3 +406,60 @@ def test_allreduce_elements_equals_full_replay_at_samples():
         full = oc.allreduce(xs, txt, R, "bf16")[0]
         got = oc.allreduce_elements([x[idx] for x in xs], idx, count, txt, R, "bf16")
         assert np.array_equal(full[idx], got)
+
+
+# ------------------------------------------------------- NEXT-4: Reduce / Broadcast / RS
+def test_reduce_equals_allreduce_at_root_and_leaves_others():
+    n, count = 5, 301
+    xs = rank_tensors("f32", count, n)
+    trees = [S.chain([4, 3, 2, 1, 0]), S.star(n, 0), [-1, 0, 1, 1, 2]]
+    red = S.header(n, "reduce") + "".join(S.tree_line(p, w, 32) for p, w in zip(trees, [2, 1, 3]))
+    allr = S.allreduce_trees(trees, [2, 1, 3], chunk=32)
+    prev = [np.full(count, 7.0, np.float32) for _ in range(n)]
+    for R in ({0, 1, 2, 3, 4}, {1, 3}, set()):
+        ys = oc.reduce(xs, red, R, "f32", y_prev=prev)
+        ref = oc.allreduce(xs, allr, R, "f32")[0]
+        assert np.array_equal(ys[0].view(np.uint32), ref.view(np.uint32))   # same trees, same order
+        assert all(np.array_equal(ys[g], prev[g]) for g in range(1, n))
+
+
+def test_reduce_int32_brute_force_and_accumulate():
+    n, count = 4, 77
+    xs = rank_tensors("i32", count, n)
+    red = S.header(n, "reduce") + S.tree_line(S.chain([1, 2, 3, 0]), 1, 16) + S.tree_line(S.star(n, 0), 2, 16)
+    y1 = oc.reduce(xs, red, {0, 1}, "i32", y_prev=[np.zeros(count, np.int32)] * n)
+    y2 = oc.reduce(xs, red, {2, 3}, "i32", accumulate=True, y_prev=y1)
+    assert np.array_equal(y2[0], oc.allreduce_exact(xs, set(range(n)), "i32"))
+
+
+def test_broadcast_copies_root_or_untouched():
+    n, count = 4, 33
+    xs = rank_tensors("bf16", count, n)
+    txt = S.header(n, "broadcast") + "".join(
+        f"bcast src=2 weight={w} chunk=16 parent={','.join(map(str, p))}\n"
+        for w, p in [(1, S.star(n, 2)), (2, S.chain([0, 1, 3, 2]))])
+    prev = [np.full(count, 0x1234, np.uint16) for _ in range(n)]
+    assert all(np.array_equal(y, xs[2]) for y in oc.broadcast(xs, txt, {0, 2}, "bf16", prev))
+    assert all(np.array_equal(y, p) for y, p in zip(oc.broadcast(xs, txt, {0, 1}, "bf16", prev), prev))
+
+
+def test_reducescatter_is_block_of_allreduce():
+    n, cnt = 4, 50
+    xs = rank_tensors("i32", n * cnt, n)
+    txt = S.header(n, "reducescatter") + "".join(
+        f"rtree dst={b} weight=1 chunk=16 parent={','.join(map(str, S.star(n, b)))}\n" for b in range(n)) \
+        + "rtree dst=1 weight=3 chunk=32 parent=1,-1,1,2 noagg=2\n"
+    for R in (set(range(n)), {0, 3}):
+        ys = oc.reducescatter(xs, txt, R, "i32")
+        full = oc.allreduce_exact(xs, R, "i32", n * cnt)
+        for b in range(n):
+            assert np.array_equal(ys[b], full[b * cnt:(b + 1) * cnt])
+    # fp32 order: one star per block rooted at b equals the allreduce star replay of that block
+    xf = rank_tensors("f32", n * cnt, n)
+    rs = S.header(n, "reducescatter") + "".join(
+        f"rtree dst={b} weight=1 chunk=16 parent={','.join(map(str, S.star(n, b)))}\n" for b in range(n))
+    ys = oc.reducescatter(xf, rs, set(range(n)), "f32")
+    for b in range(n):
+        blk = [x[b * cnt:(b + 1) * cnt] for x in xf]
+        ref = oc.allreduce(blk, S.allreduce_trees([S.star(n, b)], chunk=16), set(range(n)), "f32")[0]
+        assert np.array_equal(ys[b].view(np.uint32), ref.view(np.uint32))
