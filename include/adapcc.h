@@ -189,6 +189,30 @@ ADAPCC_API adapcc_result_t adapcc_reducescatter_lb(adapcc_comm_t comm, const voi
                                                    adapcc_dtype_t dtype, uint64_t ready_mask,
                                                    unsigned flags, adapcc_stream_t stream);
 
+/* ----------------------------------------------- zero-copy (multi-process) ---
+ * Register a device buffer so that peers can read/write it directly: the
+ * allocation holding [ptr, ptr+bytes) is exported with CUDA IPC and mapped by
+ * every peer (one bootstrap all-gather; the paper's IPC "memory pointer
+ * table").  Collective: every rank registers a buffer of the same size
+ * in the same order; ids are assigned in that order.  The buffer must stay
+ * allocated until adapcc_deregister_buffer (collective, synchronizes the
+ * device).  UNSUPPORTED on loopback communicators (already zero-copy).
+ * adapcc_collective_zc runs any collective on registered buffers with the
+ * single-copy DIRECT plan across processes: a tree's root reads every rank's
+ * input slice straight from its registered sendbuf and writes the result
+ * straight into every rank's registered recvbuf over NVLink -- no landing or
+ * broadcast slots -- bracketed by in-kernel entry/exit barriers.  Offsets
+ * (bytes, multiples of 16) and count must be identical on every rank; count
+ * has the same meaning as in the collective's own entry point. */
+ADAPCC_API adapcc_result_t adapcc_register_buffer(adapcc_comm_t comm, void* ptr, size_t bytes,
+                                                  int* reg_id);
+ADAPCC_API adapcc_result_t adapcc_deregister_buffer(adapcc_comm_t comm, int reg_id);
+ADAPCC_API adapcc_result_t adapcc_collective_zc(adapcc_comm_t comm, adapcc_coll_t coll, int send_reg,
+                                                size_t send_offset, int recv_reg, size_t recv_offset,
+                                                size_t count, adapcc_dtype_t dtype, int root,
+                                                uint64_t ready_mask, unsigned flags,
+                                                adapcc_stream_t stream);
+
 /* ------------------------------------------------------------- lifecycle --- */
 
 /* Latched device error (TIMEOUT) or SUCCESS.  Does not synchronize. */

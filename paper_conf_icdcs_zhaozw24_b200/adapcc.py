@@ -82,6 +82,9 @@ def _load():
         "adapcc_reduce_lb": [vp, pp, pp, sz, i32, i32, u64, ctypes.c_uint, vp],
         "adapcc_broadcast_lb": [vp, pp, pp, sz, i32, i32, u64, vp],
         "adapcc_reducescatter_lb": [vp, pp, pp, sz, i32, u64, ctypes.c_uint, vp],
+        "adapcc_register_buffer": [vp, vp, sz, ctypes.POINTER(i32)],
+        "adapcc_deregister_buffer": [vp, i32],
+        "adapcc_collective_zc": [vp, i32, i32, sz, i32, sz, sz, i32, i32, u64, ctypes.c_uint, vp],
         "adapcc_get_async_error": [vp],
         "adapcc_finalize": [vp],
         "adapcc_config": [vp, ctypes.c_char_p, i64],
@@ -348,6 +351,38 @@ class Communicator:
         _check(_load().adapcc_reducescatter(self._h, _ptr(send), _ptr(out), out.numel(),
                                             _dtype_code(out), m, FLAG_ACCUMULATE if accumulate else 0,
                                             _stream(stream)), "reducescatter")
+        return out
+
+    # ---- zero-copy (multi-process): registered buffers, DIRECT plan over NVLink
+    def register(self, t):
+        """Register tensor t's storage for zero-copy collectives (collective call)."""
+        rid = ctypes.c_int()
+        nbytes = t.numel() * t.element_size()
+        _check(_load().adapcc_register_buffer(self._h, ctypes.c_void_p(t.data_ptr()), nbytes,
+                                              ctypes.byref(rid)), "register_buffer")
+        regs = self.__dict__.setdefault("_regs", {})
+        regs[rid.value] = (t.data_ptr(), nbytes, t)
+        return rid.value
+
+    def deregister(self, rid):
+        _check(_load().adapcc_deregister_buffer(self._h, rid), "deregister_buffer")
+        self.__dict__.get("_regs", {}).pop(rid, None)
+
+    def _reg_of(self, t):
+        for rid, (ptr, nbytes, _) in self.__dict__.get("_regs", {}).items():
+            off = t.data_ptr() - ptr
+            if 0 <= off and off + t.numel() * t.element_size() <= nbytes:
+                return rid, off
+        raise ValueError("tensor is not inside a registered buffer (call comm.register first)")
+
+    def collective_zc(self, coll, x, out, count, root=0, ready=None, accumulate=False, stream=None):
+        """Any collective on registered tensors x / out (same offsets on every rank)."""
+        sr, so = self._reg_of(x)
+        rr, ro = self._reg_of(out)
+        m = _mask(ready, self.nranks)
+        _check(_load().adapcc_collective_zc(self._h, COLL[coll], sr, so, rr, ro, count, _dtype_code(out),
+                                            root, m, FLAG_ACCUMULATE if accumulate else 0,
+                                            _stream(stream)), coll + "_zc")
         return out
 
     # ---- loopback collectives (lists of per-virtual-rank tensors)

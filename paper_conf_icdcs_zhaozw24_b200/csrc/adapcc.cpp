@@ -7,6 +7,7 @@
 // strategy per collective and a cache of compiled plans.  Every collective
 // call is one engine launch per segment on the caller's stream.
 #include <cuda_runtime.h>
+#include <dlfcn.h>
 
 #include <algorithm>
 #include <cstdio>
@@ -61,7 +62,15 @@ struct DevPlan {
   }
 };
 
-using PlanKey = std::tuple<int, uint64_t, uint64_t, int, uint64_t, unsigned>;
+using PlanKey = std::tuple<int, uint64_t, uint64_t, int, uint64_t, unsigned, int>;  // ..., plan mode
+
+// A buffer registered for zero-copy collectives: base[q] is where rank q's
+// registered region starts in THIS process's address space (peer-mapped).
+struct RegBuf {
+  std::vector<char*> base;
+  std::vector<std::string> handle;  // per peer: IPC handle bytes (for close)
+  size_t bytes = 0;
+};
 
 int esize_of(adapcc_dtype_t d) { return d == ADAPCC_BFLOAT16 ? 2 : 4; }
 
@@ -139,6 +148,11 @@ struct adapcc_comm_s {
   int engine = 2;  // 0: LDG/STG fold, 1: TMA bulk pipeline, 2: auto by call size
   int last_engine = -1;  // kernel used by the most recent launch
   std::mutex mu;
+  adapcc_bootstrap_allgather_fn ag = nullptr;  // kept for collective registration
+  void* ag_ctx = nullptr;
+  std::map<int, RegBuf> regs;
+  int next_reg = 0;
+  std::map<std::pair<int, std::string>, std::pair<char*, int>> opened;  // (peer, handle) -> (base, refs)
 };
 
 namespace {
@@ -194,6 +208,8 @@ void release(adapcc_comm_s* c) {
   cudaSetDevice(c->device);
   cudaDeviceSynchronize();
   c->plans.clear();
+  for (auto& o : c->opened) cudaIpcCloseMemHandle(o.second.first);
+  c->opened.clear();
   if (c->loopback) {
     cudaFree(c->own_arena);
   } else {
@@ -262,9 +278,9 @@ adapcc_result_t pick_strategy(adapcc_comm_s* c, Coll coll, int root, const Strat
 }
 
 adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, const Strategy* strat, uint64_t count,
-                         adapcc_dtype_t dtype, uint64_t mask, unsigned flags,
+                         adapcc_dtype_t dtype, uint64_t mask, unsigned flags, Mode mode,
                          std::shared_ptr<DevPlan>* out) {
-  PlanKey key{(int)coll, strat->hash, count, (int)dtype, mask, flags};
+  PlanKey key{(int)coll, strat->hash, count, (int)dtype, mask, flags, (int)mode};
   auto it = c->plans.find(key);
   if (it != c->plans.end()) {
     it->second->last_tick = ++c->tick;
@@ -277,7 +293,7 @@ adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, const Strategy* strat, uin
   rq.esize = esize_of(dtype);
   rq.ready_mask = mask;
   rq.accumulate = flags & ADAPCC_FLAG_ACCUMULATE;
-  rq.mode = c->mode;
+  rq.mode = mode;
   rq.half_bytes = c->half_bytes;
   std::vector<SegmentPlan> segs;
   std::string err;
@@ -323,16 +339,20 @@ adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, const Strategy* strat, uin
   return ADAPCC_SUCCESS;
 }
 
+// zc_send / zc_recv (multi-process zero-copy): every rank's buffer as mapped
+// in this process -> the DIRECT plan runs across processes over NVLink.
 adapcc_result_t run(adapcc_comm_s* c, Coll coll, const void* const* send, void* const* recv,
                     uint64_t count, adapcc_dtype_t dtype, uint64_t mask, unsigned flags,
-                    adapcc_stream_t stream, int root = 0) {
+                    adapcc_stream_t stream, int root = 0, char* const* zc_send = nullptr,
+                    char* const* zc_recv = nullptr) {
+  const bool zc = zc_send != nullptr;
   std::lock_guard<std::mutex> lock(c->mu);
   CK(cudaSetDevice(c->device));
   const Strategy* strat = nullptr;
   adapcc_result_t r = pick_strategy(c, coll, root, &strat);
   if (r != ADAPCC_SUCCESS) return r;
   std::shared_ptr<DevPlan> plan;
-  r = get_plan(c, coll, strat, count, dtype, mask, flags, &plan);
+  r = get_plan(c, coll, strat, count, dtype, mask, flags, zc ? kDirect : c->mode, &plan);
   if (r != ADAPCC_SUCCESS) return r;
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
   cudaStreamCaptureStatus cap = cudaStreamCaptureStatusNone;
@@ -351,13 +371,17 @@ adapcc_result_t run(adapcc_comm_s* c, Coll coll, const void* const* send, void* 
     P.nranks = c->nranks;
     P.my_rank = c->loopback ? -1 : c->rank;
     P.ipc = c->loopback ? 0 : 1;
+    P.zc = zc ? 1 : 0;
     P.drop_rank = (int)c->drop_rank;
     P.half_bytes = c->half_bytes;
     P.timeout_ns = (uint64_t)std::max<int64_t>(1, c->timeout_ms) * 1000000ull;
     P.state = c->state;
     P.err = c->d_err;
     for (int q = 0; q < c->nranks; ++q) {
-      if (c->loopback || q == c->rank) {
+      if (zc) {
+        P.send[q] = zc_send[q];
+        P.recv[q] = zc_recv[q];
+      } else if (c->loopback || q == c->rank) {
         const int i = c->loopback ? q : 0;
         P.send[q] = const_cast<char*>(static_cast<const char*>(send[i]));
         P.recv[q] = static_cast<char*>(recv[i]);
@@ -424,6 +448,8 @@ adapcc_result_t adapcc_init(adapcc_comm_t* comm, int rank, int nranks, int cuda_
   c->device = cuda_device;
   c->loopback = false;
   c->mode = kStaged;
+  c->ag = ag;
+  c->ag_ctx = ag_ctx;
   adapcc_result_t r = common_init(c, scratch_bytes);
   if (r != ADAPCC_SUCCESS) { release(c); return r; }
   c->arena.assign(nranks, nullptr);
@@ -683,6 +709,120 @@ adapcc_result_t adapcc_reducescatter_lb(adapcc_comm_t c, const void* const* send
   r = check_lb(c, sendbufs, recvbufs, rbytes * c->nranks, rbytes, mask, 3);
   if (r != ADAPCC_SUCCESS) return r;
   return run(c, kReduceScatter, sendbufs, recvbufs, recvcount, dtype, mask, flags, stream);
+}
+
+// ------------------------------------------------------- zero-copy registration
+namespace {
+// base address of the allocation containing p (driver API, loaded lazily so
+// the library still loads on machines without a driver)
+bool allocation_base(void* p, char** base) {
+  using Fn = int (*)(unsigned long long*, size_t*, unsigned long long);
+  static Fn fn = [] {
+    void* h = dlopen("libcuda.so.1", RTLD_NOW | RTLD_LOCAL);
+    return h ? reinterpret_cast<Fn>(dlsym(h, "cuMemGetAddressRange_v2")) : nullptr;
+  }();
+  if (!fn) return false;
+  unsigned long long b = 0;
+  size_t sz = 0;
+  if (fn(&b, &sz, reinterpret_cast<unsigned long long>(p)) != 0) return false;
+  *base = reinterpret_cast<char*>(b);
+  return true;
+}
+}  // namespace
+
+adapcc_result_t adapcc_register_buffer(adapcc_comm_t c, void* ptr, size_t bytes, int* reg_id) {
+  if (!c || !ptr || !reg_id || misaligned(ptr)) return ADAPCC_ERR_INVALID_ARGUMENT;
+  if (c->loopback || !c->ag) return ADAPCC_ERR_UNSUPPORTED;
+  std::lock_guard<std::mutex> lock(c->mu);
+  CK(cudaSetDevice(c->device));
+  char* base = nullptr;
+  if (!allocation_base(ptr, &base)) return ADAPCC_ERR_CUDA;
+  struct Blob { cudaIpcMemHandle_t h; uint64_t offset, bytes; int32_t id, pad; };
+  Blob me{};
+  CK(cudaIpcGetMemHandle(&me.h, base));
+  me.offset = static_cast<char*>(ptr) - base;
+  me.bytes = bytes;
+  me.id = c->next_reg;
+  std::vector<Blob> all(c->nranks);
+  if (c->ag(&me, all.data(), sizeof(Blob), c->ag_ctx) != 0) return ADAPCC_ERR_BOOTSTRAP;
+  for (auto& b : all)
+    if (b.bytes != bytes || b.id != me.id) return ADAPCC_ERR_MISMATCH;
+  RegBuf rb;
+  rb.bytes = bytes;
+  rb.base.assign(c->nranks, nullptr);
+  rb.handle.assign(c->nranks, std::string());
+  for (int q = 0; q < c->nranks; ++q) {
+    if (q == c->rank) {
+      rb.base[q] = static_cast<char*>(ptr);
+      continue;
+    }
+    std::string key(reinterpret_cast<const char*>(&all[q].h), sizeof(cudaIpcMemHandle_t));
+    auto it = c->opened.find({q, key});
+    if (it == c->opened.end()) {
+      void* m = nullptr;
+      CK(cudaIpcOpenMemHandle(&m, all[q].h, cudaIpcMemLazyEnablePeerAccess));
+      it = c->opened.emplace(std::make_pair(q, key), std::make_pair(static_cast<char*>(m), 0)).first;
+    }
+    it->second.second += 1;
+    rb.base[q] = it->second.first + all[q].offset;
+    rb.handle[q] = key;
+  }
+  *reg_id = c->next_reg++;
+  c->regs[*reg_id] = std::move(rb);
+  return ADAPCC_SUCCESS;
+}
+
+adapcc_result_t adapcc_deregister_buffer(adapcc_comm_t c, int reg_id) {
+  if (!c) return ADAPCC_ERR_INVALID_ARGUMENT;
+  std::lock_guard<std::mutex> lock(c->mu);
+  auto it = c->regs.find(reg_id);
+  if (it == c->regs.end()) return ADAPCC_ERR_INVALID_ARGUMENT;
+  CK(cudaSetDevice(c->device));
+  CK(cudaDeviceSynchronize());  // no launch may still reference the mapping
+  for (int q = 0; q < c->nranks; ++q) {
+    if (q == c->rank) continue;
+    auto o = c->opened.find({q, it->second.handle[q]});
+    if (o != c->opened.end() && --o->second.second == 0) {
+      cudaIpcCloseMemHandle(o->second.first);
+      c->opened.erase(o);
+    }
+  }
+  c->regs.erase(it);
+  return ADAPCC_SUCCESS;
+}
+
+adapcc_result_t adapcc_collective_zc(adapcc_comm_t c, adapcc_coll_t coll, int send_reg,
+                                     size_t send_offset, int recv_reg, size_t recv_offset, size_t count,
+                                     adapcc_dtype_t dtype, int root, uint64_t mask, unsigned flags,
+                                     adapcc_stream_t stream) {
+  adapcc_result_t r = check_common(c, dtype, mask);
+  if (r != ADAPCC_SUCCESS) return r;
+  if (c->loopback || coll < ADAPCC_ALLREDUCE || coll > ADAPCC_REDUCESCATTER ||
+      (flags & ~ADAPCC_FLAG_ACCUMULATE))
+    return ADAPCC_ERR_INVALID_ARGUMENT;
+  if ((flags & ADAPCC_FLAG_ACCUMULATE) && coll != ADAPCC_ALLREDUCE && coll != ADAPCC_REDUCE &&
+      coll != ADAPCC_REDUCESCATTER)
+    return ADAPCC_ERR_INVALID_ARGUMENT;
+  std::vector<char*> S, D;
+  {
+    std::lock_guard<std::mutex> lock(c->mu);
+    auto si = c->regs.find(send_reg), di = c->regs.find(recv_reg);
+    if (si == c->regs.end() || di == c->regs.end()) return ADAPCC_ERR_INVALID_ARGUMENT;
+    const size_t es = esize_of(dtype), n = c->nranks;
+    size_t sb = count * es, rb = count * es;
+    if (coll == ADAPCC_ALLGATHER) rb *= n;
+    if (coll == ADAPCC_ALLTOALL) { sb *= n; rb *= n; }
+    if (coll == ADAPCC_REDUCESCATTER) sb *= n;
+    if (send_offset + sb > si->second.bytes || recv_offset + rb > di->second.bytes ||
+        (send_offset & 15) || (recv_offset & 15))
+      return ADAPCC_ERR_INVALID_ARGUMENT;
+    for (size_t q = 0; q < n; ++q) {
+      S.push_back(si->second.base[q] + send_offset);
+      D.push_back(di->second.base[q] + recv_offset);
+    }
+    if (coll == ADAPCC_ALLTOALL && overlap(S[c->rank], sb, D[c->rank], rb)) return ADAPCC_ERR_INVALID_ARGUMENT;
+  }
+  return run(c, (Coll)coll, nullptr, nullptr, count, dtype, mask, flags, stream, root, S.data(), D.data());
 }
 
 const char* adapcc_last_cuda_error(void) {

@@ -229,6 +229,13 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
     }
     __syncthreads();
   }
+  if (P.ipc && P.zc) {  // zero-copy: peers read/write our user buffers directly
+    if (blockIdx.x == 0 && threadIdx.x == 0)
+      st_release(reinterpret_cast<uint64_t*>(P.hdr[P.my_rank] + 8), epoch, true);  // entered
+    if (threadIdx.x < P.nranks && threadIdx.x != P.my_rank)
+      if (!wait_flag(reinterpret_cast<const uint64_t*>(P.hdr[threadIdx.x] + 8), epoch, P)) sh.abort = 1;
+    __syncthreads();
+  }
   constexpr int esize = Ops<DT>::kEsize;
   while (!sh.abort) {
     if (threadIdx.x == 0) {
@@ -311,6 +318,9 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
       if (P.ipc) {
         __threadfence_system();
         st_release(reinterpret_cast<uint64_t*>(P.hdr[P.my_rank]), epoch, true);
+        if (P.zc)  // our buffers stay in use until every peer has finished this call
+          for (int q = 0; q < P.nranks; ++q)
+            if (q != P.my_rank) wait_flag(reinterpret_cast<const uint64_t*>(P.hdr[q]), epoch, P);
       }
     }
   }

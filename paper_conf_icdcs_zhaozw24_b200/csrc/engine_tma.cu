@@ -339,6 +339,13 @@ __global__ void __launch_bounds__(kTmaThreads, 2) engine_tma_kernel(const __grid
       if (!wait_flag(reinterpret_cast<const uint64_t*>(P.hdr[tid]), epoch - 2, P)) sm.abort = 1;
     __syncthreads();
   }
+  if (P.ipc && P.zc) {  // zero-copy: peers read/write our user buffers directly
+    if (blockIdx.x == 0 && tid == 0)
+      st_release(reinterpret_cast<uint64_t*>(P.hdr[P.my_rank] + 8), epoch, true);  // entered
+    if (tid < P.nranks && tid != P.my_rank)
+      if (!wait_flag(reinterpret_cast<const uint64_t*>(P.hdr[tid] + 8), epoch, P)) sm.abort = 1;
+    __syncthreads();
+  }
 
   if (warp == kConsumerWarps) {
     // ================================================================ producer
@@ -446,6 +453,9 @@ __global__ void __launch_bounds__(kTmaThreads, 2) engine_tma_kernel(const __grid
       if (P.ipc) {
         __threadfence_system();
         st_release(reinterpret_cast<uint64_t*>(P.hdr[P.my_rank]), epoch, true);
+        if (P.zc)  // our buffers stay in use until every peer has finished this call
+          for (int q = 0; q < P.nranks; ++q)
+            if (q != P.my_rank) wait_flag(reinterpret_cast<const uint64_t*>(P.hdr[q]), epoch, P);
       }
     }
   }

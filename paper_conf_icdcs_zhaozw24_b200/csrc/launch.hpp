@@ -32,6 +32,7 @@ struct LaunchParams {
   int nranks;
   int my_rank;          // multi-process: this rank; loopback: -1
   int ipc;              // 1: multi-process (.sys scope, start check, done publish)
+  int zc;               // 1: zero-copy DIRECT plan across processes (entry/exit barriers)
   int drop_rank;        // test hook (loopback): tasks owned by this rank are skipped
   uint64_t half_bytes;  // bytes of one parity half of an arena
   uint64_t timeout_ns;
