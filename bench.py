@@ -48,6 +48,9 @@ def parse_args():
     p.add_argument("--e2e-steps", type=int, default=5)
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--no-parity", action="store_true")
+    p.add_argument("--test-same-gpu", action="store_true",
+                   help="N>1 code-path check on a 1-GPU box: every rank on cuda:0, gloo, no NCCL leg "
+                        "(numbers are NOT NVLink measurements)")
     return p.parse_args()
 
 
@@ -209,7 +212,7 @@ def workload_config(args, n, world):
         "workload": f"allreduce-{where}{n}-{args.dtype}-{nbytes >> 20}MiB-star{n}",
         "ranks": n, "virtual_ranks": world == 1, "bytes_per_rank": nbytes,
         "strategy": f"{n} star trees (one rooted at each rank), equal weights, chunk {args.chunk_kib} KiB",
-        "mode": args.mode if world == 1 else "staged", "ready_mask": "all",
+        "mode": args.mode if world == 1 else "zero-copy direct (registered buffers)", "ready_mask": "all",
         "l2": f"inputs {n * nbytes >> 20} MiB per step > 126 MB L2 (no flush needed)",
         "parallelism": f"{'virtual ' if world == 1 else ''}dp{n}",
     }
@@ -363,8 +366,13 @@ def run_multi(args):
     from synth import rank_tensors
 
     rank, world, local = dist_env()
-    torch.cuda.set_device(local)
-    dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    if args.test_same_gpu:
+        local = 0
+        torch.cuda.set_device(0)
+        dist.init_process_group("gloo")
+    else:
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     es = 4 if args.dtype == "f32" else 2
     nbytes = int(args.size_mib * (1 << 20)) // 16 * 16
     count = nbytes // es
@@ -393,7 +401,7 @@ def run_multi(args):
             fn()
         b.record(stream)
         torch.cuda.synchronize()
-        t = torch.tensor([a.elapsed_time(b) / steps], device="cuda")
+        t = torch.tensor([a.elapsed_time(b) / steps], device="cpu" if args.test_same_gpu else "cuda")
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         dist.barrier()
         return float(t.item())
@@ -407,7 +415,8 @@ def run_multi(args):
     z = x.clone()
 
     def nccl():
-        dist.all_reduce(z)
+        if not args.test_same_gpu:
+            dist.all_reduce(z)
 
     for _ in range(args.warmup):
         ours()
@@ -434,7 +443,7 @@ def run_multi(args):
         out_h = y.view(xh.dtype).to("cpu", non_blocking=True)
         b.record(stream)
         torch.cuda.synchronize()
-        t = torch.tensor([a.elapsed_time(b)], device="cuda")
+        t = torch.tensor([a.elapsed_time(b)], device="cpu" if args.test_same_gpu else "cuda")
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         if i > 0:
             e2e.append(float(t.item()))
@@ -463,7 +472,7 @@ def run_multi(args):
             "staged": {"value": round(busbw(nbytes, ms_staged / 1e3, world), 3), "unit": UNIT,
                        "ms_per_step": round(ms_staged, 4),
                        "path": "STAGED protocol (landing + broadcast slots in IPC arenas)"},
-            "nccl": {"value": round(busbw(nbytes, ms_nccl / 1e3, world), 3), "unit": UNIT,
+            "nccl": None if args.test_same_gpu else {"value": round(busbw(nbytes, ms_nccl / 1e3, world), 3), "unit": UNIT,
                      "ms_per_step": round(ms_nccl, 4), "version": ".".join(map(str, torch.cuda.nccl.version()))},
         }
     comm.finalize()
