@@ -1,0 +1,147 @@
+"""Relay coordinator: wait-or-proceed decisions and fault marking (NEXT-1 / NEXT-3).
+
+Host-side policy of AdapCC's adaptive relay control (§IV-C):
+
+* Decision cycles: every `cycle` the coordinator either keeps
+  waiting for all workers or starts *phase 1* -- a partial collective among
+  the ready workers, non-ready ones acting as relays -- followed by *phase 2*
+  once the late workers are ready.
+* Ski rental: waiting costs 1 per cycle (here: the cycle's
+  duration); "buying" costs the estimated phase-1 + phase-2 time.  The
+  break-even rule waits "at most until the accumulated waiting cost exceeds
+  the buying cost in a time cycle", which is 2-competitive.  The time of a
+  collective is estimated as S / B: S = 2(N-1) x tensor for
+  AllReduce, N x tensor for AlltoAll, tensor for Broadcast, with N the
+  participating workers; B = aggregate profiled link bandwidth of the graph.
+* Fault tolerance: after phase 1 completes, workers still not ready
+  after T_fault = 5 x (time since the fastest worker became ready) are marked
+  faulty and excluded.
+
+On B200 the cycle is scaled from the paper's 5 ms to the collective's own
+time scale (µs), see DESIGN.md §3 reading R2.  The coordinator is pure host
+logic; it produces the ready masks the engine consumes.
+"""
+
+from dataclasses import dataclass, field
+
+T_FAULT_FACTOR = 5.0
+
+
+def comm_volume(coll, n_participants, tensor_bytes):
+    """S of P:L135 for N participating workers."""
+    if n_participants <= 1:
+        return 0.0
+    if coll == "allreduce":
+        return 2.0 * (n_participants - 1) * tensor_bytes
+    if coll == "alltoall":
+        return float(n_participants) * tensor_bytes
+    if coll == "broadcast":
+        return float(tensor_bytes)
+    raise ValueError(coll)
+
+
+def collective_time(coll, n_participants, tensor_bytes, aggregate_bw):
+    """S / B estimate of one collective; aggregate_bw in bytes/s."""
+    return comm_volume(coll, n_participants, tensor_bytes) / aggregate_bw
+
+
+@dataclass
+class Decision:
+    action: str                 # 'wait' | 'full' | 'phase1'
+    time: float                 # when the decision is taken
+    ready: frozenset = frozenset()
+    relays: frozenset = frozenset()
+
+
+@dataclass
+class Coordinator:
+    """Break-even (ski-rental) coordinator for one collective at a time.
+
+    n            : number of workers
+    coll         : 'allreduce' | 'alltoall' | 'broadcast'
+    tensor_bytes : bytes per worker
+    link_bw      : bandwidth of one link (bytes/s); the aggregate bandwidth
+                   B of a collective among k workers is k * link_bw (every
+                   GPU's NVSwitch port, "accumulating the profiled link
+                   bandwidth in the communication graph")
+    cycle        : decision period (seconds)
+    """
+    n: int
+    coll: str
+    tensor_bytes: float
+    link_bw: float
+    cycle: float
+    waited: float = 0.0
+    history: list = field(default_factory=list)
+
+    def _t(self, k):
+        return collective_time(self.coll, k, self.tensor_bytes, max(k, 1) * self.link_bw)
+
+    def buy_cost(self, ready_count):
+        """Estimated phase 1 (ready workers) + phase 2 (late workers) time."""
+        late = self.n - ready_count
+        phase2 = self._t(late + 1) if late else 0.0   # late data reaches the others
+        return self._t(ready_count) + phase2
+
+    def full_cost(self):
+        return self._t(self.n)
+
+    def step(self, now, ready):
+        """One decision cycle at time `now` with the set of ready workers."""
+        ready = frozenset(ready)
+        if len(ready) == self.n:
+            d = Decision("full", now, ready)
+        elif ready and self.waited + self.cycle > self.buy_cost(len(ready)):
+            # waiting one more cycle would exceed the buying cost: buy (phase 1)
+            d = Decision("phase1", now, ready, frozenset(range(self.n)) - ready)
+        else:
+            self.waited += self.cycle
+            d = Decision("wait", now, ready)
+        self.history.append(d)
+        return d
+
+    def run(self, arrivals, start=0.0):
+        """Drive cycles over known arrival times (simulation / tests).
+
+        arrivals: list of per-worker ready times.  Returns (decision, finish
+        time): phase 1 starts at the decision, phase 2 starts once the last
+        worker is ready and phase 1 is done; a full collective starts when all
+        are ready.  Competitive analysis: finish - first arrival vs OPT."""
+        t = start
+        while True:
+            ready = {r for r, a in enumerate(arrivals) if a <= t}
+            d = self.step(t, ready)
+            if d.action == "full":
+                return d, t + self.full_cost()
+            if d.action == "phase1":
+                p1_end = t + self._t(len(ready))
+                late_end = max(arrivals)
+                p2 = self._t(self.n - len(ready) + 1)
+                return d, max(p1_end, late_end) + p2
+            t += self.cycle
+
+
+def offline_optimum(arrivals, n, coll, tensor_bytes, link_bw, cycle):
+    """OPT: the best decision time in hindsight (any cycle boundary)."""
+    c = Coordinator(n, coll, tensor_bytes, link_bw, cycle)
+    last = max(arrivals)
+    best = last + c.full_cost()  # wait for everyone
+    t = 0.0
+    while t < last:
+        ready = [r for r, a in enumerate(arrivals) if a <= t]
+        if ready:
+            p1_end = t + c._t(len(ready))
+            best = min(best, max(p1_end, last) + c._t(n - len(ready) + 1))
+        t += cycle
+    return best
+
+
+def faulty_workers(ready_times, phase1_end, now, factor=T_FAULT_FACTOR):
+    """after phase 1, workers not ready within T_fault = factor x (time
+    since the fastest worker became ready) are faulty.  ready_times: dict
+    worker -> ready time, or None if not ready yet."""
+    first = min(t for t in ready_times.values() if t is not None)
+    t_fault = factor * (phase1_end - first)
+    if now - phase1_end < t_fault:
+        return set()
+    return {r for r, t in ready_times.items() if t is None}
