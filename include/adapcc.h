@@ -76,6 +76,21 @@ typedef enum { ADAPCC_MODE_DIRECT = 0, ADAPCC_MODE_STAGED = 1 } adapcc_mode_t;
 /* ACCUMULATE: recvbuf += result (one rounding), the paper's phase 2 in which
  * the late ranks' data is combined with the phase-1 result. */
 #define ADAPCC_FLAG_ACCUMULATE 0x1u
+/* Late join (a relay that becomes ready during phase 1 makes
+ * "data chunks with the same offset in the buffer join the ongoing aggregation
+ * process. Then in phase 2, only partial data chunks from relay workers that
+ * have not been aggregated need to be broadcast").  AllReduce on a DIRECT plan
+ * (loopback DIRECT or adapcc_collective_zc) only; not combinable with
+ * ACCUMULATE.
+ *   LATE_JOIN (phase 1, mask R): every tree root also folds, per work piece,
+ *     the inputs of the non-ready ranks whose ready word already holds this
+ *     call's ticket (appended after the regular sources, ascending rank), and
+ *     records which ones it folded.
+ *   LATE_COMPLEMENT (phase 2, SAME mask R and buffers as phase 1): recvbuf +=
+ *     sum of the non-ready ranks' inputs that phase 1 did not fold, per piece.
+ * After both phases every rank holds the sum over all ranks. */
+#define ADAPCC_FLAG_LATE_JOIN 0x2u
+#define ADAPCC_FLAG_LATE_COMPLEMENT 0x4u
 
 /* Bootstrap all-gather the caller implements (Python: torch.distributed
  * all_gather on the process group).  Gathers bytes_per_rank from every rank
@@ -212,6 +227,15 @@ ADAPCC_API adapcc_result_t adapcc_collective_zc(adapcc_comm_t comm, adapcc_coll_
                                                 size_t count, adapcc_dtype_t dtype, int root,
                                                 uint64_t ready_mask, unsigned flags,
                                                 adapcc_stream_t stream);
+
+/* Ticket of the most recent LATE_JOIN call (0 before the first). */
+ADAPCC_API adapcc_result_t adapcc_late_ticket(adapcc_comm_t comm, uint64_t* ticket);
+/* Mark `rank` ready for late join: after all prior work on `stream` (e.g. the
+ * rank's gradient computation) its ready word becomes `ticket` (0 = the
+ * current ticket).  Multi-process: rank must be this rank (or -1);
+ * loopback: any virtual rank. */
+ADAPCC_API adapcc_result_t adapcc_signal_ready(adapcc_comm_t comm, int rank, uint64_t ticket,
+                                               adapcc_stream_t stream);
 
 /* ------------------------------------------------------------- lifecycle --- */
 

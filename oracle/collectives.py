@@ -276,3 +276,84 @@ def reducescatter(xs, strategy_text, ready, dtype, accumulate=False, y_prev=None
                 y[lo:hi] = res if res is not None else _zero(hi - lo, dtype)
         ys.append(y)
     return ys
+
+
+# --------------------------------------------------------- NEXT-1: late join
+def _root_terms(vals, sub, ready, dtype):
+    """The values a tree's root folds (kernel root: own tensor if ready, then the
+    sending children's flows; non-kernel root: its single flow, or nothing),
+    with every non-root kernel node's aggregate computed as in _tree_result."""
+    tup, flows = behavior(sub.parent, ready, sub.noagg)
+    agg_val = {}
+
+    def value(f):
+        kind, r = f
+        return vals[r] if kind == "in" else agg_val[r]
+
+    order = []
+
+    def visit(g):
+        for c in sub.children(g):
+            visit(c)
+        order.append(g)
+
+    visit(sub.root)
+    root = sub.root
+    for g in order:
+        if tup[g][2] and g != root:
+            terms = [vals[g]] if tup[g][0] else []
+            for c in sub.children(g):
+                if tup[c][3]:
+                    terms += [value(f) for f in flows[c]]
+            agg_val[g] = _fold(terms, dtype)
+    if tup[root][2]:
+        terms = [vals[root]] if tup[root][0] else []
+        for c in sub.children(root):
+            if tup[c][3]:
+                terms += [value(f) for f in flows[c]]
+        return terms
+    return [value(f) for f in flows[root]]
+
+
+def allreduce_late(xs, strategy_text, ready, dtype, included, phase=1, y_prev=None):
+    """Late join with a uniform inclusion set.
+
+    phase 1: every tree's root folds its regular terms followed by the inputs
+             of the late ranks in ``included`` (ascending rank): one rounding;
+             a single term without late inputs is copied unchanged; no term -> +0.
+    phase 2: y_prev + fold(inputs of the late ranks NOT in ``included``,
+             ascending), one rounding for the sum and one for the addition
+             (the ACCUMULATE rule); nothing left -> y_prev unchanged.
+    Late ranks = ranks not in ``ready``; ``included`` must be a subset."""
+    st = parse(strategy_text)
+    n = st.nranks
+    ready = set(ready)
+    late = sorted(set(range(n)) - ready)
+    included = sorted(set(included))
+    assert set(included) <= set(late)
+    lens = {len(x) for x in xs if x is not None}
+    count = lens.pop()
+    bounds = partition(count, ESIZE[dtype], [s.weight for s in st.subs])
+    if phase == 2:
+        rest = [r for r in late if r not in included]
+        ys = [np.array(y, copy=True) for y in y_prev]
+        if not rest:
+            return ys
+        add = xs[rest[0]].copy() if len(rest) == 1 else _fold([xs[r] for r in rest], dtype)
+        return [_accumulate(y, add, dtype) for y in ys]
+    ys = [np.empty(count, dtype=_NP[dtype]) for _ in range(n)]
+    for m, sub in enumerate(st.subs):
+        lo, hi = bounds[m], bounds[m + 1]
+        if lo == hi:
+            continue
+        vals = [x[lo:hi] if x is not None else None for x in xs]
+        terms = _root_terms(vals, sub, ready, dtype) + [xs[r][lo:hi] for r in included]
+        if not terms:
+            res = _zero(hi - lo, dtype)
+        elif len(terms) == 1:
+            res = np.array(terms[0], copy=True)
+        else:
+            res = _fold(terms, dtype)
+        for g in range(n):
+            ys[g][lo:hi] = res
+    return ys

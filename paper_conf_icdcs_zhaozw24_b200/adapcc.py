@@ -29,6 +29,8 @@ COLL = {"allreduce": 0, "allgather": 1, "alltoall": 2, "reduce": 3, "broadcast":
         "reducescatter": 5}
 MODE = {"direct": 0, "staged": 1}
 FLAG_ACCUMULATE = 0x1
+FLAG_LATE_JOIN = 0x2
+FLAG_LATE_COMPLEMENT = 0x4
 DTYPE_CODE = {"f32": 0, "bf16": 1, "i32": 2}
 
 _lib = None
@@ -85,6 +87,8 @@ def _load():
         "adapcc_register_buffer": [vp, vp, sz, ctypes.POINTER(i32)],
         "adapcc_deregister_buffer": [vp, i32],
         "adapcc_collective_zc": [vp, i32, i32, sz, i32, sz, sz, i32, i32, u64, ctypes.c_uint, vp],
+        "adapcc_late_ticket": [vp, ctypes.POINTER(u64)],
+        "adapcc_signal_ready": [vp, i32, u64, vp],
         "adapcc_get_async_error": [vp],
         "adapcc_finalize": [vp],
         "adapcc_config": [vp, ctypes.c_char_p, i64],
@@ -151,6 +155,10 @@ def _stream(stream):
     import torch
     s = stream if stream is not None else torch.cuda.current_stream()
     return ctypes.c_void_p(s.cuda_stream)
+
+
+def _late_flag(late):
+    return {None: 0, "join": FLAG_LATE_JOIN, "complement": FLAG_LATE_COMPLEMENT}[late]
 
 
 def _ptr(t):
@@ -375,14 +383,15 @@ class Communicator:
                 return rid, off
         raise ValueError("tensor is not inside a registered buffer (call comm.register first)")
 
-    def collective_zc(self, coll, x, out, count, root=0, ready=None, accumulate=False, stream=None):
+    def collective_zc(self, coll, x, out, count, root=0, ready=None, accumulate=False, stream=None,
+                      late=None):
         """Any collective on registered tensors x / out (same offsets on every rank)."""
         sr, so = self._reg_of(x)
         rr, ro = self._reg_of(out)
         m = _mask(ready, self.nranks)
+        flags = (FLAG_ACCUMULATE if accumulate else 0) | _late_flag(late)
         _check(_load().adapcc_collective_zc(self._h, COLL[coll], sr, so, rr, ro, count, _dtype_code(out),
-                                            root, m, FLAG_ACCUMULATE if accumulate else 0,
-                                            _stream(stream)), coll + "_zc")
+                                            root, m, flags, _stream(stream)), coll + "_zc")
         return out
 
     # ---- loopback collectives (lists of per-virtual-rank tensors)
@@ -399,13 +408,27 @@ class Communicator:
         self._arr_cache = (skey, dkey, S, D)
         return S, D
 
-    def allreduce_lb(self, xs, outs, ready=None, accumulate=False, stream=None):
+    def allreduce_lb(self, xs, outs, ready=None, accumulate=False, stream=None, late=None):
+        """late: None | 'join' (phase 1) | 'complement' (phase 2)."""
         m = _mask(ready, self.nranks)
-        S, D = self._arrays(xs, outs, m)
+        if late is not None:
+            # phase 2 reads the late ranks' inputs: pass every input
+            S, D = self._arrays(xs, outs, (1 << self.nranks) - 1)
+        else:
+            S, D = self._arrays(xs, outs, m)
+        flags = (FLAG_ACCUMULATE if accumulate else 0) | _late_flag(late)
         _check(_load().adapcc_allreduce_lb(self._h, S, D, outs[0].numel(), _dtype_code(outs[0]), m,
-                                           FLAG_ACCUMULATE if accumulate else 0, _stream(stream)),
-               "allreduce_lb")
+                                           flags, _stream(stream)), "allreduce_lb")
         return outs
+
+    def late_ticket(self):
+        v = ctypes.c_uint64()
+        _check(_load().adapcc_late_ticket(self._h, ctypes.byref(v)), "late_ticket")
+        return v.value
+
+    def signal_ready(self, rank=-1, ticket=0, stream=None):
+        """Mark `rank` ready for late join after the work already on `stream`."""
+        _check(_load().adapcc_signal_ready(self._h, rank, ticket, _stream(stream)), "signal_ready")
 
     def allgather_lb(self, xs, outs, ready=None, stream=None):
         m = _mask(ready, self.nranks)

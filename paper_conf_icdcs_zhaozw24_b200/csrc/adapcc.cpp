@@ -39,6 +39,7 @@ struct DevSegment {
   FlagRef* flags = nullptr;
   Item* items = nullptr;
   uint32_t nitems = 0;
+  uint64_t* late_bits = nullptr;  // per item: late ranks folded in phase 1 (late join)
 };
 
 struct DevPlan {
@@ -47,6 +48,7 @@ struct DevPlan {
   cudaEvent_t last_use = nullptr;
   uint64_t last_tick = 0;
   bool pinned = false;  // referenced by a captured CUDA graph: never evicted
+  bool joined = false;  // a LATE_JOIN call recorded late_bits (phase 2 may follow)
   ~DevPlan() {
     if (last_use) {
       cudaEventSynchronize(last_use);
@@ -57,6 +59,7 @@ struct DevPlan {
       cudaFree(s.refs);
       cudaFree(s.flags);
       cudaFree(s.items);
+      cudaFree(s.late_bits);
     }
     cudaGetLastError();  // teardown errors must not leak into a later call's check
   }
@@ -141,6 +144,7 @@ struct adapcc_comm_s {
   int64_t timeout_ms = 10000;
   int64_t max_ctas = 0;
   int64_t drop_rank = -1;
+  uint64_t late_seq = 0;  // late-join ticket of the most recent LATE_JOIN call
   int64_t piece_kib = 0;  // 0 = automatic (total traffic / (8 * grid))
   uint64_t launches = 0;
   int num_sms = 148;
@@ -235,6 +239,19 @@ adapcc_result_t check_common(adapcc_comm_t c, adapcc_dtype_t dtype, uint64_t mas
 
 bool misaligned(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15) != 0; }
 
+// ACCUMULATE, or one of LATE_JOIN / LATE_COMPLEMENT (AllReduce on a DIRECT
+// plan only: the root must be able to read a late rank's input directly).
+adapcc_result_t check_late_flags(adapcc_comm_s* c, unsigned flags, bool late_ok) {
+  (void)c;
+  const unsigned late = flags & (ADAPCC_FLAG_LATE_JOIN | ADAPCC_FLAG_LATE_COMPLEMENT);
+  if (flags & ~(ADAPCC_FLAG_ACCUMULATE | ADAPCC_FLAG_LATE_JOIN | ADAPCC_FLAG_LATE_COMPLEMENT))
+    return ADAPCC_ERR_INVALID_ARGUMENT;
+  if (late && ((flags & ADAPCC_FLAG_ACCUMULATE) || late == (ADAPCC_FLAG_LATE_JOIN | ADAPCC_FLAG_LATE_COMPLEMENT)))
+    return ADAPCC_ERR_INVALID_ARGUMENT;
+  if (late && !late_ok) return ADAPCC_ERR_UNSUPPORTED;
+  return ADAPCC_SUCCESS;
+}
+
 bool overlap(const void* a, size_t an, const void* b, size_t bn) {
   auto x = reinterpret_cast<uintptr_t>(a), y = reinterpret_cast<uintptr_t>(b);
   return x < y + bn && y < x + an;
@@ -280,6 +297,8 @@ adapcc_result_t pick_strategy(adapcc_comm_s* c, Coll coll, int root, const Strat
 adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, const Strategy* strat, uint64_t count,
                          adapcc_dtype_t dtype, uint64_t mask, unsigned flags, Mode mode,
                          std::shared_ptr<DevPlan>* out) {
+  // phase 2 of a late join runs on the phase-1 plan (same items, recorded bits)
+  if (flags & ADAPCC_FLAG_LATE_COMPLEMENT) flags = ADAPCC_FLAG_LATE_JOIN;
   PlanKey key{(int)coll, strat->hash, count, (int)dtype, mask, flags, (int)mode};
   auto it = c->plans.find(key);
   if (it != c->plans.end()) {
@@ -293,6 +312,7 @@ adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, const Strategy* strat, uin
   rq.esize = esize_of(dtype);
   rq.ready_mask = mask;
   rq.accumulate = flags & ADAPCC_FLAG_ACCUMULATE;
+  rq.late_join = flags & ADAPCC_FLAG_LATE_JOIN;
   rq.mode = mode;
   rq.half_bytes = c->half_bytes;
   std::vector<SegmentPlan> segs;
@@ -322,6 +342,10 @@ adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, const Strategy* strat, uin
     CK(up(&d.refs, sp.refs));
     CK(up(&d.flags, sp.flags));
     CK(up(&d.items, items));
+    if (rq.late_join) {
+      CK(cudaMalloc(&d.late_bits, std::max<size_t>(1, items.size()) * sizeof(uint64_t)));
+      CK(cudaMemset(d.late_bits, 0, std::max<size_t>(1, items.size()) * sizeof(uint64_t)));
+    }
     plan->segs.push_back(d);
   }
   // in loopback an empty call launches nothing; in multi-process mode every
@@ -359,6 +383,12 @@ adapcc_result_t run(adapcc_comm_s* c, Coll coll, const void* const* send, void* 
   CK(cudaStreamIsCapturing(s, &cap));
   const bool capturing = cap != cudaStreamCaptureStatusNone;
   if (capturing) plan->pinned = true;  // the graph keeps pointing at these tables
+  const int late_mode = (flags & ADAPCC_FLAG_LATE_JOIN) ? 1 : (flags & ADAPCC_FLAG_LATE_COMPLEMENT) ? 2 : 0;
+  if (late_mode == 2 && !plan->joined) return ADAPCC_ERR_INVALID_ARGUMENT;  // no phase 1 recorded
+  if (late_mode == 1) {
+    plan->joined = true;
+    ++c->late_seq;  // ticket of this phase 1: late ranks signal it (adapcc_signal_ready)
+  }
   for (const DevSegment& seg : plan->segs) {
     if (c->loopback && seg.nitems == 0) continue;
     LaunchParams P{};
@@ -372,6 +402,9 @@ adapcc_result_t run(adapcc_comm_s* c, Coll coll, const void* const* send, void* 
     P.my_rank = c->loopback ? -1 : c->rank;
     P.ipc = c->loopback ? 0 : 1;
     P.zc = zc ? 1 : 0;
+    P.late_mode = late_mode;
+    P.late_ticket = c->late_seq;
+    P.late_bits = seg.late_bits;
     P.drop_rank = (int)c->drop_rank;
     P.half_bytes = c->half_bytes;
     P.timeout_ns = (uint64_t)std::max<int64_t>(1, c->timeout_ms) * 1000000ull;
@@ -581,9 +614,13 @@ adapcc_result_t adapcc_allreduce_lb(adapcc_comm_t c, const void* const* sendbufs
                                     uint64_t mask, unsigned flags, adapcc_stream_t stream) {
   adapcc_result_t r = check_common(c, dtype, mask);
   if (r != ADAPCC_SUCCESS) return r;
-  if (flags & ~ADAPCC_FLAG_ACCUMULATE) return ADAPCC_ERR_INVALID_ARGUMENT;
+  r = check_late_flags(c, flags, c->mode == kDirect);
+  if (r != ADAPCC_SUCCESS) return r;
   const size_t bytes = count * esize_of(dtype);
-  r = check_lb(c, sendbufs, recvbufs, bytes, bytes, mask, 0);
+  // late join reads the non-ready ranks' inputs too: check every sendbuf
+  const uint64_t all = c->nranks >= 64 ? ~0ull : ((1ull << c->nranks) - 1);
+  const bool late = flags & (ADAPCC_FLAG_LATE_JOIN | ADAPCC_FLAG_LATE_COMPLEMENT);
+  r = check_lb(c, sendbufs, recvbufs, bytes, bytes, late ? all : mask, 0);
   if (r != ADAPCC_SUCCESS) return r;
   return run(c, kAllReduce, sendbufs, recvbufs, count, dtype, mask, flags, stream);
 }
@@ -797,9 +834,10 @@ adapcc_result_t adapcc_collective_zc(adapcc_comm_t c, adapcc_coll_t coll, int se
                                      adapcc_stream_t stream) {
   adapcc_result_t r = check_common(c, dtype, mask);
   if (r != ADAPCC_SUCCESS) return r;
-  if (c->loopback || coll < ADAPCC_ALLREDUCE || coll > ADAPCC_REDUCESCATTER ||
-      (flags & ~ADAPCC_FLAG_ACCUMULATE))
+  if (c->loopback || coll < ADAPCC_ALLREDUCE || coll > ADAPCC_REDUCESCATTER)
     return ADAPCC_ERR_INVALID_ARGUMENT;
+  r = check_late_flags(c, flags, coll == ADAPCC_ALLREDUCE);
+  if (r != ADAPCC_SUCCESS) return r;
   if ((flags & ADAPCC_FLAG_ACCUMULATE) && coll != ADAPCC_ALLREDUCE && coll != ADAPCC_REDUCE &&
       coll != ADAPCC_REDUCESCATTER)
     return ADAPCC_ERR_INVALID_ARGUMENT;
@@ -823,6 +861,24 @@ adapcc_result_t adapcc_collective_zc(adapcc_comm_t c, adapcc_coll_t coll, int se
     if (coll == ADAPCC_ALLTOALL && overlap(S[c->rank], sb, D[c->rank], rb)) return ADAPCC_ERR_INVALID_ARGUMENT;
   }
   return run(c, (Coll)coll, nullptr, nullptr, count, dtype, mask, flags, stream, root, S.data(), D.data());
+}
+
+// ------------------------------------------------------------ late join (NEXT-1)
+adapcc_result_t adapcc_late_ticket(adapcc_comm_t c, uint64_t* ticket) {
+  if (!c || !ticket) return ADAPCC_ERR_INVALID_ARGUMENT;
+  *ticket = c->late_seq;
+  return ADAPCC_SUCCESS;
+}
+
+adapcc_result_t adapcc_signal_ready(adapcc_comm_t c, int rank, uint64_t ticket, adapcc_stream_t stream) {
+  if (!c) return ADAPCC_ERR_INVALID_ARGUMENT;
+  if (rank < 0) rank = c->rank;
+  if (rank >= c->nranks || (!c->loopback && rank != c->rank)) return ADAPCC_ERR_INVALID_ARGUMENT;
+  if (ticket == 0) ticket = c->late_seq;
+  CK(cudaSetDevice(c->device));
+  CK(engine_signal(reinterpret_cast<uint64_t*>(c->arena[rank] + 16), ticket, !c->loopback,
+                   reinterpret_cast<cudaStream_t>(stream)));
+  return ADAPCC_SUCCESS;
 }
 
 const char* adapcc_last_cuda_error(void) {

@@ -46,9 +46,11 @@ constexpr int kThreads = 256;
 
 struct Cur {  // header of the work item being executed (staged by thread 0)
   uint64_t e0;
+  uint64_t late;            // late-join sources of this piece (bit j: late ref j)
   uint32_t ref0, flag0, chunk, len;
   uint16_t nsrc, ndst, nwait, npost, op;
-  bool dropped;
+  uint16_t tnsrc, nreg;     // task's own source count; regular sources used
+  bool dropped, force_acc;
 };
 
 struct Shared {
@@ -249,12 +251,33 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
         const Item item = P.items[it];
         const Task& t = P.tasks[item.task];
         Cur& c = sh.cur;
-        c.nsrc = t.nsrc;
+        c.tnsrc = t.nsrc;
+        c.nreg = t.nsrc;
         c.ndst = t.ndst;
         c.nwait = t.nwait;
         c.npost = t.npost;
         c.op = t.op;
         c.dropped = (int)t.owner == P.drop_rank;
+        c.late = 0;
+        c.force_acc = false;
+        if (P.late_mode && !c.dropped) {
+          if (t.nlate == 0) {
+            c.dropped = P.late_mode == 2;  // phase 2 only runs the roots' folds
+          } else {
+            const uint64_t m = late_select(P, t, it);
+            c.late = m;
+            if (P.late_mode == 2) {  // recv += sum of the late ranks not yet included
+              c.nreg = 0;
+              c.nwait = 0;
+              c.op = kOpFold;
+              c.force_acc = true;
+              c.dropped = m == 0;
+            } else if (m && t.op == kOpZero) {
+              c.op = kOpFold;
+            }
+          }
+        }
+        c.nsrc = (uint16_t)(c.nreg + __popcll(c.late));
         c.ref0 = t.ref0;
         c.flag0 = t.flag0;
         c.chunk = item.chunk;
@@ -276,7 +299,10 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
       }
       // resolve stream pointers for this piece
       if (threadIdx.x < nsrc + ndst) {
-        const BufRef r = P.refs[sh.cur.ref0 + threadIdx.x];
+        const int i = threadIdx.x;
+        const BufRef r = i < sh.cur.nreg ? P.refs[sh.cur.ref0 + i]
+                       : i < nsrc ? P.refs[sh.cur.ref0 + sh.cur.tnsrc + ndst + nth_bit(sh.cur.late, i - sh.cur.nreg)]
+                                  : P.refs[sh.cur.ref0 + sh.cur.tnsrc + (i - nsrc)];
         char* base = r.kind == kBufSend ? P.send[r.rank]
                    : r.kind == kBufRecv ? P.recv[r.rank] : P.hdr[r.rank] + half_off;
         char* p = base + r.bias + (int64_t)(sh.cur.e0 * esize);
@@ -285,8 +311,9 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
           sh.src[threadIdx.x] = p;
         } else {
           sh.dst[threadIdx.x - nsrc] = p;
-          sh.acc[threadIdx.x - nsrc] = r.accum;
-          if (r.accum) atomicOr(&sh.any_acc, 1);
+          const bool acc = r.accum || sh.cur.force_acc;
+          sh.acc[threadIdx.x - nsrc] = acc;
+          if (acc) atomicOr(&sh.any_acc, 1);
         }
       }
     }
@@ -336,6 +363,19 @@ cudaError_t engine_occupancy(int dtype, int* blocks_per_sm) {
     case kBF16: return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, engine_kernel<kBF16>, kThreads, 0);
     default: return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, engine_kernel<kI32>, kThreads, 0);
   }
+}
+
+namespace {
+__global__ void signal_kernel(uint64_t* word, uint64_t value, int sys) {
+  fence(sys);
+  st_release(word, value, sys);
+}
+}  // namespace
+
+cudaError_t engine_signal(uint64_t* word, uint64_t value, bool sys, cudaStream_t stream) {
+  cudaGetLastError();
+  signal_kernel<<<1, 1, 0, stream>>>(word, value, sys ? 1 : 0);
+  return cudaGetLastError();
 }
 
 cudaError_t engine_launch(const LaunchParams& p, int grid, cudaStream_t stream) {

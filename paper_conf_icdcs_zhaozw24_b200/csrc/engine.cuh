@@ -53,6 +53,8 @@ struct Task {
   uint32_t level;
   uint16_t op;
   uint16_t owner;           // executing rank
+  uint16_t nlate;           // late-join candidates: refs[ref0+nsrc+ndst .. +nlate) (root tasks)
+  uint16_t pad0;
 };
 
 // A work item covers elements [off, off+len) of chunk `chunk` of `task`.  A

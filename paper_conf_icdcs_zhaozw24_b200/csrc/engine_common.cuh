@@ -137,5 +137,37 @@ static __device__ __noinline__ bool wait_flag(const uint64_t* flag, uint64_t tar
 }
 
 
+// Late join ("data chunks with the same offset ... join the ongoing
+// aggregation"): which of a root task's nlate candidate ranks take part in
+// work item `item`.  Mode 1 (phase 1): candidates whose ready word
+// (arena header + 16) reached the call's ticket, recorded in late_bits[item];
+// mode 2 (phase 2): the candidates NOT recorded (only they remain to add).
+static __device__ __forceinline__ uint64_t late_select(const LaunchParams& P, const Task& t,
+                                                       uint32_t item) {
+  uint64_t m = 0;
+  if (P.late_mode == 1) {
+    for (int j = 0; j < t.nlate; ++j) {
+      const BufRef r = P.refs[t.ref0 + t.nsrc + t.ndst + j];
+      if (ld_acquire(reinterpret_cast<const uint64_t*>(P.hdr[r.rank] + 16), P.ipc) >= P.late_ticket)
+        m |= 1ull << j;
+    }
+    P.late_bits[item] = m;
+  } else if (P.late_mode == 2) {
+    const uint64_t all = t.nlate >= 64 ? ~0ull : ((1ull << t.nlate) - 1);
+    m = all & ~P.late_bits[item];
+  }
+  return m;
+}
+
+// index (into the task's late refs) of the k-th set bit of m
+static __device__ __forceinline__ int nth_bit(uint64_t m, int k) {
+  for (int j = 0; j < 64; ++j)
+    if ((m >> j) & 1) {
+      if (k == 0) return j;
+      --k;
+    }
+  return 0;
+}
+
 }  // namespace dev
 }  // namespace adapcc

@@ -259,21 +259,47 @@ __device__ __forceinline__ void consume_fold(Smem& sm, char* stages, const ItemD
 // ------------------------------------------------------------- producer
 template <int DT>
 __device__ __forceinline__ void fill_desc(const LaunchParams& P, ItemDesc& d, const Item& item,
-                                          const Task& t, uint64_t half_off, int lane) {
+                                          const Task& t, uint64_t half_off, int lane, uint32_t it,
+                                          int* nwait_eff) {
   constexpr int esize = Ops<DT>::kEsize;
   const uint64_t e0 = t.lo + (uint64_t)item.chunk * t.chunk_elems + item.off;
+  // late join (phase 1) / complement (phase 2): which candidate ranks are folded
+  uint64_t late = 0;
+  bool dropped = (int)t.owner == P.drop_rank, force_acc = false;
+  int nreg = t.nsrc, op = t.op;
+  *nwait_eff = t.nwait;
+  if (P.late_mode && !dropped) {
+    if (t.nlate == 0) {
+      dropped = P.late_mode == 2;  // phase 2 only runs the roots' folds
+    } else {
+      if (lane == 0) late = late_select(P, t, it);
+      late = __shfl_sync(0xffffffffu, late, 0);
+      if (P.late_mode == 2) {
+        nreg = 0;
+        *nwait_eff = 0;
+        op = kOpFold;
+        force_acc = true;
+        dropped = late == 0;
+      } else if (late && t.op == kOpZero) {
+        op = kOpFold;
+      }
+    }
+  }
+  const int nsrc = nreg + __popcll(late);
   int misaligned = 0;
-  for (int i = lane; i < t.nsrc + t.ndst; i += 32) {
-    const BufRef r = P.refs[t.ref0 + i];
+  for (int i = lane; i < nsrc + t.ndst; i += 32) {
+    const BufRef r = i < nreg ? P.refs[t.ref0 + i]
+                   : i < nsrc ? P.refs[t.ref0 + t.nsrc + t.ndst + nth_bit(late, i - nreg)]
+                              : P.refs[t.ref0 + t.nsrc + (i - nsrc)];
     char* base = r.kind == kBufSend ? P.send[r.rank] : r.kind == kBufRecv ? P.recv[r.rank]
                                                                          : P.hdr[r.rank] + half_off;
     char* p = base + r.bias + (int64_t)(e0 * esize);
     misaligned |= (reinterpret_cast<uintptr_t>(p) & 15) != 0;
-    if (i < t.nsrc) {
+    if (i < nsrc) {
       d.src[i] = p;
     } else {
-      d.dst[i - t.nsrc] = p;
-      d.acc[i - t.nsrc] = r.accum;
+      d.dst[i - nsrc] = p;
+      d.acc[i - nsrc] = r.accum || force_acc;
     }
   }
   for (int i = lane; i < t.npost; i += 32) {
@@ -283,21 +309,21 @@ __device__ __forceinline__ void fill_desc(const LaunchParams& P, ItemDesc& d, co
   misaligned = __any_sync(0xffffffffu, misaligned);
   __syncwarp();
   if (lane == 0) {
-    d.nsrc = t.nsrc;
+    d.nsrc = (uint16_t)nsrc;
     d.ndst = t.ndst;
-    d.op = t.op;
+    d.op = (uint16_t)op;
     d.npost = t.npost;
     d.len = item.len;
-    d.dropped = (int)t.owner == P.drop_rank;
+    d.dropped = dropped;
     int any_acc = 0;
     for (int k = 0; k < t.ndst; ++k) any_acc |= d.acc[k];
     d.any_acc = any_acc;
     const uint64_t bytes = (uint64_t)item.len * esize;
-    d.scalar_only = misaligned || t.op != kOpFold || bytes < 16;
+    d.scalar_only = misaligned || op != kOpFold || bytes < 16;
     d.vec_bytes = d.scalar_only ? 0 : (uint32_t)(bytes & ~uint64_t(15));
-    const int ks = t.nsrc < kMaxKS ? t.nsrc : kMaxKS;
+    const int ks = nsrc < kMaxKS ? (nsrc > 0 ? nsrc : 1) : kMaxKS;
     d.ks = (uint16_t)ks;
-    d.passes = (uint16_t)((t.nsrc + kMaxKS - 1) / kMaxKS);
+    d.passes = (uint16_t)((nsrc + kMaxKS - 1) / kMaxKS);
     uint32_t tile = kStageBytes / (uint32_t)ks / 4096u * 4096u;
     d.tile = tile;
     d.ntiles = d.vec_bytes ? (d.vec_bytes + tile - 1) / tile : 0;
@@ -364,11 +390,12 @@ __global__ void __launch_bounds__(kTmaThreads, 2) engine_tma_kernel(const __grid
       const Item item = stop ? Item{} : P.items[it];
       const Task& t = P.tasks[item.task];
       if (!stop) {
-        fill_desc<DT>(P, d, item, t, half_off, lane);
+        int nwait = 0;
+        fill_desc<DT>(P, d, item, t, half_off, lane, it, &nwait);
         __syncwarp();
         if (!d.dropped) {
           int ok = 1;
-          for (int i = lane; i < t.nwait; i += 32) {
+          for (int i = lane; i < nwait; i += 32) {
             const FlagRef f = P.flags[t.flag0 + i];
             const uint64_t* fl = reinterpret_cast<const uint64_t*>(P.hdr[f.rank] + half_off + f.off) + item.chunk;
             ok &= wait_flag(fl, epoch, P);

@@ -33,6 +33,9 @@ struct LaunchParams {
   int my_rank;          // multi-process: this rank; loopback: -1
   int ipc;              // 1: multi-process (.sys scope, start check, done publish)
   int zc;               // 1: zero-copy DIRECT plan across processes (entry/exit barriers)
+  int late_mode;        // 0: off; 1: late join (phase 1); 2: complement (phase 2)
+  uint64_t late_ticket; // ready word value that admits a late rank (phase 1)
+  uint64_t* late_bits;  // per work item: late candidates included in phase 1
   int drop_rank;        // test hook (loopback): tasks owned by this rank are skipped
   uint64_t half_bytes;  // bytes of one parity half of an arena
   uint64_t timeout_ns;
@@ -47,6 +50,8 @@ struct LaunchParams {
 int engine_threads();
 cudaError_t engine_occupancy(int dtype, int* blocks_per_sm);
 cudaError_t engine_launch(const LaunchParams& p, int grid, cudaStream_t stream);
+// store `value` into a ready word after all prior work on `stream` (late join)
+cudaError_t engine_signal(uint64_t* word, uint64_t value, bool sys, cudaStream_t stream);
 // engine_tma.cu: TMA bulk-copy pipeline (1 producer + 8 consumer warps, 2 CTAs/SM)
 int engine_tma_threads();
 cudaError_t engine_tma_occupancy(int dtype, int* blocks_per_sm);

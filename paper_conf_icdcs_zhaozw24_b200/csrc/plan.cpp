@@ -84,7 +84,7 @@ class Builder {
 
   int add(int owner, uint64_t lo, uint64_t hi, uint32_t ce, uint16_t op,
           const std::vector<Stream>& srcs, const std::vector<BufRef>& dsts,
-          const std::vector<FlagRef>& posts) {
+          const std::vector<FlagRef>& posts, const std::vector<BufRef>& late = {}) {
     Task t{};
     t.lo = lo;
     t.hi = hi;
@@ -97,6 +97,8 @@ class Builder {
     t.ref0 = (uint32_t)p_.refs.size();
     for (auto& s : srcs) p_.refs.push_back(s.ref);
     for (auto& d : dsts) p_.refs.push_back(d);
+    for (auto& l : late) p_.refs.push_back(l);
+    t.nlate = (uint16_t)late.size();
     t.flag0 = (uint32_t)p_.flags.size();
     uint32_t level = 0;
     uint16_t nwait = 0;
@@ -144,7 +146,8 @@ std::vector<int> bfs_order(const SubColl& s) {
 // (ReduceScatter block b); root_only: the result goes to the root's recvbuf
 // only (Reduce, ReduceScatter) instead of every rank (AllReduce).
 void plan_allreduce_tree(Builder& B, const SubColl& s, uint64_t lo, uint64_t hi, uint64_t mask,
-                         bool accumulate, Mode mode, int64_t send_bias = 0, bool root_only = false) {
+                         bool accumulate, Mode mode, int64_t send_bias = 0, bool root_only = false,
+                         bool late_join = false) {
   const int n = B.n_;
   const int es = B.esize_;
   const uint32_t ce = (uint32_t)(s.chunk / es);
@@ -157,7 +160,7 @@ void plan_allreduce_tree(Builder& B, const SubColl& s, uint64_t lo, uint64_t hi,
   std::vector<Flow> root_src =
       b.tup[root].kern ? kernel_sources(s, b, root) : b.flows[root];
   const bool zero = root_src.empty();
-  if (zero && accumulate) return;  // recvbuf untouched (reading Q7)
+  if (zero && accumulate && !late_join) return;  // recvbuf untouched (reading Q7)
 
   std::vector<BufRef> recv_all;
   for (int g = 0; g < n; ++g)
@@ -182,7 +185,13 @@ void plan_allreduce_tree(Builder& B, const SubColl& s, uint64_t lo, uint64_t hi,
     }
     std::vector<Stream> srcs;
     for (auto& f : root_src) srcs.push_back(stream_of(f));
-    B.add(root, lo, hi, ce, zero ? kOpZero : kOpFold, srcs, recv_all, {});
+    // late join: every non-ready rank is an optional source of the
+    // root's fold, included per piece if it became ready in time
+    std::vector<BufRef> late;
+    if (late_join)
+      for (int g = 0; g < n; ++g)
+        if (!((mask >> g) & 1)) late.push_back(make_ref(kBufSend, g, send_bias));
+    B.add(root, lo, hi, ce, zero ? kOpZero : kOpFold, srcs, recv_all, {}, late);
     return;
   }
 
@@ -337,7 +346,9 @@ SegmentPlan build_segment(const PlanRequest& rq,
     if (lo >= hi) continue;
     const SubColl& s = st.subs[m];
     switch (st.coll) {
-      case kAllReduce: plan_allreduce_tree(B, s, lo, hi, rq.ready_mask, rq.accumulate, rq.mode); break;
+      case kAllReduce:
+        plan_allreduce_tree(B, s, lo, hi, rq.ready_mask, rq.accumulate, rq.mode, 0, false, rq.late_join);
+        break;
       case kReduce: plan_allreduce_tree(B, s, lo, hi, rq.ready_mask, rq.accumulate, rq.mode, 0, true); break;
       case kReduceScatter:
         plan_allreduce_tree(B, s, lo, hi, rq.ready_mask, rq.accumulate, rq.mode,

@@ -40,6 +40,7 @@ struct PlanRequest {
   int esize = 4;
   uint64_t ready_mask = 0;
   bool accumulate = false;
+  bool late_join = false;   // root tasks carry the non-ready ranks as optional sources (NEXT-1)
   Mode mode = kDirect;
   uint64_t half_bytes = 0;  // arena bytes available per rank per parity half
 };

@@ -1,0 +1,109 @@
+"""Late join (NEXT-1) on the GPU vs the late-join oracle (-m gpu).
+
+Deterministic cases: the late ranks signal before phase 1 (every piece folds
+them) or never (phase 2 adds them all).  Racing case: a late rank signals from
+a side stream while phase 1 runs; the inclusion is then timing-dependent, so
+each output element must match the oracle for SOME inclusion set, with the
+same set explaining both the phase-1 and the final value (the oracle never
+consumes the GPU's decisions); int32 finals are exact."""
+
+import itertools
+
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+
+import paper_conf_icdcs_zhaozw24_b200 as pkg  # noqa: E402
+from oracle import collectives as oc  # noqa: E402
+from paper_conf_icdcs_zhaozw24_b200 import generator as G  # noqa: E402
+from synth import rank_tensors  # noqa: E402
+from tests import strategies as S  # noqa: E402
+from tests.gpu_util import bits, empty_dev, to_dev, to_host  # noqa: E402
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(autouse=True)
+def _need_gpu():
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+
+
+def _comm(n, engine):
+    c = pkg.Communicator.loopback(n, mode="direct", scratch_bytes=64 << 20)
+    c.config("engine", engine)
+    c.config("timeout_ms", 20000)
+    return c
+
+
+@pytest.mark.parametrize("engine", [0, 1])
+@pytest.mark.parametrize("dtype", ["f32", "bf16", "i32"])
+@pytest.mark.parametrize("case", ["all", "none"])
+def test_late_join_deterministic(engine, dtype, case):
+    n, count = 8, 200_003
+    R, late = {0, 1, 2, 4, 5, 7}, [3, 6]
+    text = S.allreduce_trees([S.star(n, m) for m in range(n)] + [S.chain([0, 1, 2, 3, 4, 5, 6, 7])],
+                             chunk=16384)
+    xs = rank_tensors(dtype, count, n)
+    comm = _comm(n, engine)
+    comm.set_strategy("allreduce", text)
+    dx = [to_dev(x, dtype) for x in xs]
+    dy = [empty_dev(count, dtype) for _ in range(n)]
+    if case == "all":
+        t = comm.late_ticket() + 1          # the ticket the next LATE_JOIN call will use
+        for r in late:
+            comm.signal_ready(r, ticket=t)
+    comm.allreduce_lb(dx, dy, ready=R, late="join")
+    torch.cuda.synchronize()
+    L = set(late) if case == "all" else set()
+    e1 = oc.allreduce_late(xs, text, R, dtype, L, phase=1)
+    assert all(np.array_equal(bits(to_host(y, dtype)), bits(e)) for y, e in zip(dy, e1))
+    comm.allreduce_lb(dx, dy, ready=R, late="complement")
+    torch.cuda.synchronize()
+    e2 = oc.allreduce_late(xs, text, R, dtype, L, phase=2, y_prev=e1)
+    assert all(np.array_equal(bits(to_host(y, dtype)), bits(e)) for y, e in zip(dy, e2))
+    assert comm.get_async_error() == 0
+    comm.finalize()
+
+
+@pytest.mark.parametrize("engine", [0, 1])
+@pytest.mark.parametrize("dtype", ["f32", "i32"])
+def test_late_join_racing_signal(engine, dtype):
+    n, count = 8, 4_000_003
+    R, late = {0, 1, 2, 4, 5, 7}, [3, 6]
+    text = G.allreduce_stars(n, chunk=65536)
+    xs = rank_tensors(dtype, count, n)
+    comm = _comm(n, engine)
+    comm.set_strategy("allreduce", text)
+    dx = [to_dev(x, dtype) for x in xs]
+    dy = [empty_dev(count, dtype) for _ in range(n)]
+    comm.allreduce_lb(dx, dy)  # warm-up (plans, clocks)
+    torch.cuda.synchronize()
+    side = torch.cuda.Stream()
+    main = torch.cuda.current_stream()
+    t = comm.late_ticket() + 1
+    start = torch.cuda.Event()
+    start.record(main)
+    side.wait_event(start)
+    with torch.cuda.stream(side):
+        torch.cuda._sleep(20_000)          # rank 3 finishes "compute" while phase 1 runs
+        comm.signal_ready(3, ticket=t, stream=side)
+    comm.allreduce_lb(dx, dy, ready=R, late="join")
+    y1 = [to_host(y, dtype) for y in dy]
+    comm.allreduce_lb(dx, dy, ready=R, late="complement")
+    torch.cuda.synchronize()
+    y2 = [to_host(y, dtype) for y in dy]
+    assert comm.get_async_error() == 0
+    for g in range(1, n):                   # broadcast identity
+        assert np.array_equal(bits(y1[g]), bits(y1[0])) and np.array_equal(bits(y2[g]), bits(y2[0]))
+    options = [set(c) for k in range(3) for c in itertools.combinations(late, k)]
+    ok = np.zeros(count, bool)
+    for L in options:
+        p1 = oc.allreduce_late(xs, text, R, dtype, L, phase=1)[0]
+        p2 = oc.allreduce_late(xs, text, R, dtype, L, phase=2, y_prev=[p1])[0]
+        ok |= (bits(y1[0]) == bits(p1)) & (bits(y2[0]) == bits(p2))
+    assert ok.all(), f"{(~ok).sum()} elements not explained by any inclusion set"
+    if dtype == "i32":
+        assert np.array_equal(y2[0], oc.allreduce_exact(xs, set(range(n)), "i32"))
+    comm.finalize()
