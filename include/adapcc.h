@@ -204,6 +204,20 @@ ADAPCC_API adapcc_result_t adapcc_reducescatter_lb(adapcc_comm_t comm, const voi
                                                    adapcc_dtype_t dtype, uint64_t ready_mask,
                                                    unsigned flags, adapcc_stream_t stream);
 
+/* AlltoAllv (NEXT-4; skewed MoE token dispatch): counts is a
+ * HOST array of nranks*nranks element counts, counts[s*nranks + d] from rank s
+ * to rank d, identical on every rank.  Rank s's sendbuf holds its blocks in
+ * destination order, rank d's recvbuf its blocks in source order (packed).
+ * Blocks from non-ready sources are left untouched.  The a2a lines of the
+ * AlltoAll strategy split every block by weight. */
+ADAPCC_API adapcc_result_t adapcc_alltoallv(adapcc_comm_t comm, const void* sendbuf, void* recvbuf,
+                                            const uint64_t* counts, adapcc_dtype_t dtype,
+                                            uint64_t ready_mask, adapcc_stream_t stream);
+ADAPCC_API adapcc_result_t adapcc_alltoallv_lb(adapcc_comm_t comm, const void* const* sendbufs,
+                                               void* const* recvbufs, const uint64_t* counts,
+                                               adapcc_dtype_t dtype, uint64_t ready_mask,
+                                               adapcc_stream_t stream);
+
 /* ----------------------------------------------- zero-copy (multi-process) ---
  * Register a device buffer so that peers can read/write it directly: the
  * allocation holding [ptr, ptr+bytes) is exported with CUDA IPC and mapped by

@@ -357,3 +357,21 @@ def allreduce_late(xs, strategy_text, ready, dtype, included, phase=1, y_prev=No
         for g in range(n):
             ys[g][lo:hi] = res
     return ys
+
+
+def alltoallv(xs, counts, strategy_text, ready, dtype, y_prev):
+    """AlltoAllv (NEXT-4): counts[s][d] elements of rank s's packed sendbuf
+    (destination order) land in rank d's packed recvbuf (source order), for
+    every ready s; other blocks untouched.  Pure index definition."""
+    st = parse(strategy_text)
+    if st.collective != "alltoall":
+        raise ValueError("strategy is not an alltoall strategy")
+    n = st.nranks
+    ys = [np.array(y, copy=True) for y in y_prev]
+    for s in sorted(set(ready)):
+        for d in range(n):
+            soff = sum(counts[s][:d])
+            roff = sum(counts[j][d] for j in range(s))
+            c = counts[s][d]
+            ys[d][roff:roff + c] = xs[s][soff:soff + c]
+    return ys

@@ -87,6 +87,8 @@ def _load():
         "adapcc_register_buffer": [vp, vp, sz, ctypes.POINTER(i32)],
         "adapcc_deregister_buffer": [vp, i32],
         "adapcc_collective_zc": [vp, i32, i32, sz, i32, sz, sz, i32, i32, u64, ctypes.c_uint, vp],
+        "adapcc_alltoallv": [vp, vp, vp, ctypes.POINTER(u64), i32, u64, vp],
+        "adapcc_alltoallv_lb": [vp, pp, pp, ctypes.POINTER(u64), i32, u64, vp],
         "adapcc_late_ticket": [vp, ctypes.POINTER(u64)],
         "adapcc_signal_ready": [vp, i32, u64, vp],
         "adapcc_get_async_error": [vp],
@@ -420,6 +422,23 @@ class Communicator:
         _check(_load().adapcc_allreduce_lb(self._h, S, D, outs[0].numel(), _dtype_code(outs[0]), m,
                                            flags, _stream(stream)), "allreduce_lb")
         return outs
+
+    def alltoallv_lb(self, xs, outs, counts, ready=None, stream=None):
+        """counts: nranks x nranks element counts (counts[s][d] from s to d)."""
+        m = _mask(ready, self.nranks)
+        S, D = self._arrays(xs, outs, m)
+        flat = (ctypes.c_uint64 * (self.nranks * self.nranks))(*[int(v) for row in counts for v in row])
+        _check(_load().adapcc_alltoallv_lb(self._h, S, D, flat, _dtype_code(outs[0]), m, _stream(stream)),
+               "alltoallv_lb")
+        return outs
+
+    def alltoallv(self, x, out, counts, ready=None, stream=None):
+        m = _mask(ready, self.nranks)
+        send = x if (m >> self.rank) & 1 else None
+        flat = (ctypes.c_uint64 * (self.nranks * self.nranks))(*[int(v) for row in counts for v in row])
+        _check(_load().adapcc_alltoallv(self._h, _ptr(send), _ptr(out), flat, _dtype_code(out), m,
+                                        _stream(stream)), "alltoallv")
+        return out
 
     def late_ticket(self):
         v = ctypes.c_uint64()

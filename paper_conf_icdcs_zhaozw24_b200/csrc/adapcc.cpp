@@ -296,9 +296,15 @@ adapcc_result_t pick_strategy(adapcc_comm_s* c, Coll coll, int root, const Strat
 
 adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, const Strategy* strat, uint64_t count,
                          adapcc_dtype_t dtype, uint64_t mask, unsigned flags, Mode mode,
-                         std::shared_ptr<DevPlan>* out) {
+                         std::shared_ptr<DevPlan>* out, const uint64_t* counts = nullptr) {
   // phase 2 of a late join runs on the phase-1 plan (same items, recorded bits)
   if (flags & ADAPCC_FLAG_LATE_COMPLEMENT) flags = ADAPCC_FLAG_LATE_JOIN;
+  if (counts) {  // AlltoAllv: the plan depends on the whole count matrix
+    uint64_t h = 1469598103934665603ull;
+    for (int i = 0; i < c->nranks * c->nranks; ++i) { h ^= counts[i]; h *= 1099511628211ull; }
+    count = h;
+    coll = (Coll)kNumColl;  // distinct plan-cache namespace
+  }
   PlanKey key{(int)coll, strat->hash, count, (int)dtype, mask, flags, (int)mode};
   auto it = c->plans.find(key);
   if (it != c->plans.end()) {
@@ -313,6 +319,7 @@ adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, const Strategy* strat, uin
   rq.ready_mask = mask;
   rq.accumulate = flags & ADAPCC_FLAG_ACCUMULATE;
   rq.late_join = flags & ADAPCC_FLAG_LATE_JOIN;
+  rq.counts = counts;
   rq.mode = mode;
   rq.half_bytes = c->half_bytes;
   std::vector<SegmentPlan> segs;
@@ -368,7 +375,7 @@ adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, const Strategy* strat, uin
 adapcc_result_t run(adapcc_comm_s* c, Coll coll, const void* const* send, void* const* recv,
                     uint64_t count, adapcc_dtype_t dtype, uint64_t mask, unsigned flags,
                     adapcc_stream_t stream, int root = 0, char* const* zc_send = nullptr,
-                    char* const* zc_recv = nullptr) {
+                    char* const* zc_recv = nullptr, const uint64_t* counts = nullptr) {
   const bool zc = zc_send != nullptr;
   std::lock_guard<std::mutex> lock(c->mu);
   CK(cudaSetDevice(c->device));
@@ -376,7 +383,7 @@ adapcc_result_t run(adapcc_comm_s* c, Coll coll, const void* const* send, void* 
   adapcc_result_t r = pick_strategy(c, coll, root, &strat);
   if (r != ADAPCC_SUCCESS) return r;
   std::shared_ptr<DevPlan> plan;
-  r = get_plan(c, coll, strat, count, dtype, mask, flags, zc ? kDirect : c->mode, &plan);
+  r = get_plan(c, coll, strat, count, dtype, mask, flags, zc ? kDirect : c->mode, &plan, counts);
   if (r != ADAPCC_SUCCESS) return r;
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
   cudaStreamCaptureStatus cap = cudaStreamCaptureStatusNone;
@@ -861,6 +868,55 @@ adapcc_result_t adapcc_collective_zc(adapcc_comm_t c, adapcc_coll_t coll, int se
     if (coll == ADAPCC_ALLTOALL && overlap(S[c->rank], sb, D[c->rank], rb)) return ADAPCC_ERR_INVALID_ARGUMENT;
   }
   return run(c, (Coll)coll, nullptr, nullptr, count, dtype, mask, flags, stream, root, S.data(), D.data());
+}
+
+// ---------------------------------------------------------- AlltoAllv (NEXT-4)
+static adapcc_result_t a2av_sizes(adapcc_comm_t c, const uint64_t* counts, int rank, size_t es,
+                                  size_t* sbytes, size_t* rbytes) {
+  if (!counts) return ADAPCC_ERR_INVALID_ARGUMENT;
+  uint64_t s = 0, r = 0;
+  for (int j = 0; j < c->nranks; ++j) {
+    s += counts[(size_t)rank * c->nranks + j];
+    r += counts[(size_t)j * c->nranks + rank];
+  }
+  *sbytes = s * es;
+  *rbytes = r * es;
+  return ADAPCC_SUCCESS;
+}
+
+adapcc_result_t adapcc_alltoallv(adapcc_comm_t c, const void* sendbuf, void* recvbuf, const uint64_t* counts,
+                                 adapcc_dtype_t dtype, uint64_t mask, adapcc_stream_t stream) {
+  adapcc_result_t r = check_common(c, dtype, mask);
+  if (r != ADAPCC_SUCCESS) return r;
+  if (c->loopback) return ADAPCC_ERR_INVALID_ARGUMENT;
+  size_t sb, rb;
+  r = a2av_sizes(c, counts, c->rank, esize_of(dtype), &sb, &rb);
+  if (r != ADAPCC_SUCCESS) return r;
+  const bool ready = (mask >> c->rank) & 1;
+  if ((rb && !recvbuf) || (ready && sb && !sendbuf) || misaligned(recvbuf) || (ready && misaligned(sendbuf)))
+    return ADAPCC_ERR_INVALID_ARGUMENT;
+  if (ready && sb && rb && overlap(sendbuf, sb, recvbuf, rb)) return ADAPCC_ERR_INVALID_ARGUMENT;
+  const void* s[1] = {ready ? sendbuf : nullptr};
+  void* d[1] = {recvbuf};
+  return run(c, kAllToAll, s, d, 0, dtype, mask, 0, stream, 0, nullptr, nullptr, counts);
+}
+
+adapcc_result_t adapcc_alltoallv_lb(adapcc_comm_t c, const void* const* sendbufs, void* const* recvbufs,
+                                    const uint64_t* counts, adapcc_dtype_t dtype, uint64_t mask,
+                                    adapcc_stream_t stream) {
+  adapcc_result_t r = check_common(c, dtype, mask);
+  if (r != ADAPCC_SUCCESS) return r;
+  if (!c->loopback || !sendbufs || !recvbufs) return ADAPCC_ERR_INVALID_ARGUMENT;
+  for (int q = 0; q < c->nranks; ++q) {
+    size_t sb, rb;
+    r = a2av_sizes(c, counts, q, esize_of(dtype), &sb, &rb);
+    if (r != ADAPCC_SUCCESS) return r;
+    const bool ready = (mask >> q) & 1;
+    if ((rb && !recvbufs[q]) || misaligned(recvbufs[q])) return ADAPCC_ERR_INVALID_ARGUMENT;
+    if (ready && ((sb && !sendbufs[q]) || misaligned(sendbufs[q]))) return ADAPCC_ERR_INVALID_ARGUMENT;
+    if (ready && sb && rb && overlap(sendbufs[q], sb, recvbufs[q], rb)) return ADAPCC_ERR_INVALID_ARGUMENT;
+  }
+  return run(c, kAllToAll, sendbufs, recvbufs, 0, dtype, mask, 0, stream, 0, nullptr, nullptr, counts);
 }
 
 // ------------------------------------------------------------ late join (NEXT-1)

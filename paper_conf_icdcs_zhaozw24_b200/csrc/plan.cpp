@@ -337,10 +337,55 @@ void plan_alltoall_line(Builder& B, const SubColl& s, uint64_t lo, uint64_t hi, 
   }
 }
 
+// AlltoAllv: every (s, d) block has its own count; each block is split over
+// the a2a lines by weight (Q9) and then into segment k of nseg.
+void plan_alltoallv(Builder& B, const PlanRequest& rq, uint64_t k, uint64_t nseg) {
+  const Strategy& st = *rq.st;
+  const int n = st.nranks, es = rq.esize;
+  const uint64_t unit = 16 / es;
+  std::vector<int64_t> w;
+  for (auto& s : st.subs) w.push_back(s.weight);
+  for (int src = 0; src < n; ++src) {
+    if (!((rq.ready_mask >> src) & 1)) continue;
+    for (int d = 0; d < n; ++d) {
+      const uint64_t c = rq.counts[(size_t)src * n + d];
+      if (!c) continue;
+      uint64_t soff = 0, roff = 0;
+      for (int j = 0; j < d; ++j) soff += rq.counts[(size_t)src * n + j];
+      for (int j = 0; j < src; ++j) roff += rq.counts[(size_t)j * n + d];
+      const auto b = partition(c, es, w);
+      for (size_t m = 0; m < st.subs.size(); ++m) {
+        const uint64_t step = align_up((b[m + 1] - b[m] + nseg - 1) / nseg, unit);
+        const uint64_t lo = std::min(b[m + 1], b[m] + k * step), hi = std::min(b[m + 1], b[m] + (k + 1) * step);
+        if (lo >= hi) continue;
+        const SubColl& s = st.subs[m];
+        const uint32_t ce = (uint32_t)(s.chunk / es);
+        const uint32_t nch = (uint32_t)((hi - lo + ce - 1) / ce);
+        Stream in;
+        in.ref = make_ref(kBufSend, src, (int64_t)(soff * es));
+        BufRef out = make_ref(kBufRecv, d, (int64_t)(roff * es));
+        if (rq.mode == kDirect || d == src) {
+          B.add(src, lo, hi, ce, kOpFold, {in}, {out}, {});
+          continue;
+        }
+        uint64_t off = B.alloc(d, (hi - lo) * es);
+        FlagRef fl = B.alloc_flags(d, nch);
+        B.add(src, lo, hi, ce, kOpFold, {in}, {make_ref(kBufArena, d, (int64_t)off - (int64_t)(lo * es))}, {fl});
+        B.add(d, lo, hi, ce, kOpFold, {B.slot_stream(d, off, lo, &fl)}, {out}, {});
+      }
+    }
+  }
+}
+
 SegmentPlan build_segment(const PlanRequest& rq,
-                          const std::vector<std::pair<uint64_t, uint64_t>>& ranges) {
+                          const std::vector<std::pair<uint64_t, uint64_t>>& ranges, uint64_t seg_k,
+                          uint64_t nseg) {
   const Strategy& st = *rq.st;
   Builder B(st.nranks, rq.esize, rq.half_bytes);
+  if (rq.counts) {
+    plan_alltoallv(B, rq, seg_k, nseg);
+    return B.finish();
+  }
   for (size_t m = 0; m < st.subs.size(); ++m) {
     const uint64_t lo = ranges[m].first, hi = ranges[m].second;
     if (lo >= hi) continue;
@@ -407,7 +452,13 @@ bool build_plan(const PlanRequest& rq, std::vector<SegmentPlan>* segs, std::stri
         const uint64_t a = std::min(hi, lo + k * step), b = std::min(hi, lo + (k + 1) * step);
         rr[m] = {a, b};
       }
-      SegmentPlan p = build_segment(rq, rr);
+      SegmentPlan p = build_segment(rq, rr, k, nseg);
+      if (rq.counts) {
+        uint64_t cmax = 0;
+        const int n = rq.st->nranks;
+        for (int i = 0; i < n * n; ++i) cmax = std::max<uint64_t>(cmax, rq.counts[i]);
+        max_step = std::max(max_step, align_up((cmax + nseg - 1) / nseg, unit));
+      }
       fits = fits && p.fits;
       if (!p.tasks.empty()) out.push_back(std::move(p));
     }

@@ -43,6 +43,10 @@ struct PlanRequest {
   bool late_join = false;   // root tasks carry the non-ready ranks as optional sources (NEXT-1)
   Mode mode = kDirect;
   uint64_t half_bytes = 0;  // arena bytes available per rank per parity half
+  // AlltoAllv (NEXT-4): counts[s * n + d] elements go from rank s to rank d;
+  // blocks are packed in destination order in the sendbuf and source order in
+  // the recvbuf.  nullptr for every other collective.
+  const uint64_t* counts = nullptr;
 };
 
 // Bytes at the start of each parity half reserved for per-chunk flag words.

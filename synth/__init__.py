@@ -6,4 +6,4 @@ Both the oracle and the CUDA path consume these; neither is imported here.
 """
 
 from .inputs import (rank_tensor, rank_tensors, bf16_bits_from_normal,  # noqa: F401
-                     CONFIGS, GPT2XL_LAYERS, ready_set_from_mask, mask_from_set)
+                     CONFIGS, GPT2XL_LAYERS, ready_set_from_mask, mask_from_set, moe_counts)

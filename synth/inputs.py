@@ -75,3 +75,21 @@ def mask_from_set(ready):
     for r in ready:
         m |= 1 << r
     return m
+
+
+def moe_counts(n, tokens_per_rank, hidden, zipf_a=1.2, seed=2100):
+    """Skewed top-1 MoE routing (NEXT-4, P:L309 MoE workload): every rank routes
+    `tokens_per_rank` tokens to n experts (one per rank) with Zipf(a) expert
+    popularity (a global random popularity order); returns counts[s][d] in
+    ELEMENTS (tokens x hidden).  a = 0 gives uniform routing."""
+    rng = _rng(seed)
+    order = rng.permutation(n)
+    p = 1.0 / (np.arange(1, n + 1) ** zipf_a)
+    p = p / p.sum()
+    probs = np.empty(n)
+    probs[order] = p
+    counts = []
+    for s in range(n):
+        tok = rng.multinomial(tokens_per_rank, probs)
+        counts.append([int(t) * hidden for t in tok])
+    return counts
