@@ -1,0 +1,90 @@
+"""DDP communication hook (NEXT-4) over the engine: 2 processes on one
+GPU (gloo process group, CUDA IPC communicator); gradients after backward must
+equal the average of both ranks' local gradients (-m gpu)."""
+
+import os
+import socket
+import sys
+
+import pytest
+
+torch = pytest.importorskip("torch")
+
+pytestmark = pytest.mark.gpu
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _worker(rank, n, port, q):
+    try:
+        sys.path.insert(0, ROOT)
+        import torch.distributed as dist
+        from torch.nn.parallel import DistributedDataParallel as DDP
+
+        import paper_conf_icdcs_zhaozw24_b200 as pkg
+        from paper_conf_icdcs_zhaozw24_b200.ddp import AdapccHookState, adapcc_allreduce_hook
+
+        os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+        dist.init_process_group("gloo", rank=rank, world_size=n)
+        torch.cuda.set_device(0)
+        torch.manual_seed(0)
+        model = torch.nn.Sequential(torch.nn.Linear(64, 256), torch.nn.ReLU(), torch.nn.Linear(256, 8)).cuda()
+        ref = [p.detach().clone() for p in model.parameters()]
+        comm = pkg.Communicator.init(scratch_bytes=64 << 20, device=0)
+        ddp = DDP(model, device_ids=[0], bucket_cap_mb=1)
+        ddp.register_comm_hook(AdapccHookState(comm), adapcc_allreduce_hook)
+        g = torch.Generator(device="cpu").manual_seed(100 + rank)
+        x = torch.randn(32, 64, generator=g).cuda()
+        ddp(x).square().sum().backward()
+        torch.cuda.synchronize()
+        # expected: average of every rank's local gradient of the same loss
+        local = torch.nn.Sequential(torch.nn.Linear(64, 256), torch.nn.ReLU(), torch.nn.Linear(256, 8)).cuda()
+        with torch.no_grad():
+            for p, r in zip(local.parameters(), ref):
+                p.copy_(r)
+        local(x).square().sum().backward()
+        grads = [p.grad.detach().cpu() for p in local.parameters()]
+        allg = [None] * n
+        dist.all_gather_object(allg, grads)
+        ok = True
+        for i, p in enumerate(model.parameters()):
+            exp = sum(allg[r][i] for r in range(n)) / n
+            ok &= torch.allclose(p.grad.cpu(), exp, rtol=1e-5, atol=1e-6)
+        err = comm.get_async_error()
+        comm.finalize()
+        dist.destroy_process_group()
+        q.put((rank, bool(ok) and err == 0, f"ok={ok} err={err}"))
+    except Exception as e:  # noqa: BLE001
+        import traceback
+        q.put((rank, False, traceback.format_exc() + repr(e)))
+
+
+def test_ddp_hook_two_processes_one_gpu():
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    import torch.multiprocessing as mp
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _port()
+    procs = [ctx.Process(target=_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    out = {}
+    try:
+        for _ in range(2):
+            r, ok, msg = q.get(timeout=600)
+            out[r] = (ok, msg)
+    finally:
+        for p in procs:
+            p.join(timeout=30)
+            if p.is_alive():
+                p.kill()
+    for r in range(2):
+        assert r in out and out[r][0], out.get(r)
