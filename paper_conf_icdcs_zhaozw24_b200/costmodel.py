@@ -1,0 +1,180 @@
+"""Link profiler and strategy cost model (NEXT-2, §IV-B, §IV-D).
+
+alpha-beta profiling: on a link, sending a piece of size s n times
+takes n(alpha + beta s); sending n*s at once takes alpha + beta n s; several
+(n, s) pairs give alpha and beta.  Probe rounds between instances follow the
+round-robin schedule of Fig. 5(b): in round i instance k
+probes (k + i) % N, so every round is a permutation (one flow per port).
+
+Cost model of a reduce tree, used to choose chunk sizes:
+  t_ij   = alpha_ij + beta~_ij C_m                   (chunk time on edge i -> j)
+  beta~_ij = beta_ij * sum_m N^m_ij                  (eq. 3, bandwidth sharing)
+  N^m_ij = 1 when i aggregates; |F^i_m| + sum_k N^m_ki otherwise;
+           1 for Broadcast
+  h_j    = max over in-flows (h_i + t_ij) with aggregation, h_i + t_ij without
+           (eq. 2, garbled; reading Q18)
+  T_f    = h_dst + ceil(S_m / C_m) * T_bottle, T_bottle = max edge gap on the
+           path (eqs. 5, 6); the strategy's time is max_f T_f (eq. 4)
+AllReduce = the Reduce trees followed by their reversed Broadcast, pipelined
+chunk by chunk: per tree T = h_root + depth_bcast_time +
+ceil(S_m / C_m) * max(bottleneck of both stages) -- reading R6.
+Trees are read through the product's strategy loader (host-only C ABI).
+"""
+
+import math
+
+from . import adapcc as _A
+
+# ---------------------------------------------------------------- profiler
+
+
+def solve_alpha_beta(t_many, t_once, n, s):
+    """Closed form from the two probes of P:L113:
+    t_many = n (alpha + beta s), t_once = alpha + beta n s
+    => alpha = (t_many - t_once) / (n - 1), beta = (t_once - alpha) / (n s)."""
+    alpha = (t_many - t_once) / (n - 1)
+    beta = (t_once - alpha) / (n * s)
+    return alpha, beta
+
+
+def fit_alpha_beta(samples):
+    """Least squares over (messages, bytes_each, seconds) samples of the model
+    t = messages * alpha + messages * bytes_each * beta ("several
+    measurements are performed under different values of n and s")."""
+    a11 = a12 = a22 = b1 = b2 = 0.0
+    for m, s, t in samples:
+        x1, x2 = float(m), float(m) * float(s)
+        a11 += x1 * x1
+        a12 += x1 * x2
+        a22 += x2 * x2
+        b1 += x1 * t
+        b2 += x2 * t
+    det = a11 * a22 - a12 * a12
+    return (b1 * a22 - b2 * a12) / det, (a11 * b2 - a12 * b1) / det
+
+
+def probe_rounds(n_instances):
+    """Fig. 5(b): N-1 rounds; in round i instance k probes (k + i) % N."""
+    return [[(k, (k + i) % n_instances) for k in range(n_instances)] for i in range(1, n_instances)]
+
+
+def probe_link(copy_fn, sizes=(1 << 16, 1 << 20), repeats=(1, 8), timer=None):
+    """Measure one link with the paper's two probe shapes.  copy_fn(nbytes)
+    performs one transfer and returns its duration in seconds (or timer()
+    measures it).  Returns (alpha, beta, samples)."""
+    samples = []
+    for s in sizes:
+        for n in repeats:
+            t = sum(copy_fn(s) for _ in range(n))        # n pieces of s
+            samples.append((n, s, t))
+            t1 = copy_fn(n * s)                          # one piece of n*s
+            samples.append((1, n * s, t1))
+    alpha, beta = fit_alpha_beta(samples)
+    return alpha, beta, samples
+
+
+# -------------------------------------------------------------- cost model
+def _trees(text):
+    n, coll, nsubs = _A.strategy_check(text)
+    subs = []
+    for m in range(nsubs):
+        w, chunk, parent, src = _A.strategy_sub(text, m)
+        subs.append((w, chunk, parent))
+    return n, subs
+
+
+def link_loads(parent, noagg=frozenset(), broadcast=False):
+    """N_ij for every tree edge (child -> parent) of one sub-collective."""
+    n = len(parent)
+    children = {g: [c for c in range(n) if parent[c] == g] for g in range(n)}
+    loads = {}
+
+    def out_flows(g):   # flows sent from g to its parent
+        if broadcast or g not in noagg:
+            return 1
+        return 1 + sum(out_flows(c) for c in children[g])
+
+    for g in range(n):
+        if parent[g] != -1:
+            loads[(g, parent[g])] = out_flows(g)
+    return loads
+
+
+def tree_time(parent, S_m, C_m, alpha, beta, shared_loads=None, noagg=frozenset()):
+    """T of one Reduce tree (eqs. 2, 5, 6).  alpha[i][j], beta[i][j] per link
+    (seconds, seconds per byte); shared_loads[(i, j)] = sum_m N^m_ij over all
+    sub-collectives (eq. 3), defaults to this tree's own loads."""
+    n = len(parent)
+    loads = shared_loads or link_loads(parent, noagg)
+    root = parent.index(-1)
+    children = {g: [c for c in range(n) if parent[c] == g] for g in range(n)}
+
+    def t(i, j):
+        return alpha[i][j] + beta[i][j] * loads.get((i, j), 1) * C_m
+
+    h = {}
+    bottle = 0.0
+
+    def ready(g):   # eq. 2 with aggregation: wait for the slowest in-flow
+        nonlocal bottle
+        if g in h:
+            return h[g]
+        best = 0.0
+        for c in children[g]:
+            best = max(best, ready(c) + t(c, g))
+            bottle = max(bottle, t(c, g))
+        h[g] = best
+        return best
+
+    h_root = ready(root)
+    chunks = max(1, math.ceil(S_m / C_m))
+    return h_root + chunks * bottle, h_root, bottle
+
+
+def allreduce_time(text, S, alpha, beta, esize=4):
+    """Predicted AllReduce time of a strategy for S bytes per rank: every tree
+    reduces its partition and broadcasts it back along the reversed edges, both
+    stages pipelined; the trees run concurrently sharing links (eq. 3)."""
+    n, subs = _trees(text)
+    W = sum(w for w, _, _ in subs)
+    shared = {}
+    for _, _, parent in subs:
+        for e, v in link_loads(parent).items():
+            shared[e] = shared.get(e, 0) + v
+            shared[(e[1], e[0])] = shared.get((e[1], e[0]), 0) + 1   # broadcast back
+    worst = 0.0
+    for w, chunk, parent in subs:
+        S_m = S * w / W
+        if S_m <= 0:
+            continue
+        t_red, h_red, b_red = tree_time(parent, S_m, chunk, alpha, beta, shared)
+        rev = {(j, i): 1 for (i, j) in link_loads(parent)}
+        # broadcast stage: same tree, edges reversed, depth h_bcast
+        depth = _depth(parent)
+        t_edge = max((alpha[j][i] + beta[j][i] * shared.get((j, i), 1) * chunk for (j, i) in rev), default=0.0)
+        h_b = depth * t_edge
+        chunks = max(1, math.ceil(S_m / chunk))
+        worst = max(worst, h_red + h_b + chunks * max(b_red, t_edge))
+    return worst
+
+
+def _depth(parent):
+    d = 0
+    for g in range(len(parent)):
+        k, x = 0, g
+        while parent[x] != -1:
+            x, k = parent[x], k + 1
+        d = max(d, k)
+    return d
+
+
+def best_chunk(text_for_chunk, S, alpha, beta, candidates=(1 << 14, 1 << 16, 1 << 18, 1 << 20, 1 << 22)):
+    """Chunk size C minimising the predicted time ("identifies optimized chunk
+    size to pipeline the transmission").  text_for_chunk(C) -> strategy."""
+    scored = [(allreduce_time(text_for_chunk(c), S, alpha, beta), c) for c in candidates]
+    return min(scored)[1], scored
+
+
+def uniform_links(n, alpha, beta):
+    """NVSwitch: every GPU pair has the same alpha, beta."""
+    return [[alpha] * n for _ in range(n)], [[beta] * n for _ in range(n)]

@@ -269,5 +269,66 @@ def main():
     json.dump(out, open(a.out, "w"), indent=1)
 
 
-if __name__ == "__main__":
+if __name__ == "__main__" and "--links" not in sys.argv:
     main()
+
+
+def profile_links(out_path=None):
+    """NEXT-2 on one GPU: the paper's alpha-beta probes applied to the
+    engine's own copy path (2 virtual ranks, Broadcast = one K=1 copy) and to a
+    plain device copy, then the cost model's chunk choice for NVLink numbers."""
+    import torch
+
+    import paper_conf_icdcs_zhaozw24_b200 as pkg
+    from paper_conf_icdcs_zhaozw24_b200 import costmodel as CM
+    from paper_conf_icdcs_zhaozw24_b200 import generator as G
+
+    comm = pkg.Communicator.loopback(2, mode="direct", scratch_bytes=64 << 20)
+    bufs = {}
+
+    def engine_copy(nbytes):
+        cnt = nbytes // 4
+        if cnt not in bufs:
+            bufs[cnt] = ([torch.ones(cnt, device="cuda")] * 2, [torch.empty(cnt, device="cuda") for _ in range(2)])
+        xs, ys = bufs[cnt]
+        comm.broadcast_lb(xs, ys, 0)
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        comm.broadcast_lb(xs, ys, 0)
+        e1.record()
+        torch.cuda.synchronize()
+        return e0.elapsed_time(e1) * 1e-3
+
+    def torch_copy(nbytes):
+        a = torch.ones(nbytes // 4, device="cuda")
+        b = torch.empty_like(a)
+        b.copy_(a)
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        b.copy_(a)
+        e1.record()
+        torch.cuda.synchronize()
+        return e0.elapsed_time(e1) * 1e-3
+
+    res = {}
+    for name, fn in (("engine_copy", engine_copy), ("torch_copy", torch_copy)):
+        a, b, samples = CM.probe_link(fn, sizes=(1 << 16, 1 << 22), repeats=(1, 8))
+        res[name] = {"alpha_us": round(a * 1e6, 3), "beta_GBps": round(1 / b / 1e9, 1) if b > 0 else None,
+                     "note": "one GPU: 'link' = HBM read+write of the copy"}
+    n = 8
+    alpha, beta = CM.uniform_links(n, 3e-6, 1 / 770e9)
+    best, scored = CM.best_chunk(lambda c: G.allreduce_stars(n, chunk=c), 256 << 20, alpha, beta)
+    res["nvlink_model_256MiB_8ranks"] = {"alpha_us": 3.0, "link_GBps": 770,
+                                         "best_chunk": best,
+                                         "predicted_ms": {str(c): round(t * 1e3, 4) for t, c in scored}}
+    comm.finalize()
+    print("LINKS", json.dumps(res), flush=True)
+    return res
+
+
+if __name__ == "__main__" and "--links" in sys.argv:
+    r = profile_links()
+    os.makedirs(os.path.join(ROOT, "gpurun_out"), exist_ok=True)
+    json.dump(r, open(os.path.join(ROOT, "gpurun_out", "links.json"), "w"), indent=1)
