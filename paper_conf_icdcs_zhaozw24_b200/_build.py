@@ -11,8 +11,10 @@ PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 LIB = os.path.join(PKG, "libadapcc.so")
-SOURCES = ["adapcc.cpp", "strategy.cpp", "plan.cpp", "engine.cu", "engine_tma.cu"]
-HEADERS = ["engine.cuh", "engine_common.cuh", "launch.hpp", "plan.hpp", "strategy.hpp"]
+SOURCES = ["adapcc.cpp", "strategy.cpp", "plan.cpp", "engine.cu", "engine_tma_direct.cu",
+           "engine_tma_staged.cu"]
+HEADERS = ["engine.cuh", "engine_common.cuh", "engine_tma_impl.cuh", "launch.hpp", "plan.hpp",
+           "strategy.hpp"]
 
 NVCC_FLAGS = [
     "-gencode", "arch=compute_100a,code=sm_100a",

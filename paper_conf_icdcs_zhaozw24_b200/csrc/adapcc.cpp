@@ -43,7 +43,8 @@ struct DevSegment {
 };
 
 struct DevPlan {
-  int engine = 0;      // kernel this plan's pieces were sized for
+  int engine = 0;      // 0: LDG fold kernel, 1: TMA pipeline
+  int kernel = 0;      // 0: LDG, 1: TMA for DIRECT plans, 2: TMA for STAGED plans
   std::vector<DevSegment> segs;
   cudaEvent_t last_use = nullptr;
   uint64_t last_tick = 0;
@@ -148,7 +149,9 @@ struct adapcc_comm_s {
   int64_t piece_kib = 0;  // 0 = automatic (total traffic / (8 * grid))
   uint64_t launches = 0;
   int num_sms = 148;
-  int occ[2][3] = {{1, 1, 1}, {1, 1, 1}};  // [engine][dtype] resident CTAs per SM
+  // [kernel][dtype] resident CTAs per SM; kernels: 0 LDG fold, 1 TMA (DIRECT
+  // plans), 2 TMA (STAGED plans)
+  int occ[3][3] = {{1, 1, 1}, {1, 1, 1}, {1, 1, 1}};
   int engine = 2;  // 0: LDG/STG fold, 1: TMA bulk pipeline, 2: auto by call size
   int last_engine = -1;  // kernel used by the most recent launch
   std::mutex mu;
@@ -190,8 +193,9 @@ adapcc_result_t common_init(adapcc_comm_s* c, size_t scratch) {
   CK(cudaDeviceGetAttribute(&c->num_sms, cudaDevAttrMultiProcessorCount, c->device));
   for (int d = 0; d < 3; ++d) {
     CK(engine_occupancy(d, &c->occ[0][d]));
-    CK(engine_tma_occupancy(d, &c->occ[1][d]));
-    for (int k = 0; k < 2; ++k)
+    CK(tma_direct::occupancy(d, &c->occ[1][d]));
+    CK(tma_staged::occupancy(d, &c->occ[2][d]));
+    for (int k = 0; k < 3; ++k)
       if (c->occ[k][d] < 1) c->occ[k][d] = 1;
   }
   CK(cudaMalloc(&c->state, sizeof(DevState)));
@@ -261,8 +265,8 @@ bool overlap(const void* a, size_t an, const void* b, size_t bn) {
 // launch the LDG kernel's lower fixed cost wins, above it the TMA pipeline.
 constexpr uint64_t kTmaMinTraffic = uint64_t(64) << 20;
 
-int grid_size(const adapcc_comm_s* c, adapcc_dtype_t dtype, int engine) {
-  int grid = c->num_sms * c->occ[engine][(int)dtype];
+int grid_size(const adapcc_comm_s* c, adapcc_dtype_t dtype, int kernel) {
+  int grid = c->num_sms * c->occ[kernel][(int)dtype];
   if (c->max_ctas > 0) grid = (int)std::min<int64_t>(grid, c->max_ctas);
   return std::max(grid, 1);
 }
@@ -331,11 +335,12 @@ adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, const Strategy* strat, uin
     for (auto& sp : segs) accumulate_stats(sp, c->loopback ? -1 : c->rank, rq.esize, &st);
     const uint64_t traffic = st.bytes_read + st.bytes_written;
     plan->engine = c->engine != 2 ? c->engine : (traffic / std::max<size_t>(1, segs.size()) >= kTmaMinTraffic ? 1 : 0);
+    plan->kernel = plan->engine == 0 ? 0 : (mode == kDirect ? 1 : 2);
   }
   CK(cudaEventCreateWithFlags(&plan->last_use, cudaEventDisableTiming));
   for (auto& sp : segs) {
     DevSegment d;
-    std::vector<Item> items = order_items(sp, c->loopback ? -1 : c->rank, rq.esize, grid_size(c, dtype, plan->engine),
+    std::vector<Item> items = order_items(sp, c->loopback ? -1 : c->rank, rq.esize, grid_size(c, dtype, plan->kernel),
                                           (uint64_t)c->piece_kib * 1024);
     d.nitems = (uint32_t)items.size();
     auto up = [](auto** dst, const auto& v) -> cudaError_t {
@@ -428,8 +433,9 @@ adapcc_result_t run(adapcc_comm_s* c, Coll coll, const void* const* send, void* 
       }
       P.hdr[q] = c->arena[q];
     }
-    const int grid = std::max(1, std::min<int>(grid_size(c, dtype, plan->engine), (int)std::max<uint32_t>(1, seg.nitems)));
-    CK(plan->engine ? engine_tma_launch(P, grid, s) : engine_launch(P, grid, s));
+    const int grid = std::max(1, std::min<int>(grid_size(c, dtype, plan->kernel), (int)std::max<uint32_t>(1, seg.nitems)));
+    CK(plan->kernel == 1 ? tma_direct::launch(P, grid, s)
+       : plan->kernel == 2 ? tma_staged::launch(P, grid, s) : engine_launch(P, grid, s));
     c->last_engine = plan->engine;
     ++c->launches;
   }

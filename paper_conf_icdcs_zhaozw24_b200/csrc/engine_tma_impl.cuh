@@ -15,9 +15,16 @@
 // Paper mapping: the producer is the "receive" side of the chunk pipeline
 // (wait for the chunk, then aggregate), consumers are the
 // aggregation kernel + send.
+// Compiled twice (engine_tma_direct.cu, engine_tma_staged.cu) with different
+// pipeline shapes: ADAPCC_TMA_NS names the instantiation's namespace.
 #include "engine_common.cuh"
 
+#ifndef ADAPCC_TMA_NS
+#error "include through engine_tma_direct.cu / engine_tma_staged.cu"
+#endif
+
 namespace adapcc {
+namespace ADAPCC_TMA_NS {
 namespace {
 
 using namespace dev;
@@ -25,9 +32,18 @@ using namespace dev;
 constexpr int kConsumerWarps = 8;
 constexpr int kConsumers = kConsumerWarps * 32;
 constexpr int kTmaThreads = kConsumers + 32;  // + 1 producer warp
-constexpr int kStages = 3;
-constexpr uint32_t kStageBytes = 32768;
-constexpr int kMaxKS = 8;       // sources per stage
+#ifndef ADAPCC_TMA_STAGES
+#define ADAPCC_TMA_STAGES 3      // shared-memory ring depth
+#endif
+#ifndef ADAPCC_TMA_STAGE_KB
+#define ADAPCC_TMA_STAGE_KB 32   // bytes per stage (all K source tiles of one step)
+#endif
+#ifndef ADAPCC_TMA_MINB
+#define ADAPCC_TMA_MINB 2        // resident CTAs per SM
+#endif
+constexpr int kStages = ADAPCC_TMA_STAGES;
+constexpr uint32_t kStageBytes = ADAPCC_TMA_STAGE_KB * 1024;
+constexpr int kMaxKS = (kStageBytes / 4096) < 8 ? (int)(kStageBytes / 4096) : 8;  // sources per stage
 constexpr int kQ = 2;           // item queue depth
 constexpr int kMaxPost = 4;
 
@@ -331,7 +347,7 @@ __device__ __forceinline__ void fill_desc(const LaunchParams& P, ItemDesc& d, co
 }
 
 template <int DT>
-__global__ void __launch_bounds__(kTmaThreads, 2) engine_tma_kernel(const __grid_constant__ LaunchParams P) {
+__global__ void __launch_bounds__(kTmaThreads, ADAPCC_TMA_MINB) engine_tma_kernel(const __grid_constant__ LaunchParams P) {
   extern __shared__ __align__(128) unsigned char smem_raw[];
   Smem& sm = *reinterpret_cast<Smem*>(smem_raw);
   char* stages = reinterpret_cast<char*>(smem_raw) + kSmemHeader;
@@ -500,9 +516,9 @@ cudaError_t prepare() {
 
 }  // namespace
 
-int engine_tma_threads() { return kTmaThreads; }
+int threads() { return kTmaThreads; }
 
-cudaError_t engine_tma_occupancy(int dtype, int* blocks_per_sm) {
+cudaError_t occupancy(int dtype, int* blocks_per_sm) {
   switch (dtype) {
     case kF32:
       if (cudaError_t e = prepare<kF32>()) return e;
@@ -516,7 +532,7 @@ cudaError_t engine_tma_occupancy(int dtype, int* blocks_per_sm) {
   }
 }
 
-cudaError_t engine_tma_launch(const LaunchParams& p, int grid, cudaStream_t stream) {
+cudaError_t launch(const LaunchParams& p, int grid, cudaStream_t stream) {
   cudaGetLastError();
   switch (p.dtype) {
     case kF32: prepare<kF32>(); engine_tma_kernel<kF32><<<grid, kTmaThreads, kSmemBytes, stream>>>(p); break;
@@ -526,4 +542,5 @@ cudaError_t engine_tma_launch(const LaunchParams& p, int grid, cudaStream_t stre
   return cudaGetLastError();
 }
 
+}  // namespace ADAPCC_TMA_NS
 }  // namespace adapcc

@@ -52,9 +52,17 @@ cudaError_t engine_occupancy(int dtype, int* blocks_per_sm);
 cudaError_t engine_launch(const LaunchParams& p, int grid, cudaStream_t stream);
 // store `value` into a ready word after all prior work on `stream` (late join)
 cudaError_t engine_signal(uint64_t* word, uint64_t value, bool sys, cudaStream_t stream);
-// engine_tma.cu: TMA bulk-copy pipeline (1 producer + 8 consumer warps, 2 CTAs/SM)
-int engine_tma_threads();
-cudaError_t engine_tma_occupancy(int dtype, int* blocks_per_sm);
-cudaError_t engine_tma_launch(const LaunchParams& p, int grid, cudaStream_t stream);
+// engine_tma_impl.cuh: TMA bulk-copy pipeline (1 producer + 8 consumer warps),
+// one instantiation per plan kind
+namespace tma_direct {
+int threads();
+cudaError_t occupancy(int dtype, int* blocks_per_sm);
+cudaError_t launch(const LaunchParams& p, int grid, cudaStream_t stream);
+}  // namespace tma_direct
+namespace tma_staged {
+int threads();
+cudaError_t occupancy(int dtype, int* blocks_per_sm);
+cudaError_t launch(const LaunchParams& p, int grid, cudaStream_t stream);
+}  // namespace tma_staged
 
 }  // namespace adapcc

@@ -11,8 +11,14 @@ import sys
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
-VARIANTS = {"u8b2": ("ADAPCC_UNROLL=8", "ADAPCC_MINB=2"), "u4b4": ("ADAPCC_UNROLL=4", "ADAPCC_MINB=4"),
-            "u4b2": ("ADAPCC_UNROLL=4", "ADAPCC_MINB=2"), "u16b1": ("ADAPCC_UNROLL=16", "ADAPCC_MINB=1")}
+VARIANTS = {  # TMA pipeline shapes: stages x stage KiB x CTAs/SM
+    "s3k32b2": ("ADAPCC_TMA_STAGES=3", "ADAPCC_TMA_STAGE_KB=32", "ADAPCC_TMA_MINB=2"),
+    "s4k32b1": ("ADAPCC_TMA_STAGES=4", "ADAPCC_TMA_STAGE_KB=32", "ADAPCC_TMA_MINB=1"),
+    "s6k32b1": ("ADAPCC_TMA_STAGES=6", "ADAPCC_TMA_STAGE_KB=32", "ADAPCC_TMA_MINB=1"),
+    "s5k40b1": ("ADAPCC_TMA_STAGES=5", "ADAPCC_TMA_STAGE_KB=40", "ADAPCC_TMA_MINB=1"),
+    "s4k48b1": ("ADAPCC_TMA_STAGES=4", "ADAPCC_TMA_STAGE_KB=48", "ADAPCC_TMA_MINB=1"),
+    "s3k64b1": ("ADAPCC_TMA_STAGES=3", "ADAPCC_TMA_STAGE_KB=64", "ADAPCC_TMA_MINB=1"),
+}
 
 
 def lib(v):
@@ -23,7 +29,7 @@ def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--build", action="store_true")
     ap.add_argument("--variants", default=",".join(VARIANTS))
-    ap.add_argument("--chunks", default="64,128,256,512,1024")
+    ap.add_argument("--chunks", default="256")
     ap.add_argument("--extra", default="")
     ap.add_argument("--pieces", default="0", help="ADAPCC_PIECE_KIB values (0 = auto)")
     ap.add_argument("--out", default=os.path.join(ROOT, "gpurun_out", "sweep.json"))
