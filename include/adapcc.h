@@ -293,6 +293,14 @@ ADAPCC_API adapcc_result_t adapcc_strategy_tuples(const char* strategy_text, int
 ADAPCC_API adapcc_result_t adapcc_strategy_sub(const char* strategy_text, int sub, int64_t* weight,
                                     int64_t* chunk_bytes, int32_t* parent, int32_t* src);
 
+/* Route of AlltoAll flow src -> dst in a2a sub-collective `sub` (routing
+ * variables x^f_ij, eq. 1; DESIGN.md §2 `route=`): writes the relay
+ * ranks in path order into hops (capacity nranks entries) and their number
+ * into *nhops (0 = direct).  INVALID_ARGUMENT for a non-a2a sub or ranks out
+ * of range.  Host-only. */
+ADAPCC_API adapcc_result_t adapcc_strategy_route(const char* strategy_text, int sub, int src, int dst,
+                                      int32_t* hops, int* nhops);
+
 /* Partition (DESIGN.md §3 Q9): bounds[0..nsubs] of `count` elements over all
  * sub-collectives (allreduce/alltoall), or over the bcast lines of source
  * `src` (allgather; bounds has (#lines of src)+1 entries). */

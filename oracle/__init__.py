@@ -22,9 +22,10 @@ Modules:
   bf16         -- bit-level bf16 <-> fp32 with round-to-nearest-even.
   collectives  -- allreduce (replay of the strategy's reduction order and the
                   fp64 definition), allgather, alltoall.
+  loads        -- AlltoAll flow routes (eq. 1) and link loads N_ij.
 
 Parity status of every function is in DESIGN.md §4 ("pins"); there is no
 function here without a pin.
 """
 
-from . import bf16, strategy, tuples, collectives  # noqa: F401
+from . import bf16, strategy, tuples, collectives, loads  # noqa: F401

@@ -18,11 +18,15 @@ Format (one directive per line, '#' starts a comment):
     tree  weight=<w> chunk=<C> parent=<p_0,..,p_{n-1}> [noagg=<g,..>]   (allreduce)
     ring  weight=<w> chunk=<C> order=<r_0,..,r_{n-1}>                     (allreduce)
     bcast src=<s> weight=<w> chunk=<C> parent=<p_0,..,p_{n-1}>           (allgather, broadcast)
-    a2a   weight=<w> chunk=<C>                                            (alltoall)
+    a2a   weight=<w> chunk=<C> [route=<s>:<d>:<h1>,..[;<s>:<d>:<h>,..]]  (alltoall)
     rtree dst=<b> weight=<w> chunk=<C> parent=<...> [noagg=<g,..>]       (reducescatter)
   collective reduce uses tree lines sharing one root; broadcast uses bcast
   lines sharing one src (NEXT-4 primitives: Reduce / Broadcast, P:L165,
   ReduceScatter, P:L154(1)).
+
+An a2a route entry s:d:h1,..,hk sends flow s -> d along s, h1, .., hk, d
+(routing variables x^f_ij of eq. 1); flows without an entry go
+direct.
 
 Readings: Q9 partition, Q10 chunk, Q13 ring expansion.
 """
@@ -50,6 +54,7 @@ class Sub:
     parent: list = None       # parent[g], -1 at the root (tree / bcast)
     noagg: frozenset = frozenset()   # ranks g with a_{m,g} = 0
     src: int = -1             # bcast: source (== root); rtree: destination block (== root)
+    routes: dict = field(default_factory=dict)   # a2a: (s, d) -> tuple of relay ranks
 
     @property
     def root(self):
@@ -104,6 +109,40 @@ def _check_tree(parent, n, what):
             steps += 1
             if steps > n:
                 raise StrategyError(f"{what}: cycle through rank {g}")
+
+
+def _routes(tok, n):
+    """route=s:d:h1,h2;... -> {(s, d): (h1, h2)}.  Eq. 1 asks that a
+    flow leave its source once, enter its destination once and be conserved
+    at every other node; a simple path s, h1, .., hk, d (all ranks distinct,
+    k >= 1) is exactly such a flow without cycles."""
+    out = {}
+    if tok is None:
+        return out
+    for ent in tok.split(";"):
+        parts = ent.split(":")
+        if len(parts) != 3:
+            raise StrategyError(f"route entry {ent!r} is not src:dst:hops")
+        s, d = _int(parts[0], "route src"), _int(parts[1], "route dst")
+        hops = _intlist(parts[2], "route hops")
+        path = [s] + hops + [d]
+        if any(not (0 <= g < n) for g in path):
+            raise StrategyError(f"route {ent!r} has a rank out of range")
+        if s == d:
+            raise StrategyError("route src == dst")
+        if not hops:
+            raise StrategyError("route needs at least one relay")
+        if len(set(path)) != len(path):
+            raise StrategyError(f"route {ent!r} visits a rank twice")
+        if (s, d) in out:
+            raise StrategyError(f"two routes for flow {s}->{d}")
+        out[(s, d)] = tuple(hops)
+    return out
+
+
+def flow_path(sub, s, d):
+    """Nodes of flow s -> d in a2a sub-collective `sub`: [s, h1, .., hk, d]."""
+    return [s] + list(sub.routes.get((s, d), ())) + [d]
 
 
 def parse(text):
@@ -161,7 +200,8 @@ def parse(text):
     keys = {"tree": {"weight", "chunk", "parent"}, "ring": {"weight", "chunk", "order"},
             "bcast": {"src", "weight", "chunk", "parent"}, "a2a": {"weight", "chunk"},
             "rtree": {"dst", "weight", "chunk", "parent"}}
-    optional = {"tree": {"noagg"}, "ring": set(), "bcast": set(), "a2a": set(), "rtree": {"noagg"}}
+    optional = {"tree": {"noagg"}, "ring": set(), "bcast": set(), "a2a": {"route"},
+                "rtree": {"noagg"}}
     if not raw_subs:
         raise StrategyError("no sub-collective lines")
     st = Strategy(nranks=n, collective=coll)
@@ -216,7 +256,7 @@ def parse(text):
                 raise StrategyError("bcast root must be its src")
             st.subs.append(Sub("bcast", w * n, c, parent, frozenset(), src))
         else:
-            st.subs.append(Sub("a2a", w * n, c))
+            st.subs.append(Sub("a2a", w * n, c, routes=_routes(kv.get("route"), n)))
     if len(st.subs) > MAX_SUBS:
         raise StrategyError(f"{len(st.subs)} sub-collectives > {MAX_SUBS}")
     if coll in ("allgather", "reducescatter"):

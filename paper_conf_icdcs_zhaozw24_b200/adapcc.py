@@ -102,6 +102,8 @@ def _load():
                                    ctypes.POINTER(ctypes.c_int32)],
         "adapcc_strategy_sub": [ctypes.c_char_p, i32, ctypes.POINTER(i64), ctypes.POINTER(i64),
                                 ctypes.POINTER(ctypes.c_int32), ctypes.POINTER(ctypes.c_int32)],
+        "adapcc_strategy_route": [ctypes.c_char_p, i32, i32, i32, ctypes.POINTER(ctypes.c_int32),
+                                  ctypes.POINTER(i32)],
         "adapcc_strategy_partition": [ctypes.c_char_p, u64, i32, i32, ctypes.POINTER(u64),
                                       ctypes.POINTER(i32)],
         "adapcc_plan_stats": [ctypes.c_char_p, u64, i32, u64, ctypes.c_uint, i32, i32, sz,
@@ -197,6 +199,17 @@ def strategy_sub(text, sub):
     _check(L.adapcc_strategy_sub(text.encode(), sub, ctypes.byref(w), ctypes.byref(c), par,
                                  ctypes.byref(src)), "strategy_sub")
     return w.value, c.value, list(par), src.value
+
+
+def strategy_route(text, sub, src, dst):
+    """Relay ranks of AlltoAll flow src -> dst in a2a line `sub` ([] = direct)."""
+    L = _load()
+    n, _, _ = strategy_check(text)
+    hops = (ctypes.c_int32 * n)()
+    nh = ctypes.c_int()
+    _check(L.adapcc_strategy_route(text.encode(), sub, src, dst, hops, ctypes.byref(nh)),
+           "strategy_route")
+    return list(hops[:nh.value])
 
 
 def strategy_partition(text, count, dtype, src=-1):

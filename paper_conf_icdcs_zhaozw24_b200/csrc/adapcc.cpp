@@ -1037,6 +1037,20 @@ adapcc_result_t adapcc_strategy_sub(const char* text, int sub, int64_t* weight, 
   return ADAPCC_SUCCESS;
 }
 
+adapcc_result_t adapcc_strategy_route(const char* text, int sub, int src, int dst, int32_t* hops,
+                                      int* nhops) {
+  Strategy st;
+  if (!parse_strategy(text, &st, nullptr)) return ADAPCC_ERR_INVALID_STRATEGY;
+  if (sub < 0 || sub >= (int)st.subs.size() || st.subs[sub].kind != kA2A || !nhops || src < 0 ||
+      src >= st.nranks || dst < 0 || dst >= st.nranks)
+    return ADAPCC_ERR_INVALID_ARGUMENT;
+  const std::vector<int>* h = st.subs[sub].hops(src, dst);
+  *nhops = h ? (int)h->size() : 0;
+  if (h && hops)
+    for (size_t i = 0; i < h->size(); ++i) hops[i] = (*h)[i];
+  return ADAPCC_SUCCESS;
+}
+
 adapcc_result_t adapcc_strategy_partition(const char* text, uint64_t count, adapcc_dtype_t dtype,
                                           int src, uint64_t* bounds, int* nbounds) {
   Strategy st;

@@ -18,7 +18,8 @@
 //   store-and-forward hop adds bytes on the relay's ports without adding link
 //   capacity.  Relays still receive the result (Q4).
 // AllGather: one broadcast tree per source.
-// AlltoAll: direct routes; block d of s lands in block s of d.
+// AlltoAll: block d of s lands in block s of d, direct or along the
+// flow's route (eq. 1).
 #include "plan.hpp"
 
 #include <algorithm>
@@ -311,28 +312,46 @@ void plan_allgather_tree(Builder& B, const SubColl& s, uint64_t lo, uint64_t hi,
 }
 
 // -------------------------------------------------------------- AlltoAll
+// One flow ("each GPU sends multiple flows to all other GPUs") along
+// its route src -> hops -> dst (routing variables x^f_ij, eq. 1).  Relays do
+// not aggregate (a_{m,g} = 0 for primitives without aggregation), so
+// every hop is chunk-pipelined store-and-forward, h_j = h_i + t_ij (eq. 2):
+// the holder pushes the chunk into a landing slot in the next relay's arena
+// and posts that chunk's flag.  The last holder writes the destination block
+// (DIRECT) or pushes into a landing slot that the destination copies out
+// (STAGED).
+void plan_flow(Builder& B, int src, int dst, const std::vector<int>* hops, const Stream& in,
+               const BufRef& out, uint64_t lo, uint64_t hi, uint32_t ce, Mode mode) {
+  const int es = B.esize_;
+  const uint32_t nch = (uint32_t)((hi - lo + ce - 1) / ce);
+  const uint64_t len = (hi - lo) * es;
+  Stream cur = in;
+  int at = src;
+  auto push = [&](int to) {
+    const uint64_t off = B.alloc(to, len);
+    const FlagRef fl = B.alloc_flags(to, nch);
+    B.add(at, lo, hi, ce, kOpFold, {cur}, {make_ref(kBufArena, to, (int64_t)off - (int64_t)(lo * es))}, {fl});
+    cur = B.slot_stream(to, off, lo, &fl);
+    at = to;
+  };
+  if (hops)
+    for (int h : *hops) push(h);
+  if (mode == kStaged && at != dst) push(dst);
+  B.add(at, lo, hi, ce, kOpFold, {cur}, {out}, {});
+}
+
 void plan_alltoall_line(Builder& B, const SubColl& s, uint64_t lo, uint64_t hi, uint64_t cnt,
                         uint64_t mask, Mode mode) {
   const int n = B.n_;
   const int es = B.esize_;
   const uint32_t ce = (uint32_t)(s.chunk / es);
-  const uint32_t nch = (uint32_t)((hi - lo + ce - 1) / ce);
-  const uint64_t len = (hi - lo) * es;
   for (int src = 0; src < n; ++src) {
     if (!((mask >> src) & 1)) continue;
     for (int d = 0; d < n; ++d) {
       Stream in;
       in.ref = make_ref(kBufSend, src, (int64_t)(d * cnt * es));
-      BufRef out = make_ref(kBufRecv, d, (int64_t)(src * cnt * es));
-      if (mode == kDirect || d == src) {
-        B.add(src, lo, hi, ce, kOpFold, {in}, {out}, {});
-        continue;
-      }
-      uint64_t off = B.alloc(d, len);
-      FlagRef fl = B.alloc_flags(d, nch);
-      B.add(src, lo, hi, ce, kOpFold, {in},
-            {make_ref(kBufArena, d, (int64_t)off - (int64_t)(lo * es))}, {fl});
-      B.add(d, lo, hi, ce, kOpFold, {B.slot_stream(d, off, lo, &fl)}, {out}, {});
+      plan_flow(B, src, d, s.hops(src, d), in, make_ref(kBufRecv, d, (int64_t)(src * cnt * es)), lo, hi,
+                ce, mode);
     }
   }
 }
@@ -359,19 +378,10 @@ void plan_alltoallv(Builder& B, const PlanRequest& rq, uint64_t k, uint64_t nseg
         const uint64_t lo = std::min(b[m + 1], b[m] + k * step), hi = std::min(b[m + 1], b[m] + (k + 1) * step);
         if (lo >= hi) continue;
         const SubColl& s = st.subs[m];
-        const uint32_t ce = (uint32_t)(s.chunk / es);
-        const uint32_t nch = (uint32_t)((hi - lo + ce - 1) / ce);
         Stream in;
         in.ref = make_ref(kBufSend, src, (int64_t)(soff * es));
-        BufRef out = make_ref(kBufRecv, d, (int64_t)(roff * es));
-        if (rq.mode == kDirect || d == src) {
-          B.add(src, lo, hi, ce, kOpFold, {in}, {out}, {});
-          continue;
-        }
-        uint64_t off = B.alloc(d, (hi - lo) * es);
-        FlagRef fl = B.alloc_flags(d, nch);
-        B.add(src, lo, hi, ce, kOpFold, {in}, {make_ref(kBufArena, d, (int64_t)off - (int64_t)(lo * es))}, {fl});
-        B.add(d, lo, hi, ce, kOpFold, {B.slot_stream(d, off, lo, &fl)}, {out}, {});
+        plan_flow(B, src, d, s.hops(src, d), in, make_ref(kBufRecv, d, (int64_t)(roff * es)), lo, hi,
+                  (uint32_t)(s.chunk / es), rq.mode);
       }
     }
   }

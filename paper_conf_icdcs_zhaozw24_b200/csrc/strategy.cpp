@@ -94,6 +94,46 @@ void finish_tree(SubColl* s, int n) {
   }
 }
 
+// route=<s>:<d>:<h1>,<h2>,..[;<s>:<d>:<h>,..]: each entry is one
+// flow's path (eq. 1: leaves src, enters dst, conserved at every relay).
+bool parse_routes(const std::string& v, int n, std::vector<Route>* out, std::string* err) {
+  size_t a = 0;
+  while (true) {
+    size_t b = v.find(';', a);
+    const std::string ent = v.substr(a, b == std::string::npos ? std::string::npos : b - a);
+    const size_t c1 = ent.find(':');
+    const size_t c2 = c1 == std::string::npos ? c1 : ent.find(':', c1 + 1);
+    if (c2 == std::string::npos) return fail(err, "route entry must be src:dst:hops");
+    int64_t sv = 0, dv = 0;
+    std::vector<int64_t> hv;
+    if (!parse_int(ent.substr(0, c1), &sv) || !parse_int(ent.substr(c1 + 1, c2 - c1 - 1), &dv) ||
+        !parse_list(ent.substr(c2 + 1), &hv))
+      return fail(err, "bad route entry");
+    if (sv < 0 || sv >= n || dv < 0 || dv >= n) return fail(err, "route rank out of range");
+    if (sv == dv) return fail(err, "route src == dst");
+    if (hv.empty()) return fail(err, "route needs at least one relay");
+    Route r;
+    r.src = (int)sv;
+    r.dst = (int)dv;
+    uint64_t seen = (uint64_t(1) << sv) | (uint64_t(1) << dv);
+    for (int64_t h : hv) {
+      if (h < 0 || h >= n) return fail(err, "route relay out of range");
+      if ((seen >> h) & 1) return fail(err, "route visits a rank twice");
+      seen |= uint64_t(1) << h;
+      r.hops.push_back((int)h);
+    }
+    for (const Route& o : *out)
+      if (o.src == r.src && o.dst == r.dst) return fail(err, "two routes for one flow");
+    out->push_back(std::move(r));
+    if (b == std::string::npos) break;
+    a = b + 1;
+  }
+  std::sort(out->begin(), out->end(), [](const Route& x, const Route& y) {
+    return x.src != y.src ? x.src < y.src : x.dst < y.dst;
+  });
+  return true;
+}
+
 uint64_t fnv1a(const std::string& s) {
   uint64_t h = 1469598103934665603ull;
   for (unsigned char c : s) { h ^= c; h *= 1099511628211ull; }
@@ -185,6 +225,7 @@ bool parse_strategy(const char* text, Strategy* out, std::string* err) {
     if (r.head == "rtree") { required.push_back("parent"); required.push_back("dst"); optional.push_back("noagg"); }
     if (r.head == "ring") required.push_back("order");
     if (r.head == "bcast") { required.push_back("parent"); required.push_back("src"); }
+    if (r.head == "a2a") optional.push_back("route");
     for (auto& k : required)
       if (!r.kv.count(k)) return fail(err, r.head + ": missing key " + k);
     for (auto& kv : r.kv) {
@@ -226,6 +267,7 @@ bool parse_strategy(const char* text, Strategy* out, std::string* err) {
     s.chunk = c;
     if (r.head == "a2a") {
       s.kind = kA2A;
+      if (r.kv.count("route") && !parse_routes(r.kv.at("route"), n, &s.routes, err)) return false;
       st.subs.push_back(std::move(s));
       continue;
     }
@@ -282,6 +324,12 @@ bool parse_strategy(const char* text, Strategy* out, std::string* err) {
   st.hash = fnv1a(norm);
   *out = std::move(st);
   return true;
+}
+
+const std::vector<int>* SubColl::hops(int s, int d) const {
+  for (const Route& r : routes)
+    if (r.src == s && r.dst == d) return &r.hops;
+  return nullptr;
 }
 
 std::vector<uint64_t> partition(uint64_t count, int esize, const std::vector<int64_t>& weights) {

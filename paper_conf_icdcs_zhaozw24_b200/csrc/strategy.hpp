@@ -26,6 +26,13 @@ enum Coll : int {
 constexpr int kNumColl = 6;
 enum SubKind : int { kTree = 0, kBcast = 1, kA2A = 2, kRTree = 3 };
 
+// One routed AlltoAll flow (routing variables x^f_ij, eq. 1): block
+// src -> dst travels src -> hops[0] -> ... -> hops.back() -> dst.
+struct Route {
+  int src = -1, dst = -1;
+  std::vector<int> hops;
+};
+
 struct SubColl {
   SubKind kind = kTree;
   int64_t weight = 0;          // effective integer weight (ring chains: w, others: w*n)
@@ -35,6 +42,9 @@ struct SubColl {
   int src = -1;                // bcast: source; rtree: destination block (== root)
   int root = -1;
   std::vector<std::vector<int>> children;  // ascending rank order (reading Q5)
+  std::vector<Route> routes;   // a2a: flows that do not go direct (sorted by (src, dst))
+  // a2a: relay ranks of flow src -> dst (empty = direct)
+  const std::vector<int>* hops(int src, int dst) const;
 };
 
 struct Strategy {

@@ -189,6 +189,47 @@ def alltoall_direct(n, chunk=1 << 20, lines=1):
         f"a2a weight=1 chunk={int(chunk)}\n" for _ in range(lines))
 
 
+def alltoall_routed(n, lines, chunk=1 << 20):
+    """AlltoAll with explicit routes (routing variables x^f_ij, eq. 1).
+    lines: list of (weight, {(s, d): [h1, ..]}) -- one a2a line each; flows
+    absent from a line's dict go direct."""
+    out = _header(n, "alltoall")
+    for w, routes in lines:
+        out += f"a2a weight={int(w)} chunk={int(chunk)}"
+        if routes:
+            out += " route=" + ";".join(f"{s}:{d}:{_join(h)}" for (s, d), h in sorted(routes.items()))
+        out += "\n"
+    return out
+
+
+def alltoall_detour(n, slow_edges, chunk=1 << 20, direct_weight=0, routed_weight=1):
+    """Route AlltoAll around slow links (the synthesizer's routing decision,
+    P:L171, under the load model of P:L209-211): every flow s -> d whose direct
+    edge is slow takes a two-hop path s -> h -> d through the relay h whose two
+    edges carry the fewest flows so far (both fast).  direct_weight > 0 adds a
+    direct a2a line, so that routed_weight : direct_weight of every block is
+    detoured and the rest still uses the slow edge (multi-path split)."""
+    slow = set(slow_edges)
+    load = {(i, j): 1 for i in range(n) for j in range(n) if i != j and (i, j) not in slow}
+    routes = {}
+    for (s, d) in sorted(slow):
+        best = None
+        for h in range(n):
+            if h in (s, d) or (s, h) in slow or (h, d) in slow:
+                continue
+            cost = max(load[(s, h)], load[(h, d)])
+            if best is None or cost < best[0]:
+                best = (cost, h)
+        if best is None:
+            continue                       # no fast detour: stays direct
+        h = best[1]
+        load[(s, h)] += 1
+        load[(h, d)] += 1
+        routes[(s, d)] = [h]
+    lines = [(routed_weight, routes)] + ([(direct_weight, {})] if direct_weight else [])
+    return alltoall_routed(n, lines, chunk)
+
+
 # ----------------------------------------------------- NEXT-4 primitives
 def reduce_trees(parents, weights=None, chunk=DEFAULT_CHUNK, noaggs=None):
     """Reduce: every tree must be rooted at the Reduce root."""

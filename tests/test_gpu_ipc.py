@@ -87,6 +87,16 @@ def _worker(rank, n, port, case, q):
                 torch.cuda.synchronize()
                 exp = oc.alltoall(xs, G.alltoall_direct(n), R, "f32", prev)[rank]
                 results.append(np.array_equal(bits(to_host(y, "f32")), bits(exp)))
+            if n >= 3:   # routed flows (eq. 1): store-and-forward through relay arenas
+                routed = G.alltoall_routed(n, [(1, {(0, n - 1): list(range(1, n - 1)), (n - 1, 1): [0]}),
+                                               (2, {})], chunk=4096)
+                comm.set_strategy("alltoall", routed)
+                for R in (set(range(n)), {0}):
+                    y = to_dev(prev[rank], "f32")
+                    comm.alltoall(to_dev(xs[rank], "f32"), y, ready=R)
+                    torch.cuda.synchronize()
+                    exp = oc.alltoall(xs, routed, R, "f32", prev)[rank]
+                    results.append(np.array_equal(bits(to_host(y, "f32")), bits(exp)))
         err = comm.get_async_error()
         comm.finalize()
         dist.destroy_process_group()

@@ -82,6 +82,16 @@ def _worker(rank, n, port, engine, q):
         a2a = oc.alltoall([a[:n * cnt] for a in xs], G.alltoall_direct(n), set(range(n)), "f32",
                           [np.zeros(n * cnt, np.float32)] * n)
         ok.append(np.array_equal(y[:n * cnt].cpu().numpy(), a2a[rank]))
+        if n >= 3:   # routed flows (eq. 1): each relay forwards through its own arena
+            routed = G.alltoall_routed(n, [(2, {(g, (g + 1) % n): [(g + 2) % n] for g in range(n)}), (1, {})],
+                                       chunk=4096)
+            comm.set_strategy("alltoall", routed)
+            y.zero_()
+            comm.collective_zc("alltoall", x[:n * cnt], y[:n * cnt], cnt, ready=set(range(1, n)))
+            torch.cuda.synchronize()
+            a2a = oc.alltoall([a[:n * cnt] for a in xs], routed, set(range(1, n)), "f32",
+                              [np.zeros(n * cnt, np.float32)] * n)
+            ok.append(np.array_equal(y[:n * cnt].cpu().numpy(), a2a[rank]))
         err = comm.get_async_error()
         comm.deregister(rx)
         comm.deregister(ry)
