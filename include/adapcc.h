@@ -255,6 +255,29 @@ ADAPCC_API adapcc_result_t adapcc_signal_ready(adapcc_comm_t comm, int rank, uin
 
 /* Latched device error (TIMEOUT) or SUCCESS.  Does not synchronize. */
 ADAPCC_API adapcc_result_t adapcc_get_async_error(adapcc_comm_t comm);
+/* NEXT-3 fault tolerance ("the coordinator identifies the
+ * remaining non-ready workers as faulty workers ... excluded from the training
+ * group"; "graph reconstruction" without restarting the job).
+ * Survivors exclude the ranks in dead_mask and keep the communicator: arenas,
+ * IPC mappings and registered buffers stay; a latched TIMEOUT is cleared; the
+ * device epoch restarts above every flag posted so far; every collective's
+ * strategy is reset to the survivors' default (AllReduce: one star per live
+ * rank).  Afterwards excluded ranks are never ready, own no work, and none of
+ * their buffers or arena bytes is read or written; set_strategy accepts a
+ * strategy that names them only as tree leaves (not AlltoAll relays, Reduce
+ * roots or Broadcast sources).  Collective over the SURVIVORS: each calls it
+ * with the same dead_mask and an all-gather `ag` over exactly the survivors
+ * (ascending rank order; ag may be NULL in loopback).  Host-blocking: waits for
+ * this device to drain.  Precondition: the excluded ranks' GPU work has stopped
+ * (their launches exit at the watchdog deadline).  CUDA graphs captured before
+ * the call must not be replayed after it.  INVALID_ARGUMENT: bits >= nranks,
+ * nothing left alive, or (multi-process) this rank excluded / ag NULL. */
+ADAPCC_API adapcc_result_t adapcc_exclude(adapcc_comm_t comm, uint64_t dead_mask,
+                               adapcc_bootstrap_allgather_fn ag, void* ag_ctx);
+
+/* Live ranks (all ranks until adapcc_exclude). */
+ADAPCC_API adapcc_result_t adapcc_members(adapcc_comm_t comm, uint64_t* members);
+
 /* Synchronizes the device, unmaps peers, frees everything.  comm may be NULL. */
 ADAPCC_API adapcc_result_t adapcc_finalize(adapcc_comm_t comm);
 ADAPCC_API const char* adapcc_strerror(adapcc_result_t r);
@@ -308,7 +331,10 @@ ADAPCC_API adapcc_result_t adapcc_strategy_partition(const char* strategy_text, 
                                           adapcc_dtype_t dtype, int src, uint64_t* bounds,
                                           int* nbounds);
 
-/* Plan statistics for one rank (-1 = all virtual ranks) of a call. */
+/* Plan statistics for one rank (-1 = all virtual ranks) of a call, with the
+ * live-rank set `members` (0 = all ranks; see adapcc_exclude): INVALID_STRATEGY
+ * if the strategy gives an excluded rank work, INVALID_ARGUMENT if the ready
+ * mask names one. */
 typedef struct {
   uint64_t tasks;         /* fold/copy tasks */
   uint64_t items;         /* (task, chunk) work items */
@@ -323,7 +349,7 @@ typedef struct {
 ADAPCC_API adapcc_result_t adapcc_plan_stats(const char* strategy_text, uint64_t count,
                                   adapcc_dtype_t dtype, uint64_t ready_mask, unsigned flags,
                                   adapcc_mode_t mode, int rank, size_t scratch_bytes,
-                                  adapcc_plan_stats_t* stats);
+                                  uint64_t members, adapcc_plan_stats_t* stats);
 
 #ifdef __cplusplus
 }

@@ -96,6 +96,8 @@ def _load():
         "adapcc_config": [vp, ctypes.c_char_p, i64],
         "adapcc_launch_count": [vp, ctypes.POINTER(u64)],
         "adapcc_last_engine": [vp, ctypes.POINTER(i32)],
+        "adapcc_exclude": [vp, u64, AG_FN, vp],
+        "adapcc_members": [vp, ctypes.POINTER(u64)],
         "adapcc_strategy_check": [ctypes.c_char_p, ctypes.POINTER(i32), ctypes.POINTER(i32),
                                   ctypes.POINTER(i32), ctypes.c_char_p, sz],
         "adapcc_strategy_tuples": [ctypes.c_char_p, i32, u64, ctypes.POINTER(ctypes.c_uint8),
@@ -106,7 +108,7 @@ def _load():
                                   ctypes.POINTER(i32)],
         "adapcc_strategy_partition": [ctypes.c_char_p, u64, i32, i32, ctypes.POINTER(u64),
                                       ctypes.POINTER(i32)],
-        "adapcc_plan_stats": [ctypes.c_char_p, u64, i32, u64, ctypes.c_uint, i32, i32, sz,
+        "adapcc_plan_stats": [ctypes.c_char_p, u64, i32, u64, ctypes.c_uint, i32, i32, sz, u64,
                               ctypes.POINTER(PlanStats)],
     }
     for name, args in sig.items():
@@ -222,12 +224,15 @@ def strategy_partition(text, count, dtype, src=-1):
     return list(b[:nb.value])
 
 
-def plan_stats(text, count, dtype, mask, accumulate=False, mode="direct", rank=-1, scratch_bytes=0):
+def plan_stats(text, count, dtype, mask, accumulate=False, mode="direct", rank=-1, scratch_bytes=0,
+               members=None):
+    """Byte/task accounting of a call's plan; members: live ranks (None = all)."""
     L = _load()
     st = PlanStats()
+    mm = 0 if members is None else sum(1 << g for g in members)
     _check(L.adapcc_plan_stats(text.encode(), count, DTYPE_CODE[dtype], mask,
                                FLAG_ACCUMULATE if accumulate else 0, MODE[mode], rank,
-                               scratch_bytes, ctypes.byref(st)), "plan_stats")
+                               scratch_bytes, mm, ctypes.byref(st)), "plan_stats")
     return st.as_dict()
 
 
@@ -257,6 +262,31 @@ def make_bootstrap_allgather(group=None, device=None):
     return AG_FN(ag)
 
 
+def make_store_allgather(ranks, rank, store=None, tag="adapcc"):
+    """ctypes all-gather callback over `ranks` only (ascending order), through
+    the torch.distributed key-value store -- usable after a fault, when the
+    faulty ranks cannot take part in a process-group collective (NEXT-3)."""
+    import torch.distributed as dist
+    store = store if store is not None else dist.distributed_c10d._get_default_store()
+    ranks = sorted(ranks)
+    seq = [0]
+
+    def ag(send, recv, nbytes, _ctx):
+        try:
+            seq[0] += 1
+            pre = f"{tag}/{seq[0]}/"
+            store.set(pre + str(rank), ctypes.string_at(send, nbytes))
+            keys = [pre + str(r) for r in ranks]
+            store.wait(keys)
+            blob = b"".join(bytes(store.get(k)) for k in keys)
+            ctypes.memmove(recv, blob, len(blob))
+            return 0
+        except Exception:  # noqa: BLE001 -- reported as ADAPCC_ERR_BOOTSTRAP
+            return 1
+
+    return AG_FN(ag)
+
+
 class Communicator:
     """A communicator (the paper's transmission contexts)."""
 
@@ -267,6 +297,28 @@ class Communicator:
         self.device = device
         self.loopback = loopback
         self._keep = keep
+        self.members = set(range(nranks))
+
+    def _ready_mask(self, ready):
+        return _mask(self.members if ready is None else ready, self.nranks)
+
+    # ---- fault tolerance (NEXT-3)
+    def exclude(self, dead, store=None):
+        """Exclude faulty ranks; collective over the survivors.
+        Multi-process: the survivors all-gather through the distributed store."""
+        dead = set(dead)
+        live = self.members - dead
+        mask = _mask(dead, self.nranks)
+        if self.loopback:
+            cb = AG_FN()
+        else:
+            tag = f"adapcc-exclude/{_mask(live, self.nranks)}"
+            cb = make_store_allgather(live, self.rank, store, tag)
+            self._keep_exclude = cb      # the library calls it again for registrations
+        _check(_load().adapcc_exclude(self._h, mask, cb, None), "exclude")
+        v = ctypes.c_uint64()
+        _check(_load().adapcc_members(self._h, ctypes.byref(v)), "members")
+        self.members = {g for g in range(self.nranks) if (v.value >> g) & 1}
 
     # ---- construction
     @classmethod
@@ -327,7 +379,7 @@ class Communicator:
     # ---- multi-process collectives
     def allreduce(self, x, out=None, ready=None, accumulate=False, stream=None):
         out = x if out is None else out
-        m = _mask(ready, self.nranks)
+        m = self._ready_mask(ready)
         send = x if (m >> self.rank) & 1 else None
         _check(_load().adapcc_allreduce(self._h, _ptr(send), _ptr(out), out.numel(),
                                         _dtype_code(out), m,
@@ -336,7 +388,7 @@ class Communicator:
         return out
 
     def allgather(self, x, out, ready=None, stream=None):
-        m = _mask(ready, self.nranks)
+        m = self._ready_mask(ready)
         send = x if (m >> self.rank) & 1 else None
         cnt = out.numel() // self.nranks
         _check(_load().adapcc_allgather(self._h, _ptr(send), _ptr(out), cnt, _dtype_code(out), m,
@@ -344,7 +396,7 @@ class Communicator:
         return out
 
     def alltoall(self, x, out, ready=None, stream=None):
-        m = _mask(ready, self.nranks)
+        m = self._ready_mask(ready)
         send = x if (m >> self.rank) & 1 else None
         cnt = out.numel() // self.nranks
         _check(_load().adapcc_alltoall(self._h, _ptr(send), _ptr(out), cnt, _dtype_code(out), m,
@@ -353,7 +405,7 @@ class Communicator:
 
     def reduce(self, x, out, root, ready=None, accumulate=False, stream=None):
         """Only the root's `out` is written (non-roots may pass None)."""
-        m = _mask(ready, self.nranks)
+        m = self._ready_mask(ready)
         send = x if (m >> self.rank) & 1 else None
         n_el = (out if out is not None else x).numel()
         _check(_load().adapcc_reduce(self._h, _ptr(send), _ptr(out), n_el,
@@ -362,14 +414,14 @@ class Communicator:
         return out
 
     def broadcast(self, x, out, root, ready=None, stream=None):
-        m = _mask(ready, self.nranks)
+        m = self._ready_mask(ready)
         send = x if (self.rank == root and (m >> root) & 1) else None
         _check(_load().adapcc_broadcast(self._h, _ptr(send), _ptr(out), out.numel(), _dtype_code(out),
                                         root, m, _stream(stream)), "broadcast")
         return out
 
     def reducescatter(self, x, out, ready=None, accumulate=False, stream=None):
-        m = _mask(ready, self.nranks)
+        m = self._ready_mask(ready)
         send = x if (m >> self.rank) & 1 else None
         _check(_load().adapcc_reducescatter(self._h, _ptr(send), _ptr(out), out.numel(),
                                             _dtype_code(out), m, FLAG_ACCUMULATE if accumulate else 0,
@@ -403,7 +455,7 @@ class Communicator:
         """Any collective on registered tensors x / out (same offsets on every rank)."""
         sr, so = self._reg_of(x)
         rr, ro = self._reg_of(out)
-        m = _mask(ready, self.nranks)
+        m = self._ready_mask(ready)
         flags = (FLAG_ACCUMULATE if accumulate else 0) | _late_flag(late)
         _check(_load().adapcc_collective_zc(self._h, COLL[coll], sr, so, rr, ro, count, _dtype_code(out),
                                             root, m, flags, _stream(stream)), coll + "_zc")
@@ -425,10 +477,10 @@ class Communicator:
 
     def allreduce_lb(self, xs, outs, ready=None, accumulate=False, stream=None, late=None):
         """late: None | 'join' (phase 1) | 'complement' (phase 2)."""
-        m = _mask(ready, self.nranks)
+        m = self._ready_mask(ready)
         if late is not None:
             # phase 2 reads the late ranks' inputs: pass every input
-            S, D = self._arrays(xs, outs, (1 << self.nranks) - 1)
+            S, D = self._arrays(xs, outs, _mask(self.members, self.nranks))
         else:
             S, D = self._arrays(xs, outs, m)
         flags = (FLAG_ACCUMULATE if accumulate else 0) | _late_flag(late)
@@ -438,7 +490,7 @@ class Communicator:
 
     def alltoallv_lb(self, xs, outs, counts, ready=None, stream=None):
         """counts: nranks x nranks element counts (counts[s][d] from s to d)."""
-        m = _mask(ready, self.nranks)
+        m = self._ready_mask(ready)
         S, D = self._arrays(xs, outs, m)
         flat = (ctypes.c_uint64 * (self.nranks * self.nranks))(*[int(v) for row in counts for v in row])
         _check(_load().adapcc_alltoallv_lb(self._h, S, D, flat, _dtype_code(outs[0]), m, _stream(stream)),
@@ -446,7 +498,7 @@ class Communicator:
         return outs
 
     def alltoallv(self, x, out, counts, ready=None, stream=None):
-        m = _mask(ready, self.nranks)
+        m = self._ready_mask(ready)
         send = x if (m >> self.rank) & 1 else None
         flat = (ctypes.c_uint64 * (self.nranks * self.nranks))(*[int(v) for row in counts for v in row])
         _check(_load().adapcc_alltoallv(self._h, _ptr(send), _ptr(out), flat, _dtype_code(out), m,
@@ -463,21 +515,21 @@ class Communicator:
         _check(_load().adapcc_signal_ready(self._h, rank, ticket, _stream(stream)), "signal_ready")
 
     def allgather_lb(self, xs, outs, ready=None, stream=None):
-        m = _mask(ready, self.nranks)
+        m = self._ready_mask(ready)
         S, D = self._arrays(xs, outs, m)
         _check(_load().adapcc_allgather_lb(self._h, S, D, outs[0].numel() // self.nranks,
                                            _dtype_code(outs[0]), m, _stream(stream)), "allgather_lb")
         return outs
 
     def alltoall_lb(self, xs, outs, ready=None, stream=None):
-        m = _mask(ready, self.nranks)
+        m = self._ready_mask(ready)
         S, D = self._arrays(xs, outs, m)
         _check(_load().adapcc_alltoall_lb(self._h, S, D, outs[0].numel() // self.nranks,
                                           _dtype_code(outs[0]), m, _stream(stream)), "alltoall_lb")
         return outs
 
     def reduce_lb(self, xs, outs, root, ready=None, accumulate=False, stream=None):
-        m = _mask(ready, self.nranks)
+        m = self._ready_mask(ready)
         S, D = self._arrays(xs, outs, m)
         _check(_load().adapcc_reduce_lb(self._h, S, D, outs[root].numel(), _dtype_code(outs[root]), root,
                                         m, FLAG_ACCUMULATE if accumulate else 0, _stream(stream)),
@@ -485,14 +537,14 @@ class Communicator:
         return outs
 
     def broadcast_lb(self, xs, outs, root, ready=None, stream=None):
-        m = _mask(ready, self.nranks)
+        m = self._ready_mask(ready)
         S, D = self._arrays(xs, outs, m)
         _check(_load().adapcc_broadcast_lb(self._h, S, D, outs[0].numel(), _dtype_code(outs[0]), root, m,
                                            _stream(stream)), "broadcast_lb")
         return outs
 
     def reducescatter_lb(self, xs, outs, ready=None, accumulate=False, stream=None):
-        m = _mask(ready, self.nranks)
+        m = self._ready_mask(ready)
         S, D = self._arrays(xs, outs, m)
         _check(_load().adapcc_reducescatter_lb(self._h, S, D, outs[0].numel(), _dtype_code(outs[0]), m,
                                                FLAG_ACCUMULATE if accumulate else 0, _stream(stream)),

@@ -145,3 +145,14 @@ def faulty_workers(ready_times, phase1_end, now, factor=T_FAULT_FACTOR):
     if now - phase1_end < t_fault:
         return set()
     return {r for r, t in ready_times.items() if t is None}
+
+
+def exclude_faulty(comm, ready_times, phase1_end, now, factor=T_FAULT_FACTOR, store=None):
+    """P:L139-146 end to end: identify the faulty workers with the T_fault rule
+    and exclude them from the communicator (adapcc_exclude), after which the
+    survivors continue on the same arenas with the survivors' default
+    strategy.  Returns the set excluded (empty: nothing to do yet)."""
+    faulty = faulty_workers(ready_times, phase1_end, now, factor) & set(comm.members)
+    if faulty:
+        comm.exclude(faulty, store=store)
+    return faulty

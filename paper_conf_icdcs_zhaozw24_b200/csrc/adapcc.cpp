@@ -66,7 +66,7 @@ struct DevPlan {
   }
 };
 
-using PlanKey = std::tuple<int, uint64_t, uint64_t, int, uint64_t, unsigned, int>;  // ..., plan mode
+using PlanKey = std::tuple<int, uint64_t, uint64_t, int, uint64_t, unsigned, int, uint64_t>;  // ..., mode, members
 
 // A buffer registered for zero-copy collectives: base[q] is where rank q's
 // registered region starts in THIS process's address space (peer-mapped).
@@ -85,8 +85,10 @@ std::string star(int n, int root) {
 }
 
 // Defaults; Reduce / Broadcast defaults are generated for the
-// call's root: one star tree (all trees of a Reduce share the root).
-std::string default_strategy(Coll c, int n, int root = 0) {
+// call's root: one star tree (all trees of a Reduce share the root).  After a
+// fault exclusion (NEXT-3) the AllReduce default keeps only the stars rooted at
+// live ranks; excluded ranks are leaves of every star.
+std::string default_strategy(Coll c, int n, int root = 0, uint64_t members = ~uint64_t(0)) {
   std::string s = "adapcc-strategy 1\nnranks " + std::to_string(n) + "\ncollective ";
   if (c == kReduce) return s + "reduce\ntree weight=1 chunk=262144 parent=" + star(n, root) + "\n";
   if (c == kBroadcast)
@@ -100,6 +102,7 @@ std::string default_strategy(Coll c, int n, int root = 0) {
   if (c == kAllReduce) {
     s += "allreduce\n";
     for (int m = 0; m < n; ++m) {  // n star trees, equal weights
+      if (!((members >> m) & 1)) continue;
       s += "tree weight=1 chunk=262144 parent=";
       for (int g = 0; g < n; ++g) s += (g ? "," : "") + std::to_string(g == m ? -1 : m);
       s += "\n";
@@ -145,6 +148,7 @@ struct adapcc_comm_s {
   int64_t timeout_ms = 10000;
   int64_t max_ctas = 0;
   int64_t drop_rank = -1;
+  uint64_t members = 0;   // live ranks (NEXT-3 fault exclusion); all ranks after init
   uint64_t late_seq = 0;  // late-join ticket of the most recent LATE_JOIN call
   int64_t piece_kib = 0;  // 0 = automatic (total traffic / (8 * grid))
   uint64_t launches = 0;
@@ -198,6 +202,7 @@ adapcc_result_t common_init(adapcc_comm_s* c, size_t scratch) {
     for (int k = 0; k < 3; ++k)
       if (c->occ[k][d] < 1) c->occ[k][d] = 1;
   }
+  c->members = c->nranks >= 64 ? ~uint64_t(0) : ((uint64_t(1) << c->nranks) - 1);
   CK(cudaMalloc(&c->state, sizeof(DevState)));
   CK(cudaMemset(c->state, 0, sizeof(DevState)));
   CK(cudaHostAlloc(&c->h_err, sizeof(int), cudaHostAllocMapped));
@@ -237,6 +242,9 @@ adapcc_result_t check_common(adapcc_comm_t c, adapcc_dtype_t dtype, uint64_t mas
   if (dtype != ADAPCC_FLOAT32 && dtype != ADAPCC_BFLOAT16 && dtype != ADAPCC_INT32)
     return ADAPCC_ERR_INVALID_ARGUMENT;
   if (c->nranks < 64 && (mask >> c->nranks) != 0) return ADAPCC_ERR_INVALID_ARGUMENT;
+  // an excluded rank is never ready and, in multi-process mode, makes no calls
+  if ((mask & ~c->members) || (!c->loopback && !((c->members >> c->rank) & 1)))
+    return ADAPCC_ERR_INVALID_ARGUMENT;
   if (*reinterpret_cast<volatile int*>(c->h_err)) return (adapcc_result_t)*c->h_err;
   return ADAPCC_SUCCESS;
 }
@@ -279,7 +287,7 @@ adapcc_result_t pick_strategy(adapcc_comm_s* c, Coll coll, int root, const Strat
     *out = &c->strat[coll];
     return ADAPCC_SUCCESS;
   }
-  if (root < 0 || root >= c->nranks) return ADAPCC_ERR_INVALID_ARGUMENT;
+  if (root < 0 || root >= c->nranks || !((c->members >> root) & 1)) return ADAPCC_ERR_INVALID_ARGUMENT;
   if (c->user_set[coll]) {
     const Strategy& st = c->strat[coll];
     const int sroot = coll == kReduce ? st.subs[0].root : st.subs[0].src;
@@ -309,7 +317,7 @@ adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, const Strategy* strat, uin
     count = h;
     coll = (Coll)kNumColl;  // distinct plan-cache namespace
   }
-  PlanKey key{(int)coll, strat->hash, count, (int)dtype, mask, flags, (int)mode};
+  PlanKey key{(int)coll, strat->hash, count, (int)dtype, mask, flags, (int)mode, c->members};
   auto it = c->plans.find(key);
   if (it != c->plans.end()) {
     it->second->last_tick = ++c->tick;
@@ -324,6 +332,7 @@ adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, const Strategy* strat, uin
   rq.accumulate = flags & ADAPCC_FLAG_ACCUMULATE;
   rq.late_join = flags & ADAPCC_FLAG_LATE_JOIN;
   rq.counts = counts;
+  rq.members = c->members;
   rq.mode = mode;
   rq.half_bytes = c->half_bytes;
   std::vector<SegmentPlan> segs;
@@ -418,6 +427,7 @@ adapcc_result_t run(adapcc_comm_s* c, Coll coll, const void* const* send, void* 
     P.late_ticket = c->late_seq;
     P.late_bits = seg.late_bits;
     P.drop_rank = (int)c->drop_rank;
+    P.members = c->members;
     P.half_bytes = c->half_bytes;
     P.timeout_ns = (uint64_t)std::max<int64_t>(1, c->timeout_ms) * 1000000ull;
     P.state = c->state;
@@ -547,6 +557,7 @@ adapcc_result_t adapcc_set_strategy(adapcc_comm_t c, adapcc_coll_t coll, const c
   if (!parse_strategy(text, &st, &err)) return ADAPCC_ERR_INVALID_STRATEGY;
   if (st.nranks != c->nranks || (int)st.coll != (int)coll) return ADAPCC_ERR_INVALID_STRATEGY;
   std::lock_guard<std::mutex> lock(c->mu);
+  if (!check_members(st, c->members, &err)) return ADAPCC_ERR_INVALID_STRATEGY;
   c->strat[coll] = std::move(st);
   c->user_set[coll] = true;
   return ADAPCC_SUCCESS;
@@ -607,6 +618,7 @@ static adapcc_result_t check_lb(adapcc_comm_t c, const void* const* s, void* con
                                 size_t rbytes, uint64_t mask, int kind) {
   if (!c->loopback || !s || !d) return ADAPCC_ERR_INVALID_ARGUMENT;
   for (int q = 0; q < c->nranks; ++q) {
+    if (!((c->members >> q) & 1)) continue;  // excluded: buffers never touched
     const bool ready = (mask >> q) & 1;
     if (rbytes && !d[q]) return ADAPCC_ERR_INVALID_ARGUMENT;
     if (misaligned(d[q])) return ADAPCC_ERR_INVALID_ARGUMENT;
@@ -739,11 +751,13 @@ adapcc_result_t adapcc_broadcast_lb(adapcc_comm_t c, const void* const* sendbufs
   if (!c->loopback || !sendbufs || !recvbufs || root < 0 || root >= c->nranks) return ADAPCC_ERR_INVALID_ARGUMENT;
   const size_t bytes = count * esize_of(dtype);
   for (int q = 0; q < c->nranks; ++q)
-    if ((count && !recvbufs[q]) || misaligned(recvbufs[q])) return ADAPCC_ERR_INVALID_ARGUMENT;
+    if (((c->members >> q) & 1) && ((count && !recvbufs[q]) || misaligned(recvbufs[q])))
+      return ADAPCC_ERR_INVALID_ARGUMENT;
   if ((mask >> root) & 1) {
     if ((count && !sendbufs[root]) || misaligned(sendbufs[root])) return ADAPCC_ERR_INVALID_ARGUMENT;
     for (int q = 0; q < c->nranks; ++q)
-      if (!(q == root && sendbufs[root] == recvbufs[q]) && overlap(sendbufs[root], bytes, recvbufs[q], bytes))
+      if (((c->members >> q) & 1) && !(q == root && sendbufs[root] == recvbufs[q]) &&
+          overlap(sendbufs[root], bytes, recvbufs[q], bytes))
         return ADAPCC_ERR_INVALID_ARGUMENT;
   }
   return run(c, kBroadcast, sendbufs, recvbufs, count, dtype, mask, 0, stream, root);
@@ -763,6 +777,20 @@ adapcc_result_t adapcc_reducescatter_lb(adapcc_comm_t c, const void* const* send
 
 // ------------------------------------------------------- zero-copy registration
 namespace {
+// All-gather over the live ranks (the bootstrap callback covers exactly them:
+// the original group, or the survivors' group handed to adapcc_exclude);
+// entry q of `out` is rank q's blob, zero for excluded ranks.
+int members_allgather(adapcc_comm_s* c, const void* mine, void* out, size_t bytes) {
+  const int k = __builtin_popcountll(c->members);
+  std::vector<char> tmp((size_t)k * bytes);
+  if (c->ag(mine, tmp.data(), bytes, c->ag_ctx) != 0) return 1;
+  char* o = static_cast<char*>(out);
+  std::memset(o, 0, (size_t)c->nranks * bytes);
+  for (int q = 0, i = 0; q < c->nranks; ++q)
+    if ((c->members >> q) & 1) std::memcpy(o + (size_t)q * bytes, tmp.data() + (size_t)(i++) * bytes, bytes);
+  return 0;
+}
+
 // base address of the allocation containing p (driver API, loaded lazily so
 // the library still loads on machines without a driver)
 bool allocation_base(void* p, char** base) {
@@ -794,9 +822,9 @@ adapcc_result_t adapcc_register_buffer(adapcc_comm_t c, void* ptr, size_t bytes,
   me.bytes = bytes;
   me.id = c->next_reg;
   std::vector<Blob> all(c->nranks);
-  if (c->ag(&me, all.data(), sizeof(Blob), c->ag_ctx) != 0) return ADAPCC_ERR_BOOTSTRAP;
-  for (auto& b : all)
-    if (b.bytes != bytes || b.id != me.id) return ADAPCC_ERR_MISMATCH;
+  if (members_allgather(c, &me, all.data(), sizeof(Blob)) != 0) return ADAPCC_ERR_BOOTSTRAP;
+  for (int q = 0; q < c->nranks; ++q)
+    if (((c->members >> q) & 1) && (all[q].bytes != bytes || all[q].id != me.id)) return ADAPCC_ERR_MISMATCH;
   RegBuf rb;
   rb.bytes = bytes;
   rb.base.assign(c->nranks, nullptr);
@@ -806,6 +834,7 @@ adapcc_result_t adapcc_register_buffer(adapcc_comm_t c, void* ptr, size_t bytes,
       rb.base[q] = static_cast<char*>(ptr);
       continue;
     }
+    if (!((c->members >> q) & 1)) continue;  // excluded peer: never addressed
     std::string key(reinterpret_cast<const char*>(&all[q].h), sizeof(cudaIpcMemHandle_t));
     auto it = c->opened.find({q, key});
     if (it == c->opened.end()) {
@@ -918,6 +947,7 @@ adapcc_result_t adapcc_alltoallv_lb(adapcc_comm_t c, const void* const* sendbufs
     r = a2av_sizes(c, counts, q, esize_of(dtype), &sb, &rb);
     if (r != ADAPCC_SUCCESS) return r;
     const bool ready = (mask >> q) & 1;
+    if (!((c->members >> q) & 1)) continue;
     if ((rb && !recvbufs[q]) || misaligned(recvbufs[q])) return ADAPCC_ERR_INVALID_ARGUMENT;
     if (ready && ((sb && !sendbufs[q]) || misaligned(sendbufs[q]))) return ADAPCC_ERR_INVALID_ARGUMENT;
     if (ready && sb && rb && overlap(sendbufs[q], sb, recvbufs[q], rb)) return ADAPCC_ERR_INVALID_ARGUMENT;
@@ -952,6 +982,65 @@ const char* adapcc_last_cuda_error(void) {
 adapcc_result_t adapcc_get_async_error(adapcc_comm_t c) {
   if (!c) return ADAPCC_ERR_INVALID_ARGUMENT;
   return (adapcc_result_t) * reinterpret_cast<volatile int*>(c->h_err);
+}
+
+// NEXT-3 fault tolerance: "faulty workers are excluded from the
+// training group"; the survivors keep the communicator (arenas, IPC mappings,
+// registrations) and continue with a strategy over the live ranks.
+adapcc_result_t adapcc_exclude(adapcc_comm_t c, uint64_t dead_mask, adapcc_bootstrap_allgather_fn ag,
+                               void* ag_ctx) {
+  if (!c) return ADAPCC_ERR_INVALID_ARGUMENT;
+  const uint64_t all = c->nranks >= 64 ? ~uint64_t(0) : ((uint64_t(1) << c->nranks) - 1);
+  if (dead_mask & ~all) return ADAPCC_ERR_INVALID_ARGUMENT;
+  std::lock_guard<std::mutex> lock(c->mu);
+  const uint64_t live = c->members & ~dead_mask;
+  if (!live || (!c->loopback && (!ag || !((live >> c->rank) & 1)))) return ADAPCC_ERR_INVALID_ARGUMENT;
+  CK(cudaSetDevice(c->device));
+  // 1. drain: launches that waited on the faulty rank have hit the watchdog and exited
+  CK(cudaDeviceSynchronize());
+  DevState st{};
+  CK(cudaMemcpy(&st, c->state, sizeof(DevState), cudaMemcpyDeviceToHost));
+  uint64_t epoch = st.epoch;
+  if (!c->loopback) {  // 2. agree on an epoch above every flag any survivor ever posted
+    c->members = live;
+    c->ag = ag;
+    c->ag_ctx = ag_ctx;
+    std::vector<uint64_t> e(c->nranks);
+    if (members_allgather(c, &epoch, e.data(), sizeof(uint64_t)) != 0) return ADAPCC_ERR_BOOTSTRAP;
+    for (uint64_t v : e) epoch = std::max(epoch, v);
+  }
+  epoch += 2;
+  // 3. restart the device epoch there: counters cleared, abort latch released;
+  //    this rank's "done" and "entered" words say it finished `epoch`, so the
+  //    next launch's start check (peers done >= epoch + 1 - 2) passes
+  st = DevState{};
+  st.epoch = epoch;
+  CK(cudaMemcpy(c->state, &st, sizeof(DevState), cudaMemcpyHostToDevice));
+  if (!c->loopback) {
+    const uint64_t words[2] = {epoch, epoch};
+    CK(cudaMemcpy(c->arena[c->rank], words, sizeof(words), cudaMemcpyHostToDevice));
+  }
+  *reinterpret_cast<volatile int*>(c->h_err) = 0;
+  c->members = live;
+  // 4. strategies: the survivors' defaults until set_strategy names new ones
+  for (int k = 0; k < kNumColl; ++k) {
+    if (!parse_strategy(default_strategy((Coll)k, c->nranks, 0, live).c_str(), &c->strat[k], nullptr))
+      return ADAPCC_ERR_INVALID_STRATEGY;
+    c->user_set[k] = false;
+    c->rooted[k].clear();
+  }
+  if (!c->loopback) {  // 5. barrier: nobody launches before every survivor has reset
+    int ok = 1;
+    std::vector<int> oks(c->nranks);
+    if (members_allgather(c, &ok, oks.data(), sizeof(int)) != 0) return ADAPCC_ERR_BOOTSTRAP;
+  }
+  return ADAPCC_SUCCESS;
+}
+
+adapcc_result_t adapcc_members(adapcc_comm_t c, uint64_t* members) {
+  if (!c || !members) return ADAPCC_ERR_INVALID_ARGUMENT;
+  *members = c->members;
+  return ADAPCC_SUCCESS;
 }
 
 adapcc_result_t adapcc_finalize(adapcc_comm_t c) {
@@ -1068,11 +1157,15 @@ adapcc_result_t adapcc_strategy_partition(const char* text, uint64_t count, adap
 
 adapcc_result_t adapcc_plan_stats(const char* text, uint64_t count, adapcc_dtype_t dtype,
                                   uint64_t mask, unsigned flags, adapcc_mode_t mode, int rank,
-                                  size_t scratch_bytes, adapcc_plan_stats_t* out) {
+                                  size_t scratch_bytes, uint64_t members, adapcc_plan_stats_t* out) {
   Strategy st;
   if (!parse_strategy(text, &st, nullptr)) return ADAPCC_ERR_INVALID_STRATEGY;
   if (!out || rank < -1 || rank >= st.nranks) return ADAPCC_ERR_INVALID_ARGUMENT;
+  if (members == 0) members = st.nranks >= 64 ? ~uint64_t(0) : ((uint64_t(1) << st.nranks) - 1);
+  if (mask & ~members) return ADAPCC_ERR_INVALID_ARGUMENT;
+  if (!check_members(st, members, nullptr)) return ADAPCC_ERR_INVALID_STRATEGY;
   PlanRequest rq;
+  rq.members = members;
   rq.st = &st;
   rq.count = count;
   rq.esize = esize_of(dtype);

@@ -226,7 +226,7 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
   // parity half of the arenas (epoch - 2) before we write into any arena
   if (P.ipc && epoch > 2) {
     const int r = threadIdx.x;
-    if (r < P.nranks && r != P.my_rank) {
+    if (r < P.nranks && r != P.my_rank && ((P.members >> r) & 1)) {
       if (!wait_flag(reinterpret_cast<const uint64_t*>(P.hdr[r]), epoch - 2, P)) sh.abort = 1;
     }
     __syncthreads();
@@ -234,7 +234,7 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
   if (P.ipc && P.zc) {  // zero-copy: peers read/write our user buffers directly
     if (blockIdx.x == 0 && threadIdx.x == 0)
       st_release(reinterpret_cast<uint64_t*>(P.hdr[P.my_rank] + 8), epoch, true);  // entered
-    if (threadIdx.x < P.nranks && threadIdx.x != P.my_rank)
+    if (threadIdx.x < P.nranks && threadIdx.x != P.my_rank && ((P.members >> threadIdx.x) & 1))
       if (!wait_flag(reinterpret_cast<const uint64_t*>(P.hdr[threadIdx.x] + 8), epoch, P)) sh.abort = 1;
     __syncthreads();
   }
@@ -347,7 +347,8 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
         st_release(reinterpret_cast<uint64_t*>(P.hdr[P.my_rank]), epoch, true);
         if (P.zc)  // our buffers stay in use until every peer has finished this call
           for (int q = 0; q < P.nranks; ++q)
-            if (q != P.my_rank) wait_flag(reinterpret_cast<const uint64_t*>(P.hdr[q]), epoch, P);
+            if (q != P.my_rank && ((P.members >> q) & 1))
+              wait_flag(reinterpret_cast<const uint64_t*>(P.hdr[q]), epoch, P);
       }
     }
   }

@@ -377,14 +377,14 @@ __global__ void __launch_bounds__(kTmaThreads, ADAPCC_TMA_MINB) engine_tma_kerne
   const unsigned par = (unsigned)(epoch & 1);
   const uint64_t half_off = kArenaHeader + par * P.half_bytes;
   if (P.ipc && epoch > 2) {  // peers done with the last user of this half
-    if (tid < P.nranks && tid != P.my_rank)
+    if (tid < P.nranks && tid != P.my_rank && ((P.members >> tid) & 1))
       if (!wait_flag(reinterpret_cast<const uint64_t*>(P.hdr[tid]), epoch - 2, P)) sm.abort = 1;
     __syncthreads();
   }
   if (P.ipc && P.zc) {  // zero-copy: peers read/write our user buffers directly
     if (blockIdx.x == 0 && tid == 0)
       st_release(reinterpret_cast<uint64_t*>(P.hdr[P.my_rank] + 8), epoch, true);  // entered
-    if (tid < P.nranks && tid != P.my_rank)
+    if (tid < P.nranks && tid != P.my_rank && ((P.members >> tid) & 1))
       if (!wait_flag(reinterpret_cast<const uint64_t*>(P.hdr[tid] + 8), epoch, P)) sm.abort = 1;
     __syncthreads();
   }
@@ -498,7 +498,8 @@ __global__ void __launch_bounds__(kTmaThreads, ADAPCC_TMA_MINB) engine_tma_kerne
         st_release(reinterpret_cast<uint64_t*>(P.hdr[P.my_rank]), epoch, true);
         if (P.zc)  // our buffers stay in use until every peer has finished this call
           for (int q = 0; q < P.nranks; ++q)
-            if (q != P.my_rank) wait_flag(reinterpret_cast<const uint64_t*>(P.hdr[q]), epoch, P);
+            if (q != P.my_rank && ((P.members >> q) & 1))
+              wait_flag(reinterpret_cast<const uint64_t*>(P.hdr[q]), epoch, P);
       }
     }
   }

@@ -37,6 +37,7 @@ struct LaunchParams {
   uint64_t late_ticket; // ready word value that admits a late rank (phase 1)
   uint64_t* late_bits;  // per work item: late candidates included in phase 1
   int drop_rank;        // test hook (loopback): tasks owned by this rank are skipped
+  uint64_t members;     // live ranks: excluded ranks are skipped by the IPC barriers
   uint64_t half_bytes;  // bytes of one parity half of an arena
   uint64_t timeout_ns;
   DevState* state;

@@ -50,9 +50,11 @@ BufRef make_ref(uint8_t kind, int rank, int64_t bias, bool accum = false) {
 
 class Builder {
  public:
-  Builder(int n, int esize, uint64_t half)
-      : n_(n), esize_(esize), half_(half), flag_cap_(flag_region_bytes(half)),
+  Builder(int n, int esize, uint64_t half, uint64_t members)
+      : n_(n), esize_(esize), half_(half), flag_cap_(flag_region_bytes(half)), members_(members),
         used_(n, 0), flags_used_(n, 0) {}
+
+  bool alive(int g) const { return ((members_ >> g) & 1) != 0; }
 
   // Each parity half of a rank's arena = [flag region | data region].  Flag
   // words only ever hold epochs (monotonic), so a later plan with a different
@@ -129,7 +131,7 @@ class Builder {
   }
 
   int n_, esize_;
-  uint64_t half_, flag_cap_;
+  uint64_t half_, flag_cap_, members_;
   std::vector<uint64_t> used_, flags_used_;
   SegmentPlan p_;
   std::map<std::pair<uint32_t, uint64_t>, int> producer_;
@@ -165,7 +167,7 @@ void plan_allreduce_tree(Builder& B, const SubColl& s, uint64_t lo, uint64_t hi,
 
   std::vector<BufRef> recv_all;
   for (int g = 0; g < n; ++g)
-    if (!root_only || g == s.root) recv_all.push_back(make_ref(kBufRecv, g, 0, accumulate));
+    if ((!root_only || g == s.root) && B.alive(g)) recv_all.push_back(make_ref(kBufRecv, g, 0, accumulate));
 
   if (mode == kDirect) {
     std::map<int, std::pair<uint64_t, FlagRef>> agg_slot;  // kernel node -> slot
@@ -191,7 +193,7 @@ void plan_allreduce_tree(Builder& B, const SubColl& s, uint64_t lo, uint64_t hi,
     std::vector<BufRef> late;
     if (late_join)
       for (int g = 0; g < n; ++g)
-        if (!((mask >> g) & 1)) late.push_back(make_ref(kBufSend, g, send_bias));
+        if (!((mask >> g) & 1) && B.alive(g)) late.push_back(make_ref(kBufSend, g, send_bias));
     B.add(root, lo, hi, ce, zero ? kOpZero : kOpFold, srcs, recv_all, {}, late);
     return;
   }
@@ -257,7 +259,7 @@ void plan_allreduce_tree(Builder& B, const SubColl& s, uint64_t lo, uint64_t hi,
   if (root_only) return;
   // broadcast down the reversed tree, parents before children
   for (int g : bfs_order(s)) {
-    if (g == root) continue;
+    if (g == root || !B.alive(g)) continue;  // excluded ranks are leaves (check_members)
     const int p = s.parent[g];
     auto& pd = down.at(p);
     std::vector<Stream> srcs = {B.slot_stream(p, pd.first, lo, &pd.second)};
@@ -285,12 +287,14 @@ void plan_allgather_tree(Builder& B, const SubColl& s, uint64_t lo, uint64_t hi,
   in.ref = make_ref(kBufSend, src, 0);
   if (mode == kDirect) {
     std::vector<BufRef> dsts;
-    for (int g = 0; g < n; ++g) dsts.push_back(make_ref(kBufRecv, g, slot_bias));
+    for (int g = 0; g < n; ++g)
+      if (B.alive(g)) dsts.push_back(make_ref(kBufRecv, g, slot_bias));
     B.add(src, lo, hi, ce, kOpFold, {in}, dsts, {});
     return;
   }
   std::map<int, std::pair<uint64_t, FlagRef>> down;
   for (int g : bfs_order(s)) {
+    if (!B.alive(g)) continue;  // excluded ranks are leaves (check_members)
     std::vector<Stream> srcs;
     if (g == src) {
       srcs.push_back(in);
@@ -348,6 +352,7 @@ void plan_alltoall_line(Builder& B, const SubColl& s, uint64_t lo, uint64_t hi, 
   for (int src = 0; src < n; ++src) {
     if (!((mask >> src) & 1)) continue;
     for (int d = 0; d < n; ++d) {
+      if (!B.alive(d)) continue;
       Stream in;
       in.ref = make_ref(kBufSend, src, (int64_t)(d * cnt * es));
       plan_flow(B, src, d, s.hops(src, d), in, make_ref(kBufRecv, d, (int64_t)(src * cnt * es)), lo, hi,
@@ -368,7 +373,7 @@ void plan_alltoallv(Builder& B, const PlanRequest& rq, uint64_t k, uint64_t nseg
     if (!((rq.ready_mask >> src) & 1)) continue;
     for (int d = 0; d < n; ++d) {
       const uint64_t c = rq.counts[(size_t)src * n + d];
-      if (!c) continue;
+      if (!c || !B.alive(d)) continue;
       uint64_t soff = 0, roff = 0;
       for (int j = 0; j < d; ++j) soff += rq.counts[(size_t)src * n + j];
       for (int j = 0; j < src; ++j) roff += rq.counts[(size_t)j * n + d];
@@ -391,7 +396,7 @@ SegmentPlan build_segment(const PlanRequest& rq,
                           const std::vector<std::pair<uint64_t, uint64_t>>& ranges, uint64_t seg_k,
                           uint64_t nseg) {
   const Strategy& st = *rq.st;
-  Builder B(st.nranks, rq.esize, rq.half_bytes);
+  Builder B(st.nranks, rq.esize, rq.half_bytes, rq.members);
   if (rq.counts) {
     plan_alltoallv(B, rq, seg_k, nseg);
     return B.finish();
@@ -406,6 +411,7 @@ SegmentPlan build_segment(const PlanRequest& rq,
         break;
       case kReduce: plan_allreduce_tree(B, s, lo, hi, rq.ready_mask, rq.accumulate, rq.mode, 0, true); break;
       case kReduceScatter:
+        if (!B.alive(s.src)) break;  // block of an excluded rank: no destination
         plan_allreduce_tree(B, s, lo, hi, rq.ready_mask, rq.accumulate, rq.mode,
                             (int64_t)((uint64_t)s.src * rq.count * rq.esize), true);
         break;

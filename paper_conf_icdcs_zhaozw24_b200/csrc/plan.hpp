@@ -47,6 +47,9 @@ struct PlanRequest {
   // blocks are packed in destination order in the sendbuf and source order in
   // the recvbuf.  nullptr for every other collective.
   const uint64_t* counts = nullptr;
+  // Live ranks (NEXT-3: faulty ranks excluded): an excluded rank
+  // owns no task and no buffer of it is read or written.
+  uint64_t members = ~uint64_t(0);
 };
 
 // Bytes at the start of each parity half reserved for per-chunk flag words.

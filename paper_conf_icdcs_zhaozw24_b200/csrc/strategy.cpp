@@ -326,6 +326,28 @@ bool parse_strategy(const char* text, Strategy* out, std::string* err) {
   return true;
 }
 
+bool check_members(const Strategy& st, uint64_t members, std::string* err) {
+  const int n = st.nranks;
+  auto alive = [&](int g) { return ((members >> g) & 1) != 0; };
+  for (const SubColl& s : st.subs) {
+    if (s.kind == kA2A) {
+      for (const Route& r : s.routes)
+        for (int h : r.hops)
+          if (!alive(h)) return fail(err, "an excluded rank cannot relay AlltoAll flows");
+      continue;
+    }
+    if (st.coll == kReduce && !alive(s.root)) return fail(err, "the Reduce root was excluded");
+    if (st.coll == kBroadcast && !alive(s.src)) return fail(err, "the Broadcast source was excluded");
+    // an AllGather source / ReduceScatter block owner that was excluded: the
+    // sub-collective is skipped (never ready / no destination)
+    if ((s.kind == kBcast || s.kind == kRTree) && !alive(s.src)) continue;
+    for (int g = 0; g < n; ++g)
+      if (!alive(g) && !s.children[g].empty())
+        return fail(err, "an excluded rank must be a leaf of every tree");
+  }
+  return true;
+}
+
 const std::vector<int>* SubColl::hops(int s, int d) const {
   for (const Route& r : routes)
     if (r.src == s && r.dst == d) return &r.hops;

@@ -57,6 +57,12 @@ struct Strategy {
 // Parse + validate; returns false and fills *err on failure.
 bool parse_strategy(const char* text, Strategy* out, std::string* err);
 
+// Fault tolerance (NEXT-3): after faulty ranks are excluded, a
+// strategy may still name them, but only where they have nothing to do:
+// leaves of every tree / broadcast tree whose source or destination is alive,
+// never an AlltoAll relay, never the Reduce root or Broadcast source.
+bool check_members(const Strategy& st, uint64_t members, std::string* err);
+
 // Reading Q9: bounds of `count` elements over `weights` (size M -> M+1 bounds).
 std::vector<uint64_t> partition(uint64_t count, int esize, const std::vector<int64_t>& weights);
 

@@ -230,6 +230,16 @@ def alltoall_detour(n, slow_edges, chunk=1 << 20, direct_weight=0, routed_weight
     return alltoall_routed(n, lines, chunk)
 
 
+def survivor_stars(n, alive, chunk=DEFAULT_CHUNK):
+    """AllReduce strategy after a fault exclusion (NEXT-3): one
+    star per live rank with equal weights; excluded ranks are leaves of every
+    star (the only place adapcc_exclude lets a strategy name them)."""
+    out = _header(n, "allreduce")
+    for r in sorted(alive):
+        out += f"tree weight=1 chunk={int(chunk)} parent={_join(star_parent(n, r))}\n"
+    return out
+
+
 # ----------------------------------------------------- NEXT-4 primitives
 def reduce_trees(parents, weights=None, chunk=DEFAULT_CHUNK, noaggs=None):
     """Reduce: every tree must be rooted at the Reduce root."""
