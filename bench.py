@@ -45,7 +45,7 @@ def parse_args():
     p.add_argument("--dtype", choices=["f32", "bf16"], default="f32")
     p.add_argument("--mode", choices=["direct", "staged"], default="direct")
     p.add_argument("--chunk-kib", type=int, default=256)
-    p.add_argument("--e2e-steps", type=int, default=5)
+    p.add_argument("--e2e-steps", type=int, default=8)
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--no-parity", action="store_true")
     p.add_argument("--test-same-gpu", action="store_true",
@@ -283,23 +283,12 @@ def run_single(args):
     if not args.no_parity:
         parity = sampled_parity(dy, host_in, text, n, count, args.dtype)
 
-    # end to end: pinned host inputs -> device -> allreduce -> host, every step
-    host_out = [torch.empty(count, dtype=host_in[0].dtype).pin_memory() for _ in range(n)]
-    e2e_ms = []
-    for i in range(args.e2e_steps + 1):
-        a = torch.cuda.Event(enable_timing=True)
-        b = torch.cuda.Event(enable_timing=True)
-        a.record(stream)
-        for r in range(n):
-            dx[r].view(host_in[r].dtype).copy_(host_in[r], non_blocking=True)
-        comm.allreduce_lb(dx, dy)
-        for r in range(n):
-            host_out[r].copy_(dy[r].view(host_out[r].dtype), non_blocking=True)
-        b.record(stream)
-        torch.cuda.synchronize()
-        if i > 0:
-            e2e_ms.append(a.elapsed_time(b))
-    e2e_t = sum(e2e_ms) / len(e2e_ms)
+    # end to end: pinned host inputs -> device -> allreduce -> pinned host, every
+    # step.  Steps are pipelined like a training loop's buckets: double-buffered
+    # device tensors, H2D on one copy stream and D2H on another, so step i's
+    # download overlaps step i+1's upload (PCIe is full duplex); per-step time
+    # = span of all steps / steps.
+    e2e_t = e2e_pipelined(comm, host_in, dx, dy, args.e2e_steps, tdt, lambda xs, ys: comm.allreduce_lb(xs, ys))
 
     peak, peak_src = load_peaks()
     alg_bytes = 2 * n * nbytes   # every rank's input read once + output written once
@@ -319,7 +308,9 @@ def run_single(args):
                      "kernel_ms": round(kern_ms, 4)},
         "e2e": {"value": round(busbw(nbytes, e2e_t / 1e3, n), 3), "unit": UNIT,
                 "h2d_bytes_per_step": n * nbytes, "d2h_bytes_per_step": n * nbytes,
-                "ms_per_step": round(e2e_t, 3)},
+                "ms_per_step": round(e2e_t, 3), "steps": args.e2e_steps,
+                "how": "pinned H2D of all inputs + allreduce_lb + D2H of all outputs per step; steps "
+                       "double-buffered with H2D and D2H on separate copy streams (full-duplex PCIe)"},
         "gpu_launches": launches,
         "clocks": clk.summary(),
         "parity": parity,
@@ -329,6 +320,63 @@ def run_single(args):
         out["cpu_baseline"] = cpu_baseline_block(n, args.dtype)
     comm.finalize()
     return out
+
+
+def e2e_pipelined(comm, host_in, dx, dy, steps, tdt, call, second=None):
+    """Average per-step time (ms) of `steps` end-to-end steps, each: H2D of
+    every input from pinned host memory, the collective, D2H of every output
+    into pinned host memory.  Two device buffer sets; copies on their own
+    streams; the collective on the current stream.  second = (dx2, dy2): the
+    second buffer set (e.g. registered for zero-copy), else allocated here."""
+    import torch
+    cur = torch.cuda.current_stream()
+    s_in, s_out = torch.cuda.Stream(), torch.cuda.Stream()
+    if second is None:
+        second = ([torch.empty_like(t) for t in dx], [torch.empty_like(t) for t in dy])
+    bx = [dx, second[0]]
+    by = [dy, second[1]]
+    hout = [[torch.empty(t.numel(), dtype=host_in[0].dtype).pin_memory() for t in dy] for _ in range(2)]
+    ev = lambda: torch.cuda.Event()  # noqa: E731
+    ar_done = [None, None]
+    out_done = [None, None]
+
+    def step(i):
+        b = i % 2
+        with torch.cuda.stream(s_in):
+            if ar_done[b] is not None:
+                s_in.wait_event(ar_done[b])          # the collective of step i-2 read bx[b]
+            for r, h in enumerate(host_in):
+                bx[b][r].view(h.dtype).copy_(h, non_blocking=True)
+            e_in = ev()
+            e_in.record(s_in)
+        cur.wait_event(e_in)
+        if out_done[b] is not None:
+            cur.wait_event(out_done[b])              # step i-2's download of by[b] finished
+        call(bx[b], by[b])
+        ar_done[b] = ev()
+        ar_done[b].record(cur)
+        with torch.cuda.stream(s_out):
+            s_out.wait_event(ar_done[b])
+            for r, t in enumerate(by[b]):
+                hout[b][r].copy_(t.view(hout[b][r].dtype), non_blocking=True)
+            out_done[b] = ev()
+            out_done[b].record(s_out)
+
+    for i in range(2):                                   # warm the streams and buffers
+        step(i)
+    torch.cuda.synchronize()
+    a = torch.cuda.Event(enable_timing=True)
+    z = torch.cuda.Event(enable_timing=True)
+    a.record(cur)
+    s_in.wait_stream(cur)
+    for i in range(steps):
+        step(i)
+    cur.wait_stream(s_out)
+    cur.wait_stream(s_in)
+    z.record(cur)
+    torch.cuda.synchronize()
+    assert comm.get_async_error() == 0
+    return a.elapsed_time(z) / steps
 
 
 def sampled_parity(dy, host_in, text, n, count, dtype, k=4096):
@@ -431,25 +479,24 @@ def run_multi(args):
     ms_staged = timed(ours_staged, args.steps)
     err = comm.get_async_error()
 
-    e2e = []
-    for i in range(args.e2e_steps + 1):
-        dist.barrier()
-        torch.cuda.synchronize()
-        a = torch.cuda.Event(enable_timing=True)
-        b = torch.cuda.Event(enable_timing=True)
-        a.record(stream)
-        x.view(xh.dtype).copy_(xh, non_blocking=True)
-        comm.collective_zc("allreduce", x, y, count)
-        out_h = y.view(xh.dtype).to("cpu", non_blocking=True)
-        b.record(stream)
-        torch.cuda.synchronize()
-        t = torch.tensor([a.elapsed_time(b)], device="cpu" if args.test_same_gpu else "cuda")
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        if i > 0:
-            e2e.append(float(t.item()))
-    del out_h
-    e2e_t = sum(e2e) / len(e2e)
+    # end to end (same pipelining as N=1): per rank H2D of its input, the
+    # zero-copy collective, D2H of its output; the per-step time is the max
+    # over ranks.  The second buffer pair is registered too.
+    x2, y2 = torch.empty_like(x), torch.empty_like(y)
+    comm.register(x2)
+    comm.register(y2)
+
+    def zc_call(xs, ys):
+        comm.collective_zc("allreduce", xs[0], ys[0], count)
+
+    dist.barrier()
+    e2e_local = e2e_pipelined(comm, [xh], [x], [y], args.e2e_steps, tdt, zc_call, second=([x2], [y2]))
+    t = torch.tensor([e2e_local], device="cpu" if args.test_same_gpu else "cuda")
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    e2e_t = float(t.item())
     value = busbw(nbytes, ms / 1e3, world)
+    st = pkg.adapcc.plan_stats(text, count, args.dtype, (1 << world) - 1, rank=rank)
+    dir_bytes = st["remote_bytes"] // 2   # remote loads (in) + remote stores (out), symmetric
     res = None
     if rank == 0:
         res = {
@@ -460,13 +507,18 @@ def run_multi(args):
             "config": workload_config(args, world, world),
             "algbw": round(nbytes / (ms / 1e3) / 1e9, 3),
             "pct_of_nvlink_900": round(100 * value / NVLINK_NOMINAL, 2),
-            "roofline": {"bound": "nvlink", "achieved": round(value, 1), "peak": 770.0, "unit": "GB/s",
-                         "frac": round(value / 770.0, 4), "traffic": None,
-                         "peak_source": "B200_PROFILING.md measured peer copy 770 GB/s per direction",
-                         "algorithmic_bytes_per_launch": int(2 * (world - 1) * nbytes // world)},
+            "roofline": {"bound": "nvlink", "achieved": round(dir_bytes / (ms / 1e3) / 1e9, 1), "peak": 770.0,
+                         "unit": "GB/s", "frac": round(dir_bytes / (ms / 1e3) / 1e9 / 770.0, 4), "traffic": None,
+                         "peak_source": "B200_PROFILING.md measured peer copy 770 GB/s per direction per GPU",
+                         "algorithmic_bytes_per_direction": dir_bytes,
+                         "why": "zero-copy star plan: each rank pulls the (n-1)/n S its trees reduce and "
+                                "pushes the (n-1)/n S they broadcast; loads and stores use opposite link "
+                                "directions, so (n-1)/n S must cross each direction of a GPU's NVLink"},
             "e2e": {"value": round(busbw(nbytes, e2e_t / 1e3, world), 3), "unit": UNIT,
                     "h2d_bytes_per_step": nbytes, "d2h_bytes_per_step": nbytes,
-                    "ms_per_step": round(e2e_t, 3)},
+                    "ms_per_step": round(e2e_t, 3), "steps": args.e2e_steps,
+                    "how": "per rank: pinned H2D of its input + collective_zc + D2H of its output; steps "
+                           "double-buffered (both pairs registered), copies on separate streams; max over ranks"},
             "gpu_launches": launches, "clocks": clk.summary(), "async_error": err,
             "path": "zero-copy DIRECT plan over CUDA IPC (registered buffers)",
             "staged": {"value": round(busbw(nbytes, ms_staged / 1e3, world), 3), "unit": UNIT,
