@@ -43,6 +43,9 @@ constexpr int kTmaThreads = kConsumers + 32;  // + 1 producer warp
 #endif
 constexpr int kStages = ADAPCC_TMA_STAGES;
 constexpr uint32_t kStageBytes = ADAPCC_TMA_STAGE_KB * 1024;
+// Tiles larger than one consumer round (K = 1 with accumulation: > 32 KiB;
+// K = 2, 3: > 16 KiB) exist only with stages above 32 KiB.
+constexpr bool kLargeTiles = kStageBytes > 32 * 1024;
 constexpr int kMaxKS = (kStageBytes / 4096) < 8 ? (int)(kStageBytes / 4096) : 8;  // sources per stage
 constexpr int kQ = 2;           // item queue depth
 constexpr int kMaxPost = 4;
@@ -174,30 +177,57 @@ __device__ void scalar_range(const ItemDesc& d, uint64_t e_begin, uint64_t e_end
   }
 }
 
-// Copy the tiles of a one-source item (bytes unchanged): VPT vectors per
-// thread per tile.
+// Large-tile rounds (tile > one round of the caller's VPT), kept out of line
+// so that the common one-round path keeps its register budget.
+template <int DT>
+__device__ __noinline__ void copy_rounds(const char* sb, const ItemDesc& d, int tid, uint32_t t, uint32_t nv) {
+  for (uint32_t v = tid; v < nv; v += kConsumers)
+    store_result<DT>(d, (size_t)t * d.tile + (size_t)v * 16, lds16(sb + (size_t)v * 16));
+}
+template <int DT>
+__device__ __noinline__ void fold_rounds(const char* sb, const ItemDesc& d, int tid, uint32_t t, uint32_t nv) {
+  using O = Ops<DT>;
+  for (uint32_t v = tid; v < nv; v += kConsumers) {
+    const char* pv = sb + (size_t)v * 16;
+    typename O::Acc a = O::widen(lds16(pv));
+    for (int k = 1; k < (int)d.nsrc; ++k) O::add(a, lds16(pv + (size_t)k * d.tile));
+    store_result<DT>(d, (size_t)t * d.tile + (size_t)v * 16, O::narrow(a));  // one rounding
+  }
+}
+
+// Copy the tiles of a one-source item (bytes unchanged) into destinations
+// that need the generic proxy (accumulation): VPT vectors per thread per
+// round; a tile larger than one round (VPT x 16 B x consumers) is walked in
+// rounds while the stage is held.
 template <int DT, int VPT>
 __device__ __forceinline__ void consume_copy(Smem& sm, char* stages, const ItemDesc& d, int tid,
                                              uint32_t& stage, uint32_t& sphase) {
   const bool warp_lane0 = (tid & 31) == 0;
+  constexpr uint32_t kRound = VPT * kConsumers;
   for (uint32_t t = 0; t < d.ntiles; ++t) {
     const uint32_t nv = min(d.tile, d.vec_bytes - t * d.tile) / 16;
-    uint4 raw[VPT];
     mbar_wait(&sm.full[stage], sphase);
     const char* sb = stages + (size_t)stage * kStageBytes;
+    if (!kLargeTiles || nv <= kRound) {  // one round: registers hold the tile, release the stage before storing
+      uint4 raw[VPT];
 #pragma unroll
-    for (int j = 0; j < VPT; ++j) {
-      const uint32_t v = tid + j * kConsumers;
-      if (v < nv) raw[j] = lds16(sb + (size_t)v * 16);
+      for (int j = 0; j < VPT; ++j) {
+        const uint32_t v = tid + j * kConsumers;
+        if (v < nv) raw[j] = lds16(sb + (size_t)v * 16);
+      }
+      __syncwarp();
+      if (warp_lane0) mbar_arrive(&sm.empty[stage]);
+#pragma unroll
+      for (int j = 0; j < VPT; ++j) {
+        const uint32_t v = tid + j * kConsumers;
+        if (v < nv) store_result<DT>(d, (size_t)t * d.tile + (size_t)v * 16, raw[j]);
+      }
+    } else {
+      copy_rounds<DT>(sb, d, tid, t, nv);
+      __syncwarp();
+      if (warp_lane0) mbar_arrive(&sm.empty[stage]);
     }
-    __syncwarp();
-    if (warp_lane0) mbar_arrive(&sm.empty[stage]);
     if (++stage == kStages) { stage = 0; sphase ^= 1; }
-#pragma unroll
-    for (int j = 0; j < VPT; ++j) {
-      const uint32_t v = tid + j * kConsumers;
-      if (v < nv) store_result<DT>(d, (size_t)t * d.tile + (size_t)v * 16, raw[j]);
-    }
   }
 }
 
@@ -234,14 +264,26 @@ __device__ __forceinline__ void copy_tma(Smem& sm, char* stages, const ItemDesc&
 }
 
 // Fold the tiles of a K >= 2 item: every stage holds ks source tiles; a tile
-// of K > 8 sources spans several stages (passes) accumulated in registers.
+// of K > 8 sources spans several stages (passes) accumulated in registers
+// (then the tile is at most stage / 8 bytes, one round).  A single-pass tile
+// larger than one round (VPT x 16 B x consumers: K = 2, 3 with 64 KiB stages)
+// is folded round by round while the stage is held.
 template <int DT, int VPT>
 __device__ __forceinline__ void consume_fold(Smem& sm, char* stages, const ItemDesc& d, int tid,
                                              uint32_t& stage, uint32_t& sphase) {
   using O = Ops<DT>;
   const bool warp_lane0 = (tid & 31) == 0;
+  constexpr uint32_t kRound = VPT * kConsumers;
   for (uint32_t t = 0; t < d.ntiles; ++t) {
     const uint32_t nv = min(d.tile, d.vec_bytes - t * d.tile) / 16;
+    if (kLargeTiles && nv > kRound) {  // single pass (d.passes == 1), several rounds
+      mbar_wait(&sm.full[stage], sphase);
+      fold_rounds<DT>(stages + (size_t)stage * kStageBytes, d, tid, t, nv);
+      __syncwarp();
+      if (warp_lane0) mbar_arrive(&sm.empty[stage]);
+      if (++stage == kStages) { stage = 0; sphase ^= 1; }
+      continue;
+    }
     typename O::Acc a[VPT];
     for (int p = 0; p < d.passes; ++p) {
       const int ks = min((int)d.ks, (int)d.nsrc - p * (int)d.ks);
@@ -462,7 +504,7 @@ __global__ void __launch_bounds__(kTmaThreads, ADAPCC_TMA_MINB) engine_tma_kerne
             for (uint64_t e = tid; e < d.len; e += kConsumers) reinterpret_cast<E*>(d.dst[k])[e] = E(0);
         } else {
           if (!d.scalar_only) {
-            const uint32_t vpt = d.tile / (16u * kConsumers);  // 8 (K=1), 4, 2 or 1
+            const uint32_t vpt = d.tile / (16u * kConsumers);  // tile / one round of 1 vector per thread
             if (d.nsrc == 1 && !d.any_acc) copy_tma(sm, stages, d, tid, stage, sphase);
             else if (d.nsrc == 1) consume_copy<DT, 8>(sm, stages, d, tid, stage, sphase);
             else if (vpt >= 4) consume_fold<DT, 4>(sm, stages, d, tid, stage, sphase);

@@ -141,3 +141,58 @@ def test_c5_allgather_gpt2xl_with_swap(n):
         for g in _gather(dy, idx, "bf16"):
             assert np.array_equal(g, exp), call
     comm.finalize()
+
+
+def test_c2_max_size_sampled():
+    """C2's largest point (2^30 B per rank, P:L289 sweep) at n = 8: 16 GiB of
+    inputs + outputs resident, TMA pipeline (auto), sampled parity."""
+    n, nbytes = 8, 1 << 30
+    count = nbytes // 4
+    text = G.allreduce_stars(n, chunk=262144)
+    comm = pkg.Communicator.loopback(n, scratch_bytes=64 << 20, mode="direct")
+    comm.set_strategy("allreduce", text)
+    idx = _samples(count)
+    vals, dy = [], []
+    dx = []
+    for r in range(n):   # one rank at a time keeps host memory at ~1 GiB
+        x = rank_tensors("f32", count, 1, base=1000 + r)[0]
+        vals.append(x[idx].copy())
+        dx.append(to_dev(x, "f32"))
+        del x
+        dy.append(torch.empty(count, dtype=torch.float32, device="cuda"))
+    comm.allreduce_lb(dx, dy)
+    torch.cuda.synchronize()
+    assert comm.get_async_error() == 0
+    assert comm.last_engine() == 1
+    exp = oc.allreduce_elements(vals, idx, count, text, set(range(n)), "f32")
+    for g in _gather(dy, idx, "f32"):
+        assert np.array_equal(bits(g), bits(exp))
+    comm.finalize()
+
+
+@pytest.mark.parametrize("engine", [0, 1])
+def test_byte_offsets_beyond_2_31(engine):
+    """2.25 GiB per rank (int32): byte offsets past 2^31 in every pointer path;
+    the ragged tail and the last element are sampled."""
+    n = 2
+    count = (9 << 28) // 4 + 3
+    text = G.allreduce_stars(n, chunk=1 << 20)
+    comm = pkg.Communicator.loopback(n, scratch_bytes=64 << 20, mode="direct")
+    comm.config("engine", engine)
+    comm.set_strategy("allreduce", text)
+    idx = np.unique(np.concatenate([_samples(count), np.arange(count - 64, count),
+                                    np.arange((1 << 29) - 8, (1 << 29) + 8)]))
+    vals, dx = [], []
+    for r in range(n):
+        x = rank_tensors("i32", count, 1, base=1100 + r)[0]
+        vals.append(x[idx].copy())
+        dx.append(to_dev(x, "i32"))
+        del x
+    dy = [torch.empty(count, dtype=torch.int32, device="cuda") for _ in range(n)]
+    comm.allreduce_lb(dx, dy)
+    torch.cuda.synchronize()
+    assert comm.get_async_error() == 0
+    exp = oc.allreduce_elements(vals, idx, count, text, set(range(n)), "i32")
+    for g in _gather(dy, idx, "i32"):
+        assert np.array_equal(g, exp)
+    comm.finalize()

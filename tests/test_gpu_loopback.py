@@ -303,3 +303,28 @@ def test_cuda_graph_capture_and_replay(mode, engine):
         assert comm.get_async_error() == 0
         _assert_bits([to_host(t, "f32") for t in dy], exp, f"graph replay {rep}")
     comm.finalize()
+
+
+@pytest.mark.parametrize("mode", MODES)
+@pytest.mark.parametrize("dtype", ["f32", "bf16"])
+@pytest.mark.parametrize("n", [2, 3, 5])
+def test_tma_large_items(mode, dtype, n):
+    """Items whose shared-memory tile exceeds one consumer round: K = 2, 3
+    folds and the K = 1 accumulate copy of phase 2 with 64 KiB stages (DIRECT
+    plans), chunks of 4 MiB so every item spans many tiles."""
+    count = (3 << 20) + 5
+    es = 4 if dtype == "f32" else 2
+    comm = _comm(n, mode, scratch=3 * count * es + (64 << 20), engine=1)
+    xs = rank_tensors(dtype, count, n)
+    for text in (G.allreduce_stars(n, chunk=4 << 20), G.allreduce_ring(n, chunk=4 << 20)):
+        comm.set_strategy("allreduce", text)
+        got = _run_allreduce(comm, xs, dtype, set(range(n)))
+        _assert_bits(got, oc.allreduce(xs, text, set(range(n)), dtype), f"large/{n}/{mode}")
+        # phase 1 without rank 0, phase 2 = rank 0 alone with ACCUMULATE (K = 1 + accumulate)
+        R1 = set(range(1, n))
+        p1 = _run_allreduce(comm, [x if r in R1 else None for r, x in enumerate(xs)], dtype, R1)
+        got = _run_allreduce(comm, [xs[0]] + [None] * (n - 1), dtype, {0}, accumulate=True, prev=p1)
+        exp1 = oc.allreduce(xs, text, R1, dtype)
+        _assert_bits(got, oc.allreduce(xs, text, {0}, dtype, accumulate=True, y_prev=exp1), f"large-acc/{n}/{mode}")
+    assert comm.last_engine() == 1
+    comm.finalize()
