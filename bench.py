@@ -31,7 +31,12 @@ METRIC = "AllReduce busbw GB/s vs size at 2/4/8 B200 (% of 900 GB/s) vs NCCL"
 UNIT = "GB/s"
 NVLINK_NOMINAL = 900.0
 ENGINE_NAMES = {0: "adapcc::engine_kernel (128-bit LDG/STG fold)",
-                1: "adapcc::engine_tma_kernel (TMA bulk-copy pipeline)"}
+                1: "adapcc::{ns}::engine_tma_kernel (TMA bulk-copy pipeline)"}
+
+
+def engine_name(engine, mode, dtype):
+    ns = "tma_direct" if mode == "direct" else "tma_staged"
+    return ENGINE_NAMES.get(engine, "?").format(ns=ns) + f"<{dtype}>"
 
 
 def parse_args():
@@ -304,7 +309,7 @@ def run_single(args):
         "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
                      "frac": round(achieved / peak, 4), "traffic": profile_traffic(traffic_key(comm.last_engine(), args.mode)),
                      "algorithmic_bytes_per_launch": alg_bytes, "peak_source": peak_src,
-                     "kernel": ENGINE_NAMES.get(comm.last_engine(), "?") + f"<{args.dtype}>",
+                     "kernel": engine_name(comm.last_engine(), args.mode, args.dtype),
                      "kernel_ms": round(kern_ms, 4)},
         "e2e": {"value": round(busbw(nbytes, e2e_t / 1e3, n), 3), "unit": UNIT,
                 "h2d_bytes_per_step": n * nbytes, "d2h_bytes_per_step": n * nbytes,
@@ -496,7 +501,7 @@ def run_multi(args):
     e2e_t = float(t.item())
     value = busbw(nbytes, ms / 1e3, world)
     st = pkg.adapcc.plan_stats(text, count, args.dtype, (1 << world) - 1, rank=rank)
-    dir_bytes = st["remote_bytes"] // 2   # remote loads (in) + remote stores (out), symmetric
+    dir_bytes = st["remote_bytes"]   # = bytes crossing each link direction of this GPU (symmetric plan)
     res = None
     if rank == 0:
         res = {
@@ -511,9 +516,10 @@ def run_multi(args):
                          "unit": "GB/s", "frac": round(dir_bytes / (ms / 1e3) / 1e9 / 770.0, 4), "traffic": None,
                          "peak_source": "B200_PROFILING.md measured peer copy 770 GB/s per direction per GPU",
                          "algorithmic_bytes_per_direction": dir_bytes,
-                         "why": "zero-copy star plan: each rank pulls the (n-1)/n S its trees reduce and "
-                                "pushes the (n-1)/n S they broadcast; loads and stores use opposite link "
-                                "directions, so (n-1)/n S must cross each direction of a GPU's NVLink"},
+                         "why": "zero-copy star plan, per GPU g: g's kernel pulls (n-1)/n S (its trees' "
+                                "inputs) and pushes (n-1)/n S (their results), while peers pull g's "
+                                "slices and push their results into g: 2(n-1)/n S in each direction, the "
+                                "plan's remote bytes of g (loads + stores) by symmetry"},
             "e2e": {"value": round(busbw(nbytes, e2e_t / 1e3, world), 3), "unit": UNIT,
                     "h2d_bytes_per_step": nbytes, "d2h_bytes_per_step": nbytes,
                     "ms_per_step": round(e2e_t, 3), "steps": args.e2e_steps,
