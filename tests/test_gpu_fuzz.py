@@ -1,0 +1,133 @@
+"""Randomised GPU parity sweep (-m gpu): random trees (shape, root, noagg),
+weights, chunk sizes, counts (1 element .. 3 M, ragged), masks, dtypes,
+plans (DIRECT / STAGED) and kernels (LDG, TMA, auto), every collective the
+loopback communicator offers; bit-exact against the oracle.  Seeded: a
+failure names its case and reproduces."""
+
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+
+import paper_conf_icdcs_zhaozw24_b200 as pkg  # noqa: E402
+from oracle import collectives as oc  # noqa: E402
+from paper_conf_icdcs_zhaozw24_b200 import generator as G  # noqa: E402
+from synth import rank_tensors  # noqa: E402
+from tests.gpu_util import bits, empty_dev, to_dev, to_host  # noqa: E402
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(autouse=True)
+def _need_gpu():
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+
+
+def _random_tree(rng, n):
+    """Random labelled tree: random attachment order, random root."""
+    order = [int(v) for v in rng.permutation(n)]
+    parent = [-1] * n
+    for i in range(1, n):
+        parent[order[i]] = order[int(rng.integers(0, i))]
+    return parent
+
+
+def _case(seed):
+    rng = np.random.default_rng(seed)
+    n = int(rng.integers(2, 9))
+    coll = ["allreduce", "allreduce", "allgather", "alltoall", "reducescatter"][int(rng.integers(0, 5))]
+    dtype = ["f32", "bf16", "i32"][int(rng.integers(0, 3))]
+    big = rng.random() < 0.3
+    count = int(np.exp(rng.uniform(0, np.log(3e6 if big else 2e4))))
+    if coll in ("alltoall", "allgather", "reducescatter"):
+        count = max(1, count // n)
+    chunk = 16 * int(np.exp(rng.uniform(np.log(4), np.log((8 << 20) // 16))))
+    mode = ["direct", "staged"][int(rng.integers(0, 2))]
+    engine = int(rng.integers(0, 3))
+    ready = {g for g in range(n) if rng.random() < 0.75}
+    if rng.random() < 0.2:
+        ready = set(range(n))
+    m = int(rng.integers(1, 4))
+    if coll == "allreduce":
+        parents = [_random_tree(rng, n) for _ in range(m)]
+        noaggs = [[g for g in range(n) if p[g] != -1 and rng.random() < 0.25] for p in parents]
+        text = G.allreduce_trees(parents, [int(rng.integers(1, 5)) for _ in range(m)], chunk, noaggs)
+    elif coll == "allgather":
+        text = G._header(n, "allgather")
+        for s in range(n):
+            for _ in range(int(rng.integers(1, 3))):
+                p = _random_tree(rng, n)
+                # re-root at s: swap labels of the root and s
+                r = p.index(-1)
+                sw = {r: s, s: r}
+                q = [-1] * n
+                for g in range(n):
+                    pg = p[g]
+                    q[sw.get(g, g)] = -1 if pg == -1 else sw.get(pg, pg)
+                text += f"bcast src={s} weight={int(rng.integers(1, 4))} chunk={chunk} parent={G._join(q)}\n"
+    elif coll == "alltoall":
+        lines = []
+        for _ in range(m):
+            routes = {}
+            for s in range(n):
+                for d in range(n):
+                    if s != d and n > 2 and rng.random() < 0.3:
+                        others = [g for g in range(n) if g not in (s, d)]
+                        k = int(rng.integers(1, min(3, len(others)) + 1))
+                        routes[(s, d)] = [int(v) for v in rng.choice(others, k, replace=False)]
+            lines.append((int(rng.integers(1, 4)), routes))
+        text = G.alltoall_routed(n, lines, chunk)
+    else:
+        text = G._header(n, "reducescatter")
+        for b in range(n):
+            p = _random_tree(rng, n)
+            r = p.index(-1)
+            sw = {r: b, b: r}
+            q = [-1] * n
+            for g in range(n):
+                pg = p[g]
+                q[sw.get(g, g)] = -1 if pg == -1 else sw.get(pg, pg)
+            text += f"rtree dst={b} weight=1 chunk={chunk} parent={G._join(q)}\n"
+    return dict(n=n, coll=coll, dtype=dtype, count=count, mode=mode, engine=engine, ready=ready, text=text,
+                seed=seed)
+
+
+def _eq(a, b):
+    return np.array_equal(bits(a), bits(b))
+
+
+@pytest.mark.parametrize("seed", range(300))
+def test_fuzz(seed):
+    c = _case(seed)
+    n, dtype, count, R, text = c["n"], c["dtype"], c["count"], c["ready"], c["text"]
+    es = 4 if dtype != "bf16" else 2
+    per_rank = count * (n if c["coll"] in ("alltoall", "reducescatter") else 1)
+    out_per_rank = count * (n if c["coll"] in ("alltoall", "allgather") else 1)
+    scratch = 4 * max(per_rank, out_per_rank) * es + (32 << 20)
+    comm = pkg.Communicator.loopback(n, device=0, scratch_bytes=scratch, mode=c["mode"])
+    comm.config("timeout_ms", 20000)
+    comm.config("engine", c["engine"])
+    comm.set_strategy(c["coll"], text)
+    xs = rank_tensors(dtype, per_rank, n, base=5000 + seed)
+    prev = [rank_tensors(dtype, out_per_rank, 1, base=6000 + 7 * seed + g)[0] for g in range(n)]
+    dx = [to_dev(x, dtype) if g in R else None for g, x in enumerate(xs)]
+    dy = [to_dev(p, dtype) for p in prev]
+    if c["coll"] == "allreduce":
+        acc = seed % 3 == 0
+        comm.allreduce_lb(dx, dy, ready=R, accumulate=acc)
+        exp = oc.allreduce(xs, text, R, dtype, accumulate=acc, y_prev=prev)
+    elif c["coll"] == "allgather":
+        comm.allgather_lb(dx, dy, ready=R)
+        exp = oc.allgather(xs, text, R, dtype, prev)
+    elif c["coll"] == "alltoall":
+        comm.alltoall_lb(dx, dy, ready=R)
+        exp = oc.alltoall(xs, text, R, dtype, prev)
+    else:
+        comm.reducescatter_lb(dx, dy, ready=R)
+        exp = oc.reducescatter(xs, text, R, dtype, y_prev=prev)
+    torch.cuda.synchronize()
+    assert comm.get_async_error() == 0, c
+    for g in range(n):
+        assert _eq(to_host(dy[g], dtype), exp[g]), (g, {k: v for k, v in c.items() if k != "text"}, text)
+    comm.finalize()
