@@ -33,16 +33,20 @@ def _random_tree(rng, n):
     return parent
 
 
-def _case(seed):
-    rng = np.random.default_rng(seed)
+def _case(seed, large=False):
+    rng = np.random.default_rng(seed + (100_000 if large else 0))
     n = int(rng.integers(2, 9))
     coll = ["allreduce", "allreduce", "allgather", "alltoall", "reducescatter"][int(rng.integers(0, 5))]
     dtype = ["f32", "bf16", "i32"][int(rng.integers(0, 3))]
     big = rng.random() < 0.3
     count = int(np.exp(rng.uniform(0, np.log(3e6 if big else 2e4))))
+    if large:
+        count = int(np.exp(rng.uniform(np.log(2e5), np.log(4e6))))
     if coll in ("alltoall", "allgather", "reducescatter"):
         count = max(1, count // n)
     chunk = 16 * int(np.exp(rng.uniform(np.log(4), np.log((8 << 20) // 16))))
+    if large:
+        chunk = 16 * int(np.exp(rng.uniform(np.log(4096), np.log((8 << 20) // 16))))
     mode = ["direct", "staged"][int(rng.integers(0, 2))]
     engine = int(rng.integers(0, 3))
     ready = {g for g in range(n) if rng.random() < 0.75}
@@ -99,7 +103,17 @@ def _eq(a, b):
 
 @pytest.mark.parametrize("seed", range(300))
 def test_fuzz(seed):
-    c = _case(seed)
+    _run(_case(seed))
+
+
+@pytest.mark.parametrize("seed", range(60))
+def test_fuzz_large(seed):
+    """Large counts and chunks: multi-tile items in both kernels."""
+    _run(_case(seed, large=True))
+
+
+def _run(c):
+    seed = c["seed"]
     n, dtype, count, R, text = c["n"], c["dtype"], c["count"], c["ready"], c["text"]
     es = 4 if dtype != "bf16" else 2
     per_rank = count * (n if c["coll"] in ("alltoall", "reducescatter") else 1)
