@@ -33,9 +33,9 @@ def _random_tree(rng, n):
     return parent
 
 
-def _case(seed, large=False):
+def _case(seed, large=False, n=None):
     rng = np.random.default_rng(seed + (100_000 if large else 0))
-    n = int(rng.integers(2, 9))
+    n = int(rng.integers(2, 9)) if n is None else n
     coll = ["allreduce", "allreduce", "allgather", "alltoall", "reducescatter"][int(rng.integers(0, 5))]
     dtype = ["f32", "bf16", "i32"][int(rng.integers(0, 3))]
     big = rng.random() < 0.3
