@@ -157,10 +157,14 @@ def _dtype_code(t):
     return code
 
 
-def _stream(stream):
+def _stream(stream, device=None):
+    """Raw cudaStream_t: the given torch stream, else the current stream of
+    `device` (default: the current device)."""
     import torch
-    s = stream if stream is not None else torch.cuda.current_stream()
-    return ctypes.c_void_p(s.cuda_stream)
+    if stream is not None:
+        return ctypes.c_void_p(stream.cuda_stream)
+    dev = torch.cuda.current_device() if device is None else device
+    return ctypes.c_void_p(torch._C._cuda_getCurrentRawStream(dev))
 
 
 def _late_flag(late):
@@ -345,7 +349,7 @@ class Communicator:
 
     # ---- control
     def set_strategy(self, coll, text, stream=None):
-        s = ctypes.c_void_p(0) if stream is None else _stream(stream)
+        s = ctypes.c_void_p(0) if stream is None else _stream(stream, self.device)
         _check(_load().adapcc_set_strategy(self._h, COLL[coll], text.encode(), s), "set_strategy")
 
     def config(self, key, value):
@@ -383,7 +387,7 @@ class Communicator:
         send = x if (m >> self.rank) & 1 else None
         _check(_load().adapcc_allreduce(self._h, _ptr(send), _ptr(out), out.numel(),
                                         _dtype_code(out), m,
-                                        FLAG_ACCUMULATE if accumulate else 0, _stream(stream)),
+                                        FLAG_ACCUMULATE if accumulate else 0, _stream(stream, self.device)),
                "allreduce")
         return out
 
@@ -392,7 +396,7 @@ class Communicator:
         send = x if (m >> self.rank) & 1 else None
         cnt = out.numel() // self.nranks
         _check(_load().adapcc_allgather(self._h, _ptr(send), _ptr(out), cnt, _dtype_code(out), m,
-                                        _stream(stream)), "allgather")
+                                        _stream(stream, self.device)), "allgather")
         return out
 
     def alltoall(self, x, out, ready=None, stream=None):
@@ -400,7 +404,7 @@ class Communicator:
         send = x if (m >> self.rank) & 1 else None
         cnt = out.numel() // self.nranks
         _check(_load().adapcc_alltoall(self._h, _ptr(send), _ptr(out), cnt, _dtype_code(out), m,
-                                       _stream(stream)), "alltoall")
+                                       _stream(stream, self.device)), "alltoall")
         return out
 
     def reduce(self, x, out, root, ready=None, accumulate=False, stream=None):
@@ -410,14 +414,14 @@ class Communicator:
         n_el = (out if out is not None else x).numel()
         _check(_load().adapcc_reduce(self._h, _ptr(send), _ptr(out), n_el,
                                      _dtype_code(out if out is not None else x), root, m,
-                                     FLAG_ACCUMULATE if accumulate else 0, _stream(stream)), "reduce")
+                                     FLAG_ACCUMULATE if accumulate else 0, _stream(stream, self.device)), "reduce")
         return out
 
     def broadcast(self, x, out, root, ready=None, stream=None):
         m = self._ready_mask(ready)
         send = x if (self.rank == root and (m >> root) & 1) else None
         _check(_load().adapcc_broadcast(self._h, _ptr(send), _ptr(out), out.numel(), _dtype_code(out),
-                                        root, m, _stream(stream)), "broadcast")
+                                        root, m, _stream(stream, self.device)), "broadcast")
         return out
 
     def reducescatter(self, x, out, ready=None, accumulate=False, stream=None):
@@ -425,7 +429,7 @@ class Communicator:
         send = x if (m >> self.rank) & 1 else None
         _check(_load().adapcc_reducescatter(self._h, _ptr(send), _ptr(out), out.numel(),
                                             _dtype_code(out), m, FLAG_ACCUMULATE if accumulate else 0,
-                                            _stream(stream)), "reducescatter")
+                                            _stream(stream, self.device)), "reducescatter")
         return out
 
     # ---- zero-copy (multi-process): registered buffers, DIRECT plan over NVLink
@@ -458,7 +462,7 @@ class Communicator:
         m = self._ready_mask(ready)
         flags = (FLAG_ACCUMULATE if accumulate else 0) | _late_flag(late)
         _check(_load().adapcc_collective_zc(self._h, COLL[coll], sr, so, rr, ro, count, _dtype_code(out),
-                                            root, m, flags, _stream(stream)), coll + "_zc")
+                                            root, m, flags, _stream(stream, self.device)), coll + "_zc")
         return out
 
     # ---- loopback collectives (lists of per-virtual-rank tensors)
@@ -485,7 +489,7 @@ class Communicator:
             S, D = self._arrays(xs, outs, m)
         flags = (FLAG_ACCUMULATE if accumulate else 0) | _late_flag(late)
         _check(_load().adapcc_allreduce_lb(self._h, S, D, outs[0].numel(), _dtype_code(outs[0]), m,
-                                           flags, _stream(stream)), "allreduce_lb")
+                                           flags, _stream(stream, self.device)), "allreduce_lb")
         return outs
 
     def alltoallv_lb(self, xs, outs, counts, ready=None, stream=None):
@@ -493,7 +497,7 @@ class Communicator:
         m = self._ready_mask(ready)
         S, D = self._arrays(xs, outs, m)
         flat = (ctypes.c_uint64 * (self.nranks * self.nranks))(*[int(v) for row in counts for v in row])
-        _check(_load().adapcc_alltoallv_lb(self._h, S, D, flat, _dtype_code(outs[0]), m, _stream(stream)),
+        _check(_load().adapcc_alltoallv_lb(self._h, S, D, flat, _dtype_code(outs[0]), m, _stream(stream, self.device)),
                "alltoallv_lb")
         return outs
 
@@ -502,7 +506,7 @@ class Communicator:
         send = x if (m >> self.rank) & 1 else None
         flat = (ctypes.c_uint64 * (self.nranks * self.nranks))(*[int(v) for row in counts for v in row])
         _check(_load().adapcc_alltoallv(self._h, _ptr(send), _ptr(out), flat, _dtype_code(out), m,
-                                        _stream(stream)), "alltoallv")
+                                        _stream(stream, self.device)), "alltoallv")
         return out
 
     def late_ticket(self):
@@ -512,27 +516,27 @@ class Communicator:
 
     def signal_ready(self, rank=-1, ticket=0, stream=None):
         """Mark `rank` ready for late join after the work already on `stream`."""
-        _check(_load().adapcc_signal_ready(self._h, rank, ticket, _stream(stream)), "signal_ready")
+        _check(_load().adapcc_signal_ready(self._h, rank, ticket, _stream(stream, self.device)), "signal_ready")
 
     def allgather_lb(self, xs, outs, ready=None, stream=None):
         m = self._ready_mask(ready)
         S, D = self._arrays(xs, outs, m)
         _check(_load().adapcc_allgather_lb(self._h, S, D, outs[0].numel() // self.nranks,
-                                           _dtype_code(outs[0]), m, _stream(stream)), "allgather_lb")
+                                           _dtype_code(outs[0]), m, _stream(stream, self.device)), "allgather_lb")
         return outs
 
     def alltoall_lb(self, xs, outs, ready=None, stream=None):
         m = self._ready_mask(ready)
         S, D = self._arrays(xs, outs, m)
         _check(_load().adapcc_alltoall_lb(self._h, S, D, outs[0].numel() // self.nranks,
-                                          _dtype_code(outs[0]), m, _stream(stream)), "alltoall_lb")
+                                          _dtype_code(outs[0]), m, _stream(stream, self.device)), "alltoall_lb")
         return outs
 
     def reduce_lb(self, xs, outs, root, ready=None, accumulate=False, stream=None):
         m = self._ready_mask(ready)
         S, D = self._arrays(xs, outs, m)
         _check(_load().adapcc_reduce_lb(self._h, S, D, outs[root].numel(), _dtype_code(outs[root]), root,
-                                        m, FLAG_ACCUMULATE if accumulate else 0, _stream(stream)),
+                                        m, FLAG_ACCUMULATE if accumulate else 0, _stream(stream, self.device)),
                "reduce_lb")
         return outs
 
@@ -540,13 +544,13 @@ class Communicator:
         m = self._ready_mask(ready)
         S, D = self._arrays(xs, outs, m)
         _check(_load().adapcc_broadcast_lb(self._h, S, D, outs[0].numel(), _dtype_code(outs[0]), root, m,
-                                           _stream(stream)), "broadcast_lb")
+                                           _stream(stream, self.device)), "broadcast_lb")
         return outs
 
     def reducescatter_lb(self, xs, outs, ready=None, accumulate=False, stream=None):
         m = self._ready_mask(ready)
         S, D = self._arrays(xs, outs, m)
         _check(_load().adapcc_reducescatter_lb(self._h, S, D, outs[0].numel(), _dtype_code(outs[0]), m,
-                                               FLAG_ACCUMULATE if accumulate else 0, _stream(stream)),
+                                               FLAG_ACCUMULATE if accumulate else 0, _stream(stream, self.device)),
                "reducescatter_lb")
         return outs

@@ -46,15 +46,14 @@ struct DevPlan {
   int engine = 0;      // 0: LDG fold kernel, 1: TMA pipeline
   int kernel = 0;      // 0: LDG, 1: TMA for DIRECT plans, 2: TMA for STAGED plans
   std::vector<DevSegment> segs;
-  cudaEvent_t last_use = nullptr;
+  bool launched = false;  // enqueued at least once: freeing the tables waits for the device
   uint64_t last_tick = 0;
   bool pinned = false;  // referenced by a captured CUDA graph: never evicted
   bool joined = false;  // a LATE_JOIN call recorded late_bits (phase 2 may follow)
   ~DevPlan() {
-    if (last_use) {
-      cudaEventSynchronize(last_use);
-      cudaEventDestroy(last_use);
-    }
+    // eviction is rare (plan-cache capacity), so instead of recording an event
+    // on every call the tables are freed after the device drains
+    if (launched) cudaDeviceSynchronize();
     for (auto& s : segs) {
       cudaFree(s.tasks);
       cudaFree(s.refs);
@@ -346,7 +345,6 @@ adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, const Strategy* strat, uin
     plan->engine = c->engine != 2 ? c->engine : (traffic / std::max<size_t>(1, segs.size()) >= kTmaMinTraffic ? 1 : 0);
     plan->kernel = plan->engine == 0 ? 0 : (mode == kDirect ? 1 : 2);
   }
-  CK(cudaEventCreateWithFlags(&plan->last_use, cudaEventDisableTiming));
   for (auto& sp : segs) {
     DevSegment d;
     std::vector<Item> items = order_items(sp, c->loopback ? -1 : c->rank, rq.esize, grid_size(c, dtype, plan->kernel),
@@ -449,7 +447,7 @@ adapcc_result_t run(adapcc_comm_s* c, Coll coll, const void* const* send, void* 
     c->last_engine = plan->engine;
     ++c->launches;
   }
-  if (!capturing) CK(cudaEventRecord(plan->last_use, s));
+  plan->launched = true;
   return ADAPCC_SUCCESS;
 }
 

@@ -208,8 +208,10 @@ template <int DT>
 __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __grid_constant__ LaunchParams P) {
   __shared__ Shared sh;
   const bool sys = P.ipc;
+  Item pre{};  // thread 0: this CTA's first item, loaded together with the epoch
   if (threadIdx.x == 0) {
     sh.abort = 0;
+    if (blockIdx.x < P.nitems) pre = P.items[blockIdx.x];
     // this launch's epoch = the one the previous launch published + 1
     const uint64_t e = *reinterpret_cast<volatile unsigned long long*>(&P.state->epoch) + 1;
     sh.epoch = e;
@@ -239,16 +241,22 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
     __syncthreads();
   }
   constexpr int esize = Ops<DT>::kEsize;
-  while (!sh.abort) {
+  // Item claiming: CTA b starts with item b (no atomic), later items come from
+  // the counter offset by the grid.  A CTA whose item is among the last
+  // gridDim.x stops after it: every CTA makes exactly one such claim, so those
+  // items are all taken and no CTA pays a final failed atomic (small calls run
+  // with no claim atomics at all).
+  bool first = true, last = false;
+  while (!sh.abort && !last) {
     if (threadIdx.x == 0) {
       // claim the next item and stage its header in shared memory, so that no
       // task field stays live in registers across the fold
-      const uint32_t it = atomicAdd(&P.state->work[par], 1u);
+      const uint32_t it = first ? blockIdx.x : gridDim.x + atomicAdd(&P.state->work[par], 1u);
       sh.item = it;
       sh.bad_align = 0;
       sh.any_acc = 0;
       if (it < P.nitems) {
-        const Item item = P.items[it];
+        const Item item = first ? pre : P.items[it];
         const Task& t = P.tasks[item.task];
         Cur& c = sh.cur;
         c.tnsrc = t.nsrc;
@@ -287,6 +295,8 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
     }
     __syncthreads();
     if (sh.item >= P.nitems) break;
+    first = false;
+    last = (uint64_t)sh.item + gridDim.x >= P.nitems;
     const int nsrc = sh.cur.nsrc, ndst = sh.cur.ndst;
     const bool dropped = sh.cur.dropped;
     if (!dropped) {

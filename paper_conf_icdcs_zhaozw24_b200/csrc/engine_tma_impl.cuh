@@ -434,13 +434,18 @@ __global__ void __launch_bounds__(kTmaThreads, ADAPCC_TMA_MINB) engine_tma_kerne
   if (warp == kConsumerWarps) {
     // ================================================================ producer
     uint32_t stage = 0, sphase = 0, qi = 0, qphase = 0;
+    // claiming as in the LDG kernel: item blockIdx.x first, then the counter
+    // offset by the grid; stop after an item among the last gridDim.x
+    bool first = true, last = false;
     for (;;) {
       uint32_t it = 0;
       int stop_i = 0;
       if (lane == 0) {
-        it = atomicAdd(&P.state->work[par], 1u);
+        if (!last) it = first ? blockIdx.x : gridDim.x + atomicAdd(&P.state->work[par], 1u);
         mbar_wait(&sm.qempty[qi], qphase ^ 1);  // queue slot free
-        stop_i = it >= P.nitems || *reinterpret_cast<volatile int*>(&sm.abort) != 0;
+        stop_i = last || it >= P.nitems || *reinterpret_cast<volatile int*>(&sm.abort) != 0;
+        first = false;
+        last = last || (uint64_t)it + gridDim.x >= P.nitems;
       }
       it = __shfl_sync(0xffffffffu, it, 0);
       bool stop = __shfl_sync(0xffffffffu, stop_i, 0) != 0;
