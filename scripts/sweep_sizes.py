@@ -62,7 +62,8 @@ def main():
             xs = [torch.randn(count // n or 1, device="cuda").to(tdt) for _ in range(n)]
             ys = [torch.empty(n * xs[0].numel(), device="cuda", dtype=tdt) for _ in range(n)]
             call = lambda: comm.allgather_lb(xs, ys)  # noqa: E731
-            factor, alg_bytes = (n - 1.0) / n, n * nbytes + n * n * xs[0].numel() * es
+            # DIRECT: every shard read once, written to all n outputs
+            factor, alg_bytes = (n - 1.0) / n, n * n * xs[0].numel() * es + n * xs[0].numel() * es
         else:
             xs = [torch.randn(count, device="cuda").to(tdt) for _ in range(n)]
             ys = [torch.empty_like(x) for x in xs]
