@@ -15,6 +15,10 @@ Cost model of a reduce tree, used to choose chunk sizes:
            (eq. 2, garbled; reading Q18)
   T_f    = h_dst + ceil(S_m / C_m) * T_bottle, T_bottle = max edge gap on the
            path (eqs. 5, 6); the strategy's time is max_f T_f (eq. 4)
+AlltoAll (P:L209-211): N_ij = number of flows (all lines) traversing (i, j);
+relays do not aggregate, so a flow's first chunk reaches its destination at
+h = sum of t_ij along its route (eq. 2, a = 0) and the flow ends at
+h + ceil(S_m / C_m) * (its slowest edge) (eqs. 5, 6).
 AllReduce = the Reduce trees followed by their reversed Broadcast, pipelined
 chunk by chunk: per tree T = h_root + depth_bcast_time +
 ceil(S_m / C_m) * max(bottleneck of both stages) -- reading R6.
@@ -155,6 +159,55 @@ def allreduce_time(text, S, alpha, beta, esize=4):
         h_b = depth * t_edge
         chunks = max(1, math.ceil(S_m / chunk))
         worst = max(worst, h_red + h_b + chunks * max(b_red, t_edge))
+    return worst
+
+
+def alltoall_paths(text):
+    """Per a2a line m: (weight, chunk, {(s, d): [s, h1, .., d]}) read through
+    the product's loader (adapcc_strategy_route)."""
+    n, coll, nsubs = _A.strategy_check(text)
+    out = []
+    for m in range(nsubs):
+        w, chunk, _, _ = _A.strategy_sub(text, m)
+        paths = {(s, d): [s] + _A.strategy_route(text, m, s, d) + [d]
+                 for s in range(n) for d in range(n) if s != d}
+        out.append((w, chunk, paths))
+    return n, out
+
+
+def alltoall_link_loads(text, ready=None):
+    """N_ij = sum over all lines' flows of x^f_ij (P:L209-211 with eq. 3's
+    sum over sub-collectives).  ready: sources that send (default all)."""
+    n, lines = alltoall_paths(text)
+    src = set(range(n)) if ready is None else set(ready)
+    loads = {}
+    for _, _, paths in lines:
+        for (s, _), p in paths.items():
+            if s not in src:
+                continue
+            for e in zip(p[:-1], p[1:]):
+                loads[e] = loads.get(e, 0) + 1
+    return loads
+
+
+def alltoall_time(text, S, alpha, beta, ready=None):
+    """Predicted AlltoAll time, S bytes per (source, destination) block split
+    over the a2a lines by weight; flows of every line share links (eq. 3)."""
+    n, lines = alltoall_paths(text)
+    src = set(range(n)) if ready is None else set(ready)
+    loads = alltoall_link_loads(text, ready)
+    W = sum(w for w, _, _ in lines)
+    worst = 0.0
+    for w, chunk, paths in lines:
+        S_m = S * w / W
+        if S_m <= 0:
+            continue
+        chunks = max(1, math.ceil(S_m / chunk))
+        for (s, _), p in paths.items():
+            if s not in src:
+                continue
+            ts = [alpha[i][j] + beta[i][j] * loads[(i, j)] * chunk for i, j in zip(p[:-1], p[1:])]
+            worst = max(worst, sum(ts) + chunks * max(ts))
     return worst
 
 

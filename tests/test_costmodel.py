@@ -73,3 +73,54 @@ def test_chunk_tradeoff_latency_vs_pipelining():
     chain = G.allreduce_trees([G.chain_parent(list(range(n)))], chunk=best)
     assert CM.allreduce_time(chain, S, alpha, beta) >= CM.allreduce_time(G.allreduce_stars(n, chunk=best), S,
                                                                           alpha, beta)
+
+
+# ------------------------------------------------------------- AlltoAll (routes)
+def test_alltoall_loads_match_oracle():
+    """Product cost model's N_ij (via the C loader) = the oracle's (own parser)."""
+    import random
+
+    from oracle import loads as OL
+    from paper_conf_icdcs_zhaozw24_b200 import generator as G
+    rng = random.Random(21)
+    for _ in range(20):
+        n = rng.randint(3, 8)
+        lines = []
+        for _ in range(rng.randint(1, 3)):
+            routes = {}
+            for s in range(n):
+                for d in range(n):
+                    if s != d and rng.random() < 0.3:
+                        others = [g for g in range(n) if g not in (s, d)]
+                        routes[(s, d)] = rng.sample(others, rng.randint(1, min(2, len(others))))
+            lines.append((rng.randint(1, 3), routes))
+        text = G.alltoall_routed(n, lines)
+        R = {g for g in range(n) if rng.random() < 0.7} or {0}
+        exp = {}
+        for N in OL.alltoall_link_loads(text, R):
+            for e, v in N.items():
+                exp[e] = exp.get(e, 0) + v
+        assert CM.alltoall_link_loads(text, R) == exp
+
+
+def test_alltoall_time_closed_form_direct():
+    """Direct flows on a uniform switch: every edge carries one flow, so
+    T = t + ceil(S/C) t with t = alpha + beta C (eqs. 2, 5, 6)."""
+    from paper_conf_icdcs_zhaozw24_b200 import generator as G
+    n, C, S = 8, 1 << 20, 16 << 20
+    a, b = 2e-6, 1 / 700e9
+    A_, B_ = CM.uniform_links(n, a, b)
+    t = a + b * C
+    assert CM.alltoall_time(G.alltoall_direct(n, chunk=C), S, A_, B_) == pytest.approx(t + (S // C) * t)
+
+
+def test_alltoall_detour_around_a_slow_link_pays_off():
+    """A 10x slower link (heterogeneous links, the paper's motivation):
+    routing its flows through a relay beats the direct path in the model."""
+    from paper_conf_icdcs_zhaozw24_b200 import generator as G
+    n, C, S = 4, 1 << 20, 64 << 20
+    A_, B_ = CM.uniform_links(n, 2e-6, 1 / 700e9)
+    B_[0][1] = B_[1][0] = 10 / 700e9
+    direct = CM.alltoall_time(G.alltoall_direct(n, chunk=C), S, A_, B_)
+    detour = CM.alltoall_time(G.alltoall_detour(n, [(0, 1), (1, 0)], chunk=C), S, A_, B_)
+    assert detour < 0.5 * direct
