@@ -21,8 +21,8 @@ class AdapccHookState:
         self.ready = ready            # None = every rank
 
     def contributors(self):
-        if self.ready is None:
-            return self.comm.nranks
+        if self.ready is None:              # every live rank (all, unless some were excluded)
+            return len(self.comm.members)
         if isinstance(self.ready, int):
             return bin(self.ready).count("1")
         return len(set(self.ready))
