@@ -332,6 +332,7 @@ adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, const Strategy* strat, uin
   rq.late_join = flags & ADAPCC_FLAG_LATE_JOIN;
   rq.counts = counts;
   rq.members = c->members;
+  rq.grid = grid_size(c, dtype, 0);
   rq.mode = mode;
   rq.half_bytes = c->half_bytes;
   std::vector<SegmentPlan> segs;

@@ -50,9 +50,18 @@ BufRef make_ref(uint8_t kind, int rank, int64_t bias, bool accum = false) {
 
 class Builder {
  public:
-  Builder(int n, int esize, uint64_t half, uint64_t members)
+  Builder(int n, int esize, uint64_t half, uint64_t members, uint64_t unit_cap)
       : n_(n), esize_(esize), half_(half), flag_cap_(flag_region_bytes(half)), members_(members),
-        used_(n, 0), flags_used_(n, 0) {}
+        unit_cap_(unit_cap), used_(n, 0), flags_used_(n, 0) {}
+
+  // Pipelining unit (elements) of a sub-collective with chunk C_m: C_m, or a
+  // smaller unit when the call is too small to give every CTA work at C_m
+  // (reading R8: the strategy's chunk is the largest unit the engine moves
+  // between flags; results do not depend on it).
+  uint32_t chunk_elems(int64_t chunk_bytes) const {
+    const uint64_t b = unit_cap_ ? std::min<uint64_t>((uint64_t)chunk_bytes, unit_cap_) : (uint64_t)chunk_bytes;
+    return (uint32_t)(b / esize_);
+  }
 
   bool alive(int g) const { return ((members_ >> g) & 1) != 0; }
 
@@ -131,7 +140,7 @@ class Builder {
   }
 
   int n_, esize_;
-  uint64_t half_, flag_cap_, members_;
+  uint64_t half_, flag_cap_, members_, unit_cap_;
   std::vector<uint64_t> used_, flags_used_;
   SegmentPlan p_;
   std::map<std::pair<uint32_t, uint64_t>, int> producer_;
@@ -153,7 +162,7 @@ void plan_allreduce_tree(Builder& B, const SubColl& s, uint64_t lo, uint64_t hi,
                          bool late_join = false) {
   const int n = B.n_;
   const int es = B.esize_;
-  const uint32_t ce = (uint32_t)(s.chunk / es);
+  const uint32_t ce = B.chunk_elems(s.chunk);
   const uint32_t nch = (uint32_t)((hi - lo + ce - 1) / ce);
   const uint64_t len = (hi - lo) * es;
   const TreeBehavior b = tree_behavior(s, mask);
@@ -279,7 +288,7 @@ void plan_allgather_tree(Builder& B, const SubColl& s, uint64_t lo, uint64_t hi,
   const int es = B.esize_;
   const int src = s.src;
   if (!((mask >> src) & 1)) return;  // non-ready source: slots untouched (Q12)
-  const uint32_t ce = (uint32_t)(s.chunk / es);
+  const uint32_t ce = B.chunk_elems(s.chunk);
   const uint32_t nch = (uint32_t)((hi - lo + ce - 1) / ce);
   const uint64_t len = (hi - lo) * es;
   const int64_t slot_bias = slot_bias_override >= 0 ? slot_bias_override : (int64_t)(src * cnt * es);
@@ -348,7 +357,7 @@ void plan_alltoall_line(Builder& B, const SubColl& s, uint64_t lo, uint64_t hi, 
                         uint64_t mask, Mode mode) {
   const int n = B.n_;
   const int es = B.esize_;
-  const uint32_t ce = (uint32_t)(s.chunk / es);
+  const uint32_t ce = B.chunk_elems(s.chunk);
   for (int src = 0; src < n; ++src) {
     if (!((mask >> src) & 1)) continue;
     for (int d = 0; d < n; ++d) {
@@ -386,7 +395,7 @@ void plan_alltoallv(Builder& B, const PlanRequest& rq, uint64_t k, uint64_t nseg
         Stream in;
         in.ref = make_ref(kBufSend, src, (int64_t)(soff * es));
         plan_flow(B, src, d, s.hops(src, d), in, make_ref(kBufRecv, d, (int64_t)(roff * es)), lo, hi,
-                  (uint32_t)(s.chunk / es), rq.mode);
+                  B.chunk_elems(s.chunk), rq.mode);
       }
     }
   }
@@ -396,7 +405,15 @@ SegmentPlan build_segment(const PlanRequest& rq,
                           const std::vector<std::pair<uint64_t, uint64_t>>& ranges, uint64_t seg_k,
                           uint64_t nseg) {
   const Strategy& st = *rq.st;
-  Builder B(st.nranks, rq.esize, rq.half_bytes, rq.members);
+  // unit cap: about two flagged units per CTA over the call's bytes per rank
+  // (x n ranks), 4 KiB-aligned, at least 16 KiB
+  uint64_t unit_cap = 0;
+  if (rq.grid > 0 && !rq.counts) {
+    const uint64_t per_rank = rq.count * (uint64_t)rq.esize *
+                              ((st.coll == kAllToAll || st.coll == kAllGather || st.coll == kReduceScatter) ? st.nranks : 1);
+    unit_cap = std::max<uint64_t>(16384, per_rank * st.nranks / (2ull * rq.grid) / 4096 * 4096);
+  }
+  Builder B(st.nranks, rq.esize, rq.half_bytes, rq.members, unit_cap);
   if (rq.counts) {
     plan_alltoallv(B, rq, seg_k, nseg);
     return B.finish();

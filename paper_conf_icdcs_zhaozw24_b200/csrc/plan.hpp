@@ -50,6 +50,9 @@ struct PlanRequest {
   // Live ranks (NEXT-3: faulty ranks excluded): an excluded rank
   // owns no task and no buffer of it is read or written.
   uint64_t members = ~uint64_t(0);
+  // CTAs the call will run on (0: pipeline in units of the strategy's chunks
+  // only); small calls subdivide chunks so that every CTA gets work (R8).
+  int grid = 0;
 };
 
 // Bytes at the start of each parity half reserved for per-chunk flag words.

@@ -56,6 +56,29 @@ def main():
         torch.cuda.synchronize()
         return e0.elapsed_time(e1) / iters
 
+    def timeit_graph(fn, iters=100, reps=5):
+        """Device time per call with the host out of the loop (CUDA graph of
+        `iters` back-to-back calls), SURVEY §8(d) d-5."""
+        s = torch.cuda.Stream()
+        s.wait_stream(torch.cuda.current_stream())
+        with torch.cuda.stream(s):
+            fn()
+            torch.cuda.synchronize()
+            g = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(g, stream=s):
+                for _ in range(iters):
+                    fn()
+        torch.cuda.synchronize()
+        g.replay()
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        for _ in range(reps):
+            g.replay()
+        e1.record()
+        torch.cuda.synchronize()
+        return e0.elapsed_time(e1) / (iters * reps)
+
     def sampled_ok(ys, xs, text, R, count, dtype, k=2048):
         idx = np.unique(np.random.default_rng(5).integers(0, count, size=k))
         exp = oc.allreduce_elements([x[idx] if x is not None else None for x in xs], idx, count, text, R, dtype)
@@ -78,9 +101,11 @@ def main():
             dx = [dev(x, "f32") for x in xs]
             dy = [torch.empty_like(t) for t in dx]
             ms = timeit(lambda: comm.allreduce_lb(dx, dy), iters=200)
+            ms_g = timeit_graph(lambda: comm.allreduce_lb(dx, dy))
             exp = oc.allreduce(xs, text, {0, 1}, "f32")
             ok = all(np.array_equal(host_bits(dy[g], "f32"), exp[g].view(np.uint32)) for g in range(n))
             res.append({"mode": mode, "us": round(ms * 1e3, 2), "busbw": round(count * 4 / ms / 1e6 * 1.0, 2),
+                        "us_graph": round(ms_g * 1e3, 2), "busbw_graph": round(count * 4 / ms_g / 1e6, 2),
                         "parity_bit_exact": ok, "kernel": comm.last_engine()})
             comm.finalize()
         out["C1"] = res
