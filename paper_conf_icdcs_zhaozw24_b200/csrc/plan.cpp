@@ -407,11 +407,17 @@ SegmentPlan build_segment(const PlanRequest& rq,
   const Strategy& st = *rq.st;
   // unit cap: about two flagged units per CTA over the call's bytes per rank
   // (x n ranks), 4 KiB-aligned, at least 16 KiB
+  // and never above 1 MiB: one CTA moves a unit between flags, and larger
+  // units serialise a chunk on one SM (measured: ring / double-binary trees
+  // lose 40-60 % with 4 MiB units)
   uint64_t unit_cap = 0;
-  if (rq.grid > 0 && !rq.counts) {
-    const uint64_t per_rank = rq.count * (uint64_t)rq.esize *
-                              ((st.coll == kAllToAll || st.coll == kAllGather || st.coll == kReduceScatter) ? st.nranks : 1);
-    unit_cap = std::max<uint64_t>(16384, per_rank * st.nranks / (2ull * rq.grid) / 4096 * 4096);
+  if (rq.grid > 0) {
+    unit_cap = uint64_t(1) << 20;
+    if (!rq.counts) {
+      const uint64_t per_rank = rq.count * (uint64_t)rq.esize *
+                                ((st.coll == kAllToAll || st.coll == kAllGather || st.coll == kReduceScatter) ? st.nranks : 1);
+      unit_cap = std::min(unit_cap, std::max<uint64_t>(16384, per_rank * st.nranks / (2ull * rq.grid) / 4096 * 4096));
+    }
   }
   Builder B(st.nranks, rq.esize, rq.half_bytes, rq.members, unit_cap);
   if (rq.counts) {
@@ -523,6 +529,12 @@ std::vector<Item> order_items(const SegmentPlan& p, int rank, int esize, int gri
   const uint64_t align = 512;  // elements: keeps every piece 16-byte aligned
   struct Key { uint64_t a; uint32_t level, task, chunk, off, len; };
   std::vector<Key> keys;
+  // Claim order: key (chunk + level x lag).  Any lag >= 1 claims an item after
+  // the same chunk's items one level down (its only dependencies), which keeps
+  // the persistent grid deadlock-free.  The lag spaces a dependency about two
+  // in-flight windows (grid x queue depth) ahead of its consumer, so a claimed
+  // item rarely waits: lag = ceil(2 x grid / items per (chunk, level)).
+  uint64_t lag = 1;
   for (uint32_t t = 0; t < p.tasks.size(); ++t) {
     const Task& T = p.tasks[t];
     if (rank >= 0 && T.owner != rank) continue;
@@ -536,10 +548,19 @@ std::vector<Item> order_items(const SegmentPlan& p, int rank, int esize, int gri
       const uint64_t c0 = T.lo + (uint64_t)c * T.chunk_elems;
       const uint64_t clen = std::min<uint64_t>(T.hi, c0 + T.chunk_elems) - c0;
       for (uint64_t off = 0; off < clen; off += piece)
-        keys.push_back({(uint64_t)c + T.level, T.level, t, c, (uint32_t)off,
+        keys.push_back({(uint64_t)c, T.level, t, c, (uint32_t)off,
                         (uint32_t)std::min<uint64_t>(piece, clen - off)});
     }
   }
+  if (p.max_level > 0 && !keys.empty()) {
+    std::vector<uint64_t> chunks_at(p.max_level + 1, 0);
+    for (const Key& k : keys) chunks_at[k.level] = std::max<uint64_t>(chunks_at[k.level], (uint64_t)k.chunk + 1);
+    uint64_t slots = 0;
+    for (uint64_t v : chunks_at) slots += v;
+    const uint64_t per = std::max<uint64_t>(1, keys.size() / std::max<uint64_t>(1, slots));
+    lag = std::max<uint64_t>(1, (2ull * std::max(grid, 1) + per - 1) / per);
+  }
+  for (Key& k : keys) k.a = (uint64_t)k.chunk + (uint64_t)k.level * lag;
   std::sort(keys.begin(), keys.end(), [](const Key& x, const Key& y) {
     return std::tie(x.a, x.level, x.task, x.chunk, x.off) <
            std::tie(y.a, y.level, y.task, y.chunk, y.off);
