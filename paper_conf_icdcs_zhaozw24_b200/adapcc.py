@@ -303,8 +303,17 @@ class Communicator:
         self._keep = keep
         self.members = set(range(nranks))
 
+    @property
+    def members(self):
+        return self._members
+
+    @members.setter
+    def members(self, live):
+        self._members = set(live)
+        self._members_mask = _mask(self._members, self.nranks)
+
     def _ready_mask(self, ready):
-        return _mask(self.members if ready is None else ready, self.nranks)
+        return self._members_mask if ready is None else _mask(ready, self.nranks)
 
     # ---- fault tolerance (NEXT-3)
     def exclude(self, dead, store=None):
@@ -467,16 +476,16 @@ class Communicator:
 
     # ---- loopback collectives (lists of per-virtual-rank tensors)
     def _arrays(self, xs, outs, m):
+        """ctypes pointer arrays for the _lb calls, reused while the pointers repeat."""
+        key = [x.data_ptr() if x is not None and (m >> r) & 1 else 0 for r, x in enumerate(xs)]
+        key += [o.data_ptr() if o is not None else 0 for o in outs]
+        cached = self.__dict__.get("_arr_cache")
+        if cached is not None and cached[0] == key:
+            return cached[1], cached[2]
         n = self.nranks
-        skey = tuple((xs[r].data_ptr() if ((m >> r) & 1 and xs[r] is not None) else 0)
-                     for r in range(n))
-        dkey = tuple((o.data_ptr() if o is not None else 0) for o in outs)
-        cached = getattr(self, "_arr_cache", None)
-        if cached is not None and cached[0] == skey and cached[1] == dkey:
-            return cached[2], cached[3]
-        S = (ctypes.c_void_p * n)(*skey)
-        D = (ctypes.c_void_p * n)(*dkey)
-        self._arr_cache = (skey, dkey, S, D)
+        S = (ctypes.c_void_p * n)(*key[:n])
+        D = (ctypes.c_void_p * n)(*key[n:])
+        self._arr_cache = (key, S, D)
         return S, D
 
     def allreduce_lb(self, xs, outs, ready=None, accumulate=False, stream=None, late=None):

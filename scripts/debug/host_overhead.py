@@ -41,3 +41,13 @@ def burst():
 t0 = time.perf_counter()
 for _ in range(500): burst()
 print("burst of 8 + sync per call", (time.perf_counter() - t0) / 4000 * 1e6)
+# host-only enqueue cost: stream blocked by a long sleep kernel, 500 enqueues
+for name, fn in [("ctypes allreduce_lb", lambda: L.adapcc_allreduce_lb(comm._h, S, D, cnt, 0, m, 0, st)),
+                 ("python allreduce_lb", lambda: comm.allreduce_lb(xs, ys)),
+                 ("torch add_", lambda: xs[0].add_(0))]:
+    torch.cuda._sleep(int(2e9))
+    t0 = time.perf_counter()
+    for _ in range(500): fn()
+    t1 = time.perf_counter()
+    torch.cuda.synchronize()
+    print(f"{name:40s} host-only {(t1-t0)/500*1e6:7.2f} us/call")
