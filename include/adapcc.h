@@ -287,8 +287,17 @@ ADAPCC_API const char* adapcc_last_cuda_error(void);
 /* Runtime knobs.  key: "timeout_ms" (watchdog, default 10000; env
  * ADAPCC_TIMEOUT_MS), "max_ctas" (grid cap, 0 = #SMs x occupancy; env
  * ADAPCC_NCTAS), "engine" (2 = auto by call size, default; 1 = TMA bulk-copy
- * pipeline; 0 = 128-bit LDG/STG fold; env ADAPCC_ENGINE), "debug_drop_rank" (loopback test hook:
- * virtual rank r posts nothing, so its consumers hit the watchdog; -1 = off). */
+ * pipeline; 0 = 128-bit LDG/STG fold; env ADAPCC_ENGINE), "piece_kib" (traffic per work
+ * piece of flag-free tasks, 0 = automatic, default; env ADAPCC_PIECE_KIB), "taper" (the last
+ * ~2 x grid flag-free items are cut into this many sub-pieces, 0..64; 0 = automatic,
+ * default: 2 once a call has >= 4 items per CTA, else off; 1 = off;
+ * env ADAPCC_TAPER), "debug_check" (multi-process: 1 = every launch first compares a hash
+ * of its call -- collective, strategy, count, dtype, mask, flags, live ranks, segment, zero-copy
+ * registrations -- with every live peer's for the same launch, in the arena headers, before any
+ * byte moves; a mismatch latches ADAPCC_ERR_MISMATCH instead of corrupting data or hanging until
+ * the watchdog; 0 = off, default; env ADAPCC_DEBUG), "debug_drop_rank" (loopback test hook:
+ * virtual rank r posts nothing, so its consumers hit the watchdog; -1 = off).  Changing engine / piece_kib / taper empties the
+ * plan cache (plans a captured CUDA graph uses stay alive); results never depend on them. */
 ADAPCC_API adapcc_result_t adapcc_config(adapcc_comm_t comm, const char* key, int64_t value);
 
 /* Number of engine kernel launches this communicator has issued. */

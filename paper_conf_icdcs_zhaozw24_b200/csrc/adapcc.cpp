@@ -50,6 +50,7 @@ struct DevPlan {
   uint64_t last_tick = 0;
   bool pinned = false;  // referenced by a captured CUDA graph: never evicted
   bool joined = false;  // a LATE_JOIN call recorded late_bits (phase 2 may follow)
+  uint64_t sig = 0;     // hash of the plan key: the call every rank must agree on (debug check)
   ~DevPlan() {
     // eviction is rare (plan-cache capacity), so instead of recording an event
     // on every call the tables are freed after the device drains
@@ -143,13 +144,16 @@ struct adapcc_comm_s {
   bool user_set[kNumColl] = {};          // set_strategy was called for this collective
   std::map<int, Strategy> rooted[kNumColl];  // default Reduce/Broadcast strategies per root
   std::map<PlanKey, std::shared_ptr<DevPlan>> plans;
+  std::vector<std::shared_ptr<DevPlan>> retired;  // out of the cache, still used by a captured graph
   uint64_t tick = 0;  // plan-cache clock (least recently used plan is evicted)
   int64_t timeout_ms = 10000;
   int64_t max_ctas = 0;
   int64_t drop_rank = -1;
   uint64_t members = 0;   // live ranks (NEXT-3 fault exclusion); all ranks after init
   uint64_t late_seq = 0;  // late-join ticket of the most recent LATE_JOIN call
-  int64_t piece_kib = 0;  // 0 = automatic (total traffic / (8 * grid))
+  int64_t piece_kib = 0;  // 0 = automatic (plan.cpp:order_items)
+  int64_t taper = 0;      // tail items cut into this many sub-pieces (1 = off, 0 = auto)
+  int64_t check_sig = 0;  // debug: kernels compare call signatures across ranks (ADAPCC_DEBUG)
   uint64_t launches = 0;
   int num_sms = 148;
   // [kernel][dtype] resident CTAs per SM; kernels: 0 LDG fold, 1 TMA (DIRECT
@@ -192,6 +196,8 @@ adapcc_result_t common_init(adapcc_comm_s* c, size_t scratch) {
   c->max_ctas = env_int("ADAPCC_NCTAS", 0);
   c->engine = (int)std::min<int64_t>(2, std::max<int64_t>(0, env_int("ADAPCC_ENGINE", 2)));
   c->piece_kib = env_int("ADAPCC_PIECE_KIB", 0);
+  c->taper = std::min<int64_t>(64, std::max<int64_t>(0, env_int("ADAPCC_TAPER", 0)));
+  c->check_sig = env_int("ADAPCC_DEBUG", 0) != 0;
   CK(cudaSetDevice(c->device));
   CK(cudaDeviceGetAttribute(&c->num_sms, cudaDevAttrMultiProcessorCount, c->device));
   for (int d = 0; d < 3; ++d) {
@@ -220,6 +226,7 @@ void release(adapcc_comm_s* c) {
   cudaSetDevice(c->device);
   cudaDeviceSynchronize();
   c->plans.clear();
+  c->retired.clear();
   for (auto& o : c->opened) cudaIpcCloseMemHandle(o.second.first);
   c->opened.clear();
   if (c->loopback) {
@@ -246,6 +253,12 @@ adapcc_result_t check_common(adapcc_comm_t c, adapcc_dtype_t dtype, uint64_t mas
     return ADAPCC_ERR_INVALID_ARGUMENT;
   if (*reinterpret_cast<volatile int*>(c->h_err)) return (adapcc_result_t)*c->h_err;
   return ADAPCC_SUCCESS;
+}
+
+// FNV-1a over 64-bit words (call signatures of the debug check)
+uint64_t fnv(uint64_t h, uint64_t v) {
+  for (int i = 0; i < 8; ++i) { h ^= (v >> (8 * i)) & 0xff; h *= 1099511628211ull; }
+  return h;
 }
 
 bool misaligned(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15) != 0; }
@@ -340,6 +353,13 @@ adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, const Strategy* strat, uin
   if (!build_plan(rq, &segs, &err)) return ADAPCC_ERR_OOM;
   auto plan = std::make_shared<DevPlan>();
   {
+    uint64_t h = 1469598103934665603ull;
+    for (uint64_t v : {(uint64_t)coll, strat->hash, count, (uint64_t)dtype, mask, (uint64_t)flags, (uint64_t)mode,
+                       c->members, (uint64_t)segs.size()})
+      h = fnv(h, v);
+    plan->sig = h;
+  }
+  {
     PlanStats st;
     for (auto& sp : segs) accumulate_stats(sp, c->loopback ? -1 : c->rank, rq.esize, &st);
     const uint64_t traffic = st.bytes_read + st.bytes_written;
@@ -349,7 +369,7 @@ adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, const Strategy* strat, uin
   for (auto& sp : segs) {
     DevSegment d;
     std::vector<Item> items = order_items(sp, c->loopback ? -1 : c->rank, rq.esize, grid_size(c, dtype, plan->kernel),
-                                          (uint64_t)c->piece_kib * 1024);
+                                          (uint64_t)c->piece_kib * 1024, (int)c->taper);
     d.nitems = (uint32_t)items.size();
     auto up = [](auto** dst, const auto& v) -> cudaError_t {
       using T = typename std::decay_t<decltype(v)>::value_type;
@@ -388,7 +408,7 @@ adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, const Strategy* strat, uin
 adapcc_result_t run(adapcc_comm_s* c, Coll coll, const void* const* send, void* const* recv,
                     uint64_t count, adapcc_dtype_t dtype, uint64_t mask, unsigned flags,
                     adapcc_stream_t stream, int root = 0, char* const* zc_send = nullptr,
-                    char* const* zc_recv = nullptr, const uint64_t* counts = nullptr) {
+                    char* const* zc_recv = nullptr, const uint64_t* counts = nullptr, uint64_t sig_extra = 0) {
   const bool zc = zc_send != nullptr;
   std::lock_guard<std::mutex> lock(c->mu);
   CK(cudaSetDevice(c->device));
@@ -409,7 +429,8 @@ adapcc_result_t run(adapcc_comm_s* c, Coll coll, const void* const* send, void* 
     plan->joined = true;
     ++c->late_seq;  // ticket of this phase 1: late ranks signal it (adapcc_signal_ready)
   }
-  for (const DevSegment& seg : plan->segs) {
+  for (size_t si = 0; si < plan->segs.size(); ++si) {
+    const DevSegment& seg = plan->segs[si];
     if (c->loopback && seg.nitems == 0) continue;
     LaunchParams P{};
     P.tasks = seg.tasks;
@@ -429,6 +450,8 @@ adapcc_result_t run(adapcc_comm_s* c, Coll coll, const void* const* send, void* 
     P.members = c->members;
     P.half_bytes = c->half_bytes;
     P.timeout_ns = (uint64_t)std::max<int64_t>(1, c->timeout_ms) * 1000000ull;
+    P.check_sig = !c->loopback && c->check_sig;
+    P.sig = fnv(fnv(plan->sig, si), sig_extra);
     P.state = c->state;
     P.err = c->d_err;
     for (int q = 0; q < c->nranks; ++q) {
@@ -901,7 +924,11 @@ adapcc_result_t adapcc_collective_zc(adapcc_comm_t c, adapcc_coll_t coll, int se
     }
     if (coll == ADAPCC_ALLTOALL && overlap(S[c->rank], sb, D[c->rank], rb)) return ADAPCC_ERR_INVALID_ARGUMENT;
   }
-  return run(c, (Coll)coll, nullptr, nullptr, count, dtype, mask, flags, stream, root, S.data(), D.data());
+  uint64_t extra = 1469598103934665603ull;
+  for (uint64_t v : {(uint64_t)send_reg, (uint64_t)send_offset, (uint64_t)recv_reg, (uint64_t)recv_offset})
+    extra = fnv(extra, v);
+  return run(c, (Coll)coll, nullptr, nullptr, count, dtype, mask, flags, stream, root, S.data(), D.data(), nullptr,
+             extra);
 }
 
 // ---------------------------------------------------------- AlltoAllv (NEXT-4)
@@ -1047,6 +1074,14 @@ adapcc_result_t adapcc_finalize(adapcc_comm_t c) {
   return ADAPCC_SUCCESS;
 }
 
+// Empties the plan cache.  Plans captured into a CUDA graph stay alive until
+// finalize (the graph keeps pointing at their tables).
+static void drop_plans(adapcc_comm_t c) {
+  for (auto& kv : c->plans)
+    if (kv.second->pinned) c->retired.push_back(kv.second);
+  c->plans.clear();
+}
+
 adapcc_result_t adapcc_config(adapcc_comm_t c, const char* key, int64_t value) {
   if (!c || !key) return ADAPCC_ERR_INVALID_ARGUMENT;
   std::lock_guard<std::mutex> lock(c->mu);
@@ -1054,9 +1089,15 @@ adapcc_result_t adapcc_config(adapcc_comm_t c, const char* key, int64_t value) {
   else if (!std::strcmp(key, "max_ctas")) { if (value < 0) return ADAPCC_ERR_INVALID_ARGUMENT; c->max_ctas = value; }
   else if (!std::strcmp(key, "engine")) {
     if (value < 0 || value > 2) return ADAPCC_ERR_INVALID_ARGUMENT;
-    if (value != c->engine) c->plans.clear();  // pieces are sized for the engine's grid
+    if (value != c->engine) drop_plans(c);  // pieces are sized for the engine's grid
     c->engine = (int)value;
   }
+  else if (!std::strcmp(key, "piece_kib") || !std::strcmp(key, "taper")) {
+    if (value < 0 || (key[0] == 't' && value > 64)) return ADAPCC_ERR_INVALID_ARGUMENT;
+    (key[0] == 't' ? c->taper : c->piece_kib) = value;
+    drop_plans(c);  // items are cut at plan time
+  }
+  else if (!std::strcmp(key, "debug_check")) c->check_sig = value != 0;
   else if (!std::strcmp(key, "debug_drop_rank")) {
     if (!c->loopback || value < -1 || value >= c->nranks) return ADAPCC_ERR_INVALID_ARGUMENT;
     c->drop_rank = value;

@@ -233,11 +233,12 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
     }
     __syncthreads();
   }
+  if (P.ipc && P.check_sig && !check_call_sig(P, epoch)) sh.abort = 1;  // before any byte moves
   if (P.ipc && P.zc) {  // zero-copy: peers read/write our user buffers directly
     if (blockIdx.x == 0 && threadIdx.x == 0)
-      st_release(reinterpret_cast<uint64_t*>(P.hdr[P.my_rank] + 8), epoch, true);  // entered
+      st_release(reinterpret_cast<uint64_t*>(P.hdr[P.my_rank] + ArenaHeader::kEntered), epoch, true);  // entered
     if (threadIdx.x < P.nranks && threadIdx.x != P.my_rank && ((P.members >> threadIdx.x) & 1))
-      if (!wait_flag(reinterpret_cast<const uint64_t*>(P.hdr[threadIdx.x] + 8), epoch, P)) sh.abort = 1;
+      if (!wait_flag(reinterpret_cast<const uint64_t*>(P.hdr[threadIdx.x] + ArenaHeader::kEntered), epoch, P)) sh.abort = 1;
     __syncthreads();
   }
   constexpr int esize = Ops<DT>::kEsize;
@@ -297,7 +298,7 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
     if (sh.item >= P.nitems) break;
     first = false;
     last = (uint64_t)sh.item + gridDim.x >= P.nitems;
-    const int nsrc = sh.cur.nsrc, ndst = sh.cur.ndst;
+    const int nsrc = sh.cur.nsrc, ndst = sh.cur.ndst, npost = sh.cur.npost;
     const bool dropped = sh.cur.dropped;
     if (!dropped) {
       // input flags, one waiter thread per flag
@@ -332,7 +333,9 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
     if (!dropped) {
       fold_chunk<DT>(sh, nsrc, ndst, sh.cur.len, sh.cur.op);
       __syncthreads();
-      if (threadIdx.x == 0 && sh.cur.npost) {
+      // npost was read before the barrier: after it, only thread 0 touches
+      // sh.cur (it rewrites it for the next item)
+      if (threadIdx.x == 0 && npost) {
         const uint64_t e = sh.epoch;
         const char* const* hdr = P.hdr;
         fence(sys);  // the chunk's bytes (incl. remote NVLink stores) before its flag

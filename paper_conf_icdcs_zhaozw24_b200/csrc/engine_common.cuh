@@ -137,6 +137,36 @@ static __device__ __noinline__ bool wait_flag(const uint64_t* flag, uint64_t tar
 }
 
 
+// Debug-mode call check (mismatched calls fail loudly instead of
+// corrupting data or hanging).  Block 0 publishes this rank's call signature
+// for `epoch` in its arena header (slot epoch & 3: peers run at most one epoch
+// apart, the parity-half start check bounds them); every CTA then compares it
+// with every live peer's signature for the same epoch before moving any byte.
+// A mismatch latches ADAPCC_ERR_MISMATCH and raises the abort flag.  Returns
+// false on mismatch or watchdog timeout.  Called by all threads of the CTA.
+static __device__ bool check_call_sig(const LaunchParams& P, uint64_t epoch) {
+  const int slot = (int)(epoch & 3);
+  if (blockIdx.x == 0 && threadIdx.x == 0) {
+    char* me = P.hdr[P.my_rank];
+    *reinterpret_cast<volatile uint64_t*>(me + ArenaHeader::kSig + 8 * slot) = P.sig;
+    st_release(reinterpret_cast<uint64_t*>(me + ArenaHeader::kSigEpoch + 8 * slot), epoch, true);
+  }
+  int bad = 0;
+  const int r = threadIdx.x;
+  if (r < P.nranks && r != P.my_rank && ((P.members >> r) & 1)) {
+    const char* peer = P.hdr[r];
+    if (!wait_flag(reinterpret_cast<const uint64_t*>(peer + ArenaHeader::kSigEpoch + 8 * slot), epoch, P)) {
+      bad = 1;
+    } else if (*reinterpret_cast<const volatile uint64_t*>(peer + ArenaHeader::kSig + 8 * slot) != P.sig) {
+      *reinterpret_cast<volatile int*>(P.err) = 8;  // ADAPCC_ERR_MISMATCH
+      atomicExch(&P.state->abort, 1u);
+      __threadfence_system();
+      bad = 1;
+    }
+  }
+  return __syncthreads_or(bad) == 0;
+}
+
 // Late join ("data chunks with the same offset ... join the ongoing
 // aggregation"): which of a root task's nlate candidate ranks take part in
 // work item `item`.  Mode 1 (phase 1): candidates whose ready word
@@ -148,7 +178,8 @@ static __device__ __forceinline__ uint64_t late_select(const LaunchParams& P, co
   if (P.late_mode == 1) {
     for (int j = 0; j < t.nlate; ++j) {
       const BufRef r = P.refs[t.ref0 + t.nsrc + t.ndst + j];
-      if (ld_acquire(reinterpret_cast<const uint64_t*>(P.hdr[r.rank] + 16), P.ipc) >= P.late_ticket)
+      if (ld_acquire(reinterpret_cast<const uint64_t*>(P.hdr[r.rank] + ArenaHeader::kReady), P.ipc) >=
+          P.late_ticket)
         m |= 1ull << j;
     }
     P.late_bits[item] = m;

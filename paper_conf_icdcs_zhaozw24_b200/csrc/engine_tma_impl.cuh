@@ -423,11 +423,12 @@ __global__ void __launch_bounds__(kTmaThreads, ADAPCC_TMA_MINB) engine_tma_kerne
       if (!wait_flag(reinterpret_cast<const uint64_t*>(P.hdr[tid]), epoch - 2, P)) sm.abort = 1;
     __syncthreads();
   }
+  if (P.ipc && P.check_sig && !check_call_sig(P, epoch)) sm.abort = 1;  // before any byte moves
   if (P.ipc && P.zc) {  // zero-copy: peers read/write our user buffers directly
     if (blockIdx.x == 0 && tid == 0)
-      st_release(reinterpret_cast<uint64_t*>(P.hdr[P.my_rank] + 8), epoch, true);  // entered
+      st_release(reinterpret_cast<uint64_t*>(P.hdr[P.my_rank] + ArenaHeader::kEntered), epoch, true);  // entered
     if (tid < P.nranks && tid != P.my_rank && ((P.members >> tid) & 1))
-      if (!wait_flag(reinterpret_cast<const uint64_t*>(P.hdr[tid] + 8), epoch, P)) sm.abort = 1;
+      if (!wait_flag(reinterpret_cast<const uint64_t*>(P.hdr[tid] + ArenaHeader::kEntered), epoch, P)) sm.abort = 1;
     __syncthreads();
   }
 
@@ -440,9 +441,11 @@ __global__ void __launch_bounds__(kTmaThreads, ADAPCC_TMA_MINB) engine_tma_kerne
     for (;;) {
       uint32_t it = 0;
       int stop_i = 0;
+      if (lane == 0 && !last) it = first ? blockIdx.x : gridDim.x + atomicAdd(&P.state->work[par], 1u);
+      // queue slot free: every lane waits (acquire), since every lane rewrites
+      // the slot's descriptor that the consumers of item i - kQ were reading
+      mbar_wait(&sm.qempty[qi], qphase ^ 1);
       if (lane == 0) {
-        if (!last) it = first ? blockIdx.x : gridDim.x + atomicAdd(&P.state->work[par], 1u);
-        mbar_wait(&sm.qempty[qi], qphase ^ 1);  // queue slot free
         stop_i = last || it >= P.nitems || *reinterpret_cast<volatile int*>(&sm.abort) != 0;
         first = false;
         last = last || (uint64_t)it + gridDim.x >= P.nitems;

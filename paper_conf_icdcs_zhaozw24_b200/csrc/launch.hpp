@@ -40,11 +40,23 @@ struct LaunchParams {
   uint64_t members;     // live ranks: excluded ranks are skipped by the IPC barriers
   uint64_t half_bytes;  // bytes of one parity half of an arena
   uint64_t timeout_ns;
+  uint64_t sig;         // call signature (debug check): hash of the call every rank must agree on
+  int check_sig;        // 1: multi-process debug mode, compare `sig` with every peer's before any data moves
   DevState* state;
   int* err;             // host-mapped error word
   char* send[kMaxRanksDev];
   char* recv[kMaxRanksDev];
   char* hdr[kMaxRanksDev];  // arena base of each rank (peer-mapped): [header | half 0 | half 1]
+};
+
+// Words of the 4 KiB arena header (byte offsets).  Each rank writes only its
+// own header; peers read it over NVLink.
+struct ArenaHeader {
+  static constexpr int kDone = 0;      // last epoch this rank finished (parity-half reuse, exit barrier)
+  static constexpr int kEntered = 8;   // zero-copy: epoch this rank's kernel entered
+  static constexpr int kReady = 16;    // late join: ticket this rank signalled ready for
+  static constexpr int kSig = 64;      // debug check: call signature of epoch e in slot e & 3 ...
+  static constexpr int kSigEpoch = 96; // ... published by epoch e in slot e & 3 (release)
 };
 
 // engine.cu: 128-bit LDG/STG fold (256 threads, 2 CTAs/SM)

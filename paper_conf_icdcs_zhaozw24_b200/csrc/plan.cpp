@@ -513,7 +513,7 @@ bool build_plan(const PlanRequest& rq, std::vector<SegmentPlan>* segs, std::stri
 }
 
 std::vector<Item> order_items(const SegmentPlan& p, int rank, int esize, int grid,
-                              uint64_t piece_bytes) {
+                              uint64_t piece_bytes, int taper) {
   // Work balance: tasks that post no flags are cut into pieces of roughly
   // equal traffic so that the grid sees >= ~8 items per CTA.
   uint64_t total = 0;
@@ -565,9 +565,36 @@ std::vector<Item> order_items(const SegmentPlan& p, int rank, int esize, int gri
     return std::tie(x.a, x.level, x.task, x.chunk, x.off) <
            std::tie(y.a, y.level, y.task, y.chunk, y.off);
   });
-  std::vector<Item> items(keys.size());
-  for (size_t i = 0; i < keys.size(); ++i)
-    items[i] = {keys[i].task, keys[i].chunk, keys[i].off, keys[i].len};
+  // Tail taper: CTAs claim items dynamically, so a launch ends when its last
+  // items finish; with uniform pieces the grid idles for about half an item
+  // at the end.  The last ~2 x grid items of flag-free tasks are cut into
+  // `taper` consecutive sub-pieces (same key position, so the claim order
+  // stays topological: sub-pieces wait on the same flags and post none).
+  // taper 0 = automatic: 2 once the call has >= 4 items per CTA (measured,
+  // profiles/taper_*_r01.json: +1-3 % from 16 MiB per rank up; with fewer
+  // items the extra claims cost more than the shorter tail saves).
+  if (taper <= 0) taper = keys.size() >= 4ull * (uint64_t)std::max(grid, 1) ? 2 : 1;
+  std::vector<uint8_t> split(keys.size(), 0);
+  if (taper > 1) {
+    uint64_t want = 2ull * std::max(grid, 1);
+    for (size_t i = keys.size(); i-- > 0 && want > 0;) {
+      if (p.tasks[keys[i].task].npost != 0 || keys[i].len < (uint64_t)taper * align) continue;
+      split[i] = 1;
+      --want;
+    }
+  }
+  std::vector<Item> items;
+  items.reserve(keys.size());
+  for (size_t i = 0; i < keys.size(); ++i) {
+    const Key& k = keys[i];
+    if (!split[i]) {
+      items.push_back({k.task, k.chunk, k.off, k.len});
+      continue;
+    }
+    const uint32_t sub = (uint32_t)((k.len + (uint64_t)taper * align - 1) / ((uint64_t)taper * align) * align);
+    for (uint32_t o = 0; o < k.len; o += sub)
+      items.push_back({k.task, k.chunk, k.off + o, std::min<uint32_t>(sub, k.len - o)});
+  }
   return items;
 }
 
