@@ -53,6 +53,7 @@ def parse_args():
     p.add_argument("--e2e-steps", type=int, default=8)
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--no-parity", action="store_true")
+    p.add_argument("--no-sweep", action="store_true", help="skip the busbw-vs-size sweep")
     p.add_argument("--test-same-gpu", action="store_true",
                    help="N>1 code-path check on a 1-GPU box: every rank on cuda:0, gloo, no NCCL leg "
                         "(numbers are NOT NVLink measurements)")
@@ -147,6 +148,63 @@ class ClockSampler:
         med = s[len(s) // 2] if s else None
         return {"sm_mhz": med, "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons),
                 "samples": len(s)}
+
+
+# ------------------------------------------------------------- size sweep
+SWEEP_SIZES = [1 << s for s in range(10, 29, 2)]   # bytes per rank: 1 KiB .. 256 MiB, x4 steps
+
+
+def time_point(fn, reduce_max=None, graph=True):
+    """Per-call device time (ms) of back-to-back calls, two ways: plain
+    enqueue on the current stream ("ms", host enqueue included when it is the
+    bottleneck) and a CUDA graph of the same calls ("ms_graph", device time
+    only).  >= ~10 ms per measurement.  reduce_max: max over ranks (N>1)."""
+    import torch
+    cur = torch.cuda.current_stream()
+    for _ in range(3):
+        fn()
+    torch.cuda.synchronize()
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    a.record(cur)
+    fn()
+    b.record(cur)
+    torch.cuda.synchronize()
+    one = max(a.elapsed_time(b), 1e-3)
+    iters = int(min(1000, max(5, 10.0 / one)))
+    if reduce_max:
+        iters = int(reduce_max(float(iters), op="min"))   # same count on every rank
+        reduce_max(0.0)                                   # barrier
+    a.record(cur)
+    for _ in range(iters):
+        fn()
+    b.record(cur)
+    torch.cuda.synchronize()
+    ms = a.elapsed_time(b) / iters
+    if not graph:
+        return (reduce_max(ms) if reduce_max else ms), None
+    s = torch.cuda.Stream()
+    s.wait_stream(cur)
+    with torch.cuda.stream(s):
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g, stream=s):
+            for _ in range(iters):
+                fn()
+    torch.cuda.synchronize()
+    if reduce_max:
+        reduce_max(0.0)
+    g.replay()
+    torch.cuda.synchronize()
+    if reduce_max:
+        reduce_max(0.0)
+    a.record(cur)
+    g.replay()
+    b.record(cur)
+    torch.cuda.synchronize()
+    msg = a.elapsed_time(b) / iters
+    del g
+    if reduce_max:
+        ms, msg = reduce_max(ms), reduce_max(msg)
+    return ms, msg
 
 
 # ------------------------------------------------------------------ oracle leg
@@ -296,6 +354,18 @@ def run_single(args):
     e2e_t = e2e_pipelined(comm, host_in, dx, dy, args.e2e_steps, tdt, lambda xs, ys: comm.allreduce_lb(xs, ys))
 
     peak, peak_src = load_peaks()
+    sweep = None
+    if not args.no_sweep:   # BASELINE metric is busbw vs size: every x4 size up to the bench size
+        sweep = []
+        for sb in [b for b in SWEEP_SIZES if b <= nbytes]:
+            c = sb // es
+            xs_, ys_ = [t[:c] for t in dx], [t[:c] for t in dy]
+            ms_, msg_ = time_point(lambda: comm.allreduce_lb(xs_, ys_))
+            sweep.append({"bytes_per_rank": sb, "us": round(ms_ * 1e3, 2), "us_graph": round(msg_ * 1e3, 2),
+                          "busbw": round(busbw(sb, ms_ / 1e3, n), 2),
+                          "busbw_graph": round(busbw(sb, msg_ / 1e3, n), 2),
+                          "hbm_frac_graph": round(2 * n * sb / (msg_ / 1e3) / 1e9 / peak, 4)})
+        assert comm.get_async_error() == 0
     alg_bytes = 2 * n * nbytes   # every rank's input read once + output written once
     achieved = alg_bytes / (kern_ms / 1e3) / 1e9
     out = {
@@ -320,6 +390,10 @@ def run_single(args):
         "clocks": clk.summary(),
         "parity": parity,
         "nccl": None,
+        "sweep": sweep,
+        "sweep_how": "same call at every x4 size (slices of the bench buffers), back-to-back enqueue (us) "
+                     "and a CUDA graph of the same calls (us_graph, device time); sizes whose 2nS fit the "
+                     "126 MB L2 run partly from L2",
     }
     if not args.no_cpu_baseline:
         out["cpu_baseline"] = cpu_baseline_block(n, args.dtype)
@@ -409,6 +483,37 @@ def sampled_parity(dy, host_in, text, n, count, dtype, k=4096):
 
 
 # ---------------------------------------------------------------- our arm, N>1
+def multi_sampled_parity(comm, x, y, xh, text, world, rank, count, dtype, k=4096):
+    """One fresh zero-copy AllReduce, then every rank's input and output at the
+    same seeded indices go to rank 0, which replays the strategy on them with
+    the oracle and counts bit mismatches (None on other ranks)."""
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+
+    from oracle import collectives as oc
+    y.fill_(float("nan"))
+    comm.collective_zc("allreduce", x, y, count)
+    torch.cuda.synchronize()
+    rng = np.random.default_rng(11)
+    idx = np.unique(np.concatenate([rng.integers(0, count, size=k), [0, count - 1]]))
+    ti = torch.from_numpy(idx).to(y.device)
+    a = xh.numpy()[idx]
+    g = y.index_select(0, ti)
+    g = g.view(torch.int16).cpu().numpy() if dtype == "bf16" else g.cpu().numpy()
+    mine = (a.view(np.uint16) if dtype == "bf16" else a, g.view(np.uint16) if dtype == "bf16" else g)
+    got = [None] * world
+    dist.all_gather_object(got, mine)
+    if rank != 0:
+        return None
+    exp = oc.allreduce_elements([v[0] for v in got], idx, count, text, set(range(world)), dtype)
+    ebits = exp.view(np.uint16) if dtype == "bf16" else exp.view(np.uint32)
+    bad = sum(int(np.count_nonzero((v[1].view(np.uint16) if dtype == "bf16" else v[1].view(np.uint32)) != ebits))
+              for v in got)
+    return {"samples_per_rank": int(len(idx)), "ranks": world, "mismatches": bad,
+            "reference": "oracle.allreduce_elements (strategy-order replay) on every rank's sampled inputs, bit-exact"}
+
+
 def run_multi(args):
     import numpy as np
     import torch
@@ -500,6 +605,27 @@ def run_multi(args):
     dist.all_reduce(t, op=dist.ReduceOp.MAX)
     e2e_t = float(t.item())
     value = busbw(nbytes, ms / 1e3, world)
+
+    def reduce_max(v, op="max"):
+        t = torch.tensor([v], dtype=torch.float64, device="cpu" if args.test_same_gpu else "cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX if op == "max" else dist.ReduceOp.MIN)
+        return float(t.item())
+
+    sweep = None
+    if not args.no_sweep:   # busbw vs size, ours (zero-copy) and NCCL on the same buffers, max over ranks
+        sweep = []
+        for sb in [b for b in SWEEP_SIZES if b <= nbytes]:
+            c = sb // es
+            xs_, ys_, zs_ = x[:c], y[:c], z[:c]
+            ms_, msg_ = time_point(lambda: comm.collective_zc("allreduce", xs_, ys_, c), reduce_max)
+            pt = {"bytes_per_rank": sb, "us": round(ms_ * 1e3, 2), "us_graph": round(msg_ * 1e3, 2),
+                  "busbw": round(busbw(sb, ms_ / 1e3, world), 2),
+                  "busbw_graph": round(busbw(sb, msg_ / 1e3, world), 2)}
+            if not args.test_same_gpu:
+                nms, _ = time_point(lambda: dist.all_reduce(zs_), reduce_max, graph=False)
+                pt.update({"nccl_us": round(nms * 1e3, 2), "nccl_busbw": round(busbw(sb, nms / 1e3, world), 2)})
+            sweep.append(pt)
+    parity = None if args.no_parity else multi_sampled_parity(comm, x, y, xh, text, world, rank, count, args.dtype)
     st = pkg.adapcc.plan_stats(text, count, args.dtype, (1 << world) - 1, rank=rank)
     dir_bytes = st["remote_bytes"]   # = bytes crossing each link direction of this GPU (symmetric plan)
     res = None
@@ -525,7 +651,11 @@ def run_multi(args):
                     "ms_per_step": round(e2e_t, 3), "steps": args.e2e_steps,
                     "how": "per rank: pinned H2D of its input + collective_zc + D2H of its output; steps "
                            "double-buffered (both pairs registered), copies on separate streams; max over ranks"},
-            "gpu_launches": launches, "clocks": clk.summary(), "async_error": err,
+            "gpu_launches": launches, "clocks": clk.summary(), "async_error": err, "parity": parity,
+            "sweep": sweep,
+            "sweep_how": "every x4 size up to the bench size, slices of the registered buffers; ours = "
+                         "zero-copy AllReduce, nccl = dist.all_reduce on the same sizes; back-to-back "
+                         "enqueue (us; NCCL likewise) and, ours only, a CUDA graph (us_graph); max over ranks",
             "path": "zero-copy DIRECT plan over CUDA IPC (registered buffers)",
             "staged": {"value": round(busbw(nbytes, ms_staged / 1e3, world), 3), "unit": UNIT,
                        "ms_per_step": round(ms_staged, 4),

@@ -290,7 +290,7 @@ ADAPCC_API const char* adapcc_last_cuda_error(void);
  * pipeline; 0 = 128-bit LDG/STG fold; env ADAPCC_ENGINE), "piece_kib" (traffic per work
  * piece of flag-free tasks, 0 = automatic, default; env ADAPCC_PIECE_KIB), "taper" (the last
  * ~2 x grid flag-free items are cut into this many sub-pieces, 0..64; 0 = automatic,
- * default: 2 once a call has >= 4 items per CTA, else off; 1 = off;
+ * default: halve those of >= 384 KiB of traffic; 1 = off;
  * env ADAPCC_TAPER), "debug_check" (multi-process: 1 = every launch first compares a hash
  * of its call -- collective, strategy, count, dtype, mask, flags, live ranks, segment, zero-copy
  * registrations -- with every live peer's for the same launch, in the arena headers, before any

@@ -40,6 +40,8 @@ struct DevSegment {
   Item* items = nullptr;
   uint32_t nitems = 0;
   uint64_t* late_bits = nullptr;  // per item: late ranks folded in phase 1 (late join)
+  uint4* first = nullptr;         // LDG kernel: per-CTA first-item blobs (launch.hpp)
+  uint32_t nfirst = 0, first_words = 0;
 };
 
 struct DevPlan {
@@ -61,6 +63,7 @@ struct DevPlan {
       cudaFree(s.flags);
       cudaFree(s.items);
       cudaFree(s.late_bits);
+      cudaFree(s.first);
     }
     cudaGetLastError();  // teardown errors must not leak into a later call's check
   }
@@ -154,6 +157,7 @@ struct adapcc_comm_s {
   int64_t piece_kib = 0;  // 0 = automatic (plan.cpp:order_items)
   int64_t taper = 0;      // tail items cut into this many sub-pieces (1 = off, 0 = auto)
   int64_t check_sig = 0;  // debug: kernels compare call signatures across ranks (ADAPCC_DEBUG)
+  int64_t first_blob = 1; // LDG kernel: per-CTA first-item blobs (ADAPCC_FIRST_BLOB=0 disables)
   uint64_t launches = 0;
   int num_sms = 148;
   // [kernel][dtype] resident CTAs per SM; kernels: 0 LDG fold, 1 TMA (DIRECT
@@ -198,6 +202,7 @@ adapcc_result_t common_init(adapcc_comm_s* c, size_t scratch) {
   c->piece_kib = env_int("ADAPCC_PIECE_KIB", 0);
   c->taper = std::min<int64_t>(64, std::max<int64_t>(0, env_int("ADAPCC_TAPER", 0)));
   c->check_sig = env_int("ADAPCC_DEBUG", 0) != 0;
+  c->first_blob = env_int("ADAPCC_FIRST_BLOB", 1) != 0;
   CK(cudaSetDevice(c->device));
   CK(cudaDeviceGetAttribute(&c->num_sms, cudaDevAttrMultiProcessorCount, c->device));
   for (int d = 0; d < 3; ++d) {
@@ -382,6 +387,28 @@ adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, const Strategy* strat, uin
     CK(up(&d.refs, sp.refs));
     CK(up(&d.flags, sp.flags));
     CK(up(&d.items, items));
+    if (plan->kernel == 0 && c->first_blob) {
+      // first-item blobs: CTA b's first item is items[b] whatever the grid
+      const uint32_t nf = std::min<uint32_t>(d.nitems, (uint32_t)grid_size(c, dtype, 0));
+      uint32_t words = 0;
+      for (uint32_t b = 0; b < nf; ++b) {
+        const Task& t = sp.tasks[items[b].task];
+        words = std::max<uint32_t>(words, (uint32_t)kBlobRef0 + t.nsrc + t.ndst + t.nlate);
+      }
+      if (nf > 0 && words <= (uint32_t)kFirstMaxWords) {
+        std::vector<uint4> blob((size_t)nf * words, uint4{0, 0, 0, 0});
+        for (uint32_t b = 0; b < nf; ++b) {
+          const Task& t = sp.tasks[items[b].task];
+          char* w = reinterpret_cast<char*>(&blob[(size_t)b * words]);
+          std::memcpy(w, &items[b], sizeof(Item));
+          std::memcpy(w + 16, &t, sizeof(Task));
+          std::memcpy(w + 16 * kBlobRef0, &sp.refs[t.ref0], sizeof(BufRef) * (t.nsrc + t.ndst + t.nlate));
+        }
+        CK(up(&d.first, blob));
+        d.nfirst = nf;
+        d.first_words = words;
+      }
+    }
     if (rq.late_join) {
       CK(cudaMalloc(&d.late_bits, std::max<size_t>(1, items.size()) * sizeof(uint64_t)));
       CK(cudaMemset(d.late_bits, 0, std::max<size_t>(1, items.size()) * sizeof(uint64_t)));
@@ -438,6 +465,9 @@ adapcc_result_t run(adapcc_comm_s* c, Coll coll, const void* const* send, void* 
     P.flags = seg.flags;
     P.items = seg.items;
     P.nitems = seg.nitems;
+    P.first = seg.first;
+    P.nfirst = seg.nfirst;
+    P.first_words = seg.first_words;
     P.dtype = (int)dtype;
     P.nranks = c->nranks;
     P.my_rank = c->loopback ? -1 : c->rank;
@@ -1098,6 +1128,10 @@ adapcc_result_t adapcc_config(adapcc_comm_t c, const char* key, int64_t value) {
     drop_plans(c);  // items are cut at plan time
   }
   else if (!std::strcmp(key, "debug_check")) c->check_sig = value != 0;
+  else if (!std::strcmp(key, "first_blob")) {
+    c->first_blob = value != 0;
+    drop_plans(c);
+  }
   else if (!std::strcmp(key, "debug_drop_rank")) {
     if (!c->loopback || value < -1 || value >= c->nranks) return ADAPCC_ERR_INVALID_ARGUMENT;
     c->drop_rank = value;

@@ -51,9 +51,11 @@ struct Cur {  // header of the work item being executed (staged by thread 0)
   uint16_t nsrc, ndst, nwait, npost, op;
   uint16_t tnsrc, nreg;     // task's own source count; regular sources used
   bool dropped, force_acc;
+  bool from_blob;           // refs come from the first-item blob in shared memory
 };
 
 struct Shared {
+  uint4 blob[kFirstMaxWords];  // this CTA's first item: Item | Task | refs
   Cur cur;
   const char* src[kMaxFold];
   char* dst[kMaxDst];
@@ -209,9 +211,13 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
   __shared__ Shared sh;
   const bool sys = P.ipc;
   Item pre{};  // thread 0: this CTA's first item, loaded together with the epoch
+  // first item, its task and refs in one round trip (plan-time blob)
+  const bool use_blob = blockIdx.x < P.nfirst;
+  if (use_blob && threadIdx.x < P.first_words)
+    sh.blob[threadIdx.x] = P.first[(size_t)blockIdx.x * P.first_words + threadIdx.x];
   if (threadIdx.x == 0) {
     sh.abort = 0;
-    if (blockIdx.x < P.nitems) pre = P.items[blockIdx.x];
+    if (!use_blob && blockIdx.x < P.nitems) pre = P.items[blockIdx.x];
     // this launch's epoch = the one the previous launch published + 1
     const uint64_t e = *reinterpret_cast<volatile unsigned long long*>(&P.state->epoch) + 1;
     sh.epoch = e;
@@ -257,9 +263,11 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
       sh.bad_align = 0;
       sh.any_acc = 0;
       if (it < P.nitems) {
-        const Item item = first ? pre : P.items[it];
-        const Task& t = P.tasks[item.task];
+        const bool fb = first && blockIdx.x < P.nfirst;  // (recomputed: keeps no register live)
+        const Item item = fb ? *reinterpret_cast<const Item*>(&sh.blob[0]) : first ? pre : P.items[it];
+        const Task& t = fb ? *reinterpret_cast<const Task*>(&sh.blob[1]) : P.tasks[item.task];
         Cur& c = sh.cur;
+        c.from_blob = fb;
         c.tnsrc = t.nsrc;
         c.nreg = t.nsrc;
         c.ndst = t.ndst;
@@ -311,9 +319,12 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
       // resolve stream pointers for this piece
       if (threadIdx.x < nsrc + ndst) {
         const int i = threadIdx.x;
-        const BufRef r = i < sh.cur.nreg ? P.refs[sh.cur.ref0 + i]
-                       : i < nsrc ? P.refs[sh.cur.ref0 + sh.cur.tnsrc + ndst + nth_bit(sh.cur.late, i - sh.cur.nreg)]
-                                  : P.refs[sh.cur.ref0 + sh.cur.tnsrc + (i - nsrc)];
+        // index of this stream's ref, relative to the task's first ref
+        const uint32_t j = i < sh.cur.nreg ? i
+                         : i < nsrc ? sh.cur.tnsrc + ndst + nth_bit(sh.cur.late, i - sh.cur.nreg)
+                                    : sh.cur.tnsrc + (i - nsrc);
+        const BufRef r = sh.cur.from_blob ? *reinterpret_cast<const BufRef*>(&sh.blob[kBlobRef0 + j])
+                                          : P.refs[sh.cur.ref0 + j];
         char* base = r.kind == kBufSend ? P.send[r.rank]
                    : r.kind == kBufRecv ? P.recv[r.rank] : P.hdr[r.rank] + half_off;
         char* p = base + r.bias + (int64_t)(sh.cur.e0 * esize);
@@ -349,7 +360,10 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
   }
   __syncthreads();
   if (threadIdx.x == 0) {
-    fence(sys);
+    // across processes the done word published to peers must follow every
+    // CTA's data; in loopback only the next launch reads anything, after
+    // this one completes, so counting needs no fence
+    if (sys) fence(sys);
     const unsigned done = atomicAdd(&P.state->done[par], 1u);
     if (done == gridDim.x - 1) {
       // last CTA: publish the epoch for the next launch on this stream and,

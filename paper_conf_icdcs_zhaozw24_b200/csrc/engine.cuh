@@ -19,6 +19,10 @@ namespace adapcc {
 constexpr int kMaxFold = 64;   // max sources of one fold (<= ranks)
 constexpr int kMaxDst = 65;    // max destinations of one task (<= ranks + 1)
 constexpr int kArenaHeader = 4096;  // per-rank arena header (done epoch)
+// LDG kernel: per-CTA "first item" blob = Item, Task, then the task's refs
+// (sources, destinations, late candidates), in 16-byte words; plans whose
+// first items need more words go without blobs.
+constexpr int kFirstMaxWords = 72;
 
 enum BufKind : uint8_t { kBufSend = 0, kBufRecv = 1, kBufArena = 2 };
 enum DType : int { kF32 = 0, kBF16 = 1, kI32 = 2 };
@@ -67,5 +71,9 @@ struct Item {
   uint32_t off;   // elements from the chunk start
   uint32_t len;   // elements
 };
+static_assert(sizeof(Item) == 16, "Item layout");
+
+// first-item blob layout (16-byte words): [0] Item, [1, kBlobRef0) Task, then refs
+constexpr int kBlobRef0 = 1 + (int)((sizeof(Task) + 15) / 16);
 
 }  // namespace adapcc

@@ -28,6 +28,11 @@ struct LaunchParams {
   const FlagRef* flags;
   const Item* items;
   uint32_t nitems;
+  // LDG kernel: CTA b < nfirst reads its first item (items[b]), that item's
+  // task and refs as ONE blob of first_words 16-byte words at first + b *
+  // first_words, loaded in a single round trip together with the epoch
+  const uint4* first;
+  uint32_t nfirst, first_words;
   int dtype;
   int nranks;
   int my_rank;          // multi-process: this rank; loopback: -1

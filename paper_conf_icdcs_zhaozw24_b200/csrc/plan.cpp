@@ -570,15 +570,19 @@ std::vector<Item> order_items(const SegmentPlan& p, int rank, int esize, int gri
   // at the end.  The last ~2 x grid items of flag-free tasks are cut into
   // `taper` consecutive sub-pieces (same key position, so the claim order
   // stays topological: sub-pieces wait on the same flags and post none).
-  // taper 0 = automatic: 2 once the call has >= 4 items per CTA (measured,
-  // profiles/taper_*_r01.json: +1-3 % from 16 MiB per rank up; with fewer
-  // items the extra claims cost more than the shorter tail saves).
-  if (taper <= 0) taper = keys.size() >= 4ull * (uint64_t)std::max(grid, 1) ? 2 : 1;
+  // taper 0 = automatic: halve only items of >= 384 KiB of traffic (measured,
+  // profiles/taper_*_r01.json: +1-3 % from 16 MiB per rank up, where pieces
+  // are 448-512 KiB; halving ~110-230 KiB pieces costs more in per-item
+  // overhead than the shorter tail saves).
+  const bool auto_taper = taper <= 0;
+  if (auto_taper) taper = 2;
   std::vector<uint8_t> split(keys.size(), 0);
   if (taper > 1) {
     uint64_t want = 2ull * std::max(grid, 1);
     for (size_t i = keys.size(); i-- > 0 && want > 0;) {
-      if (p.tasks[keys[i].task].npost != 0 || keys[i].len < (uint64_t)taper * align) continue;
+      const Task& T = p.tasks[keys[i].task];
+      if (T.npost != 0 || keys[i].len < (uint64_t)taper * align) continue;
+      if (auto_taper && (uint64_t)keys[i].len * esize * (T.nsrc + T.ndst) < (384u << 10)) continue;
       split[i] = 1;
       --want;
     }

@@ -9,6 +9,8 @@ C3  partial AllReduce, 8 ranks, stragglers {3,6}: T_adapcc = end of phase 2 (pha
     T_wait = t_s + T_full, straggler lag t_s simulated by a 1-CTA spin kernel on a compute stream
 C4  AlltoAll 8 ranks, [8][512][4096] bf16 per rank
 C5  AllGather of GPT-2-XL row shards, 48 layers x 4 weights, strategy swap at call 96
+G1  local chunk reduction: Reduce of k in {2, 8} virtual 1 GiB inputs into one
+    1 GiB output (one star tree rooted at 0), fp32 and bf16; GB/s = (k+1) S / t vs the HBM peak
 Timing: CUDA events on the launching stream, warm-up first; busbw factors as nccl-tests.
 Every config also checks parity on sampled outputs against the oracle.
 """
@@ -25,7 +27,7 @@ sys.path.insert(0, ROOT)
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--out", default=os.path.join(ROOT, "gpurun_out", "configs.json"))
-    ap.add_argument("--only", default="C1,C2,C3,C4,C5")
+    ap.add_argument("--only", default="C1,C2,C3,C4,C5,G1")
     a = ap.parse_args()
 
     import numpy as np
@@ -289,6 +291,42 @@ def main():
             print("C5", res[-1], flush=True)
             comm.finalize()
         out["C5"] = res
+
+    # ------------------------------------------------------------------ G1
+    if "G1" in only:
+        res = []
+        pk = os.path.join(ROOT, "MEASURED_PEAKS.json")
+        peak = json.load(open(pk))["hbm_gbs"] if os.path.exists(pk) else 6650.0
+        nbytes = 1 << 30
+        for dtype in ("f32", "bf16"):
+            es = 4 if dtype == "f32" else 2
+            count = nbytes // es
+            tdt = torch.float32 if dtype == "f32" else torch.bfloat16
+            for k in (2, 8):
+                comm = pkg.Communicator.loopback(k, mode="direct", scratch_bytes=64 << 20)
+                text = G.reduce_trees([G.star_parent(k, 0)], chunk=1 << 20)
+                comm.set_strategy("reduce", text)
+                g = torch.Generator(device="cuda").manual_seed(7)
+                dx = [torch.randn(count, device="cuda", generator=g).to(tdt) for _ in range(k)]
+                dy = [torch.empty(count, device="cuda", dtype=tdt)] + [None] * (k - 1)
+                ms = timeit(lambda: comm.reduce_lb(dx, dy, root=0), iters=10)
+                gbs = (k + 1) * nbytes / ms / 1e6
+                # parity: the single star's fold order (root's own input, then 1..k-1) at sampled indices
+                idx = np.unique(np.random.default_rng(5).integers(0, count, size=2048))
+                ti = torch.from_numpy(idx).cuda()
+                vals = [host_bits(x.index_select(0, ti), dtype) for x in dx]
+                vals = [v.view(np.float32) if dtype == "f32" else v for v in vals]
+                exp = oc.allreduce_elements(vals, idx, count, G.allreduce_trees([G.star_parent(k, 0)]),
+                                            set(range(k)), dtype)
+                eb = exp.view(np.uint16) if dtype == "bf16" else exp.view(np.uint32)
+                ok = bool(np.array_equal(host_bits(dy[0].index_select(0, ti), dtype), eb))
+                res.append({"dtype": dtype, "k": k, "ms": round(ms, 4), "gbs": round(gbs, 1),
+                            "hbm_frac": round(gbs / peak, 4), "parity": ok, "kernel": comm.last_engine()})
+                print("G1", res[-1], flush=True)
+                del dx, dy
+                comm.finalize()
+                torch.cuda.empty_cache()
+        out["G1"] = res
 
     os.makedirs(os.path.dirname(a.out), exist_ok=True)
     json.dump(out, open(a.out, "w"), indent=1)

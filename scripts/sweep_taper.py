@@ -27,6 +27,7 @@ def main():
     ap.add_argument("--engine", type=int, default=2)
     ap.add_argument("--tapers", default="1,2,4,8")
     ap.add_argument("--pieces", default="0")
+    ap.add_argument("--blobs", default="1", help="first_blob settings (LDG kernel first-item blobs)")
     ap.add_argument("--min-log2", type=int, default=20)
     ap.add_argument("--max-log2", type=int, default=28)
     ap.add_argument("--out", default=os.path.join(ROOT, "gpurun_out", "taper.json"))
@@ -50,7 +51,8 @@ def main():
         comm.set_strategy("allreduce", G.allreduce_stars(n, chunk=256 << 10))
     else:
         comm.set_strategy("alltoall", G.alltoall_direct(n, chunk=256 << 10))
-    settings = [(int(p), int(t)) for p in a.pieces.split(",") for t in a.tapers.split(",")]
+    settings = [(int(p), int(t), int(b)) for p in a.pieces.split(",") for t in a.tapers.split(",")
+                for b in a.blobs.split(",")]
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     res = []
     for lg in range(a.min_log2, a.max_log2 + 1):
@@ -60,9 +62,10 @@ def main():
         ys = [torch.empty_like(x) for x in xs]
         fn = comm.allreduce_lb if a.coll == "allreduce" else comm.alltoall_lb
         graphs = {}
-        for (pc, tp) in settings:
+        for (pc, tp, bl) in settings:
             comm.config("piece_kib", pc)
             comm.config("taper", tp)
+            comm.config("first_blob", bl)
             for _ in range(3):
                 fn(xs, ys)
             torch.cuda.synchronize()
@@ -75,7 +78,7 @@ def main():
             with torch.cuda.graph(g):
                 for _ in range(iters):
                     fn(xs, ys)
-            graphs[(pc, tp)] = (g, iters)
+            graphs[(pc, tp, bl)] = (g, iters)
         times = {s: [] for s in settings}
         for _ in range(3):
             for s in settings:
@@ -89,7 +92,8 @@ def main():
                 times[s].append(e0.elapsed_time(e1) / iters)
         for s in settings:
             ms = statistics.median(times[s])
-            res.append({"bytes_per_rank": nbytes, "piece_kib": s[0], "taper": s[1], "us": round(ms * 1e3, 3),
+            res.append({"bytes_per_rank": nbytes, "piece_kib": s[0], "taper": s[1], "first_blob": s[2],
+                        "us": round(ms * 1e3, 3),
                         "hbm_frac": round(2 * n * nbytes / (ms * 1e-3) / 1e9 / peak, 4)})
             print(json.dumps(res[-1]), flush=True)
         del graphs, xs, ys

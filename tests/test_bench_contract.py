@@ -1,0 +1,68 @@
+"""bench.py keeps the driver's JSON-line contract (one line, required keys).
+
+CPU: the reference arm (the oracle timed on the host).  GPU (-m gpu): our arm
+at N=1 (loopback) and the N>1 code path with 2 processes on one GPU
+(--test-same-gpu), each with sampled oracle parity at 0 mismatches.
+"""
+
+import json
+import os
+import subprocess
+import sys
+
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+KEYS = {"metric", "value", "unit", "n_gpus", "steps", "warmup", "ms_per_step", "higher_is_better",
+        "scaling", "vs_baseline", "dtype", "data", "config", "e2e"}
+
+
+def _run(cmd, timeout=600, env=None):
+    e = dict(os.environ)
+    e.update(env or {})
+    p = subprocess.run(cmd, cwd=ROOT, capture_output=True, text=True, timeout=timeout, env=e)
+    assert p.returncode == 0, p.stderr[-3000:]
+    lines = [ln for ln in p.stdout.splitlines() if ln.startswith("{")]
+    assert len(lines) == 1, p.stdout[-3000:]
+    return json.loads(lines[0])
+
+
+def test_reference_arm_contract():
+    d = _run([sys.executable, "bench.py", "--impl", "reference", "--steps", "2", "--warmup", "1"])
+    assert KEYS <= d.keys()
+    assert d["impl"] == "reference" and d["value"] > 0 and d["unit"] == "GB/s"
+    assert d["cpu_baseline"]["kind"] == "oracle" and d["cpu_baseline"]["cores"] == 1
+    assert d["e2e"]["h2d_bytes_per_step"] == 0 and d["e2e"]["value"] == d["value"]
+    assert d["config"]["workload"].startswith("allreduce-loopback-vr8")
+
+
+@pytest.mark.gpu
+def test_ours_single_gpu_contract():
+    torch = pytest.importorskip("torch")
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    d = _run([sys.executable, "bench.py", "--steps", "3", "--warmup", "3", "--size-mib", "16",
+              "--no-cpu-baseline", "--e2e-steps", "2"])
+    assert KEYS | {"roofline", "gpu_launches", "clocks", "parity"} <= d.keys()
+    assert d["n_gpus"] == 1 and d["value"] > 0 and d["gpu_launches"] == 3
+    assert d["parity"]["mismatches"] == 0
+    r = d["roofline"]
+    assert r["bound"] == "hbm" and r["achieved"] > 0 and abs(r["frac"] - r["achieved"] / r["peak"]) < 1e-3
+    assert d["e2e"]["h2d_bytes_per_step"] == 8 * (16 << 20)
+    sw = d["sweep"]   # busbw vs size: every x4 size from 1 KiB up to the bench size
+    assert [p["bytes_per_rank"] for p in sw] == [1 << s for s in range(10, 25, 2)]
+    assert all(p["busbw"] > 0 and p["busbw_graph"] > 0 for p in sw)
+
+
+@pytest.mark.gpu
+def test_ours_two_ranks_same_gpu_contract():
+    torch = pytest.importorskip("torch")
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    d = _run([sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
+              "--master-addr", "127.0.0.1", "--master-port", "29517", "bench.py", "--gpus", "2",
+              "--steps", "3", "--warmup", "3", "--size-mib", "8", "--e2e-steps", "2", "--test-same-gpu"])
+    assert KEYS | {"roofline", "gpu_launches", "parity", "staged"} <= d.keys()
+    assert d["n_gpus"] == 2 and d["async_error"] == 0
+    assert d["parity"]["mismatches"] == 0 and d["parity"]["ranks"] == 2
+    assert [p["bytes_per_rank"] for p in d["sweep"]] == [1 << s for s in range(10, 24, 2)]
