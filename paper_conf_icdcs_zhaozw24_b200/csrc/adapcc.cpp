@@ -8,6 +8,7 @@
 // call is one engine launch per segment on the caller's stream.
 #include <cuda_runtime.h>
 #include <dlfcn.h>
+#include <nvtx3/nvToolsExt.h>  // header-only NVTX ranges: free unless a profiler (nsys) is attached
 
 #include <algorithm>
 #include <cstdio>
@@ -437,6 +438,12 @@ adapcc_result_t run(adapcc_comm_s* c, Coll coll, const void* const* send, void* 
                     adapcc_stream_t stream, int root = 0, char* const* zc_send = nullptr,
                     char* const* zc_recv = nullptr, const uint64_t* counts = nullptr, uint64_t sig_extra = 0) {
   const bool zc = zc_send != nullptr;
+  // tracing: one NVTX range per collective call on the host timeline
+  static const char* const kRange[kNumColl + 1] = {"adapcc::allreduce", "adapcc::allgather", "adapcc::alltoall",
+                                                   "adapcc::reduce", "adapcc::broadcast", "adapcc::reducescatter",
+                                                   "adapcc::alltoallv"};
+  nvtxRangePushA(kRange[counts ? kNumColl : (int)coll]);
+  struct Pop { ~Pop() { nvtxRangePop(); } } pop;
   std::lock_guard<std::mutex> lock(c->mu);
   CK(cudaSetDevice(c->device));
   const Strategy* strat = nullptr;

@@ -48,6 +48,10 @@ constexpr uint32_t kStageBytes = ADAPCC_TMA_STAGE_KB * 1024;
 constexpr bool kLargeTiles = kStageBytes > 32 * 1024;
 constexpr int kMaxKS = (kStageBytes / 4096) < 8 ? (int)(kStageBytes / 4096) : 8;  // sources per stage
 constexpr int kQ = 2;           // item queue depth
+#ifndef ADAPCC_FOLD_TMA
+#define ADAPCC_FOLD_TMA 1        // K >= 2 folds stored by TMA bulk stores from shared memory
+#endif
+constexpr bool kFoldTma = ADAPCC_FOLD_TMA != 0;
 constexpr int kMaxPost = 4;
 
 struct ItemDesc {
@@ -136,6 +140,10 @@ __device__ __forceinline__ void consumer_sync() {
   asm volatile("bar.sync 1, %0;" ::"n"(kConsumers) : "memory");
 }
 __device__ __forceinline__ uint4 lds16(const char* p) { return *reinterpret_cast<const uint4*>(p); }
+__device__ __forceinline__ void sts16(char* p, uint4 v) { *reinterpret_cast<uint4*>(p) = v; }
+__device__ __forceinline__ void fence_proxy_async_smem() {  // generic-proxy smem writes -> async proxy (TMA)
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
 
 // ------------------------------------------------------------ consumers
 template <int DT>
@@ -260,6 +268,50 @@ __device__ __forceinline__ void copy_tma(Smem& sm, char* stages, const ItemDesc&
     const uint32_t total = stage + d.ntiles;
     sphase ^= (total / kStages) & 1;
     stage = total % kStages;
+  }
+}
+
+// Fold the tiles of a K >= 2 item whose destinations are all plain stores
+// (no accumulation) and whose sources fit one stage: the consumers fold each
+// vector in shared memory, in place over source 0's tile, and one thread
+// stores the folded tile to every destination with TMA bulk stores (as
+// copy_tma does for K = 1).  Consumer threads then issue no global stores at
+// all; a stage is released once its bulk stores have read it.
+template <int DT>
+__device__ __forceinline__ void consume_fold_tma(Smem& sm, char* stages, const ItemDesc& d, int tid,
+                                                 uint32_t& stage, uint32_t& sphase) {
+  using O = Ops<DT>;
+  const uint32_t tile = d.tile, vec_bytes = d.vec_bytes, ntiles = d.ntiles;
+  const int ks = d.nsrc, ndst = d.ndst;
+  int prev = -1;  // tid 0: the stage whose bulk stores may still be reading it
+  for (uint32_t t = 0; t < ntiles; ++t) {
+    const uint32_t tb = min(tile, vec_bytes - t * tile);
+    const uint32_t nv = tb / 16;
+    mbar_wait(&sm.full[stage], sphase);
+    char* sb = stages + (size_t)stage * kStageBytes;
+#pragma unroll 2
+    for (uint32_t v = tid; v < nv; v += kConsumers) {
+      char* pv = sb + (size_t)v * 16;
+      typename O::Acc a = O::widen(lds16(pv));
+      for (int k = 1; k < ks; ++k) O::add(a, lds16(pv + (size_t)k * tile));
+      sts16(pv, O::narrow(a));  // one rounding; each thread overwrites only vectors it read
+    }
+    fence_proxy_async_smem();
+    consumer_sync();  // the whole folded tile is in shared memory
+    if (tid == 0) {
+      for (int k = 0; k < ndst; ++k) tma_store(d.dst[k] + (size_t)t * tile, sb, tb);
+      tma_store_commit();
+      if (prev >= 0) {
+        tma_store_wait_read<1>();
+        mbar_arrive_cnt(&sm.empty[prev], kConsumerWarps);
+      }
+      prev = (int)stage;
+    }
+    if (++stage == kStages) { stage = 0; sphase ^= 1; }
+  }
+  if (tid == 0 && prev >= 0) {
+    tma_store_wait_read<0>();
+    mbar_arrive_cnt(&sm.empty[prev], kConsumerWarps);
   }
 }
 
@@ -514,6 +566,12 @@ __global__ void __launch_bounds__(kTmaThreads, ADAPCC_TMA_MINB) engine_tma_kerne
           if (!d.scalar_only) {
             const uint32_t vpt = d.tile / (16u * kConsumers);  // tile / one round of 1 vector per thread
             if (d.nsrc == 1 && !d.any_acc) copy_tma(sm, stages, d, tid, stage, sphase);
+            // TMA-stored fold where per-thread stores are the cost: tiles above 16 KiB (K = 2, 3 in
+            // 64 KiB stages, else fold_rounds; G1 k = 2: 0.86 -> 1.02 of the copy peak) or >= 3
+            // destinations (star roots); with 1-2 destinations of small tiles the register path,
+            // which frees the stage before storing, is as fast or faster (G1 k = 8: 1.08 vs 1.04)
+            else if (kFoldTma && !d.any_acc && d.passes == 1 && (d.tile > 16384 || d.ndst >= 3))
+              consume_fold_tma<DT>(sm, stages, d, tid, stage, sphase);
             else if (d.nsrc == 1) consume_copy<DT, 8>(sm, stages, d, tid, stage, sphase);
             else if (vpt >= 4) consume_fold<DT, 4>(sm, stages, d, tid, stage, sphase);
             else if (vpt >= 2) consume_fold<DT, 2>(sm, stages, d, tid, stage, sphase);

@@ -401,6 +401,9 @@ void plan_alltoallv(Builder& B, const PlanRequest& rq, uint64_t k, uint64_t nseg
   }
 }
 
+SegmentPlan build_units(const PlanRequest& rq, const std::vector<std::pair<uint64_t, uint64_t>>& ranges,
+                        uint64_t seg_k, uint64_t nseg, uint64_t unit_cap);
+
 SegmentPlan build_segment(const PlanRequest& rq,
                           const std::vector<std::pair<uint64_t, uint64_t>>& ranges, uint64_t seg_k,
                           uint64_t nseg) {
@@ -419,6 +422,20 @@ SegmentPlan build_segment(const PlanRequest& rq,
       unit_cap = std::min(unit_cap, std::max<uint64_t>(16384, per_rank * st.nranks / (2ull * rq.grid) / 4096 * 4096));
     }
   }
+  SegmentPlan p = build_units(rq, ranges, seg_k, nseg, unit_cap);
+  // The cap only matters where units pipeline between flags.  A flag-free
+  // plan (DIRECT star / AllGather / AlltoAll) keeps C_m: its work balance
+  // comes from pieces (order_items), and capped units would only shrink them
+  // (AlltoAll at 1 MiB per rank: 2 item rounds instead of 1, 5.4 -> 7.0 us).
+  bool flagged = false;
+  for (const Task& t : p.tasks) flagged |= t.nwait != 0 || t.npost != 0;
+  if (!flagged && unit_cap) p = build_units(rq, ranges, seg_k, nseg, 0);
+  return p;
+}
+
+SegmentPlan build_units(const PlanRequest& rq, const std::vector<std::pair<uint64_t, uint64_t>>& ranges,
+                        uint64_t seg_k, uint64_t nseg, uint64_t unit_cap) {
+  const Strategy& st = *rq.st;
   Builder B(st.nranks, rq.esize, rq.half_bytes, rq.members, unit_cap);
   if (rq.counts) {
     plan_alltoallv(B, rq, seg_k, nseg);
