@@ -291,12 +291,18 @@ ADAPCC_API const char* adapcc_last_cuda_error(void);
  * piece of flag-free tasks, 0 = automatic, default; env ADAPCC_PIECE_KIB), "taper" (the last
  * ~2 x grid flag-free items are cut into this many sub-pieces, 0..64; 0 = automatic,
  * default: halve those of >= 384 KiB of traffic; 1 = off;
- * env ADAPCC_TAPER), "debug_check" (multi-process: 1 = every launch first compares a hash
+ * env ADAPCC_TAPER), "sched" (LDG fold kernel: 0 = CTAs claim items from a counter; 1 or 2 =
+ * static schedule, default: CTA b runs items b, b + grid, ... and prefetches each item's
+ * descriptor blob while it folds the previous one -- plans whose blobs exceed 64 MiB claim
+ * dynamically; env ADAPCC_SCHED), "pdl" (1 = launch engine kernels as programmatic dependent
+ * launches: a kernel's prologue overlaps the previous kernel on the stream, default; 0 = off;
+ * env ADAPCC_PDL), "first_blob" (LDG fold kernel: 1 = item descriptors as per-item blobs,
+ * default; 0 = plain item/task/ref tables; env ADAPCC_FIRST_BLOB), "debug_check" (multi-process: 1 = every launch first compares a hash
  * of its call -- collective, strategy, count, dtype, mask, flags, live ranks, segment, zero-copy
  * registrations -- with every live peer's for the same launch, in the arena headers, before any
  * byte moves; a mismatch latches ADAPCC_ERR_MISMATCH instead of corrupting data or hanging until
  * the watchdog; 0 = off, default; env ADAPCC_DEBUG), "debug_drop_rank" (loopback test hook:
- * virtual rank r posts nothing, so its consumers hit the watchdog; -1 = off).  Changing engine / piece_kib / taper empties the
+ * virtual rank r posts nothing, so its consumers hit the watchdog; -1 = off).  Changing engine / piece_kib / taper / sched / first_blob empties the
  * plan cache (plans a captured CUDA graph uses stay alive); results never depend on them. */
 ADAPCC_API adapcc_result_t adapcc_config(adapcc_comm_t comm, const char* key, int64_t value);
 

@@ -33,6 +33,7 @@ namespace {
 
 constexpr size_t kDefaultScratch = size_t(1) << 30;
 constexpr int kPlanCacheCap = 64;
+constexpr uint64_t kMaxBlobBytes = uint64_t(64) << 20;  // per segment: larger plans claim dynamically
 
 struct DevSegment {
   Task* tasks = nullptr;
@@ -43,6 +44,7 @@ struct DevSegment {
   uint64_t* late_bits = nullptr;  // per item: late ranks folded in phase 1 (late join)
   uint4* first = nullptr;         // LDG kernel: per-CTA first-item blobs (launch.hpp)
   uint32_t nfirst = 0, first_words = 0;
+  uint32_t sched_static = 0;      // LDG kernel: every item has a blob, CTA b runs b, b + grid, ...
 };
 
 struct DevPlan {
@@ -159,6 +161,8 @@ struct adapcc_comm_s {
   int64_t taper = 0;      // tail items cut into this many sub-pieces (1 = off, 0 = auto)
   int64_t check_sig = 0;  // debug: kernels compare call signatures across ranks (ADAPCC_DEBUG)
   int64_t first_blob = 1; // LDG kernel: per-CTA first-item blobs (ADAPCC_FIRST_BLOB=0 disables)
+  int64_t pdl = 1;        // programmatic dependent launch of the engine kernels (ADAPCC_PDL)
+  int64_t sched = 2;      // LDG kernel: 0 dynamic claims, 1 static blob schedule, 2 auto (ADAPCC_SCHED)
   uint64_t launches = 0;
   int num_sms = 148;
   // [kernel][dtype] resident CTAs per SM; kernels: 0 LDG fold, 1 TMA (DIRECT
@@ -204,6 +208,8 @@ adapcc_result_t common_init(adapcc_comm_s* c, size_t scratch) {
   c->taper = std::min<int64_t>(64, std::max<int64_t>(0, env_int("ADAPCC_TAPER", 0)));
   c->check_sig = env_int("ADAPCC_DEBUG", 0) != 0;
   c->first_blob = env_int("ADAPCC_FIRST_BLOB", 1) != 0;
+  c->pdl = env_int("ADAPCC_PDL", 1) != 0;
+  c->sched = std::min<int64_t>(2, std::max<int64_t>(0, env_int("ADAPCC_SCHED", 2)));
   CK(cudaSetDevice(c->device));
   CK(cudaDeviceGetAttribute(&c->num_sms, cudaDevAttrMultiProcessorCount, c->device));
   for (int d = 0; d < 3; ++d) {
@@ -289,7 +295,10 @@ bool overlap(const void* a, size_t an, const void* b, size_t bn) {
 
 // Measured crossover (profiles/sizes_*_r01.json): below ~64 MiB of traffic per
 // launch the LDG kernel's lower fixed cost wins, above it the TMA pipeline.
-constexpr uint64_t kTmaMinTraffic = uint64_t(64) << 20;
+// auto engine: the TMA pipeline from 128 MiB of traffic per launch; below, the
+// LDG fold's lower fixed cost wins (profiles/pieces_r01.json: 8 virtual ranks
+// x 4 MiB = 64 MiB of traffic, LDG 10.4 us vs TMA 13.4 us)
+constexpr uint64_t kTmaMinTraffic = uint64_t(128) << 20;
 
 int grid_size(const adapcc_comm_s* c, adapcc_dtype_t dtype, int kernel) {
   int grid = c->num_sms * c->occ[kernel][(int)dtype];
@@ -375,7 +384,7 @@ adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, const Strategy* strat, uin
   for (auto& sp : segs) {
     DevSegment d;
     std::vector<Item> items = order_items(sp, c->loopback ? -1 : c->rank, rq.esize, grid_size(c, dtype, plan->kernel),
-                                          (uint64_t)c->piece_kib * 1024, (int)c->taper);
+                                          (uint64_t)c->piece_kib * 1024, (int)c->taper, plan->kernel != 0);
     d.nitems = (uint32_t)items.size();
     auto up = [](auto** dst, const auto& v) -> cudaError_t {
       using T = typename std::decay_t<decltype(v)>::value_type;
@@ -389,13 +398,22 @@ adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, const Strategy* strat, uin
     CK(up(&d.flags, sp.flags));
     CK(up(&d.items, items));
     if (plan->kernel == 0 && c->first_blob) {
-      // first-item blobs: CTA b's first item is items[b] whatever the grid
-      const uint32_t nf = std::min<uint32_t>(d.nitems, (uint32_t)grid_size(c, dtype, 0));
+      // Item blobs (launch.hpp): item i, its task and the task's refs in one
+      // run of 16-byte words.  Static schedule: every item gets one, CTA b runs
+      // items b, b + grid, ... and prefetches the next blob while it folds (no
+      // claim atomic and no item -> task -> refs chain per item).  Otherwise
+      // only CTA b's first item (items[b]) has one, whatever the grid.
+      auto words_of = [&](uint32_t i) {
+        const Task& t = sp.tasks[items[i].task];
+        return (uint32_t)kBlobRef0 + t.nsrc + t.ndst + t.nlate;
+      };
+      uint32_t all_words = 0;
+      for (uint32_t i = 0; i < d.nitems; ++i) all_words = std::max(all_words, words_of(i));
+      const bool stat = c->sched != 0 && d.nitems > 0 && all_words <= (uint32_t)kFirstMaxWords &&
+                        (uint64_t)d.nitems * all_words * 16 <= kMaxBlobBytes;
+      const uint32_t nf = stat ? d.nitems : std::min<uint32_t>(d.nitems, (uint32_t)grid_size(c, dtype, 0));
       uint32_t words = 0;
-      for (uint32_t b = 0; b < nf; ++b) {
-        const Task& t = sp.tasks[items[b].task];
-        words = std::max<uint32_t>(words, (uint32_t)kBlobRef0 + t.nsrc + t.ndst + t.nlate);
-      }
+      for (uint32_t b = 0; b < nf; ++b) words = std::max(words, words_of(b));
       if (nf > 0 && words <= (uint32_t)kFirstMaxWords) {
         std::vector<uint4> blob((size_t)nf * words, uint4{0, 0, 0, 0});
         for (uint32_t b = 0; b < nf; ++b) {
@@ -408,6 +426,7 @@ adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, const Strategy* strat, uin
         CK(up(&d.first, blob));
         d.nfirst = nf;
         d.first_words = words;
+        d.sched_static = stat ? 1 : 0;
       }
     }
     if (rq.late_join) {
@@ -475,6 +494,7 @@ adapcc_result_t run(adapcc_comm_s* c, Coll coll, const void* const* send, void* 
     P.first = seg.first;
     P.nfirst = seg.nfirst;
     P.first_words = seg.first_words;
+    P.sched_static = seg.sched_static;
     P.dtype = (int)dtype;
     P.nranks = c->nranks;
     P.my_rank = c->loopback ? -1 : c->rank;
@@ -503,8 +523,9 @@ adapcc_result_t run(adapcc_comm_s* c, Coll coll, const void* const* send, void* 
       P.hdr[q] = c->arena[q];
     }
     const int grid = std::max(1, std::min<int>(grid_size(c, dtype, plan->kernel), (int)std::max<uint32_t>(1, seg.nitems)));
-    CK(plan->kernel == 1 ? tma_direct::launch(P, grid, s)
-       : plan->kernel == 2 ? tma_staged::launch(P, grid, s) : engine_launch(P, grid, s));
+    const bool pdl = c->pdl != 0;
+    CK(plan->kernel == 1 ? tma_direct::launch(P, grid, s, pdl)
+       : plan->kernel == 2 ? tma_staged::launch(P, grid, s, pdl) : engine_launch(P, grid, s, pdl));
     c->last_engine = plan->engine;
     ++c->launches;
   }
@@ -1135,6 +1156,12 @@ adapcc_result_t adapcc_config(adapcc_comm_t c, const char* key, int64_t value) {
     drop_plans(c);  // items are cut at plan time
   }
   else if (!std::strcmp(key, "debug_check")) c->check_sig = value != 0;
+  else if (!std::strcmp(key, "pdl")) c->pdl = value != 0;
+  else if (!std::strcmp(key, "sched")) {
+    if (value < 0 || value > 2) return ADAPCC_ERR_INVALID_ARGUMENT;
+    c->sched = value;
+    drop_plans(c);  // blobs are built at plan time
+  }
   else if (!std::strcmp(key, "first_blob")) {
     c->first_blob = value != 0;
     drop_plans(c);

@@ -51,11 +51,11 @@ struct Cur {  // header of the work item being executed (staged by thread 0)
   uint16_t nsrc, ndst, nwait, npost, op;
   uint16_t tnsrc, nreg;     // task's own source count; regular sources used
   bool dropped, force_acc;
-  bool from_blob;           // refs come from the first-item blob in shared memory
+  int8_t blob;              // refs come from blob buffer `blob` in shared memory (-1: from P.refs)
 };
 
 struct Shared {
-  uint4 blob[kFirstMaxWords];  // this CTA's first item: Item | Task | refs
+  uint4 blob[2][kFirstMaxWords];  // item blobs: Item | Task | refs (static schedule: double-buffered)
   Cur cur;
   const char* src[kMaxFold];
   char* dst[kMaxDst];
@@ -66,6 +66,14 @@ struct Shared {
   int abort;
   int any_acc;
 };
+
+// 16-byte global -> shared copy that completes asynchronously (blob prefetch)
+__device__ __forceinline__ void cp_async16(void* smem, const void* gmem) {
+  const unsigned s = (unsigned)__cvta_generic_to_shared(smem);
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(s), "l"(gmem) : "memory");
+  asm volatile("cp.async.commit_group;\n" ::: "memory");
+}
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;\n" ::: "memory"); }
 
 // ---------------------------------------------------------------- vector fold
 // Thread t handles vectors base, base + 256, ..., base + (U-1)*256 of a
@@ -214,10 +222,16 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
   // first item, its task and refs in one round trip (plan-time blob)
   const bool use_blob = blockIdx.x < P.nfirst;
   if (use_blob && threadIdx.x < P.first_words)
-    sh.blob[threadIdx.x] = P.first[(size_t)blockIdx.x * P.first_words + threadIdx.x];
+    sh.blob[0][threadIdx.x] = P.first[(size_t)blockIdx.x * P.first_words + threadIdx.x];
+  const bool stat = P.sched_static != 0;
+  int buf = 0;  // blob buffer of the current item (static schedule)
+  if (threadIdx.x == 0 && !use_blob && blockIdx.x < P.nitems) pre = P.items[blockIdx.x];
+  // the plan tables above are immutable; the epoch, counters, arenas and user
+  // buffers below belong to the stream order (PDL: the previous launch)
+  pdl_trigger();
+  pdl_wait();
   if (threadIdx.x == 0) {
     sh.abort = 0;
-    if (!use_blob && blockIdx.x < P.nitems) pre = P.items[blockIdx.x];
     // this launch's epoch = the one the previous launch published + 1
     const uint64_t e = *reinterpret_cast<volatile unsigned long long*>(&P.state->epoch) + 1;
     sh.epoch = e;
@@ -258,16 +272,17 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
     if (threadIdx.x == 0) {
       // claim the next item and stage its header in shared memory, so that no
       // task field stays live in registers across the fold
-      const uint32_t it = first ? blockIdx.x : gridDim.x + atomicAdd(&P.state->work[par], 1u);
+      const uint32_t it = first ? blockIdx.x : stat ? sh.item + gridDim.x
+                                                    : gridDim.x + atomicAdd(&P.state->work[par], 1u);
       sh.item = it;
       sh.bad_align = 0;
       sh.any_acc = 0;
       if (it < P.nitems) {
-        const bool fb = first && blockIdx.x < P.nfirst;  // (recomputed: keeps no register live)
-        const Item item = fb ? *reinterpret_cast<const Item*>(&sh.blob[0]) : first ? pre : P.items[it];
-        const Task& t = fb ? *reinterpret_cast<const Task*>(&sh.blob[1]) : P.tasks[item.task];
+        const bool fb = stat || (first && blockIdx.x < P.nfirst);  // (recomputed: keeps no register live)
+        const Item item = fb ? *reinterpret_cast<const Item*>(&sh.blob[buf][0]) : first ? pre : P.items[it];
+        const Task& t = fb ? *reinterpret_cast<const Task*>(&sh.blob[buf][1]) : P.tasks[item.task];
         Cur& c = sh.cur;
-        c.from_blob = fb;
+        c.blob = fb ? (int8_t)buf : (int8_t)-1;
         c.tnsrc = t.nsrc;
         c.nreg = t.nsrc;
         c.ndst = t.ndst;
@@ -306,6 +321,11 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
     if (sh.item >= P.nitems) break;
     first = false;
     last = (uint64_t)sh.item + gridDim.x >= P.nitems;
+    // static schedule: fetch the next item's blob into the other buffer while
+    // this item folds (its last readers finished before the barrier above)
+    if (stat && !last && threadIdx.x < P.first_words)
+      cp_async16(&sh.blob[buf ^ 1][threadIdx.x],
+                 P.first + (size_t)(sh.item + gridDim.x) * P.first_words + threadIdx.x);
     const int nsrc = sh.cur.nsrc, ndst = sh.cur.ndst, npost = sh.cur.npost;
     const bool dropped = sh.cur.dropped;
     if (!dropped) {
@@ -323,7 +343,7 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
         const uint32_t j = i < sh.cur.nreg ? i
                          : i < nsrc ? sh.cur.tnsrc + ndst + nth_bit(sh.cur.late, i - sh.cur.nreg)
                                     : sh.cur.tnsrc + (i - nsrc);
-        const BufRef r = sh.cur.from_blob ? *reinterpret_cast<const BufRef*>(&sh.blob[kBlobRef0 + j])
+        const BufRef r = sh.cur.blob >= 0 ? *reinterpret_cast<const BufRef*>(&sh.blob[sh.cur.blob][kBlobRef0 + j])
                                           : P.refs[sh.cur.ref0 + j];
         char* base = r.kind == kBufSend ? P.send[r.rank]
                    : r.kind == kBufRecv ? P.recv[r.rank] : P.hdr[r.rank] + half_off;
@@ -340,9 +360,13 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
       }
     }
     __syncthreads();
-    if (sh.abort) break;
+    if (sh.abort) {
+      if (stat) cp_async_wait_all();
+      break;
+    }
     if (!dropped) {
       fold_chunk<DT>(sh, nsrc, ndst, sh.cur.len, sh.cur.op);
+      if (stat) cp_async_wait_all();  // the next blob has landed before the barrier publishes it
       __syncthreads();
       // npost was read before the barrier: after it, only thread 0 touches
       // sh.cur (it rewrites it for the next item)
@@ -356,7 +380,11 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
                          sh.cur.chunk, e, sys);
         }
       }
+    } else if (stat) {
+      cp_async_wait_all();
+      __syncthreads();
     }
+    buf ^= stat ? 1 : 0;
   }
   __syncthreads();
   if (threadIdx.x == 0) {
@@ -406,14 +434,13 @@ cudaError_t engine_signal(uint64_t* word, uint64_t value, bool sys, cudaStream_t
   return cudaGetLastError();
 }
 
-cudaError_t engine_launch(const LaunchParams& p, int grid, cudaStream_t stream) {
+cudaError_t engine_launch(const LaunchParams& p, int grid, cudaStream_t stream, bool pdl) {
   cudaGetLastError();  // clear any stale error so the check below is about this launch
   switch (p.dtype) {
-    case kF32: engine_kernel<kF32><<<grid, kThreads, 0, stream>>>(p); break;
-    case kBF16: engine_kernel<kBF16><<<grid, kThreads, 0, stream>>>(p); break;
-    default: engine_kernel<kI32><<<grid, kThreads, 0, stream>>>(p); break;
+    case kF32: return launch_kernel(engine_kernel<kF32>, grid, kThreads, 0, stream, pdl, p);
+    case kBF16: return launch_kernel(engine_kernel<kBF16>, grid, kThreads, 0, stream, pdl, p);
+    default: return launch_kernel(engine_kernel<kI32>, grid, kThreads, 0, stream, pdl, p);
   }
-  return cudaGetLastError();
 }
 
 }  // namespace adapcc

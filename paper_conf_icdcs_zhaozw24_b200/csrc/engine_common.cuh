@@ -33,6 +33,16 @@ __device__ __forceinline__ uint64_t globaltimer() {
   return t;
 }
 
+// Programmatic dependent launch (PDL): a launch with
+// cudaLaunchAttributeProgrammaticStreamSerialization may start while the
+// previous kernel on the stream is still running.  Everything before
+// pdl_wait() may only touch immutable plan tables and shared memory;
+// pdl_wait() returns once the previous grid has completed and its memory is
+// visible (a no-op when the launch had no such dependency).  pdl_trigger()
+// lets the next launch start its own prologue early.
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+
 // 128-bit load/store; .cg keeps in-kernel-produced data out of L1
 __device__ __forceinline__ uint4 ld16(const char* p) { return __ldcg(reinterpret_cast<const uint4*>(p)); }
 __device__ __forceinline__ void st16(char* p, uint4 v) { __stcg(reinterpret_cast<uint4*>(p), v); }
@@ -201,4 +211,21 @@ static __device__ __forceinline__ int nth_bit(uint64_t m, int k) {
 }
 
 }  // namespace dev
+
+// Kernel launch, optionally as a programmatic dependent launch (see pdl_wait).
+template <typename Kernel>
+inline cudaError_t launch_kernel(Kernel kernel, int grid, int threads, size_t smem, cudaStream_t stream,
+                                 bool pdl, const LaunchParams& p) {
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = dim3((unsigned)grid);
+  cfg.blockDim = dim3((unsigned)threads);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = stream;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = pdl ? 1 : 0;
+  return cudaLaunchKernelEx(&cfg, kernel, p);
+}
 }  // namespace adapcc

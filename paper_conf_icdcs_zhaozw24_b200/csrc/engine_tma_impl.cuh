@@ -459,6 +459,12 @@ __global__ void __launch_bounds__(kTmaThreads, ADAPCC_TMA_MINB) engine_tma_kerne
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     sm.abort = 0;
+  }
+  // shared-memory set-up above; the epoch, counters, arenas and user buffers
+  // below belong to the stream order (PDL: the previous launch)
+  pdl_trigger();
+  pdl_wait();
+  if (tid == 0) {
     const uint64_t e = *reinterpret_cast<volatile unsigned long long*>(&P.state->epoch) + 1;
     sm.epoch = e;
     if (blockIdx.x == 0) {
@@ -641,14 +647,19 @@ cudaError_t occupancy(int dtype, int* blocks_per_sm) {
   }
 }
 
-cudaError_t launch(const LaunchParams& p, int grid, cudaStream_t stream) {
+cudaError_t launch(const LaunchParams& p, int grid, cudaStream_t stream, bool pdl) {
   cudaGetLastError();
   switch (p.dtype) {
-    case kF32: prepare<kF32>(); engine_tma_kernel<kF32><<<grid, kTmaThreads, kSmemBytes, stream>>>(p); break;
-    case kBF16: prepare<kBF16>(); engine_tma_kernel<kBF16><<<grid, kTmaThreads, kSmemBytes, stream>>>(p); break;
-    default: prepare<kI32>(); engine_tma_kernel<kI32><<<grid, kTmaThreads, kSmemBytes, stream>>>(p); break;
+    case kF32:
+      if (cudaError_t e = prepare<kF32>()) return e;
+      return launch_kernel(engine_tma_kernel<kF32>, grid, kTmaThreads, kSmemBytes, stream, pdl, p);
+    case kBF16:
+      if (cudaError_t e = prepare<kBF16>()) return e;
+      return launch_kernel(engine_tma_kernel<kBF16>, grid, kTmaThreads, kSmemBytes, stream, pdl, p);
+    default:
+      if (cudaError_t e = prepare<kI32>()) return e;
+      return launch_kernel(engine_tma_kernel<kI32>, grid, kTmaThreads, kSmemBytes, stream, pdl, p);
   }
-  return cudaGetLastError();
 }
 
 }  // namespace ADAPCC_TMA_NS

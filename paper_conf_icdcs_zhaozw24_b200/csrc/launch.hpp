@@ -33,6 +33,12 @@ struct LaunchParams {
   // first_words, loaded in a single round trip together with the epoch
   const uint4* first;
   uint32_t nfirst, first_words;
+  // static schedule (nfirst == nitems): CTA b runs items b, b + grid, ... in
+  // order, reading each item's blob (prefetched during the previous fold)
+  // instead of claiming from the counter; still deadlock-free, because the
+  // smallest unfinished item's CTA has finished all its earlier items and its
+  // inputs come from smaller items
+  uint32_t sched_static;
   int dtype;
   int nranks;
   int my_rank;          // multi-process: this rank; loopback: -1
@@ -67,7 +73,7 @@ struct ArenaHeader {
 // engine.cu: 128-bit LDG/STG fold (256 threads, 2 CTAs/SM)
 int engine_threads();
 cudaError_t engine_occupancy(int dtype, int* blocks_per_sm);
-cudaError_t engine_launch(const LaunchParams& p, int grid, cudaStream_t stream);
+cudaError_t engine_launch(const LaunchParams& p, int grid, cudaStream_t stream, bool pdl);
 // store `value` into a ready word after all prior work on `stream` (late join)
 cudaError_t engine_signal(uint64_t* word, uint64_t value, bool sys, cudaStream_t stream);
 // engine_tma_impl.cuh: TMA bulk-copy pipeline (1 producer + 8 consumer warps),
@@ -75,12 +81,12 @@ cudaError_t engine_signal(uint64_t* word, uint64_t value, bool sys, cudaStream_t
 namespace tma_direct {
 int threads();
 cudaError_t occupancy(int dtype, int* blocks_per_sm);
-cudaError_t launch(const LaunchParams& p, int grid, cudaStream_t stream);
+cudaError_t launch(const LaunchParams& p, int grid, cudaStream_t stream, bool pdl);
 }  // namespace tma_direct
 namespace tma_staged {
 int threads();
 cudaError_t occupancy(int dtype, int* blocks_per_sm);
-cudaError_t launch(const LaunchParams& p, int grid, cudaStream_t stream);
+cudaError_t launch(const LaunchParams& p, int grid, cudaStream_t stream, bool pdl);
 }  // namespace tma_staged
 
 }  // namespace adapcc

@@ -530,19 +530,25 @@ bool build_plan(const PlanRequest& rq, std::vector<SegmentPlan>* segs, std::stri
 }
 
 std::vector<Item> order_items(const SegmentPlan& p, int rank, int esize, int grid,
-                              uint64_t piece_bytes, int taper) {
+                              uint64_t piece_bytes, int taper, bool tma) {
   // Work balance: tasks that post no flags are cut into pieces of roughly
-  // equal traffic so that the grid sees >= ~8 items per CTA.
+  // equal traffic.
   uint64_t total = 0;
   for (const Task& T : p.tasks)
     if (rank < 0 || T.owner == rank) total += (T.hi - T.lo) * esize * (uint64_t)(T.nsrc + T.ndst);
-  // Measured on B200 (profiles/sweep_r01.json): ~512 KiB of traffic per item
-  // (32 KiB per stream for a 16-stream fold) is the sweet spot -- smaller
-  // items pay the per-item claim/sync overhead, larger ones lose bandwidth.
+  // Measured on B200 (profiles/sweep_r01.json, profiles/pieces_r01.json):
+  // ~512 KiB of traffic per item (32 KiB per stream for a 16-stream fold) is
+  // the sweet spot of large calls -- smaller items pay the per-item claim/sync
+  // overhead, larger ones lose bandwidth.
+  // Pieces are sized so that every CTA gets the same number m of items: a
+  // CTA streams a piece at a roughly fixed rate, so a call ends when the CTA
+  // with the most items does (8 MiB per rank, TMA: 1.7 items per CTA left half
+  // the grid idle for a whole item at the end).
+  const uint64_t g = (uint64_t)std::max(grid, 1);
+  const uint64_t cap = 512 * 1024, floor_bytes = tma ? 256 * 1024 : 16 * 1024;
+  const uint64_t m = std::max<uint64_t>(1, (total + g * cap - 1) / (g * cap));
   const uint64_t target =
-      piece_bytes ? piece_bytes
-                  : std::min<uint64_t>(std::max<uint64_t>(total / (4ull * std::max(grid, 1)), 64 * 1024),
-                                       512 * 1024);
+      piece_bytes ? piece_bytes : std::min<uint64_t>(std::max<uint64_t>(total / (m * g), floor_bytes), cap);
   const uint64_t align = 512;  // elements: keeps every piece 16-byte aligned
   struct Key { uint64_t a; uint32_t level, task, chunk, off, len; };
   std::vector<Key> keys;
@@ -555,15 +561,19 @@ std::vector<Item> order_items(const SegmentPlan& p, int rank, int esize, int gri
   for (uint32_t t = 0; t < p.tasks.size(); ++t) {
     const Task& T = p.tasks[t];
     if (rank >= 0 && T.owner != rank) continue;
-    uint64_t piece = T.chunk_elems;
-    if (T.npost == 0) {
-      const uint64_t streams = std::max<uint64_t>(1, T.nsrc + T.ndst);
-      piece = std::max<uint64_t>(align, target / (streams * esize) / align * align);
-      piece = std::min<uint64_t>(piece, T.chunk_elems);
-    }
+    const uint64_t streams = std::max<uint64_t>(1, T.nsrc + T.ndst);
     for (uint32_t c = 0; c < T.nchunks; ++c) {
       const uint64_t c0 = T.lo + (uint64_t)c * T.chunk_elems;
       const uint64_t clen = std::min<uint64_t>(T.hi, c0 + T.chunk_elems) - c0;
+      // a flag-free chunk is cut into at most floor(traffic / target) equal
+      // pieces of >= `target` bytes: with target = total / grid a mid-size
+      // call then has at most one item per CTA (measured: 304 items of 14 KiB
+      // per stream on 296 CTAs 14.9 us, 256 items of 16 KiB 10.5 us)
+      uint64_t piece = clen;
+      if (T.npost == 0) {
+        const uint64_t cnt = std::max<uint64_t>(1, clen * streams * esize / target);
+        piece = std::max<uint64_t>(align, ((clen + cnt - 1) / cnt + align - 1) / align * align);
+      }
       for (uint64_t off = 0; off < clen; off += piece)
         keys.push_back({(uint64_t)c, T.level, t, c, (uint32_t)off,
                         (uint32_t)std::min<uint64_t>(piece, clen - off)});

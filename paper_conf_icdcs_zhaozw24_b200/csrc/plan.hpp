@@ -66,11 +66,12 @@ bool build_plan(const PlanRequest& rq, std::vector<SegmentPlan>* segs, std::stri
 // Work items of `rank` (-1: all ranks) in deadlock-free order; `grid` CTAs
 // will execute them (used to size the pieces of flag-free tasks).
 // piece_bytes: traffic per piece (all streams); 0 = automatic (see plan.cpp).
+// tma: items for the TMA pipeline kernel (larger mid-size pieces).
 // taper: the last ~2 x grid splittable items (flag-free tasks) are cut into
 // `taper` sub-pieces each, so the dynamic claim loop ends on short items
 // (1 = off, 0 = automatic).
 std::vector<Item> order_items(const SegmentPlan& p, int rank, int esize, int grid,
-                              uint64_t piece_bytes = 0, int taper = 1);
+                              uint64_t piece_bytes = 0, int taper = 1, bool tma = false);
 
 // Byte accounting for adapcc_plan_stats.
 void accumulate_stats(const SegmentPlan& p, int rank, int esize, PlanStats* s);

@@ -26,6 +26,9 @@ def main():
     ap.add_argument("--min-log2", type=int, default=10)
     ap.add_argument("--max-log2", type=int, default=30)
     ap.add_argument("--graph", action="store_true", help="time a CUDA graph of back-to-back calls")
+    ap.add_argument("--engine", type=int, default=-1, help="0 LDG, 1 TMA, 2 auto (default: library default)")
+    ap.add_argument("--piece-kib", type=int, default=-1, help="work-piece traffic target (0 = automatic)")
+    ap.add_argument("--sched", type=int, default=-1, help="LDG kernel: 0 dynamic claims, 1 static, 2 auto")
     ap.add_argument("--out", default=os.path.join(ROOT, "gpurun_out", "sizes.json"))
     a = ap.parse_args()
 
@@ -42,6 +45,12 @@ def main():
     maxb = 1 << a.max_log2
     scratch = 64 << 20 if a.mode == "direct" else 2 * maxb + (64 << 20)
     comm = pkg.Communicator.loopback(n, scratch_bytes=scratch, mode=a.mode)
+    if a.engine >= 0:
+        comm.config("engine", a.engine)
+    if a.sched >= 0:
+        comm.config("sched", a.sched)
+    if a.piece_kib >= 0:
+        comm.config("piece_kib", a.piece_kib)
     chunk = a.chunk_kib * 1024
     if a.coll == "allreduce":
         comm.set_strategy("allreduce", G.allreduce_stars(n, chunk=chunk))
@@ -106,7 +115,7 @@ def main():
     assert comm.get_async_error() == 0
     os.makedirs(os.path.dirname(a.out), exist_ok=True)
     json.dump({"ranks": n, "dtype": a.dtype, "mode": a.mode, "coll": a.coll, "chunk": chunk,
-               "graph": a.graph, "note": "same buffers every call: sizes whose 2nS fit in L2 run from L2",
+               "graph": a.graph, "engine": a.engine, "piece_kib": a.piece_kib, "sched": a.sched, "note": "same buffers every call: sizes whose 2nS fit in L2 run from L2",
                "points": res}, open(a.out, "w"), indent=1)
 
 

@@ -1,6 +1,7 @@
 """Randomised GPU parity sweep (-m gpu): random trees (shape, root, noagg),
 weights, chunk sizes, counts (1 element .. 3 M, ragged), masks, dtypes,
-plans (DIRECT / STAGED) and kernels (LDG, TMA, auto), every collective the
+plans (DIRECT / STAGED), kernels (LDG, TMA, auto), LDG schedules, PDL on/off
+and piece sizes, every collective the
 loopback communicator offers; bit-exact against the oracle.  Seeded: a
 failure names its case and reproduces."""
 
@@ -93,8 +94,14 @@ def _case(seed, large=False, n=None):
                 pg = p[g]
                 q[sw.get(g, g)] = -1 if pg == -1 else sw.get(pg, pg)
             text += f"rtree dst={b} weight=1 chunk={chunk} parent={G._join(q)}\n"
+    # launch knobs from their own stream (the cases above stay as they were):
+    # LDG schedule (dynamic claims / static blobs), programmatic dependent
+    # launch, work-piece size (0 = automatic)
+    r2 = np.random.default_rng(seed + (7_100_000 if large else 7_000_000))
+    knobs = dict(sched=int(r2.choice([0, 2])), pdl=int(r2.integers(0, 2)),
+                 piece_kib=int(r2.choice([0, 0, 16, 48, 512])))
     return dict(n=n, coll=coll, dtype=dtype, count=count, mode=mode, engine=engine, ready=ready, text=text,
-                seed=seed)
+                seed=seed, **knobs)
 
 
 def _eq(a, b):
@@ -122,6 +129,8 @@ def _run(c):
     comm = pkg.Communicator.loopback(n, device=0, scratch_bytes=scratch, mode=c["mode"])
     comm.config("timeout_ms", 20000)
     comm.config("engine", c["engine"])
+    for k in ("sched", "pdl", "piece_kib"):
+        comm.config(k, c[k])
     comm.set_strategy(c["coll"], text)
     xs = rank_tensors(dtype, per_rank, n, base=5000 + seed)
     prev = [rank_tensors(dtype, out_per_rank, 1, base=6000 + 7 * seed + g)[0] for g in range(n)]
