@@ -1,7 +1,4 @@
+python scripts/debug/ab_configs.py --coll allreduce --sizes 10,16,20,21,22,23,24,25 --reps 5 --configs 'engine=2;engine=1;engine=0' 2>&1 | tail -8
+python scripts/debug/ab_configs.py --coll alltoall --sizes 10,20,22,23,24 --reps 5 --configs 'engine=2' 2>&1 | tail -5
+for s in 1048576 4194304; do python scripts/trace_report.py --bytes-per-rank $s --out gpurun_out/tr/b_ar_$s > /dev/null 2>gpurun_out/tr/err_$s.log; done
 timeout 1500 python -m pytest tests -m gpu -x -q -p no:cacheprovider > gpurun_out/t_all.log 2>&1; tail -2 gpurun_out/t_all.log
-timeout 300 python bench.py > gpurun_out/bench2.json 2> gpurun_out/bench2.err
-python scripts/sweep_sizes.py --graph --out gpurun_out/sizes_ar_r01b.json > /dev/null 2>>gpurun_out/st_err.log
-python scripts/sweep_sizes.py --graph --coll alltoall --out gpurun_out/sizes_a2a_r01b.json > /dev/null 2>>gpurun_out/st_err.log
-python scripts/sweep_sizes.py --graph --coll allgather --out gpurun_out/sizes_ag_r01b.json > /dev/null 2>>gpurun_out/st_err.log
-python scripts/sweep_sizes.py --graph --dtype bf16 --out gpurun_out/sizes_ar_bf16_r01b.json > /dev/null 2>>gpurun_out/st_err.log
-python scripts/debug/launch_floor.py > gpurun_out/floor3.json 2>&1

@@ -306,6 +306,22 @@ ADAPCC_API const char* adapcc_last_cuda_error(void);
  * plan cache (plans a captured CUDA graph uses stay alive); results never depend on them. */
 ADAPCC_API adapcc_result_t adapcc_config(adapcc_comm_t comm, const char* key, int64_t value);
 
+/* In-kernel trace (debug / tuning; SURVEY §5 tracing).  Enable with adapcc_config(comm, "trace",
+ * capacity) -- capacity = records kept (0 = off, the default; changing it drains the device and
+ * drops the old buffer).  While on, every engine launch appends one 48-byte record per work item
+ * it executes and one per CTA, with %globaltimer times in ns:
+ *   struct { uint32_t launch, cta, item, task; uint64_t t0, t1, t2, bytes; }
+ *   item record (item != 0xFFFFFFFF): t0 claimed, t1 inputs ready (flags acquired), t2 done
+ *     (stores issued, flags posted); bytes = traffic of the item over all its streams;
+ *   CTA record (item == 0xFFFFFFFF): t0 entry, t1 after the stream-order wait and epoch read,
+ *     t2 exit.
+ * Records beyond the capacity are dropped.  adapcc_trace_read drains the device, copies up to
+ * max_records records to host memory `records`, reports how many were copied and how many were
+ * written in total (n_total > capacity: some were dropped), and empties the buffer.  Returns
+ * ADAPCC_ERR_UNSUPPORTED while tracing is off.  Tracing adds one atomic per record. */
+ADAPCC_API adapcc_result_t adapcc_trace_read(adapcc_comm_t comm, void* records, uint32_t max_records,
+                                             uint32_t* n_copied, uint32_t* n_total);
+
 /* Number of engine kernel launches this communicator has issued. */
 ADAPCC_API adapcc_result_t adapcc_launch_count(adapcc_comm_t comm, uint64_t* count);
 /* Kernel of the most recent launch: 0 = LDG/STG fold, 1 = TMA pipeline, -1 = none. */

@@ -96,6 +96,8 @@ def _load():
         "adapcc_config": [vp, ctypes.c_char_p, i64],
         "adapcc_launch_count": [vp, ctypes.POINTER(u64)],
         "adapcc_last_engine": [vp, ctypes.POINTER(i32)],
+        "adapcc_trace_read": [vp, vp, ctypes.c_uint32, ctypes.POINTER(ctypes.c_uint32),
+                              ctypes.POINTER(ctypes.c_uint32)],
         "adapcc_exclude": [vp, u64, AG_FN, vp],
         "adapcc_members": [vp, ctypes.POINTER(u64)],
         "adapcc_strategy_check": [ctypes.c_char_p, ctypes.POINTER(i32), ctypes.POINTER(i32),
@@ -371,6 +373,21 @@ class Communicator:
         v = ctypes.c_uint64()
         _check(_load().adapcc_launch_count(self._h, ctypes.byref(v)), "launch_count")
         return v.value
+
+    def trace(self, max_records=1 << 20):
+        """Drain the in-kernel trace (enable with config("trace", capacity)).
+
+        Returns (records, n_total): a numpy structured array with fields
+        launch, cta, item, task, t0, t1, t2, bytes (include/adapcc.h,
+        adapcc_trace_read) and the number of records the kernels wrote."""
+        import numpy as np
+        dt = np.dtype([("launch", "<u4"), ("cta", "<u4"), ("item", "<u4"), ("task", "<u4"),
+                       ("t0", "<u8"), ("t1", "<u8"), ("t2", "<u8"), ("bytes", "<u8")])
+        buf = np.zeros(max_records, dtype=dt)
+        n, tot = ctypes.c_uint32(), ctypes.c_uint32()
+        _check(_load().adapcc_trace_read(self._h, buf.ctypes.data, max_records, ctypes.byref(n),
+                                         ctypes.byref(tot)), "trace_read")
+        return buf[:n.value].copy(), tot.value
 
     def last_engine(self):
         """Kernel of the most recent launch: 0 LDG/STG fold, 1 TMA pipeline."""

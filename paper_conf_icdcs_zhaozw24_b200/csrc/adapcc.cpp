@@ -161,6 +161,9 @@ struct adapcc_comm_s {
   int64_t taper = 0;      // tail items cut into this many sub-pieces (1 = off, 0 = auto)
   int64_t check_sig = 0;  // debug: kernels compare call signatures across ranks (ADAPCC_DEBUG)
   int64_t first_blob = 1; // LDG kernel: per-CTA first-item blobs (ADAPCC_FIRST_BLOB=0 disables)
+  TraceRec* trace = nullptr;  // in-kernel trace buffer (adapcc_config("trace", capacity))
+  unsigned* trace_n = nullptr;
+  uint32_t trace_cap = 0;
   int64_t pdl = 1;        // programmatic dependent launch of the engine kernels (ADAPCC_PDL)
   int64_t sched = 2;      // LDG kernel: 0 dynamic claims, 1 static blob schedule, 2 auto (ADAPCC_SCHED)
   uint64_t launches = 0;
@@ -250,6 +253,8 @@ void release(adapcc_comm_s* c) {
     }
   }
   cudaFree(c->state);
+  cudaFree(c->trace);
+  cudaFree(c->trace_n);
   cudaFreeHost(c->h_err);
   delete c;
 }
@@ -397,7 +402,7 @@ adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, const Strategy* strat, uin
     CK(up(&d.refs, sp.refs));
     CK(up(&d.flags, sp.flags));
     CK(up(&d.items, items));
-    if (plan->kernel == 0 && c->first_blob) {
+    if (c->first_blob) {
       // Item blobs (launch.hpp): item i, its task and the task's refs in one
       // run of 16-byte words.  Static schedule: every item gets one, CTA b runs
       // items b, b + grid, ... and prefetches the next blob while it folds (no
@@ -409,9 +414,9 @@ adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, const Strategy* strat, uin
       };
       uint32_t all_words = 0;
       for (uint32_t i = 0; i < d.nitems; ++i) all_words = std::max(all_words, words_of(i));
-      const bool stat = c->sched != 0 && d.nitems > 0 && all_words <= (uint32_t)kFirstMaxWords &&
+      const bool stat = plan->kernel == 0 && c->sched != 0 && d.nitems > 0 && all_words <= (uint32_t)kFirstMaxWords &&
                         (uint64_t)d.nitems * all_words * 16 <= kMaxBlobBytes;
-      const uint32_t nf = stat ? d.nitems : std::min<uint32_t>(d.nitems, (uint32_t)grid_size(c, dtype, 0));
+      const uint32_t nf = stat ? d.nitems : std::min<uint32_t>(d.nitems, (uint32_t)grid_size(c, dtype, plan->kernel));
       uint32_t words = 0;
       for (uint32_t b = 0; b < nf; ++b) words = std::max(words, words_of(b));
       if (nf > 0 && words <= (uint32_t)kFirstMaxWords) {
@@ -511,6 +516,10 @@ adapcc_result_t run(adapcc_comm_s* c, Coll coll, const void* const* send, void* 
     P.sig = fnv(fnv(plan->sig, si), sig_extra);
     P.state = c->state;
     P.err = c->d_err;
+    P.trace = c->trace;
+    P.trace_n = c->trace_n;
+    P.trace_cap = c->trace_cap;
+    P.launch_seq = (uint32_t)c->launches;
     for (int q = 0; q < c->nranks; ++q) {
       if (zc) {
         P.send[q] = zc_send[q];
@@ -1157,6 +1166,28 @@ adapcc_result_t adapcc_config(adapcc_comm_t c, const char* key, int64_t value) {
   }
   else if (!std::strcmp(key, "debug_check")) c->check_sig = value != 0;
   else if (!std::strcmp(key, "pdl")) c->pdl = value != 0;
+  else if (!std::strcmp(key, "trace")) {  // capacity in records; 0 = off
+    if (value < 0 || value > (int64_t(1) << 26)) return ADAPCC_ERR_INVALID_ARGUMENT;
+    if (cudaSetDevice(c->device) != cudaSuccess || cudaDeviceSynchronize() != cudaSuccess) return ADAPCC_ERR_CUDA;
+    cudaFree(c->trace);
+    cudaFree(c->trace_n);
+    c->trace = nullptr;
+    c->trace_n = nullptr;
+    c->trace_cap = 0;
+    if (value > 0) {
+      if (cudaMalloc(&c->trace, (size_t)value * sizeof(TraceRec)) != cudaSuccess ||
+          cudaMalloc(&c->trace_n, sizeof(unsigned)) != cudaSuccess ||
+          cudaMemset(c->trace_n, 0, sizeof(unsigned)) != cudaSuccess) {
+        cudaGetLastError();
+        cudaFree(c->trace);
+        cudaFree(c->trace_n);
+        c->trace = nullptr;
+        c->trace_n = nullptr;
+        return ADAPCC_ERR_OOM;
+      }
+      c->trace_cap = (uint32_t)value;
+    }
+  }
   else if (!std::strcmp(key, "sched")) {
     if (value < 0 || value > 2) return ADAPCC_ERR_INVALID_ARGUMENT;
     c->sched = value;
@@ -1170,6 +1201,25 @@ adapcc_result_t adapcc_config(adapcc_comm_t c, const char* key, int64_t value) {
     if (!c->loopback || value < -1 || value >= c->nranks) return ADAPCC_ERR_INVALID_ARGUMENT;
     c->drop_rank = value;
   } else return ADAPCC_ERR_INVALID_ARGUMENT;
+  return ADAPCC_SUCCESS;
+}
+
+adapcc_result_t adapcc_trace_read(adapcc_comm_t c, void* records, uint32_t max_records, uint32_t* n_copied,
+                                  uint32_t* n_total) {
+  if (!c || !n_copied || (max_records && !records)) return ADAPCC_ERR_INVALID_ARGUMENT;
+  std::lock_guard<std::mutex> lock(c->mu);
+  *n_copied = 0;
+  if (n_total) *n_total = 0;
+  if (!c->trace) return ADAPCC_ERR_UNSUPPORTED;
+  CK(cudaSetDevice(c->device));
+  CK(cudaDeviceSynchronize());
+  unsigned n = 0;
+  CK(cudaMemcpy(&n, c->trace_n, sizeof(n), cudaMemcpyDeviceToHost));
+  const uint32_t have = std::min<uint32_t>(n, c->trace_cap), k = std::min<uint32_t>(have, max_records);
+  if (k) CK(cudaMemcpy(records, c->trace, (size_t)k * sizeof(TraceRec), cudaMemcpyDeviceToHost));
+  CK(cudaMemset(c->trace_n, 0, sizeof(unsigned)));
+  *n_copied = k;
+  if (n_total) *n_total = n;
   return ADAPCC_SUCCESS;
 }
 

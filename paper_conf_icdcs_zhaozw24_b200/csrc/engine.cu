@@ -55,6 +55,8 @@ struct Cur {  // header of the work item being executed (staged by thread 0)
 };
 
 struct Shared {
+  uint64_t tr0, tr1;           // trace: item claimed / inputs ready
+  char* base[3][kMaxRanksDev];  // P.send / P.recv / P.hdr (indexed by BufKind), copied from the params
   uint4 blob[2][kFirstMaxWords];  // item blobs: Item | Task | refs (static schedule: double-buffered)
   Cur cur;
   const char* src[kMaxFold];
@@ -218,6 +220,7 @@ template <int DT>
 __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __grid_constant__ LaunchParams P) {
   __shared__ Shared sh;
   const bool sys = P.ipc;
+  const uint64_t t_entry = P.trace ? globaltimer() : 0;
   Item pre{};  // thread 0: this CTA's first item, loaded together with the epoch
   // first item, its task and refs in one round trip (plan-time blob)
   const bool use_blob = blockIdx.x < P.nfirst;
@@ -225,6 +228,13 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
     sh.blob[0][threadIdx.x] = P.first[(size_t)blockIdx.x * P.first_words + threadIdx.x];
   const bool stat = P.sched_static != 0;
   int buf = 0;  // blob buffer of the current item (static schedule)
+  // buffer bases into shared memory: dynamically indexed kernel parameters
+  // are constant-bank loads that miss on a cold launch (~1 us measured with
+  // the in-kernel trace); done before the stream-order wait
+  for (int i = threadIdx.x; i < 3 * P.nranks; i += kThreads) {
+    const int k = i / P.nranks, q = i - k * P.nranks;
+    sh.base[k][q] = k == 0 ? P.send[q] : k == 1 ? P.recv[q] : P.hdr[q];
+  }
   if (threadIdx.x == 0 && !use_blob && blockIdx.x < P.nitems) pre = P.items[blockIdx.x];
   // the plan tables above are immutable; the epoch, counters, arenas and user
   // buffers below belong to the stream order (PDL: the previous launch)
@@ -241,6 +251,7 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
     }
   }
   __syncthreads();
+  const uint64_t t_ready = P.trace ? globaltimer() : 0;
   const uint64_t epoch = sh.epoch;
   const unsigned par = (unsigned)(epoch & 1);
   const uint64_t half_off = kArenaHeader + par * P.half_bytes;
@@ -275,6 +286,7 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
       const uint32_t it = first ? blockIdx.x : stat ? sh.item + gridDim.x
                                                     : gridDim.x + atomicAdd(&P.state->work[par], 1u);
       sh.item = it;
+      if (P.trace) sh.tr0 = globaltimer();
       sh.bad_align = 0;
       sh.any_acc = 0;
       if (it < P.nitems) {
@@ -333,7 +345,7 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
       if (threadIdx.x < sh.cur.nwait) {
         const FlagRef f = P.flags[sh.cur.flag0 + threadIdx.x];
         const uint64_t* fl =
-            reinterpret_cast<const uint64_t*>(P.hdr[f.rank] + half_off + f.off) + sh.cur.chunk;
+            reinterpret_cast<const uint64_t*>(sh.base[kBufArena][f.rank] + half_off + f.off) + sh.cur.chunk;
         if (!wait_flag(fl, epoch, P)) sh.abort = 1;
       }
       // resolve stream pointers for this piece
@@ -345,8 +357,7 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
                                     : sh.cur.tnsrc + (i - nsrc);
         const BufRef r = sh.cur.blob >= 0 ? *reinterpret_cast<const BufRef*>(&sh.blob[sh.cur.blob][kBlobRef0 + j])
                                           : P.refs[sh.cur.ref0 + j];
-        char* base = r.kind == kBufSend ? P.send[r.rank]
-                   : r.kind == kBufRecv ? P.recv[r.rank] : P.hdr[r.rank] + half_off;
+        char* base = sh.base[r.kind][r.rank] + (r.kind == kBufArena ? half_off : 0);
         char* p = base + r.bias + (int64_t)(sh.cur.e0 * esize);
         if (reinterpret_cast<uintptr_t>(p) & 15) atomicOr(&sh.bad_align, 1);
         if (threadIdx.x < nsrc) {
@@ -360,6 +371,7 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
       }
     }
     __syncthreads();
+    if (P.trace && threadIdx.x == 0) sh.tr1 = globaltimer();
     if (sh.abort) {
       if (stat) cp_async_wait_all();
       break;
@@ -380,6 +392,9 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
                          sh.cur.chunk, e, sys);
         }
       }
+      if (P.trace && threadIdx.x == 0)
+        trace_put(P, sh.item, 0, sh.tr0, sh.tr1, globaltimer(),
+                  (uint64_t)sh.cur.len * esize * (uint64_t)(sh.cur.nsrc + sh.cur.ndst));
     } else if (stat) {
       cp_async_wait_all();
       __syncthreads();
@@ -387,6 +402,7 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
     buf ^= stat ? 1 : 0;
   }
   __syncthreads();
+  if (P.trace && threadIdx.x == 0) trace_put(P, kTraceCta, 0, t_entry, t_ready, globaltimer(), 0);
   if (threadIdx.x == 0) {
     // across processes the done word published to peers must follow every
     // CTA's data; in loopback only the next launch reads anything, after

@@ -43,6 +43,13 @@ __device__ __forceinline__ uint64_t globaltimer() {
 __device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
 __device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
 
+// appends one trace record (tracing is a debug mode: one atomic per record)
+__device__ __forceinline__ void trace_put(const LaunchParams& P, uint32_t item, uint32_t task, uint64_t t0,
+                                          uint64_t t1, uint64_t t2, uint64_t bytes) {
+  const unsigned i = atomicAdd(P.trace_n, 1u);
+  if (i < P.trace_cap) P.trace[i] = TraceRec{P.launch_seq, blockIdx.x, item, task, t0, t1, t2, bytes};
+}
+
 // 128-bit load/store; .cg keeps in-kernel-produced data out of L1
 __device__ __forceinline__ uint4 ld16(const char* p) { return __ldcg(reinterpret_cast<const uint4*>(p)); }
 __device__ __forceinline__ void st16(char* p, uint4 v) { __stcg(reinterpret_cast<uint4*>(p), v); }

@@ -65,6 +65,8 @@ struct ItemDesc {
   uint16_t nsrc, ndst, op, npost, passes, ks;
   uint8_t acc[kMaxDst];
   uint8_t stop, dropped, scalar_only, any_acc;
+  uint32_t item;        // trace: item index, claim and inputs-ready times
+  uint64_t tr0, tr1;
 };
 
 struct Smem {
@@ -76,6 +78,8 @@ struct Smem {
   int abort;
   int pad;
   ItemDesc q[kQ];
+  uint4 blob[kFirstMaxWords];  // this CTA's first item: Item | Task | refs (plan-time blob)
+  char* base[3][kMaxRanksDev];  // P.send / P.recv / P.hdr (indexed by BufKind), copied from the params
 };
 
 constexpr size_t kSmemHeader = (sizeof(Smem) + 127) / 128 * 128;
@@ -368,9 +372,11 @@ __device__ __forceinline__ void consume_fold(Smem& sm, char* stages, const ItemD
 
 // ------------------------------------------------------------- producer
 template <int DT>
-__device__ __forceinline__ void fill_desc(const LaunchParams& P, ItemDesc& d, const Item& item,
-                                          const Task& t, uint64_t half_off, int lane, uint32_t it,
-                                          int* nwait_eff) {
+// R: the task's refs (R[0] = refs[t.ref0]), in global memory or in the
+// CTA's first-item blob
+__device__ __forceinline__ void fill_desc(const LaunchParams& P, char* const (*base)[kMaxRanksDev],
+                                          ItemDesc& d, const Item& item, const Task& t, const BufRef* R,
+                                          uint64_t half_off, int lane, uint32_t it, int* nwait_eff) {
   constexpr int esize = Ops<DT>::kEsize;
   const uint64_t e0 = t.lo + (uint64_t)item.chunk * t.chunk_elems + item.off;
   // late join (phase 1) / complement (phase 2): which candidate ranks are folded
@@ -398,12 +404,10 @@ __device__ __forceinline__ void fill_desc(const LaunchParams& P, ItemDesc& d, co
   const int nsrc = nreg + __popcll(late);
   int misaligned = 0;
   for (int i = lane; i < nsrc + t.ndst; i += 32) {
-    const BufRef r = i < nreg ? P.refs[t.ref0 + i]
-                   : i < nsrc ? P.refs[t.ref0 + t.nsrc + t.ndst + nth_bit(late, i - nreg)]
-                              : P.refs[t.ref0 + t.nsrc + (i - nsrc)];
-    char* base = r.kind == kBufSend ? P.send[r.rank] : r.kind == kBufRecv ? P.recv[r.rank]
-                                                                         : P.hdr[r.rank] + half_off;
-    char* p = base + r.bias + (int64_t)(e0 * esize);
+    const BufRef r = i < nreg ? R[i]
+                   : i < nsrc ? R[t.nsrc + t.ndst + nth_bit(late, i - nreg)]
+                              : R[t.nsrc + (i - nsrc)];
+    char* p = base[r.kind][r.rank] + (r.kind == kBufArena ? half_off : 0) + r.bias + (int64_t)(e0 * esize);
     misaligned |= (reinterpret_cast<uintptr_t>(p) & 15) != 0;
     if (i < nsrc) {
       d.src[i] = p;
@@ -414,7 +418,7 @@ __device__ __forceinline__ void fill_desc(const LaunchParams& P, ItemDesc& d, co
   }
   for (int i = lane; i < t.npost; i += 32) {
     const FlagRef f = P.flags[t.flag0 + t.nwait + i];
-    d.post[i] = reinterpret_cast<uint64_t*>(P.hdr[f.rank] + half_off + f.off) + item.chunk;
+    d.post[i] = reinterpret_cast<uint64_t*>(base[kBufArena][f.rank] + half_off + f.off) + item.chunk;
   }
   misaligned = __any_sync(0xffffffffu, misaligned);
   __syncwarp();
@@ -448,6 +452,7 @@ __global__ void __launch_bounds__(kTmaThreads, ADAPCC_TMA_MINB) engine_tma_kerne
   const int tid = threadIdx.x;
   const int warp = tid >> 5, lane = tid & 31;
   const bool sys = P.ipc;
+  const uint64_t t_entry = P.trace ? globaltimer() : 0;
   if (tid == 0) {
     for (int s = 0; s < kStages; ++s) {
       mbar_init(&sm.full[s], 1);
@@ -459,6 +464,21 @@ __global__ void __launch_bounds__(kTmaThreads, ADAPCC_TMA_MINB) engine_tma_kerne
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     sm.abort = 0;
+  }
+  // the producer's first item, its task and refs: one round trip of
+  // immutable plan data, issued before the stream-order wait below
+  const bool use_blob = blockIdx.x < P.nfirst;
+  if (warp == kConsumerWarps) {
+    if (use_blob)
+      for (uint32_t i = lane; i < P.first_words; i += 32)
+        sm.blob[i] = P.first[(size_t)blockIdx.x * P.first_words + i];
+    // buffer bases into shared memory (dynamically indexed parameters are
+    // constant-bank loads that miss on a cold launch)
+    for (int i = lane; i < 3 * P.nranks; i += 32) {
+      const int k = i / P.nranks, q = i - k * P.nranks;
+      sm.base[k][q] = k == 0 ? P.send[q] : k == 1 ? P.recv[q] : P.hdr[q];
+    }
+    __syncwarp();
   }
   // shared-memory set-up above; the epoch, counters, arenas and user buffers
   // below belong to the stream order (PDL: the previous launch)
@@ -473,6 +493,7 @@ __global__ void __launch_bounds__(kTmaThreads, ADAPCC_TMA_MINB) engine_tma_kerne
     }
   }
   __syncthreads();
+  const uint64_t t_ready = P.trace ? globaltimer() : 0;
   const uint64_t epoch = sm.epoch;
   const unsigned par = (unsigned)(epoch & 1);
   const uint64_t half_off = kArenaHeader + par * P.half_bytes;
@@ -500,6 +521,7 @@ __global__ void __launch_bounds__(kTmaThreads, ADAPCC_TMA_MINB) engine_tma_kerne
       uint32_t it = 0;
       int stop_i = 0;
       if (lane == 0 && !last) it = first ? blockIdx.x : gridDim.x + atomicAdd(&P.state->work[par], 1u);
+      const uint64_t tr0 = P.trace ? globaltimer() : 0;
       // queue slot free: every lane waits (acquire), since every lane rewrites
       // the slot's descriptor that the consumers of item i - kQ were reading
       mbar_wait(&sm.qempty[qi], qphase ^ 1);
@@ -511,17 +533,19 @@ __global__ void __launch_bounds__(kTmaThreads, ADAPCC_TMA_MINB) engine_tma_kerne
       it = __shfl_sync(0xffffffffu, it, 0);
       bool stop = __shfl_sync(0xffffffffu, stop_i, 0) != 0;
       ItemDesc& d = sm.q[qi];
-      const Item item = stop ? Item{} : P.items[it];
-      const Task& t = P.tasks[item.task];
+      const bool fb = use_blob && it == blockIdx.x;  // this CTA's first item (blob in shared memory)
+      const Item item = stop ? Item{} : fb ? *reinterpret_cast<const Item*>(&sm.blob[0]) : P.items[it];
+      const Task& t = fb ? *reinterpret_cast<const Task*>(&sm.blob[1]) : P.tasks[item.task];
       if (!stop) {
         int nwait = 0;
-        fill_desc<DT>(P, d, item, t, half_off, lane, it, &nwait);
+        const BufRef* R = fb ? reinterpret_cast<const BufRef*>(&sm.blob[kBlobRef0]) : P.refs + t.ref0;
+        fill_desc<DT>(P, sm.base, d, item, t, R, half_off, lane, it, &nwait);
         __syncwarp();
         if (!d.dropped) {
           int ok = 1;
           for (int i = lane; i < nwait; i += 32) {
             const FlagRef f = P.flags[t.flag0 + i];
-            const uint64_t* fl = reinterpret_cast<const uint64_t*>(P.hdr[f.rank] + half_off + f.off) + item.chunk;
+            const uint64_t* fl = reinterpret_cast<const uint64_t*>(sm.base[kBufArena][f.rank] + half_off + f.off) + item.chunk;
             ok &= wait_flag(fl, epoch, P);
           }
           if (!__all_sync(0xffffffffu, ok)) {
@@ -532,6 +556,11 @@ __global__ void __launch_bounds__(kTmaThreads, ADAPCC_TMA_MINB) engine_tma_kerne
       }
       if (lane == 0) {
         d.stop = stop;
+        if (P.trace) {
+          d.item = it;
+          d.tr0 = tr0;
+          d.tr1 = globaltimer();
+        }
         fence_proxy_async();      // acquired peer/arena data -> async-proxy (TMA) reads
         mbar_arrive(&sm.qfull[qi]);
       }
@@ -594,16 +623,25 @@ __global__ void __launch_bounds__(kTmaThreads, ADAPCC_TMA_MINB) engine_tma_kerne
           for (int i = 0; i < d.npost; ++i) st_release(d.post[i], epoch, sys);
         }
       }
+      if (P.trace && tid == 0 && !d.dropped)
+        trace_put(P, d.item, 0, d.tr0, d.tr1, globaltimer(), d.len * Ops<DT>::kEsize * (uint64_t)(d.nsrc + d.ndst));
       consumer_sync();    // all consumers are done reading the descriptor
       if (tid == 0) mbar_arrive(&sm.qempty[qi]);
       if (++qi == kQ) { qi = 0; qphase ^= 1; }
     }
   }
   __syncthreads();
+  if (P.trace && tid == 0) trace_put(P, kTraceCta, 0, t_entry, t_ready, globaltimer(), 0);
   if (tid == 0) {
-    tma_store_wait_all();  // this CTA's bulk stores are complete before it counts as done
-    fence_proxy_async();
-    fence(sys);
+    // across processes this CTA's bulk stores are complete before it counts as
+    // done (peers read the published word); in loopback only the next launch
+    // reads the epoch, after this grid has completed, so the count goes first
+    // and the store drain overlaps it
+    if (sys) {
+      tma_store_wait_all();
+      fence_proxy_async();
+      fence(sys);
+    }
     const unsigned done = atomicAdd(&P.state->done[par], 1u);
     if (done == gridDim.x - 1) {
       *reinterpret_cast<volatile unsigned long long*>(&P.state->epoch) = epoch;
@@ -616,6 +654,7 @@ __global__ void __launch_bounds__(kTmaThreads, ADAPCC_TMA_MINB) engine_tma_kerne
               wait_flag(reinterpret_cast<const uint64_t*>(P.hdr[q]), epoch, P);
       }
     }
+    if (!sys) tma_store_wait_all();  // bulk stores complete before the CTA exits
   }
 }
 

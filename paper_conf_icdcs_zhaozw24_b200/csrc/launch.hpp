@@ -22,6 +22,22 @@ struct DevState {
   unsigned long long epoch;  // last completed launch
 };
 
+// In-kernel trace record (adapcc_config("trace", capacity)): one per work
+// item a CTA executes plus one per CTA and launch (item == kTraceCta), times
+// from %globaltimer (ns).  Item: t0 claimed, t1 inputs ready (flags acquired),
+// t2 done (stores issued, flags posted).  CTA: t0 entry, t1 after the stream-
+// order wait and the epoch read, t2 exit.
+struct TraceRec {
+  uint32_t launch;  // launch sequence number of the communicator
+  uint32_t cta;
+  uint32_t item;
+  uint32_t task;
+  uint64_t t0, t1, t2;
+  uint64_t bytes;   // traffic of the item (sources + destinations)
+};
+static_assert(sizeof(TraceRec) == 48, "TraceRec layout");
+constexpr uint32_t kTraceCta = 0xFFFFFFFFu;
+
 struct LaunchParams {
   const Task* tasks;
   const BufRef* refs;
@@ -53,6 +69,10 @@ struct LaunchParams {
   uint64_t timeout_ns;
   uint64_t sig;         // call signature (debug check): hash of the call every rank must agree on
   int check_sig;        // 1: multi-process debug mode, compare `sig` with every peer's before any data moves
+  TraceRec* trace;        // nullptr: tracing off
+  unsigned* trace_n;      // records written (may exceed trace_cap: the excess is dropped)
+  uint32_t trace_cap;
+  uint32_t launch_seq;
   DevState* state;
   int* err;             // host-mapped error word
   char* send[kMaxRanksDev];
