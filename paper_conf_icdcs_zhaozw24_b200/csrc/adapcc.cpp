@@ -45,6 +45,7 @@ struct DevSegment {
   uint4* first = nullptr;         // LDG kernel: per-CTA first-item blobs (launch.hpp)
   uint32_t nfirst = 0, first_words = 0;
   uint32_t sched_static = 0;      // LDG kernel: every item has a blob, CTA b runs b, b + grid, ...
+  uint32_t arena_free = 0;        // no arena streams, flag waits or posts (launch.hpp)
 };
 
 struct DevPlan {
@@ -391,6 +392,12 @@ adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, const Strategy* strat, uin
     std::vector<Item> items = order_items(sp, c->loopback ? -1 : c->rank, rq.esize, grid_size(c, dtype, plan->kernel),
                                           (uint64_t)c->piece_kib * 1024, (int)c->taper, plan->kernel != 0);
     d.nitems = (uint32_t)items.size();
+    d.arena_free = 1;
+    for (const Task& t : sp.tasks) {
+      if (t.nwait || t.npost) d.arena_free = 0;
+      for (uint32_t k = 0; k < (uint32_t)t.nsrc + t.ndst + t.nlate; ++k)
+        if (sp.refs[t.ref0 + k].kind == kBufArena) d.arena_free = 0;
+    }
     auto up = [](auto** dst, const auto& v) -> cudaError_t {
       using T = typename std::decay_t<decltype(v)>::value_type;
       size_t bytes = std::max<size_t>(1, v.size()) * sizeof(T);
@@ -500,6 +507,7 @@ adapcc_result_t run(adapcc_comm_s* c, Coll coll, const void* const* send, void* 
     P.nfirst = seg.nfirst;
     P.first_words = seg.first_words;
     P.sched_static = seg.sched_static;
+    P.arena_free = seg.arena_free;
     P.dtype = (int)dtype;
     P.nranks = c->nranks;
     P.my_rank = c->loopback ? -1 : c->rank;

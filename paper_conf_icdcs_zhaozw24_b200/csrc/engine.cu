@@ -228,14 +228,99 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
     sh.blob[0][threadIdx.x] = P.first[(size_t)blockIdx.x * P.first_words + threadIdx.x];
   const bool stat = P.sched_static != 0;
   int buf = 0;  // blob buffer of the current item (static schedule)
-  // buffer bases into shared memory: dynamically indexed kernel parameters
-  // are constant-bank loads that miss on a cold launch (~1 us measured with
-  // the in-kernel trace); done before the stream-order wait
+  // buffer bases into shared memory (indexed by BufKind): read once per CTA,
+  // before the stream-order wait
   for (int i = threadIdx.x; i < 3 * P.nranks; i += kThreads) {
     const int k = i / P.nranks, q = i - k * P.nranks;
     sh.base[k][q] = k == 0 ? P.send[q] : k == 1 ? P.recv[q] : P.hdr[q];
   }
   if (threadIdx.x == 0 && !use_blob && blockIdx.x < P.nitems) pre = P.items[blockIdx.x];
+  constexpr int esize = Ops<DT>::kEsize;
+
+  // thread 0: stage item `it`'s header in shared memory, so that no task field
+  // stays live in registers across the fold (fb: from blob buffer b)
+  auto stage = [&](uint32_t it, bool fb, int b, bool is_first) {
+    sh.item = it;
+    if (P.trace) sh.tr0 = globaltimer();
+    sh.bad_align = 0;
+    sh.any_acc = 0;
+    if (it >= P.nitems) return;
+    const Item item = fb ? *reinterpret_cast<const Item*>(&sh.blob[b][0]) : is_first ? pre : P.items[it];
+    const Task& t = fb ? *reinterpret_cast<const Task*>(&sh.blob[b][1]) : P.tasks[item.task];
+    Cur& c = sh.cur;
+    c.blob = fb ? (int8_t)b : (int8_t)-1;
+    c.tnsrc = t.nsrc;
+    c.nreg = t.nsrc;
+    c.ndst = t.ndst;
+    c.nwait = t.nwait;
+    c.npost = t.npost;
+    c.op = t.op;
+    c.dropped = (int)t.owner == P.drop_rank;
+    c.late = 0;
+    c.force_acc = false;
+    if (P.late_mode && !c.dropped) {
+      if (t.nlate == 0) {
+        c.dropped = P.late_mode == 2;  // phase 2 only runs the roots' folds
+      } else {
+        const uint64_t m = late_select(P, t, it);
+        c.late = m;
+        if (P.late_mode == 2) {  // recv += sum of the late ranks not yet included
+          c.nreg = 0;
+          c.nwait = 0;
+          c.op = kOpFold;
+          c.force_acc = true;
+          c.dropped = m == 0;
+        } else if (m && t.op == kOpZero) {
+          c.op = kOpFold;
+        }
+      }
+    }
+    c.nsrc = (uint16_t)(c.nreg + __popcll(c.late));
+    c.ref0 = t.ref0;
+    c.flag0 = t.flag0;
+    c.chunk = item.chunk;
+    c.len = item.len;
+    c.e0 = t.lo + (uint64_t)item.chunk * t.chunk_elems + item.off;
+  };
+  // threads < nsrc + ndst: resolve the staged item's stream pointers.  Arena
+  // streams get `hoff` (the parity half); returns whether this thread's
+  // stream is an arena stream.
+  auto resolve = [&](uint64_t hoff) -> bool {
+    const int nsrc = sh.cur.nsrc, ndst = sh.cur.ndst;
+    if (threadIdx.x >= nsrc + ndst) return false;
+    const int i = threadIdx.x;
+    // index of this stream's ref, relative to the task's first ref
+    const uint32_t j = i < sh.cur.nreg ? i
+                     : i < nsrc ? sh.cur.tnsrc + ndst + nth_bit(sh.cur.late, i - sh.cur.nreg)
+                                : sh.cur.tnsrc + (i - nsrc);
+    const BufRef r = sh.cur.blob >= 0 ? *reinterpret_cast<const BufRef*>(&sh.blob[sh.cur.blob][kBlobRef0 + j])
+                                      : P.refs[sh.cur.ref0 + j];
+    const bool arena = r.kind == kBufArena;
+    char* p = sh.base[r.kind][r.rank] + (arena ? hoff : 0) + r.bias + (int64_t)(sh.cur.e0 * esize);
+    if (reinterpret_cast<uintptr_t>(p) & 15) atomicOr(&sh.bad_align, 1);  // (hoff is 256-byte aligned)
+    if (i < nsrc) {
+      sh.src[i] = p;
+    } else {
+      sh.dst[i - nsrc] = p;
+      const bool acc = r.accum || sh.cur.force_acc;
+      sh.acc[i - nsrc] = acc;
+      if (acc) atomicOr(&sh.any_acc, 1);
+    }
+    return arena;
+  };
+  // The first item of a blob CTA is staged and resolved here, before the
+  // stream-order wait: under PDL this overlaps the previous kernel instead of
+  // sitting between the epoch read and the first load (~0.8 us, in-kernel
+  // trace).  Arena pointers get the parity half once the epoch is known.
+  // Late join decides per item from ready words, so it stages after the wait.
+  const bool prestage = use_blob && P.late_mode == 0;
+  bool my_arena = false;
+  if (prestage) {
+    __syncthreads();  // blob words and buffer bases
+    if (threadIdx.x == 0) stage(blockIdx.x, true, 0, true);
+    __syncthreads();
+    if (sh.item < P.nitems && !sh.cur.dropped) my_arena = resolve(0);
+  }
   // the plan tables above are immutable; the epoch, counters, arenas and user
   // buffers below belong to the stream order (PDL: the previous launch)
   pdl_trigger();
@@ -272,64 +357,22 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
       if (!wait_flag(reinterpret_cast<const uint64_t*>(P.hdr[threadIdx.x] + ArenaHeader::kEntered), epoch, P)) sh.abort = 1;
     __syncthreads();
   }
-  constexpr int esize = Ops<DT>::kEsize;
   // Item claiming: CTA b starts with item b (no atomic), later items come from
   // the counter offset by the grid.  A CTA whose item is among the last
   // gridDim.x stops after it: every CTA makes exactly one such claim, so those
   // items are all taken and no CTA pays a final failed atomic (small calls run
   // with no claim atomics at all).
-  bool first = true, last = false;
+  bool first = true, last = false, staged = prestage;
   while (!sh.abort && !last) {
-    if (threadIdx.x == 0) {
-      // claim the next item and stage its header in shared memory, so that no
-      // task field stays live in registers across the fold
-      const uint32_t it = first ? blockIdx.x : stat ? sh.item + gridDim.x
-                                                    : gridDim.x + atomicAdd(&P.state->work[par], 1u);
-      sh.item = it;
-      if (P.trace) sh.tr0 = globaltimer();
-      sh.bad_align = 0;
-      sh.any_acc = 0;
-      if (it < P.nitems) {
-        const bool fb = stat || (first && blockIdx.x < P.nfirst);  // (recomputed: keeps no register live)
-        const Item item = fb ? *reinterpret_cast<const Item*>(&sh.blob[buf][0]) : first ? pre : P.items[it];
-        const Task& t = fb ? *reinterpret_cast<const Task*>(&sh.blob[buf][1]) : P.tasks[item.task];
-        Cur& c = sh.cur;
-        c.blob = fb ? (int8_t)buf : (int8_t)-1;
-        c.tnsrc = t.nsrc;
-        c.nreg = t.nsrc;
-        c.ndst = t.ndst;
-        c.nwait = t.nwait;
-        c.npost = t.npost;
-        c.op = t.op;
-        c.dropped = (int)t.owner == P.drop_rank;
-        c.late = 0;
-        c.force_acc = false;
-        if (P.late_mode && !c.dropped) {
-          if (t.nlate == 0) {
-            c.dropped = P.late_mode == 2;  // phase 2 only runs the roots' folds
-          } else {
-            const uint64_t m = late_select(P, t, it);
-            c.late = m;
-            if (P.late_mode == 2) {  // recv += sum of the late ranks not yet included
-              c.nreg = 0;
-              c.nwait = 0;
-              c.op = kOpFold;
-              c.force_acc = true;
-              c.dropped = m == 0;
-            } else if (m && t.op == kOpZero) {
-              c.op = kOpFold;
-            }
-          }
-        }
-        c.nsrc = (uint16_t)(c.nreg + __popcll(c.late));
-        c.ref0 = t.ref0;
-        c.flag0 = t.flag0;
-        c.chunk = item.chunk;
-        c.len = item.len;
-        c.e0 = t.lo + (uint64_t)item.chunk * t.chunk_elems + item.off;
+    if (!staged) {
+      if (threadIdx.x == 0) {
+        const uint32_t it = first ? blockIdx.x : stat ? sh.item + gridDim.x
+                                                      : gridDim.x + atomicAdd(&P.state->work[par], 1u);
+        const bool fb = stat || (first && use_blob);
+        stage(it, fb, buf, first);
       }
+      __syncthreads();
     }
-    __syncthreads();
     if (sh.item >= P.nitems) break;
     first = false;
     last = (uint64_t)sh.item + gridDim.x >= P.nitems;
@@ -348,28 +391,15 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
             reinterpret_cast<const uint64_t*>(sh.base[kBufArena][f.rank] + half_off + f.off) + sh.cur.chunk;
         if (!wait_flag(fl, epoch, P)) sh.abort = 1;
       }
-      // resolve stream pointers for this piece
-      if (threadIdx.x < nsrc + ndst) {
+      if (!staged) {
+        resolve(half_off);
+      } else if (my_arena) {  // pre-staged before the epoch was known
         const int i = threadIdx.x;
-        // index of this stream's ref, relative to the task's first ref
-        const uint32_t j = i < sh.cur.nreg ? i
-                         : i < nsrc ? sh.cur.tnsrc + ndst + nth_bit(sh.cur.late, i - sh.cur.nreg)
-                                    : sh.cur.tnsrc + (i - nsrc);
-        const BufRef r = sh.cur.blob >= 0 ? *reinterpret_cast<const BufRef*>(&sh.blob[sh.cur.blob][kBlobRef0 + j])
-                                          : P.refs[sh.cur.ref0 + j];
-        char* base = sh.base[r.kind][r.rank] + (r.kind == kBufArena ? half_off : 0);
-        char* p = base + r.bias + (int64_t)(sh.cur.e0 * esize);
-        if (reinterpret_cast<uintptr_t>(p) & 15) atomicOr(&sh.bad_align, 1);
-        if (threadIdx.x < nsrc) {
-          sh.src[threadIdx.x] = p;
-        } else {
-          sh.dst[threadIdx.x - nsrc] = p;
-          const bool acc = r.accum || sh.cur.force_acc;
-          sh.acc[threadIdx.x - nsrc] = acc;
-          if (acc) atomicOr(&sh.any_acc, 1);
-        }
+        if (i < nsrc) sh.src[i] += half_off;
+        else sh.dst[i - nsrc] += half_off;
       }
     }
+    staged = false;
     __syncthreads();
     if (P.trace && threadIdx.x == 0) sh.tr1 = globaltimer();
     if (sh.abort) {

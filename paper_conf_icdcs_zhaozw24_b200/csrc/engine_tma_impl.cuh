@@ -472,13 +472,23 @@ __global__ void __launch_bounds__(kTmaThreads, ADAPCC_TMA_MINB) engine_tma_kerne
     if (use_blob)
       for (uint32_t i = lane; i < P.first_words; i += 32)
         sm.blob[i] = P.first[(size_t)blockIdx.x * P.first_words + i];
-    // buffer bases into shared memory (dynamically indexed parameters are
-    // constant-bank loads that miss on a cold launch)
+    // buffer bases into shared memory (indexed by BufKind)
     for (int i = lane; i < 3 * P.nranks; i += 32) {
       const int k = i / P.nranks, q = i - k * P.nranks;
       sm.base[k][q] = k == 0 ? P.send[q] : k == 1 ? P.recv[q] : P.hdr[q];
     }
     __syncwarp();
+    // A plan without arena streams or flags (DIRECT: loopback and zero-copy)
+    // describes its first item before the stream-order wait: its pointers do
+    // not depend on the epoch's parity half, so under PDL this overlaps the
+    // previous kernel.  Late join decides per item from ready words: after.
+    if (use_blob && P.arena_free && P.late_mode == 0) {
+      int nwait = 0;
+      fill_desc<DT>(P, sm.base, sm.q[0], *reinterpret_cast<const Item*>(&sm.blob[0]),
+                    *reinterpret_cast<const Task*>(&sm.blob[1]),
+                    reinterpret_cast<const BufRef*>(&sm.blob[kBlobRef0]), 0, lane, blockIdx.x, &nwait);
+      __syncwarp();
+    }
   }
   // shared-memory set-up above; the epoch, counters, arenas and user buffers
   // below belong to the stream order (PDL: the previous launch)
@@ -538,9 +548,11 @@ __global__ void __launch_bounds__(kTmaThreads, ADAPCC_TMA_MINB) engine_tma_kerne
       const Task& t = fb ? *reinterpret_cast<const Task*>(&sm.blob[1]) : P.tasks[item.task];
       if (!stop) {
         int nwait = 0;
-        const BufRef* R = fb ? reinterpret_cast<const BufRef*>(&sm.blob[kBlobRef0]) : P.refs + t.ref0;
-        fill_desc<DT>(P, sm.base, d, item, t, R, half_off, lane, it, &nwait);
-        __syncwarp();
+        if (!(fb && P.arena_free && P.late_mode == 0)) {  // (else described before the wait, above)
+          const BufRef* R = fb ? reinterpret_cast<const BufRef*>(&sm.blob[kBlobRef0]) : P.refs + t.ref0;
+          fill_desc<DT>(P, sm.base, d, item, t, R, half_off, lane, it, &nwait);
+          __syncwarp();
+        }
         if (!d.dropped) {
           int ok = 1;
           for (int i = lane; i < nwait; i += 32) {

@@ -55,6 +55,10 @@ struct LaunchParams {
   // smallest unfinished item's CTA has finished all its earlier items and its
   // inputs come from smaller items
   uint32_t sched_static;
+  // 1: no task has arena streams, flag waits or posts (DIRECT plans): item
+  // pointers do not depend on the epoch (the TMA kernel describes its first
+  // item before the stream-order wait)
+  uint32_t arena_free;
   int dtype;
   int nranks;
   int my_rank;          // multi-process: this rank; loopback: -1
