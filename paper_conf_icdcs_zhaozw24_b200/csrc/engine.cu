@@ -315,6 +315,7 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
   // Late join decides per item from ready words, so it stages after the wait.
   const bool prestage = use_blob && P.late_mode == 0;
   bool my_arena = false;
+  if (threadIdx.x == 0) sh.abort = 0;
   if (prestage) {
     __syncthreads();  // blob words and buffer bases
     if (threadIdx.x == 0) stage(blockIdx.x, true, 0, true);
@@ -325,19 +326,28 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
   // buffers below belong to the stream order (PDL: the previous launch)
   pdl_trigger();
   pdl_wait();
-  if (threadIdx.x == 0) {
-    sh.abort = 0;
-    // this launch's epoch = the one the previous launch published + 1
-    const uint64_t e = *reinterpret_cast<volatile unsigned long long*>(&P.state->epoch) + 1;
-    sh.epoch = e;
-    if (blockIdx.x == 0) {  // re-arm the other parity's counters for the next launch
-      P.state->work[(e + 1) & 1] = 0;
-      P.state->done[(e + 1) & 1] = 0;
+  // Lazy epoch: a loopback plan without arena streams or flags whose CTAs
+  // need no claim counter only uses the epoch to count itself done at the
+  // end, so its load stays in flight during the fold instead of costing a
+  // round trip and a barrier up front.
+  const bool lazy = !P.ipc && P.arena_free && prestage && (stat || P.nitems <= gridDim.x);
+  uint64_t e_lazy = 0;
+  if (lazy) {
+    if (threadIdx.x == 0) e_lazy = *reinterpret_cast<volatile unsigned long long*>(&P.state->epoch) + 1;
+  } else {
+    if (threadIdx.x == 0) {
+      // this launch's epoch = the one the previous launch published + 1
+      const uint64_t e = *reinterpret_cast<volatile unsigned long long*>(&P.state->epoch) + 1;
+      sh.epoch = e;
+      if (blockIdx.x == 0) {  // re-arm the other parity's counters for the next launch
+        P.state->work[(e + 1) & 1] = 0;
+        P.state->done[(e + 1) & 1] = 0;
+      }
     }
+    __syncthreads();
   }
-  __syncthreads();
   const uint64_t t_ready = P.trace ? globaltimer() : 0;
-  const uint64_t epoch = sh.epoch;
+  const uint64_t epoch = lazy ? 0 : sh.epoch;  // (lazy: unused before the end)
   const unsigned par = (unsigned)(epoch & 1);
   const uint64_t half_off = kArenaHeader + par * P.half_bytes;
   // multi-process: every peer must have finished the call that last used this
@@ -438,11 +448,16 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
     // CTA's data; in loopback only the next launch reads anything, after
     // this one completes, so counting needs no fence
     if (sys) fence(sys);
-    const unsigned done = atomicAdd(&P.state->done[par], 1u);
+    const uint64_t ep = lazy ? e_lazy : epoch;
+    if (lazy && blockIdx.x == 0) {  // re-arm the other parity's counters for the next launch
+      P.state->work[(ep + 1) & 1] = 0;
+      P.state->done[(ep + 1) & 1] = 0;
+    }
+    const unsigned done = atomicAdd(&P.state->done[ep & 1], 1u);
     if (done == gridDim.x - 1) {
       // last CTA: publish the epoch for the next launch on this stream and,
       // across processes, "this rank finished epoch" to the peers
-      *reinterpret_cast<volatile unsigned long long*>(&P.state->epoch) = epoch;
+      *reinterpret_cast<volatile unsigned long long*>(&P.state->epoch) = ep;
       if (P.ipc) {
         __threadfence_system();
         st_release(reinterpret_cast<uint64_t*>(P.hdr[P.my_rank]), epoch, true);
