@@ -1,3 +1,6 @@
-python scripts/debug/ab_configs.py --coll allreduce --sizes 10,16,18,20,21,22 --reps 5 --configs 'engine=2;sched=0' 2>&1 | tail -6
-python scripts/debug/ab_configs.py --coll alltoall --sizes 10,20,22 --reps 5 --configs 'engine=2' 2>&1 | tail -3
-timeout 1500 python -m pytest tests -m gpu -x -q -p no:cacheprovider > gpurun_out/t_all.log 2>&1; tail -2 gpurun_out/t_all.log
+mkdir -p gpurun_out/trace
+python scripts/trace_report.py --bytes-per-rank 1048576 --out gpurun_out/trace/allreduce_1MiB > /dev/null 2>gpurun_out/trace/err1.log
+python scripts/trace_report.py --bytes-per-rank 8388608 --out gpurun_out/trace/allreduce_8MiB > /dev/null 2>gpurun_out/trace/err2.log
+python scripts/trace_report.py --bytes-per-rank 268435456 --calls 4 --out gpurun_out/trace/allreduce_256MiB > /dev/null 2>gpurun_out/trace/err3.log
+python scripts/trace_report.py --bytes-per-rank 16777216 --mode staged --out gpurun_out/trace/allreduce_staged_16MiB > /dev/null 2>gpurun_out/trace/err4.log
+python scripts/trace_report.py --coll alltoall --bytes-per-rank 33554432 --out gpurun_out/trace/alltoall_32MiB > /dev/null 2>gpurun_out/trace/err5.log
