@@ -601,8 +601,12 @@ std::vector<Item> order_items(const SegmentPlan& p, int rank, int esize, int gri
   // profiles/taper_*_r01.json: +1-3 % from 16 MiB per rank up, where pieces
   // are 448-512 KiB; halving ~110-230 KiB pieces costs more in per-item
   // overhead than the shorter tail saves).
+  // Automatic taper only from m >= 3 items per CTA: with one or two balanced
+  // rounds the last round is already even, and halving its items only adds
+  // per-item overhead (8 MiB per rank, m = 2: 26.3 us tapered, 24.8 us not;
+  // 16 MiB, m = 4: 46.0 vs 46.3 us, profiles/ab/taper_r01.txt).
   const bool auto_taper = taper <= 0;
-  if (auto_taper) taper = 2;
+  if (auto_taper) taper = (piece_bytes || m >= 3) ? 2 : 1;
   std::vector<uint8_t> split(keys.size(), 0);
   if (taper > 1) {
     uint64_t want = 2ull * std::max(grid, 1);
