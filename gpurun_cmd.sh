@@ -1,3 +1,3 @@
-timeout 1500 python -m pytest tests -m gpu -x -q -p no:cacheprovider > gpurun_out/t_all.log 2>&1; tail -2 gpurun_out/t_all.log
-timeout 1200 python scripts/bench_configs.py --out gpurun_out/configs_new.json > gpurun_out/configs_new.log 2>&1; tail -3 gpurun_out/configs_new.log
-python scripts/debug/host_overhead.py > gpurun_out/host_overhead.txt 2>&1
+python scripts/debug/ab_configs.py --coll allgather --sizes 23,24,25,26 --reps 5 --configs 'engine=0;engine=1;engine=0,sched=0' 2>&1 | tail -4
+python scripts/debug/ab_configs.py --coll allreduce --sizes 23,24,25 --reps 5 --configs 'engine=0;engine=1' 2>&1 | tail -3
+python scripts/debug/ab_configs.py --coll alltoall --sizes 23,24,25 --reps 5 --configs 'engine=0;engine=1' 2>&1 | tail -3

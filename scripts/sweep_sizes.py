@@ -21,7 +21,7 @@ def main():
     ap.add_argument("--ranks", type=int, default=8)
     ap.add_argument("--dtype", default="f32", choices=["f32", "bf16"])
     ap.add_argument("--mode", default="direct", choices=["direct", "staged"])
-    ap.add_argument("--coll", default="allreduce", choices=["allreduce", "allgather", "alltoall"])
+    ap.add_argument("--coll", default="allreduce", choices=["allreduce", "allgather", "alltoall", "reducescatter", "reduce", "broadcast"])
     ap.add_argument("--chunk-kib", type=int, default=256)
     ap.add_argument("--min-log2", type=int, default=10)
     ap.add_argument("--max-log2", type=int, default=30)
@@ -56,8 +56,11 @@ def main():
         comm.set_strategy("allreduce", G.allreduce_stars(n, chunk=chunk))
     elif a.coll == "allgather":
         comm.set_strategy("allgather", G.allgather_stars(n, chunk=chunk))
-    else:
+    elif a.coll == "alltoall":
         comm.set_strategy("alltoall", G.alltoall_direct(n, chunk=chunk))
+    elif a.coll == "reducescatter":
+        comm.set_strategy("reducescatter", G.reducescatter_stars(n, chunk=chunk))
+    # reduce / broadcast: the library's default star rooted at the call's root (rank 0)
     res = []
     for lg in range(a.min_log2, a.max_log2 + 1):
         nbytes = 1 << lg
@@ -73,11 +76,27 @@ def main():
             call = lambda: comm.allgather_lb(xs, ys)  # noqa: E731
             # DIRECT: every shard read once, written to all n outputs
             factor, alg_bytes = (n - 1.0) / n, n * n * xs[0].numel() * es + n * xs[0].numel() * es
-        else:
+        elif a.coll == "alltoall":
             xs = [torch.randn(count, device="cuda").to(tdt) for _ in range(n)]
             ys = [torch.empty_like(x) for x in xs]
             call = lambda: comm.alltoall_lb(xs, ys)  # noqa: E731
             factor, alg_bytes = (n - 1.0) / n, 2 * n * nbytes
+        elif a.coll == "reducescatter":  # bytes_per_rank = input per rank (n blocks), nccl-tests convention
+            xs = [torch.randn(count // n * n or n, device="cuda").to(tdt) for _ in range(n)]
+            ys = [torch.empty(xs[0].numel() // n, device="cuda", dtype=tdt) for _ in range(n)]
+            call = lambda: comm.reducescatter_lb(xs, ys)  # noqa: E731
+            # DIRECT: every input read once, every output block written once
+            factor, alg_bytes = (n - 1.0) / n, (n + 1) * xs[0].numel() * es
+        elif a.coll == "reduce":
+            xs = [torch.randn(count, device="cuda").to(tdt) for _ in range(n)]
+            ys = [torch.empty_like(x) for x in xs]
+            call = lambda: comm.reduce_lb(xs, ys, 0)  # noqa: E731
+            factor, alg_bytes = 1.0, (n + 1) * nbytes
+        else:
+            xs = [torch.randn(count, device="cuda").to(tdt) for _ in range(n)]
+            ys = [torch.empty_like(x) for x in xs]
+            call = lambda: comm.broadcast_lb(xs, ys, 0)  # noqa: E731
+            factor, alg_bytes = 1.0, (n + 1) * nbytes
         for _ in range(5):
             call()
         torch.cuda.synchronize()
