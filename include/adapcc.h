@@ -382,6 +382,29 @@ ADAPCC_API adapcc_result_t adapcc_plan_stats(const char* strategy_text, uint64_t
                                   adapcc_mode_t mode, int rank, size_t scratch_bytes,
                                   uint64_t members, adapcc_plan_stats_t* stats);
 
+/* Host-only inspection of the work items the engine would execute for one segment (launch) of a
+ * call: the plan compiler's output (DESIGN.md §6 "Work items", "Pieces"), for CPU tests of the
+ * host logic.  grid = CTAs of the launch (pieces are sized for it), tma = 1 for the TMA pipeline's
+ * piece rule, piece_kib / taper as adapcc_config (0 = automatic).  Items come in claim order; an
+ * item covers elements [off, off + len) of chunk `chunk` of task `task` (element offsets from the
+ * chunk start).  Tasks are listed with their element range, chunking, stream counts, flag counts
+ * and dependency level.  Up to max_items / max_tasks entries are copied; *n_items / *n_tasks get
+ * the full counts.  segment >= the number of segments: INVALID_ARGUMENT. */
+typedef struct { uint32_t task, chunk, off, len; } adapcc_item_t;
+typedef struct {
+  uint64_t lo, hi;                  /* elements covered */
+  uint32_t chunk_elems, nchunks;
+  uint16_t nsrc, ndst, nwait, npost;
+  uint32_t level;                   /* dependency depth: waits only on posts of lower levels */
+  uint32_t owner;                   /* executing rank */
+} adapcc_task_info_t;
+ADAPCC_API adapcc_result_t adapcc_plan_items(const char* strategy_text, uint64_t count,
+                                  adapcc_dtype_t dtype, uint64_t ready_mask, unsigned flags,
+                                  adapcc_mode_t mode, int rank, size_t scratch_bytes, int grid,
+                                  int tma, uint32_t piece_kib, int taper, int segment,
+                                  adapcc_item_t* items, uint32_t max_items, uint32_t* n_items,
+                                  adapcc_task_info_t* tasks, uint32_t max_tasks, uint32_t* n_tasks);
+
 #ifdef __cplusplus
 }
 #endif

@@ -6,5 +6,5 @@ ctypes binding and ``generator`` emits strategy text.
 """
 
 from . import coordinator, costmodel, ddp, generator  # noqa: F401
-from .adapcc import (AdapccError, Communicator, plan_stats, strategy_check,  # noqa: F401
+from .adapcc import (AdapccError, Communicator, plan_items, plan_stats, strategy_check,  # noqa: F401
                      strategy_partition, strategy_sub, strategy_tuples, lib_path)

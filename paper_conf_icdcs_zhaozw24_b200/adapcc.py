@@ -112,6 +112,9 @@ def _load():
                                       ctypes.POINTER(i32)],
         "adapcc_plan_stats": [ctypes.c_char_p, u64, i32, u64, ctypes.c_uint, i32, i32, sz, u64,
                               ctypes.POINTER(PlanStats)],
+        "adapcc_plan_items": [ctypes.c_char_p, u64, i32, u64, ctypes.c_uint, i32, i32, sz, i32, i32,
+                              ctypes.c_uint32, i32, i32, vp, ctypes.c_uint32, ctypes.POINTER(ctypes.c_uint32),
+                              vp, ctypes.c_uint32, ctypes.POINTER(ctypes.c_uint32)],
     }
     for name, args in sig.items():
         f = getattr(L, name)
@@ -240,6 +243,26 @@ def plan_stats(text, count, dtype, mask, accumulate=False, mode="direct", rank=-
                                FLAG_ACCUMULATE if accumulate else 0, MODE[mode], rank,
                                scratch_bytes, mm, ctypes.byref(st)), "plan_stats")
     return st.as_dict()
+
+
+def plan_items(text, count, dtype, mask, grid, tma=False, accumulate=False, mode="direct", rank=-1,
+               scratch_bytes=0, piece_kib=0, taper=0, segment=0):
+    """Work items (claim order) and tasks of one segment of a call's plan, as
+    numpy structured arrays (include/adapcc.h adapcc_plan_items)."""
+    import numpy as np
+    L = _load()
+    idt = np.dtype([("task", "<u4"), ("chunk", "<u4"), ("off", "<u4"), ("len", "<u4")])
+    tdt = np.dtype([("lo", "<u8"), ("hi", "<u8"), ("chunk_elems", "<u4"), ("nchunks", "<u4"),
+                    ("nsrc", "<u2"), ("ndst", "<u2"), ("nwait", "<u2"), ("npost", "<u2"),
+                    ("level", "<u4"), ("owner", "<u4")])
+    ni, nt = ctypes.c_uint32(), ctypes.c_uint32()
+    args = (text.encode(), count, DTYPE_CODE[dtype], mask, FLAG_ACCUMULATE if accumulate else 0, MODE[mode],
+            rank, scratch_bytes, grid, 1 if tma else 0, piece_kib, taper, segment)
+    _check(L.adapcc_plan_items(*args, None, 0, ctypes.byref(ni), None, 0, ctypes.byref(nt)), "plan_items")
+    items, tasks = np.zeros(ni.value, dtype=idt), np.zeros(nt.value, dtype=tdt)
+    _check(L.adapcc_plan_items(*args, items.ctypes.data, ni.value, ctypes.byref(ni), tasks.ctypes.data,
+                               nt.value, ctypes.byref(nt)), "plan_items")
+    return items, tasks
 
 
 # --------------------------------------------------------------- communicator

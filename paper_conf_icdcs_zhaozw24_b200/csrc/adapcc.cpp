@@ -1357,4 +1357,46 @@ adapcc_result_t adapcc_plan_stats(const char* text, uint64_t count, adapcc_dtype
   return ADAPCC_SUCCESS;
 }
 
+adapcc_result_t adapcc_plan_items(const char* text, uint64_t count, adapcc_dtype_t dtype, uint64_t mask,
+                                  unsigned flags, adapcc_mode_t mode, int rank, size_t scratch_bytes, int grid,
+                                  int tma, uint32_t piece_kib, int taper, int segment, adapcc_item_t* items,
+                                  uint32_t max_items, uint32_t* n_items, adapcc_task_info_t* tasks,
+                                  uint32_t max_tasks, uint32_t* n_tasks) {
+  Strategy st;
+  if (!text || !parse_strategy(text, &st, nullptr)) return ADAPCC_ERR_INVALID_STRATEGY;
+  if (rank < -1 || rank >= st.nranks || grid < 1 || segment < 0 || taper < 0 || taper > 64 || !n_items ||
+      !n_tasks || (max_items && !items) || (max_tasks && !tasks))
+    return ADAPCC_ERR_INVALID_ARGUMENT;
+  const uint64_t members = st.nranks >= 64 ? ~uint64_t(0) : ((uint64_t(1) << st.nranks) - 1);
+  if (mask & ~members) return ADAPCC_ERR_INVALID_ARGUMENT;
+  PlanRequest rq;
+  rq.members = members;
+  rq.st = &st;
+  rq.count = count;
+  rq.esize = esize_of(dtype);
+  rq.ready_mask = mask;
+  rq.accumulate = flags & ADAPCC_FLAG_ACCUMULATE;
+  rq.late_join = flags & ADAPCC_FLAG_LATE_JOIN;
+  rq.mode = (Mode)mode;
+  rq.grid = grid;
+  const size_t scratch = scratch_bytes ? scratch_bytes : kDefaultScratch;
+  if (scratch < (size_t)kArenaHeader + 2 * (4096 + 65536)) return ADAPCC_ERR_INVALID_ARGUMENT;
+  rq.half_bytes = ((scratch - kArenaHeader) / 2) / 256 * 256;
+  std::vector<SegmentPlan> segs;
+  if (!build_plan(rq, &segs, nullptr)) return ADAPCC_ERR_OOM;
+  if ((size_t)segment >= segs.size()) return ADAPCC_ERR_INVALID_ARGUMENT;
+  const SegmentPlan& sp = segs[segment];
+  const std::vector<Item> it = order_items(sp, rank, rq.esize, grid, (uint64_t)piece_kib * 1024, taper, tma != 0);
+  *n_items = (uint32_t)it.size();
+  for (uint32_t i = 0; i < std::min<uint32_t>(max_items, *n_items); ++i)
+    items[i] = adapcc_item_t{it[i].task, it[i].chunk, it[i].off, it[i].len};
+  *n_tasks = (uint32_t)sp.tasks.size();
+  for (uint32_t i = 0; i < std::min<uint32_t>(max_tasks, *n_tasks); ++i) {
+    const Task& t = sp.tasks[i];
+    tasks[i] = adapcc_task_info_t{t.lo, t.hi, t.chunk_elems, t.nchunks, t.nsrc, t.ndst, t.nwait, t.npost,
+                                  t.level, t.owner};
+  }
+  return ADAPCC_SUCCESS;
+}
+
 }  // extern "C"

@@ -19,7 +19,7 @@ run() {
   echo "== exit $?" >> gpurun_out/sanitize_$tool.log
 }
 LB=tests/test_gpu_loopback.py
-MORE="tests/test_gpu_primitives.py tests/test_gpu_late_join.py tests/test_gpu_a2a_routes.py"
+MORE="tests/test_gpu_primitives.py tests/test_gpu_late_join.py tests/test_gpu_a2a_routes.py tests/test_gpu_trace.py"
 # leak-check off: the only leaks reported are PyTorch caching-allocator segments alive at exit
 run memcheck "$LB $MORE" "not watchdog"
 run racecheck "$LB" "(allreduce_parity and f32 and (stars8 or dbinary)) or (alltoall and bf16) or c1_config or (tma_large_items and f32)"
