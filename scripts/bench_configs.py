@@ -8,6 +8,7 @@ C3  partial AllReduce, 8 ranks, stragglers {3,6}: T_adapcc = end of phase 2 (pha
     ready ranks at t=0 with relays, phase 2 ACCUMULATE once the stragglers are ready) vs
     T_wait = t_s + T_full, straggler lag t_s simulated by a 1-CTA spin kernel on a compute stream
 C4  AlltoAll 8 ranks, [8][512][4096] bf16 per rank
+C4v AlltoAllv MoE dispatch, 8 ranks x 4096 tokens x 4096 bf16, Zipf(a) top-1 routing, a in {0, 1.2, 2}
 C5  AllGather of GPT-2-XL row shards, 48 layers x 4 weights, strategy swap at call 96
 G1  local chunk reduction: Reduce of k in {2, 8} virtual 1 GiB inputs into one
     1 GiB output (one star tree rooted at 0), fp32 and bf16; GB/s = (k+1) S / t vs the HBM peak
@@ -27,7 +28,7 @@ sys.path.insert(0, ROOT)
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--out", default=os.path.join(ROOT, "gpurun_out", "configs.json"))
-    ap.add_argument("--only", default="C1,C2,C3,C4,C5,G1")
+    ap.add_argument("--only", default="C1,C2,C3,C4,C4v,C5,G1")
     a = ap.parse_args()
 
     import numpy as np
@@ -242,6 +243,40 @@ def main():
             print("C4", res[-1], flush=True)
             comm.finalize()
         out["C4"] = res
+
+    # ------------------------------------------------------------------ C4v
+    # AlltoAllv MoE dispatch (NEXT-4): 8 ranks x 4096 tokens x hidden 4096 bf16 per rank, top-1
+    # routing with Zipf(a) expert popularity (a = 0: uniform), DIRECT plan; algorithmic bytes =
+    # every token read once and written once; busbw counts the tokens that leave their rank.
+    if "C4v" in only:
+        from synth.inputs import moe_counts
+        res = []
+        n, tok, hid = 8, 4096, 4096
+        text = G.alltoall_direct(n, chunk=1 << 20)
+        for a_zipf in (0.0, 1.2, 2.0):
+            counts = moe_counts(n, tok, hid, zipf_a=a_zipf)
+            send = [sum(counts[s]) for s in range(n)]
+            recv = [sum(counts[s][d] for s in range(n)) for d in range(n)]
+            xs = [rank_tensors("bf16", send[s], 1, base=2200 + s)[0] for s in range(n)]
+            comm = pkg.Communicator.loopback(n, mode="direct", scratch_bytes=64 << 20)
+            comm.set_strategy("alltoall", text)
+            dx = [dev(x, "bf16") for x in xs]
+            dy = [torch.empty(recv[d], dtype=torch.bfloat16, device="cuda") for d in range(n)]
+            ms = timeit_graph(lambda: comm.alltoallv_lb(dx, dy, counts))
+            prev = [np.zeros(recv[d], np.uint16) for d in range(n)]
+            exp = oc.alltoallv(xs, counts, text, set(range(n)), "bf16", prev)
+            comm.alltoallv_lb(dx, dy, counts)
+            torch.cuda.synchronize()
+            ok = all(np.array_equal(host_bits(dy[d], "bf16"), exp[d]) for d in range(n))
+            moved = sum(counts[s][d] for s in range(n) for d in range(n) if s != d) * 2
+            total = sum(send) * 2
+            res.append({"zipf_a": a_zipf, "max_recv_tokens": max(recv) // hid, "min_recv_tokens": min(recv) // hid,
+                        "ms_graph": round(ms, 4), "busbw_per_rank": round(moved / n / ms / 1e6, 1),
+                        "hbm_frac": round(2 * total / ms / 1e6 / 6545.6, 4), "parity": ok,
+                        "kernel": comm.last_engine()})
+            print("C4v", res[-1], flush=True)
+            comm.finalize()
+        out["C4v"] = res
 
     # ------------------------------------------------------------------ C5
     if "C5" in only:
