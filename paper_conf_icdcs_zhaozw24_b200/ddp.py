@@ -7,18 +7,27 @@ The paper exposes "a communication hook for PyTorch DDP".  Usage:
 
 Each gradient bucket is averaged in place by one engine launch on the current
 stream (the STAGED protocol, or the zero-copy DIRECT plan when the bucket's
-storage was registered with comm.register).  `ready` may restrict the
-aggregation to the ready ranks (partial aggregation); the bucket is then
-divided by the number of contributing ranks.
+storage was registered with comm.register).  With auto_register=True the hook
+registers every bucket buffer the first time it sees it, so a training loop
+runs zero-copy from its first step without touching DDP internals.  DDP
+launches buckets in index order on every rank, which keeps the collective
+registrations in the same order everywhere; DDP rebuilds its buckets once
+after the first iteration, so each bucket is registered at most twice.
+`ready` may restrict the aggregation to the ready ranks (partial
+aggregation); the bucket is then divided by the number of contributing ranks.
 """
 
 import torch
 
 
 class AdapccHookState:
-    def __init__(self, comm, ready=None):
+    def __init__(self, comm, ready=None, auto_register=False):
         self.comm = comm
         self.ready = ready            # None = every rank
+        self.auto_register = auto_register
+        self.registered = 0           # buffers this hook registered
+        self.zero_copy_calls = 0
+        self.staged_calls = 0
 
     def contributors(self):
         if self.ready is None:              # every live rank (all, unless some were excluded)
@@ -33,9 +42,19 @@ def adapcc_allreduce_hook(state, bucket):
     comm = state.comm
     try:
         comm._reg_of(buf)
+        registered = True
+    except ValueError:
+        registered = False
+    if not registered and state.auto_register:
+        comm.register(buf)   # collective: every rank reaches this bucket in the same order
+        state.registered += 1
+        registered = True
+    if registered:
         comm.collective_zc("allreduce", buf, buf, buf.numel(), ready=state.ready)
-    except ValueError:   # bucket not registered: STAGED protocol through the arenas
+        state.zero_copy_calls += 1
+    else:                # bucket not registered: STAGED protocol through the arenas
         comm.allreduce(buf, buf, ready=state.ready)
+        state.staged_calls += 1
     buf.div_(state.contributors())
     fut = torch.futures.Future()
     fut.set_result(buf)

@@ -22,7 +22,7 @@ def _port():
     return p
 
 
-def _worker(rank, n, port, q):
+def _worker(rank, n, port, q, auto_register=False, steps=1):
     try:
         sys.path.insert(0, ROOT)
         import torch.distributed as dist
@@ -39,24 +39,29 @@ def _worker(rank, n, port, q):
         ref = [p.detach().clone() for p in model.parameters()]
         comm = pkg.Communicator.init(scratch_bytes=64 << 20, device=0)
         ddp = DDP(model, device_ids=[0], bucket_cap_mb=1)
-        ddp.register_comm_hook(AdapccHookState(comm), adapcc_allreduce_hook)
+        state = AdapccHookState(comm, auto_register=auto_register)
+        ddp.register_comm_hook(state, adapcc_allreduce_hook)
         g = torch.Generator(device="cpu").manual_seed(100 + rank)
-        x = torch.randn(32, 64, generator=g).cuda()
-        ddp(x).square().sum().backward()
-        torch.cuda.synchronize()
-        # expected: average of every rank's local gradient of the same loss
-        local = torch.nn.Sequential(torch.nn.Linear(64, 256), torch.nn.ReLU(), torch.nn.Linear(256, 8)).cuda()
-        with torch.no_grad():
-            for p, r in zip(local.parameters(), ref):
-                p.copy_(r)
-        local(x).square().sum().backward()
-        grads = [p.grad.detach().cpu() for p in local.parameters()]
-        allg = [None] * n
-        dist.all_gather_object(allg, grads)
         ok = True
-        for i, p in enumerate(model.parameters()):
-            exp = sum(allg[r][i] for r in range(n)) / n
-            ok &= torch.allclose(p.grad.cpu(), exp, rtol=1e-5, atol=1e-6)
+        for step in range(steps):   # parameters stay fixed: every step checks the same reduction
+            ddp.zero_grad(set_to_none=False)
+            x = torch.randn(32, 64, generator=g).cuda()
+            ddp(x).square().sum().backward()
+            torch.cuda.synchronize()
+            # expected: average of every rank's local gradient of the same loss
+            local = torch.nn.Sequential(torch.nn.Linear(64, 256), torch.nn.ReLU(), torch.nn.Linear(256, 8)).cuda()
+            with torch.no_grad():
+                for p, r in zip(local.parameters(), ref):
+                    p.copy_(r)
+            local(x).square().sum().backward()
+            grads = [p.grad.detach().cpu() for p in local.parameters()]
+            allg = [None] * n
+            dist.all_gather_object(allg, grads)
+            for i, p in enumerate(model.parameters()):
+                exp = sum(allg[r][i] for r in range(n)) / n
+                ok &= torch.allclose(p.grad.cpu(), exp, rtol=1e-5, atol=1e-6)
+        if auto_register:  # every bucket went zero-copy, none through the arenas
+            ok &= state.registered > 0 and state.staged_calls == 0 and state.zero_copy_calls > 0
         err = comm.get_async_error()
         comm.finalize()
         dist.destroy_process_group()
@@ -66,14 +71,14 @@ def _worker(rank, n, port, q):
         q.put((rank, False, traceback.format_exc() + repr(e)))
 
 
-def test_ddp_hook_two_processes_one_gpu():
+def _run(auto_register, steps):
     if not torch.cuda.is_available():
         pytest.skip("no GPU")
     import torch.multiprocessing as mp
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _port()
-    procs = [ctx.Process(target=_worker, args=(r, 2, port, q)) for r in range(2)]
+    procs = [ctx.Process(target=_worker, args=(r, 2, port, q, auto_register, steps)) for r in range(2)]
     for p in procs:
         p.start()
     out = {}
@@ -88,3 +93,13 @@ def test_ddp_hook_two_processes_one_gpu():
                 p.kill()
     for r in range(2):
         assert r in out and out[r][0], out.get(r)
+
+
+def test_ddp_hook_two_processes_one_gpu():
+    _run(auto_register=False, steps=1)
+
+
+def test_ddp_hook_auto_register_zero_copy():
+    """auto_register: buckets are registered on first sight (and again after DDP's bucket rebuild)
+    and every step runs the zero-copy DIRECT plan; gradients stay the cross-rank average."""
+    _run(auto_register=True, steps=3)

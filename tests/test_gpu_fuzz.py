@@ -5,6 +5,8 @@ and piece sizes, every collective the
 loopback communicator offers; bit-exact against the oracle.  Seeded: a
 failure names its case and reproduces."""
 
+import os
+
 import numpy as np
 import pytest
 
@@ -108,7 +110,10 @@ def _eq(a, b):
     return np.array_equal(bits(a), bits(b))
 
 
-@pytest.mark.parametrize("seed", range(300))
+FUZZ_CASES = int(os.environ.get("ADAPCC_FUZZ_CASES", "1000"))  # widen the sweep for one-off soak runs
+
+
+@pytest.mark.parametrize("seed", range(FUZZ_CASES))
 def test_fuzz(seed):
     _run(_case(seed))
 

@@ -1,7 +1,9 @@
 """Randomised parity sweep of the multi-process paths (-m gpu): 3 processes on
 one GPU (CUDA IPC, gloo bootstrap), the seeded cases of test_gpu_fuzz.py with
-n = 3, each run through the STAGED protocol and through the zero-copy DIRECT
-plan on registered buffers; every process checks its own output bit-exactly."""
+n = 3 (kernels, LDG schedules, PDL and piece sizes included), each run through
+the STAGED protocol and through the zero-copy DIRECT plan on registered
+buffers; every process checks its own output bit-exactly.
+ADAPCC_IPC_FUZZ_CASES sets the number of cases (default 240)."""
 
 import os
 import socket
@@ -14,7 +16,8 @@ torch = pytest.importorskip("torch")
 
 pytestmark = pytest.mark.gpu
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-N, CASES = 3, 120
+N = 3
+CASES = int(os.environ.get("ADAPCC_IPC_FUZZ_CASES", "240"))
 
 
 def _free_port():
@@ -67,6 +70,8 @@ def _worker(rank, port, q):
                 exp = oc.reducescatter(xs, text, R, dtype, y_prev=prev)[rank]
             comm.set_strategy(coll, text)
             comm.config("engine", c["engine"])
+            for k in ("sched", "pdl", "piece_kib"):  # same seeded launch knobs on every rank
+                comm.config(k, c[k])
             for path in ("staged", "zc"):
                 if path == "staged":
                     x = to_dev(xs[rank], dtype)
