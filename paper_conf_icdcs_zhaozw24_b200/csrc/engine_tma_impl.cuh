@@ -53,6 +53,10 @@ constexpr int kQ = 2;           // item queue depth
 #endif
 constexpr bool kFoldTma = ADAPCC_FOLD_TMA != 0;
 constexpr int kMaxPost = 4;
+// ACCUMULATE (phase 2, recv += result) with every tile in shared memory: the
+// producer also loads each accumulating destination's tile, so a stage holds
+// nsrc + nacc tiles of at least 512 B (acc_tma in the item descriptor)
+constexpr int kMaxAccTiles = 24;
 
 struct ItemDesc {
   const char* src[kMaxFold];
@@ -65,6 +69,8 @@ struct ItemDesc {
   uint16_t nsrc, ndst, op, npost, passes, ks;
   uint8_t acc[kMaxDst];
   uint8_t stop, dropped, scalar_only, any_acc;
+  uint8_t acc_tma;            // accumulating destinations are loaded by TMA and stored from the stage
+  uint8_t acc_slot[kMaxDst];  // acc_tma: stage tile of destination k's recv (0 = plain destination)
   uint32_t item;        // trace: item index, claim and inputs-ready times
   uint64_t tr0, tr1;
 };
@@ -275,6 +281,65 @@ __device__ __forceinline__ void copy_tma(Smem& sm, char* stages, const ItemDesc&
   }
 }
 
+// ACCUMULATE items (acc_tma): a stage holds the K source tiles and, after
+// them, the current tile of every accumulating destination.  The consumers
+// fold the sources (one rounding), write the result over source 0's tile when
+// a plain destination needs it, and add it into each recv tile in place (one
+// more rounding, as store_result does); one thread then bulk-stores every
+// destination's tile.  No consumer global load or store is left.
+template <int DT>
+__device__ __forceinline__ void consume_acc_tma(Smem& sm, char* stages, const ItemDesc& d, int tid,
+                                                uint32_t& stage, uint32_t& sphase) {
+  using O = Ops<DT>;
+  const uint32_t tile = d.tile;
+  const int ks = d.nsrc, ndst = d.ndst;
+  bool plain = false;
+  for (int k = 0; k < ndst; ++k) plain |= !d.acc[k];
+  int prev = -1;  // tid 0: the stage whose bulk stores may still be reading it
+  for (uint32_t t = 0; t < d.ntiles; ++t) {
+    const uint32_t tb = min(tile, d.vec_bytes - t * tile);
+    const uint32_t nv = tb / 16;
+    mbar_wait(&sm.full[stage], sphase);
+    char* sb = stages + (size_t)stage * kStageBytes;
+    for (uint32_t v = tid; v < nv; v += kConsumers) {
+      char* pv = sb + (size_t)v * 16;
+      uint4 r;
+      if (ks == 1) {
+        r = lds16(pv);
+      } else {
+        typename O::Acc a = O::widen(lds16(pv));
+        for (int k = 1; k < ks; ++k) O::add(a, lds16(pv + (size_t)k * tile));
+        r = O::narrow(a);
+        if (plain) sts16(pv, r);
+      }
+      for (int k = 0; k < ndst; ++k) {
+        if (!d.acc[k]) continue;
+        char* q = pv + (size_t)d.acc_slot[k] * tile;
+        typename O::Acc b = O::widen(lds16(q));
+        O::add(b, r);
+        sts16(q, O::narrow(b));
+      }
+    }
+    fence_proxy_async_smem();
+    consumer_sync();  // every tile of this stage is final in shared memory
+    if (tid == 0) {
+      for (int k = 0; k < ndst; ++k)
+        tma_store(d.dst[k] + (size_t)t * tile, sb + (size_t)(d.acc[k] ? d.acc_slot[k] : 0) * tile, tb);
+      tma_store_commit();
+      if (prev >= 0) {
+        tma_store_wait_read<1>();
+        mbar_arrive_cnt(&sm.empty[prev], kConsumerWarps);
+      }
+      prev = (int)stage;
+    }
+    if (++stage == kStages) { stage = 0; sphase ^= 1; }
+  }
+  if (tid == 0 && prev >= 0) {
+    tma_store_wait_read<0>();
+    mbar_arrive_cnt(&sm.empty[prev], kConsumerWarps);
+  }
+}
+
 // Fold the tiles of a K >= 2 item whose destinations are all plain stores
 // (no accumulation) and whose sources fit one stage: the consumers fold each
 // vector in shared memory, in place over source 0's tile, and one thread
@@ -441,6 +506,23 @@ __device__ __forceinline__ void fill_desc(const LaunchParams& P, char* const (*b
     uint32_t tile = kStageBytes / (uint32_t)ks / 4096u * 4096u;
     d.tile = tile;
     d.ntiles = d.vec_bytes ? (d.vec_bytes + tile - 1) / tile : 0;
+    // Phase 2 (ACCUMULATE): recv += result used to be a load, add and store
+    // per destination per vector, one memory latency after another; with the
+    // recv tiles brought in by TMA next to the sources, the read-modify-write
+    // happens in shared memory and leaves by bulk stores.
+    int nacc = 0;
+    for (int k = 0; k < t.ndst; ++k) nacc += d.acc[k] ? 1 : 0;
+    d.acc_tma = kFoldTma && nacc > 0 && !d.scalar_only && nsrc >= 1 && nsrc <= kMaxKS &&
+                nsrc + nacc <= kMaxAccTiles;
+    if (d.acc_tma) {
+      int j = 0;
+      for (int k = 0; k < t.ndst; ++k) d.acc_slot[k] = d.acc[k] ? (uint8_t)(nsrc + j++) : (uint8_t)0;
+      const uint32_t at = kStageBytes / (uint32_t)(nsrc + nacc) / 512u * 512u;
+      d.ks = (uint16_t)nsrc;
+      d.passes = 1;
+      d.tile = at;
+      d.ntiles = (d.vec_bytes + at - 1) / at;
+    }
   }
 }
 
@@ -584,12 +666,20 @@ __global__ void __launch_bounds__(kTmaThreads, ADAPCC_TMA_MINB) engine_tma_kerne
           for (int p = 0; p < d.passes; ++p) {
             if (lane == 0) {
               const int ks = min((int)d.ks, (int)d.nsrc - p * (int)d.ks);
+              int nacc = 0;
+              if (d.acc_tma)
+                for (int k = 0; k < d.ndst; ++k) nacc += d.acc[k] ? 1 : 0;
               mbar_wait(&sm.empty[stage], sphase ^ 1);
-              mbar_expect_tx(&sm.full[stage], (uint32_t)ks * tb);
+              mbar_expect_tx(&sm.full[stage], (uint32_t)(ks + nacc) * tb);
               char* sb = stages + (size_t)stage * kStageBytes;
               for (int j = 0; j < ks; ++j)
                 tma_load(sb + (size_t)j * d.tile, d.src[p * d.ks + j] + (size_t)tt * d.tile, tb,
                          &sm.full[stage]);
+              if (d.acc_tma)  // the accumulating destinations' current recv tiles
+                for (int k = 0; k < d.ndst; ++k)
+                  if (d.acc[k])
+                    tma_load(sb + (size_t)d.acc_slot[k] * d.tile, d.dst[k] + (size_t)tt * d.tile, tb,
+                             &sm.full[stage]);
             }
             if (++stage == kStages) { stage = 0; sphase ^= 1; }
           }
@@ -612,7 +702,8 @@ __global__ void __launch_bounds__(kTmaThreads, ADAPCC_TMA_MINB) engine_tma_kerne
         } else {
           if (!d.scalar_only) {
             const uint32_t vpt = d.tile / (16u * kConsumers);  // tile / one round of 1 vector per thread
-            if (d.nsrc == 1 && !d.any_acc) copy_tma(sm, stages, d, tid, stage, sphase);
+            if (d.acc_tma) consume_acc_tma<DT>(sm, stages, d, tid, stage, sphase);
+            else if (d.nsrc == 1 && !d.any_acc) copy_tma(sm, stages, d, tid, stage, sphase);
             // TMA-stored fold where per-thread stores are the cost: tiles above 16 KiB (K = 2, 3 in
             // 64 KiB stages, else fold_rounds; G1 k = 2: 0.86 -> 1.02 of the copy peak) or >= 3
             // destinations (star roots); with 1-2 destinations of small tiles the register path,

@@ -215,6 +215,50 @@ def main():
                                             "lags": lags,
                                             "rel_err_vs_full_sum": float(np.max(np.abs(got - full)) /
                                                                          np.max(np.abs(full)))}
+            # Per-piece late join (NEXT-1) on the DIRECT plan: phase 1 starts at t = 0 with the
+            # stragglers as late candidates; their compute stream signals them ready after the lag, so
+            # every piece claimed after that folds them in; phase 2 (LATE_COMPLEMENT) adds them only to
+            # the pieces that had already passed.  T_wait uses the DIRECT plan's own T_full.
+            dcomm = pkg.Communicator.loopback(n, mode="direct", scratch_bytes=64 << 20)
+            dcomm.set_strategy("allreduce", G.allreduce_stars(n))
+            t_full_d = timeit(lambda: dcomm.allreduce_lb(dx, dy), iters=10)
+            for _ in range(2):  # warm the LATE_JOIN plan (phase 2 runs on the same plan)
+                dcomm.allreduce_lb(dx, dy, ready=R1, late="join")
+                dcomm.allreduce_lb(dx, dy, ready=R1, late="complement")
+            torch.cuda.synchronize()
+            lags = {}
+            for f in (0.0, 0.25, 0.5, 1.0, 2.0):
+                ts = f * t_full_d
+                torch.cuda.synchronize()
+                a0 = torch.cuda.Event(enable_timing=True)
+                a1 = torch.cuda.Event(enable_timing=True)
+                ready_ev = torch.cuda.Event()
+                ticket = dcomm.late_ticket() + 1
+                a0.record(s_comm)
+                s_comp.wait_event(a0)
+                with torch.cuda.stream(s_comp):
+                    if ts > 0:
+                        torch.cuda._sleep(int(ts * cyc_per_ms))
+                    for r in sorted(R2):
+                        dcomm.signal_ready(rank=r, ticket=ticket, stream=s_comp)
+                    ready_ev.record(s_comp)
+                with torch.cuda.stream(s_comm):
+                    dcomm.allreduce_lb(dx, dy, ready=R1, late="join")
+                    s_comm.wait_event(ready_ev)
+                    dcomm.allreduce_lb(dx, dy, ready=R1, late="complement")
+                    a1.record(s_comm)
+                torch.cuda.synchronize()
+                t_adapcc = a0.elapsed_time(a1)
+                t_wait = ts + t_full_d
+                lags[str(f)] = {"t_s_ms": round(ts, 4), "T_adapcc_ms": round(t_adapcc, 4),
+                                "T_wait_ms": round(t_wait, 4), "speedup": round(t_wait / t_adapcc, 3)}
+            assert dcomm.get_async_error() == 0
+            full = oc.allreduce_exact([x[:4096] for x in xs], set(range(n)), "f32")
+            got = dy[0][:4096].cpu().numpy().astype(np.float64)
+            point["variants"]["late join per piece (DIRECT, NEXT-1)"] = {
+                "T_full_direct_ms": round(t_full_d, 4), "lags": lags,
+                "rel_err_vs_full_sum": float(np.max(np.abs(got - full)) / np.max(np.abs(full)))}
+            dcomm.finalize()
             res.append(point)
             print("C3", json.dumps(point)[:400], flush=True)
             del dx, dy
