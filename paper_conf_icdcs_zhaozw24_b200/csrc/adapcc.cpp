@@ -42,6 +42,8 @@ struct DevSegment {
   Item* items = nullptr;
   uint32_t nitems = 0;
   uint64_t* late_bits = nullptr;  // per item: late ranks folded in phase 1 (late join)
+  uint32_t* late_list = nullptr;  // 2 x nitems: items phase 1 left incomplete (per ticket parity)
+  uint32_t* late_count = nullptr; // 2 counts
   uint4* first = nullptr;         // LDG kernel: per-CTA first-item blobs (launch.hpp)
   uint32_t nfirst = 0, first_words = 0;
   uint32_t sched_static = 0;      // LDG kernel: every item has a blob, CTA b runs b, b + grid, ...
@@ -67,6 +69,8 @@ struct DevPlan {
       cudaFree(s.flags);
       cudaFree(s.items);
       cudaFree(s.late_bits);
+      cudaFree(s.late_list);
+      cudaFree(s.late_count);
       cudaFree(s.first);
     }
     cudaGetLastError();  // teardown errors must not leak into a later call's check
@@ -421,7 +425,8 @@ adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, const Strategy* strat, uin
       };
       uint32_t all_words = 0;
       for (uint32_t i = 0; i < d.nitems; ++i) all_words = std::max(all_words, words_of(i));
-      const bool stat = plan->kernel == 0 && c->sched != 0 && d.nitems > 0 && all_words <= (uint32_t)kFirstMaxWords &&
+      // (late-join plans claim dynamically: phase 2 runs phase 1's list of incomplete items)
+      const bool stat = plan->kernel == 0 && c->sched != 0 && !rq.late_join && d.nitems > 0 && all_words <= (uint32_t)kFirstMaxWords &&
                         (uint64_t)d.nitems * all_words * 16 <= kMaxBlobBytes;
       const uint32_t nf = stat ? d.nitems : std::min<uint32_t>(d.nitems, (uint32_t)grid_size(c, dtype, plan->kernel));
       uint32_t words = 0;
@@ -444,6 +449,9 @@ adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, const Strategy* strat, uin
     if (rq.late_join) {
       CK(cudaMalloc(&d.late_bits, std::max<size_t>(1, items.size()) * sizeof(uint64_t)));
       CK(cudaMemset(d.late_bits, 0, std::max<size_t>(1, items.size()) * sizeof(uint64_t)));
+      CK(cudaMalloc(&d.late_list, 2 * std::max<size_t>(1, items.size()) * sizeof(uint32_t)));
+      CK(cudaMalloc(&d.late_count, 2 * sizeof(uint32_t)));
+      CK(cudaMemset(d.late_count, 0, 2 * sizeof(uint32_t)));
     }
     plan->segs.push_back(d);
   }
@@ -516,6 +524,8 @@ adapcc_result_t run(adapcc_comm_s* c, Coll coll, const void* const* send, void* 
     P.late_mode = late_mode;
     P.late_ticket = c->late_seq;
     P.late_bits = seg.late_bits;
+    P.late_list = seg.late_list;
+    P.late_count = seg.late_count;
     P.drop_rank = (int)c->drop_rank;
     P.members = c->members;
     P.half_bytes = c->half_bytes;

@@ -64,6 +64,8 @@ struct Shared {
   uint8_t acc[kMaxDst];
   uint64_t epoch;
   uint32_t item;
+  uint32_t claim;              // claim index of `item` (= item, or its position in the phase-2 list)
+  uint32_t nclaim;             // claimable indices (nitems, or the phase-2 list length)
   int bad_align;
   int abort;
   int any_acc;
@@ -318,7 +320,10 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
   if (threadIdx.x == 0) sh.abort = 0;
   if (prestage) {
     __syncthreads();  // blob words and buffer bases
-    if (threadIdx.x == 0) stage(blockIdx.x, true, 0, true);
+    if (threadIdx.x == 0) {
+      sh.claim = blockIdx.x;
+      stage(blockIdx.x, true, 0, true);
+    }
     __syncthreads();
     if (sh.item < P.nitems && !sh.cur.dropped) my_arena = resolve(0);
   }
@@ -326,6 +331,12 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
   // buffers below belong to the stream order (PDL: the previous launch)
   pdl_trigger();
   pdl_wait();
+  if (threadIdx.x == 0) {
+    sh.nclaim = (P.late_mode == 2 && P.late_list && !stat)
+                    ? *reinterpret_cast<volatile uint32_t*>(&P.late_count[P.late_ticket & 1]) : P.nitems;
+    // phase 1: empty the other ticket parity's list for the next phase 1
+    if (P.late_mode == 1 && blockIdx.x == 0) P.late_count[(P.late_ticket + 1) & 1] = 0;
+  }
   // Lazy epoch: a loopback plan without arena streams or flags whose CTAs
   // need no claim counter only uses the epoch to count itself done at the
   // end, so its load stays in flight during the fold instead of costing a
@@ -373,19 +384,26 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
   // items are all taken and no CTA pays a final failed atomic (small calls run
   // with no claim atomics at all).
   bool first = true, last = false, staged = prestage;
+  // Phase 2 of a late join claims positions in phase 1's list of incomplete
+  // items (no waits in phase 2, so any order is deadlock-free)
+  const bool listed = P.late_mode == 2 && P.late_list != nullptr && !stat;
   while (!sh.abort && !last) {
     if (!staged) {
       if (threadIdx.x == 0) {
-        const uint32_t it = first ? blockIdx.x : stat ? sh.item + gridDim.x
-                                                      : gridDim.x + atomicAdd(&P.state->work[par], 1u);
-        const bool fb = stat || (first && use_blob);
-        stage(it, fb, buf, first);
+        const uint32_t k = first ? blockIdx.x : stat ? sh.item + gridDim.x
+                                                     : gridDim.x + atomicAdd(&P.state->work[par], 1u);
+        sh.claim = k;
+        uint32_t it = k;
+        if (listed) it = k < sh.nclaim ? P.late_list[(size_t)(P.late_ticket & 1) * P.nitems + k] : P.nitems;
+        // (a listed phase-2 item is not the CTA's first item: no blob, no preloaded item)
+        const bool fb = stat || (first && use_blob && !listed);
+        stage(it, fb, buf, first && !listed);
       }
       __syncthreads();
     }
     if (sh.item >= P.nitems) break;
     first = false;
-    last = (uint64_t)sh.item + gridDim.x >= P.nitems;
+    last = (uint64_t)sh.claim + gridDim.x >= (listed ? sh.nclaim : P.nitems);
     // static schedule: fetch the next item's blob into the other buffer while
     // this item folds (its last readers finished before the barrier above)
     if (stat && !last && threadIdx.x < P.first_words)
@@ -457,6 +475,9 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
     if (done == gridDim.x - 1) {
       // last CTA: publish the epoch for the next launch on this stream and,
       // across processes, "this rank finished epoch" to the peers
+      // phase 2 consumed its list (every CTA is past its claims): empty it, so
+      // a replayed phase 1 with the same ticket starts a fresh one
+      if (P.late_mode == 2 && P.late_count) P.late_count[P.late_ticket & 1] = 0;
       *reinterpret_cast<volatile unsigned long long*>(&P.state->epoch) = ep;
       if (P.ipc) {
         __threadfence_system();

@@ -200,6 +200,11 @@ static __device__ __forceinline__ uint64_t late_select(const LaunchParams& P, co
         m |= 1ull << j;
     }
     P.late_bits[item] = m;
+    const uint64_t all = t.nlate >= 64 ? ~0ull : ((1ull << t.nlate) - 1);
+    if (all & ~m) {  // phase 2 has something to add here
+      const unsigned par = (unsigned)(P.late_ticket & 1);
+      P.late_list[(size_t)par * P.nitems + atomicAdd(&P.late_count[par], 1u)] = item;
+    }
   } else if (P.late_mode == 2) {
     const uint64_t all = t.nlate >= 64 ? ~0ull : ((1ull << t.nlate) - 1);
     m = all & ~P.late_bits[item];

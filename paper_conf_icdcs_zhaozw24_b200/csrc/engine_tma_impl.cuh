@@ -582,6 +582,8 @@ __global__ void __launch_bounds__(kTmaThreads, ADAPCC_TMA_MINB) engine_tma_kerne
     if (blockIdx.x == 0) {
       P.state->work[(e + 1) & 1] = 0;
       P.state->done[(e + 1) & 1] = 0;
+      // phase 1: empty the other ticket parity's list for the next phase 1
+      if (P.late_mode == 1) P.late_count[(P.late_ticket + 1) & 1] = 0;
     }
   }
   __syncthreads();
@@ -609,23 +611,34 @@ __global__ void __launch_bounds__(kTmaThreads, ADAPCC_TMA_MINB) engine_tma_kerne
     // claiming as in the LDG kernel: item blockIdx.x first, then the counter
     // offset by the grid; stop after an item among the last gridDim.x
     bool first = true, last = false;
+    // Phase 2 of a late join (LATE_COMPLEMENT) has work only in the items
+    // phase 1 listed as incomplete: claims index that list (no waits in phase
+    // 2, so any order is deadlock-free) and everything else is never touched.
+    const bool listed = P.late_mode == 2 && P.late_list != nullptr;
+    const uint32_t nclaim = listed ? *reinterpret_cast<volatile uint32_t*>(&P.late_count[P.late_ticket & 1])
+                                   : P.nitems;
     for (;;) {
       uint32_t it = 0;
       int stop_i = 0;
-      if (lane == 0 && !last) it = first ? blockIdx.x : gridDim.x + atomicAdd(&P.state->work[par], 1u);
+      if (lane == 0 && !last) {
+        it = first ? blockIdx.x : gridDim.x + atomicAdd(&P.state->work[par], 1u);
+        last = (uint64_t)it + gridDim.x >= nclaim;
+        if (listed) it = it < nclaim ? P.late_list[(size_t)(P.late_ticket & 1) * P.nitems + it] : P.nitems;
+      } else if (lane == 0) {
+        it = P.nitems;
+      }
       const uint64_t tr0 = P.trace ? globaltimer() : 0;
       // queue slot free: every lane waits (acquire), since every lane rewrites
       // the slot's descriptor that the consumers of item i - kQ were reading
       mbar_wait(&sm.qempty[qi], qphase ^ 1);
       if (lane == 0) {
-        stop_i = last || it >= P.nitems || *reinterpret_cast<volatile int*>(&sm.abort) != 0;
+        stop_i = it >= P.nitems || *reinterpret_cast<volatile int*>(&sm.abort) != 0;
         first = false;
-        last = last || (uint64_t)it + gridDim.x >= P.nitems;
       }
       it = __shfl_sync(0xffffffffu, it, 0);
       bool stop = __shfl_sync(0xffffffffu, stop_i, 0) != 0;
       ItemDesc& d = sm.q[qi];
-      const bool fb = use_blob && it == blockIdx.x;  // this CTA's first item (blob in shared memory)
+      const bool fb = use_blob && !listed && it == blockIdx.x;  // this CTA's first item (blob in shared memory)
       const Item item = stop ? Item{} : fb ? *reinterpret_cast<const Item*>(&sm.blob[0]) : P.items[it];
       const Task& t = fb ? *reinterpret_cast<const Task*>(&sm.blob[1]) : P.tasks[item.task];
       if (!stop) {
@@ -747,6 +760,9 @@ __global__ void __launch_bounds__(kTmaThreads, ADAPCC_TMA_MINB) engine_tma_kerne
     }
     const unsigned done = atomicAdd(&P.state->done[par], 1u);
     if (done == gridDim.x - 1) {
+      // phase 2 consumed its list (every CTA is past its claims): empty it, so
+      // a replayed phase 1 with the same ticket starts a fresh one
+      if (P.late_mode == 2 && P.late_count) P.late_count[P.late_ticket & 1] = 0;
       *reinterpret_cast<volatile unsigned long long*>(&P.state->epoch) = epoch;
       if (P.ipc) {
         __threadfence_system();

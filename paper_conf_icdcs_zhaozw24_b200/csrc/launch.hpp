@@ -67,6 +67,11 @@ struct LaunchParams {
   int late_mode;        // 0: off; 1: late join (phase 1); 2: complement (phase 2)
   uint64_t late_ticket; // ready word value that admits a late rank (phase 1)
   uint64_t* late_bits;  // per work item: late candidates included in phase 1
+  // Phase 1 lists the items that missed a late rank (late_list[par * nitems +
+  // i], i < late_count[par], par = late_ticket & 1); phase 2 runs exactly those.
+  // Phase 1's block 0 clears the other parity's count for the next phase 1.
+  uint32_t* late_list;
+  uint32_t* late_count;
   int drop_rank;        // test hook (loopback): tasks owned by this rank are skipped
   uint64_t members;     // live ranks: excluded ranks are skipped by the IPC barriers
   uint64_t half_bytes;  // bytes of one parity half of an arena

@@ -39,7 +39,7 @@ def _comm(n, engine):
 
 @pytest.mark.parametrize("engine", [0, 1])
 @pytest.mark.parametrize("dtype", ["f32", "bf16", "i32"])
-@pytest.mark.parametrize("case", ["all", "none"])
+@pytest.mark.parametrize("case", ["all", "none", "one"])
 def test_late_join_deterministic(engine, dtype, case):
     n, count = 8, 200_003
     R, late = {0, 1, 2, 4, 5, 7}, [3, 6]
@@ -50,13 +50,14 @@ def test_late_join_deterministic(engine, dtype, case):
     comm.set_strategy("allreduce", text)
     dx = [to_dev(x, dtype) for x in xs]
     dy = [empty_dev(count, dtype) for _ in range(n)]
-    if case == "all":
+    if case in ("all", "one"):
         t = comm.late_ticket() + 1          # the ticket the next LATE_JOIN call will use
-        for r in late:
+        for r in (late if case == "all" else late[:1]):
             comm.signal_ready(r, ticket=t)
     comm.allreduce_lb(dx, dy, ready=R, late="join")
     torch.cuda.synchronize()
-    L = set(late) if case == "all" else set()
+    # "one": rank 3 joins every piece, rank 6 none -> phase 2 runs every root piece, adding only 6
+    L = set(late) if case == "all" else {late[0]} if case == "one" else set()
     e1 = oc.allreduce_late(xs, text, R, dtype, L, phase=1)
     assert all(np.array_equal(bits(to_host(y, dtype)), bits(e)) for y, e in zip(dy, e1))
     comm.allreduce_lb(dx, dy, ready=R, late="complement")
