@@ -533,9 +533,16 @@ std::vector<Item> order_items(const SegmentPlan& p, int rank, int esize, int gri
                               uint64_t piece_bytes, int taper, bool tma) {
   // Work balance: tasks that post no flags are cut into pieces of roughly
   // equal traffic.
+  // streams of a task: sources + destinations, an accumulating destination
+  // twice (recv is read and written)
+  auto streams_of = [&](const Task& T) {
+    uint64_t s = (uint64_t)T.nsrc + T.ndst;
+    for (uint32_t k = 0; k < T.ndst; ++k) s += p.refs[T.ref0 + T.nsrc + k].accum ? 1 : 0;
+    return std::max<uint64_t>(1, s);
+  };
   uint64_t total = 0;
   for (const Task& T : p.tasks)
-    if (rank < 0 || T.owner == rank) total += (T.hi - T.lo) * esize * (uint64_t)(T.nsrc + T.ndst);
+    if (rank < 0 || T.owner == rank) total += (T.hi - T.lo) * esize * streams_of(T);
   // Measured on B200 (profiles/sweep_r01.json, profiles/pieces_r01.json):
   // ~512 KiB of traffic per item (32 KiB per stream for a 16-stream fold) is
   // the sweet spot of large calls -- smaller items pay the per-item claim/sync
@@ -561,7 +568,7 @@ std::vector<Item> order_items(const SegmentPlan& p, int rank, int esize, int gri
   for (uint32_t t = 0; t < p.tasks.size(); ++t) {
     const Task& T = p.tasks[t];
     if (rank >= 0 && T.owner != rank) continue;
-    const uint64_t streams = std::max<uint64_t>(1, T.nsrc + T.ndst);
+    const uint64_t streams = streams_of(T);
     for (uint32_t c = 0; c < T.nchunks; ++c) {
       const uint64_t c0 = T.lo + (uint64_t)c * T.chunk_elems;
       const uint64_t clen = std::min<uint64_t>(T.hi, c0 + T.chunk_elems) - c0;
@@ -613,7 +620,7 @@ std::vector<Item> order_items(const SegmentPlan& p, int rank, int esize, int gri
     for (size_t i = keys.size(); i-- > 0 && want > 0;) {
       const Task& T = p.tasks[keys[i].task];
       if (T.npost != 0 || keys[i].len < (uint64_t)taper * align) continue;
-      if (auto_taper && (uint64_t)keys[i].len * esize * (T.nsrc + T.ndst) < (384u << 10)) continue;
+      if (auto_taper && (uint64_t)keys[i].len * esize * streams_of(T) < (384u << 10)) continue;
       split[i] = 1;
       --want;
     }
