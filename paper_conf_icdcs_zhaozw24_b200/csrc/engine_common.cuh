@@ -212,6 +212,36 @@ static __device__ __forceinline__ uint64_t late_select(const LaunchParams& P, co
   return m;
 }
 
+// late_select for a whole warp (the TMA kernel's producer): lane j checks
+// candidate j (and j + 32, ...), so the ref and ready-word loads of all
+// candidates are in flight together instead of one candidate after another.
+// Same result and side effects as late_select; every lane returns the mask.
+static __device__ __forceinline__ uint64_t late_select_warp(const LaunchParams& P, const Task& t,
+                                                            uint32_t item, int lane) {
+  const uint64_t all = t.nlate >= 64 ? ~0ull : ((1ull << t.nlate) - 1);
+  if (P.late_mode == 2) return all & ~P.late_bits[item];
+  if (P.late_mode != 1) return 0;
+  uint64_t m = 0;
+  for (int j0 = 0; j0 < t.nlate; j0 += 32) {
+    const int j = j0 + lane;
+    bool ok = false;
+    if (j < t.nlate) {
+      const BufRef r = P.refs[t.ref0 + t.nsrc + t.ndst + j];
+      ok = ld_acquire(reinterpret_cast<const uint64_t*>(P.hdr[r.rank] + ArenaHeader::kReady), P.ipc) >=
+           P.late_ticket;
+    }
+    m |= (uint64_t)__ballot_sync(0xffffffffu, ok) << j0;
+  }
+  if (lane == 0) {
+    P.late_bits[item] = m;
+    if (all & ~m) {  // phase 2 has something to add here
+      const unsigned par = (unsigned)(P.late_ticket & 1);
+      P.late_list[(size_t)par * P.nitems + atomicAdd(&P.late_count[par], 1u)] = item;
+    }
+  }
+  return m;
+}
+
 // index (into the task's late refs) of the k-th set bit of m
 static __device__ __forceinline__ int nth_bit(uint64_t m, int k) {
   for (int j = 0; j < 64; ++j)

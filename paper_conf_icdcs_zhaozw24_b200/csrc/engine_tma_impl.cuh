@@ -453,8 +453,7 @@ __device__ __forceinline__ void fill_desc(const LaunchParams& P, char* const (*b
     if (t.nlate == 0) {
       dropped = P.late_mode == 2;  // phase 2 only runs the roots' folds
     } else {
-      if (lane == 0) late = late_select(P, t, it);
-      late = __shfl_sync(0xffffffffu, late, 0);
+      late = late_select_warp(P, t, it, lane);
       if (P.late_mode == 2) {
         nreg = 0;
         *nwait_eff = 0;
