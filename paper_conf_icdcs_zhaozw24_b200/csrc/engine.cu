@@ -317,7 +317,10 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
   // Late join decides per item from ready words, so it stages after the wait.
   const bool prestage = use_blob && P.late_mode == 0;
   bool my_arena = false;
-  if (threadIdx.x == 0) sh.abort = 0;
+  if (threadIdx.x == 0) {
+    sh.abort = 0;
+    sh.nclaim = P.nitems;  // (phase 2 of a late join: its list length, set after the wait)
+  }
   if (prestage) {
     __syncthreads();  // blob words and buffer bases
     if (threadIdx.x == 0) {
@@ -331,12 +334,6 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
   // buffers below belong to the stream order (PDL: the previous launch)
   pdl_trigger();
   pdl_wait();
-  if (threadIdx.x == 0) {
-    sh.nclaim = (P.late_mode == 2 && P.late_list && !stat)
-                    ? *reinterpret_cast<volatile uint32_t*>(&P.late_count[P.late_ticket & 1]) : P.nitems;
-    // phase 1: empty the other ticket parity's list for the next phase 1
-    if (P.late_mode == 1 && blockIdx.x == 0) P.late_count[(P.late_ticket + 1) & 1] = 0;
-  }
   // Lazy epoch: a loopback plan without arena streams or flags whose CTAs
   // need no claim counter only uses the epoch to count itself done at the
   // end, so its load stays in flight during the fold instead of costing a
@@ -347,6 +344,11 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
     if (threadIdx.x == 0) e_lazy = *reinterpret_cast<volatile unsigned long long*>(&P.state->epoch) + 1;
   } else {
     if (threadIdx.x == 0) {
+      // late join (never lazy): phase 2 claims positions in phase 1's list;
+      // phase 1 empties the other ticket parity's list for the next phase 1
+      if (P.late_mode == 2 && P.late_list && !stat)
+        sh.nclaim = *reinterpret_cast<volatile uint32_t*>(&P.late_count[P.late_ticket & 1]);
+      if (P.late_mode == 1 && blockIdx.x == 0) P.late_count[(P.late_ticket + 1) & 1] = 0;
       // this launch's epoch = the one the previous launch published + 1
       const uint64_t e = *reinterpret_cast<volatile unsigned long long*>(&P.state->epoch) + 1;
       sh.epoch = e;
