@@ -108,3 +108,40 @@ def test_late_join_racing_signal(engine, dtype):
     if dtype == "i32":
         assert np.array_equal(y2[0], oc.allreduce_exact(xs, set(range(n)), "i32"))
     comm.finalize()
+
+
+@pytest.mark.parametrize("engine", [0, 1])
+def test_late_join_graph_replay(engine):
+    """Phase 1 + phase 2 captured in one CUDA graph (the ticket is baked in) and replayed: every replay
+    rebuilds phase 1's list of incomplete pieces from scratch (phase 2 empties its list when it ends),
+    so rank 6 is added exactly once per replay (int32, exact) while rank 3 joins every piece."""
+    n, count = 8, 300_007
+    R, late = {0, 1, 2, 4, 5, 7}, [3, 6]
+    text = G.allreduce_stars(n, chunk=65536)
+    xs = rank_tensors("i32", count, n)
+    comm = _comm(n, engine)
+    comm.set_strategy("allreduce", text)
+    dx = [to_dev(x, "i32") for x in xs]
+    dy = [empty_dev(count, "i32") for _ in range(n)]
+    s = torch.cuda.Stream()
+    s.wait_stream(torch.cuda.current_stream())
+    with torch.cuda.stream(s):
+        comm.allreduce_lb(dx, dy, ready=R, late="join")       # plan built outside the capture
+        comm.allreduce_lb(dx, dy, ready=R, late="complement")
+        torch.cuda.synchronize()
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g, stream=s):
+            t = comm.late_ticket() + 1
+            comm.signal_ready(late[0], ticket=t, stream=s)
+            comm.allreduce_lb(dx, dy, ready=R, late="join", stream=s)
+            comm.allreduce_lb(dx, dy, ready=R, late="complement", stream=s)
+    full = oc.allreduce(xs, text, set(range(n)), "i32")
+    for _ in range(3):
+        for y in dy:
+            y.zero_()
+        g.replay()
+        torch.cuda.synchronize()
+        assert comm.get_async_error() == 0
+        for y, e in zip(dy, full):
+            assert np.array_equal(bits(to_host(y, "i32")), bits(e))
+    comm.finalize()
