@@ -1,2 +1,1 @@
-timeout 600 python -m pytest tests/test_gpu_late_join.py -x -q -p no:cacheprovider -k graph 2>&1 | tail -15
-timeout 1800 python -m pytest tests -m gpu -x -q -p no:cacheprovider > gpurun_out/t_all.log 2>&1; tail -2 gpurun_out/t_all.log
+ncu --set full --clock-control none -k regex:engine -s 2 -c 1 -o gpurun_out/prof_acc16 python scripts/debug/acc_one.py > gpurun_out/ncu_acc.log 2>&1; tail -2 gpurun_out/ncu_acc.log
