@@ -1,1 +1,3 @@
-ncu --set full --clock-control none -k regex:engine -s 2 -c 1 -o gpurun_out/prof_acc16 python scripts/debug/acc_one.py > gpurun_out/ncu_acc.log 2>&1; tail -2 gpurun_out/ncu_acc.log
+python scripts/debug/acc_engines.py 2>&1 | tail -4
+python scripts/debug/late_timing.py 2>&1 | tail -1
+timeout 900 python -m pytest tests/test_gpu_late_join.py tests/test_gpu_fuzz.py tests/test_gpu_loopback.py tests/test_gpu_primitives.py -x -q -p no:cacheprovider 2>&1 | tail -2
