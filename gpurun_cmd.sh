@@ -1,3 +1,3 @@
-python scripts/debug/acc_engines.py 2>&1 | tail -4
-python scripts/debug/late_timing.py 2>&1 | tail -1
-timeout 900 python -m pytest tests/test_gpu_late_join.py tests/test_gpu_fuzz.py tests/test_gpu_loopback.py tests/test_gpu_primitives.py -x -q -p no:cacheprovider 2>&1 | tail -2
+bash scripts/profile.sh r01 > gpurun_out/profile_run.log 2>&1
+python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/smoke.log 2>&1
+tail -1 gpurun_out/bench_r01.json | cut -c1-160; cat gpurun_out/smoke.log
