@@ -389,7 +389,11 @@ adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, const Strategy* strat, uin
     for (auto& sp : segs) accumulate_stats(sp, c->loopback ? -1 : c->rank, rq.esize, &st);
     const uint64_t traffic = st.bytes_read + st.bytes_written;
     plan->engine = c->engine != 2 ? c->engine : (traffic / std::max<size_t>(1, segs.size()) >= kTmaMinTraffic ? 1 : 0);
-    plan->kernel = plan->engine == 0 ? 0 : (mode == kDirect ? 1 : 2);
+    // ACCUMULATE (phase 2) stages nsrc + nacc tiles per ring slot and is
+    // latency-bound: the 2 CTAs/SM x 3 x 32 KiB shape of the STAGED
+    // instantiation beats 1 x 3 x 64 KiB on DIRECT plans too
+    // (profiles/acc_variants_r01.json: 256 MiB/rank 868 -> 801 us).
+    plan->kernel = plan->engine == 0 ? 0 : (mode == kDirect && !rq.accumulate ? 1 : 2);
   }
   for (auto& sp : segs) {
     DevSegment d;

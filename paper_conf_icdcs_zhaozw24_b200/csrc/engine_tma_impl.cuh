@@ -676,22 +676,26 @@ __global__ void __launch_bounds__(kTmaThreads, ADAPCC_TMA_MINB) engine_tma_kerne
         for (uint32_t tt = 0; tt < d.ntiles; ++tt) {
           const uint32_t tb = min(d.tile, d.vec_bytes - tt * d.tile);
           for (int p = 0; p < d.passes; ++p) {
+            const int ks = min((int)d.ks, (int)d.nsrc - p * (int)d.ks);
             if (lane == 0) {
-              const int ks = min((int)d.ks, (int)d.nsrc - p * (int)d.ks);
               int nacc = 0;
               if (d.acc_tma)
                 for (int k = 0; k < d.ndst; ++k) nacc += d.acc[k] ? 1 : 0;
               mbar_wait(&sm.empty[stage], sphase ^ 1);
               mbar_expect_tx(&sm.full[stage], (uint32_t)(ks + nacc) * tb);
-              char* sb = stages + (size_t)stage * kStageBytes;
-              for (int j = 0; j < ks; ++j)
-                tma_load(sb + (size_t)j * d.tile, d.src[p * d.ks + j] + (size_t)tt * d.tile, tb,
-                         &sm.full[stage]);
-              if (d.acc_tma)  // the accumulating destinations' current recv tiles
-                for (int k = 0; k < d.ndst; ++k)
-                  if (d.acc[k])
-                    tma_load(sb + (size_t)d.acc_slot[k] * d.tile, d.dst[k] + (size_t)tt * d.tile, tb,
-                             &sm.full[stage]);
+            }
+            __syncwarp();
+            // One bulk load per lane: a stage's K source tiles (and, with
+            // acc_tma, the accumulating destinations' recv tiles) are issued
+            // warp-parallel instead of one after another from lane 0.
+            char* sb = stages + (size_t)stage * kStageBytes;
+            if (lane < ks) {
+              tma_load(sb + (size_t)lane * d.tile, d.src[p * d.ks + lane] + (size_t)tt * d.tile, tb,
+                       &sm.full[stage]);
+            } else if (d.acc_tma) {
+              for (int k = 0; k < d.ndst; ++k)
+                if (d.acc[k] && d.acc_slot[k] == lane)
+                  tma_load(sb + (size_t)lane * d.tile, d.dst[k] + (size_t)tt * d.tile, tb, &sm.full[stage]);
             }
             if (++stage == kStages) { stage = 0; sphase ^= 1; }
           }
