@@ -166,6 +166,7 @@ struct adapcc_comm_s {
   int64_t taper = 0;      // tail items cut into this many sub-pieces (1 = off, 0 = auto)
   int64_t check_sig = 0;  // debug: kernels compare call signatures across ranks (ADAPCC_DEBUG)
   int64_t first_blob = 1; // LDG kernel: per-CTA first-item blobs (ADAPCC_FIRST_BLOB=0 disables)
+  int64_t tma_shape = 0;  // tuning: 0 = auto, 1 / 2 = force the 1 x 3 x 64 / 2 x 3 x 32 KiB TMA ring (ADAPCC_TMA_SHAPE)
   TraceRec* trace = nullptr;  // in-kernel trace buffer (adapcc_config("trace", capacity))
   unsigned* trace_n = nullptr;
   uint32_t trace_cap = 0;
@@ -216,6 +217,7 @@ adapcc_result_t common_init(adapcc_comm_s* c, size_t scratch) {
   c->taper = std::min<int64_t>(64, std::max<int64_t>(0, env_int("ADAPCC_TAPER", 0)));
   c->check_sig = env_int("ADAPCC_DEBUG", 0) != 0;
   c->first_blob = env_int("ADAPCC_FIRST_BLOB", 1) != 0;
+  c->tma_shape = env_int("ADAPCC_TMA_SHAPE", 0);
   c->pdl = env_int("ADAPCC_PDL", 1) != 0;
   c->sched = std::min<int64_t>(2, std::max<int64_t>(0, env_int("ADAPCC_SCHED", 2)));
   CK(cudaSetDevice(c->device));
@@ -394,6 +396,7 @@ adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, const Strategy* strat, uin
     // instantiation beats 1 x 3 x 64 KiB on DIRECT plans too
     // (profiles/acc_variants_r01.json: 256 MiB/rank 868 -> 801 us).
     plan->kernel = plan->engine == 0 ? 0 : (mode == kDirect && !rq.accumulate ? 1 : 2);
+    if (plan->kernel != 0 && (c->tma_shape == 1 || c->tma_shape == 2)) plan->kernel = (int)c->tma_shape;
   }
   for (auto& sp : segs) {
     DevSegment d;
