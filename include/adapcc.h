@@ -297,7 +297,9 @@ ADAPCC_API const char* adapcc_last_cuda_error(void);
  * dynamically; env ADAPCC_SCHED), "pdl" (1 = launch engine kernels as programmatic dependent
  * launches: a kernel's prologue overlaps the previous kernel on the stream, default; 0 = off;
  * env ADAPCC_PDL), "first_blob" (LDG fold kernel: 1 = item descriptors as per-item blobs,
- * default; 0 = plain item/task/ref tables; env ADAPCC_FIRST_BLOB), "trace" (in-kernel trace capacity in
+ * default; 0 = plain item/task/ref tables; env ADAPCC_FIRST_BLOB; env only: ADAPCC_TMA_SHAPE
+ * forces the TMA ring of every TMA launch, 1 = 1 CTA/SM x 3 x 64 KiB, 2 = 2 CTAs/SM x 3 x 32 KiB,
+ * 0 = automatic, default: ACCUMULATE and STAGED plans 2, others 1), "trace" (in-kernel trace capacity in
  * records, 0 = off, default; see adapcc_trace_read), "debug_check" (multi-process: 1 = every launch first compares a hash
  * of its call -- collective, strategy, count, dtype, mask, flags, live ranks, segment, zero-copy
  * registrations -- with every live peer's for the same launch, in the arena headers, before any
