@@ -4,7 +4,10 @@ Metric (BASELINE.json): AllReduce busbw (GB/s) = algbw * 2(n-1)/n, algbw =
 bytes per rank / time per call (nccl-tests convention).
 
   python bench.py                      # N=1: 8 virtual ranks on one B200 (loopback)
-  torchrun --nproc-per-node N bench.py --gpus N   # N>1: one process per GPU, CUDA IPC
+  python bench.py --gpus N             # N>1: re-launches itself under torch.distributed.run,
+                                       #      one process per GPU, CUDA IPC (fails without N GPUs)
+  torchrun --nproc-per-node N bench.py --gpus N   # the same, launched by the caller
+  python bench.py --gpus N --test-same-gpu        # N>1 code path, N processes on cuda:0
   python bench.py --impl reference     # the CPU oracle timed on the host (reference arm)
 
 N=1 workload: BASELINE config C2's multi-tree AllReduce at the paper's
@@ -42,8 +45,8 @@ def engine_name(engine, mode, dtype):
 def parse_args():
     p = argparse.ArgumentParser()
     p.add_argument("--gpus", type=int, default=1)
-    p.add_argument("--steps", type=int, default=100)
-    p.add_argument("--warmup", type=int, default=10)
+    p.add_argument("--steps", type=int, default=20)
+    p.add_argument("--warmup", type=int, default=5)
     p.add_argument("--impl", choices=["ours", "reference"], default="ours")
     p.add_argument("--vranks", type=int, default=8, help="virtual ranks at N=1")
     p.add_argument("--size-mib", type=float, default=256.0, help="bytes per rank (MiB)")
@@ -208,60 +211,65 @@ def time_point(fn, reduce_max=None, graph=True):
 
 
 # ------------------------------------------------------------------ oracle leg
-def oracle_sample_busbw(n, dtype, count, reps=1):
-    """Time the CPU oracle (as it stands) on a bounded sample; 1 host core."""
-    import numpy as np  # noqa: F401
-
-    from oracle import collectives as oc
-    from paper_conf_icdcs_zhaozw24_b200 import generator as G
-    from synth import rank_tensors
+def pin_one_core():
     try:
         os.sched_setaffinity(0, {sorted(os.sched_getaffinity(0))[0]})
     except Exception:  # noqa: BLE001
         pass
-    xs = rank_tensors(dtype, count, n)
-    text = G.allreduce_stars(n, chunk=262144)
-    es = 4 if dtype == "f32" else 2
+
+
+def oracle_replay(xs, text, n, dtype):
+    """The CPU oracle (as it stands) on the whole workload: (outputs, seconds)."""
+    from oracle import collectives as oc
     t0 = time.perf_counter()
-    for _ in range(reps):
-        oc.allreduce(xs, text, set(range(n)), dtype)
-    dt = (time.perf_counter() - t0) / reps
-    return busbw(count * es, dt, n), dt
+    ys = oc.allreduce(xs, text, set(range(n)), dtype)
+    return ys, time.perf_counter() - t0
 
 
-def cpu_baseline_block(n, dtype, target_s=15.0):
-    count = 1 << 20
-    v, dt = oracle_sample_busbw(n, dtype, count)
-    reps = max(1, min(200, int(target_s / max(dt, 1e-6))))
-    v, dt = oracle_sample_busbw(n, dtype, count, reps=reps)
+def cpu_baseline_block(xs, text, n, dtype, first_s, target_s=15.0):
+    """The oracle timed on the bench workload itself (every rank's full
+    tensor), one host core; `first_s` = the replay parity already timed."""
     es = 4 if dtype == "f32" else 2
-    return {"value": round(v, 4), "unit": UNIT, "cores": 1, "kind": "oracle",
-            "sample": f"{n} simulated ranks x {count} {dtype} elements ({count * es >> 20} MiB/rank), "
-                      f"{reps} reps, numpy single thread pinned to 1 core of {os.cpu_count()}"}
+    reps = max(0, min(20, int(round(target_s / max(first_s, 1e-6))) - 1))
+    times = [first_s]
+    pin_one_core()
+    for _ in range(reps):
+        times.append(oracle_replay(xs, text, n, dtype)[1])
+    t = sum(times) / len(times)
+    return {"value": round(busbw(len(xs[0]) * es, t, n), 4), "unit": UNIT, "cores": 1, "kind": "oracle",
+            "sample": f"the full bench workload ({n} simulated ranks x {len(xs[0]) * es >> 20} MiB {dtype}, "
+                      f"strategy-order replay), {len(times)} reps, mean {t:.2f} s, numpy single thread pinned "
+                      f"to 1 core of {os.cpu_count()}"}
 
 
 def run_reference(args):
+    """Reference arm of this tier: the CPU oracle, as it stands, timed on the
+    host on this arm's own workload (N ranks x size-mib per step, N = 8
+    virtual ranks at --gpus 1).  Under torchrun only rank 0 runs it."""
+    from paper_conf_icdcs_zhaozw24_b200 import generator as G
+    from synth import rank_tensors
     r, w, _ = dist_env()
     if r != 0:
         return None
-    n = args.vranks if w == 1 else w
-    count = 1 << 20
+    ngpus = max(w, args.gpus)
+    n = args.vranks if ngpus == 1 else ngpus
     es = 4 if args.dtype == "f32" else 2
+    count = int(args.size_mib * (1 << 20)) // 16 * 16 // es
+    xs = rank_tensors(args.dtype, count, n)
+    text = G.allreduce_stars(n, chunk=args.chunk_kib * 1024)
+    pin_one_core()
     for _ in range(args.warmup):
-        oracle_sample_busbw(n, args.dtype, count)
-    times = []
-    for _ in range(args.steps):
-        _, dt = oracle_sample_busbw(n, args.dtype, count)
-        times.append(dt)
+        oracle_replay(xs, text, n, args.dtype)
+    times = [oracle_replay(xs, text, n, args.dtype)[1] for _ in range(args.steps)]
     t = sum(times) / len(times)
     v = busbw(count * es, t, n)
-    sample = (f"{n} simulated ranks x {count} {args.dtype} elements per step "
-              f"({count * es >> 20} MiB/rank), numpy 1 core of {os.cpu_count()}")
+    sample = (f"the whole workload every step: {n} simulated ranks x {count * es >> 20} MiB {args.dtype} "
+              f"(strategy-order replay of {n} star trees), numpy single thread pinned to 1 core of {os.cpu_count()}")
     return {
         "impl": "reference", "metric": METRIC, "value": round(v, 4), "unit": UNIT,
-        "n_gpus": w, "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(t * 1e3, 3),
+        "n_gpus": ngpus, "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(t * 1e3, 3),
         "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": args.dtype,
-        "data": "synthetic", "config": workload_config(args, n, w),
+        "data": "synthetic", "config": workload_config(args, n, ngpus),
         "cpu_baseline": {"value": round(v, 4), "unit": UNIT, "cores": 1, "kind": "oracle",
                          "sample": sample},
         "e2e": {"value": round(v, 4), "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
@@ -278,6 +286,7 @@ def workload_config(args, n, world):
         "mode": args.mode if world == 1 else "zero-copy direct (registered buffers)", "ready_mask": "all",
         "l2": f"inputs {n * nbytes >> 20} MiB per step > 126 MB L2 (no flush needed)",
         "parallelism": f"{'virtual ' if world == 1 else ''}dp{n}",
+        "same_gpu": bool(world > 1 and getattr(args, "test_same_gpu", False)),
     }
 
 
@@ -341,10 +350,15 @@ def run_single(args):
     kern_ms = sum(per) / len(per)
     value = busbw(nbytes, ms / 1e3, n)
 
-    # parity on sampled outputs at full size (oracle, one element at a time)
-    parity = None
-    if not args.no_parity:
-        parity = sampled_parity(dy, host_in, text, n, count, args.dtype)
+    # parity at the bench point: EVERY output element of every rank against
+    # the oracle's strategy-order replay of the same inputs, bit-exact
+    parity, xs_np, oracle_s = None, None, None
+    if not args.no_parity or not args.no_cpu_baseline:
+        xs_np = [h.numpy().view(np.uint16) if args.dtype == "bf16" else h.numpy() for h in host_in]
+        ys, oracle_s = oracle_replay(xs_np, text, n, args.dtype)
+        if not args.no_parity:
+            parity = complete_parity(dy, ys, args.dtype)
+        del ys
 
     # end to end: pinned host inputs -> device -> allreduce -> pinned host, every
     # step.  Steps are pipelined like a training loop's buckets: double-buffered
@@ -396,7 +410,7 @@ def run_single(args):
                      "126 MB L2 run partly from L2",
     }
     if not args.no_cpu_baseline:
-        out["cpu_baseline"] = cpu_baseline_block(n, args.dtype)
+        out["cpu_baseline"] = cpu_baseline_block(xs_np, text, n, args.dtype, oracle_s)
     comm.finalize()
     return out
 
@@ -458,60 +472,52 @@ def e2e_pipelined(comm, host_in, dx, dy, steps, tdt, call, second=None):
     return a.elapsed_time(z) / steps
 
 
-def sampled_parity(dy, host_in, text, n, count, dtype, k=4096):
+def complete_parity(dy, ys, dtype):
+    """Bit mismatches of every output element of every rank (device tensors
+    dy) against the oracle's outputs ys."""
     import numpy as np
     import torch
-
-    from oracle import collectives as oc
-    rng = np.random.default_rng(11)
-    idx = np.unique(np.concatenate([rng.integers(0, count, size=k), [0, count - 1]]))
-    ti = torch.from_numpy(idx).cuda()
-    vals = []
-    for h in host_in:
-        a = h.numpy()
-        vals.append(a[idx].view(np.uint16) if dtype == "bf16" else a[idx])
-    exp = oc.allreduce_elements(vals, idx, count, text, set(range(n)), dtype)
     bad = 0
-    for y in dy:
-        g = y.index_select(0, ti)
-        g = g.view(torch.int16).cpu().numpy().view(np.uint16) if dtype == "bf16" else g.cpu().numpy()
-        ebits = exp.view(np.uint16) if dtype == "bf16" else exp.view(np.uint32)
-        gbits = g.view(np.uint16) if dtype == "bf16" else g.view(np.uint32)
-        bad += int(np.count_nonzero(ebits != gbits))
-    return {"samples_per_rank": int(len(idx)), "ranks": n, "mismatches": bad,
-            "reference": "oracle.allreduce_elements (strategy-order replay), bit-exact"}
+    for y, e in zip(dy, ys):
+        g = y.view(torch.int16).cpu().numpy().view(np.uint16) if dtype == "bf16" else y.cpu().numpy().view(np.uint32)
+        bad += int(np.count_nonzero(g != (e.view(np.uint16) if dtype == "bf16" else e.view(np.uint32))))
+    return {"complete": True, "elements_per_rank": int(dy[0].numel()), "ranks": len(dy), "mismatches": bad,
+            "reference": "oracle.allreduce (strategy-order replay) on the same inputs, every element, bit-exact"}
 
 
 # ---------------------------------------------------------------- our arm, N>1
-def multi_sampled_parity(comm, x, y, xh, text, world, rank, count, dtype, k=4096):
-    """One fresh zero-copy AllReduce, then every rank's input and output at the
-    same seeded indices go to rank 0, which replays the strategy on them with
-    the oracle and counts bit mismatches (None on other ranks)."""
+def multi_complete_parity(comm, x, y, text, world, rank, count, dtype):
+    """One fresh zero-copy AllReduce checked completely: rank 0 regenerates
+    every rank's seeded input, replays the strategy with the oracle and
+    compares its own output element by element; every other rank sends the
+    SHA-256 of its whole output, which must equal the hash of the oracle's
+    output for that rank (all outputs of an AllReduce are bitwise identical,
+    but each rank is checked against its own expected bytes).  None on ranks > 0."""
+    import hashlib
+
     import numpy as np
     import torch
     import torch.distributed as dist
 
-    from oracle import collectives as oc
+    from synth import rank_tensors
     y.fill_(float("nan"))
     comm.collective_zc("allreduce", x, y, count)
     torch.cuda.synchronize()
-    rng = np.random.default_rng(11)
-    idx = np.unique(np.concatenate([rng.integers(0, count, size=k), [0, count - 1]]))
-    ti = torch.from_numpy(idx).to(y.device)
-    a = xh.numpy()[idx]
-    g = y.index_select(0, ti)
-    g = g.view(torch.int16).cpu().numpy() if dtype == "bf16" else g.cpu().numpy()
-    mine = (a.view(np.uint16) if dtype == "bf16" else a, g.view(np.uint16) if dtype == "bf16" else g)
+    g = y.view(torch.int16).cpu().numpy().view(np.uint16) if dtype == "bf16" else y.cpu().numpy().view(np.uint32)
     got = [None] * world
-    dist.all_gather_object(got, mine)
+    dist.all_gather_object(got, hashlib.sha256(g.tobytes()).hexdigest())
     if rank != 0:
         return None
-    exp = oc.allreduce_elements([v[0] for v in got], idx, count, text, set(range(world)), dtype)
-    ebits = exp.view(np.uint16) if dtype == "bf16" else exp.view(np.uint32)
-    bad = sum(int(np.count_nonzero((v[1].view(np.uint16) if dtype == "bf16" else v[1].view(np.uint32)) != ebits))
-              for v in got)
-    return {"samples_per_rank": int(len(idx)), "ranks": world, "mismatches": bad,
-            "reference": "oracle.allreduce_elements (strategy-order replay) on every rank's sampled inputs, bit-exact"}
+    xs = [rank_tensors(dtype, count, 1, base=1000 + r)[0] for r in range(world)]
+    ys, _ = oracle_replay(xs, text, world, dtype)
+    e0 = ys[0].view(np.uint16) if dtype == "bf16" else ys[0].view(np.uint32)
+    bad0 = int(np.count_nonzero(g != e0))
+    bad_ranks = [q for q in range(1, world)
+                 if got[q] != hashlib.sha256(ys[q].tobytes()).hexdigest()]
+    return {"complete": True, "elements_per_rank": int(count), "ranks": world, "mismatches": bad0,
+            "ranks_mismatched": ([0] if bad0 else []) + bad_ranks,
+            "reference": "oracle.allreduce (strategy-order replay) of every rank's seeded input; rank 0 "
+                         "element by element, ranks > 0 by SHA-256 of the whole output, bit-exact"}
 
 
 def run_multi(args):
@@ -625,7 +631,7 @@ def run_multi(args):
                 nms, _ = time_point(lambda: dist.all_reduce(zs_), reduce_max, graph=False)
                 pt.update({"nccl_us": round(nms * 1e3, 2), "nccl_busbw": round(busbw(sb, nms / 1e3, world), 2)})
             sweep.append(pt)
-    parity = None if args.no_parity else multi_sampled_parity(comm, x, y, xh, text, world, rank, count, args.dtype)
+    parity = None if args.no_parity else multi_complete_parity(comm, x, y, text, world, rank, count, args.dtype)
     st = pkg.adapcc.plan_stats(text, count, args.dtype, (1 << world) - 1, rank=rank)
     dir_bytes = st["remote_bytes"]   # = bytes crossing each link direction of this GPU (symmetric plan)
     res = None
@@ -668,18 +674,53 @@ def run_multi(args):
     return res
 
 
+def free_port():
+    import socket
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def self_launch(args):
+    """--gpus N without a launcher: re-run this script as N ranks under
+    torch.distributed.run (one process per GPU, 127.0.0.1 rendezvous).
+    Without N visible GPUs it fails loudly unless --test-same-gpu is given
+    (then all N ranks share cuda:0 and the numbers are not NVLink numbers)."""
+    if not args.test_same_gpu:
+        import torch
+        have = torch.cuda.device_count()
+        if have < args.gpus:
+            print(f"bench.py: --gpus {args.gpus} needs {args.gpus} visible GPUs, found {have} "
+                  f"(use --test-same-gpu to run the N-rank code path on one GPU)", file=sys.stderr)
+            return 2
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr=127.0.0.1", f"--master-port={free_port()}", os.path.abspath(__file__), *sys.argv[1:]]
+    return subprocess.run(cmd, cwd=ROOT).returncode
+
+
 def main():
     args = parse_args()
     _, world, _ = dist_env()
+    if args.gpus < 1:
+        print("bench.py: --gpus must be >= 1", file=sys.stderr)
+        return 2
+    if "WORLD_SIZE" in os.environ and world != args.gpus:
+        print(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={world}", file=sys.stderr)
+        return 2
     if args.impl == "reference":
-        out = run_reference(args)
+        out = run_reference(args)        # CPU only: no launcher needed, rank 0 prints
+    elif args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        return self_launch(args)
     elif world > 1:
         out = run_multi(args)
     else:
         out = run_single(args)
     if out is not None:
         print(json.dumps(out), flush=True)
+    return 0
 
 
 if __name__ == "__main__":
-    main()
+    sys.exit(main())

@@ -88,6 +88,10 @@ typedef enum { ADAPCC_MODE_DIRECT = 0, ADAPCC_MODE_STAGED = 1 } adapcc_mode_t;
  *     records which ones it folded.
  *   LATE_COMPLEMENT (phase 2, SAME mask R and buffers as phase 1): recvbuf +=
  *     sum of the non-ready ranks' inputs that phase 1 did not fold, per piece.
+ *     It complements the most recent LATE_JOIN call of the same plan (same
+ *     strategy, count, dtype, mask and buffers kind); phase-1 / phase-2 pairs
+ *     of different plans may interleave.  A second LATE_COMPLEMENT after the
+ *     same phase 1 adds nothing.  No phase 1 of this plan yet: INVALID_ARGUMENT.
  * After both phases every rank holds the sum over all ranks. */
 #define ADAPCC_FLAG_LATE_JOIN 0x2u
 #define ADAPCC_FLAG_LATE_COMPLEMENT 0x4u
@@ -286,7 +290,7 @@ ADAPCC_API const char* adapcc_last_cuda_error(void);
 
 /* Runtime knobs.  key: "timeout_ms" (watchdog, default 10000; env
  * ADAPCC_TIMEOUT_MS), "max_ctas" (grid cap, 0 = #SMs x occupancy; env
- * ADAPCC_NCTAS), "engine" (2 = auto by call size, default; 1 = TMA bulk-copy
+ * ADAPCC_NCTAS; a change empties the plan cache, since pieces are sized for the grid), "engine" (2 = auto by call size, default; 1 = TMA bulk-copy
  * pipeline; 0 = 128-bit LDG/STG fold; env ADAPCC_ENGINE), "piece_kib" (traffic per work
  * piece of flag-free tasks, 0 = automatic, default; env ADAPCC_PIECE_KIB), "taper" (the last
  * ~2 x grid flag-free items are cut into this many sub-pieces, 0..64; 0 = automatic,

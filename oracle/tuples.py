@@ -72,18 +72,6 @@ def behavior(parent, ready, noagg=frozenset()):
     return tup, flows
 
 
-def kernel_sources(parent, ready, noagg, g, flows=None):
-    """Ordered inputs folded by kernel node g: own tensor (if ready), then the
-    flows of its sending children by ascending rank (reading Q5)."""
-    tup, fl = behavior(parent, ready, noagg) if flows is None else flows
-    n = len(parent)
-    src = [("in", g)] if tup[g][0] else []
-    for c in range(n):
-        if parent[c] == g and tup[c][3]:
-            src += fl[c]
-    return src
-
-
 def broadcast_tuples(parent):
     """Broadcast stage of AllReduce = the reduce tree reversed (Q8):
     every non-root receives, nobody aggregates, a rank sends iff it has

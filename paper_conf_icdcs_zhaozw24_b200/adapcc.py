@@ -246,7 +246,7 @@ def plan_stats(text, count, dtype, mask, accumulate=False, mode="direct", rank=-
 
 
 def plan_items(text, count, dtype, mask, grid, tma=False, accumulate=False, mode="direct", rank=-1,
-               scratch_bytes=0, piece_kib=0, taper=0, segment=0):
+               scratch_bytes=0, piece_kib=0, taper=0, segment=0, late=None):
     """Work items (claim order) and tasks of one segment of a call's plan, as
     numpy structured arrays (include/adapcc.h adapcc_plan_items)."""
     import numpy as np
@@ -256,7 +256,8 @@ def plan_items(text, count, dtype, mask, grid, tma=False, accumulate=False, mode
                     ("nsrc", "<u2"), ("ndst", "<u2"), ("nwait", "<u2"), ("npost", "<u2"),
                     ("level", "<u4"), ("owner", "<u4")])
     ni, nt = ctypes.c_uint32(), ctypes.c_uint32()
-    args = (text.encode(), count, DTYPE_CODE[dtype], mask, FLAG_ACCUMULATE if accumulate else 0, MODE[mode],
+    flags = (FLAG_ACCUMULATE if accumulate else 0) | _late_flag(late)
+    args = (text.encode(), count, DTYPE_CODE[dtype], mask, flags, MODE[mode],
             rank, scratch_bytes, grid, 1 if tma else 0, piece_kib, taper, segment)
     _check(L.adapcc_plan_items(*args, None, 0, ctypes.byref(ni), None, 0, ctypes.byref(nt)), "plan_items")
     items, tasks = np.zeros(ni.value, dtype=idt), np.zeros(nt.value, dtype=tdt)

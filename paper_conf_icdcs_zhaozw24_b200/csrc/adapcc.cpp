@@ -42,8 +42,8 @@ struct DevSegment {
   Item* items = nullptr;
   uint32_t nitems = 0;
   uint64_t* late_bits = nullptr;  // per item: late ranks folded in phase 1 (late join)
-  uint32_t* late_list = nullptr;  // 2 x nitems: items phase 1 left incomplete (per ticket parity)
-  uint32_t* late_count = nullptr; // 2 counts
+  uint32_t* late_list = nullptr;  // nitems: items phase 1 left incomplete
+  unsigned long long* late_count = nullptr;  // (gen << 32 | count), epoch of the last phase 1 (launch.hpp)
   uint4* first = nullptr;         // LDG kernel: per-CTA first-item blobs (launch.hpp)
   uint32_t nfirst = 0, first_words = 0;
   uint32_t sched_static = 0;      // LDG kernel: every item has a blob, CTA b runs b, b + grid, ...
@@ -456,9 +456,10 @@ adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, const Strategy* strat, uin
     if (rq.late_join) {
       CK(cudaMalloc(&d.late_bits, std::max<size_t>(1, items.size()) * sizeof(uint64_t)));
       CK(cudaMemset(d.late_bits, 0, std::max<size_t>(1, items.size()) * sizeof(uint64_t)));
-      CK(cudaMalloc(&d.late_list, 2 * std::max<size_t>(1, items.size()) * sizeof(uint32_t)));
-      CK(cudaMalloc(&d.late_count, 2 * sizeof(uint32_t)));
-      CK(cudaMemset(d.late_count, 0, 2 * sizeof(uint32_t)));
+      CK(cudaMalloc(&d.late_list, std::max<size_t>(1, items.size()) * sizeof(uint32_t)));
+      CK(cudaMalloc(&d.late_count, 2 * sizeof(unsigned long long)));
+      const unsigned long long init[2] = {0ull, ~0ull};  // empty list, no phase 1 recorded
+      CK(cudaMemcpy(d.late_count, init, sizeof(init), cudaMemcpyHostToDevice));
     }
     plan->segs.push_back(d);
   }
@@ -556,10 +557,14 @@ adapcc_result_t run(adapcc_comm_s* c, Coll coll, const void* const* send, void* 
       }
       P.hdr[q] = c->arena[q];
     }
-    const int grid = std::max(1, std::min<int>(grid_size(c, dtype, plan->kernel), (int)std::max<uint32_t>(1, seg.nitems)));
+    // phase 2 of a late join accumulates into every destination: on the TMA
+    // engine it takes the ACCUMULATE shape (2 x 3 x 32 KiB) whatever the plan's
+    // kernel; item order is grid-independent, so the plan is shared
+    const int kernel = (late_mode == 2 && plan->kernel == 1 && c->tma_shape != 1) ? 2 : plan->kernel;
+    const int grid = std::max(1, std::min<int>(grid_size(c, dtype, kernel), (int)std::max<uint32_t>(1, seg.nitems)));
     const bool pdl = c->pdl != 0;
-    CK(plan->kernel == 1 ? tma_direct::launch(P, grid, s, pdl)
-       : plan->kernel == 2 ? tma_staged::launch(P, grid, s, pdl) : engine_launch(P, grid, s, pdl));
+    CK(kernel == 1 ? tma_direct::launch(P, grid, s, pdl)
+       : kernel == 2 ? tma_staged::launch(P, grid, s, pdl) : engine_launch(P, grid, s, pdl));
     c->last_engine = plan->engine;
     ++c->launches;
   }
@@ -1178,7 +1183,11 @@ adapcc_result_t adapcc_config(adapcc_comm_t c, const char* key, int64_t value) {
   if (!c || !key) return ADAPCC_ERR_INVALID_ARGUMENT;
   std::lock_guard<std::mutex> lock(c->mu);
   if (!std::strcmp(key, "timeout_ms")) { if (value < 1) return ADAPCC_ERR_INVALID_ARGUMENT; c->timeout_ms = value; }
-  else if (!std::strcmp(key, "max_ctas")) { if (value < 0) return ADAPCC_ERR_INVALID_ARGUMENT; c->max_ctas = value; }
+  else if (!std::strcmp(key, "max_ctas")) {
+    if (value < 0) return ADAPCC_ERR_INVALID_ARGUMENT;
+    if (value != c->max_ctas) drop_plans(c);  // pieces, taper and first-item blobs are sized for the grid
+    c->max_ctas = value;
+  }
   else if (!std::strcmp(key, "engine")) {
     if (value < 0 || value > 2) return ADAPCC_ERR_INVALID_ARGUMENT;
     if (value != c->engine) drop_plans(c);  // pieces are sized for the engine's grid

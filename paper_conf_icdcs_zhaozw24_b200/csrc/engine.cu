@@ -264,7 +264,7 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
       if (t.nlate == 0) {
         c.dropped = P.late_mode == 2;  // phase 2 only runs the roots' folds
       } else {
-        const uint64_t m = late_select(P, t, it);
+        const uint64_t m = late_select(P, t, it, sh.epoch);
         c.late = m;
         if (P.late_mode == 2) {  // recv += sum of the late ranks not yet included
           c.nreg = 0;
@@ -344,11 +344,8 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
     if (threadIdx.x == 0) e_lazy = *reinterpret_cast<volatile unsigned long long*>(&P.state->epoch) + 1;
   } else {
     if (threadIdx.x == 0) {
-      // late join (never lazy): phase 2 claims positions in phase 1's list;
-      // phase 1 empties the other ticket parity's list for the next phase 1
-      if (P.late_mode == 2 && P.late_list && !stat)
-        sh.nclaim = *reinterpret_cast<volatile uint32_t*>(&P.late_count[P.late_ticket & 1]);
-      if (P.late_mode == 1 && blockIdx.x == 0) P.late_count[(P.late_ticket + 1) & 1] = 0;
+      // late join (never lazy): phase 2 claims positions in phase 1's list
+      if (P.late_mode == 2 && P.late_list && !stat) sh.nclaim = late_listed(P);
       // this launch's epoch = the one the previous launch published + 1
       const uint64_t e = *reinterpret_cast<volatile unsigned long long*>(&P.state->epoch) + 1;
       sh.epoch = e;
@@ -396,7 +393,7 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
                                                      : gridDim.x + atomicAdd(&P.state->work[par], 1u);
         sh.claim = k;
         uint32_t it = k;
-        if (listed) it = k < sh.nclaim ? P.late_list[(size_t)(P.late_ticket & 1) * P.nitems + k] : P.nitems;
+        if (listed) it = k < sh.nclaim ? P.late_list[k] : P.nitems;
         // (a listed phase-2 item is not the CTA's first item: no blob, no preloaded item)
         const bool fb = stat || (first && use_blob && !listed);
         stage(it, fb, buf, first && !listed);
@@ -477,9 +474,9 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
     if (done == gridDim.x - 1) {
       // last CTA: publish the epoch for the next launch on this stream and,
       // across processes, "this rank finished epoch" to the peers
-      // phase 2 consumed its list (every CTA is past its claims): empty it, so
-      // a replayed phase 1 with the same ticket starts a fresh one
-      if (P.late_mode == 2 && P.late_count) P.late_count[P.late_ticket & 1] = 0;
+      // late join: phase 1 validates its list for phase 2; phase 2 consumed it
+      // (every CTA is past its claims), so a repeated phase 2 adds nothing
+      if (P.late_mode && P.late_count) P.late_count[1] = P.late_mode == 1 ? ep : ~0ull;
       *reinterpret_cast<volatile unsigned long long*>(&P.state->epoch) = ep;
       if (P.ipc) {
         __threadfence_system();

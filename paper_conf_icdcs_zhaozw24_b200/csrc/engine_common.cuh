@@ -189,8 +189,30 @@ static __device__ bool check_call_sig(const LaunchParams& P, uint64_t epoch) {
 // work item `item`.  Mode 1 (phase 1): candidates whose ready word
 // (arena header + 16) reached the call's ticket, recorded in late_bits[item];
 // mode 2 (phase 2): the candidates NOT recorded (only they remain to add).
+// Position of the next entry in the plan's phase-2 list for the phase-1
+// launch of `epoch`: the first append of a new launch (gen differs) restarts
+// the count at 0 (launch.hpp, late_count).
+static __device__ __forceinline__ uint32_t late_append(const LaunchParams& P, uint64_t epoch) {
+  const unsigned long long gen = (unsigned long long)(uint32_t)epoch;
+  unsigned long long old = *reinterpret_cast<volatile unsigned long long*>(&P.late_count[0]), nw;
+  for (;;) {
+    nw = (old >> 32) == gen ? old + 1 : ((gen << 32) | 1ull);
+    const unsigned long long prev = atomicCAS(&P.late_count[0], old, nw);
+    if (prev == old) break;
+    old = prev;
+  }
+  return (uint32_t)nw - 1u;
+}
+
+// Entries phase 2 runs: the list of the last completed phase 1, if any.
+static __device__ __forceinline__ uint32_t late_listed(const LaunchParams& P) {
+  const unsigned long long w = *reinterpret_cast<volatile unsigned long long*>(&P.late_count[0]);
+  const unsigned long long g = *reinterpret_cast<volatile unsigned long long*>(&P.late_count[1]);
+  return g != ~0ull && (w >> 32) == (unsigned long long)(uint32_t)g ? (uint32_t)w : 0u;
+}
+
 static __device__ __forceinline__ uint64_t late_select(const LaunchParams& P, const Task& t,
-                                                       uint32_t item) {
+                                                       uint32_t item, uint64_t epoch) {
   uint64_t m = 0;
   if (P.late_mode == 1) {
     for (int j = 0; j < t.nlate; ++j) {
@@ -201,10 +223,7 @@ static __device__ __forceinline__ uint64_t late_select(const LaunchParams& P, co
     }
     P.late_bits[item] = m;
     const uint64_t all = t.nlate >= 64 ? ~0ull : ((1ull << t.nlate) - 1);
-    if (all & ~m) {  // phase 2 has something to add here
-      const unsigned par = (unsigned)(P.late_ticket & 1);
-      P.late_list[(size_t)par * P.nitems + atomicAdd(&P.late_count[par], 1u)] = item;
-    }
+    if (all & ~m) P.late_list[late_append(P, epoch)] = item;  // phase 2 has something to add here
   } else if (P.late_mode == 2) {
     const uint64_t all = t.nlate >= 64 ? ~0ull : ((1ull << t.nlate) - 1);
     m = all & ~P.late_bits[item];
@@ -217,7 +236,7 @@ static __device__ __forceinline__ uint64_t late_select(const LaunchParams& P, co
 // candidates are in flight together instead of one candidate after another.
 // Same result and side effects as late_select; every lane returns the mask.
 static __device__ __forceinline__ uint64_t late_select_warp(const LaunchParams& P, const Task& t,
-                                                            uint32_t item, int lane) {
+                                                            uint32_t item, int lane, uint64_t epoch) {
   const uint64_t all = t.nlate >= 64 ? ~0ull : ((1ull << t.nlate) - 1);
   if (P.late_mode == 2) return all & ~P.late_bits[item];
   if (P.late_mode != 1) return 0;
@@ -234,10 +253,7 @@ static __device__ __forceinline__ uint64_t late_select_warp(const LaunchParams& 
   }
   if (lane == 0) {
     P.late_bits[item] = m;
-    if (all & ~m) {  // phase 2 has something to add here
-      const unsigned par = (unsigned)(P.late_ticket & 1);
-      P.late_list[(size_t)par * P.nitems + atomicAdd(&P.late_count[par], 1u)] = item;
-    }
+    if (all & ~m) P.late_list[late_append(P, epoch)] = item;  // phase 2 has something to add here
   }
   return m;
 }

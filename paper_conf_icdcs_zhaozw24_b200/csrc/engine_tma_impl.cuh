@@ -57,6 +57,10 @@ constexpr int kMaxPost = 4;
 // producer also loads each accumulating destination's tile, so a stage holds
 // nsrc + nacc tiles of at least 512 B (acc_tma in the item descriptor)
 constexpr int kMaxAccTiles = 24;
+// tuning overrides (ADAPCC_TMA_STAGE_KB / _STAGES) must leave at least one
+// 4 KiB source tile and one 512-byte ACCUMULATE tile per stage
+static_assert(kStageBytes % 4096 == 0 && kStageBytes >= kMaxAccTiles * 512, "TMA stage too small");
+static_assert(kMaxKS >= 1 && kStages >= 2, "TMA pipeline shape");
 
 struct ItemDesc {
   const char* src[kMaxFold];
@@ -441,7 +445,8 @@ template <int DT>
 // CTA's first-item blob
 __device__ __forceinline__ void fill_desc(const LaunchParams& P, char* const (*base)[kMaxRanksDev],
                                           ItemDesc& d, const Item& item, const Task& t, const BufRef* R,
-                                          uint64_t half_off, int lane, uint32_t it, int* nwait_eff) {
+                                          uint64_t half_off, int lane, uint32_t it, int* nwait_eff,
+                                          uint64_t epoch) {
   constexpr int esize = Ops<DT>::kEsize;
   const uint64_t e0 = t.lo + (uint64_t)item.chunk * t.chunk_elems + item.off;
   // late join (phase 1) / complement (phase 2): which candidate ranks are folded
@@ -453,7 +458,7 @@ __device__ __forceinline__ void fill_desc(const LaunchParams& P, char* const (*b
     if (t.nlate == 0) {
       dropped = P.late_mode == 2;  // phase 2 only runs the roots' folds
     } else {
-      late = late_select_warp(P, t, it, lane);
+      late = late_select_warp(P, t, it, lane, epoch);
       if (P.late_mode == 2) {
         nreg = 0;
         *nwait_eff = 0;
@@ -567,7 +572,7 @@ __global__ void __launch_bounds__(kTmaThreads, ADAPCC_TMA_MINB) engine_tma_kerne
       int nwait = 0;
       fill_desc<DT>(P, sm.base, sm.q[0], *reinterpret_cast<const Item*>(&sm.blob[0]),
                     *reinterpret_cast<const Task*>(&sm.blob[1]),
-                    reinterpret_cast<const BufRef*>(&sm.blob[kBlobRef0]), 0, lane, blockIdx.x, &nwait);
+                    reinterpret_cast<const BufRef*>(&sm.blob[kBlobRef0]), 0, lane, blockIdx.x, &nwait, 0);
       __syncwarp();
     }
   }
@@ -581,8 +586,6 @@ __global__ void __launch_bounds__(kTmaThreads, ADAPCC_TMA_MINB) engine_tma_kerne
     if (blockIdx.x == 0) {
       P.state->work[(e + 1) & 1] = 0;
       P.state->done[(e + 1) & 1] = 0;
-      // phase 1: empty the other ticket parity's list for the next phase 1
-      if (P.late_mode == 1) P.late_count[(P.late_ticket + 1) & 1] = 0;
     }
   }
   __syncthreads();
@@ -614,15 +617,14 @@ __global__ void __launch_bounds__(kTmaThreads, ADAPCC_TMA_MINB) engine_tma_kerne
     // phase 1 listed as incomplete: claims index that list (no waits in phase
     // 2, so any order is deadlock-free) and everything else is never touched.
     const bool listed = P.late_mode == 2 && P.late_list != nullptr;
-    const uint32_t nclaim = listed ? *reinterpret_cast<volatile uint32_t*>(&P.late_count[P.late_ticket & 1])
-                                   : P.nitems;
+    const uint32_t nclaim = listed ? late_listed(P) : P.nitems;
     for (;;) {
       uint32_t it = 0;
       int stop_i = 0;
       if (lane == 0 && !last) {
         it = first ? blockIdx.x : gridDim.x + atomicAdd(&P.state->work[par], 1u);
         last = (uint64_t)it + gridDim.x >= nclaim;
-        if (listed) it = it < nclaim ? P.late_list[(size_t)(P.late_ticket & 1) * P.nitems + it] : P.nitems;
+        if (listed) it = it < nclaim ? P.late_list[it] : P.nitems;
       } else if (lane == 0) {
         it = P.nitems;
       }
@@ -644,7 +646,7 @@ __global__ void __launch_bounds__(kTmaThreads, ADAPCC_TMA_MINB) engine_tma_kerne
         int nwait = 0;
         if (!(fb && P.arena_free && P.late_mode == 0)) {  // (else described before the wait, above)
           const BufRef* R = fb ? reinterpret_cast<const BufRef*>(&sm.blob[kBlobRef0]) : P.refs + t.ref0;
-          fill_desc<DT>(P, sm.base, d, item, t, R, half_off, lane, it, &nwait);
+          fill_desc<DT>(P, sm.base, d, item, t, R, half_off, lane, it, &nwait, epoch);
           __syncwarp();
         }
         if (!d.dropped) {
@@ -677,11 +679,13 @@ __global__ void __launch_bounds__(kTmaThreads, ADAPCC_TMA_MINB) engine_tma_kerne
           const uint32_t tb = min(d.tile, d.vec_bytes - tt * d.tile);
           for (int p = 0; p < d.passes; ++p) {
             const int ks = min((int)d.ks, (int)d.nsrc - p * (int)d.ks);
+            // every issuing lane acquires the stage's release (its TMA load
+            // overwrites what the consumers read); lane 0 arms the tx count
+            mbar_wait(&sm.empty[stage], sphase ^ 1);
             if (lane == 0) {
               int nacc = 0;
               if (d.acc_tma)
                 for (int k = 0; k < d.ndst; ++k) nacc += d.acc[k] ? 1 : 0;
-              mbar_wait(&sm.empty[stage], sphase ^ 1);
               mbar_expect_tx(&sm.full[stage], (uint32_t)(ks + nacc) * tb);
             }
             __syncwarp();
@@ -763,9 +767,9 @@ __global__ void __launch_bounds__(kTmaThreads, ADAPCC_TMA_MINB) engine_tma_kerne
     }
     const unsigned done = atomicAdd(&P.state->done[par], 1u);
     if (done == gridDim.x - 1) {
-      // phase 2 consumed its list (every CTA is past its claims): empty it, so
-      // a replayed phase 1 with the same ticket starts a fresh one
-      if (P.late_mode == 2 && P.late_count) P.late_count[P.late_ticket & 1] = 0;
+      // late join: phase 1 validates its list for phase 2; phase 2 consumed it
+      // (every CTA is past its claims), so a repeated phase 2 adds nothing
+      if (P.late_mode && P.late_count) P.late_count[1] = P.late_mode == 1 ? epoch : ~0ull;
       *reinterpret_cast<volatile unsigned long long*>(&P.state->epoch) = epoch;
       if (P.ipc) {
         __threadfence_system();

@@ -67,11 +67,18 @@ struct LaunchParams {
   int late_mode;        // 0: off; 1: late join (phase 1); 2: complement (phase 2)
   uint64_t late_ticket; // ready word value that admits a late rank (phase 1)
   uint64_t* late_bits;  // per work item: late candidates included in phase 1
-  // Phase 1 lists the items that missed a late rank (late_list[par * nitems +
-  // i], i < late_count[par], par = late_ticket & 1); phase 2 runs exactly those.
-  // Phase 1's block 0 clears the other parity's count for the next phase 1.
+  // Phase 1 lists the items that missed a late rank (late_list[i], i < count)
+  // and phase 2 runs exactly those.  late_count[0] = (gen << 32) | count, where
+  // gen is the low 32 bits of the epoch of the phase-1 launch that appended:
+  // the first append of a launch with a new gen restarts the count, so a list
+  // never holds a stale entry (no reset step, CUDA-graph replays included).
+  // late_count[1] = epoch of the last completed phase 1 of this plan (written
+  // by its last CTA; ~0 after a phase 2 consumed the list): phase 2 runs the
+  // list only if its gen matches, so a phase 1 that listed nothing, or a
+  // repeated phase 2, adds nothing.  Both words are per plan: phase 1 / phase 2
+  // pairs of different plans may interleave on a stream.
   uint32_t* late_list;
-  uint32_t* late_count;
+  unsigned long long* late_count;
   int drop_rank;        // test hook (loopback): tasks owned by this rank are skipped
   uint64_t members;     // live ranks: excluded ranks are skipped by the IPC barriers
   uint64_t half_bytes;  // bytes of one parity half of an arena

@@ -28,12 +28,32 @@ def _run(cmd, timeout=600, env=None):
 
 
 def test_reference_arm_contract():
-    d = _run([sys.executable, "bench.py", "--impl", "reference", "--steps", "2", "--warmup", "1"])
+    d = _run([sys.executable, "bench.py", "--impl", "reference", "--steps", "2", "--warmup", "1",
+              "--size-mib", "4"])
     assert KEYS <= d.keys()
     assert d["impl"] == "reference" and d["value"] > 0 and d["unit"] == "GB/s"
     assert d["cpu_baseline"]["kind"] == "oracle" and d["cpu_baseline"]["cores"] == 1
     assert d["e2e"]["h2d_bytes_per_step"] == 0 and d["e2e"]["value"] == d["value"]
-    assert d["config"]["workload"].startswith("allreduce-loopback-vr8")
+    # the oracle runs the arm's own workload (not a smaller sample under its label)
+    assert d["config"]["workload"] == "allreduce-loopback-vr8-f32-4MiB-star8"
+    assert d["config"]["bytes_per_rank"] == 4 << 20 and "4 MiB" in d["cpu_baseline"]["sample"]
+
+
+def test_reference_arm_reports_n_gpus():
+    d = _run([sys.executable, "bench.py", "--impl", "reference", "--gpus", "2", "--steps", "1",
+              "--warmup", "1", "--size-mib", "1"])
+    assert d["n_gpus"] == 2 and d["config"]["ranks"] == 2
+
+
+def test_multi_gpu_without_gpus_fails_loudly():
+    """--gpus N with fewer than N visible GPUs (this CPU box has none) must not
+    fall back to a 1-GPU run: exit code != 0 and no JSON line."""
+    e = dict(os.environ, CUDA_VISIBLE_DEVICES="")
+    p = subprocess.run([sys.executable, "bench.py", "--gpus", "2", "--steps", "1", "--warmup", "1"],
+                       cwd=ROOT, capture_output=True, text=True, timeout=300, env=e)
+    assert p.returncode != 0
+    assert not [ln for ln in p.stdout.splitlines() if ln.startswith("{")]
+    assert "--gpus 2" in p.stderr
 
 
 @pytest.mark.gpu
@@ -45,7 +65,8 @@ def test_ours_single_gpu_contract():
               "--no-cpu-baseline", "--e2e-steps", "2"])
     assert KEYS | {"roofline", "gpu_launches", "clocks", "parity"} <= d.keys()
     assert d["n_gpus"] == 1 and d["value"] > 0 and d["gpu_launches"] == 3
-    assert d["parity"]["mismatches"] == 0
+    assert d["parity"]["complete"] and d["parity"]["mismatches"] == 0
+    assert d["parity"]["elements_per_rank"] == (16 << 20) // 4 and d["parity"]["ranks"] == 8
     r = d["roofline"]
     assert r["bound"] == "hbm" and r["achieved"] > 0 and abs(r["frac"] - r["achieved"] / r["peak"]) < 1e-3
     assert d["e2e"]["h2d_bytes_per_step"] == 8 * (16 << 20)
@@ -59,10 +80,11 @@ def test_ours_two_ranks_same_gpu_contract():
     torch = pytest.importorskip("torch")
     if not torch.cuda.is_available():
         pytest.skip("no GPU")
-    d = _run([sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
-              "--master-addr", "127.0.0.1", "--master-port", "29517", "bench.py", "--gpus", "2",
+    # no launcher: bench.py re-launches itself as 2 ranks (both on cuda:0)
+    d = _run([sys.executable, "bench.py", "--gpus", "2",
               "--steps", "3", "--warmup", "3", "--size-mib", "8", "--e2e-steps", "2", "--test-same-gpu"])
     assert KEYS | {"roofline", "gpu_launches", "parity", "staged"} <= d.keys()
-    assert d["n_gpus"] == 2 and d["async_error"] == 0
-    assert d["parity"]["mismatches"] == 0 and d["parity"]["ranks"] == 2
+    assert d["n_gpus"] == 2 and d["async_error"] == 0 and d["config"]["same_gpu"]
+    assert d["parity"]["complete"] and d["parity"]["mismatches"] == 0 and d["parity"]["ranks"] == 2
+    assert d["parity"]["ranks_mismatched"] == []
     assert [p["bytes_per_rank"] for p in d["sweep"]] == [1 << s for s in range(10, 24, 2)]

@@ -33,12 +33,13 @@ def _worker(rank, n, port, q, auto_register=False, steps=1):
 
         os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
         dist.init_process_group("gloo", rank=rank, world_size=n)
-        torch.cuda.set_device(0)
+        dev = rank % torch.cuda.device_count()  # one GPU per rank when the box has them
+        torch.cuda.set_device(dev)
         torch.manual_seed(0)
         model = torch.nn.Sequential(torch.nn.Linear(64, 256), torch.nn.ReLU(), torch.nn.Linear(256, 8)).cuda()
         ref = [p.detach().clone() for p in model.parameters()]
-        comm = pkg.Communicator.init(scratch_bytes=64 << 20, device=0)
-        ddp = DDP(model, device_ids=[0], bucket_cap_mb=1)
+        comm = pkg.Communicator.init(scratch_bytes=64 << 20, device=dev)
+        ddp = DDP(model, device_ids=[dev], bucket_cap_mb=1)
         state = AdapccHookState(comm, auto_register=auto_register)
         ddp.register_comm_hook(state, adapcc_allreduce_hook)
         g = torch.Generator(device="cpu").manual_seed(100 + rank)

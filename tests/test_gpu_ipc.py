@@ -1,6 +1,6 @@
 """Multi-process IPC path on ONE GPU (-m gpu).
 
-n processes share cuda:0, bootstrap over a gloo process group (127.0.0.1),
+n processes (one GPU each, or all on cuda:0 on a 1-GPU box) bootstrap over a gloo process group (127.0.0.1),
 export/open each other's arenas with CUDA IPC and run the STAGED protocol with
 system-scope flags -- the exact code path of the 8-GPU NVSwitch deployment,
 time-sliced on one device.  Each process checks its own recvbuf against the
@@ -43,8 +43,9 @@ def _worker(rank, n, port, case, q):
         os.environ["MASTER_ADDR"] = "127.0.0.1"
         os.environ["MASTER_PORT"] = str(port)
         dist.init_process_group("gloo", rank=rank, world_size=n)
-        torch.cuda.set_device(0)
-        comm = pkg.Communicator.init(scratch_bytes=64 << 20, device=0)
+        dev = rank % torch.cuda.device_count()  # one GPU per rank when the box has them
+        torch.cuda.set_device(dev)
+        comm = pkg.Communicator.init(scratch_bytes=64 << 20, device=dev)
         comm.config("timeout_ms", 60000)
         results = []
         if case == "allreduce":

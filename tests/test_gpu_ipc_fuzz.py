@@ -41,8 +41,9 @@ def _worker(rank, port, q):
 
         os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
         dist.init_process_group("gloo", rank=rank, world_size=N)
-        torch.cuda.set_device(0)
-        comm = pkg.Communicator.init(scratch_bytes=256 << 20, device=0)
+        dev = rank % torch.cuda.device_count()  # one GPU per rank when the box has them
+        torch.cuda.set_device(dev)
+        comm = pkg.Communicator.init(scratch_bytes=256 << 20, device=dev)
         comm.config("timeout_ms", 60000)
         cap = 3 * (1 << 20) * N + 64
         bx = torch.zeros(cap, dtype=torch.int32, device="cuda")

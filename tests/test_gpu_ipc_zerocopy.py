@@ -37,8 +37,9 @@ def _worker(rank, n, port, engine, q):
 
         os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
         dist.init_process_group("gloo", rank=rank, world_size=n)
-        torch.cuda.set_device(0)
-        comm = pkg.Communicator.init(scratch_bytes=64 << 20, device=0)
+        dev = rank % torch.cuda.device_count()  # one GPU per rank when the box has them
+        torch.cuda.set_device(dev)
+        comm = pkg.Communicator.init(scratch_bytes=64 << 20, device=dev)
         comm.config("timeout_ms", 60000)
         comm.config("engine", engine)
         ok = []
@@ -119,6 +120,85 @@ def test_zero_copy_one_gpu(n, engine):
     try:
         for _ in range(n):
             r, ok, msg = q.get(timeout=600)
+            out[r] = (ok, msg)
+    finally:
+        for p in procs:
+            p.join(timeout=30)
+            if p.is_alive():
+                p.kill()
+    for r in range(n):
+        assert r in out and out[r][0], out.get(r)
+
+
+def _big_worker(rank, n, port, mib, q):
+    """The N>1 bench path at bench-like size: >= 64 MiB per rank, zero-copy
+    DIRECT on the TMA engine (and the STAGED protocol beside it), every
+    element of this rank's output against the oracle replay."""
+    try:
+        sys.path.insert(0, ROOT)
+        import torch.distributed as dist
+
+        import paper_conf_icdcs_zhaozw24_b200 as pkg
+        from oracle import collectives as oc
+        from paper_conf_icdcs_zhaozw24_b200 import generator as G
+        from synth import rank_tensors
+        from tests.gpu_util import bits, to_dev, to_host
+
+        os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+        dist.init_process_group("gloo", rank=rank, world_size=n)
+        dev = rank % torch.cuda.device_count()
+        torch.cuda.set_device(dev)
+        nbytes = mib << 20
+        comm = pkg.Communicator.init(scratch_bytes=2 * nbytes + (64 << 20), device=dev)
+        comm.config("timeout_ms", 120000)
+        msgs = []
+        for dtype in ("f32", "bf16"):
+            es = 4 if dtype == "f32" else 2
+            count = nbytes // es - 8 * 3 - 5       # ragged: not a multiple of any tile
+            text = G.allreduce_stars(n, chunk=262144)
+            comm.set_strategy("allreduce", text)
+            xs = rank_tensors(dtype, count, n)
+            exp = oc.allreduce(xs, text, set(range(n)), dtype)[rank]
+            x = to_dev(xs[rank], dtype)
+            y = torch.empty_like(x)
+            rx, ry = comm.register(x), comm.register(y)
+            for engine, path in ((1, "zc"), (0, "zc"), (2, "staged")):
+                comm.config("engine", engine)
+                y.view(torch.uint8).fill_(0x5A)
+                if path == "zc":
+                    comm.collective_zc("allreduce", x, y, count)
+                else:
+                    comm.allreduce(x, y)
+                torch.cuda.synchronize()
+                bad = int(np.count_nonzero(bits(to_host(y, dtype)) != bits(exp)))
+                msgs.append(f"{dtype}/{path}/engine{engine}: {bad} bad")
+            comm.deregister(rx)
+            comm.deregister(ry)
+            del x, y
+        err = comm.get_async_error()
+        comm.finalize()
+        dist.destroy_process_group()
+        q.put((rank, err == 0 and all(m.endswith(": 0 bad") for m in msgs), f"{msgs} err={err}"))
+    except Exception as e:  # noqa: BLE001
+        import traceback
+        q.put((rank, False, traceback.format_exc() + repr(e)))
+
+
+def test_zero_copy_three_ranks_64mib_complete():
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+    import torch.multiprocessing as mp
+    n, mib = 3, 64
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _port()
+    procs = [ctx.Process(target=_big_worker, args=(r, n, port, mib, q)) for r in range(n)]
+    for p in procs:
+        p.start()
+    out = {}
+    try:
+        for _ in range(n):
+            r, ok, msg = q.get(timeout=900)
             out[r] = (ok, msg)
     finally:
         for p in procs:

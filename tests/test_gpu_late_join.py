@@ -3,9 +3,11 @@
 Deterministic cases: the late ranks signal before phase 1 (every piece folds
 them) or never (phase 2 adds them all).  Racing case: a late rank signals from
 a side stream while phase 1 runs; the inclusion is then timing-dependent, so
-each output element must match the oracle for SOME inclusion set, with the
-same set explaining both the phase-1 and the final value (the oracle never
-consumes the GPU's decisions); int32 finals are exact."""
+every work piece (the plan's unit of inclusion, from adapcc_plan_items) must
+match the oracle for ONE inclusion set, the same set explaining both the
+phase-1 and the final value of all its elements (the oracle never consumes
+the GPU's decisions), and the race must produce a mixed outcome; int32
+finals are exact."""
 
 import itertools
 
@@ -68,45 +70,109 @@ def test_late_join_deterministic(engine, dtype, case):
     comm.finalize()
 
 
+def _piece_ranges(text, count, dtype, R, grid, engine):
+    """Element ranges [a, b) of the work pieces of the LATE_JOIN plan the
+    kernel runs (same grid, same item cutting): the unit of inclusion."""
+    mask = sum(1 << r for r in R)
+    items, tasks = pkg.adapcc.plan_items(text, count, dtype, mask, grid, tma=engine == 1, late="join")
+    t = tasks[items["task"]]
+    a = t["lo"] + items["chunk"].astype(np.uint64) * t["chunk_elems"] + items["off"]
+    return np.stack([a, a + items["len"]], axis=1).astype(np.int64)
+
+
 @pytest.mark.parametrize("engine", [0, 1])
 @pytest.mark.parametrize("dtype", ["f32", "i32"])
 def test_late_join_racing_signal(engine, dtype):
-    n, count = 8, 4_000_003
+    """Rank 3 signals from a side stream while phase 1 runs.  Per work piece
+    (chunks "with the same offset" join), ONE inclusion set must
+    explain every element of the piece in both phases; across lags the race
+    must produce a mixed outcome (some pieces with rank 3, some without)."""
+    n, count, grid = 8, 4_000_003, 128
     R, late = {0, 1, 2, 4, 5, 7}, [3, 6]
     text = G.allreduce_stars(n, chunk=65536)
     xs = rank_tensors(dtype, count, n)
     comm = _comm(n, engine)
+    comm.config("max_ctas", grid)       # the piece cut below uses the same grid
     comm.set_strategy("allreduce", text)
     dx = [to_dev(x, dtype) for x in xs]
     dy = [empty_dev(count, dtype) for _ in range(n)]
     comm.allreduce_lb(dx, dy)  # warm-up (plans, clocks)
     torch.cuda.synchronize()
-    side = torch.cuda.Stream()
-    main = torch.cuda.current_stream()
-    t = comm.late_ticket() + 1
-    start = torch.cuda.Event()
-    start.record(main)
-    side.wait_event(start)
-    with torch.cuda.stream(side):
-        torch.cuda._sleep(20_000)          # rank 3 finishes "compute" while phase 1 runs
-        comm.signal_ready(3, ticket=t, stream=side)
-    comm.allreduce_lb(dx, dy, ready=R, late="join")
-    y1 = [to_host(y, dtype) for y in dy]
-    comm.allreduce_lb(dx, dy, ready=R, late="complement")
-    torch.cuda.synchronize()
-    y2 = [to_host(y, dtype) for y in dy]
-    assert comm.get_async_error() == 0
-    for g in range(1, n):                   # broadcast identity
-        assert np.array_equal(bits(y1[g]), bits(y1[0])) and np.array_equal(bits(y2[g]), bits(y2[0]))
+    pieces = _piece_ranges(text, count, dtype, R, grid, engine)
+    covered = np.zeros(count, np.int32)
+    for a, b in pieces:
+        covered[a:b] += 1
+    assert (covered == 1).all(), "pieces must tile the tensor"
     options = [set(c) for k in range(3) for c in itertools.combinations(late, k)]
-    ok = np.zeros(count, bool)
+    expect = []
     for L in options:
         p1 = oc.allreduce_late(xs, text, R, dtype, L, phase=1)[0]
         p2 = oc.allreduce_late(xs, text, R, dtype, L, phase=2, y_prev=[p1])[0]
-        ok |= (bits(y1[0]) == bits(p1)) & (bits(y2[0]) == bits(p2))
-    assert ok.all(), f"{(~ok).sum()} elements not explained by any inclusion set"
-    if dtype == "i32":
-        assert np.array_equal(y2[0], oc.allreduce_exact(xs, set(range(n)), "i32"))
+        expect.append((bits(p1), bits(p2)))
+    side = torch.cuda.Stream()
+    main = torch.cuda.current_stream()
+    outcomes = set()
+    for lag in (2_000, 10_000, 20_000, 40_000, 80_000, 160_000):
+        t = comm.late_ticket() + 1
+        start = torch.cuda.Event()
+        start.record(main)
+        side.wait_event(start)
+        with torch.cuda.stream(side):
+            torch.cuda._sleep(lag)             # rank 3 finishes "compute" while phase 1 runs
+            comm.signal_ready(3, ticket=t, stream=side)
+        comm.allreduce_lb(dx, dy, ready=R, late="join")
+        y1 = [to_host(y, dtype) for y in dy]
+        comm.allreduce_lb(dx, dy, ready=R, late="complement")
+        torch.cuda.synchronize()
+        y2 = [to_host(y, dtype) for y in dy]
+        assert comm.get_async_error() == 0
+        for g in range(1, n):                   # broadcast identity
+            assert np.array_equal(bits(y1[g]), bits(y1[0])) and np.array_equal(bits(y2[g]), bits(y2[0]))
+        match = [(bits(y1[0]) == e1) & (bits(y2[0]) == e2) for e1, e2 in expect]
+        csum = [np.concatenate([[0], np.cumsum(m)]) for m in match]
+        for a, b in pieces:
+            fits = [k for k in range(len(options)) if csum[k][b] - csum[k][a] == b - a]
+            assert fits, f"piece [{a},{b}) not explained by one inclusion set (lag {lag})"
+            outcomes.add(3 in options[fits[0]] if len(fits) == 1 else None)
+        if dtype == "i32":
+            assert np.array_equal(y2[0], oc.allreduce_exact(xs, set(range(n)), "i32"))
+        if True in outcomes and False in outcomes:
+            break
+    assert True in outcomes and False in outcomes, f"no mixed outcome in any lag: {outcomes}"
+    comm.finalize()
+
+
+@pytest.mark.parametrize("engine", [0, 1])
+def test_late_join_interleaved_plans(engine):
+    """Phase-1 / phase-2 pairs of two plans interleave on one stream
+    (phase 1 A, phase 1 B, phase 2 A, phase 2 B): each phase 2 complements
+    its own plan's phase 1.  A second phase 2 adds nothing."""
+    n = 8
+    R, late = {0, 1, 2, 4, 5, 7}, [3, 6]
+    text = G.allreduce_stars(n, chunk=65536)
+    comm = _comm(n, engine)
+    comm.set_strategy("allreduce", text)
+    cA, cB = 1_000_003, 600_011
+    xA, xB = rank_tensors("i32", cA, n), rank_tensors("i32", cB, n, base=1500)
+    dA, dB = [to_dev(x, "i32") for x in xA], [to_dev(x, "i32") for x in xB]
+    yA, yB = [empty_dev(cA, "i32") for _ in range(n)], [empty_dev(cB, "i32") for _ in range(n)]
+    tA = comm.late_ticket() + 1
+    comm.signal_ready(3, ticket=tA)             # rank 3 joins A's phase 1, not B's (ticket tA + 1)
+    comm.allreduce_lb(dA, yA, ready=R, late="join")
+    comm.allreduce_lb(dB, yB, ready=R, late="join")
+    torch.cuda.synchronize()
+    eA1 = oc.allreduce_late(xA, text, R, "i32", {3}, phase=1)
+    eB1 = oc.allreduce_late(xB, text, R, "i32", set(), phase=1)
+    assert all(np.array_equal(to_host(y, "i32"), e) for y, e in zip(yA, eA1))
+    assert all(np.array_equal(to_host(y, "i32"), e) for y, e in zip(yB, eB1))
+    comm.allreduce_lb(dA, yA, ready=R, late="complement")
+    comm.allreduce_lb(dB, yB, ready=R, late="complement")
+    comm.allreduce_lb(dA, yA, ready=R, late="complement")   # nothing left to add
+    torch.cuda.synchronize()
+    assert comm.get_async_error() == 0
+    fA, fB = oc.allreduce_exact(xA, set(range(n)), "i32"), oc.allreduce_exact(xB, set(range(n)), "i32")
+    assert all(np.array_equal(to_host(y, "i32"), fA) for y in yA)
+    assert all(np.array_equal(to_host(y, "i32"), fB) for y in yB)
     comm.finalize()
 
 
