@@ -303,7 +303,12 @@ ADAPCC_API const char* adapcc_last_cuda_error(void);
  * env ADAPCC_PDL), "first_blob" (LDG fold kernel: 1 = item descriptors as per-item blobs,
  * default; 0 = plain item/task/ref tables; env ADAPCC_FIRST_BLOB; env only: ADAPCC_TMA_SHAPE
  * forces the TMA ring of every TMA launch, 1 = 1 CTA/SM x 3 x 64 KiB, 2 = 2 CTAs/SM x 3 x 32 KiB,
- * 0 = automatic, default: ACCUMULATE and STAGED plans 2, others 1), "trace" (in-kernel trace capacity in
+ * 0 = automatic, default: STAGED plans (and ACCUMULATE plans with acc_red off) 2, others 1),
+ * "acc_red" (TMA kernel, accumulating destinations -- ACCUMULATE phase 2, LATE_COMPLEMENT: 1 = the
+ * folded tile leaves the stage by TMA bulk reduce-adds, recv += result performed in L2
+ * (cp.reduce.async.bulk .add, fp32 / bf16 round to nearest even without flushing subnormals,
+ * int32 wraps), default; 0 = recv tiles are TMA-loaded into the stage, added in shared memory
+ * and bulk-stored; env ADAPCC_ACC_RED; a change empties the plan cache), "trace" (in-kernel trace capacity in
  * records, 0 = off, default; see adapcc_trace_read), "debug_check" (multi-process: 1 = every launch first compares a hash
  * of its call -- collective, strategy, count, dtype, mask, flags, live ranks, segment, zero-copy
  * registrations -- with every live peer's for the same launch, in the arena headers, before any

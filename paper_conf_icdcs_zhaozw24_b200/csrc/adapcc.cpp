@@ -171,6 +171,7 @@ struct adapcc_comm_s {
   unsigned* trace_n = nullptr;
   uint32_t trace_cap = 0;
   int64_t pdl = 1;        // programmatic dependent launch of the engine kernels (ADAPCC_PDL)
+  int64_t acc_red = 1;    // TMA kernel: recv += result by bulk reduce-add in L2 (ADAPCC_ACC_RED)
   int64_t sched = 2;      // LDG kernel: 0 dynamic claims, 1 static blob schedule, 2 auto (ADAPCC_SCHED)
   uint64_t launches = 0;
   int num_sms = 148;
@@ -219,6 +220,7 @@ adapcc_result_t common_init(adapcc_comm_s* c, size_t scratch) {
   c->first_blob = env_int("ADAPCC_FIRST_BLOB", 1) != 0;
   c->tma_shape = env_int("ADAPCC_TMA_SHAPE", 0);
   c->pdl = env_int("ADAPCC_PDL", 1) != 0;
+  c->acc_red = env_int("ADAPCC_ACC_RED", 1) != 0;
   c->sched = std::min<int64_t>(2, std::max<int64_t>(0, env_int("ADAPCC_SCHED", 2)));
   CK(cudaSetDevice(c->device));
   CK(cudaDeviceGetAttribute(&c->num_sms, cudaDevAttrMultiProcessorCount, c->device));
@@ -391,11 +393,12 @@ adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, const Strategy* strat, uin
     for (auto& sp : segs) accumulate_stats(sp, c->loopback ? -1 : c->rank, rq.esize, &st);
     const uint64_t traffic = st.bytes_read + st.bytes_written;
     plan->engine = c->engine != 2 ? c->engine : (traffic / std::max<size_t>(1, segs.size()) >= kTmaMinTraffic ? 1 : 0);
-    // ACCUMULATE (phase 2) stages nsrc + nacc tiles per ring slot and is
-    // latency-bound: the 2 CTAs/SM x 3 x 32 KiB shape of the STAGED
-    // instantiation beats 1 x 3 x 64 KiB on DIRECT plans too
-    // (profiles/acc_variants_r01.json: 256 MiB/rank 868 -> 801 us).
-    plan->kernel = plan->engine == 0 ? 0 : (mode == kDirect && !rq.accumulate ? 1 : 2);
+    // ACCUMULATE (phase 2): with bulk reduce-adds (acc_red, default) a stage
+    // holds only the sources and DIRECT plans keep the 1 x 3 x 64 KiB ring
+    // (profiles/acc_r02.json); the shared-memory read-modify-write (acc_red
+    // off) stages nsrc + nacc tiles per slot and is latency-bound, where the
+    // 2 CTAs/SM x 3 x 32 KiB shape wins (profiles/acc_variants_r01.json).
+    plan->kernel = plan->engine == 0 ? 0 : (mode == kDirect && (!rq.accumulate || c->acc_red) ? 1 : 2);
     if (plan->kernel != 0 && (c->tma_shape == 1 || c->tma_shape == 2)) plan->kernel = (int)c->tma_shape;
   }
   for (auto& sp : segs) {
@@ -530,6 +533,7 @@ adapcc_result_t run(adapcc_comm_s* c, Coll coll, const void* const* send, void* 
     P.ipc = c->loopback ? 0 : 1;
     P.zc = zc ? 1 : 0;
     P.late_mode = late_mode;
+    P.acc_red = c->acc_red ? 1 : 0;
     P.late_ticket = c->late_seq;
     P.late_bits = seg.late_bits;
     P.late_list = seg.late_list;
@@ -557,10 +561,10 @@ adapcc_result_t run(adapcc_comm_s* c, Coll coll, const void* const* send, void* 
       }
       P.hdr[q] = c->arena[q];
     }
-    // phase 2 of a late join accumulates into every destination: on the TMA
-    // engine it takes the ACCUMULATE shape (2 x 3 x 32 KiB) whatever the plan's
-    // kernel; item order is grid-independent, so the plan is shared
-    const int kernel = (late_mode == 2 && plan->kernel == 1 && c->tma_shape != 1) ? 2 : plan->kernel;
+    // phase 2 of a late join accumulates into every destination: without
+    // acc_red it takes the ACCUMULATE shape (2 x 3 x 32 KiB) whatever the
+    // plan's kernel; item order is grid-independent, so the plan is shared
+    const int kernel = (late_mode == 2 && plan->kernel == 1 && !c->acc_red && c->tma_shape != 1) ? 2 : plan->kernel;
     const int grid = std::max(1, std::min<int>(grid_size(c, dtype, kernel), (int)std::max<uint32_t>(1, seg.nitems)));
     const bool pdl = c->pdl != 0;
     CK(kernel == 1 ? tma_direct::launch(P, grid, s, pdl)
@@ -1200,6 +1204,10 @@ adapcc_result_t adapcc_config(adapcc_comm_t c, const char* key, int64_t value) {
   }
   else if (!std::strcmp(key, "debug_check")) c->check_sig = value != 0;
   else if (!std::strcmp(key, "pdl")) c->pdl = value != 0;
+  else if (!std::strcmp(key, "acc_red")) {
+    if ((value != 0) != (c->acc_red != 0)) drop_plans(c);  // the TMA ring shape of ACCUMULATE plans depends on it
+    c->acc_red = value != 0;
+  }
   else if (!std::strcmp(key, "trace")) {  // capacity in records; 0 = off
     if (value < 0 || value > (int64_t(1) << 26)) return ADAPCC_ERR_INVALID_ARGUMENT;
     if (cudaSetDevice(c->device) != cudaSuccess || cudaDeviceSynchronize() != cudaSuccess) return ADAPCC_ERR_CUDA;

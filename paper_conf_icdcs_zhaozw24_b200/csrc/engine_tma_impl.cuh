@@ -74,6 +74,7 @@ struct ItemDesc {
   uint8_t acc[kMaxDst];
   uint8_t stop, dropped, scalar_only, any_acc;
   uint8_t acc_tma;            // accumulating destinations are loaded by TMA and stored from the stage
+  uint8_t acc_red;            // accumulating destinations take bulk reduce-adds of the folded tile
   uint8_t acc_slot[kMaxDst];  // acc_tma: stage tile of destination k's recv (0 = plain destination)
   uint32_t item;        // trace: item index, claim and inputs-ready times
   uint64_t tr0, tr1;
@@ -135,6 +136,30 @@ __device__ __forceinline__ void tma_store(void* gdst, const void* ssrc, uint32_t
   asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(gdst), "r"(su32(ssrc)),
                "r"(bytes)
                : "memory");
+}
+// TMA bulk reduction shared -> global: dst[i] = dst[i] + src[i], performed
+// by the memory system (L2) as one read-modify-write per element -- recv +=
+// result without bringing recv into the SM (SASS UBLKRED ... .RN).  fp32 adds
+// round to nearest even, bf16 (.noftz) rounds the exact sum once to bf16
+// (reading Q6), int32 wraps (.u32 add = the same bits as .s32).
+template <int DT>
+__device__ __forceinline__ void tma_red_add(void* gdst, const void* ssrc, uint32_t bytes) {
+  if constexpr (DT == kF32)
+    asm volatile("cp.reduce.async.bulk.global.shared::cta.bulk_group.add.f32 [%0], [%1], %2;" ::"l"(gdst),
+                 "r"(su32(ssrc)), "r"(bytes) : "memory");
+  else if constexpr (DT == kBF16)
+    asm volatile("cp.reduce.async.bulk.global.shared::cta.bulk_group.add.noftz.bf16 [%0], [%1], %2;" ::"l"(gdst),
+                 "r"(su32(ssrc)), "r"(bytes) : "memory");
+  else
+    asm volatile("cp.reduce.async.bulk.global.shared::cta.bulk_group.add.u32 [%0], [%1], %2;" ::"l"(gdst),
+                 "r"(su32(ssrc)), "r"(bytes) : "memory");
+}
+// one destination tile leaves the stage: plain bulk store, or bulk reduce-add
+// into an accumulating destination (acc_red)
+template <int DT>
+__device__ __forceinline__ void tma_put(void* gdst, const void* ssrc, uint32_t bytes, bool acc) {
+  if (acc) tma_red_add<DT>(gdst, ssrc, bytes);
+  else tma_store(gdst, ssrc, bytes);
 }
 __device__ __forceinline__ void tma_store_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
 template <int N>
@@ -257,6 +282,7 @@ __device__ __forceinline__ void consume_copy(Smem& sm, char* stages, const ItemD
 // thread waits for each loaded stage and issues the D bulk stores straight
 // from shared memory; a stage is released once its stores have read it.
 // Other consumer threads only advance their ring position.
+template <int DT>
 __device__ __forceinline__ void copy_tma(Smem& sm, char* stages, const ItemDesc& d, int tid,
                                          uint32_t& stage, uint32_t& sphase) {
   if (tid == 0) {
@@ -265,7 +291,7 @@ __device__ __forceinline__ void copy_tma(Smem& sm, char* stages, const ItemDesc&
       const uint32_t tb = min(d.tile, d.vec_bytes - t * d.tile);
       mbar_wait(&sm.full[stage], sphase);
       const char* sb = stages + (size_t)stage * kStageBytes;
-      for (int k = 0; k < d.ndst; ++k) tma_store(d.dst[k] + (size_t)t * d.tile, sb, tb);
+      for (int k = 0; k < d.ndst; ++k) tma_put<DT>(d.dst[k] + (size_t)t * d.tile, sb, tb, d.acc[k]);
       tma_store_commit();
       if (prev >= 0) {
         tma_store_wait_read<1>();
@@ -372,7 +398,7 @@ __device__ __forceinline__ void consume_fold_tma(Smem& sm, char* stages, const I
     fence_proxy_async_smem();
     consumer_sync();  // the whole folded tile is in shared memory
     if (tid == 0) {
-      for (int k = 0; k < ndst; ++k) tma_store(d.dst[k] + (size_t)t * tile, sb, tb);
+      for (int k = 0; k < ndst; ++k) tma_put<DT>(d.dst[k] + (size_t)t * tile, sb, tb, d.acc[k]);
       tma_store_commit();
       if (prev >= 0) {
         tma_store_wait_read<1>();
@@ -436,6 +462,37 @@ __device__ __forceinline__ void consume_fold(Smem& sm, char* stages, const ItemD
       const uint32_t v = tid + j * kConsumers;
       if (v < nv) store_result<DT>(d, (size_t)t * d.tile + (size_t)v * 16, O::narrow(a[j]));  // one rounding
     }
+  }
+}
+
+// Single-pass fold whose tile is larger than one register round: every tile
+// is folded round by round (fold_rounds) while its stage is held.
+template <int DT>
+__device__ __forceinline__ void consume_fold_held(Smem& sm, char* stages, const ItemDesc& d, int tid,
+                                                  uint32_t& stage, uint32_t& sphase) {
+  for (uint32_t t = 0; t < d.ntiles; ++t) {
+    const uint32_t nv = min(d.tile, d.vec_bytes - t * d.tile) / 16;
+    mbar_wait(&sm.full[stage], sphase);
+    fold_rounds<DT>(stages + (size_t)stage * kStageBytes, d, tid, t, nv);
+    __syncwarp();
+    if ((tid & 31) == 0) mbar_arrive(&sm.empty[stage]);
+    if (++stage == kStages) { stage = 0; sphase ^= 1; }
+  }
+}
+
+// One-source item with generic-proxy destinations (accumulation without
+// acc_red / acc_tma): every tile is copied round by round while its stage is
+// held (rare path, kept small so it does not set the kernel's register budget)
+template <int DT>
+__device__ __forceinline__ void consume_copy_held(Smem& sm, char* stages, const ItemDesc& d, int tid,
+                                                  uint32_t& stage, uint32_t& sphase) {
+  for (uint32_t t = 0; t < d.ntiles; ++t) {
+    const uint32_t nv = min(d.tile, d.vec_bytes - t * d.tile) / 16;
+    mbar_wait(&sm.full[stage], sphase);
+    copy_rounds<DT>(stages + (size_t)stage * kStageBytes, d, tid, t, nv);
+    __syncwarp();
+    if ((tid & 31) == 0) mbar_arrive(&sm.empty[stage]);
+    if (++stage == kStages) { stage = 0; sphase ^= 1; }
   }
 }
 
@@ -516,7 +573,10 @@ __device__ __forceinline__ void fill_desc(const LaunchParams& P, char* const (*b
     // happens in shared memory and leaves by bulk stores.
     int nacc = 0;
     for (int k = 0; k < t.ndst; ++k) nacc += d.acc[k] ? 1 : 0;
-    d.acc_tma = kFoldTma && nacc > 0 && !d.scalar_only && nsrc >= 1 && nsrc <= kMaxKS &&
+    // accumulating destinations by bulk reduce-add (default): the stage holds
+    // only the sources; the folded tile goes to every destination by TMA
+    d.acc_red = kFoldTma && P.acc_red && nacc > 0 && !d.scalar_only && nsrc >= 1 && nsrc <= kMaxKS;
+    d.acc_tma = kFoldTma && !d.acc_red && nacc > 0 && !d.scalar_only && nsrc >= 1 && nsrc <= kMaxKS &&
                 nsrc + nacc <= kMaxAccTiles;
     if (d.acc_tma) {
       int j = 0;
@@ -531,7 +591,14 @@ __device__ __forceinline__ void fill_desc(const LaunchParams& P, char* const (*b
 }
 
 template <int DT>
-__global__ void __launch_bounds__(kTmaThreads, ADAPCC_TMA_MINB) engine_tma_kernel(const __grid_constant__ LaunchParams P) {
+#ifdef ADAPCC_TMA_MAXNREG
+// explicit register budget: __launch_bounds__(288, 2) alone makes ptxas cap
+// at 96 registers and spill, although 112 x 288 x 2 fits the register file
+__global__ void __maxnreg__(ADAPCC_TMA_MAXNREG)
+#else
+__global__ void __launch_bounds__(kTmaThreads, ADAPCC_TMA_MINB)
+#endif
+engine_tma_kernel(const __grid_constant__ LaunchParams P) {
   extern __shared__ __align__(128) unsigned char smem_raw[];
   Smem& sm = *reinterpret_cast<Smem*>(smem_raw);
   char* stages = reinterpret_cast<char*>(smem_raw) + kSmemHeader;
@@ -681,7 +748,12 @@ __global__ void __launch_bounds__(kTmaThreads, ADAPCC_TMA_MINB) engine_tma_kerne
             const int ks = min((int)d.ks, (int)d.nsrc - p * (int)d.ks);
             // every issuing lane acquires the stage's release (its TMA load
             // overwrites what the consumers read); lane 0 arms the tx count
+#ifndef ADAPCC_LANE0_EMPTY_WAIT
             mbar_wait(&sm.empty[stage], sphase ^ 1);
+#else
+            if (lane == 0) mbar_wait(&sm.empty[stage], sphase ^ 1);
+            __syncwarp();
+#endif
             if (lane == 0) {
               int nacc = 0;
               if (d.acc_tma)
@@ -723,15 +795,28 @@ __global__ void __launch_bounds__(kTmaThreads, ADAPCC_TMA_MINB) engine_tma_kerne
           if (!d.scalar_only) {
             const uint32_t vpt = d.tile / (16u * kConsumers);  // tile / one round of 1 vector per thread
             if (d.acc_tma) consume_acc_tma<DT>(sm, stages, d, tid, stage, sphase);
-            else if (d.nsrc == 1 && !d.any_acc) copy_tma(sm, stages, d, tid, stage, sphase);
+            else if (d.nsrc == 1 && (!d.any_acc || d.acc_red)) copy_tma<DT>(sm, stages, d, tid, stage, sphase);
+            else if (d.acc_red) consume_fold_tma<DT>(sm, stages, d, tid, stage, sphase);
             // TMA-stored fold where per-thread stores are the cost: tiles above 16 KiB (K = 2, 3 in
             // 64 KiB stages, else fold_rounds; G1 k = 2: 0.86 -> 1.02 of the copy peak) or >= 3
             // destinations (star roots); with 1-2 destinations of small tiles the register path,
             // which frees the stage before storing, is as fast or faster (G1 k = 8: 1.08 vs 1.04)
             else if (kFoldTma && !d.any_acc && d.passes == 1 && (d.tile > 16384 || d.ndst >= 3))
               consume_fold_tma<DT>(sm, stages, d, tid, stage, sphase);
-            else if (d.nsrc == 1) consume_copy<DT, 8>(sm, stages, d, tid, stage, sphase);
-            else if (vpt >= 4) consume_fold<DT, 4>(sm, stages, d, tid, stage, sphase);
+            else if (d.nsrc == 1) {
+              // (32 KiB stages: the 8-vector register round of consume_copy set the whole
+              // kernel's register budget and made it spill at 2 CTAs/SM -- 96 registers)
+              if constexpr (kLargeTiles) consume_copy<DT, 8>(sm, stages, d, tid, stage, sphase);
+              else consume_copy_held<DT>(sm, stages, d, tid, stage, sphase);
+            }
+            else if (vpt >= 4) {
+              if constexpr (DT == kBF16) {  // 4 x 8 fp32 accumulators per thread spill at 2 CTAs/SM
+                if (!d.any_acc) consume_fold_tma<DT>(sm, stages, d, tid, stage, sphase);
+                else consume_fold_held<DT>(sm, stages, d, tid, stage, sphase);
+              } else {
+                consume_fold<DT, 4>(sm, stages, d, tid, stage, sphase);
+              }
+            }
             else if (vpt >= 2) consume_fold<DT, 2>(sm, stages, d, tid, stage, sphase);
             else consume_fold<DT, 1>(sm, stages, d, tid, stage, sphase);
           }

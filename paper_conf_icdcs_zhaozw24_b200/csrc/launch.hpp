@@ -65,6 +65,7 @@ struct LaunchParams {
   int ipc;              // 1: multi-process (.sys scope, start check, done publish)
   int zc;               // 1: zero-copy DIRECT plan across processes (entry/exit barriers)
   int late_mode;        // 0: off; 1: late join (phase 1); 2: complement (phase 2)
+  int acc_red;          // TMA kernel: accumulating destinations by bulk reduce-add (else smem read-modify-write)
   uint64_t late_ticket; // ready word value that admits a late rank (phase 1)
   uint64_t* late_bits;  // per work item: late candidates included in phase 1
   // Phase 1 lists the items that missed a late rank (late_list[i], i < count)

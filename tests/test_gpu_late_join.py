@@ -109,22 +109,34 @@ def test_late_join_racing_signal(engine, dtype):
         p1 = oc.allreduce_late(xs, text, R, dtype, L, phase=1)[0]
         p2 = oc.allreduce_late(xs, text, R, dtype, L, phase=2, y_prev=[p1])[0]
         expect.append((bits(p1), bits(p2)))
-    side = torch.cuda.Stream()
-    main = torch.cuda.current_stream()
+    from cuda.bindings import driver as cu
+    # explicit streams only: a stream memory op on the legacy default stream
+    # would wait for the side stream, which waits for it (deadlock)
+    side, main = torch.cuda.Stream(), torch.cuda.Stream()
+    main.wait_stream(torch.cuda.current_stream())
     outcomes = set()
     for lag in (2_000, 10_000, 20_000, 40_000, 80_000, 160_000):
         t = comm.late_ticket() + 1
-        start = torch.cuda.Event()
-        start.record(main)
-        side.wait_event(start)
+        # the lag starts when phase 1 is next on the main stream: the side
+        # stream waits (stream memory op) for a word main writes right before
+        # launching phase 1, sleeps `lag` cycles, then rank 3 signals
+        go = torch.zeros(4, dtype=torch.int32, device="cuda")
+        torch.cuda.synchronize()
+        (e,) = cu.cuStreamWaitValue32(cu.CUstream(side.cuda_stream), cu.CUdeviceptr(go.data_ptr()), 1,
+                                      cu.CUstreamWaitValue_flags.CU_STREAM_WAIT_VALUE_GEQ)
+        assert e == cu.CUresult.CUDA_SUCCESS, e
         with torch.cuda.stream(side):
             torch.cuda._sleep(lag)             # rank 3 finishes "compute" while phase 1 runs
             comm.signal_ready(3, ticket=t, stream=side)
-        comm.allreduce_lb(dx, dy, ready=R, late="join")
+        (e,) = cu.cuStreamWriteValue32(cu.CUstream(main.cuda_stream), cu.CUdeviceptr(go.data_ptr()), 1, 0)
+        assert e == cu.CUresult.CUDA_SUCCESS, e
+        comm.allreduce_lb(dx, dy, ready=R, late="join", stream=main)
+        main.synchronize()
         y1 = [to_host(y, dtype) for y in dy]
-        comm.allreduce_lb(dx, dy, ready=R, late="complement")
-        torch.cuda.synchronize()
+        comm.allreduce_lb(dx, dy, ready=R, late="complement", stream=main)
+        main.synchronize()
         y2 = [to_host(y, dtype) for y in dy]
+        side.synchronize()
         assert comm.get_async_error() == 0
         for g in range(1, n):                   # broadcast identity
             assert np.array_equal(bits(y1[g]), bits(y1[0])) and np.array_equal(bits(y2[g]), bits(y2[0]))
@@ -139,6 +151,7 @@ def test_late_join_racing_signal(engine, dtype):
         if True in outcomes and False in outcomes:
             break
     assert True in outcomes and False in outcomes, f"no mixed outcome in any lag: {outcomes}"
+    torch.cuda.synchronize()
     comm.finalize()
 
 

@@ -117,17 +117,20 @@ def test_c1_config_bit_exact(mode, engine):
     comm.finalize()
 
 
+@pytest.mark.parametrize("acc_red", [1, 0])
 @pytest.mark.parametrize("mode", MODES)
 @pytest.mark.parametrize("dtype", ["f32", "bf16", "i32"])
 @pytest.mark.parametrize("engine", ENGINES)
-def test_phase1_phase2_accumulate(mode, dtype, engine):
-    """C3 shape (reduced): stragglers {3,6} relay in phase 1, join with ACCUMULATE."""
+def test_phase1_phase2_accumulate(mode, dtype, engine, acc_red):
+    """C3 shape (reduced): stragglers {3,6} relay in phase 1, join with ACCUMULATE
+    (TMA kernel: bulk reduce-add into recv, or the shared-memory read-modify-write)."""
     n, count = 8, 65_537
     R1, R2 = {0, 1, 2, 4, 5, 7}, {3, 6}
     xs = rank_tensors(dtype, count, n)
     t1 = G.allreduce_mask_aware_stars(n, R1, chunk=8192)
     t2 = G.allreduce_mask_aware_stars(n, R2, chunk=8192)
     comm = _comm(n, mode, engine=engine)
+    comm.config("acc_red", acc_red)
     comm.set_strategy("allreduce", t1)
     y1 = _run_allreduce(comm, [x if r in R1 else None for r, x in enumerate(xs)], dtype, R1)
     e1 = oc.allreduce(xs, t1, R1, dtype)
@@ -327,4 +330,48 @@ def test_tma_large_items(mode, dtype, n):
         exp1 = oc.allreduce(xs, text, R1, dtype)
         _assert_bits(got, oc.allreduce(xs, text, {0}, dtype, accumulate=True, y_prev=exp1), f"large-acc/{n}/{mode}")
     assert comm.last_engine() == 1
+    comm.finalize()
+
+
+def _subnormal_case(dtype, count, rng):
+    """prev / x pairs whose sums are subnormal, start subnormal, or cancel to
+    +-0 (reading Q16: IEEE, no flush to zero)."""
+    if dtype == "f32":
+        tiny = np.float32(1.1754944e-38)   # smallest normal
+        prev = (rng.integers(-40, 40, count).astype(np.float32) * np.float32(2.0 ** -140)) + \
+            np.where(rng.random(count) < 0.5, tiny, -tiny).astype(np.float32)
+        x = (rng.integers(-40, 40, count).astype(np.float32) * np.float32(2.0 ** -141)) - prev * np.float32(0.75)
+        return prev.astype(np.float32), x.astype(np.float32)
+    # bf16 bit patterns: exponent field 0 or 1 (subnormal / smallest normals), random signs
+    def pat():
+        e = rng.integers(0, 2, count).astype(np.uint16) << 7
+        m = rng.integers(0, 128, count).astype(np.uint16)
+        s = (rng.integers(0, 2, count).astype(np.uint16) << 15)
+        return (s | e | m).astype(np.uint16)
+    return pat(), pat()
+
+
+@pytest.mark.parametrize("acc_red", [1, 0])
+@pytest.mark.parametrize("dtype", ["f32", "bf16"])
+@pytest.mark.parametrize("engine", ENGINES)
+def test_accumulate_subnormals_ieee(dtype, engine, acc_red):
+    """ACCUMULATE (phase 2) where recv, the result and recv + result are
+    subnormal: the engine (incl. the L2 bulk reduce-add) must not flush to
+    zero -- bit-exact with the oracle's IEEE replay (reading Q16).  K = 1
+    (single late rank) and K = 2 (two late ranks, folded first)."""
+    n, count = 3, (1 << 20) + 37
+    rng = np.random.default_rng(5)
+    prev, x1 = _subnormal_case(dtype, count, rng)
+    _, x2 = _subnormal_case(dtype, count, rng)
+    xs = [None, x1, x2]
+    text = G.allreduce_stars(n, chunk=65536)
+    comm = _comm(n, "direct", engine=engine)
+    comm.config("acc_red", acc_red)
+    comm.set_strategy("allreduce", text)
+    for R in ({1}, {1, 2}):
+        got = _run_allreduce(comm, [x if r in R else None for r, x in enumerate(xs)], dtype, R,
+                             accumulate=True, prev=[prev] * n)
+        _assert_bits(got, oc.allreduce(xs, text, R, dtype, accumulate=True, y_prev=[prev] * n),
+                     f"subnormal/{dtype}/{sorted(R)}")
+    assert comm.get_async_error() == 0
     comm.finalize()
