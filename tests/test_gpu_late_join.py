@@ -87,7 +87,7 @@ def test_late_join_racing_signal(engine, dtype):
     (chunks "with the same offset" join), ONE inclusion set must
     explain every element of the piece in both phases; across lags the race
     must produce a mixed outcome (some pieces with rank 3, some without)."""
-    n, count, grid = 8, 4_000_003, 128
+    n, count, grid = 8, 4_000_003, 32
     R, late = {0, 1, 2, 4, 5, 7}, [3, 6]
     text = G.allreduce_stars(n, chunk=65536)
     xs = rank_tensors(dtype, count, n)
@@ -109,27 +109,19 @@ def test_late_join_racing_signal(engine, dtype):
         p1 = oc.allreduce_late(xs, text, R, dtype, L, phase=1)[0]
         p2 = oc.allreduce_late(xs, text, R, dtype, L, phase=2, y_prev=[p1])[0]
         expect.append((bits(p1), bits(p2)))
-    from cuda.bindings import driver as cu
-    # explicit streams only: a stream memory op on the legacy default stream
-    # would wait for the side stream, which waits for it (deadlock)
     side, main = torch.cuda.Stream(), torch.cuda.Stream()
     main.wait_stream(torch.cuda.current_stream())
     outcomes = set()
-    for lag in (2_000, 10_000, 20_000, 40_000, 80_000, 160_000):
+    # grid 32: phase 1 runs for hundreds of microseconds, so a lag sweep lands
+    # the signal inside it despite the host's launch jitter
+    for lag in (20_000, 50_000, 100_000, 200_000, 400_000, 800_000, 1_600_000):
         t = comm.late_ticket() + 1
-        # the lag starts when phase 1 is next on the main stream: the side
-        # stream waits (stream memory op) for a word main writes right before
-        # launching phase 1, sleeps `lag` cycles, then rank 3 signals
-        go = torch.zeros(4, dtype=torch.int32, device="cuda")
-        torch.cuda.synchronize()
-        (e,) = cu.cuStreamWaitValue32(cu.CUstream(side.cuda_stream), cu.CUdeviceptr(go.data_ptr()), 1,
-                                      cu.CUstreamWaitValue_flags.CU_STREAM_WAIT_VALUE_GEQ)
-        assert e == cu.CUresult.CUDA_SUCCESS, e
+        start = torch.cuda.Event()
+        start.record(main)
+        side.wait_event(start)
         with torch.cuda.stream(side):
             torch.cuda._sleep(lag)             # rank 3 finishes "compute" while phase 1 runs
             comm.signal_ready(3, ticket=t, stream=side)
-        (e,) = cu.cuStreamWriteValue32(cu.CUstream(main.cuda_stream), cu.CUdeviceptr(go.data_ptr()), 1, 0)
-        assert e == cu.CUresult.CUDA_SUCCESS, e
         comm.allreduce_lb(dx, dy, ready=R, late="join", stream=main)
         main.synchronize()
         y1 = [to_host(y, dtype) for y in dy]
