@@ -44,11 +44,11 @@ def raw(rep):
 def main():
     tag = sys.argv[1] if len(sys.argv) > 1 else "r01"
     res = {}
-    for name in ("direct_tma", "direct_ldg", "staged_tma", "staged_ldg"):
-        key = "allreduce_loopback_" + name
-        rep = os.path.join(ROOT, "gpurun_out", f"prof_{name}_{tag}.ncu-rep")
-        if not os.path.exists(rep):
-            continue
+    import glob
+    reps = sorted(glob.glob(os.path.join(ROOT, "gpurun_out", f"prof_*_{tag}.ncu-rep")))
+    for rep in reps:
+        name = os.path.basename(rep)[len("prof_"):-len(f"_{tag}.ncu-rep")]
+        key = name if name.startswith("acc") else "allreduce_loopback_" + name
         d = raw(rep)
         t = d["gpu__time_duration.sum"]["value"]
         t_s = t * 1e-6 if d["gpu__time_duration.sum"]["unit"] == "us" else t * 1e-9 if d["gpu__time_duration.sum"]["unit"] == "ns" else t * 1e-3
@@ -57,7 +57,7 @@ def main():
                     "dram_bytes_per_launch": int(rd + wr), "dram_read": int(rd), "dram_write": int(wr),
                     "duration_s_ncu": t_s, "dram_gbs_ncu": (rd + wr) / t_s / 1e9,
                     "metrics": {k: v["value"] for k, v in d.items()}}
-    path = os.path.join(ROOT, "profiles", "ncu_summary.json")
+    path = os.path.join(ROOT, "profiles", "ncu_summary.json" if tag == "r01" else f"ncu_summary_{tag}.json")
     json.dump(res, open(path, "w"), indent=1)
     print(json.dumps(res, indent=1))
 
