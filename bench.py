@@ -157,11 +157,12 @@ class ClockSampler:
 SWEEP_SIZES = [1 << s for s in range(10, 29, 2)]   # bytes per rank: 1 KiB .. 256 MiB, x4 steps
 
 
-def time_point(fn, reduce_max=None, graph=True):
+def time_point(fn, reduce_max=None, graph=True, fn_graph=None):
     """Per-call device time (ms) of back-to-back calls, two ways: plain
     enqueue on the current stream ("ms", host enqueue included when it is the
     bottleneck) and a CUDA graph of the same calls ("ms_graph", device time
-    only).  >= ~10 ms per measurement.  reduce_max: max over ranks (N>1)."""
+    only; fn_graph, default fn, must enqueue on the current stream).
+    >= ~10 ms per measurement.  reduce_max: max over ranks (N>1)."""
     import torch
     cur = torch.cuda.current_stream()
     for _ in range(3):
@@ -191,7 +192,7 @@ def time_point(fn, reduce_max=None, graph=True):
         g = torch.cuda.CUDAGraph()
         with torch.cuda.graph(g, stream=s):
             for _ in range(iters):
-                fn()
+                (fn_graph or fn)()
     torch.cuda.synchronize()
     if reduce_max:
         reduce_max(0.0)
@@ -374,8 +375,11 @@ def run_single(args):
         for sb in [b for b in SWEEP_SIZES if b <= nbytes]:
             c = sb // es
             xs_, ys_ = [t[:c] for t in dx], [t[:c] for t in dy]
-            ms_, msg_ = time_point(lambda: comm.allreduce_lb(xs_, ys_))
+            call = comm.prepare_allreduce_lb(xs_, ys_)     # host fast path: one C call per AllReduce
+            ms_, msg_ = time_point(call, fn_graph=lambda: comm.allreduce_lb(xs_, ys_))
+            msp_, _ = time_point(lambda: comm.allreduce_lb(xs_, ys_), graph=False)
             sweep.append({"bytes_per_rank": sb, "us": round(ms_ * 1e3, 2), "us_graph": round(msg_ * 1e3, 2),
+                          "us_api": round(msp_ * 1e3, 2),
                           "busbw": round(busbw(sb, ms_ / 1e3, n), 2),
                           "busbw_graph": round(busbw(sb, msg_ / 1e3, n), 2),
                           "hbm_frac_graph": round(2 * n * sb / (msg_ / 1e3) / 1e9 / peak, 4)})
@@ -405,8 +409,10 @@ def run_single(args):
         "parity": parity,
         "nccl": None,
         "sweep": sweep,
-        "sweep_how": "same call at every x4 size (slices of the bench buffers), back-to-back enqueue (us) "
-                     "and a CUDA graph of the same calls (us_graph, device time); sizes whose 2nS fit the "
+        "sweep_how": "same call at every x4 size (slices of the bench buffers): back-to-back enqueue of a "
+                     "prepared call (us: Communicator.prepare_allreduce_lb, one C call per AllReduce), of the "
+                     "per-call API (us_api: allreduce_lb marshals its arguments every call), and a CUDA graph "
+                     "of the same calls (us_graph, device time); busbw from us; sizes whose 2nS fit the "
                      "126 MB L2 run partly from L2",
     }
     if not args.no_cpu_baseline:
@@ -623,7 +629,8 @@ def run_multi(args):
         for sb in [b for b in SWEEP_SIZES if b <= nbytes]:
             c = sb // es
             xs_, ys_, zs_ = x[:c], y[:c], z[:c]
-            ms_, msg_ = time_point(lambda: comm.collective_zc("allreduce", xs_, ys_, c), reduce_max)
+            call = comm.prepare_collective_zc("allreduce", xs_, ys_, c)
+            ms_, msg_ = time_point(call, reduce_max, fn_graph=lambda: comm.collective_zc("allreduce", xs_, ys_, c))
             pt = {"bytes_per_rank": sb, "us": round(ms_ * 1e3, 2), "us_graph": round(msg_ * 1e3, 2),
                   "busbw": round(busbw(sb, ms_ / 1e3, world), 2),
                   "busbw_graph": round(busbw(sb, msg_ / 1e3, world), 2)}

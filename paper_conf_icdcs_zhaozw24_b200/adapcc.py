@@ -317,6 +317,26 @@ def make_store_allgather(ranks, rank, store=None, tag="adapcc"):
     return AG_FN(ag)
 
 
+class PreparedCall:
+    """One collective call with its C arguments converted once (ctypes values),
+    re-enqueued by calling it: the per-call host cost is one C call
+    (Communicator.prepare_*).  Keeps references to the tensors it names."""
+
+    __slots__ = ("_fn", "_args", "_where", "_keep")
+
+    def __init__(self, fn, args, where, keep=None):
+        conv = []
+        for a, t in zip(args, fn.argtypes):
+            conv.append(a if isinstance(a, (ctypes._SimpleCData, ctypes.Array, ctypes._Pointer)) or a is None
+                        else t(a))
+        self._fn, self._args, self._where, self._keep = fn, tuple(conv), where, keep
+
+    def __call__(self):
+        code = self._fn(*self._args)
+        if code:
+            raise AdapccError(code, self._where)
+
+
 class Communicator:
     """A communicator (the paper's transmission contexts)."""
 
@@ -529,8 +549,7 @@ class Communicator:
         self._arr_cache = (key, S, D)
         return S, D
 
-    def allreduce_lb(self, xs, outs, ready=None, accumulate=False, stream=None, late=None):
-        """late: None | 'join' (phase 1) | 'complement' (phase 2)."""
+    def _allreduce_lb_args(self, xs, outs, ready, accumulate, stream, late):
         m = self._ready_mask(ready)
         if late is not None:
             # phase 2 reads the late ranks' inputs: pass every input
@@ -538,9 +557,43 @@ class Communicator:
         else:
             S, D = self._arrays(xs, outs, m)
         flags = (FLAG_ACCUMULATE if accumulate else 0) | _late_flag(late)
-        _check(_load().adapcc_allreduce_lb(self._h, S, D, outs[0].numel(), _dtype_code(outs[0]), m,
-                                           flags, _stream(stream, self.device)), "allreduce_lb")
+        return (self._h, S, D, outs[0].numel(), _dtype_code(outs[0]), m, flags, _stream(stream, self.device))
+
+    def allreduce_lb(self, xs, outs, ready=None, accumulate=False, stream=None, late=None):
+        """late: None | 'join' (phase 1) | 'complement' (phase 2)."""
+        _check(_load().adapcc_allreduce_lb(*self._allreduce_lb_args(xs, outs, ready, accumulate, stream, late)),
+               "allreduce_lb")
         return outs
+
+    # ---- prepared calls: every argument marshalled once
+    def prepare_allreduce_lb(self, xs, outs, ready=None, accumulate=False, stream=None, late=None):
+        """A persistent loopback AllReduce: the returned callable enqueues the
+        same call (same tensors, mask, flags and stream -- the current stream
+        at prepare time unless given) with one C call and no per-call
+        marshalling.  The tensors must stay alive and keep their storage."""
+        return PreparedCall(_load().adapcc_allreduce_lb,
+                            self._allreduce_lb_args(xs, outs, ready, accumulate, stream, late),
+                            "allreduce_lb", keep=(xs, outs))
+
+    def prepare_allreduce(self, x, out=None, ready=None, accumulate=False, stream=None):
+        """A persistent multi-process AllReduce (see prepare_allreduce_lb)."""
+        out = x if out is None else out
+        m = self._ready_mask(ready)
+        send = x if (m >> self.rank) & 1 else None
+        args = (self._h, _ptr(send), _ptr(out), out.numel(), _dtype_code(out), m,
+                FLAG_ACCUMULATE if accumulate else 0, _stream(stream, self.device))
+        return PreparedCall(_load().adapcc_allreduce, args, "allreduce", keep=(x, out))
+
+    def prepare_collective_zc(self, coll, x, out, count, root=0, ready=None, accumulate=False, stream=None,
+                              late=None):
+        """A persistent zero-copy collective on registered tensors (see prepare_allreduce_lb)."""
+        sr, so = self._reg_of(x)
+        rr, ro = self._reg_of(out)
+        m = self._ready_mask(ready)
+        flags = (FLAG_ACCUMULATE if accumulate else 0) | _late_flag(late)
+        args = (self._h, COLL[coll], sr, so, rr, ro, count, _dtype_code(out), root, m, flags,
+                _stream(stream, self.device))
+        return PreparedCall(_load().adapcc_collective_zc, args, coll + "_zc", keep=(x, out))
 
     def alltoallv_lb(self, xs, outs, counts, ready=None, stream=None):
         """counts: nranks x nranks element counts (counts[s][d] from s to d)."""

@@ -495,7 +495,8 @@ adapcc_result_t run(adapcc_comm_s* c, Coll coll, const void* const* send, void* 
   nvtxRangePushA(kRange[counts ? kNumColl : (int)coll]);
   struct Pop { ~Pop() { nvtxRangePop(); } } pop;
   std::lock_guard<std::mutex> lock(c->mu);
-  CK(cudaSetDevice(c->device));
+  int cur_dev = -1;  // (cudaGetDevice reads thread state; cudaSetDevice is only needed on a change)
+  if (cudaGetDevice(&cur_dev) != cudaSuccess || cur_dev != c->device) CK(cudaSetDevice(c->device));
   const Strategy* strat = nullptr;
   adapcc_result_t r = pick_strategy(c, coll, root, &strat);
   if (r != ADAPCC_SUCCESS) return r;

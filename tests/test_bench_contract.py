@@ -88,3 +88,21 @@ def test_ours_two_ranks_same_gpu_contract():
     assert d["parity"]["complete"] and d["parity"]["mismatches"] == 0 and d["parity"]["ranks"] == 2
     assert d["parity"]["ranks_mismatched"] == []
     assert [p["bytes_per_rank"] for p in d["sweep"]] == [1 << s for s in range(10, 24, 2)]
+
+
+def test_prepared_call_marshals_once():
+    """PreparedCall converts every argument to its ctypes type once (host fast
+    path); calling it re-issues exactly those arguments (CPU: a stub C function)."""
+    import ctypes
+    from paper_conf_icdcs_zhaozw24_b200.adapcc import PreparedCall
+    seen = []
+
+    @ctypes.CFUNCTYPE(ctypes.c_int, ctypes.c_void_p, ctypes.c_size_t, ctypes.c_uint64)
+    def stub(h, n, m):
+        seen.append((h, n, m))
+        return 0
+    pc = PreparedCall(stub, (ctypes.c_void_p(16), 1024, 0xFF), "stub")
+    assert all(isinstance(a, ctypes._SimpleCData) for a in pc._args)
+    pc()
+    pc()
+    assert seen == [(16, 1024, 0xFF)] * 2
