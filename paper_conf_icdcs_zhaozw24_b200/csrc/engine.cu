@@ -56,7 +56,6 @@ struct Cur {  // header of the work item being executed (staged by thread 0)
 
 struct Shared {
   uint64_t tr0, tr1;           // trace: item claimed / inputs ready
-  char* base[3][kMaxRanksDev];  // P.send / P.recv / P.hdr (indexed by BufKind), copied from the params
   uint4 blob[2][kFirstMaxWords];  // item blobs: Item | Task | refs (static schedule: double-buffered)
   Cur cur;
   const char* src[kMaxFold];
@@ -218,9 +217,10 @@ __device__ void fold_chunk(const Shared& sh, int nsrc, int ndst, uint64_t n, int
   if ((uint64_t)nvec * VE < n) fold_scalar<DT>(sh, nsrc, ndst, (uint64_t)nvec * VE, n);
 }
 
-template <int DT>
-__global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __grid_constant__ LaunchParams P) {
+template <int DT, int NR>
+__global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __grid_constant__ LaunchParamsT<NR> P) {
   __shared__ Shared sh;
+  __shared__ char* sbase[3][NR];  // P.send / P.recv / P.hdr (indexed by BufKind), copied from the params
   const bool sys = P.ipc;
   const uint64_t t_entry = P.trace ? globaltimer() : 0;
   Item pre{};  // thread 0: this CTA's first item, loaded together with the epoch
@@ -234,7 +234,7 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
   // before the stream-order wait
   for (int i = threadIdx.x; i < 3 * P.nranks; i += kThreads) {
     const int k = i / P.nranks, q = i - k * P.nranks;
-    sh.base[k][q] = k == 0 ? P.send[q] : k == 1 ? P.recv[q] : P.hdr[q];
+    sbase[k][q] = k == 0 ? P.send[q] : k == 1 ? P.recv[q] : P.hdr[q];
   }
   if (threadIdx.x == 0 && !use_blob && blockIdx.x < P.nitems) pre = P.items[blockIdx.x];
   constexpr int esize = Ops<DT>::kEsize;
@@ -298,7 +298,7 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
     const BufRef r = sh.cur.blob >= 0 ? *reinterpret_cast<const BufRef*>(&sh.blob[sh.cur.blob][kBlobRef0 + j])
                                       : P.refs[sh.cur.ref0 + j];
     const bool arena = r.kind == kBufArena;
-    char* p = sh.base[r.kind][r.rank] + (arena ? hoff : 0) + r.bias + (int64_t)(sh.cur.e0 * esize);
+    char* p = sbase[r.kind][r.rank] + (arena ? hoff : 0) + r.bias + (int64_t)(sh.cur.e0 * esize);
     if (reinterpret_cast<uintptr_t>(p) & 15) atomicOr(&sh.bad_align, 1);  // (hoff is 256-byte aligned)
     if (i < nsrc) {
       sh.src[i] = p;
@@ -415,7 +415,7 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
       if (threadIdx.x < sh.cur.nwait) {
         const FlagRef f = P.flags[sh.cur.flag0 + threadIdx.x];
         const uint64_t* fl =
-            reinterpret_cast<const uint64_t*>(sh.base[kBufArena][f.rank] + half_off + f.off) + sh.cur.chunk;
+            reinterpret_cast<const uint64_t*>(sbase[kBufArena][f.rank] + half_off + f.off) + sh.cur.chunk;
         if (!wait_flag(fl, epoch, P)) sh.abort = 1;
       }
       if (!staged) {
@@ -496,9 +496,9 @@ int engine_threads() { return kThreads; }
 
 cudaError_t engine_occupancy(int dtype, int* blocks_per_sm) {
   switch (dtype) {
-    case kF32: return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, engine_kernel<kF32>, kThreads, 0);
-    case kBF16: return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, engine_kernel<kBF16>, kThreads, 0);
-    default: return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, engine_kernel<kI32>, kThreads, 0);
+    case kF32: return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, engine_kernel<kF32, kMaxRanksDev>, kThreads, 0);
+    case kBF16: return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, engine_kernel<kBF16, kMaxRanksDev>, kThreads, 0);
+    default: return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, engine_kernel<kI32, kMaxRanksDev>, kThreads, 0);
   }
 }
 
@@ -515,13 +515,21 @@ cudaError_t engine_signal(uint64_t* word, uint64_t value, bool sys, cudaStream_t
   return cudaGetLastError();
 }
 
+namespace {
+template <int NR>
+cudaError_t launch_nr(const LaunchParamsT<NR>& p, int grid, cudaStream_t stream, bool pdl) {
+  switch (p.dtype) {
+    case kF32: return launch_kernel(engine_kernel<kF32, NR>, grid, kThreads, 0, stream, pdl, p);
+    case kBF16: return launch_kernel(engine_kernel<kBF16, NR>, grid, kThreads, 0, stream, pdl, p);
+    default: return launch_kernel(engine_kernel<kI32, NR>, grid, kThreads, 0, stream, pdl, p);
+  }
+}
+}  // namespace
+
 cudaError_t engine_launch(const LaunchParams& p, int grid, cudaStream_t stream, bool pdl) {
   cudaGetLastError();  // clear any stale error so the check below is about this launch
-  switch (p.dtype) {
-    case kF32: return launch_kernel(engine_kernel<kF32>, grid, kThreads, 0, stream, pdl, p);
-    case kBF16: return launch_kernel(engine_kernel<kBF16>, grid, kThreads, 0, stream, pdl, p);
-    default: return launch_kernel(engine_kernel<kI32>, grid, kThreads, 0, stream, pdl, p);
-  }
+  if (p.nranks <= kNarrowRanks) return launch_nr(narrow(p), grid, stream, pdl);
+  return launch_nr(p, grid, stream, pdl);
 }
 
 }  // namespace adapcc

@@ -44,7 +44,8 @@ __device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;"
 __device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
 
 // appends one trace record (tracing is a debug mode: one atomic per record)
-__device__ __forceinline__ void trace_put(const LaunchParams& P, uint32_t item, uint32_t task, uint64_t t0,
+template <class LP>
+__device__ __forceinline__ void trace_put(const LP& P, uint32_t item, uint32_t task, uint64_t t0,
                                           uint64_t t1, uint64_t t2, uint64_t bytes) {
   const unsigned i = atomicAdd(P.trace_n, 1u);
   if (i < P.trace_cap) P.trace[i] = TraceRec{P.launch_seq, blockIdx.x, item, task, t0, t1, t2, bytes};
@@ -135,7 +136,8 @@ template <> struct Ops<kI32> {
 
 
 // spin until *flag >= target; false on watchdog timeout or abort
-static __device__ __noinline__ bool wait_flag(const uint64_t* flag, uint64_t target, const LaunchParams& P) {
+template <class LP>
+static __device__ __noinline__ bool wait_flag(const uint64_t* flag, uint64_t target, const LP& P) {
   const bool sys = P.ipc;
   if (ld_acquire(flag, sys) >= target) return true;
   const uint64_t t0 = globaltimer();
@@ -161,7 +163,8 @@ static __device__ __noinline__ bool wait_flag(const uint64_t* flag, uint64_t tar
 // with every live peer's signature for the same epoch before moving any byte.
 // A mismatch latches ADAPCC_ERR_MISMATCH and raises the abort flag.  Returns
 // false on mismatch or watchdog timeout.  Called by all threads of the CTA.
-static __device__ bool check_call_sig(const LaunchParams& P, uint64_t epoch) {
+template <class LP>
+static __device__ bool check_call_sig(const LP& P, uint64_t epoch) {
   const int slot = (int)(epoch & 3);
   if (blockIdx.x == 0 && threadIdx.x == 0) {
     char* me = P.hdr[P.my_rank];
@@ -192,7 +195,8 @@ static __device__ bool check_call_sig(const LaunchParams& P, uint64_t epoch) {
 // Position of the next entry in the plan's phase-2 list for the phase-1
 // launch of `epoch`: the first append of a new launch (gen differs) restarts
 // the count at 0 (launch.hpp, late_count).
-static __device__ __forceinline__ uint32_t late_append(const LaunchParams& P, uint64_t epoch) {
+template <class LP>
+static __device__ __forceinline__ uint32_t late_append(const LP& P, uint64_t epoch) {
   const unsigned long long gen = (unsigned long long)(uint32_t)epoch;
   unsigned long long old = *reinterpret_cast<volatile unsigned long long*>(&P.late_count[0]), nw;
   for (;;) {
@@ -205,13 +209,15 @@ static __device__ __forceinline__ uint32_t late_append(const LaunchParams& P, ui
 }
 
 // Entries phase 2 runs: the list of the last completed phase 1, if any.
-static __device__ __forceinline__ uint32_t late_listed(const LaunchParams& P) {
+template <class LP>
+static __device__ __forceinline__ uint32_t late_listed(const LP& P) {
   const unsigned long long w = *reinterpret_cast<volatile unsigned long long*>(&P.late_count[0]);
   const unsigned long long g = *reinterpret_cast<volatile unsigned long long*>(&P.late_count[1]);
   return g != ~0ull && (w >> 32) == (unsigned long long)(uint32_t)g ? (uint32_t)w : 0u;
 }
 
-static __device__ __forceinline__ uint64_t late_select(const LaunchParams& P, const Task& t,
+template <class LP>
+static __device__ __forceinline__ uint64_t late_select(const LP& P, const Task& t,
                                                        uint32_t item, uint64_t epoch) {
   uint64_t m = 0;
   if (P.late_mode == 1) {
@@ -235,7 +241,8 @@ static __device__ __forceinline__ uint64_t late_select(const LaunchParams& P, co
 // candidate j (and j + 32, ...), so the ref and ready-word loads of all
 // candidates are in flight together instead of one candidate after another.
 // Same result and side effects as late_select; every lane returns the mask.
-static __device__ __forceinline__ uint64_t late_select_warp(const LaunchParams& P, const Task& t,
+template <class LP>
+static __device__ __forceinline__ uint64_t late_select_warp(const LP& P, const Task& t,
                                                             uint32_t item, int lane, uint64_t epoch) {
   const uint64_t all = t.nlate >= 64 ? ~0ull : ((1ull << t.nlate) - 1);
   if (P.late_mode == 2) return all & ~P.late_bits[item];
@@ -271,9 +278,9 @@ static __device__ __forceinline__ int nth_bit(uint64_t m, int k) {
 }  // namespace dev
 
 // Kernel launch, optionally as a programmatic dependent launch (see pdl_wait).
-template <typename Kernel>
+template <typename Kernel, class LP>
 inline cudaError_t launch_kernel(Kernel kernel, int grid, int threads, size_t smem, cudaStream_t stream,
-                                 bool pdl, const LaunchParams& p) {
+                                 bool pdl, const LP& p) {
   cudaLaunchConfig_t cfg{};
   cfg.gridDim = dim3((unsigned)grid);
   cfg.blockDim = dim3((unsigned)threads);

@@ -90,7 +90,6 @@ struct Smem {
   int pad;
   ItemDesc q[kQ];
   uint4 blob[kFirstMaxWords];  // this CTA's first item: Item | Task | refs (plan-time blob)
-  char* base[3][kMaxRanksDev];  // P.send / P.recv / P.hdr (indexed by BufKind), copied from the params
 };
 
 constexpr size_t kSmemHeader = (sizeof(Smem) + 127) / 128 * 128;
@@ -497,10 +496,10 @@ __device__ __forceinline__ void consume_copy_held(Smem& sm, char* stages, const 
 }
 
 // ------------------------------------------------------------- producer
-template <int DT>
 // R: the task's refs (R[0] = refs[t.ref0]), in global memory or in the
 // CTA's first-item blob
-__device__ __forceinline__ void fill_desc(const LaunchParams& P, char* const (*base)[kMaxRanksDev],
+template <int DT, class LP>
+__device__ __forceinline__ void fill_desc(const LP& P, char* const (*base)[LP::kRanks],
                                           ItemDesc& d, const Item& item, const Task& t, const BufRef* R,
                                           uint64_t half_off, int lane, uint32_t it, int* nwait_eff,
                                           uint64_t epoch) {
@@ -590,17 +589,17 @@ __device__ __forceinline__ void fill_desc(const LaunchParams& P, char* const (*b
   }
 }
 
-template <int DT>
+template <int DT, int NR>
 #ifdef ADAPCC_TMA_MAXNREG
-// explicit register budget: __launch_bounds__(288, 2) alone makes ptxas cap
-// at 96 registers and spill, although 112 x 288 x 2 fits the register file
+// explicit register budget (tuning only, see engine_tma_staged.cu)
 __global__ void __maxnreg__(ADAPCC_TMA_MAXNREG)
 #else
 __global__ void __launch_bounds__(kTmaThreads, ADAPCC_TMA_MINB)
 #endif
-engine_tma_kernel(const __grid_constant__ LaunchParams P) {
+engine_tma_kernel(const __grid_constant__ LaunchParamsT<NR> P) {
   extern __shared__ __align__(128) unsigned char smem_raw[];
   Smem& sm = *reinterpret_cast<Smem*>(smem_raw);
+  __shared__ char* sbase[3][NR];  // P.send / P.recv / P.hdr (indexed by BufKind), copied from the params
   char* stages = reinterpret_cast<char*>(smem_raw) + kSmemHeader;
   const int tid = threadIdx.x;
   const int warp = tid >> 5, lane = tid & 31;
@@ -628,7 +627,7 @@ engine_tma_kernel(const __grid_constant__ LaunchParams P) {
     // buffer bases into shared memory (indexed by BufKind)
     for (int i = lane; i < 3 * P.nranks; i += 32) {
       const int k = i / P.nranks, q = i - k * P.nranks;
-      sm.base[k][q] = k == 0 ? P.send[q] : k == 1 ? P.recv[q] : P.hdr[q];
+      sbase[k][q] = k == 0 ? P.send[q] : k == 1 ? P.recv[q] : P.hdr[q];
     }
     __syncwarp();
     // A plan without arena streams or flags (DIRECT: loopback and zero-copy)
@@ -637,7 +636,7 @@ engine_tma_kernel(const __grid_constant__ LaunchParams P) {
     // previous kernel.  Late join decides per item from ready words: after.
     if (use_blob && P.arena_free && P.late_mode == 0) {
       int nwait = 0;
-      fill_desc<DT>(P, sm.base, sm.q[0], *reinterpret_cast<const Item*>(&sm.blob[0]),
+      fill_desc<DT>(P, sbase, sm.q[0], *reinterpret_cast<const Item*>(&sm.blob[0]),
                     *reinterpret_cast<const Task*>(&sm.blob[1]),
                     reinterpret_cast<const BufRef*>(&sm.blob[kBlobRef0]), 0, lane, blockIdx.x, &nwait, 0);
       __syncwarp();
@@ -713,14 +712,14 @@ engine_tma_kernel(const __grid_constant__ LaunchParams P) {
         int nwait = 0;
         if (!(fb && P.arena_free && P.late_mode == 0)) {  // (else described before the wait, above)
           const BufRef* R = fb ? reinterpret_cast<const BufRef*>(&sm.blob[kBlobRef0]) : P.refs + t.ref0;
-          fill_desc<DT>(P, sm.base, d, item, t, R, half_off, lane, it, &nwait, epoch);
+          fill_desc<DT>(P, sbase, d, item, t, R, half_off, lane, it, &nwait, epoch);
           __syncwarp();
         }
         if (!d.dropped) {
           int ok = 1;
           for (int i = lane; i < nwait; i += 32) {
             const FlagRef f = P.flags[t.flag0 + i];
-            const uint64_t* fl = reinterpret_cast<const uint64_t*>(sm.base[kBufArena][f.rank] + half_off + f.off) + item.chunk;
+            const uint64_t* fl = reinterpret_cast<const uint64_t*>(sbase[kBufArena][f.rank] + half_off + f.off) + item.chunk;
             ok &= wait_flag(fl, epoch, P);
           }
           if (!__all_sync(0xffffffffu, ok)) {
@@ -869,14 +868,29 @@ engine_tma_kernel(const __grid_constant__ LaunchParams P) {
   }
 }
 
-template <int DT>
+template <int DT, int NR>
 cudaError_t prepare() {
   static bool done = false;
   if (done) return cudaSuccess;
-  cudaError_t e = cudaFuncSetAttribute(engine_tma_kernel<DT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+  cudaError_t e = cudaFuncSetAttribute(engine_tma_kernel<DT, NR>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        (int)kSmemBytes);
   done = e == cudaSuccess;
   return e;
+}
+
+template <int NR>
+cudaError_t launch_nr(const LaunchParamsT<NR>& p, int grid, cudaStream_t stream, bool pdl) {
+  switch (p.dtype) {
+    case kF32:
+      if (cudaError_t e = prepare<kF32, NR>()) return e;
+      return launch_kernel(engine_tma_kernel<kF32, NR>, grid, kTmaThreads, kSmemBytes, stream, pdl, p);
+    case kBF16:
+      if (cudaError_t e = prepare<kBF16, NR>()) return e;
+      return launch_kernel(engine_tma_kernel<kBF16, NR>, grid, kTmaThreads, kSmemBytes, stream, pdl, p);
+    default:
+      if (cudaError_t e = prepare<kI32, NR>()) return e;
+      return launch_kernel(engine_tma_kernel<kI32, NR>, grid, kTmaThreads, kSmemBytes, stream, pdl, p);
+  }
 }
 
 }  // namespace
@@ -886,30 +900,24 @@ int threads() { return kTmaThreads; }
 cudaError_t occupancy(int dtype, int* blocks_per_sm) {
   switch (dtype) {
     case kF32:
-      if (cudaError_t e = prepare<kF32>()) return e;
-      return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, engine_tma_kernel<kF32>, kTmaThreads, kSmemBytes);
+      if (cudaError_t e = prepare<kF32, kMaxRanksDev>()) return e;
+      return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, engine_tma_kernel<kF32, kMaxRanksDev>,
+                                                           kTmaThreads, kSmemBytes);
     case kBF16:
-      if (cudaError_t e = prepare<kBF16>()) return e;
-      return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, engine_tma_kernel<kBF16>, kTmaThreads, kSmemBytes);
+      if (cudaError_t e = prepare<kBF16, kMaxRanksDev>()) return e;
+      return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, engine_tma_kernel<kBF16, kMaxRanksDev>,
+                                                           kTmaThreads, kSmemBytes);
     default:
-      if (cudaError_t e = prepare<kI32>()) return e;
-      return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, engine_tma_kernel<kI32>, kTmaThreads, kSmemBytes);
+      if (cudaError_t e = prepare<kI32, kMaxRanksDev>()) return e;
+      return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, engine_tma_kernel<kI32, kMaxRanksDev>,
+                                                           kTmaThreads, kSmemBytes);
   }
 }
 
 cudaError_t launch(const LaunchParams& p, int grid, cudaStream_t stream, bool pdl) {
   cudaGetLastError();
-  switch (p.dtype) {
-    case kF32:
-      if (cudaError_t e = prepare<kF32>()) return e;
-      return launch_kernel(engine_tma_kernel<kF32>, grid, kTmaThreads, kSmemBytes, stream, pdl, p);
-    case kBF16:
-      if (cudaError_t e = prepare<kBF16>()) return e;
-      return launch_kernel(engine_tma_kernel<kBF16>, grid, kTmaThreads, kSmemBytes, stream, pdl, p);
-    default:
-      if (cudaError_t e = prepare<kI32>()) return e;
-      return launch_kernel(engine_tma_kernel<kI32>, grid, kTmaThreads, kSmemBytes, stream, pdl, p);
-  }
+  if (p.nranks <= kNarrowRanks) return launch_nr(narrow(p), grid, stream, pdl);
+  return launch_nr(p, grid, stream, pdl);
 }
 
 }  // namespace ADAPCC_TMA_NS

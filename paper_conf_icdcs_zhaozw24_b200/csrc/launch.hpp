@@ -38,7 +38,12 @@ struct TraceRec {
 static_assert(sizeof(TraceRec) == 48, "TraceRec layout");
 constexpr uint32_t kTraceCta = 0xFFFFFFFFu;
 
-struct LaunchParams {
+// Scalar part of the launch parameters; the per-rank pointer arrays follow in
+// LaunchParamsT<NR>.  Kernel parameters are copied into every launch, and a
+// launch with 1.8 KB of them costs ~1.5 us more host time than one with a few
+// bytes (scripts/debug/host_floor.cu): calls over <= 8 ranks launch the
+// kernels instantiated for 8-entry arrays.
+struct LaunchCore {
   const Task* tasks;
   const BufRef* refs;
   const FlagRef* flags;
@@ -92,10 +97,30 @@ struct LaunchParams {
   uint32_t launch_seq;
   DevState* state;
   int* err;             // host-mapped error word
-  char* send[kMaxRanksDev];
-  char* recv[kMaxRanksDev];
-  char* hdr[kMaxRanksDev];  // arena base of each rank (peer-mapped): [header | half 0 | half 1]
 };
+
+template <int NR>
+struct LaunchParamsT : LaunchCore {
+  static constexpr int kRanks = NR;
+  char* send[NR];
+  char* recv[NR];
+  char* hdr[NR];  // arena base of each rank (peer-mapped): [header | half 0 | half 1]
+};
+constexpr int kNarrowRanks = 8;
+using LaunchParams = LaunchParamsT<kMaxRanksDev>;  // what the host fills
+using LaunchParamsNarrow = LaunchParamsT<kNarrowRanks>;
+
+// the same call in the narrow parameter block (nranks <= kNarrowRanks)
+inline LaunchParamsNarrow narrow(const LaunchParams& p) {
+  LaunchParamsNarrow n;
+  static_cast<LaunchCore&>(n) = static_cast<const LaunchCore&>(p);
+  for (int q = 0; q < kNarrowRanks; ++q) {
+    n.send[q] = p.send[q];
+    n.recv[q] = p.recv[q];
+    n.hdr[q] = p.hdr[q];
+  }
+  return n;
+}
 
 // Words of the 4 KiB arena header (byte offsets).  Each rank writes only its
 // own header; peers read it over NVLink.

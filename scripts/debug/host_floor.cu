@@ -9,6 +9,10 @@
 
 #include "../../include/adapcc.h"
 
+struct Big { char b[1792]; };
+__global__ void empty_big(const __grid_constant__ Big p) { if (p.b[threadIdx.x & 1023] == 123) asm volatile("trap;"); }
+__global__ void empty_small(int x) { if (x == 123) asm volatile("trap;"); }
+
 __global__ void spin(long long cycles) {
   const long long t0 = clock64();
   while (clock64() - t0 < cycles) {
@@ -33,7 +37,7 @@ int main() {
   };
   for (int i = 0; i < 200; ++i) call();
   cudaStreamSynchronize(s);
-  const int K = 2000;
+  const int K = 300;
   // (1) host-only: stream held by a long spin kernel, K enqueues
   spin<<<1, 1, 0, s>>>(4000000000LL);
   auto t0 = std::chrono::steady_clock::now();
@@ -42,6 +46,35 @@ int main() {
   cudaStreamSynchronize(s);
   printf("host enqueue only (stream blocked): %.3f us/call\n",
          std::chrono::duration<double, std::micro>(t1 - t0).count() / K);
+  {  // host-only costs of the pieces: bookkeeping without a launch, raw launches
+    auto spin_then = [&](auto f) {
+      spin<<<1, 1, 0, s>>>(2000000000LL);
+      auto a0 = std::chrono::steady_clock::now();
+      for (int i = 0; i < K; ++i) f();
+      auto a1 = std::chrono::steady_clock::now();
+      cudaStreamSynchronize(s);
+      return std::chrono::duration<double, std::micro>(a1 - a0).count() / K;
+    };
+    printf("adapcc_allreduce_lb count=0 (no launch): %.3f us\n", spin_then([&] {
+      adapcc_allreduce_lb(c, (const void* const*)x.data(), (void* const*)y.data(), 0, ADAPCC_FLOAT32, (1u << n) - 1, 0, s);
+    }));
+    Big big{};
+    for (int pdl = 0; pdl < 2; ++pdl) {
+      cudaLaunchConfig_t cfg{};
+      cfg.gridDim = dim3(148);
+      cfg.blockDim = dim3(256);
+      cfg.stream = s;
+      cudaLaunchAttribute at[1];
+      at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+      at[0].val.programmaticStreamSerializationAllowed = 1;
+      cfg.attrs = at;
+      cfg.numAttrs = pdl;
+      printf("cudaLaunchKernelEx 1792-B param, pdl=%d: %.3f us\n", pdl,
+             spin_then([&] { cudaLaunchKernelEx(&cfg, empty_big, big); }));
+      printf("cudaLaunchKernelEx 4-B param, pdl=%d: %.3f us\n", pdl,
+             spin_then([&] { cudaLaunchKernelEx(&cfg, empty_small, 1); }));
+    }
+  }
   // (2) back to back: wall time per call incl. device execution
   cudaEvent_t a, b;
   cudaEventCreate(&a);

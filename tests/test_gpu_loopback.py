@@ -375,3 +375,31 @@ def test_accumulate_subnormals_ieee(dtype, engine, acc_red):
                      f"subnormal/{dtype}/{sorted(R)}")
     assert comm.get_async_error() == 0
     comm.finalize()
+
+
+@pytest.mark.parametrize("mode", MODES)
+@pytest.mark.parametrize("engine", ENGINES)
+@pytest.mark.parametrize("n", [9, 16, 64])
+def test_wide_rank_counts(n, mode, engine):
+    """More than 8 ranks: the kernels instantiated for 64-entry pointer arrays
+    (<= 8 ranks launch the narrow parameter block, launch.hpp)."""
+    count = 10_007
+    comm = _comm(n, mode, scratch=16 << 20, engine=engine)
+    xs = rank_tensors("i32", count, n)
+    text = G.allreduce_stars(n, chunk=8192)
+    comm.set_strategy("allreduce", text)
+    R = set(range(n)) - {n // 2}
+    got = _run_allreduce(comm, xs, "i32", R)
+    _assert_bits(got, oc.allreduce(xs, text, R, "i32"), f"wide/{n}")
+    cnt = 257
+    ag = G.allgather_stars(n, chunk=4096)
+    comm.set_strategy("allgather", ag)
+    xg = rank_tensors("f32", cnt, n)
+    dy = [empty_dev(n * cnt, "f32") for _ in range(n)]
+    comm.allgather_lb([to_dev(x, "f32") for x in xg], dy)
+    torch.cuda.synchronize()
+    full = np.concatenate(xg)
+    for g in range(n):
+        assert np.array_equal(bits(to_host(dy[g], "f32")), bits(full)), g
+    assert comm.get_async_error() == 0
+    comm.finalize()
