@@ -248,6 +248,25 @@ ADAPCC_API adapcc_result_t adapcc_collective_zc(adapcc_comm_t comm, adapcc_coll_
 
 /* Ticket of the most recent LATE_JOIN call (0 before the first). */
 ADAPCC_API adapcc_result_t adapcc_late_ticket(adapcc_comm_t comm, uint64_t* ticket);
+
+/* Link probe (NEXT-2: the paper's alpha-beta link profiling, §IV-B,
+ * P:L109-115).  Rank `src` (-1 = this rank; loopback: any virtual rank) sends
+ * `messages` back-to-back messages of `bytes` (multiple of 16, > 0, at most
+ * one parity half's data region) to EVERY rank in dst_mask at once, through
+ * engine 0 (copy engines: cudaMemcpyAsync, one stream per destination) or 1
+ * (SM: TMA bulk copies global -> shared -> peer, one kernel per message).
+ * One repetition is captured in a CUDA graph and replayed `iters` times
+ * between CUDA events; *seconds = mean time of one repetition (so a
+ * repetition of m messages of s bytes is the paper's t = m (alpha + beta s)).
+ * Data goes from the sender's arena (half 0) to the receivers' arenas (half 1):
+ * the call first synchronizes the device, and in multi-process mode it is a
+ * collective -- every live rank calls it (with its own src / dst_mask, 0 =
+ * only take part) and the timed replays start after a bootstrap barrier, so
+ * a probe round of the Fig. 5(b) schedule runs all its flows at once.
+ * dst_mask must not contain src or excluded ranks.  Errors: INVALID_ARGUMENT,
+ * CUDA, BOOTSTRAP. */
+ADAPCC_API adapcc_result_t adapcc_link_probe(adapcc_comm_t comm, int src, uint64_t dst_mask, size_t bytes,
+                                             int messages, int engine, int iters, double* seconds);
 /* Mark `rank` ready for late join: after all prior work on `stream` (e.g. the
  * rank's gradient computation) its ready word becomes `ticket` (0 = the
  * current ticket).  Multi-process: rank must be this rank (or -1);
@@ -304,6 +323,9 @@ ADAPCC_API const char* adapcc_last_cuda_error(void);
  * default; 0 = plain item/task/ref tables; env ADAPCC_FIRST_BLOB; env only: ADAPCC_TMA_SHAPE
  * forces the TMA ring of every TMA launch, 1 = 1 CTA/SM x 3 x 64 KiB, 2 = 2 CTAs/SM x 3 x 32 KiB,
  * 0 = automatic, default: STAGED plans (and ACCUMULATE plans with acc_red off) 2, others 1),
+ * "default_chunk" (chunk C_m in bytes of every default strategy -- the ones in effect for collectives
+ * without adapcc_set_strategy; multiple of 16, default 262144; e.g. the cost model's choice from
+ * a link profile, costmodel.py; strategies set by the caller are kept),
  * "acc_red" (TMA kernel, accumulating destinations -- ACCUMULATE phase 2, LATE_COMPLEMENT: 1 = the
  * folded tile leaves the stage by TMA bulk reduce-adds, recv += result performed in L2
  * (cp.reduce.async.bulk .add, fp32 / bf16 round to nearest even without flushing subnormals,

@@ -90,6 +90,7 @@ def _load():
         "adapcc_alltoallv": [vp, vp, vp, ctypes.POINTER(u64), i32, u64, vp],
         "adapcc_alltoallv_lb": [vp, pp, pp, ctypes.POINTER(u64), i32, u64, vp],
         "adapcc_late_ticket": [vp, ctypes.POINTER(u64)],
+        "adapcc_link_probe": [vp, i32, u64, sz, i32, i32, i32, ctypes.POINTER(ctypes.c_double)],
         "adapcc_signal_ready": [vp, i32, u64, vp],
         "adapcc_get_async_error": [vp],
         "adapcc_finalize": [vp],
@@ -611,6 +612,16 @@ class Communicator:
         _check(_load().adapcc_alltoallv(self._h, _ptr(send), _ptr(out), flat, _dtype_code(out), m,
                                         _stream(stream, self.device)), "alltoallv")
         return out
+
+    def link_probe(self, dst, nbytes, messages=1, engine="sm", iters=20, src=-1):
+        """Seconds per repetition of `messages` messages of `nbytes` from `src`
+        (-1 = this rank) to every rank in `dst` at once (adapcc_link_probe);
+        engine "sm" (TMA bulk copies) or "ce" (copy engines).  Multi-process:
+        a collective -- every rank calls it (dst may be empty)."""
+        v = ctypes.c_double()
+        _check(_load().adapcc_link_probe(self._h, src, _mask(set(dst), self.nranks), nbytes, messages,
+                                         {"ce": 0, "sm": 1}[engine], iters, ctypes.byref(v)), "link_probe")
+        return v.value
 
     def late_ticket(self):
         v = ctypes.c_uint64()

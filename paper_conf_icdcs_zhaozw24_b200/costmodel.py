@@ -77,6 +77,109 @@ def probe_link(copy_fn, sizes=(1 << 16, 1 << 20), repeats=(1, 8), timer=None):
     return alpha, beta, samples
 
 
+def profile_links(comm, sizes=(1 << 16, 1 << 22), repeats=(1, 8), engine="sm", iters=20, gather=None):
+    """Per-link alpha / beta on the device, through
+    adapcc_link_probe (graph-captured messages, so alpha is the device's
+    per-message cost rather than host launch noise).
+
+    Multi-process: the N-1 rounds of Fig. 5(b) (probe_rounds): in round i rank
+    k probes (k + i) % N while every other rank probes its own partner (one
+    flow per port); per link the paper's two shapes, m messages of s
+    and one message of m*s, for every (s, m), least-squares fit.
+    `gather(obj) -> list per rank` shares the rows (default: the
+    torch.distributed default group).  Loopback (n virtual ranks on one GPU):
+    virtual rank 0 probes each q in turn; every "link" is the HBM copy path.
+    Also times the fan-out 1 -> all others at the largest size (the N>1 bench's
+    P2P ceiling).  Returns a JSON-able dict."""
+    n, me = comm.nranks, comm.rank
+    rounds = [[(0, q)] for q in range(1, n)] if comm.loopback else probe_rounds(n)
+    rows = {}
+    for rnd in rounds:
+        mine = rnd if comm.loopback else [p for p in rnd if p[0] == me]
+        for (i, j) in mine:
+            samples = []
+            for s in sizes:
+                for m in repeats:
+                    for msgs, nb in ((m, s), (1, m * s)):
+                        t = comm.link_probe({j}, nb, messages=msgs, engine=engine, iters=iters,
+                                            src=i if comm.loopback else -1)
+                        samples.append((msgs, nb, t))
+            a, b = fit_alpha_beta(samples)
+            rows[(i, j)] = {"alpha_s": a, "beta_s_per_byte": b, "samples": samples}
+    # fan-out 1 -> n-1 (rank 0 sends, the others only take part)
+    big = max(sizes) * max(repeats)
+    fan_dst = set(range(1, n)) if (comm.loopback or me == 0) else set()
+    t_fan = comm.link_probe(fan_dst, big, engine=engine, iters=max(2, iters // 4), src=0 if comm.loopback else -1)
+    mine = {"rows": {f"{i}->{j}": v for (i, j), v in rows.items()},
+            "fanout": {"src": 0, "bytes_per_dst": big, "seconds": t_fan} if fan_dst else None}
+    if comm.loopback:
+        per_rank = [mine]
+    else:
+        if gather is None:
+            import torch.distributed as dist
+
+            def gather(obj):
+                out = [None] * dist.get_world_size()
+                dist.all_gather_object(out, obj)
+                return out
+        per_rank = gather(mine)
+    alpha = [[None] * n for _ in range(n)]
+    beta = [[None] * n for _ in range(n)]
+    samples = {}
+    for pr in per_rank:
+        for key, v in pr["rows"].items():
+            i, j = (int(x) for x in key.split("->"))
+            alpha[i][j], beta[i][j] = v["alpha_s"], v["beta_s_per_byte"]
+            samples[key] = v["samples"]
+    fan = [pr["fanout"] for pr in per_rank if pr["fanout"]]
+    gbps = [[(1.0 / b / 1e9 if b and b > 0 else None) for b in row] for row in beta]
+    return {"n": n, "engine": engine, "loopback": comm.loopback, "sizes": list(sizes), "repeats": list(repeats),
+            "alpha_us": [[(a * 1e6 if a is not None else None) for a in row] for row in alpha],
+            "beta_GBps": gbps, "samples": samples,
+            "fanout": [{"src": f["src"], "dsts": n - 1, "bytes_per_dst": f["bytes_per_dst"], "seconds": f["seconds"],
+                        "GBps_per_dst": f["bytes_per_dst"] / f["seconds"] / 1e9 if f["seconds"] else None,
+                        "GBps_out": (n - 1) * f["bytes_per_dst"] / f["seconds"] / 1e9 if f["seconds"] else None}
+                       for f in fan]}
+
+
+def links_to_model(profile):
+    """alpha[i][j] (s) and beta[i][j] (s/byte) matrices for the cost model;
+    links the profile did not measure take the mean of the measured ones."""
+    n = profile["n"]
+    a_all = [a for row in profile["alpha_us"] for a in row if a is not None]
+    g_all = [g for row in profile["beta_GBps"] for g in row if g]
+    a0 = (sum(a_all) / len(a_all)) * 1e-6 if a_all else 3e-6
+    b0 = 1.0 / ((sum(g_all) / len(g_all)) * 1e9) if g_all else 1.0 / 770e9
+    alpha = [[(profile["alpha_us"][i][j] * 1e-6 if profile["alpha_us"][i][j] is not None else a0) for j in range(n)]
+             for i in range(n)]
+    beta = [[(1.0 / (profile["beta_GBps"][i][j] * 1e9) if profile["beta_GBps"][i][j] else b0) for j in range(n)]
+            for i in range(n)]
+    return alpha, beta
+
+
+def per_gpu_bandwidth(profile):
+    """Per-GPU link bandwidth (GB/s) for generator.mask_aware_star_weights(bw=):
+    the slowest measured outgoing link of each GPU (one NVSwitch port each)."""
+    n = profile["n"]
+    out = []
+    for i in range(n):
+        g = [profile["beta_GBps"][i][j] for j in range(n) if j != i and profile["beta_GBps"][i][j]]
+        out.append(min(g) if g else None)
+    known = [x for x in out if x]
+    fill = sum(known) / len(known) if known else 1.0
+    return [x if x else fill for x in out]
+
+
+def chunk_from_profile(profile, S, text_for_chunk=None, candidates=(1 << 14, 1 << 16, 1 << 18, 1 << 20, 1 << 22)):
+    """The cost model's chunk for S bytes per rank on the profiled links
+    (default strategy: n star trees), plus the predicted times."""
+    from . import generator as G
+    n = profile["n"]
+    alpha, beta = links_to_model(profile)
+    fn = text_for_chunk or (lambda c: G.allreduce_stars(n, chunk=c))
+    return best_chunk(fn, S, alpha, beta, candidates)
+
+
 # -------------------------------------------------------------- cost model
 def _trees(text):
     n, coll, nsubs = _A.strategy_check(text)

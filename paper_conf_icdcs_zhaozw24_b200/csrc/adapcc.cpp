@@ -99,29 +99,30 @@ std::string star(int n, int root) {
 // call's root: one star tree (all trees of a Reduce share the root).  After a
 // fault exclusion (NEXT-3) the AllReduce default keeps only the stars rooted at
 // live ranks; excluded ranks are leaves of every star.
-std::string default_strategy(Coll c, int n, int root = 0, uint64_t members = ~uint64_t(0)) {
+std::string default_strategy(Coll c, int n, int root = 0, uint64_t members = ~uint64_t(0), int64_t chunk = 262144) {
+  const std::string ck = std::to_string(chunk);
   std::string s = "adapcc-strategy 1\nnranks " + std::to_string(n) + "\ncollective ";
-  if (c == kReduce) return s + "reduce\ntree weight=1 chunk=262144 parent=" + star(n, root) + "\n";
+  if (c == kReduce) return s + "reduce\ntree weight=1 chunk=" + ck + " parent=" + star(n, root) + "\n";
   if (c == kBroadcast)
-    return s + "broadcast\nbcast src=" + std::to_string(root) + " weight=1 chunk=262144 parent=" + star(n, root) + "\n";
+    return s + "broadcast\nbcast src=" + std::to_string(root) + " weight=1 chunk=" + ck + " parent=" + star(n, root) + "\n";
   if (c == kReduceScatter) {
     s += "reducescatter\n";
     for (int b = 0; b < n; ++b)
-      s += "rtree dst=" + std::to_string(b) + " weight=1 chunk=262144 parent=" + star(n, b) + "\n";
+      s += "rtree dst=" + std::to_string(b) + " weight=1 chunk=" + ck + " parent=" + star(n, b) + "\n";
     return s;
   }
   if (c == kAllReduce) {
     s += "allreduce\n";
     for (int m = 0; m < n; ++m) {  // n star trees, equal weights
       if (!((members >> m) & 1)) continue;
-      s += "tree weight=1 chunk=262144 parent=";
+      s += "tree weight=1 chunk=" + ck + " parent=";
       for (int g = 0; g < n; ++g) s += (g ? "," : "") + std::to_string(g == m ? -1 : m);
       s += "\n";
     }
   } else if (c == kAllGather) {
     s += "allgather\n";
     for (int src = 0; src < n; ++src) {
-      s += "bcast src=" + std::to_string(src) + " weight=1 chunk=262144 parent=";
+      s += "bcast src=" + std::to_string(src) + " weight=1 chunk=" + ck + " parent=";
       for (int g = 0; g < n; ++g) s += (g ? "," : "") + std::to_string(g == src ? -1 : src);
       s += "\n";
     }
@@ -172,6 +173,7 @@ struct adapcc_comm_s {
   uint32_t trace_cap = 0;
   int64_t pdl = 1;        // programmatic dependent launch of the engine kernels (ADAPCC_PDL)
   int64_t acc_red = 1;    // TMA kernel: recv += result by bulk reduce-add in L2 (ADAPCC_ACC_RED)
+  int64_t default_chunk = 262144;  // C_m of the default strategies (a link profile may set it)
   int64_t sched = 2;      // LDG kernel: 0 dynamic claims, 1 static blob schedule, 2 auto (ADAPCC_SCHED)
   uint64_t launches = 0;
   int num_sms = 148;
@@ -339,7 +341,7 @@ adapcc_result_t pick_strategy(adapcc_comm_s* c, Coll coll, int root, const Strat
   auto it = c->rooted[coll].find(root);
   if (it == c->rooted[coll].end()) {
     Strategy st;
-    if (!parse_strategy(default_strategy(coll, c->nranks, root).c_str(), &st, nullptr))
+    if (!parse_strategy(default_strategy(coll, c->nranks, root, c->members, c->default_chunk).c_str(), &st, nullptr))
       return ADAPCC_ERR_INVALID_STRATEGY;
     it = c->rooted[coll].emplace(root, std::move(st)).first;
   }
@@ -1083,6 +1085,96 @@ adapcc_result_t adapcc_alltoallv_lb(adapcc_comm_t c, const void* const* sendbufs
   return run(c, kAllToAll, sendbufs, recvbufs, 0, dtype, mask, 0, stream, 0, nullptr, nullptr, counts);
 }
 
+// ----------------------------------------------------------- link probe (NEXT-2)
+adapcc_result_t adapcc_link_probe(adapcc_comm_t c, int src, uint64_t dst_mask, size_t bytes, int messages,
+                                  int engine, int iters, double* seconds) {
+  if (!c || !seconds || messages < 1 || iters < 1 || (engine != 0 && engine != 1) || (bytes & 15) || !bytes)
+    return ADAPCC_ERR_INVALID_ARGUMENT;
+  if (src < 0) src = c->rank;
+  const uint64_t all = c->nranks >= 64 ? ~uint64_t(0) : ((uint64_t(1) << c->nranks) - 1);
+  if (src >= c->nranks || (!c->loopback && src != c->rank) || (dst_mask & ~all) || ((dst_mask >> src) & 1) ||
+      (dst_mask & ~c->members))
+    return ADAPCC_ERR_INVALID_ARGUMENT;
+  const uint64_t flag_cap = flag_region_bytes(c->half_bytes);
+  if (bytes > c->half_bytes - flag_cap) return ADAPCC_ERR_INVALID_ARGUMENT;
+  std::lock_guard<std::mutex> lock(c->mu);
+  CK(cudaSetDevice(c->device));
+  CK(cudaDeviceSynchronize());  // no collective is using the arenas
+  *seconds = 0.0;
+  // source: the sender's arena, half 0 data region; destinations: each
+  // receiver's arena, half 1 data region (scratch between collective calls)
+  const char* sp = c->arena[src] + kArenaHeader + flag_cap;
+  std::vector<char*> dst;
+  for (int q = 0; q < c->nranks; ++q)
+    if ((dst_mask >> q) & 1) dst.push_back(c->arena[q] + kArenaHeader + c->half_bytes + flag_cap);
+  auto barrier = [&]() -> adapcc_result_t {  // multi-process: every rank probes at the same time
+    if (c->loopback) return ADAPCC_SUCCESS;
+    int ok = 1;
+    std::vector<int> oks(c->nranks);
+    return members_allgather(c, &ok, oks.data(), sizeof(int)) ? ADAPCC_ERR_BOOTSTRAP : ADAPCC_SUCCESS;
+  };
+  cudaStream_t s = nullptr;
+  std::vector<cudaStream_t> ps(dst.size(), nullptr);
+  std::vector<cudaEvent_t> ev(dst.size() + 3, nullptr);
+  cudaGraph_t g = nullptr;
+  cudaGraphExec_t ge = nullptr;
+  adapcc_result_t r = ADAPCC_SUCCESS;
+  auto cleanup = [&] {
+    if (ge) cudaGraphExecDestroy(ge);
+    if (g) cudaGraphDestroy(g);
+    for (auto e : ev) if (e) cudaEventDestroy(e);
+    for (auto p : ps) if (p) cudaStreamDestroy(p);
+    if (s) cudaStreamDestroy(s);
+  };
+#define PK(expr)                                      \
+  do {                                                \
+    cudaError_t _e = (expr);                          \
+    if (_e != cudaSuccess) {                          \
+      cleanup();                                      \
+      return cuda_fail(_e, __LINE__);                 \
+    }                                                 \
+  } while (0)
+  PK(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
+  for (auto& e : ev) PK(cudaEventCreate(&e));
+  if (!dst.empty()) {
+    // one repetition = `messages` back-to-back messages, captured once in a
+    // CUDA graph: its replays carry no host launch overhead, so alpha is the
+    // device's per-message cost (P:L113 probes)
+    PK(cudaStreamBeginCapture(s, cudaStreamCaptureModeThreadLocal));
+    if (engine == 1) {
+      for (int m = 0; m < messages; ++m)
+        PK(probe_launch(sp, dst.data(), (int)dst.size(), bytes, 4 * c->num_sms, s));
+    } else {  // copy engines: one stream per destination, forked from / joined into s
+      PK(cudaEventRecord(ev[0], s));
+      for (size_t k = 0; k < dst.size(); ++k) {
+        PK(cudaStreamCreateWithFlags(&ps[k], cudaStreamNonBlocking));
+        PK(cudaStreamWaitEvent(ps[k], ev[0], 0));
+        for (int m = 0; m < messages; ++m)
+          PK(cudaMemcpyAsync(dst[k], sp, bytes, cudaMemcpyDeviceToDevice, ps[k]));
+        PK(cudaEventRecord(ev[3 + k], ps[k]));
+        PK(cudaStreamWaitEvent(s, ev[3 + k], 0));
+      }
+    }
+    PK(cudaStreamEndCapture(s, &g));
+    PK(cudaGraphInstantiate(&ge, g, 0));
+    PK(cudaGraphLaunch(ge, s));  // warm-up (and first touch of the peers' pages)
+    PK(cudaStreamSynchronize(s));
+  }
+  if ((r = barrier()) != ADAPCC_SUCCESS) { cleanup(); return r; }
+  if (!dst.empty()) {
+    PK(cudaEventRecord(ev[1], s));
+    for (int i = 0; i < iters; ++i) PK(cudaGraphLaunch(ge, s));
+    PK(cudaEventRecord(ev[2], s));
+    PK(cudaStreamSynchronize(s));
+    float ms = 0.f;
+    PK(cudaEventElapsedTime(&ms, ev[1], ev[2]));
+    *seconds = (double)ms * 1e-3 / iters;
+  }
+#undef PK
+  cleanup();
+  return barrier();
+}
+
 // ------------------------------------------------------------ late join (NEXT-1)
 adapcc_result_t adapcc_late_ticket(adapcc_comm_t c, uint64_t* ticket) {
   if (!c || !ticket) return ADAPCC_ERR_INVALID_ARGUMENT;
@@ -1152,7 +1244,7 @@ adapcc_result_t adapcc_exclude(adapcc_comm_t c, uint64_t dead_mask, adapcc_boots
   c->members = live;
   // 4. strategies: the survivors' defaults until set_strategy names new ones
   for (int k = 0; k < kNumColl; ++k) {
-    if (!parse_strategy(default_strategy((Coll)k, c->nranks, 0, live).c_str(), &c->strat[k], nullptr))
+    if (!parse_strategy(default_strategy((Coll)k, c->nranks, 0, live, c->default_chunk).c_str(), &c->strat[k], nullptr))
       return ADAPCC_ERR_INVALID_STRATEGY;
     c->user_set[k] = false;
     c->rooted[k].clear();
@@ -1202,6 +1294,18 @@ adapcc_result_t adapcc_config(adapcc_comm_t c, const char* key, int64_t value) {
     if (value < 0 || (key[0] == 't' && value > 64)) return ADAPCC_ERR_INVALID_ARGUMENT;
     (key[0] == 't' ? c->taper : c->piece_kib) = value;
     drop_plans(c);  // items are cut at plan time
+  }
+  else if (!std::strcmp(key, "default_chunk")) {
+    // C_m of every default strategy (a decision variable; e.g. the
+    // cost model's choice from a link profile); user strategies are kept
+    if (value < 16 || value % 16 || value > (int64_t(1) << 31)) return ADAPCC_ERR_INVALID_ARGUMENT;
+    c->default_chunk = value;
+    for (int k = 0; k < kNumColl; ++k) {
+      c->rooted[k].clear();
+      if (c->user_set[k]) continue;
+      if (!parse_strategy(default_strategy((Coll)k, c->nranks, 0, c->members, value).c_str(), &c->strat[k], nullptr))
+        return ADAPCC_ERR_INVALID_STRATEGY;
+    }
   }
   else if (!std::strcmp(key, "debug_check")) c->check_sig = value != 0;
   else if (!std::strcmp(key, "pdl")) c->pdl = value != 0;

@@ -136,6 +136,10 @@ struct ArenaHeader {
 int engine_threads();
 cudaError_t engine_occupancy(int dtype, int* blocks_per_sm);
 cudaError_t engine_launch(const LaunchParams& p, int grid, cudaStream_t stream, bool pdl);
+// probe.cu: one probe message -- `bytes` from src to each of dst[0..ndst) by
+// TMA bulk copies (link profiling, NEXT-2)
+cudaError_t probe_launch(const char* src, char* const* dst, int ndst, uint64_t bytes, int grid,
+                         cudaStream_t stream);
 // store `value` into a ready word after all prior work on `stream` (late join)
 cudaError_t engine_signal(uint64_t* word, uint64_t value, bool sys, cudaStream_t stream);
 // engine_tma_impl.cuh: TMA bulk-copy pipeline (1 producer + 8 consumer warps),

@@ -27,4 +27,4 @@ for cnt in (256, 4096, 65536):
               f"{(t1-t0)/K*1e6:6.2f} (wall)   host-only {(h1-h0)/300*1e6:6.2f} us/call")
     comm.finalize()
 PY
-bash scripts/debug/host_floor.sh > gpurun_out/host_floor2.log 2>&1
+
