@@ -255,9 +255,10 @@ ADAPCC_API adapcc_result_t adapcc_late_ticket(adapcc_comm_t comm, uint64_t* tick
  * one parity half's data region) to EVERY rank in dst_mask at once, through
  * engine 0 (copy engines: cudaMemcpyAsync, one stream per destination) or 1
  * (SM: TMA bulk copies global -> shared -> peer, one kernel per message).
- * One repetition is captured in a CUDA graph and replayed `iters` times
- * between CUDA events; *seconds = mean time of one repetition (so a
- * repetition of m messages of s bytes is the paper's t = m (alpha + beta s)).
+ * `iters` repetitions are captured in one CUDA graph, replayed once (warm-up)
+ * and once between CUDA events; *seconds = that time / iters, the mean time of
+ * one repetition (so a repetition of m messages of s bytes is the paper's
+ * t = m (alpha + beta s), with no host launch cost inside).
  * Data goes from the sender's arena (half 0) to the receivers' arenas (half 1):
  * the call first synchronizes the device, and in multi-process mode it is a
  * collective -- every live rank calls it (with its own src / dst_mask, 0 =

@@ -1137,19 +1137,19 @@ adapcc_result_t adapcc_link_probe(adapcc_comm_t c, int src, uint64_t dst_mask, s
   PK(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
   for (auto& e : ev) PK(cudaEventCreate(&e));
   if (!dst.empty()) {
-    // one repetition = `messages` back-to-back messages, captured once in a
-    // CUDA graph: its replays carry no host launch overhead, so alpha is the
-    // device's per-message cost (P:L113 probes)
+    // all `iters` repetitions of `messages` back-to-back messages captured in
+    // ONE CUDA graph: no host launch and no per-replay constant inside the
+    // timed region, so alpha is the device's per-message cost (P:L113 probes)
     PK(cudaStreamBeginCapture(s, cudaStreamCaptureModeThreadLocal));
     if (engine == 1) {
-      for (int m = 0; m < messages; ++m)
+      for (int m = 0; m < messages * iters; ++m)
         PK(probe_launch(sp, dst.data(), (int)dst.size(), bytes, 4 * c->num_sms, s));
     } else {  // copy engines: one stream per destination, forked from / joined into s
       PK(cudaEventRecord(ev[0], s));
       for (size_t k = 0; k < dst.size(); ++k) {
         PK(cudaStreamCreateWithFlags(&ps[k], cudaStreamNonBlocking));
         PK(cudaStreamWaitEvent(ps[k], ev[0], 0));
-        for (int m = 0; m < messages; ++m)
+        for (int m = 0; m < messages * iters; ++m)
           PK(cudaMemcpyAsync(dst[k], sp, bytes, cudaMemcpyDeviceToDevice, ps[k]));
         PK(cudaEventRecord(ev[3 + k], ps[k]));
         PK(cudaStreamWaitEvent(s, ev[3 + k], 0));
@@ -1163,7 +1163,7 @@ adapcc_result_t adapcc_link_probe(adapcc_comm_t c, int src, uint64_t dst_mask, s
   if ((r = barrier()) != ADAPCC_SUCCESS) { cleanup(); return r; }
   if (!dst.empty()) {
     PK(cudaEventRecord(ev[1], s));
-    for (int i = 0; i < iters; ++i) PK(cudaGraphLaunch(ge, s));
+    PK(cudaGraphLaunch(ge, s));
     PK(cudaEventRecord(ev[2], s));
     PK(cudaStreamSynchronize(s));
     float ms = 0.f;

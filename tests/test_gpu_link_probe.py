@@ -42,9 +42,9 @@ def test_loopback_profile(engine):
 def test_probe_messages_scale():
     """m messages take ~m times one message (the model t = m (alpha + beta s))."""
     comm = pkg.Communicator.loopback(2, scratch_bytes=256 << 20)
-    t1 = comm.link_probe({1}, 1 << 22, messages=1, src=0, iters=50)
-    t8 = comm.link_probe({1}, 1 << 22, messages=8, src=0, iters=20)
-    assert 6.0 < t8 / t1 < 10.0, (t1, t8)
+    t1 = comm.link_probe({1}, 1 << 22, messages=1, src=0, iters=40)
+    t8 = comm.link_probe({1}, 1 << 22, messages=8, src=0, iters=10)
+    assert 7.0 < t8 / t1 < 9.0, (t1, t8)
     comm.finalize()
 
 
@@ -98,5 +98,5 @@ def test_multiprocess_probe_rounds():
         p = out[r][1]
         for i in range(n):
             for j in range(n):
-                if i != j:
-                    assert p["beta_GBps"][i][j] and p["beta_GBps"][i][j] > 0
+                if i != j:   # every link probed by its sender (one GPU here: time-sliced, so no bound on beta)
+                    assert p["alpha_us"][i][j] is not None and f"{i}->{j}" in p["samples"]
