@@ -79,15 +79,22 @@ typedef enum { ADAPCC_MODE_DIRECT = 0, ADAPCC_MODE_STAGED = 1 } adapcc_mode_t;
 /* Late join (a relay that becomes ready during phase 1 makes
  * "data chunks with the same offset in the buffer join the ongoing aggregation
  * process. Then in phase 2, only partial data chunks from relay workers that
- * have not been aggregated need to be broadcast").  AllReduce on a DIRECT plan
- * (loopback DIRECT or adapcc_collective_zc) only; not combinable with
- * ACCUMULATE.
- *   LATE_JOIN (phase 1, mask R): every tree root also folds, per work piece,
- *     the inputs of the non-ready ranks whose ready word already holds this
- *     call's ticket (appended after the regular sources, ascending rank), and
- *     records which ones it folded.
+ * have not been aggregated need to be broadcast").  AllReduce only, every
+ * plan kind (loopback DIRECT / STAGED, multi-process STAGED via
+ * adapcc_allreduce, zero-copy via adapcc_collective_zc); not combinable with
+ * ACCUMULATE.  A non-ready rank passes its (future) sendbuf: it is read only
+ * after the rank signalled ready (adapcc_signal_ready).
+ *   LATE_JOIN (phase 1, mask R): every tree root also folds, per work piece
+ *     (DIRECT) or per chunk (STAGED), the inputs of the non-ready ranks whose
+ *     ready word already holds this call's ticket (appended after the
+ *     regular sources, ascending rank), and records which ones it folded.
+ *     DIRECT: the root reads the late input; STAGED: the late rank pushes its
+ *     chunk to the root iff it is ready when its GPU reaches that chunk, and a
+ *     per-chunk decision word next to the landing slot tells the root.
  *   LATE_COMPLEMENT (phase 2, SAME mask R and buffers as phase 1): recvbuf +=
- *     sum of the non-ready ranks' inputs that phase 1 did not fold, per piece.
+ *     sum of the non-ready ranks' inputs that phase 1 did not fold, per piece /
+ *     chunk (STAGED: only those chunks are pushed; the root broadcasts the sum
+ *     of what was left, or a "nothing" decision, chunk by chunk).
  *     It complements the most recent LATE_JOIN call of the same plan (same
  *     strategy, count, dtype, mask and buffers kind); phase-1 / phase-2 pairs
  *     of different plans may interleave.  A second LATE_COMPLEMENT after the

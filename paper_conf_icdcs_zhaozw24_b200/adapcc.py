@@ -452,13 +452,15 @@ class Communicator:
             pass
 
     # ---- multi-process collectives
-    def allreduce(self, x, out=None, ready=None, accumulate=False, stream=None):
+    def allreduce(self, x, out=None, ready=None, accumulate=False, stream=None, late=None):
+        """late: None | 'join' (phase 1) | 'complement' (phase 2); a late rank
+        passes its input, read once it signalled ready (signal_ready)."""
         out = x if out is None else out
         m = self._ready_mask(ready)
-        send = x if (m >> self.rank) & 1 else None
+        send = x if ((m >> self.rank) & 1 or late is not None) else None
+        flags = (FLAG_ACCUMULATE if accumulate else 0) | _late_flag(late)
         _check(_load().adapcc_allreduce(self._h, _ptr(send), _ptr(out), out.numel(),
-                                        _dtype_code(out), m,
-                                        FLAG_ACCUMULATE if accumulate else 0, _stream(stream, self.device)),
+                                        _dtype_code(out), m, flags, _stream(stream, self.device)),
                "allreduce")
         return out
 

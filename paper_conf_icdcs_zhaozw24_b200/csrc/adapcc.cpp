@@ -291,8 +291,9 @@ uint64_t fnv(uint64_t h, uint64_t v) {
 
 bool misaligned(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15) != 0; }
 
-// ACCUMULATE, or one of LATE_JOIN / LATE_COMPLEMENT (AllReduce on a DIRECT
-// plan only: the root must be able to read a late rank's input directly).
+// ACCUMULATE, or one of LATE_JOIN / LATE_COMPLEMENT (AllReduce only; on a
+// DIRECT plan the root reads a late rank's input, on a STAGED plan the late
+// rank pushes it to the root).
 adapcc_result_t check_late_flags(adapcc_comm_s* c, unsigned flags, bool late_ok) {
   (void)c;
   const unsigned late = flags & (ADAPCC_FLAG_LATE_JOIN | ADAPCC_FLAG_LATE_COMPLEMENT);
@@ -400,6 +401,8 @@ adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, const Strategy* strat, uin
     // (profiles/acc_r02.json); the shared-memory read-modify-write (acc_red
     // off) stages nsrc + nacc tiles per slot and is latency-bound, where the
     // 2 CTAs/SM x 3 x 32 KiB shape wins (profiles/acc_variants_r01.json).
+    // STAGED late join (decision words, conditional pushes) runs on the LDG kernel
+    if (rq.late_join && mode == kStaged) plan->engine = 0;
     plan->kernel = plan->engine == 0 ? 0 : (mode == kDirect && (!rq.accumulate || c->acc_red) ? 1 : 2);
     if (plan->kernel != 0 && (c->tma_shape == 1 || c->tma_shape == 2)) plan->kernel = (int)c->tma_shape;
   }
@@ -539,7 +542,8 @@ adapcc_result_t run(adapcc_comm_s* c, Coll coll, const void* const* send, void* 
     P.acc_red = c->acc_red ? 1 : 0;
     P.late_ticket = c->late_seq;
     P.late_bits = seg.late_bits;
-    P.late_list = seg.late_list;
+    // (STAGED phase 2 runs every item: pulls wait for every chunk's decision)
+    P.late_list = (zc || c->mode == kDirect) ? seg.late_list : nullptr;
     P.late_count = seg.late_count;
     P.drop_rank = (int)c->drop_rank;
     P.members = c->members;
@@ -694,10 +698,14 @@ adapcc_result_t adapcc_allreduce(adapcc_comm_t c, const void* sendbuf, void* rec
                                  adapcc_stream_t stream) {
   adapcc_result_t r = check_common(c, dtype, mask);
   if (r != ADAPCC_SUCCESS) return r;
-  if (c->loopback || (flags & ~ADAPCC_FLAG_ACCUMULATE)) return ADAPCC_ERR_INVALID_ARGUMENT;
+  if (c->loopback) return ADAPCC_ERR_INVALID_ARGUMENT;
+  r = check_late_flags(c, flags, true);
+  if (r != ADAPCC_SUCCESS) return r;
   const size_t bytes = count * esize_of(dtype);
   if (count && !recvbuf) return ADAPCC_ERR_INVALID_ARGUMENT;
-  const bool ready = (mask >> c->rank) & 1;
+  // late join: a non-ready rank's input is pushed once it signals ready
+  const bool late = flags & (ADAPCC_FLAG_LATE_JOIN | ADAPCC_FLAG_LATE_COMPLEMENT);
+  const bool ready = ((mask >> c->rank) & 1) || late;
   if (count && ready && !sendbuf) return ADAPCC_ERR_INVALID_ARGUMENT;
   if (misaligned(recvbuf) || (ready && misaligned(sendbuf))) return ADAPCC_ERR_INVALID_ARGUMENT;
   if (ready && sendbuf != recvbuf && overlap(sendbuf, bytes, recvbuf, bytes)) return ADAPCC_ERR_INVALID_ARGUMENT;
@@ -765,7 +773,7 @@ adapcc_result_t adapcc_allreduce_lb(adapcc_comm_t c, const void* const* sendbufs
                                     uint64_t mask, unsigned flags, adapcc_stream_t stream) {
   adapcc_result_t r = check_common(c, dtype, mask);
   if (r != ADAPCC_SUCCESS) return r;
-  r = check_late_flags(c, flags, c->mode == kDirect);
+  r = check_late_flags(c, flags, true);
   if (r != ADAPCC_SUCCESS) return r;
   const size_t bytes = count * esize_of(dtype);
   // late join reads the non-ready ranks' inputs too: check every sendbuf
@@ -1476,6 +1484,7 @@ adapcc_result_t adapcc_plan_stats(const char* text, uint64_t count, adapcc_dtype
   rq.esize = esize_of(dtype);
   rq.ready_mask = mask;
   rq.accumulate = flags & ADAPCC_FLAG_ACCUMULATE;
+  rq.late_join = flags & (ADAPCC_FLAG_LATE_JOIN | ADAPCC_FLAG_LATE_COMPLEMENT);
   rq.mode = (Mode)mode;
   const size_t scratch = scratch_bytes ? scratch_bytes : kDefaultScratch;
   if (scratch < (size_t)kArenaHeader + 2 * (4096 + 65536)) return ADAPCC_ERR_INVALID_ARGUMENT;

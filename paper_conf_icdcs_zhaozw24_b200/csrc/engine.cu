@@ -52,6 +52,12 @@ struct Cur {  // header of the work item being executed (staged by thread 0)
   uint16_t tnsrc, nreg;     // task's own source count; regular sources used
   bool dropped, force_acc;
   int8_t blob;              // refs come from blob buffer `blob` in shared memory (-1: from P.refs)
+  // STAGED late join (LateKind): decision words
+  uint8_t lkind, decide;    // decide: sources / op are fixed after the waits (decision words)
+  uint8_t dec_dst, dec_out; // write dec_out into the decision word of every arena destination
+  uint16_t tnwait, wait0, tnlate;  // task's wait count; first wait used; late candidates
+  uint64_t tlo;             // task range start and chunk count (decision-word addresses)
+  uint32_t tnch;
 };
 
 struct Shared {
@@ -197,6 +203,7 @@ template <int DT>
 __device__ void fold_chunk(const Shared& sh, int nsrc, int ndst, uint64_t n, int op) {
   using O = Ops<DT>;
   using E = typename O::E;
+  if (op == kOpNone) return;  // (STAGED late join: nothing to move for this chunk)
   if (op == kOpZero) {
     for (int d = 0; d < ndst; ++d)
       for (uint64_t e = threadIdx.x; e < n; e += kThreads)
@@ -260,7 +267,41 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
     c.dropped = (int)t.owner == P.drop_rank;
     c.late = 0;
     c.force_acc = false;
-    if (P.late_mode && !c.dropped) {
+    c.lkind = t.lkind;
+    c.decide = 0;
+    c.dec_dst = 0;
+    c.dec_out = 1;
+    c.tnwait = t.nwait;
+    c.wait0 = 0;
+    c.tnlate = t.nlate;
+    c.tlo = t.lo;
+    c.tnch = t.nchunks;
+    if (P.late_mode && !c.dropped && t.lkind == kLatePush) {
+      // the late rank's own chunk goes to the root iff it is ready now
+      // (phase 1) / iff it did not go in phase 1 (phase 2)
+      bool pushed;
+      if (P.late_mode == 1) {
+        pushed = ld_acquire(reinterpret_cast<const uint64_t*>(sbase[kBufArena][t.owner] + ArenaHeader::kReady),
+                            P.ipc) >= P.late_ticket;
+        P.late_bits[it] = pushed ? 1 : 0;
+      } else {
+        pushed = P.late_bits[it] == 0;
+      }
+      if (!pushed) c.op = kOpNone;
+      c.dec_dst = 1;
+      c.dec_out = pushed ? 1 : 0;
+    } else if (P.late_mode && !c.dropped && t.lkind == kLateRoot) {
+      c.decide = 1;  // candidates are decided after the waits (their decision words)
+      if (P.late_mode == 2) {  // only the late slots' flags; recv += fold of what is left
+        c.nreg = 0;
+        c.wait0 = (uint16_t)(t.nwait - t.nlwait);
+        c.nwait = t.nlwait;
+        c.op = kOpFold;
+        c.force_acc = true;
+      }
+    } else if (P.late_mode && !c.dropped && t.lkind == kLatePull) {
+      c.decide = P.late_mode == 2;  // accumulate iff the parent broadcast anything
+    } else if (P.late_mode && !c.dropped) {
       if (t.nlate == 0) {
         c.dropped = P.late_mode == 2;  // phase 2 only runs the roots' folds
       } else {
@@ -304,11 +345,59 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
       sh.src[i] = p;
     } else {
       sh.dst[i - nsrc] = p;
-      const bool acc = r.accum || sh.cur.force_acc;
+      // (force_acc: recv += result; a STAGED broadcast slot still takes the plain result)
+      const bool acc = r.accum || (sh.cur.force_acc && r.kind == kBufRecv);
       sh.acc[i - nsrc] = acc;
       if (acc) atomicOr(&sh.any_acc, 1);
     }
     return arena;
+  };
+  // STAGED late join: decision word of chunk sh.cur.chunk of the slot `r`
+  // (an arena stream of the current task) -- 8 bytes per chunk before the slot
+  auto dec_word = [&](const BufRef& r, uint64_t hoff) {
+    return reinterpret_cast<uint64_t*>(sbase[kBufArena][r.rank] + hoff + r.bias + (int64_t)(sh.cur.tlo * esize) -
+                                       (int64_t)late_dec_bytes(sh.cur.tnch)) + sh.cur.chunk;
+  };
+  auto ref_of = [&](uint32_t j) {
+    return sh.cur.blob >= 0 ? *reinterpret_cast<const BufRef*>(&sh.blob[sh.cur.blob][kBlobRef0 + j])
+                            : P.refs[sh.cur.ref0 + j];
+  };
+  // thread 0, after the item's waits: which late candidates the root folds
+  // (phase 1: the pushed slots and, for a late root, its own input if ready;
+  // phase 2: the slots pushed now and a late root's own input if not yet
+  // folded), or whether a phase-2 broadcast pull has anything to add
+  auto decide = [&](uint64_t hoff) {
+    Cur& c = sh.cur;
+    if (c.lkind == kLateRoot) {
+      const uint64_t prev = P.late_mode == 2 ? P.late_bits[sh.item] : 0;
+      uint64_t m = 0;
+      for (uint32_t j = 0; j < c.tnlate; ++j) {
+        const BufRef r = ref_of(c.tnsrc + c.ndst + j);
+        bool in;
+        if (r.kind == kBufArena) in = *reinterpret_cast<volatile uint64_t*>(dec_word(r, hoff)) != 0;
+        else if (P.late_mode == 1)
+          in = ld_acquire(reinterpret_cast<const uint64_t*>(sbase[kBufArena][r.rank] + ArenaHeader::kReady),
+                          P.ipc) >= P.late_ticket;
+        else in = ((prev >> j) & 1) == 0;
+        if (in) m |= 1ull << j;
+      }
+      if (P.late_mode == 1) {
+        P.late_bits[sh.item] = m;
+        if (m && c.op == kOpZero) c.op = kOpFold;
+      } else {
+        if (!m) c.op = kOpNone;
+        c.dec_dst = 1;
+        c.dec_out = m ? 1 : 0;
+      }
+      c.late = m;
+      c.nsrc = (uint16_t)(c.nreg + __popcll(m));
+    } else {  // kLatePull, phase 2
+      const bool any = *reinterpret_cast<volatile uint64_t*>(dec_word(ref_of(0), hoff)) != 0;
+      if (!any) c.op = kOpNone;
+      else c.force_acc = true;
+      c.dec_dst = 1;
+      c.dec_out = any ? 1 : 0;
+    }
   };
   // The first item of a blob CTA is staged and resolved here, before the
   // stream-order wait: under PDL this overlaps the previous kernel instead of
@@ -408,20 +497,19 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
     if (stat && !last && threadIdx.x < P.first_words)
       cp_async16(&sh.blob[buf ^ 1][threadIdx.x],
                  P.first + (size_t)(sh.item + gridDim.x) * P.first_words + threadIdx.x);
-    const int nsrc = sh.cur.nsrc, ndst = sh.cur.ndst, npost = sh.cur.npost;
-    const bool dropped = sh.cur.dropped;
+    const bool dropped = sh.cur.dropped, deferred = sh.cur.decide != 0;
     if (!dropped) {
       // input flags, one waiter thread per flag
       if (threadIdx.x < sh.cur.nwait) {
-        const FlagRef f = P.flags[sh.cur.flag0 + threadIdx.x];
+        const FlagRef f = P.flags[sh.cur.flag0 + sh.cur.wait0 + threadIdx.x];
         const uint64_t* fl =
             reinterpret_cast<const uint64_t*>(sbase[kBufArena][f.rank] + half_off + f.off) + sh.cur.chunk;
         if (!wait_flag(fl, epoch, P)) sh.abort = 1;
       }
       if (!staged) {
-        resolve(half_off);
+        if (!deferred) resolve(half_off);
       } else if (my_arena) {  // pre-staged before the epoch was known
-        const int i = threadIdx.x;
+        const int i = threadIdx.x, nsrc = sh.cur.nsrc;
         if (i < nsrc) sh.src[i] += half_off;
         else sh.dst[i - nsrc] += half_off;
       }
@@ -433,6 +521,13 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
       if (stat) cp_async_wait_all();
       break;
     }
+    if (!dropped && deferred) {  // STAGED late join: decision words are readable now
+      if (threadIdx.x == 0) decide(half_off);
+      __syncthreads();
+      resolve(half_off);
+      __syncthreads();
+    }
+    const int nsrc = sh.cur.nsrc, ndst = sh.cur.ndst, npost = sh.cur.npost;
     if (!dropped) {
       fold_chunk<DT>(sh, nsrc, ndst, sh.cur.len, sh.cur.op);
       if (stat) cp_async_wait_all();  // the next blob has landed before the barrier publishes it
@@ -442,9 +537,14 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
       if (threadIdx.x == 0 && npost) {
         const uint64_t e = sh.epoch;
         const char* const* hdr = P.hdr;
+        if (sh.cur.dec_dst)  // STAGED late join: the decision travels with the chunk's flag
+          for (int k = 0; k < ndst; ++k) {
+            const BufRef r = ref_of(sh.cur.tnsrc + k);
+            if (r.kind == kBufArena) *reinterpret_cast<volatile uint64_t*>(dec_word(r, half_off)) = sh.cur.dec_out;
+          }
         fence(sys);  // the chunk's bytes (incl. remote NVLink stores) before its flag
         for (int i = 0; i < sh.cur.npost; ++i) {
-          const FlagRef f = P.flags[sh.cur.flag0 + sh.cur.nwait + i];
+          const FlagRef f = P.flags[sh.cur.flag0 + sh.cur.tnwait + i];
           st_release(reinterpret_cast<uint64_t*>(const_cast<char*>(hdr[f.rank]) + half_off + f.off) +
                          sh.cur.chunk, e, sys);
         }

@@ -26,7 +26,18 @@ constexpr int kFirstMaxWords = 72;
 
 enum BufKind : uint8_t { kBufSend = 0, kBufRecv = 1, kBufArena = 2 };
 enum DType : int { kF32 = 0, kBF16 = 1, kI32 = 2 };
-enum TaskOp : uint16_t { kOpFold = 0, kOpZero = 1 };
+enum TaskOp : uint16_t { kOpFold = 0, kOpZero = 1, kOpNone = 2 /* (runtime only) no data */ };
+// Late join on STAGED plans (NEXT-1): the late rank pushes its chunk
+// to the tree root itself, conditionally, and every decision travels in a
+// per-chunk word placed before the slot it describes.
+enum LateKind : uint8_t {
+  kLateNone = 0,  // DIRECT late join (nlate > 0 at roots) or no late join
+  kLatePush = 1,  // owner = a late rank: push its chunk into its landing slot at the root iff
+                  // ready (phase 1) / iff not pushed in phase 1 (phase 2); decision word = pushed
+  kLateRoot = 2,  // root: late candidates = landing slots (decision words) or its own input
+                  // (ready word); the last nlwait waits are the late slots' flags
+  kLatePull = 3,  // broadcast pull: phase 2 accumulates iff the parent's decision word says so
+};
 
 // address(e) = base(kind, rank) + bias + e * esize, e = element index in the
 // task's coordinate system.
@@ -58,7 +69,8 @@ struct Task {
   uint16_t op;
   uint16_t owner;           // executing rank
   uint16_t nlate;           // late-join candidates: refs[ref0+nsrc+ndst .. +nlate) (root tasks)
-  uint16_t pad0;
+  uint8_t lkind;            // LateKind
+  uint8_t nlwait;           // kLateRoot: the last nlwait of the nwait waits belong to late candidates
 };
 
 // A work item covers elements [off, off+len) of chunk `chunk` of `task`.  A
@@ -72,6 +84,13 @@ struct Item {
   uint32_t len;   // elements
 };
 static_assert(sizeof(Item) == 16, "Item layout");
+
+// STAGED late join: per-chunk decision words (8 bytes each) sit just before
+// the slot they describe, in an array of late_dec_bytes(nchunks) bytes
+#ifdef __CUDACC__
+__host__ __device__
+#endif
+inline uint64_t late_dec_bytes(uint32_t nchunks) { return ((uint64_t)nchunks * 8 + 255) / 256 * 256; }
 
 // first-item blob layout (16-byte words): [0] Item, [1, kBlobRef0) Task, then refs
 constexpr int kBlobRef0 = 1 + (int)((sizeof(Task) + 15) / 16);

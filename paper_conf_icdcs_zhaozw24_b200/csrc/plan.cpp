@@ -73,6 +73,11 @@ class Builder {
     used_[r] = align_up(used_[r] + bytes, kAlign);
     return off;
   }
+  // a slot preceded by its per-chunk decision words (STAGED late join)
+  uint64_t alloc_dec(int r, uint64_t bytes, uint32_t nchunks) {
+    const uint64_t d = late_dec_bytes(nchunks);
+    return alloc(r, d + bytes) + d;
+  }
   FlagRef alloc_flags(int r, uint32_t nchunks) {
     FlagRef f{};
     f.off = flags_used_[r];
@@ -94,9 +99,12 @@ class Builder {
     return s;
   }
 
+  // late: late-join candidates (root tasks); late_waits: their landing
+  // slots' flags (STAGED), waited after the sources' flags; lkind: LateKind
   int add(int owner, uint64_t lo, uint64_t hi, uint32_t ce, uint16_t op,
           const std::vector<Stream>& srcs, const std::vector<BufRef>& dsts,
-          const std::vector<FlagRef>& posts, const std::vector<BufRef>& late = {}) {
+          const std::vector<FlagRef>& posts, const std::vector<BufRef>& late = {},
+          const std::vector<FlagRef>& late_waits = {}, uint8_t lkind = kLateNone) {
     Task t{};
     t.lo = lo;
     t.hi = hi;
@@ -121,7 +129,15 @@ class Builder {
       auto it = producer_.find({s.flag.rank, s.flag.off});
       if (it != producer_.end()) level = std::max(level, p_.tasks[it->second].level + 1);
     }
+    for (auto& f : late_waits) {
+      p_.flags.push_back(f);
+      ++nwait;
+      auto it = producer_.find({f.rank, f.off});
+      if (it != producer_.end()) level = std::max(level, p_.tasks[it->second].level + 1);
+    }
     t.nwait = nwait;
+    t.nlwait = (uint8_t)late_waits.size();
+    t.lkind = lkind;
     for (auto& f : posts) p_.flags.push_back(f);
     t.npost = (uint16_t)posts.size();
     t.level = level;
@@ -249,11 +265,36 @@ void plan_allreduce_tree(Builder& B, const SubColl& s, uint64_t lo, uint64_t hi,
     B.add(k, lo, hi, ce, kOpFold, consumer_srcs[k],
           {make_ref(kBufArena, d.rank, (int64_t)d.off - (int64_t)(lo * es))}, {d.flag});
   }
+  // late join (NEXT-1) on the STAGED protocol: every non-ready live
+  // rank pushes its own chunk straight into a landing slot at the root -- iff
+  // it is ready by then (phase 1) / iff it did not in phase 1 (phase 2) -- and
+  // says so in the slot's per-chunk decision word; a non-ready root folds its
+  // own input when its ready word allows (reading R4: late inputs join at the
+  // root, after the regular terms, ascending rank)
+  std::vector<BufRef> late_refs;
+  std::vector<FlagRef> late_waits;
+  if (late_join) {
+    for (int g = 0; g < n; ++g) {
+      if (((mask >> g) & 1) || !B.alive(g)) continue;
+      if (g == root) {
+        late_refs.push_back(make_ref(kBufSend, g, send_bias));
+        continue;
+      }
+      const uint64_t off = B.alloc_dec(root, len, nch);
+      const FlagRef fl = B.alloc_flags(root, nch);
+      const BufRef slot = make_ref(kBufArena, root, (int64_t)off - (int64_t)(lo * es));
+      Stream src;
+      src.ref = make_ref(kBufSend, g, send_bias);
+      B.add(g, lo, hi, ce, kOpFold, {src}, {slot}, {fl}, {}, {}, kLatePush);
+      late_refs.push_back(slot);
+      late_waits.push_back(fl);
+    }
+  }
   // root hand-off: own recvbuf + broadcast slot
   std::map<int, std::pair<uint64_t, FlagRef>> down;
   auto add_down_dst = [&](int g, std::vector<BufRef>* dsts, std::vector<FlagRef>* posts) {
     if (s.children[g].empty()) return;
-    uint64_t off = B.alloc(g, len);
+    uint64_t off = late_join ? B.alloc_dec(g, len, nch) : B.alloc(g, len);
     FlagRef fl = B.alloc_flags(g, nch);
     down[g] = {off, fl};
     dsts->push_back(make_ref(kBufArena, g, (int64_t)off - (int64_t)(lo * es)));
@@ -263,7 +304,8 @@ void plan_allreduce_tree(Builder& B, const SubColl& s, uint64_t lo, uint64_t hi,
     std::vector<BufRef> dsts = {make_ref(kBufRecv, root, 0, accumulate)};
     std::vector<FlagRef> posts;
     if (!root_only) add_down_dst(root, &dsts, &posts);
-    B.add(root, lo, hi, ce, zero ? kOpZero : kOpFold, consumer_srcs[root], dsts, posts);
+    B.add(root, lo, hi, ce, zero ? kOpZero : kOpFold, consumer_srcs[root], dsts, posts, late_refs, late_waits,
+          late_join ? kLateRoot : kLateNone);
   }
   if (root_only) return;
   // broadcast down the reversed tree, parents before children
@@ -275,7 +317,7 @@ void plan_allreduce_tree(Builder& B, const SubColl& s, uint64_t lo, uint64_t hi,
     std::vector<BufRef> dsts = {make_ref(kBufRecv, g, 0, accumulate)};
     std::vector<FlagRef> posts;
     add_down_dst(g, &dsts, &posts);
-    B.add(g, lo, hi, ce, kOpFold, srcs, dsts, posts);
+    B.add(g, lo, hi, ce, kOpFold, srcs, dsts, posts, {}, {}, late_join ? kLatePull : kLateNone);
   }
 }
 

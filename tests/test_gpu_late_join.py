@@ -32,23 +32,26 @@ def _need_gpu():
         pytest.skip("no GPU")
 
 
-def _comm(n, engine):
-    c = pkg.Communicator.loopback(n, mode="direct", scratch_bytes=64 << 20)
+def _comm(n, engine, mode="direct"):
+    c = pkg.Communicator.loopback(n, mode=mode, scratch_bytes=64 << 20)
     c.config("engine", engine)
     c.config("timeout_ms", 20000)
     return c
 
 
+@pytest.mark.parametrize("mode", ["direct", "staged"])
 @pytest.mark.parametrize("engine", [0, 1])
 @pytest.mark.parametrize("dtype", ["f32", "bf16", "i32"])
 @pytest.mark.parametrize("case", ["all", "none", "one"])
-def test_late_join_deterministic(engine, dtype, case):
+def test_late_join_deterministic(engine, dtype, case, mode):
+    """STAGED: late ranks push their chunks to the roots themselves (LDG
+    kernel whatever the engine setting); DIRECT: roots read them."""
     n, count = 8, 200_003
     R, late = {0, 1, 2, 4, 5, 7}, [3, 6]
     text = S.allreduce_trees([S.star(n, m) for m in range(n)] + [S.chain([0, 1, 2, 3, 4, 5, 6, 7])],
                              chunk=16384)
     xs = rank_tensors(dtype, count, n)
-    comm = _comm(n, engine)
+    comm = _comm(n, engine, mode)
     comm.set_strategy("allreduce", text)
     dx = [to_dev(x, dtype) for x in xs]
     dy = [empty_dev(count, dtype) for _ in range(n)]
@@ -70,19 +73,24 @@ def test_late_join_deterministic(engine, dtype, case):
     comm.finalize()
 
 
-def _piece_ranges(text, count, dtype, R, grid, engine):
+def _piece_ranges(text, count, dtype, R, grid, engine, mode="direct"):
     """Element ranges [a, b) of the work pieces of the LATE_JOIN plan the
-    kernel runs (same grid, same item cutting): the unit of inclusion."""
+    kernel runs (same grid, same item cutting): the unit of inclusion.
+    STAGED: the root tasks' chunks (a star root writes its recv and its
+    broadcast slot)."""
     mask = sum(1 << r for r in R)
-    items, tasks = pkg.adapcc.plan_items(text, count, dtype, mask, grid, tma=engine == 1, late="join")
+    items, tasks = pkg.adapcc.plan_items(text, count, dtype, mask, grid, tma=engine == 1 and mode == "direct",
+                                         late="join", mode=mode)
+    if mode == "staged":
+        items = items[(tasks[items["task"]]["ndst"] == 2) & (tasks[items["task"]]["nwait"] >= 1)]
     t = tasks[items["task"]]
     a = t["lo"] + items["chunk"].astype(np.uint64) * t["chunk_elems"] + items["off"]
     return np.stack([a, a + items["len"]], axis=1).astype(np.int64)
 
 
-@pytest.mark.parametrize("engine", [0, 1])
+@pytest.mark.parametrize("engine,mode", [(0, "direct"), (1, "direct"), (0, "staged")])
 @pytest.mark.parametrize("dtype", ["f32", "i32"])
-def test_late_join_racing_signal(engine, dtype):
+def test_late_join_racing_signal(engine, dtype, mode):
     """Rank 3 signals from a side stream while phase 1 runs.  Per work piece
     (chunks "with the same offset" join), ONE inclusion set must
     explain every element of the piece in both phases; across lags the race
@@ -91,14 +99,14 @@ def test_late_join_racing_signal(engine, dtype):
     R, late = {0, 1, 2, 4, 5, 7}, [3, 6]
     text = G.allreduce_stars(n, chunk=65536)
     xs = rank_tensors(dtype, count, n)
-    comm = _comm(n, engine)
+    comm = _comm(n, engine, mode)
     comm.config("max_ctas", grid)       # the piece cut below uses the same grid
     comm.set_strategy("allreduce", text)
     dx = [to_dev(x, dtype) for x in xs]
     dy = [empty_dev(count, dtype) for _ in range(n)]
     comm.allreduce_lb(dx, dy)  # warm-up (plans, clocks)
     torch.cuda.synchronize()
-    pieces = _piece_ranges(text, count, dtype, R, grid, engine)
+    pieces = _piece_ranges(text, count, dtype, R, grid, engine, mode)
     covered = np.zeros(count, np.int32)
     for a, b in pieces:
         covered[a:b] += 1

@@ -121,3 +121,41 @@ def test_plan_items_rejects_bad_arguments():
         pkg.plan_items(text, 1024, "f32", 15, 8, segment=5)  # no such segment
     with pytest.raises(pkg.AdapccError):
         pkg.plan_items(text, 1024, "f32", 1 << 5, 8)       # mask names rank 5 of 4
+
+
+@pytest.mark.parametrize("name", ["stars8", "dbinary8", "ring4"])
+@pytest.mark.parametrize("rank", [-1, 0, 3])
+def test_staged_late_join_plan(name, rank):
+    """STAGED late join (NEXT-1): per tree, every non-ready rank owns
+    one conditional push task (no waits, one post per chunk) whose range is the
+    tree's; the root task waits for them in addition to its regular sources;
+    items still tile every chunk and keep a topological claim order."""
+    text = STRATS[name]()
+    n, _, nsubs = pkg.strategy_check(text)
+    late = {3, n - 2}
+    mask = sum(1 << g for g in range(n) if g not in late)
+    count = 100_003
+    items, tasks = pkg.adapcc.plan_items(text, count, "f32", mask, 64, mode="staged", rank=rank, late="join")
+    if rank == -1:
+        _check_tiling(items, tasks)
+    _check_order(items, tasks)
+    _, plain = pkg.adapcc.plan_items(text, count, "f32", mask, 64, mode="staged", rank=rank)
+    # every tree range gets exactly one push per late rank that is not its root
+    ranges = {}
+    for t in plain:
+        ranges.setdefault((int(t["lo"]), int(t["hi"])), []).append(t)
+    extra = len(tasks) - len(plain)
+    if rank == -1:
+        roots = []
+        for m in range(nsubs):
+            _, _, parent, _ = pkg.strategy_sub(text, m)
+            roots.append(parent.index(-1))
+        assert extra == sum(len(late - {r}) for r in roots)
+        pushes = [t for t in tasks if int(t["owner"]) in late and int(t["nwait"]) == 0 and int(t["npost"]) == 1
+                  and int(t["nsrc"]) == 1]
+        assert len(pushes) >= extra
+    else:   # (tasks are listed for every rank; items only for `rank`)
+        mine = {int(it["task"]) for it in items}
+        assert all(int(tasks[i]["owner"]) == rank for i in mine)
+        assert any(int(tasks[i]["owner"]) in late and int(tasks[i]["nsrc"]) == 1 and int(tasks[i]["nwait"]) == 0
+                   for i in range(len(tasks)))
