@@ -282,6 +282,22 @@ ADAPCC_API adapcc_result_t adapcc_link_probe(adapcc_comm_t comm, int src, uint64
 ADAPCC_API adapcc_result_t adapcc_signal_ready(adapcc_comm_t comm, int rank, uint64_t ticket,
                                                adapcc_stream_t stream);
 
+/* Readiness board (NEXT-1 online coordinator): a page of host
+ * memory, mapped into the device, whose word r holds the ticket rank r last
+ * signalled ready for -- adapcc_signal_ready's kernel writes it (system-scope
+ * release) next to the arena word, so a host thread can poll readiness at a
+ * microsecond cycle without touching the device.  Words 64..127 are free for
+ * the coordinator's own use (its decision channel).  *shared = 1 when every
+ * rank's word is visible on this host: always in loopback; in multi-process
+ * mode when the ranks share a node and POSIX shared memory works (the page is
+ * created by rank 0 at adapcc_init and mapped by every rank); 0 = only this
+ * rank's word is maintained.  The page lives until adapcc_finalize. */
+ADAPCC_API adapcc_result_t adapcc_ready_board(adapcc_comm_t comm, volatile uint64_t** board, int* shared);
+/* Benchmark utility: one thread spins on %globaltimer for `ns` nanoseconds on
+ * `stream` (the controlled straggler of SURVEY §8(d) d-5: a late rank's
+ * "computation" that occupies one SM slot, not the GPU). */
+ADAPCC_API adapcc_result_t adapcc_spin(adapcc_comm_t comm, uint64_t ns, adapcc_stream_t stream);
+
 /* ------------------------------------------------------------- lifecycle --- */
 
 /* Latched device error (TIMEOUT) or SUCCESS.  Does not synchronize. */

@@ -92,6 +92,8 @@ def _load():
         "adapcc_late_ticket": [vp, ctypes.POINTER(u64)],
         "adapcc_link_probe": [vp, i32, u64, sz, i32, i32, i32, ctypes.POINTER(ctypes.c_double)],
         "adapcc_signal_ready": [vp, i32, u64, vp],
+        "adapcc_ready_board": [vp, ctypes.POINTER(ctypes.c_void_p), ctypes.POINTER(i32)],
+        "adapcc_spin": [vp, u64, vp],
         "adapcc_get_async_error": [vp],
         "adapcc_finalize": [vp],
         "adapcc_config": [vp, ctypes.c_char_p, i64],
@@ -624,6 +626,18 @@ class Communicator:
         _check(_load().adapcc_link_probe(self._h, src, _mask(set(dst), self.nranks), nbytes, messages,
                                          {"ce": 0, "sm": 1}[engine], iters, ctypes.byref(v)), "link_probe")
         return v.value
+
+    def ready_board(self):
+        """(address, shared) of the host-mapped readiness board (adapcc_ready_board):
+        word r = the ticket rank r last signalled ready for; words 64..127 are
+        the coordinator's.  shared: every rank's word is visible here."""
+        p, sh = ctypes.c_void_p(), ctypes.c_int()
+        _check(_load().adapcc_ready_board(self._h, ctypes.byref(p), ctypes.byref(sh)), "ready_board")
+        return p.value, bool(sh.value)
+
+    def spin(self, ns, stream=None):
+        """Enqueue a one-thread %globaltimer spin of `ns` nanoseconds (controlled straggler)."""
+        _check(_load().adapcc_spin(self._h, int(ns), _stream(stream, self.device)), "spin")
 
     def late_ticket(self):
         v = ctypes.c_uint64()

@@ -156,3 +156,120 @@ def exclude_faulty(comm, ready_times, phase1_end, now, factor=T_FAULT_FACTOR, st
     if faulty:
         comm.exclude(faulty, store=store)
     return faulty
+
+
+# ------------------------------------------------------- online coordinator
+BOARD_DECISION = 64      # readiness-board words: 64 sequence, 65 action, 66 mask (adapcc_ready_board)
+_ACTIONS = {"full": 1, "phase1": 2}
+
+
+class ReadyBoard:
+    """Host view of the communicator's readiness board (adapcc_ready_board):
+    word r holds the ticket rank r last signalled ready for, written by the
+    device (system-scope release) right after the rank's computation; the
+    decision area carries the leader's decisions to the other ranks of the
+    node.  Reads are plain host loads -- no device round trip (the
+    coordinator "receives communication requests from each worker")."""
+
+    def __init__(self, comm):
+        import ctypes
+        addr, self.shared = comm.ready_board()
+        self.n = comm.nranks
+        self.words = (ctypes.c_uint64 * 128).from_address(addr)
+
+    def ready(self, ticket):
+        w = self.words
+        return frozenset(r for r in range(self.n) if w[r] >= ticket)
+
+    def publish(self, seq, action, mask):
+        w = self.words
+        w[BOARD_DECISION + 1] = _ACTIONS[action]
+        w[BOARD_DECISION + 2] = mask
+        w[BOARD_DECISION] = seq            # last: followers read seq first (x86 stores stay ordered)
+
+    def wait_decision(self, seq, timeout, clock):
+        w = self.words
+        t0 = clock()
+        while w[BOARD_DECISION] < seq:
+            if clock() - t0 > timeout:
+                raise TimeoutError("coordinator decision not published")
+        action = {v: k for k, v in _ACTIONS.items()}[int(w[BOARD_DECISION + 1])]
+        return action, int(w[BOARD_DECISION + 2])
+
+
+class OnlineCoordinator:
+    """The relay coordinator on the hot path: one AllReduce per
+    call, driven by real readiness.
+
+    Every decision cycle the leader (rank 0, or the loopback process) reads
+    the readiness board -- which ranks signalled this collective's ticket --
+    and applies the break-even rule (Coordinator.step); it publishes "full"
+    (everyone ready) or "phase1" (ready ranks aggregate, the others relay) on
+    the board, and every rank issues the same LATE_JOIN call with that mask
+    (late ranks' chunks still join the ongoing aggregation chunk by chunk,
+    P:L131).  Each rank then polls the board until every late rank signalled
+    and issues LATE_COMPLEMENT (phase 2: only the chunks phase 1 missed).
+
+    issue(mask, late) enqueues this rank's collective call: late = 'join' |
+    'complement'.  Ranks signal readiness with comm.signal_ready(ticket=
+    coordinator.ticket()) after their computation (the ticket of the
+    collective the coordinator runs next).  policy: a Coordinator (fresh per
+    call: its waited time accumulates); cycle: seconds between decisions
+    (the paper's 5 ms, scaled to the collective's time scale, reading R2)."""
+
+    def __init__(self, comm, policy_factory, cycle=5e-6, timeout=30.0, clock=None):
+        import time
+        self.comm = comm
+        self.board = ReadyBoard(comm)
+        self.policy_factory = policy_factory
+        self.cycle = cycle
+        self.timeout = timeout
+        self.clock = clock or time.perf_counter
+        self.seq = 0
+        self.leader = comm.loopback or comm.rank == 0
+        if not comm.loopback and comm.nranks > 1 and not self.board.shared:
+            raise RuntimeError("online coordinator needs a node-shared readiness board (POSIX shared memory)")
+
+    def ticket(self):
+        """Ticket of the next collective (its phase 1 is the next LATE_JOIN call)."""
+        return self.comm.late_ticket() + 1
+
+    def allreduce(self, issue):
+        n, clock = self.comm.nranks, self.clock
+        all_mask = (1 << n) - 1
+        t = self.ticket()
+        self.seq += 1
+        t0 = clock()
+        if self.leader:
+            policy = self.policy_factory()
+            nxt = t0
+            while True:
+                ready = self.board.ready(t)
+                d = policy.step(clock() - t0, ready)
+                if d.action != "wait":
+                    break
+                if clock() - t0 > self.timeout:
+                    raise TimeoutError("no worker became ready")
+                nxt += self.cycle
+                while clock() < nxt:
+                    pass
+            mask = all_mask if d.action == "full" else sum(1 << r for r in d.ready)
+            if not self.comm.loopback:
+                self.board.publish(self.seq, d.action, mask)
+            action = d.action
+        else:
+            action, mask = self.board.wait_decision(self.seq, self.timeout, clock)
+        t_decide = clock()
+        issue(mask, "join")                   # phase 1 (or the full collective: nobody is late)
+        late = all_mask & ~mask
+        t_late = None
+        if late:
+            while True:                       # phase 2 once every late rank is ready
+                if all((self.board.words[r] >= t) for r in range(n) if (late >> r) & 1):
+                    break
+                if clock() - t0 > self.timeout:
+                    raise TimeoutError("late ranks never became ready (fault: see exclude_faulty)")
+            t_late = clock()
+            issue(mask, "complement")
+        return {"action": action, "mask": mask, "ticket": t, "decided_after_s": t_decide - t0,
+                "phase2_after_s": None if t_late is None else t_late - t0}

@@ -8,9 +8,13 @@
 // call is one engine launch per segment on the caller's stream.
 #include <cuda_runtime.h>
 #include <dlfcn.h>
+#include <fcntl.h>
+#include <sys/mman.h>
+#include <unistd.h>
 #include <nvtx3/nvToolsExt.h>  // header-only NVTX ranges: free unless a profiler (nsys) is attached
 
 #include <algorithm>
+#include <chrono>
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
@@ -188,6 +192,16 @@ struct adapcc_comm_s {
   std::map<int, RegBuf> regs;
   int next_reg = 0;
   std::map<std::pair<int, std::string>, std::pair<char*, int>> opened;  // (peer, handle) -> (base, refs)
+  // Readiness board (NEXT-1 online coordinator): kBoardWords host words,
+  // mapped into the device; word r = the ticket rank r signalled ready for
+  // (adapcc_signal_ready writes it next to the arena word), words 64.. are the
+  // coordinator's decision area.  Multi-process: one POSIX shared-memory page
+  // per communicator, registered by every rank, so every rank's host sees
+  // every rank's readiness without a device round trip.
+  uint64_t* h_board = nullptr;
+  uint64_t* d_board = nullptr;
+  bool board_shm = false;    // shared across the ranks of the node
+  bool board_pinned = false; // cudaHostAlloc'ed (else registered mmap)
 };
 
 namespace {
@@ -247,10 +261,55 @@ adapcc_result_t common_init(adapcc_comm_s* c, size_t scratch) {
   return ADAPCC_SUCCESS;
 }
 
+constexpr size_t kBoardBytes = 4096;
+
+// private board: a mapped pinned page (loopback, or a node without /dev/shm)
+adapcc_result_t board_private(adapcc_comm_s* c) {
+  void* h = nullptr;
+  if (cudaHostAlloc(&h, kBoardBytes, cudaHostAllocMapped | cudaHostAllocPortable) != cudaSuccess) return ADAPCC_ERR_CUDA;
+  std::memset(h, 0, kBoardBytes);
+  c->h_board = static_cast<uint64_t*>(h);
+  c->board_pinned = true;
+  CK(cudaHostGetDevicePointer(reinterpret_cast<void**>(&c->d_board), h, 0));
+  return ADAPCC_SUCCESS;
+}
+
+// shared board: rank 0 creates the page, every rank maps and registers it
+bool board_shared(adapcc_comm_s* c, const char* name, bool create) {
+  const int fd = shm_open(name, O_RDWR | (create ? O_CREAT | O_EXCL : 0), 0600);
+  if (fd < 0) return false;
+  if (create && ftruncate(fd, kBoardBytes) != 0) { close(fd); return false; }
+  void* p = mmap(nullptr, kBoardBytes, PROT_READ | PROT_WRITE, MAP_SHARED, fd, 0);
+  close(fd);
+  if (p == MAP_FAILED) return false;
+  if (create) std::memset(p, 0, kBoardBytes);
+  if (cudaHostRegister(p, kBoardBytes, cudaHostRegisterMapped | cudaHostRegisterPortable) != cudaSuccess ||
+      cudaHostGetDevicePointer(reinterpret_cast<void**>(&c->d_board), p, 0) != cudaSuccess) {
+    cudaGetLastError();
+    munmap(p, kBoardBytes);
+    return false;
+  }
+  c->h_board = static_cast<uint64_t*>(p);
+  c->board_shm = true;
+  return true;
+}
+
+void board_free(adapcc_comm_s* c) {
+  if (!c->h_board) return;
+  if (c->board_pinned) {
+    cudaFreeHost(c->h_board);
+  } else {
+    cudaHostUnregister(c->h_board);
+    munmap(c->h_board, kBoardBytes);
+  }
+  c->h_board = c->d_board = nullptr;
+}
+
 void release(adapcc_comm_s* c) {
   if (!c) return;
   cudaSetDevice(c->device);
   cudaDeviceSynchronize();
+  board_free(c);
   c->plans.clear();
   c->retired.clear();
   for (auto& o : c->opened) cudaIpcCloseMemHandle(o.second.first);
@@ -619,6 +678,7 @@ adapcc_result_t adapcc_init_loopback(adapcc_comm_t* comm, int nranks, int cuda_d
   if (cudaMemset(c->own_arena, 0, c->arena_bytes * nranks) != cudaSuccess ||
       cudaDeviceSynchronize() != cudaSuccess) { release(c); return ADAPCC_ERR_CUDA; }
   for (int q = 0; q < nranks; ++q) c->arena.push_back(c->own_arena + q * c->arena_bytes);
+  if ((r = board_private(c)) != ADAPCC_SUCCESS) { release(c); return r; }
   *comm = c;
   return ADAPCC_SUCCESS;
 }
@@ -646,13 +706,19 @@ adapcc_result_t adapcc_init(adapcc_comm_t* comm, int rank, int nranks, int cuda_
     release(c);
     return ADAPCC_ERR_CUDA;
   }
-  // handle exchange: the paper's set-up AllGather of IPC handles
-  struct Blob { cudaIpcMemHandle_t h; uint64_t arena_bytes; int32_t nranks, rank; };
+  // handle exchange: the paper's set-up AllGather of IPC handles;
+  // rank 0 also names (and creates) the node's readiness board
+  struct Blob { cudaIpcMemHandle_t h; uint64_t arena_bytes; int32_t nranks, rank; char board[48]; };
   Blob me{};
   if (cudaIpcGetMemHandle(&me.h, mine) != cudaSuccess) { release(c); return ADAPCC_ERR_CUDA; }
   me.arena_bytes = c->arena_bytes;
   me.nranks = nranks;
   me.rank = rank;
+  if (rank == 0) {
+    const auto t = std::chrono::steady_clock::now().time_since_epoch().count();
+    std::snprintf(me.board, sizeof(me.board), "/adapcc-%d-%llx", (int)getpid(), (unsigned long long)t);
+    if (!board_shared(c, me.board, true)) me.board[0] = 0;  // no shared memory: private boards
+  }
   std::vector<Blob> all(nranks);
   if (ag(&me, all.data(), sizeof(Blob), ag_ctx) != 0) { release(c); return ADAPCC_ERR_BOOTSTRAP; }
   for (int q = 0; q < nranks; ++q) {
@@ -670,10 +736,21 @@ adapcc_result_t adapcc_init(adapcc_comm_t* comm, int rank, int nranks, int cuda_
     }
     c->arena[q] = static_cast<char*>(p);
   }
+  if (rank != 0 && all[0].board[0]) board_shared(c, all[0].board, false);
+  if (!c->h_board && (r = board_private(c)) != ADAPCC_SUCCESS) { release(c); return r; }
   // second exchange doubles as a barrier: every peer has mapped every arena
-  int ok = 1;
+  // (and the board); the board's name can then go (the mappings stay)
+  int ok = c->board_shm ? 1 : 0;
   std::vector<int> oks(nranks);
   if (ag(&ok, oks.data(), sizeof(int), ag_ctx) != 0) { release(c); return ADAPCC_ERR_BOOTSTRAP; }
+  if (rank == 0 && all[0].board[0]) shm_unlink(all[0].board);
+  for (int q = 0; q < nranks; ++q)
+    if (!oks[q] && c->board_shm) {  // someone could not map it: everybody uses a private board
+      board_free(c);
+      c->board_shm = false;
+      if ((r = board_private(c)) != ADAPCC_SUCCESS) { release(c); return r; }
+      break;
+    }
   *comm = c;
   return ADAPCC_SUCCESS;
 }
@@ -1197,7 +1274,21 @@ adapcc_result_t adapcc_signal_ready(adapcc_comm_t c, int rank, uint64_t ticket, 
   if (ticket == 0) ticket = c->late_seq;
   CK(cudaSetDevice(c->device));
   CK(engine_signal(reinterpret_cast<uint64_t*>(c->arena[rank] + 16), ticket, !c->loopback,
-                   reinterpret_cast<cudaStream_t>(stream)));
+                   c->d_board ? c->d_board + rank : nullptr, reinterpret_cast<cudaStream_t>(stream)));
+  return ADAPCC_SUCCESS;
+}
+
+adapcc_result_t adapcc_ready_board(adapcc_comm_t c, volatile uint64_t** board, int* shared) {
+  if (!c || !board) return ADAPCC_ERR_INVALID_ARGUMENT;
+  *board = c->h_board;
+  if (shared) *shared = c->loopback || c->board_shm ? 1 : 0;
+  return c->h_board ? ADAPCC_SUCCESS : ADAPCC_ERR_UNSUPPORTED;
+}
+
+adapcc_result_t adapcc_spin(adapcc_comm_t c, uint64_t ns, adapcc_stream_t stream) {
+  if (!c) return ADAPCC_ERR_INVALID_ARGUMENT;
+  CK(cudaSetDevice(c->device));
+  CK(engine_spin(ns, reinterpret_cast<cudaStream_t>(stream)));
   return ADAPCC_SUCCESS;
 }
 

@@ -603,15 +603,27 @@ cudaError_t engine_occupancy(int dtype, int* blocks_per_sm) {
 }
 
 namespace {
-__global__ void signal_kernel(uint64_t* word, uint64_t value, int sys) {
+__global__ void signal_kernel(uint64_t* word, uint64_t value, int sys, uint64_t* board) {
   fence(sys);
   st_release(word, value, sys);
+  if (board) st_release(board, value, true);  // host-visible readiness board (coordinator)
+}
+__global__ void spin_kernel(uint64_t ns) {
+  const uint64_t t0 = globaltimer();
+  while (globaltimer() - t0 < ns) {
+  }
 }
 }  // namespace
 
-cudaError_t engine_signal(uint64_t* word, uint64_t value, bool sys, cudaStream_t stream) {
+cudaError_t engine_signal(uint64_t* word, uint64_t value, bool sys, uint64_t* board, cudaStream_t stream) {
   cudaGetLastError();
-  signal_kernel<<<1, 1, 0, stream>>>(word, value, sys ? 1 : 0);
+  signal_kernel<<<1, 1, 0, stream>>>(word, value, sys ? 1 : 0, board);
+  return cudaGetLastError();
+}
+
+cudaError_t engine_spin(uint64_t ns, cudaStream_t stream) {
+  cudaGetLastError();
+  spin_kernel<<<1, 1, 0, stream>>>(ns);
   return cudaGetLastError();
 }
 

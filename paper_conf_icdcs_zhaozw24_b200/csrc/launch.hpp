@@ -141,7 +141,10 @@ cudaError_t engine_launch(const LaunchParams& p, int grid, cudaStream_t stream, 
 cudaError_t probe_launch(const char* src, char* const* dst, int ndst, uint64_t bytes, int grid,
                          cudaStream_t stream);
 // store `value` into a ready word after all prior work on `stream` (late join)
-cudaError_t engine_signal(uint64_t* word, uint64_t value, bool sys, cudaStream_t stream);
+// (and into board, a host-mapped readiness word, if not null)
+cudaError_t engine_signal(uint64_t* word, uint64_t value, bool sys, uint64_t* board, cudaStream_t stream);
+// one thread spinning on %globaltimer for `ns` (controlled straggler, benchmarks)
+cudaError_t engine_spin(uint64_t ns, cudaStream_t stream);
 // engine_tma_impl.cuh: TMA bulk-copy pipeline (1 producer + 8 consumer warps),
 // one instantiation per plan kind
 namespace tma_direct {

@@ -1,0 +1,137 @@
+"""The online coordinator on the GPU (-m gpu, NEXT-1 P:L129-137): real
+readiness (ranks signal through the device onto the host-mapped board, two
+stragglers after a controlled %globaltimer spin), the coordinator -- not the
+test -- decides wait / full / phase 1 and issues LATE_JOIN / LATE_COMPLEMENT;
+int32 results equal the full sum exactly, and every recvbuf is identical."""
+
+import os
+import socket
+import sys
+
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+
+import paper_conf_icdcs_zhaozw24_b200 as pkg  # noqa: E402
+from oracle import collectives as oc  # noqa: E402
+from paper_conf_icdcs_zhaozw24_b200 import coordinator as C  # noqa: E402
+from paper_conf_icdcs_zhaozw24_b200 import generator as G  # noqa: E402
+from synth import rank_tensors  # noqa: E402
+from tests.gpu_util import empty_dev, to_dev, to_host  # noqa: E402
+
+pytestmark = pytest.mark.gpu
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(autouse=True)
+def _need_gpu():
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+
+
+def _policy(n, S, buy_s):
+    p = C.Coordinator(n, "allreduce", S, 100e9, 5e-6)
+    p.buy_cost = lambda k: buy_s        # calibrated buying cost (seconds)
+    return p
+
+
+@pytest.mark.parametrize("mode", ["direct", "staged"])
+@pytest.mark.parametrize("lag_us,buy_us,expect", [(3000, 50, "phase1"), (0, 100_000, "full")])
+def test_coordinator_drives_the_calls(mode, lag_us, buy_us, expect):
+    n, count = 8, 2_000_003
+    R, late = {0, 1, 2, 4, 5, 7}, [3, 6]
+    xs = rank_tensors("i32", count, n)
+    comm = pkg.Communicator.loopback(n, mode=mode, scratch_bytes=64 << 20)
+    comm.set_strategy("allreduce", G.allreduce_stars(n, chunk=65536))
+    dx = [to_dev(x, "i32") for x in xs]
+    dy = [empty_dev(count, "i32") for _ in range(n)]
+    cs = torch.cuda.Stream(priority=-1)      # communication: high priority
+    side = torch.cuda.Stream()               # the stragglers' "computation"
+    coord = C.OnlineCoordinator(comm, lambda: _policy(n, count * 4, buy_us * 1e-6), cycle=2e-6)
+    full = oc.allreduce_exact(xs, set(range(n)), "i32")
+    for it in range(3):
+        t = coord.ticket()
+        for r in R:
+            comm.signal_ready(r, ticket=t, stream=cs)
+        for r in late:
+            comm.spin(lag_us * 1000, stream=side)
+            comm.signal_ready(r, ticket=t, stream=side)
+        res = coord.allreduce(lambda m, lt: comm.allreduce_lb(dx, dy, ready=m, late=lt, stream=cs))
+        torch.cuda.synchronize()
+        assert comm.get_async_error() == 0
+        assert res["action"] == expect, res
+        for y in dy:
+            assert np.array_equal(to_host(y, "i32"), full), (it, res)
+    comm.finalize()
+
+
+def _port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _worker(rank, n, port, q):
+    try:
+        sys.path.insert(0, ROOT)
+        import torch.distributed as dist
+        os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+        dist.init_process_group("gloo", rank=rank, world_size=n)
+        dev = rank % torch.cuda.device_count()
+        torch.cuda.set_device(dev)
+        comm = pkg.Communicator.init(scratch_bytes=64 << 20, device=dev)
+        comm.config("timeout_ms", 60000)
+        count = 500_009
+        xs = rank_tensors("i32", count, n)
+        x, y = to_dev(xs[rank], "i32"), empty_dev(count, "i32")
+        late = n - 1
+        coord = C.OnlineCoordinator(comm, lambda: _policy(n, count * 4, 100e-6), cycle=5e-6)
+        cs = torch.cuda.Stream(priority=-1)
+        side = torch.cuda.Stream()
+        ok = []
+        for it in range(3):
+            t = coord.ticket()
+            dist.barrier()
+            if rank == late:
+                comm.spin(20_000_000, stream=side)        # 20 ms straggler
+                comm.signal_ready(ticket=t, stream=side)
+            else:
+                comm.signal_ready(ticket=t, stream=cs)
+            res = coord.allreduce(lambda m, lt: comm.allreduce(x, y, ready=m, late=lt, stream=cs))
+            torch.cuda.synchronize()
+            ok.append((res["action"], np.array_equal(to_host(y, "i32"), oc.allreduce_exact(xs, set(range(n)), "i32"))))
+        err = comm.get_async_error()
+        comm.finalize()
+        dist.destroy_process_group()
+        q.put((rank, err == 0 and all(a == "phase1" and b for a, b in ok), f"{ok} err={err} shared={coord.board.shared}"))
+    except Exception as e:  # noqa: BLE001
+        import traceback
+        q.put((rank, False, traceback.format_exc() + repr(e)))
+
+
+def test_coordinator_multiprocess_shared_board():
+    """3 processes: rank 0 decides from the node-shared board and publishes;
+    every rank issues the same phase-1 / phase-2 calls (STAGED protocol)."""
+    import torch.multiprocessing as mp
+    n = 3
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _port()
+    ps = [ctx.Process(target=_worker, args=(r, n, port, q)) for r in range(n)]
+    for p in ps:
+        p.start()
+    out = {}
+    try:
+        for _ in range(n):
+            r, ok, msg = q.get(timeout=300)
+            out[r] = (ok, msg)
+    finally:
+        for p in ps:
+            p.join(timeout=30)
+            if p.is_alive():
+                p.kill()
+    for r in range(n):
+        assert r in out and out[r][0], out.get(r)
