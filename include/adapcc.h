@@ -255,6 +255,12 @@ ADAPCC_API adapcc_result_t adapcc_collective_zc(adapcc_comm_t comm, adapcc_coll_
 
 /* Ticket of the most recent LATE_JOIN call (0 before the first). */
 ADAPCC_API adapcc_result_t adapcc_late_ticket(adapcc_comm_t comm, uint64_t* ticket);
+/* Consume a ticket without a LATE_JOIN call (host only; collective in the
+ * sense that every rank must advance at the same point of its call
+ * sequence): a coordinator that runs a plain AllReduce because everyone was
+ * ready still retires the readiness signals of that round.  *ticket (may be
+ * NULL) = the consumed ticket. */
+ADAPCC_API adapcc_result_t adapcc_late_advance(adapcc_comm_t comm, uint64_t* ticket);
 
 /* Link probe (NEXT-2: the paper's alpha-beta link profiling, §IV-B,
  * P:L109-115).  Rank `src` (-1 = this rank; loopback: any virtual rank) sends

@@ -90,6 +90,7 @@ def _load():
         "adapcc_alltoallv": [vp, vp, vp, ctypes.POINTER(u64), i32, u64, vp],
         "adapcc_alltoallv_lb": [vp, pp, pp, ctypes.POINTER(u64), i32, u64, vp],
         "adapcc_late_ticket": [vp, ctypes.POINTER(u64)],
+        "adapcc_late_advance": [vp, ctypes.POINTER(u64)],
         "adapcc_link_probe": [vp, i32, u64, sz, i32, i32, i32, ctypes.POINTER(ctypes.c_double)],
         "adapcc_signal_ready": [vp, i32, u64, vp],
         "adapcc_ready_board": [vp, ctypes.POINTER(ctypes.c_void_p), ctypes.POINTER(i32)],
@@ -638,6 +639,12 @@ class Communicator:
     def spin(self, ns, stream=None):
         """Enqueue a one-thread %globaltimer spin of `ns` nanoseconds (controlled straggler)."""
         _check(_load().adapcc_spin(self._h, int(ns), _stream(stream, self.device)), "spin")
+
+    def late_advance(self):
+        """Consume the next ticket without a LATE_JOIN call (adapcc_late_advance)."""
+        v = ctypes.c_uint64()
+        _check(_load().adapcc_late_advance(self._h, ctypes.byref(v)), "late_advance")
+        return v.value
 
     def late_ticket(self):
         v = ctypes.c_uint64()

@@ -210,8 +210,10 @@ class OnlineCoordinator:
     P:L131).  Each rank then polls the board until every late rank signalled
     and issues LATE_COMPLEMENT (phase 2: only the chunks phase 1 missed).
 
-    issue(mask, late) enqueues this rank's collective call: late = 'join' |
-    'complement'.  Ranks signal readiness with comm.signal_ready(ticket=
+    issue(mask, late) enqueues this rank's collective call: late = None (a
+    plain AllReduce over everyone: the "full" decision, after which the
+    round's ticket is retired with adapcc_late_advance), 'join' (phase 1) or
+    'complement' (phase 2).  Ranks signal readiness with comm.signal_ready(ticket=
     coordinator.ticket()) after their computation (the ticket of the
     collective the coordinator runs next).  policy: a Coordinator (fresh per
     call: its waited time accumulates); cycle: seconds between decisions
@@ -260,7 +262,11 @@ class OnlineCoordinator:
         else:
             action, mask = self.board.wait_decision(self.seq, self.timeout, clock)
         t_decide = clock()
-        issue(mask, "join")                   # phase 1 (or the full collective: nobody is late)
+        if action == "full":                  # nobody is late: the plain (fastest) plan
+            self.comm.late_advance()          # ... and this round's signals are retired
+            issue(mask, None)
+        else:
+            issue(mask, "join")               # phase 1
         late = all_mask & ~mask
         t_late = None
         if late:

@@ -1267,6 +1267,14 @@ adapcc_result_t adapcc_late_ticket(adapcc_comm_t c, uint64_t* ticket) {
   return ADAPCC_SUCCESS;
 }
 
+adapcc_result_t adapcc_late_advance(adapcc_comm_t c, uint64_t* ticket) {
+  if (!c) return ADAPCC_ERR_INVALID_ARGUMENT;
+  std::lock_guard<std::mutex> lock(c->mu);
+  ++c->late_seq;
+  if (ticket) *ticket = c->late_seq;
+  return ADAPCC_SUCCESS;
+}
+
 adapcc_result_t adapcc_signal_ready(adapcc_comm_t c, int rank, uint64_t ticket, adapcc_stream_t stream) {
   if (!c) return ADAPCC_ERR_INVALID_ARGUMENT;
   if (rank < 0) rank = c->rank;

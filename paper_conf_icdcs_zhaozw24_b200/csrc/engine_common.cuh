@@ -194,18 +194,19 @@ static __device__ bool check_call_sig(const LP& P, uint64_t epoch) {
 // mode 2 (phase 2): the candidates NOT recorded (only they remain to add).
 // Position of the next entry in the plan's phase-2 list for the phase-1
 // launch of `epoch`: the first append of a new launch (gen differs) restarts
-// the count at 0 (launch.hpp, late_count).
+// the count at 0 with one compare-and-swap; every later append of the launch
+// is a plain atomicAdd on the count half (no retry loop: a CAS per append
+// serialised a phase 1 that lists hundreds of items, launch.hpp late_count).
 template <class LP>
 static __device__ __forceinline__ uint32_t late_append(const LP& P, uint64_t epoch) {
   const unsigned long long gen = (unsigned long long)(uint32_t)epoch;
-  unsigned long long old = *reinterpret_cast<volatile unsigned long long*>(&P.late_count[0]), nw;
-  for (;;) {
-    nw = (old >> 32) == gen ? old + 1 : ((gen << 32) | 1ull);
-    const unsigned long long prev = atomicCAS(&P.late_count[0], old, nw);
-    if (prev == old) break;
-    old = prev;
+  unsigned long long old = *reinterpret_cast<volatile unsigned long long*>(&P.late_count[0]);
+  while ((old >> 32) != gen) {
+    const unsigned long long prev = atomicCAS(&P.late_count[0], old, (gen << 32) | 1ull);
+    if (prev == old) return 0u;   // this launch's first entry
+    old = prev;                   // someone else moved it: retry only while the gen is stale
   }
-  return (uint32_t)nw - 1u;
+  return (uint32_t)atomicAdd(&P.late_count[0], 1ull);
 }
 
 // Entries phase 2 runs: the list of the last completed phase 1, if any.

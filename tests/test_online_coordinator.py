@@ -25,6 +25,10 @@ class FakeComm:
     def late_ticket(self):
         return self._ticket
 
+    def late_advance(self):
+        self._ticket += 1
+        return self._ticket
+
 
 def _policy(n, buy_after):
     """A Coordinator whose buying cost is buy_after seconds."""
@@ -41,7 +45,8 @@ def test_all_ready_runs_one_full_call():
     calls = []
     oc = C.OnlineCoordinator(comm, lambda: _policy(4, 1.0), cycle=1e-5)
     res = oc.allreduce(lambda m, late: calls.append((m, late)))
-    assert res["action"] == "full" and calls == [(0b1111, "join")]
+    assert res["action"] == "full" and calls == [(0b1111, None)]
+    assert comm.late_ticket() == 5          # the round's ticket is retired
 
 
 def test_phase1_then_phase2_after_late_ranks_signal():
