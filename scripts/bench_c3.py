@@ -104,15 +104,15 @@ def main():
 
             def run_coord(name, ts_ns):
                 co = coord[name]
-                torch.cuda.synchronize()
                 t = co.ticket()
+                for r in R:                             # the ready ranks finished before t = 0
+                    comm.signal_ready(r, ticket=t, stream=cs)
+                torch.cuda.synchronize()
                 e0, e1 = ev(), ev()
                 e0.record(side)
                 comm.spin(ts_ns, stream=side)           # the stragglers' computation
                 for r in LATE:
                     comm.signal_ready(r, ticket=t, stream=side)
-                for r in R:
-                    comm.signal_ready(r, ticket=t, stream=cs)
                 res = co.allreduce(lambda m, lt: comm.allreduce_lb(xs, ys, ready=m, late=lt, stream=cs))
                 e1.record(cs)
                 torch.cuda.synchronize()
