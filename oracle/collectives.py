@@ -94,11 +94,47 @@ def allreduce(xs, strategy_text, ready, dtype, accumulate=False, y_prev=None):
     return ys
 
 
+def _nvls_result(vals, ready, dtype):
+    """An nvls sub-collective (reading R9): the NVSwitch sums the ready ranks'
+    values in an order it does not disclose (PTX multimem.ld_reduce), so the
+    oracle is the plain definition -- the exact sum (fp64 accumulation of the
+    fp32 / bf16-widened values), rounded once to the working precision (RNE);
+    int32 wraps mod 2^32.  GPU parity on fp32 / bf16 is a tolerance check
+    against this (nvls_tolerance); int32 is bit-exact."""
+    ready = sorted(r for r in ready if vals[r] is not None)
+    if not ready:
+        return None
+    if dtype == "i32":
+        tot = np.zeros(len(vals[ready[0]]), dtype=np.int64)
+        for r in ready:
+            tot = tot + vals[r].astype(np.int64)
+        return (tot & 0xFFFFFFFF).astype(np.uint32).view(np.int32)
+    acc = np.zeros(len(vals[ready[0]]), dtype=np.float64)
+    for r in ready:
+        acc = acc + (_bf.to_f32(vals[r]) if dtype == "bf16" else vals[r]).astype(np.float64)
+    f32 = acc.astype(np.float32)
+    return _bf.from_f32_rne(f32) if dtype == "bf16" else f32
+
+
+def nvls_tolerance(dtype, k):
+    """Normwise bound |y - exact| <= tol * sum_r |x_r| for a switch reduction
+    of k terms in any order: fp32 adds: (k-1) u + u (the final rounding),
+    u = 2^-24; bf16 with fp32 accumulation (.acc::f32) and one rounding to
+    bf16: (k-1) 2^-24 + 2^-8.  int32: 0 (exact)."""
+    if dtype == "i32":
+        return 0.0
+    u = 2.0 ** -24
+    return (max(k - 1, 0) + 1) * u if dtype == "f32" else max(k - 1, 0) * u + 2.0 ** -8
+
+
 def _tree_result(vals, sub, ready, dtype):
     """Result of one reduce tree over the elements in ``vals`` (vals[r]: rank r's
     values, None if not ready): bottom-up tuples, fold at every
     kernel node (own first, then sending children ascending, Q5), the root's
-    aggregate or its single flow; None when no ready rank is in the tree."""
+    aggregate or its single flow; None when no ready rank is in the tree.
+    An nvls sub-collective reduces through the switch (_nvls_result)."""
+    if sub.kind == "nvls":
+        return _nvls_result(vals, ready, dtype)
     tup, flows = behavior(sub.parent, ready, sub.noagg)
     agg_val = {}
 

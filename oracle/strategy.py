@@ -20,9 +20,14 @@ Format (one directive per line, '#' starts a comment):
     bcast src=<s> weight=<w> chunk=<C> parent=<p_0,..,p_{n-1}>           (allgather, broadcast)
     a2a   weight=<w> chunk=<C> [route=<s>:<d>:<h1>,..[;<s>:<d>:<h>,..]]  (alltoall)
     rtree dst=<b> weight=<w> chunk=<C> parent=<...> [noagg=<g,..>]       (reducescatter)
+    nvls  weight=<w> chunk=<C>                                            (allreduce)
   collective reduce uses tree lines sharing one root; broadcast uses bcast
   lines sharing one src (NEXT-4 primitives: Reduce / Broadcast, P:L165,
   ReduceScatter, P:L154(1)).
+
+An nvls line reduces its partition through the NVSwitch (multimem
+ld_reduce / st, NEXT-2): the switch is the aggregation point, every rank
+receives the result (reading R9: the summation order is the switch's).
 
 An a2a route entry s:d:h1,..,hk sends flow s -> d along s, h1, .., hk, d
 (routing variables x^f_ij of eq. 1); flows without an entry go
@@ -48,7 +53,7 @@ class StrategyError(ValueError):
 @dataclass
 class Sub:
     """One sub-collective m after ring expansion."""
-    kind: str                 # 'tree' (allreduce), 'bcast' (allgather), 'a2a'
+    kind: str                 # 'tree' | 'nvls' (allreduce), 'bcast' (allgather), 'a2a', 'rtree'
     weight: int               # effective integer weight (see expand_weights)
     chunk: int                # C_m in bytes (P:L176)
     parent: list = None       # parent[g], -1 at the root (tree / bcast)
@@ -182,7 +187,7 @@ def parse(text):
                             "reducescatter"):
                 raise StrategyError(f"unknown collective {coll!r}")
             continue
-        if head not in ("tree", "ring", "bcast", "a2a", "rtree"):
+        if head not in ("tree", "ring", "bcast", "a2a", "rtree", "nvls"):
             raise StrategyError(f"unknown directive {head!r}")
         kv = {}
         for t in toks[1:]:
@@ -195,13 +200,13 @@ def parse(text):
         raw_subs.append((head, kv))
     if n is None or coll is None:
         raise StrategyError("missing nranks or collective line")
-    allowed = {"allreduce": ("tree", "ring"), "allgather": ("bcast",), "alltoall": ("a2a",),
+    allowed = {"allreduce": ("tree", "ring", "nvls"), "allgather": ("bcast",), "alltoall": ("a2a",),
                "reduce": ("tree",), "broadcast": ("bcast",), "reducescatter": ("rtree",)}[coll]
     keys = {"tree": {"weight", "chunk", "parent"}, "ring": {"weight", "chunk", "order"},
             "bcast": {"src", "weight", "chunk", "parent"}, "a2a": {"weight", "chunk"},
-            "rtree": {"dst", "weight", "chunk", "parent"}}
+            "rtree": {"dst", "weight", "chunk", "parent"}, "nvls": {"weight", "chunk"}}
     optional = {"tree": {"noagg"}, "ring": set(), "bcast": set(), "a2a": {"route"},
-                "rtree": {"noagg"}}
+                "rtree": {"noagg"}, "nvls": set()}
     if not raw_subs:
         raise StrategyError("no sub-collective lines")
     st = Strategy(nranks=n, collective=coll)
@@ -255,6 +260,8 @@ def parse(text):
             if parent[src] != -1:
                 raise StrategyError("bcast root must be its src")
             st.subs.append(Sub("bcast", w * n, c, parent, frozenset(), src))
+        elif head == "nvls":
+            st.subs.append(Sub("nvls", w * n, c))
         else:
             st.subs.append(Sub("a2a", w * n, c, routes=_routes(kv.get("route"), n)))
     if len(st.subs) > MAX_SUBS:

@@ -150,6 +150,11 @@ BAD = [
     "adapcc-strategy 1\nnranks 2\ncollective alltoall\na2a weight=1\n",
     "adapcc-strategy 1\nnranks 2\nnranks 2\ncollective alltoall\na2a weight=1 chunk=16\n",
     "adapcc-strategy 1\nnranks 2\ncollective alltoall\na2a weight=1x chunk=16\n",
+    # nvls (NEXT-2 switch reduction): allreduce only, weight and chunk only
+    "adapcc-strategy 1\nnranks 2\ncollective allgather\nnvls weight=1 chunk=16\n",
+    "adapcc-strategy 1\nnranks 2\ncollective allreduce\nnvls weight=1 chunk=16 parent=-1,0\n",
+    "adapcc-strategy 1\nnranks 2\ncollective allreduce\nnvls weight=1\n",
+    "adapcc-strategy 1\nnranks 2\ncollective allreduce\nnvls weight=0 chunk=16\n",
 ]
 
 
@@ -463,3 +468,47 @@ def test_reducescatter_is_block_of_allreduce():
         blk = [x[b * cnt:(b + 1) * cnt] for x in xf]
         ref = oc.allreduce(blk, S.allreduce_trees([S.star(n, b)], chunk=16), set(range(n)), "f32")[0]
         assert np.array_equal(ys[b].view(np.uint32), ref.view(np.uint32))
+
+
+# ------------------------------------------------------------ nvls (NEXT-2)
+NVLS = ("adapcc-strategy 1\nnranks {n}\ncollective allreduce\nnvls weight=3 chunk=4096\n"
+        "tree weight=1 chunk=4096 parent={star}\n")
+
+
+def _nvls_text(n):
+    return NVLS.format(n=n, star=",".join(["-1"] + ["0"] * (n - 1)))
+
+
+@pytest.mark.parametrize("n", [2, 3, 5])
+def test_nvls_int32_is_the_brute_force_sum(n):
+    """An nvls partition is the switch's sum over the ready ranks: int32 adds
+    commute exactly, so it equals brute force mod 2^32 for every mask."""
+    xs = rank_tensors("i32", 4099, n)
+    text = _nvls_text(n)
+    for k in range(1, n + 1):
+        for R in itertools.combinations(range(n), k):
+            got = oc.allreduce(xs, text, set(R), "i32")
+            exp = oc.allreduce_exact(xs, set(R), "i32")
+            assert all(np.array_equal(g, exp) for g in got)
+
+
+def test_nvls_float_within_switch_bound_and_integer_exact():
+    """fp32 / bf16: within the any-order bound of nvls_tolerance against the
+    fp64 definition; integer-valued fp32 (partial sums < 2^24) is exact."""
+    n = 8
+    text = _nvls_text(n)
+    st = ost.parse(text)
+    lo, hi = ost.partition(20_000, 4, [s.weight for s in st.subs])[:2]
+    for dtype in ("f32", "bf16"):
+        xs = rank_tensors(dtype, 20_000, n)
+        got = oc.allreduce(xs, text, set(range(n)), dtype)[0]
+        ex = oc.allreduce_exact(xs, set(range(n)), dtype)
+        vals = [(obf.to_f32(x) if dtype == "bf16" else x).astype(np.float64) for x in xs]
+        den = np.sum(np.abs(np.stack(vals)), axis=0)
+        g = (obf.to_f32(got) if dtype == "bf16" else got).astype(np.float64)
+        err = np.abs(g[lo:hi] - ex[lo:hi]) / den[lo:hi]
+        assert err.max() <= oc.nvls_tolerance(dtype, n)
+        assert oc.nvls_tolerance(dtype, n) < (1e-6 if dtype == "f32" else 1e-2)
+    xi = rank_tensors("f32", 20_000, n, dist="intval")
+    got = oc.allreduce(xi, text, set(range(n)), "f32")[0]
+    assert np.array_equal(got[lo:hi].astype(np.float64), oc.allreduce_exact(xi, set(range(n)), "f32")[lo:hi])
