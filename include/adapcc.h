@@ -253,6 +253,24 @@ ADAPCC_API adapcc_result_t adapcc_collective_zc(adapcc_comm_t comm, adapcc_coll_
                                                 uint64_t ready_mask, unsigned flags,
                                                 adapcc_stream_t stream);
 
+/* NVLS switch reduction (NEXT-2): set up a multicast team over every rank's
+ * GPU (NVSwitch multicast objects, cuMulticast*) bound to `bytes` (rounded
+ * up to the multicast granularity) of library-owned scratch per rank; after
+ * it AllReduce strategies may contain `nvls weight=<w> chunk=<C>` lines,
+ * whose partition every rank copies into its scratch, slice owners sum in
+ * the switch (multimem.ld_reduce) and store to every rank at once
+ * (multimem.st), and every rank copies out -- ~S per GPU and direction over
+ * NVLink instead of the 2(n-1)/n S of P2P trees.  The switch defines the fp32
+ * summation order (oracle: tolerance mode, int32 exact); nvls lines need the
+ * whole ready mask and no late join (UNSUPPORTED otherwise) and run on the
+ * LDG kernel.  Collective over every rank (multi-process only; loopback:
+ * UNSUPPORTED).  Any failure on any rank (no multicast support, driver entry
+ * points, pidfd_getfd of rank 0's exported handle, binding) makes every rank
+ * return UNSUPPORTED and `why` (may be NULL) says why; an nvls line then
+ * makes its calls return UNSUPPORTED.  Calling it again replaces the team.
+ * Off by default. */
+ADAPCC_API adapcc_result_t adapcc_nvls_setup(adapcc_comm_t comm, size_t bytes, char* why, size_t why_len);
+
 /* Ticket of the most recent LATE_JOIN call (0 before the first). */
 ADAPCC_API adapcc_result_t adapcc_late_ticket(adapcc_comm_t comm, uint64_t* ticket);
 /* Consume a ticket without a LATE_JOIN call (host only; collective in the

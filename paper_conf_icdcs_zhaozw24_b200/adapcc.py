@@ -90,6 +90,7 @@ def _load():
         "adapcc_alltoallv": [vp, vp, vp, ctypes.POINTER(u64), i32, u64, vp],
         "adapcc_alltoallv_lb": [vp, pp, pp, ctypes.POINTER(u64), i32, u64, vp],
         "adapcc_late_ticket": [vp, ctypes.POINTER(u64)],
+        "adapcc_nvls_setup": [vp, sz, ctypes.c_char_p, sz],
         "adapcc_late_advance": [vp, ctypes.POINTER(u64)],
         "adapcc_link_probe": [vp, i32, u64, sz, i32, i32, i32, ctypes.POINTER(ctypes.c_double)],
         "adapcc_signal_ready": [vp, i32, u64, vp],
@@ -639,6 +640,15 @@ class Communicator:
     def spin(self, ns, stream=None):
         """Enqueue a one-thread %globaltimer spin of `ns` nanoseconds (controlled straggler)."""
         _check(_load().adapcc_spin(self._h, int(ns), _stream(stream, self.device)), "spin")
+
+    def nvls_setup(self, nbytes=256 << 20):
+        """Multicast team + NVLS scratch (adapcc_nvls_setup, collective).
+        Returns (ok, reason); ok False when the box cannot multicast."""
+        why = ctypes.create_string_buffer(256)
+        code = _load().adapcc_nvls_setup(self._h, nbytes, why, 256)
+        if code not in (SUCCESS, UNSUPPORTED):
+            raise AdapccError(code, "nvls_setup: " + why.value.decode())
+        return code == SUCCESS, why.value.decode()
 
     def late_advance(self):
         """Consume the next ticket without a LATE_JOIN call (adapcc_late_advance)."""

@@ -6,8 +6,10 @@
 // after one bootstrap all-gather of handles (Fig. 10), plus the
 // strategy per collective and a cache of compiled plans.  Every collective
 // call is one engine launch per segment on the caller's stream.
+#include <cuda.h>  // driver API types only: the functions are resolved with dlopen (NVLS setup)
 #include <cuda_runtime.h>
 #include <dlfcn.h>
+#include <sys/syscall.h>
 #include <fcntl.h>
 #include <sys/mman.h>
 #include <unistd.h>
@@ -202,6 +204,14 @@ struct adapcc_comm_s {
   uint64_t* d_board = nullptr;
   bool board_shm = false;    // shared across the ranks of the node
   bool board_pinned = false; // cudaHostAlloc'ed (else registered mmap)
+  // NVLS (NEXT-2): a multicast object over every rank's device, bound to a
+  // scratch allocation per rank; nvls_uc / nvls_mc = its unicast / multicast
+  // virtual addresses (adapcc_nvls_setup)
+  char* nvls_uc = nullptr;
+  char* nvls_mc = nullptr;
+  uint64_t nvls_bytes = 0;
+  unsigned long long nvls_mc_handle = 0, nvls_phys = 0;
+  int nvls_fd = -1;
 };
 
 namespace {
@@ -305,11 +315,14 @@ void board_free(adapcc_comm_s* c) {
   c->h_board = c->d_board = nullptr;
 }
 
+void nvls_release(adapcc_comm_s* c);
+
 void release(adapcc_comm_s* c) {
   if (!c) return;
   cudaSetDevice(c->device);
   cudaDeviceSynchronize();
   board_free(c);
+  nvls_release(c);
   c->plans.clear();
   c->retired.clear();
   for (auto& o : c->opened) cudaIpcCloseMemHandle(o.second.first);
@@ -439,9 +452,10 @@ adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, const Strategy* strat, uin
   rq.grid = grid_size(c, dtype, 0);
   rq.mode = mode;
   rq.half_bytes = c->half_bytes;
+  rq.nvls_bytes = c->nvls_bytes;
   std::vector<SegmentPlan> segs;
   std::string err;
-  if (!build_plan(rq, &segs, &err)) return ADAPCC_ERR_OOM;
+  if (!build_plan(rq, &segs, &err)) return err.rfind("unsupported", 0) == 0 ? ADAPCC_ERR_UNSUPPORTED : ADAPCC_ERR_OOM;
   auto plan = std::make_shared<DevPlan>();
   {
     uint64_t h = 1469598103934665603ull;
@@ -460,8 +474,11 @@ adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, const Strategy* strat, uin
     // (profiles/acc_r02.json); the shared-memory read-modify-write (acc_red
     // off) stages nsrc + nacc tiles per slot and is latency-bound, where the
     // 2 CTAs/SM x 3 x 32 KiB shape wins (profiles/acc_variants_r01.json).
-    // STAGED late join (decision words, conditional pushes) runs on the LDG kernel
+    // STAGED late join (decision words, conditional pushes) and NVLS
+    // (multimem) tasks run on the LDG kernel
     if (rq.late_join && mode == kStaged) plan->engine = 0;
+    for (auto& sp : segs)
+      if (sp.nvls) plan->engine = 0;
     plan->kernel = plan->engine == 0 ? 0 : (mode == kDirect && (!rq.accumulate || c->acc_red) ? 1 : 2);
     if (plan->kernel != 0 && (c->tma_shape == 1 || c->tma_shape == 2)) plan->kernel = (int)c->tma_shape;
   }
@@ -612,6 +629,8 @@ adapcc_result_t run(adapcc_comm_s* c, Coll coll, const void* const* send, void* 
     P.sig = fnv(fnv(plan->sig, si), sig_extra);
     P.state = c->state;
     P.err = c->d_err;
+    P.nvls_uc = c->nvls_uc;
+    P.nvls_mc = c->nvls_mc;
     P.trace = c->trace;
     P.trace_n = c->trace_n;
     P.trace_cap = c->trace_cap;
@@ -1170,6 +1189,224 @@ adapcc_result_t adapcc_alltoallv_lb(adapcc_comm_t c, const void* const* sendbufs
   return run(c, kAllToAll, sendbufs, recvbufs, 0, dtype, mask, 0, stream, 0, nullptr, nullptr, counts);
 }
 
+// ------------------------------------------------------------ NVLS (NEXT-2)
+}  // extern "C"
+namespace {
+// driver entry points for the multicast set-up, resolved at run time (the
+// library must load on machines without a driver)
+struct Drv {
+  CUresult (*DeviceGet)(CUdevice*, int);
+  CUresult (*DeviceGetAttribute)(int*, CUdevice_attribute, CUdevice);
+  CUresult (*MulticastCreate)(CUmemGenericAllocationHandle*, const CUmulticastObjectProp*);
+  CUresult (*MulticastGetGranularity)(size_t*, const CUmulticastObjectProp*, CUmulticastGranularity_flags);
+  CUresult (*MulticastAddDevice)(CUmemGenericAllocationHandle, CUdevice);
+  CUresult (*MulticastBindMem)(CUmemGenericAllocationHandle, size_t, CUmemGenericAllocationHandle, size_t, size_t,
+                               unsigned long long);
+  CUresult (*MulticastUnbind)(CUmemGenericAllocationHandle, CUdevice, size_t, size_t);
+  CUresult (*MemCreate)(CUmemGenericAllocationHandle*, size_t, const CUmemAllocationProp*, unsigned long long);
+  CUresult (*MemRelease)(CUmemGenericAllocationHandle);
+  CUresult (*MemAddressReserve)(CUdeviceptr*, size_t, size_t, CUdeviceptr, unsigned long long);
+  CUresult (*MemAddressFree)(CUdeviceptr, size_t);
+  CUresult (*MemMap)(CUdeviceptr, size_t, size_t, CUmemGenericAllocationHandle, unsigned long long);
+  CUresult (*MemUnmap)(CUdeviceptr, size_t);
+  CUresult (*MemSetAccess)(CUdeviceptr, size_t, const CUmemAccessDesc*, size_t);
+  CUresult (*MemExportToShareableHandle)(void*, CUmemGenericAllocationHandle, CUmemAllocationHandleType,
+                                         unsigned long long);
+  CUresult (*MemImportFromShareableHandle)(CUmemGenericAllocationHandle*, void*, CUmemAllocationHandleType);
+  bool ok = false;
+};
+
+const Drv& drv() {
+  static Drv d = [] {
+    Drv x{};
+    void* h = dlopen("libcuda.so.1", RTLD_NOW | RTLD_LOCAL);
+    if (!h) return x;
+    bool all = true;
+    auto get = [&](auto& fn, const char* name) {
+      fn = reinterpret_cast<std::remove_reference_t<decltype(fn)>>(dlsym(h, name));
+      all = all && fn != nullptr;
+    };
+    get(x.DeviceGet, "cuDeviceGet");
+    get(x.DeviceGetAttribute, "cuDeviceGetAttribute");
+    get(x.MulticastCreate, "cuMulticastCreate");
+    get(x.MulticastGetGranularity, "cuMulticastGetGranularity");
+    get(x.MulticastAddDevice, "cuMulticastAddDevice");
+    get(x.MulticastBindMem, "cuMulticastBindMem");
+    get(x.MulticastUnbind, "cuMulticastUnbind");
+    get(x.MemCreate, "cuMemCreate");
+    get(x.MemRelease, "cuMemRelease");
+    get(x.MemAddressReserve, "cuMemAddressReserve");
+    get(x.MemAddressFree, "cuMemAddressFree");
+    get(x.MemMap, "cuMemMap");
+    get(x.MemUnmap, "cuMemUnmap");
+    get(x.MemSetAccess, "cuMemSetAccess");
+    get(x.MemExportToShareableHandle, "cuMemExportToShareableHandle");
+    get(x.MemImportFromShareableHandle, "cuMemImportFromShareableHandle");
+    x.ok = all;
+    return x;
+  }();
+  return d;
+}
+
+void nvls_free(adapcc_comm_s* c) {
+  const Drv& d = drv();
+  if (!d.ok) return;
+  cudaDeviceSynchronize();
+  CUdevice dev;
+  d.DeviceGet(&dev, c->device);
+  if (c->nvls_mc) {
+    d.MemUnmap((CUdeviceptr)c->nvls_mc, c->nvls_bytes);
+    d.MemAddressFree((CUdeviceptr)c->nvls_mc, c->nvls_bytes);
+  }
+  if (c->nvls_uc) {
+    d.MemUnmap((CUdeviceptr)c->nvls_uc, c->nvls_bytes);
+    d.MemAddressFree((CUdeviceptr)c->nvls_uc, c->nvls_bytes);
+  }
+  if (c->nvls_mc_handle && c->nvls_phys) d.MulticastUnbind(c->nvls_mc_handle, dev, 0, c->nvls_bytes);
+  if (c->nvls_phys) d.MemRelease(c->nvls_phys);
+  if (c->nvls_mc_handle) d.MemRelease(c->nvls_mc_handle);
+  if (c->nvls_fd >= 0) close(c->nvls_fd);
+  c->nvls_uc = c->nvls_mc = nullptr;
+  c->nvls_mc_handle = c->nvls_phys = 0;
+  c->nvls_bytes = 0;
+  c->nvls_fd = -1;
+}
+
+void nvls_release(adapcc_comm_s* c) {
+  if (c->nvls_bytes || c->nvls_mc_handle || c->nvls_phys) nvls_free(c);
+}
+
+// plans depend on whether NVLS scratch exists (nvls lines plan against it)
+void drop_plans_nvls(adapcc_comm_s* c) {
+  for (auto& kv : c->plans)
+    if (kv.second->pinned) c->retired.push_back(kv.second);
+  c->plans.clear();
+}
+}  // namespace
+extern "C" {
+
+adapcc_result_t adapcc_nvls_setup(adapcc_comm_t c, size_t bytes, char* why, size_t why_len) {
+  auto say = [&](const char* m) {
+    if (why && why_len) {
+      std::strncpy(why, m, why_len - 1);
+      why[why_len - 1] = 0;
+    }
+  };
+  if (!c || !bytes) return ADAPCC_ERR_INVALID_ARGUMENT;
+  if (c->loopback) { say("loopback: one device, no multicast team"); return ADAPCC_ERR_UNSUPPORTED; }
+  const uint64_t all = c->nranks >= 64 ? ~uint64_t(0) : ((uint64_t(1) << c->nranks) - 1);
+  if (c->members != all) { say("a rank was excluded: the multicast team is incomplete"); return ADAPCC_ERR_UNSUPPORTED; }
+  std::lock_guard<std::mutex> lock(c->mu);
+  CK(cudaSetDevice(c->device));
+  CK(cudaDeviceSynchronize());
+  if (c->nvls_bytes) nvls_free(c);
+  const Drv& d = drv();
+  std::string reason;
+  // every step ends with an all-gather of success flags, so that all ranks
+  // either finish the set-up or give up together
+  auto agree = [&](bool ok, const char* what) -> adapcc_result_t {
+    int mine = ok ? 1 : 0;
+    std::vector<int> v(c->nranks);
+    if (members_allgather(c, &mine, v.data(), sizeof(int)) != 0) return ADAPCC_ERR_BOOTSTRAP;
+    for (int x : v)
+      if (!x) {
+        if (reason.empty()) reason = ok ? std::string("a peer failed: ") + what : std::string(what);
+        return ADAPCC_ERR_UNSUPPORTED;
+      }
+    return ADAPCC_SUCCESS;
+  };
+  auto bail = [&](adapcc_result_t r) {
+    nvls_free(c);
+    say(reason.c_str());
+    drop_plans_nvls(c);
+    return r;
+  };
+  CUdevice dev = 0;
+  int mc_ok = 0;
+  bool ok = d.ok && d.DeviceGet(&dev, c->device) == CUDA_SUCCESS &&
+            d.DeviceGetAttribute(&mc_ok, CU_DEVICE_ATTRIBUTE_MULTICAST_SUPPORTED, dev) == CUDA_SUCCESS && mc_ok;
+  adapcc_result_t r = agree(ok, d.ok ? "device without multicast support" : "driver without multicast entry points");
+  if (r) return bail(r);
+  CUmulticastObjectProp mp{};
+  mp.numDevices = (unsigned)c->nranks;
+  mp.handleTypes = CU_MEM_HANDLE_TYPE_POSIX_FILE_DESCRIPTOR;
+  mp.size = bytes;
+  size_t gran = 0;
+  ok = d.MulticastGetGranularity(&gran, &mp, CU_MULTICAST_GRANULARITY_RECOMMENDED) == CUDA_SUCCESS && gran;
+  if ((r = agree(ok, "cuMulticastGetGranularity"))) return bail(r);
+  const size_t size = (bytes + gran - 1) / gran * gran;
+  mp.size = size;
+  c->nvls_bytes = size;
+  // rank 0 creates the multicast object and exports it as a file descriptor;
+  // the others duplicate that descriptor out of rank 0's process (pidfd_getfd)
+  struct Share { int64_t pid; int32_t fd; int32_t ok; };
+  Share me{(int64_t)getpid(), -1, 1};
+  if (c->rank == 0) {
+    CUmemGenericAllocationHandle h = 0;
+    int fd = -1;
+    me.ok = d.MulticastCreate(&h, &mp) == CUDA_SUCCESS &&
+            d.MemExportToShareableHandle(&fd, h, CU_MEM_HANDLE_TYPE_POSIX_FILE_DESCRIPTOR, 0) == CUDA_SUCCESS;
+    c->nvls_mc_handle = h;
+    c->nvls_fd = fd;
+    me.fd = fd;
+  }
+  std::vector<Share> sh(c->nranks);
+  if (members_allgather(c, &me, sh.data(), sizeof(Share)) != 0) return bail(ADAPCC_ERR_BOOTSTRAP);
+  if ((r = agree(sh[0].ok != 0, "cuMulticastCreate / export"))) return bail(r);
+  if (c->rank != 0) {
+#ifndef SYS_pidfd_open
+#define SYS_pidfd_open 434
+#endif
+#ifndef SYS_pidfd_getfd
+#define SYS_pidfd_getfd 438
+#endif
+    const int pfd = (int)syscall(SYS_pidfd_open, (pid_t)sh[0].pid, 0);
+    const int fd = pfd >= 0 ? (int)syscall(SYS_pidfd_getfd, pfd, sh[0].fd, 0) : -1;
+    if (pfd >= 0) close(pfd);
+    CUmemGenericAllocationHandle h = 0;
+    ok = fd >= 0 && d.MemImportFromShareableHandle(&h, reinterpret_cast<void*>((intptr_t)fd),
+                                                   CU_MEM_HANDLE_TYPE_POSIX_FILE_DESCRIPTOR) == CUDA_SUCCESS;
+    c->nvls_mc_handle = h;
+    c->nvls_fd = fd;
+  } else {
+    ok = true;
+  }
+  if ((r = agree(ok, "importing the multicast handle (pidfd_getfd)"))) return bail(r);
+  ok = d.MulticastAddDevice(c->nvls_mc_handle, dev) == CUDA_SUCCESS;
+  if ((r = agree(ok, "cuMulticastAddDevice"))) return bail(r);
+  CUmemAllocationProp ap{};
+  ap.type = CU_MEM_ALLOCATION_TYPE_PINNED;
+  ap.location.type = CU_MEM_LOCATION_TYPE_DEVICE;
+  ap.location.id = c->device;
+  CUmemGenericAllocationHandle ph = 0;
+  ok = d.MemCreate(&ph, size, &ap, 0) == CUDA_SUCCESS;
+  c->nvls_phys = ok ? ph : 0;
+  ok = ok && d.MulticastBindMem(c->nvls_mc_handle, 0, ph, 0, size, 0) == CUDA_SUCCESS;
+  if ((r = agree(ok, "cuMemCreate / cuMulticastBindMem"))) return bail(r);
+  CUmemAccessDesc acc{};
+  acc.location.type = CU_MEM_LOCATION_TYPE_DEVICE;
+  acc.location.id = c->device;
+  acc.flags = CU_MEM_ACCESS_FLAGS_PROT_READWRITE;
+  CUdeviceptr uva = 0, mva = 0;
+  ok = d.MemAddressReserve(&uva, size, gran, 0, 0) == CUDA_SUCCESS;
+  if (ok) {
+    ok = d.MemMap(uva, size, 0, ph, 0) == CUDA_SUCCESS && d.MemSetAccess(uva, size, &acc, 1) == CUDA_SUCCESS;
+    if (ok) c->nvls_uc = reinterpret_cast<char*>(uva);
+    else d.MemAddressFree(uva, size);
+  }
+  ok = ok && d.MemAddressReserve(&mva, size, gran, 0, 0) == CUDA_SUCCESS;
+  if (ok) {
+    ok = d.MemMap(mva, size, 0, c->nvls_mc_handle, 0) == CUDA_SUCCESS &&
+         d.MemSetAccess(mva, size, &acc, 1) == CUDA_SUCCESS;
+    if (ok) c->nvls_mc = reinterpret_cast<char*>(mva);
+    else d.MemAddressFree(mva, size);
+  }
+  if ((r = agree(ok, "mapping the unicast / multicast addresses"))) return bail(r);
+  drop_plans_nvls(c);
+  say("ok");
+  return ADAPCC_SUCCESS;
+}
+
 // ----------------------------------------------------------- link probe (NEXT-2)
 adapcc_result_t adapcc_link_probe(adapcc_comm_t c, int src, uint64_t dst_mask, size_t bytes, int messages,
                                   int engine, int iters, double* seconds) {
@@ -1588,8 +1825,10 @@ adapcc_result_t adapcc_plan_stats(const char* text, uint64_t count, adapcc_dtype
   const size_t scratch = scratch_bytes ? scratch_bytes : kDefaultScratch;
   if (scratch < (size_t)kArenaHeader + 2 * (4096 + 65536)) return ADAPCC_ERR_INVALID_ARGUMENT;
   rq.half_bytes = ((scratch - kArenaHeader) / 2) / 256 * 256;
+  rq.nvls_bytes = uint64_t(1) << 30;  // host-only planning: as if 1 GiB of NVLS scratch were set up
   std::vector<SegmentPlan> segs;
-  if (!build_plan(rq, &segs, nullptr)) return ADAPCC_ERR_OOM;
+  std::string perr;
+  if (!build_plan(rq, &segs, &perr)) return perr.rfind("unsupported", 0) == 0 ? ADAPCC_ERR_UNSUPPORTED : ADAPCC_ERR_OOM;
   PlanStats s;
   for (auto& p : segs) accumulate_stats(p, rank, rq.esize, &s);
   s.segments = segs.size();
@@ -1629,8 +1868,10 @@ adapcc_result_t adapcc_plan_items(const char* text, uint64_t count, adapcc_dtype
   const size_t scratch = scratch_bytes ? scratch_bytes : kDefaultScratch;
   if (scratch < (size_t)kArenaHeader + 2 * (4096 + 65536)) return ADAPCC_ERR_INVALID_ARGUMENT;
   rq.half_bytes = ((scratch - kArenaHeader) / 2) / 256 * 256;
+  rq.nvls_bytes = uint64_t(1) << 30;  // host-only planning: as if 1 GiB of NVLS scratch were set up
   std::vector<SegmentPlan> segs;
-  if (!build_plan(rq, &segs, nullptr)) return ADAPCC_ERR_OOM;
+  std::string perr;
+  if (!build_plan(rq, &segs, &perr)) return perr.rfind("unsupported", 0) == 0 ? ADAPCC_ERR_UNSUPPORTED : ADAPCC_ERR_OOM;
   if ((size_t)segment >= segs.size()) return ADAPCC_ERR_INVALID_ARGUMENT;
   const SegmentPlan& sp = segs[segment];
   const std::vector<Item> it = order_items(sp, rank, rq.esize, grid, (uint64_t)piece_kib * 1024, taper, tma != 0);

@@ -74,6 +74,7 @@ struct Shared {
   int bad_align;
   int abort;
   int any_acc;
+  int nvls_alias;              // the item touches the NVLS scratch (unicast and multicast aliases)
 };
 
 // 16-byte global -> shared copy that completes asynchronously (blob prefetch)
@@ -170,6 +171,39 @@ __device__ __forceinline__ void fold_vec(const Shared& sh, int nsrc, int ndst, u
   }
 }
 
+// NVLS (NEXT-2 switch reduction): every 16-byte vector of the multicast
+// source is summed over all ranks' copies by the NVSwitch (multimem
+// ld_reduce; fp32 adds in the switch's order, bf16 accumulated in fp32 and
+// rounded once, int32 wrapping) and the sum is stored to every rank's copy of
+// the multicast destination (multimem.st).
+template <int DT>
+__device__ __forceinline__ uint4 mm_ld_reduce(const char* p) {
+  uint4 v;
+  if constexpr (DT == kF32)
+    asm volatile("multimem.ld_reduce.relaxed.sys.global.add.v4.f32 {%0,%1,%2,%3}, [%4];"
+                 : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p) : "memory");
+  else if constexpr (DT == kBF16)
+    asm volatile("multimem.ld_reduce.relaxed.sys.global.add.acc::f32.v4.bf16x2 {%0,%1,%2,%3}, [%4];"
+                 : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p) : "memory");
+  else {
+    asm volatile("multimem.ld_reduce.relaxed.sys.global.add.u32 %0, [%1];" : "=r"(v.x) : "l"(p) : "memory");
+    asm volatile("multimem.ld_reduce.relaxed.sys.global.add.u32 %0, [%1];" : "=r"(v.y) : "l"(p + 4) : "memory");
+    asm volatile("multimem.ld_reduce.relaxed.sys.global.add.u32 %0, [%1];" : "=r"(v.z) : "l"(p + 8) : "memory");
+    asm volatile("multimem.ld_reduce.relaxed.sys.global.add.u32 %0, [%1];" : "=r"(v.w) : "l"(p + 12) : "memory");
+  }
+  return v;
+}
+__device__ __forceinline__ void mm_st(char* p, uint4 v) {
+  asm volatile("multimem.st.relaxed.sys.global.v4.f32 [%0], {%1,%2,%3,%4};" ::"l"(p), "r"(v.x), "r"(v.y), "r"(v.z),
+               "r"(v.w) : "memory");
+}
+template <int DT, class SH>
+__device__ void nvls_vec(const SH& sh, uint32_t nvec) {
+  for (uint32_t v = threadIdx.x; v < nvec; v += kThreads)
+    mm_st(sh.dst[0] + (size_t)v * 16, mm_ld_reduce<DT>(sh.src[0] + (size_t)v * 16));
+}
+__device__ __forceinline__ void fence_proxy_alias() { asm volatile("fence.proxy.alias;" ::: "memory"); }
+
 // element path (misaligned slots / ragged tail): e in [e_begin, e_end)
 template <int DT>
 __device__ __forceinline__ void fold_scalar(const Shared& sh, int nsrc, int ndst, uint64_t e_begin,
@@ -204,6 +238,10 @@ __device__ void fold_chunk(const Shared& sh, int nsrc, int ndst, uint64_t n, int
   using O = Ops<DT>;
   using E = typename O::E;
   if (op == kOpNone) return;  // (STAGED late join: nothing to move for this chunk)
+  if (op == kOpNvls) {        // (planned on whole 16-byte vectors only)
+    nvls_vec<DT>(sh, (uint32_t)(n * O::kEsize / 16));
+    return;
+  }
   if (op == kOpZero) {
     for (int d = 0; d < ndst; ++d)
       for (uint64_t e = threadIdx.x; e < n; e += kThreads)
@@ -227,7 +265,8 @@ __device__ void fold_chunk(const Shared& sh, int nsrc, int ndst, uint64_t n, int
 template <int DT, int NR>
 __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __grid_constant__ LaunchParamsT<NR> P) {
   __shared__ Shared sh;
-  __shared__ char* sbase[3][NR];  // P.send / P.recv / P.hdr (indexed by BufKind), copied from the params
+  // P.send / P.recv / P.hdr / NVLS scratch (unicast, multicast), indexed by BufKind
+  __shared__ char* sbase[kNumBufKinds][NR];
   const bool sys = P.ipc;
   const uint64_t t_entry = P.trace ? globaltimer() : 0;
   Item pre{};  // thread 0: this CTA's first item, loaded together with the epoch
@@ -239,9 +278,9 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
   int buf = 0;  // blob buffer of the current item (static schedule)
   // buffer bases into shared memory (indexed by BufKind): read once per CTA,
   // before the stream-order wait
-  for (int i = threadIdx.x; i < 3 * P.nranks; i += kThreads) {
+  for (int i = threadIdx.x; i < kNumBufKinds * P.nranks; i += kThreads) {
     const int k = i / P.nranks, q = i - k * P.nranks;
-    sbase[k][q] = k == 0 ? P.send[q] : k == 1 ? P.recv[q] : P.hdr[q];
+    sbase[k][q] = k == 0 ? P.send[q] : k == 1 ? P.recv[q] : k == 2 ? P.hdr[q] : k == 3 ? P.nvls_uc : P.nvls_mc;
   }
   if (threadIdx.x == 0 && !use_blob && blockIdx.x < P.nitems) pre = P.items[blockIdx.x];
   constexpr int esize = Ops<DT>::kEsize;
@@ -253,6 +292,7 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
     if (P.trace) sh.tr0 = globaltimer();
     sh.bad_align = 0;
     sh.any_acc = 0;
+    sh.nvls_alias = 0;
     if (it >= P.nitems) return;
     const Item item = fb ? *reinterpret_cast<const Item*>(&sh.blob[b][0]) : is_first ? pre : P.items[it];
     const Task& t = fb ? *reinterpret_cast<const Task*>(&sh.blob[b][1]) : P.tasks[item.task];
@@ -341,6 +381,7 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
     const bool arena = r.kind == kBufArena;
     char* p = sbase[r.kind][r.rank] + (arena ? hoff : 0) + r.bias + (int64_t)(sh.cur.e0 * esize);
     if (reinterpret_cast<uintptr_t>(p) & 15) atomicOr(&sh.bad_align, 1);  // (hoff is 256-byte aligned)
+    if (r.kind >= kBufNvlsUc) atomicOr(&sh.nvls_alias, 1);
     if (i < nsrc) {
       sh.src[i] = p;
     } else {
@@ -528,8 +569,13 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
       __syncthreads();
     }
     const int nsrc = sh.cur.nsrc, ndst = sh.cur.ndst, npost = sh.cur.npost;
+    const bool alias = sh.nvls_alias != 0;
     if (!dropped) {
+      // NVLS scratch is written through one address alias (unicast or
+      // multicast) and read through the other: proxy fences on both sides
+      if (alias) fence_proxy_alias();
       fold_chunk<DT>(sh, nsrc, ndst, sh.cur.len, sh.cur.op);
+      if (alias) fence_proxy_alias();
       if (stat) cp_async_wait_all();  // the next blob has landed before the barrier publishes it
       __syncthreads();
       // npost was read before the barrier: after it, only thread 0 touches

@@ -24,9 +24,13 @@ constexpr int kArenaHeader = 4096;  // per-rank arena header (done epoch)
 // first items need more words go without blobs.
 constexpr int kFirstMaxWords = 72;
 
-enum BufKind : uint8_t { kBufSend = 0, kBufRecv = 1, kBufArena = 2 };
+enum BufKind : uint8_t { kBufSend = 0, kBufRecv = 1, kBufArena = 2,
+                         kBufNvlsUc = 3,   // this rank's NVLS scratch, unicast address (adapcc_nvls_setup)
+                         kBufNvlsMc = 4 }; // the NVLS scratch, multicast address (every rank's copy at once)
+constexpr int kNumBufKinds = 5;
 enum DType : int { kF32 = 0, kBF16 = 1, kI32 = 2 };
-enum TaskOp : uint16_t { kOpFold = 0, kOpZero = 1, kOpNone = 2 /* (runtime only) no data */ };
+enum TaskOp : uint16_t { kOpFold = 0, kOpZero = 1, kOpNone = 2 /* (runtime only) no data */,
+                         kOpNvls = 3 /* dst(mc) = switch sum of src(mc) over every rank: multimem.ld_reduce + st */ };
 // Late join on STAGED plans (NEXT-1): the late rank pushes its chunk
 // to the tree root itself, conditionally, and every decision travels in a
 // per-chunk word placed before the slot it describes.

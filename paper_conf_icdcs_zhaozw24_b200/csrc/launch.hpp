@@ -97,6 +97,8 @@ struct LaunchCore {
   uint32_t launch_seq;
   DevState* state;
   int* err;             // host-mapped error word
+  char* nvls_uc;        // NVLS scratch of this rank: unicast / multicast address (nullptr: no NVLS)
+  char* nvls_mc;
 };
 
 template <int NR>

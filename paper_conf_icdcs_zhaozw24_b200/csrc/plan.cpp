@@ -88,8 +88,15 @@ class Builder {
   bool fits() const {
     for (int r = 0; r < n_; ++r)
       if (flags_used_[r] > flag_cap_ || flag_cap_ + used_[r] > half_) return false;
-    return true;
+    return nvls_used_ <= nvls_cap_;
   }
+  // NVLS scratch: the same offsets on every rank (one multicast address)
+  uint64_t nvls_alloc(uint64_t bytes) {
+    const uint64_t off = nvls_used_;
+    nvls_used_ = align_up(nvls_used_ + bytes, kAlign);
+    return off;
+  }
+  uint64_t nvls_used_ = 0, nvls_cap_ = 0;
 
   // Slot holding elements [lo,hi) of a stream at rank r: address(e) = base + off + (e-lo)*esize
   Stream slot_stream(int r, uint64_t off, uint64_t lo, const FlagRef* f) {
@@ -145,6 +152,17 @@ class Builder {
     for (auto& f : posts) producer_[{f.rank, f.off}] = idx;
     p_.tasks.push_back(t);
     p_.max_level = std::max(p_.max_level, level);
+    return idx;
+  }
+
+  // a task with one source stream whose chunk is ready after ALL of `waits`'
+  // flags (NVLS: every rank copied its part in)
+  int add_multiwait(int owner, uint64_t lo, uint64_t hi, uint32_t ce, uint16_t op, const std::vector<Stream>& waits,
+                    const std::vector<BufRef>& dsts, const std::vector<FlagRef>& posts) {
+    std::vector<FlagRef> extra;
+    for (size_t i = 1; i < waits.size(); ++i) extra.push_back(waits[i].flag);
+    const int idx = add(owner, lo, hi, ce, op, {waits[0]}, dsts, posts, {}, extra, kLateNone);
+    p_.tasks[idx].nlwait = 0;
     return idx;
   }
 
@@ -321,6 +339,83 @@ void plan_allreduce_tree(Builder& B, const SubColl& s, uint64_t lo, uint64_t hi,
   }
 }
 
+// ----------------------------------------------------------------- NVLS
+// An nvls sub-collective (NEXT-2; the NVSwitch as the aggregation point --
+// the B200 counterpart of the paper's switch / NIC nodes of the communication
+// graph): every rank copies its partition into its multicast-bound
+// scratch (one flag per slice owner), slice owner k sums slice k over all
+// ranks' copies in the switch and stores the sum to all of them at once
+// (multimem ld_reduce + st, one flag to every rank), and every rank copies
+// the sums out to its recvbuf.  Per GPU and direction ~S crosses NVLink
+// instead of 2(n-1)/n S for P2P trees.  The switch sums every rank's copy,
+// so it needs the whole mask; the sub-16-byte tail of the last partition
+// goes through a star tree at rank 0.
+void plan_nvls(Builder& B, const SubColl& s, uint64_t lo, uint64_t hi, uint64_t mask, bool accumulate, Mode mode,
+               bool late_join, std::string* unsupported) {
+  const int n = B.n_;
+  const int es = B.esize_;
+  const uint64_t all = n >= 64 ? ~uint64_t(0) : ((uint64_t(1) << n) - 1);
+  if (B.nvls_cap_ == 0) { *unsupported = "nvls line without NVLS scratch (adapcc_nvls_setup)"; return; }
+  if ((mask & all) != all || B.members_ != all) {
+    *unsupported = "nvls lines reduce every rank's copy: the whole mask is required";
+    return;
+  }
+  if (late_join) { *unsupported = "late join on nvls lines"; return; }
+  const uint64_t unit = 16 / es;
+  const uint64_t hal = lo + (hi - lo) / unit * unit;
+  if (hal < hi) {  // ragged tail: a star tree rooted at rank 0
+    SubColl star;
+    star.kind = kTree;
+    star.weight = 1;
+    star.chunk = s.chunk;
+    star.parent.assign(n, 0);
+    star.parent[0] = -1;
+    star.root = 0;
+    star.children.assign(n, {});
+    for (int g = 1; g < n; ++g) star.children[0].push_back(g);
+    plan_allreduce_tree(B, star, hal, hi, mask, accumulate, mode, 0, false, false);
+  }
+  if (hal <= lo) return;
+  const uint64_t L = hal - lo, bytes = L * es;
+  const uint64_t in_off = B.nvls_alloc(bytes), out_off = B.nvls_alloc(bytes);
+  const int64_t in_bias = (int64_t)in_off - (int64_t)(lo * es), out_bias = (int64_t)out_off - (int64_t)(lo * es);
+  const uint32_t ce = std::max<uint32_t>((uint32_t)unit, B.chunk_elems(s.chunk) / (uint32_t)unit * (uint32_t)unit);
+  const uint64_t units = L / unit;
+  for (int k = 0; k < n; ++k) {  // slice k: reduced by rank k
+    const uint64_t a = lo + units * k / n * unit, b = lo + units * (k + 1) / n * unit;
+    if (a >= b) continue;
+    const uint32_t nch = (uint32_t)((b - a + ce - 1) / ce);
+    std::vector<FlagRef> fin(n), fout(n);
+    for (int q = 0; q < n; ++q) {
+      fin[q] = B.alloc_flags(k, nch);   // "rank q copied slice k in", at rank k
+      fout[q] = B.alloc_flags(q, nch);  // "slice k is summed", at rank q
+    }
+    for (int q = 0; q < n; ++q) {
+      Stream src;
+      src.ref = make_ref(kBufSend, q, 0);
+      B.add(q, a, b, ce, kOpFold, {src}, {make_ref(kBufNvlsUc, q, in_bias)}, {fin[q]});
+    }
+    std::vector<Stream> waits;
+    for (int q = 0; q < n; ++q) {
+      Stream w;
+      w.ref = make_ref(kBufNvlsMc, k, in_bias);
+      w.wait = true;
+      w.flag = fin[q];
+      waits.push_back(w);
+    }
+    // one source stream (the multicast input), waited for through n flags
+    B.add_multiwait(k, a, b, ce, kOpNvls, waits, {make_ref(kBufNvlsMc, k, out_bias)}, fout);
+    for (int q = 0; q < n; ++q) {
+      Stream src;
+      src.ref = make_ref(kBufNvlsUc, q, out_bias);
+      src.wait = true;
+      src.flag = fout[q];
+      B.add(q, a, b, ce, kOpFold, {src}, {make_ref(kBufRecv, q, 0, accumulate)}, {});
+    }
+  }
+  B.p_.nvls = true;
+}
+
 // ------------------------------------------------------------- AllGather
 // slot_bias < 0: AllGather (source s lands in slot s of every recvbuf);
 // otherwise Broadcast (lands at that byte offset).
@@ -479,6 +574,7 @@ SegmentPlan build_units(const PlanRequest& rq, const std::vector<std::pair<uint6
                         uint64_t seg_k, uint64_t nseg, uint64_t unit_cap) {
   const Strategy& st = *rq.st;
   Builder B(st.nranks, rq.esize, rq.half_bytes, rq.members, unit_cap);
+  B.nvls_cap_ = rq.nvls_bytes;
   if (rq.counts) {
     plan_alltoallv(B, rq, seg_k, nseg);
     return B.finish();
@@ -489,7 +585,8 @@ SegmentPlan build_units(const PlanRequest& rq, const std::vector<std::pair<uint6
     const SubColl& s = st.subs[m];
     switch (st.coll) {
       case kAllReduce:
-        plan_allreduce_tree(B, s, lo, hi, rq.ready_mask, rq.accumulate, rq.mode, 0, false, rq.late_join);
+        if (s.kind == kNvls) plan_nvls(B, s, lo, hi, rq.ready_mask, rq.accumulate, rq.mode, rq.late_join, &B.p_.unsupported);
+        else plan_allreduce_tree(B, s, lo, hi, rq.ready_mask, rq.accumulate, rq.mode, 0, false, rq.late_join);
         break;
       case kReduce: plan_allreduce_tree(B, s, lo, hi, rq.ready_mask, rq.accumulate, rq.mode, 0, true); break;
       case kReduceScatter:
@@ -551,6 +648,10 @@ bool build_plan(const PlanRequest& rq, std::vector<SegmentPlan>* segs, std::stri
         rr[m] = {a, b};
       }
       SegmentPlan p = build_segment(rq, rr, k, nseg);
+      if (!p.unsupported.empty()) {
+        if (err) *err = "unsupported: " + p.unsupported;
+        return false;
+      }
       if (rq.counts) {
         uint64_t cmax = 0;
         const int n = rq.st->nranks;

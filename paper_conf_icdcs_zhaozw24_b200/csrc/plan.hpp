@@ -32,6 +32,8 @@ struct SegmentPlan {
   std::vector<uint64_t> arena_used;  // per rank, bytes inside one parity half
   uint32_t max_level = 0;
   bool fits = true;                  // flags and data fit their regions
+  bool nvls = false;                 // has NVLS tasks (LDG kernel only)
+  std::string unsupported;           // non-empty: the call cannot run (reason)
 };
 
 struct PlanRequest {
@@ -53,6 +55,9 @@ struct PlanRequest {
   // CTAs the call will run on (0: pipeline in units of the strategy's chunks
   // only); small calls subdivide chunks so that every CTA gets work (R8).
   int grid = 0;
+  // NVLS scratch bytes per rank (adapcc_nvls_setup; 0 = none): nvls lines
+  // need it, the whole mask, and a multi-process communicator
+  uint64_t nvls_bytes = 0;
 };
 
 // Bytes at the start of each parity half reserved for per-chunk flag words.

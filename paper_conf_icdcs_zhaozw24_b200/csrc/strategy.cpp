@@ -192,7 +192,7 @@ bool parse_strategy(const char* text, Strategy* out, std::string* err) {
       else return fail(err, "unknown collective");
       continue;
     }
-    if (t[0] != "tree" && t[0] != "ring" && t[0] != "bcast" && t[0] != "a2a" && t[0] != "rtree")
+    if (t[0] != "tree" && t[0] != "ring" && t[0] != "bcast" && t[0] != "a2a" && t[0] != "rtree" && t[0] != "nvls")
       return fail(err, "unknown directive " + t[0]);
     Raw r;
     r.head = t[0];
@@ -212,7 +212,7 @@ bool parse_strategy(const char* text, Strategy* out, std::string* err) {
   st.nranks = n;
   st.coll = (Coll)coll;
   for (const Raw& r : raws) {
-    const bool ok_kind = (coll == kAllReduce && (r.head == "tree" || r.head == "ring")) ||
+    const bool ok_kind = (coll == kAllReduce && (r.head == "tree" || r.head == "ring" || r.head == "nvls")) ||
                          (coll == kAllGather && r.head == "bcast") ||
                          (coll == kAllToAll && r.head == "a2a") ||
                          (coll == kReduce && r.head == "tree") ||
@@ -265,6 +265,11 @@ bool parse_strategy(const char* text, Strategy* out, std::string* err) {
     SubColl s;
     s.weight = w * n;
     s.chunk = c;
+    if (r.head == "nvls") {  // the switch reduces and multicasts: no graph to give
+      s.kind = kNvls;
+      st.subs.push_back(std::move(s));
+      continue;
+    }
     if (r.head == "a2a") {
       s.kind = kA2A;
       if (r.kv.count("route") && !parse_routes(r.kv.at("route"), n, &s.routes, err)) return false;
@@ -330,6 +335,11 @@ bool check_members(const Strategy& st, uint64_t members, std::string* err) {
   const int n = st.nranks;
   auto alive = [&](int g) { return ((members >> g) & 1) != 0; };
   for (const SubColl& s : st.subs) {
+    if (s.kind == kNvls) {  // the multicast team is every rank of the communicator
+      if (members != (n >= 64 ? ~uint64_t(0) : ((uint64_t(1) << n) - 1)))
+        return fail(err, "an nvls line needs every rank (the multicast team)");
+      continue;
+    }
     if (s.kind == kA2A) {
       for (const Route& r : s.routes)
         for (int h : r.hops)

@@ -24,7 +24,8 @@ enum Coll : int {
   kReduce = 3, kBroadcast = 4, kReduceScatter = 5  // NEXT-4 primitives
 };
 constexpr int kNumColl = 6;
-enum SubKind : int { kTree = 0, kBcast = 1, kA2A = 2, kRTree = 3 };
+enum SubKind : int { kTree = 0, kBcast = 1, kA2A = 2, kRTree = 3,
+                     kNvls = 4 /* allreduce partition reduced by the NVSwitch (multimem, NEXT-2) */ };
 
 // One routed AlltoAll flow (routing variables x^f_ij, eq. 1): block
 // src -> dst travels src -> hops[0] -> ... -> hops.back() -> dst.

@@ -167,6 +167,17 @@ def allreduce_mask_aware_stars(n, ready, chunk=DEFAULT_CHUNK, bw=None, relays_as
 
 
 # ------------------------------------------------------------------- allgather
+def allreduce_nvls(n, chunk=DEFAULT_CHUNK, nvls_weight=1, star_weight=0):
+    """NVLS switch reduction (NEXT-2): one nvls line (the NVSwitch reduces and
+    multicasts its partition) plus, with star_weight > 0, n star trees sharing
+    the rest (weights are per line, reading Q9)."""
+    lines = [f"nvls weight={nvls_weight} chunk={chunk}"]
+    if star_weight:
+        for m in range(n):
+            lines.append(f"tree weight={star_weight} chunk={chunk} parent={_join(star_parent(n, m))}")
+    return _header(n, "allreduce") + "\n".join(lines) + "\n"
+
+
 def allgather_stars(n, chunk=DEFAULT_CHUNK):
     """One Broadcast per source, each a star from the source."""
     out = _header(n, "allgather")
