@@ -57,6 +57,9 @@ def parse_args():
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--no-parity", action="store_true")
     p.add_argument("--no-sweep", action="store_true", help="skip the busbw-vs-size sweep")
+    p.add_argument("--no-nccl-legs", action="store_true",
+                   help="N>1: skip the NCCL_ALGO / NVLS leg runs (separate torchrun jobs)")
+    p.add_argument("--nccl-leg", default=None, help=argparse.SUPPRESS)   # internal: one NCCL variant
     p.add_argument("--test-same-gpu", action="store_true",
                    help="N>1 code-path check on a 1-GPU box: every rank on cuda:0, gloo, no NCCL leg "
                         "(numbers are NOT NVLink measurements)")
@@ -408,6 +411,7 @@ def run_single(args):
         "clocks": clk.summary(),
         "parity": parity,
         "nccl": None,
+        "paper_context": PAPER_CONTEXT,
         "sweep": sweep,
         "sweep_how": "same call at every x4 size (slices of the bench buffers): back-to-back enqueue of a "
                      "prepared call (us: Communicator.prepare_allreduce_lb, one C call per AllReduce), of the "
@@ -526,6 +530,96 @@ def multi_complete_parity(comm, x, y, text, world, rank, count, dtype):
                          "element by element, ranks > 0 by SHA-256 of the whole output, bit-exact"}
 
 
+PAPER_CONTEXT = {
+    "claims": ["up to 2x communication speed-up vs NCCL (P:L7, P:L31, P:L319)",
+               "up to 31% training throughput improvement vs NCCL (P:L7, P:L321)",
+               "AllReduce 1.06x-1.29x vs NCCL / MSCCL (P:L291, P:L301)"],
+    "hardware": "6 servers: 4 x (4 A100, NVLink, 100 Gbps RDMA) + 2 x (4 V100, NVLink, 50 Gbps), CUDA 11.3 (P:L279)",
+    "note": "context only: a multi-server RDMA/TCP testbed with stragglers, not one NVSwitch node",
+}
+NCCL_LEGS = {"default": {}, "ring": {"NCCL_ALGO": "Ring"}, "tree": {"NCCL_ALGO": "Tree"},
+             "nvls": {"NCCL_ALGO": "NVLS"}, "nvls_off": {"NCCL_NVLS_ENABLE": "0"}}
+
+
+def p2p_ceiling(comm, world, rank, nbytes=64 << 20):
+    """In-run NVLink ceiling (adapcc_link_probe, graph-captured): copy engine
+    and TMA-store kernel, 1 -> 1 (every rank to its right neighbour at once, a
+    permutation round) and 1 -> n-1 (rank 0 to everyone); seconds are the max
+    over ranks; GB/s per direction of the sender."""
+    import torch
+    import torch.distributed as dist
+    out = {}
+    dev = "cpu" if dist.get_backend() == "gloo" else "cuda"
+    for eng in ("sm", "ce"):
+        t1 = comm.link_probe({(rank + 1) % world}, nbytes, engine=eng, iters=8)
+        tf = comm.link_probe(set(range(1, world)) if rank == 0 else set(), nbytes, engine=eng, iters=4)
+        t = torch.tensor([t1, tf], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        t1, tf = float(t[0]), float(t[1])
+        out[eng] = {"one_to_one_GBps": round(nbytes / t1 / 1e9, 1),
+                    "one_to_all_GBps_per_dst": round(nbytes / tf / 1e9, 1),
+                    "one_to_all_GBps_out": round((world - 1) * nbytes / tf / 1e9, 1)}
+    out["bytes"] = nbytes
+    return out
+
+
+def run_nccl_leg(args):
+    """One NCCL variant (environment set by the parent): busbw vs size for
+    fp32 and bf16, max over ranks; rank 0 prints one JSON line."""
+    import torch
+    import torch.distributed as dist
+    rank, world, local = dist_env()
+    torch.cuda.set_device(local)
+    dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    nbytes = int(args.size_mib * (1 << 20)) // 16 * 16
+    buf = torch.randn(nbytes // 4, device="cuda")
+
+    def reduce_max(v, op="max"):
+        t = torch.tensor([v], dtype=torch.float64, device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX if op == "max" else dist.ReduceOp.MIN)
+        return float(t.item())
+
+    res = {}
+    for dt, tdt, es in (("f32", torch.float32, 4), ("bf16", torch.bfloat16, 2)):
+        pts = []
+        z = buf.view(tdt)
+        for sb in [b for b in SWEEP_SIZES if b <= nbytes]:
+            zs = z[:sb // es]
+            ms, _ = time_point(lambda: dist.all_reduce(zs), reduce_max, graph=False)
+            pts.append({"bytes_per_rank": sb, "us": round(ms * 1e3, 2), "busbw": round(busbw(sb, ms / 1e3, world), 2)})
+        res[dt] = pts
+    if rank == 0:
+        print(json.dumps({"nccl_leg": args.nccl_leg, "env": NCCL_LEGS[args.nccl_leg], "sweep": res,
+                          "version": ".".join(map(str, torch.cuda.nccl.version()))}), flush=True)
+    dist.destroy_process_group()
+    return None
+
+
+def nccl_legs(args, world):
+    """Rank 0, after the main run: every NCCL variant as its own torchrun job
+    (NCCL reads NCCL_ALGO / NCCL_NVLS_ENABLE when it starts)."""
+    out = {}
+    for name, env in NCCL_LEGS.items():
+        e = dict(os.environ)
+        for k in list(e):
+            if k in ("RANK", "WORLD_SIZE", "LOCAL_RANK", "LOCAL_WORLD_SIZE", "MASTER_ADDR", "MASTER_PORT",
+                     "GROUP_RANK", "GROUP_WORLD_SIZE", "ROLE_RANK", "ROLE_WORLD_SIZE", "ROLE_NAME") or \
+                    k.startswith("TORCHELASTIC_"):
+                e.pop(k)
+        e.update(env)
+        cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={world}",
+               "--master-addr=127.0.0.1", f"--master-port={free_port()}", os.path.abspath(__file__),
+               "--gpus", str(world), "--nccl-leg", name, "--size-mib", str(args.size_mib)]
+        try:
+            p = subprocess.run(cmd, cwd=ROOT, capture_output=True, text=True, timeout=600, env=e)
+            lines = [ln for ln in p.stdout.splitlines() if ln.startswith("{")]
+            out[name] = json.loads(lines[-1]) if p.returncode == 0 and lines else \
+                {"unavailable": f"rc={p.returncode}: {p.stderr.strip().splitlines()[-1] if p.stderr.strip() else ''}"[:300]}
+        except Exception as ex:  # noqa: BLE001
+            out[name] = {"unavailable": repr(ex)[:300]}
+    return out
+
+
 def run_multi(args):
     import numpy as np
     import torch
@@ -560,6 +654,7 @@ def run_multi(args):
     # zero-copy: x / y registered once (CUDA IPC), DIRECT plan over NVLink
     comm.register(x)
     comm.register(y)
+    probes = p2p_ceiling(comm, world, rank)
 
     def timed(fn, steps):
         dist.barrier()
@@ -625,21 +720,41 @@ def run_multi(args):
 
     sweep = None
     if not args.no_sweep:   # busbw vs size, ours (zero-copy) and NCCL on the same buffers, max over ranks
-        sweep = []
-        for sb in [b for b in SWEEP_SIZES if b <= nbytes]:
-            c = sb // es
-            xs_, ys_, zs_ = x[:c], y[:c], z[:c]
-            call = comm.prepare_collective_zc("allreduce", xs_, ys_, c)
-            ms_, msg_ = time_point(call, reduce_max, fn_graph=lambda: comm.collective_zc("allreduce", xs_, ys_, c))
-            pt = {"bytes_per_rank": sb, "us": round(ms_ * 1e3, 2), "us_graph": round(msg_ * 1e3, 2),
-                  "busbw": round(busbw(sb, ms_ / 1e3, world), 2),
-                  "busbw_graph": round(busbw(sb, msg_ / 1e3, world), 2)}
-            if not args.test_same_gpu:
-                nms, _ = time_point(lambda: dist.all_reduce(zs_), reduce_max, graph=False)
-                pt.update({"nccl_us": round(nms * 1e3, 2), "nccl_busbw": round(busbw(sb, nms / 1e3, world), 2)})
-            sweep.append(pt)
+        sweep = {}
+        # fp32 and bf16 (C2): the other dtype reuses the registered bytes (timing only)
+        for sdt in [args.dtype] + [d for d in ("f32", "bf16") if d != args.dtype]:
+            sdt_t = torch.float32 if sdt == "f32" else torch.bfloat16
+            ses = 4 if sdt == "f32" else 2
+            xv, yv, zv = x.view(sdt_t), y.view(sdt_t), z.view(sdt_t)
+            pts = []
+            for sb in [b for b in SWEEP_SIZES if b <= nbytes]:
+                c = sb // ses
+                xs_, ys_, zs_ = xv[:c], yv[:c], zv[:c]
+                call = comm.prepare_collective_zc("allreduce", xs_, ys_, c)
+                ms_, msg_ = time_point(call, reduce_max,
+                                       fn_graph=lambda: comm.collective_zc("allreduce", xs_, ys_, c))
+                pt = {"bytes_per_rank": sb, "us": round(ms_ * 1e3, 2), "us_graph": round(msg_ * 1e3, 2),
+                      "busbw": round(busbw(sb, ms_ / 1e3, world), 2),
+                      "busbw_graph": round(busbw(sb, msg_ / 1e3, world), 2)}
+                if not args.test_same_gpu:
+                    nms, _ = time_point(lambda: dist.all_reduce(zs_), reduce_max, graph=False)
+                    pt.update({"nccl_us": round(nms * 1e3, 2), "nccl_busbw": round(busbw(sb, nms / 1e3, world), 2)})
+                pts.append(pt)
+            sweep[sdt] = pts
+    # NVLS switch reduction (NEXT-2): off by default, measured when the box can multicast
+    nvls = {"value": None, "reason": None}
+    ok_nv, why_nv = comm.nvls_setup(2 * nbytes + (16 << 20))
+    if ok_nv:
+        comm.set_strategy("allreduce", G.allreduce_nvls(world, chunk=args.chunk_kib * 1024))
+        ms_nv = timed(lambda: comm.allreduce(x, y), args.steps)
+        nvls.update({"value": round(busbw(nbytes, ms_nv / 1e3, world), 3), "unit": UNIT,
+                     "ms_per_step": round(ms_nv, 4), "path": "nvls line: multimem ld_reduce + st (STAGED copy in/out)"})
+        comm.set_strategy("allreduce", text)
+    else:
+        nvls["reason"] = why_nv
     parity = None if args.no_parity else multi_complete_parity(comm, x, y, text, world, rank, count, args.dtype)
     st = pkg.adapcc.plan_stats(text, count, args.dtype, (1 << world) - 1, rank=rank)
+    peak_dir = probes["sm"]["one_to_one_GBps"]
     dir_bytes = st["remote_bytes"]   # = bytes crossing each link direction of this GPU (symmetric plan)
     res = None
     if rank == 0:
@@ -651,9 +766,11 @@ def run_multi(args):
             "config": workload_config(args, world, world),
             "algbw": round(nbytes / (ms / 1e3) / 1e9, 3),
             "pct_of_nvlink_900": round(100 * value / NVLINK_NOMINAL, 2),
-            "roofline": {"bound": "nvlink", "achieved": round(dir_bytes / (ms / 1e3) / 1e9, 1), "peak": 770.0,
-                         "unit": "GB/s", "frac": round(dir_bytes / (ms / 1e3) / 1e9 / 770.0, 4), "traffic": None,
-                         "peak_source": "B200_PROFILING.md measured peer copy 770 GB/s per direction per GPU",
+            "roofline": {"bound": "nvlink" if not args.test_same_gpu else "hbm (all ranks on one GPU)",
+                         "achieved": round(dir_bytes / (ms / 1e3) / 1e9, 1), "peak": peak_dir,
+                         "unit": "GB/s", "frac": round(dir_bytes / (ms / 1e3) / 1e9 / peak_dir, 4), "traffic": None,
+                         "peak_source": "measured in this run: TMA-store probe 1 -> 1 per direction "
+                                        "(adapcc_link_probe, max over ranks); 900 nominal",
                          "algorithmic_bytes_per_direction": dir_bytes,
                          "why": "zero-copy star plan, per GPU g: g's kernel pulls (n-1)/n S (its trees' "
                                 "inputs) and pushes (n-1)/n S (their results), while peers pull g's "
@@ -670,6 +787,7 @@ def run_multi(args):
                          "zero-copy AllReduce, nccl = dist.all_reduce on the same sizes; back-to-back "
                          "enqueue (us; NCCL likewise) and, ours only, a CUDA graph (us_graph); max over ranks",
             "path": "zero-copy DIRECT plan over CUDA IPC (registered buffers)",
+            "p2p_ceiling": probes, "nvls": nvls, "paper_context": PAPER_CONTEXT,
             "staged": {"value": round(busbw(nbytes, ms_staged / 1e3, world), 3), "unit": UNIT,
                        "ms_per_step": round(ms_staged, 4),
                        "path": "STAGED protocol (landing + broadcast slots in IPC arenas)"},
@@ -678,6 +796,10 @@ def run_multi(args):
         }
     comm.finalize()
     dist.destroy_process_group()
+    if rank == 0 and not args.test_same_gpu and not args.no_nccl_legs:
+        del x, y, z, x2, y2
+        torch.cuda.empty_cache()
+        res["nccl_legs"] = nccl_legs(args, world)
     return res
 
 
@@ -716,7 +838,9 @@ def main():
     if "WORLD_SIZE" in os.environ and world != args.gpus:
         print(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={world}", file=sys.stderr)
         return 2
-    if args.impl == "reference":
+    if args.nccl_leg:
+        out = run_nccl_leg(args)
+    elif args.impl == "reference":
         out = run_reference(args)        # CPU only: no launcher needed, rank 0 prints
     elif args.gpus > 1 and "WORLD_SIZE" not in os.environ:
         return self_launch(args)

@@ -87,7 +87,11 @@ def test_ours_two_ranks_same_gpu_contract():
     assert d["n_gpus"] == 2 and d["async_error"] == 0 and d["config"]["same_gpu"]
     assert d["parity"]["complete"] and d["parity"]["mismatches"] == 0 and d["parity"]["ranks"] == 2
     assert d["parity"]["ranks_mismatched"] == []
-    assert [p["bytes_per_rank"] for p in d["sweep"]] == [1 << s for s in range(10, 24, 2)]
+    for dt in ("f32", "bf16"):   # C2 sweeps both dtypes
+        assert [p["bytes_per_rank"] for p in d["sweep"][dt]] == [1 << s for s in range(10, 24, 2)]
+    assert d["p2p_ceiling"]["sm"]["one_to_one_GBps"] > 0 and d["roofline"]["peak"] > 0
+    assert d["nvls"]["value"] is None and d["nvls"]["reason"]        # one GPU: no multicast team
+    assert "2x" in d["paper_context"]["claims"][0]
 
 
 def test_prepared_call_marshals_once():
