@@ -15,7 +15,7 @@ Format (one directive per line, '#' starts a comment):
     adapcc-strategy 1
     nranks <n>                                  1 <= n <= 64
     collective allreduce|allgather|alltoall
-    tree  weight=<w> chunk=<C> parent=<p_0,..,p_{n-1}> [noagg=<g,..>]   (allreduce)
+    tree  weight=<w> chunk=<C> parent=<p_0,..,p_{n-1}> [noagg=<g,..>] [relay=store|bypass]   (allreduce)
     ring  weight=<w> chunk=<C> order=<r_0,..,r_{n-1}>                     (allreduce)
     bcast src=<s> weight=<w> chunk=<C> parent=<p_0,..,p_{n-1}>           (allgather, broadcast)
     a2a   weight=<w> chunk=<C> [route=<s>:<d>:<h1>,..[;<s>:<d>:<h>,..]]  (alltoall)
@@ -60,6 +60,8 @@ class Sub:
     noagg: frozenset = frozenset()   # ranks g with a_{m,g} = 0
     src: int = -1             # bcast: source (== root); rtree: destination block (== root)
     routes: dict = field(default_factory=dict)   # a2a: (s, d) -> tuple of relay ranks
+    relay: str = "bypass"     # tree: how a pure relay forwards its single flow (data path only:
+                              # the bytes arrive unchanged either way, so results do not depend on it)
 
     @property
     def root(self):
@@ -205,7 +207,7 @@ def parse(text):
     keys = {"tree": {"weight", "chunk", "parent"}, "ring": {"weight", "chunk", "order"},
             "bcast": {"src", "weight", "chunk", "parent"}, "a2a": {"weight", "chunk"},
             "rtree": {"dst", "weight", "chunk", "parent"}, "nvls": {"weight", "chunk"}}
-    optional = {"tree": {"noagg"}, "ring": set(), "bcast": set(), "a2a": {"route"},
+    optional = {"tree": {"noagg", "relay"}, "ring": set(), "bcast": set(), "a2a": {"route"},
                 "rtree": {"noagg"}, "nvls": set()}
     if not raw_subs:
         raise StrategyError("no sub-collective lines")
@@ -240,7 +242,10 @@ def parse(text):
                     raise StrategyError("rtree root must be its dst")
                 st.subs.append(Sub("rtree", w * n, c, parent, frozenset(noagg), dst))
             else:
-                st.subs.append(Sub("tree", w * n, c, parent, frozenset(noagg)))
+                relay = kv.get("relay", "bypass")
+                if relay not in ("store", "bypass"):
+                    raise StrategyError("relay must be store or bypass")
+                st.subs.append(Sub("tree", w * n, c, parent, frozenset(noagg), relay=relay))
         elif head == "ring":
             order = _intlist(kv["order"], "order")
             if sorted(order) != list(range(n)):

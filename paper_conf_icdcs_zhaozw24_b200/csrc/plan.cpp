@@ -188,6 +188,44 @@ std::vector<int> bfs_order(const SubColl& s) {
 }
 
 // ------------------------------------------------------------- AllReduce
+// relay=store (relays forward "as intermediaries, relaying tensor
+// data from other workers"): a pure relay -- not ready, no kernel, one
+// incoming flow (P:L154(2)) -- receives that flow into its own arena and
+// forwards it, chunk by chunk, instead of being bypassed.  The behaviour
+// tuples are unchanged; for planning the relay's emitted flow becomes its
+// stored copy (Flow kAgg at the relay, a one-source "fold" = a byte copy), so
+// every consumer still folds the same bytes at the same position.
+struct RelayPlan {
+  std::vector<uint8_t> store;             // per rank: a store-and-forward relay
+  std::vector<std::vector<Flow>> src;     // its single incoming flow
+};
+
+RelayPlan store_relays(const SubColl& s, TreeBehavior* b) {
+  const int n = (int)s.parent.size();
+  RelayPlan rp;
+  rp.store.assign(n, 0);
+  rp.src.assign(n, {});
+  if (!s.relay_store) return rp;
+  for (int g : b->postorder) {  // children first: a relay below a relay forwards the stored copy
+    const Tuple& t = b->tup[g];
+    std::vector<Flow> f;
+    if (t.kern) {
+      f.push_back({Flow::kAgg, g});
+    } else {
+      if (t.act) f.push_back({Flow::kIn, g});
+      for (int c : s.children[g])
+        if (b->tup[c].send) f.insert(f.end(), b->flows[c].begin(), b->flows[c].end());
+    }
+    if (!t.kern && !t.act && t.recv && t.send && f.size() == 1 && g != s.root) {
+      rp.store[g] = 1;
+      rp.src[g] = f;
+      f = {{Flow::kAgg, g}};
+    }
+    b->flows[g] = f;
+  }
+  return rp;
+}
+
 // send_bias: byte offset of the tree's block inside every rank's sendbuf
 // (ReduceScatter block b); root_only: the result goes to the root's recvbuf
 // only (Reduce, ReduceScatter) instead of every rank (AllReduce).
@@ -199,7 +237,8 @@ void plan_allreduce_tree(Builder& B, const SubColl& s, uint64_t lo, uint64_t hi,
   const uint32_t ce = B.chunk_elems(s.chunk);
   const uint32_t nch = (uint32_t)((hi - lo + ce - 1) / ce);
   const uint64_t len = (hi - lo) * es;
-  const TreeBehavior b = tree_behavior(s, mask);
+  TreeBehavior b = tree_behavior(s, mask);
+  const RelayPlan rp = store_relays(s, &b);
   const int root = s.root;
 
   // sources folded at the root (kernel) or its single flow (no kernel)
@@ -220,12 +259,12 @@ void plan_allreduce_tree(Builder& B, const SubColl& s, uint64_t lo, uint64_t hi,
       return B.slot_stream(f.rank, as.first, lo, &as.second);
     };
     for (int k : b.postorder) {
-      if (!b.tup[k].kern || k == root) continue;
+      if (!(b.tup[k].kern || rp.store[k]) || k == root) continue;
       uint64_t off = B.alloc(k, len);
       FlagRef fl = B.alloc_flags(k, nch);
       agg_slot[k] = {off, fl};
       std::vector<Stream> srcs;
-      for (auto& f : kernel_sources(s, b, k)) srcs.push_back(stream_of(f));
+      for (auto& f : rp.store[k] ? rp.src[k] : kernel_sources(s, b, k)) srcs.push_back(stream_of(f));
       B.add(k, lo, hi, ce, kOpFold, srcs,
             {make_ref(kBufArena, k, (int64_t)off - (int64_t)(lo * es))}, {fl});
     }
@@ -247,10 +286,10 @@ void plan_allreduce_tree(Builder& B, const SubColl& s, uint64_t lo, uint64_t hi,
   std::map<int, std::vector<Stream>> consumer_srcs;
   std::vector<int> consumers;
   for (int k : b.postorder)
-    if (b.tup[k].kern && k != root) consumers.push_back(k);
+    if ((b.tup[k].kern || rp.store[k]) && k != root) consumers.push_back(k);
   consumers.push_back(root);
   for (int c : consumers) {
-    const std::vector<Flow> L = (c == root) ? root_src : kernel_sources(s, b, c);
+    const std::vector<Flow> L = (c == root) ? root_src : rp.store[c] ? rp.src[c] : kernel_sources(s, b, c);
     std::vector<Stream> srcs;
     for (const Flow& f : L) {
       if (f.kind == Flow::kIn && f.rank == c) {

@@ -221,7 +221,7 @@ bool parse_strategy(const char* text, Strategy* out, std::string* err) {
     if (!ok_kind) return fail(err, "directive " + r.head + " not valid for this collective");
     std::vector<std::string> required = {"weight", "chunk"};
     std::vector<std::string> optional;
-    if (r.head == "tree") { required.push_back("parent"); optional.push_back("noagg"); }
+    if (r.head == "tree") { required.push_back("parent"); optional.push_back("noagg"); optional.push_back("relay"); }
     if (r.head == "rtree") { required.push_back("parent"); required.push_back("dst"); optional.push_back("noagg"); }
     if (r.head == "ring") required.push_back("order");
     if (r.head == "bcast") { required.push_back("parent"); required.push_back("src"); }
@@ -288,6 +288,11 @@ bool parse_strategy(const char* text, Strategy* out, std::string* err) {
         if (!parse_int(r.kv.at("dst"), &dst) || dst < 0 || dst >= n) return fail(err, "bad rtree dst");
         if (s.root != dst) return fail(err, "rtree root must be its dst");
         s.src = (int)dst;
+      }
+      if (r.kv.count("relay")) {
+        const std::string& v = r.kv.at("relay");
+        if (v != "store" && v != "bypass") return fail(err, "relay must be store or bypass");
+        s.relay_store = v == "store";
       }
       if (r.kv.count("noagg")) {
         std::vector<int64_t> na;

@@ -40,6 +40,7 @@ struct SubColl {
   int64_t chunk = 0;           // C_m, bytes, multiple of 16
   std::vector<int> parent;     // tree / bcast; -1 at the root
   uint64_t noagg = 0;          // bit g: a_{m,g} = 0
+  bool relay_store = false;    // tree: pure relays store-and-forward through their arena (relay=store)
   int src = -1;                // bcast: source; rtree: destination block (== root)
   int root = -1;
   std::vector<std::vector<int>> children;  // ascending rank order (reading Q5)

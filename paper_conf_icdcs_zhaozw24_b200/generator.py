@@ -51,7 +51,8 @@ def binary_tree_parent(order):
 
 
 # ------------------------------------------------------------------- allreduce
-def allreduce_trees(parents, weights=None, chunk=DEFAULT_CHUNK, noaggs=None):
+def allreduce_trees(parents, weights=None, chunk=DEFAULT_CHUNK, noaggs=None, relay=None):
+    """relay: None (the default, bypass) or 'store' / 'bypass' on every tree line."""
     n = len(parents[0])
     weights = weights if weights is not None else [1] * len(parents)
     noaggs = noaggs or [()] * len(parents)
@@ -60,6 +61,8 @@ def allreduce_trees(parents, weights=None, chunk=DEFAULT_CHUNK, noaggs=None):
         out += f"tree weight={int(w)} chunk={int(chunk)} parent={_join(p)}"
         if na:
             out += f" noagg={_join(na)}"
+        if relay:
+            out += f" relay={relay}"
         out += "\n"
     return out
 

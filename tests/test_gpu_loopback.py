@@ -403,3 +403,23 @@ def test_wide_rank_counts(n, mode, engine):
         assert np.array_equal(bits(to_host(dy[g], "f32")), bits(full)), g
     assert comm.get_async_error() == 0
     comm.finalize()
+
+
+@pytest.mark.parametrize("relay", ["store", "bypass"])
+@pytest.mark.parametrize("mode", MODES)
+@pytest.mark.parametrize("engine", ENGINES)
+@pytest.mark.parametrize("dtype", ["f32", "bf16", "i32"])
+def test_relay_store_bit_exact(relay, mode, engine, dtype):
+    """relay=store: pure relays forward through their own arena,
+    chunk by chunk; the result is bit-identical to the oracle (and to the
+    bypass data path) for chains of relays, binary trees and stars."""
+    n, count = 7, 300_007
+    parents = [[-1, 0, 1, 2, 3, 4, 5], [-1, 0, 0, 1, 1, 2, 2], S.star(n, 3)]
+    text = G.allreduce_trees(parents, weights=[3, 2, 1], chunk=32768, relay=relay)
+    comm = _comm(n, mode, scratch=128 << 20, engine=engine)
+    comm.set_strategy("allreduce", text)
+    xs = rank_tensors(dtype, count, n)
+    for R in ({0, 6}, {0, 3, 4}, set(range(n)) - {1, 2, 5}, {6}):
+        got = _run_allreduce(comm, xs, dtype, R)
+        _assert_bits(got, oc.allreduce(xs, text, R, dtype), f"relay={relay}/{sorted(R)}")
+    comm.finalize()

@@ -150,6 +150,11 @@ BAD = [
     "adapcc-strategy 1\nnranks 2\ncollective alltoall\na2a weight=1\n",
     "adapcc-strategy 1\nnranks 2\nnranks 2\ncollective alltoall\na2a weight=1 chunk=16\n",
     "adapcc-strategy 1\nnranks 2\ncollective alltoall\na2a weight=1x chunk=16\n",
+    # relay=store|bypass on tree lines only
+    "adapcc-strategy 1\nnranks 2\ncollective allreduce\ntree weight=1 chunk=16 parent=-1,0 relay=copy\n",
+    "adapcc-strategy 1\nnranks 2\ncollective reduce\ntree weight=1 chunk=16 parent=-1,0 relay=stored\n",
+    "adapcc-strategy 1\nnranks 2\ncollective allgather\nbcast src=0 weight=1 chunk=16 parent=-1,0 relay=store\n"
+    "bcast src=1 weight=1 chunk=16 parent=1,-1\n",
     # nvls (NEXT-2 switch reduction): allreduce only, weight and chunk only
     "adapcc-strategy 1\nnranks 2\ncollective allgather\nnvls weight=1 chunk=16\n",
     "adapcc-strategy 1\nnranks 2\ncollective allreduce\nnvls weight=1 chunk=16 parent=-1,0\n",
