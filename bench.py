@@ -375,6 +375,10 @@ def run_single(args):
     sweep = None
     if not args.no_sweep:   # BASELINE metric is busbw vs size: every x4 size up to the bench size
         sweep = []
+        warm = comm.prepare_allreduce_lb([t[:256] for t in dx], [t[:256] for t in dy])
+        for _ in range(2000):      # host warm-up (clocks, caches) before the smallest point
+            warm()
+        torch.cuda.synchronize()
         for sb in [b for b in SWEEP_SIZES if b <= nbytes]:
             c = sb // es
             xs_, ys_ = [t[:c] for t in dx], [t[:c] for t in dy]

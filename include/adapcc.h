@@ -263,8 +263,13 @@ ADAPCC_API adapcc_result_t adapcc_collective_zc(adapcc_comm_t comm, adapcc_coll_
  * NVLink instead of the 2(n-1)/n S of P2P trees.  The switch defines the fp32
  * summation order (oracle: tolerance mode, int32 exact); nvls lines need the
  * whole ready mask and no late join (UNSUPPORTED otherwise) and run on the
- * LDG kernel.  Collective over every rank (multi-process only; loopback:
- * UNSUPPORTED).  Any failure on any rank (no multicast support, driver entry
+ * LDG kernel.  Collective over every rank.  Loopback (one device, no
+ * multicast team): the switch is EMULATED -- each virtual rank gets its own
+ * scratch and the kernel sums the n copies in ascending rank order and
+ * stores the sum to all of them, so the plan (copy in, per-slice flags,
+ * switch step, copy out, ragged tail) runs and is tested on one GPU; only
+ * multimem itself is not exercised there.  Multi-process: any failure on any
+ * rank (no multicast support, driver entry
  * points, pidfd_getfd of rank 0's exported handle, binding) makes every rank
  * return UNSUPPORTED and `why` (may be NULL) says why; an nvls line then
  * makes its calls return UNSUPPORTED.  Calling it again replaces the team.

@@ -212,6 +212,7 @@ struct adapcc_comm_s {
   uint64_t nvls_bytes = 0;
   unsigned long long nvls_mc_handle = 0, nvls_phys = 0;
   int nvls_fd = -1;
+  uint64_t nvls_stride = 0;  // loopback emulation: per-virtual-rank scratch stride (cudaMalloc'ed)
 };
 
 namespace {
@@ -631,6 +632,7 @@ adapcc_result_t run(adapcc_comm_s* c, Coll coll, const void* const* send, void* 
     P.err = c->d_err;
     P.nvls_uc = c->nvls_uc;
     P.nvls_mc = c->nvls_mc;
+    P.nvls_stride = c->nvls_stride;
     P.trace = c->trace;
     P.trace_n = c->trace_n;
     P.trace_cap = c->trace_cap;
@@ -1249,6 +1251,13 @@ const Drv& drv() {
 }
 
 void nvls_free(adapcc_comm_s* c) {
+  if (c->nvls_stride) {  // loopback emulation
+    cudaDeviceSynchronize();
+    cudaFree(c->nvls_uc);
+    c->nvls_uc = c->nvls_mc = nullptr;
+    c->nvls_bytes = c->nvls_stride = 0;
+    return;
+  }
   const Drv& d = drv();
   if (!d.ok) return;
   cudaDeviceSynchronize();
@@ -1273,7 +1282,7 @@ void nvls_free(adapcc_comm_s* c) {
 }
 
 void nvls_release(adapcc_comm_s* c) {
-  if (c->nvls_bytes || c->nvls_mc_handle || c->nvls_phys) nvls_free(c);
+  if (c->nvls_bytes || c->nvls_mc_handle || c->nvls_phys || c->nvls_stride) nvls_free(c);
 }
 
 // plans depend on whether NVLS scratch exists (nvls lines plan against it)
@@ -1293,7 +1302,19 @@ adapcc_result_t adapcc_nvls_setup(adapcc_comm_t c, size_t bytes, char* why, size
     }
   };
   if (!c || !bytes) return ADAPCC_ERR_INVALID_ARGUMENT;
-  if (c->loopback) { say("loopback: one device, no multicast team"); return ADAPCC_ERR_UNSUPPORTED; }
+  if (c->loopback) {  // one device: no multicast team -- emulate the switch (plan + engine test bed)
+    std::lock_guard<std::mutex> lock(c->mu);
+    CK(cudaSetDevice(c->device));
+    if (c->nvls_bytes) nvls_free(c);
+    const uint64_t size = (bytes + (uint64_t(2) << 20) - 1) / (uint64_t(2) << 20) * (uint64_t(2) << 20);
+    char* p = nullptr;
+    if (cudaMalloc(&p, size * c->nranks) != cudaSuccess) { cudaGetLastError(); return ADAPCC_ERR_OOM; }
+    c->nvls_uc = c->nvls_mc = p;
+    c->nvls_stride = c->nvls_bytes = size;
+    drop_plans_nvls(c);
+    say("loopback emulation: per-virtual-rank scratch, the kernel sums the copies in ascending rank order");
+    return ADAPCC_SUCCESS;
+  }
   const uint64_t all = c->nranks >= 64 ? ~uint64_t(0) : ((uint64_t(1) << c->nranks) - 1);
   if (c->members != all) { say("a rank was excluded: the multicast team is incomplete"); return ADAPCC_ERR_UNSUPPORTED; }
   std::lock_guard<std::mutex> lock(c->mu);

@@ -202,6 +202,23 @@ __device__ void nvls_vec(const SH& sh, uint32_t nvec) {
   for (uint32_t v = threadIdx.x; v < nvec; v += kThreads)
     mm_st(sh.dst[0] + (size_t)v * 16, mm_ld_reduce<DT>(sh.src[0] + (size_t)v * 16));
 }
+// Loopback emulation of the switch (adapcc_nvls_setup on one device): the
+// multicast address is virtual rank 0's copy; every rank's copy sits at the
+// same offset from its own unicast base (uc[q]); the sum runs over the n
+// copies in ascending rank order (fp32 adds, bf16 accumulated in fp32 and
+// rounded once, int32 wrapping) and is stored to every copy.
+template <int DT, class SH>
+__device__ void nvls_vec_emul(const SH& sh, uint32_t nvec, char* const* uc, const char* mc, int n) {
+  using O = Ops<DT>;
+  const size_t so = (size_t)(sh.src[0] - mc), dof = (size_t)(sh.dst[0] - mc);
+  for (uint32_t v = threadIdx.x; v < nvec; v += kThreads) {
+    const size_t o = (size_t)v * 16;
+    typename O::Acc a = O::widen(ld16(uc[0] + so + o));
+    for (int q = 1; q < n; ++q) O::add(a, ld16(uc[q] + so + o));
+    const uint4 r = O::narrow(a);
+    for (int q = 0; q < n; ++q) st16(uc[q] + dof + o, r);
+  }
+}
 __device__ __forceinline__ void fence_proxy_alias() { asm volatile("fence.proxy.alias;" ::: "memory"); }
 
 // element path (misaligned slots / ragged tail): e in [e_begin, e_end)
@@ -234,12 +251,14 @@ __device__ __forceinline__ void fold_scalar(const Shared& sh, int nsrc, int ndst
 }
 
 template <int DT>
-__device__ void fold_chunk(const Shared& sh, int nsrc, int ndst, uint64_t n, int op) {
+__device__ void fold_chunk(const Shared& sh, int nsrc, int ndst, uint64_t n, int op,
+                           char* const* nvls_uc = nullptr, const char* nvls_mc = nullptr, int nranks = 0) {
   using O = Ops<DT>;
   using E = typename O::E;
   if (op == kOpNone) return;  // (STAGED late join: nothing to move for this chunk)
   if (op == kOpNvls) {        // (planned on whole 16-byte vectors only)
-    nvls_vec<DT>(sh, (uint32_t)(n * O::kEsize / 16));
+    if (nvls_uc) nvls_vec_emul<DT>(sh, (uint32_t)(n * O::kEsize / 16), nvls_uc, nvls_mc, nranks);
+    else nvls_vec<DT>(sh, (uint32_t)(n * O::kEsize / 16));
     return;
   }
   if (op == kOpZero) {
@@ -280,7 +299,8 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
   // before the stream-order wait
   for (int i = threadIdx.x; i < kNumBufKinds * P.nranks; i += kThreads) {
     const int k = i / P.nranks, q = i - k * P.nranks;
-    sbase[k][q] = k == 0 ? P.send[q] : k == 1 ? P.recv[q] : k == 2 ? P.hdr[q] : k == 3 ? P.nvls_uc : P.nvls_mc;
+    sbase[k][q] = k == 0 ? P.send[q] : k == 1 ? P.recv[q] : k == 2 ? P.hdr[q]
+                : k == 3 ? P.nvls_uc + (uint64_t)q * P.nvls_stride : P.nvls_mc;
   }
   if (threadIdx.x == 0 && !use_blob && blockIdx.x < P.nitems) pre = P.items[blockIdx.x];
   constexpr int esize = Ops<DT>::kEsize;
@@ -574,7 +594,8 @@ __global__ void __launch_bounds__(kThreads, ADAPCC_MINB) engine_kernel(const __g
       // NVLS scratch is written through one address alias (unicast or
       // multicast) and read through the other: proxy fences on both sides
       if (alias) fence_proxy_alias();
-      fold_chunk<DT>(sh, nsrc, ndst, sh.cur.len, sh.cur.op);
+      fold_chunk<DT>(sh, nsrc, ndst, sh.cur.len, sh.cur.op, P.nvls_stride ? sbase[kBufNvlsUc] : nullptr,
+                     sbase[kBufNvlsMc][0], P.nranks);
       if (alias) fence_proxy_alias();
       if (stat) cp_async_wait_all();  // the next blob has landed before the barrier publishes it
       __syncthreads();

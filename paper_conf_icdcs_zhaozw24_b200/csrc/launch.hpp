@@ -99,6 +99,8 @@ struct LaunchCore {
   int* err;             // host-mapped error word
   char* nvls_uc;        // NVLS scratch of this rank: unicast / multicast address (nullptr: no NVLS)
   char* nvls_mc;
+  uint64_t nvls_stride; // 0: a real multicast team; > 0: loopback emulation -- virtual rank q's scratch is
+                        // nvls_uc + q * nvls_stride and the kernel sums / stores the n copies itself
 };
 
 template <int NR>

@@ -26,15 +26,61 @@ def _need_gpu():
         pytest.skip("no GPU")
 
 
-def test_loopback_refuses_nvls():
+def test_nvls_line_without_setup_is_refused():
     comm = pkg.Communicator.loopback(4)
-    ok, why = comm.nvls_setup(64 << 20)
-    assert not ok and "loopback" in why
     comm.set_strategy("allreduce", G.allreduce_nvls(4))
     xs = [torch.ones(4096, device="cuda") for _ in range(4)]
     with pytest.raises(pkg.AdapccError) as e:
         comm.allreduce_lb(xs, [torch.empty_like(x) for x in xs])
     assert e.value.code == pkg.adapcc.UNSUPPORTED
+    comm.finalize()
+
+
+@pytest.mark.parametrize("mode", ["direct", "staged"])
+@pytest.mark.parametrize("n", [2, 5, 8])
+def test_nvls_plan_on_emulated_switch(mode, n):
+    """Loopback emulates the switch (each virtual rank has its own scratch,
+    the kernel sums the copies): the whole NVLS plan -- copy in, per-slice
+    flags, the switch step, copy out, the ragged tail through a star -- runs
+    against the oracle's tolerance mode (int32 exact), with nvls lines mixed
+    with star trees, ACCUMULATE, and a partial mask refused."""
+    from oracle import bf16 as obf
+    from oracle import collectives as oc
+    from synth import rank_tensors
+    from tests.gpu_util import bits, empty_dev, to_dev, to_host
+    comm = pkg.Communicator.loopback(n, mode=mode, scratch_bytes=64 << 20)
+    ok, why = comm.nvls_setup(32 << 20)
+    assert ok, why
+    text = G.allreduce_nvls(n, chunk=1 << 16, nvls_weight=5, star_weight=1)
+    comm.set_strategy("allreduce", text)
+    for dtype in ("i32", "f32", "bf16"):
+        for count in (1 << 20, (1 << 20) + 3, 777):
+            xs = rank_tensors(dtype, count, n)
+            dy = [empty_dev(count, dtype) for _ in range(n)]
+            comm.allreduce_lb([to_dev(x, dtype) for x in xs], dy)
+            torch.cuda.synchronize()
+            exp = oc.allreduce(xs, text, set(range(n)), dtype)
+            got = [to_host(y, dtype) for y in dy]
+            for g in range(1, n):
+                assert np.array_equal(bits(got[g]), bits(got[0]))      # every rank the same bytes
+            if dtype == "i32":
+                assert np.array_equal(got[0], exp[0])
+            else:
+                f = (lambda a: obf.to_f32(a).astype(np.float64)) if dtype == "bf16" else (lambda a: a.astype(np.float64))
+                den = np.sum(np.abs(np.stack([f(x) for x in xs])), axis=0) + 1e-30
+                assert np.max(np.abs(f(got[0]) - f(exp[0])) / den) <= oc.nvls_tolerance(dtype, n) * 1.001
+    # ACCUMULATE (phase 2 on top of a previous result), int32 exact
+    xs = rank_tensors("i32", 100_003, n)
+    prev = rank_tensors("i32", 100_003, n, base=1700)
+    dy = [to_dev(p, "i32") for p in prev]
+    comm.allreduce_lb([to_dev(x, "i32") for x in xs], dy, accumulate=True)
+    torch.cuda.synchronize()
+    exp = oc.allreduce(xs, text, set(range(n)), "i32", accumulate=True, y_prev=prev)
+    assert all(np.array_equal(to_host(y, "i32"), e) for y, e in zip(dy, exp))
+    with pytest.raises(pkg.AdapccError) as e:          # the switch sums every copy: whole mask only
+        comm.allreduce_lb([to_dev(x, "i32") for x in xs], dy, ready=set(range(1, n)))
+    assert e.value.code == pkg.adapcc.UNSUPPORTED
+    assert comm.get_async_error() == 0
     comm.finalize()
 
 
@@ -124,3 +170,4 @@ def test_nvls_multiprocess():
     assert len(oks) == 1, out                      # every rank agrees
     if not out[0]["ok"]:
         pytest.skip("no multicast team on this box: " + out[0]["why"])
+    assert out[0]["checks"] and all(ok for _, ok in out[0]["checks"])
