@@ -475,9 +475,7 @@ adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, const Strategy* strat, uin
     // (profiles/acc_r02.json); the shared-memory read-modify-write (acc_red
     // off) stages nsrc + nacc tiles per slot and is latency-bound, where the
     // 2 CTAs/SM x 3 x 32 KiB shape wins (profiles/acc_variants_r01.json).
-    // STAGED late join (decision words, conditional pushes) and NVLS
-    // (multimem) tasks run on the LDG kernel
-    if (rq.late_join && mode == kStaged) plan->engine = 0;
+    // NVLS (multimem) tasks run on the LDG kernel
     for (auto& sp : segs)
       if (sp.nvls) plan->engine = 0;
     plan->kernel = plan->engine == 0 ? 0 : (mode == kDirect && (!rq.accumulate || c->acc_red) ? 1 : 2);

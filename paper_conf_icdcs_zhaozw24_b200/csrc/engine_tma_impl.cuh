@@ -75,6 +75,10 @@ struct ItemDesc {
   uint8_t stop, dropped, scalar_only, any_acc;
   uint8_t acc_tma;            // accumulating destinations are loaded by TMA and stored from the stage
   uint8_t acc_red;            // accumulating destinations take bulk reduce-adds of the folded tile
+  uint8_t need_decide;        // STAGED late join: sources / op are fixed after the waits (decision words)
+  uint8_t ndec, dec_val;      // STAGED late join: decision words to write before the posts, and their value
+  uint16_t wait0;             // first of the task's waits this item waits for
+  uint64_t* dec[2];
   uint8_t acc_slot[kMaxDst];  // acc_tma: stage tile of destination k's recv (0 = plain destination)
   uint32_t item;        // trace: item index, claim and inputs-ready times
   uint64_t tr0, tr1;
@@ -496,21 +500,80 @@ __device__ __forceinline__ void consume_copy_held(Smem& sm, char* stages, const 
 }
 
 // ------------------------------------------------------------- producer
+// STAGED late join: decision word of chunk `chunk` of the slot `r` of task t
+template <int DT, class LP>
+__device__ __forceinline__ uint64_t* dec_word(char* const (*base)[LP::kRanks], const BufRef& r, const Task& t,
+                                              uint64_t half_off, uint32_t chunk) {
+  return reinterpret_cast<uint64_t*>(base[kBufArena][r.rank] + half_off + r.bias +
+                                     (int64_t)(t.lo * Ops<DT>::kEsize) - (int64_t)late_dec_bytes(t.nchunks)) + chunk;
+}
+
 // R: the task's refs (R[0] = refs[t.ref0]), in global memory or in the
-// CTA's first-item blob
+// CTA's first-item blob.  decided: STAGED late join, second pass after the
+// item's waits with `decision` = the late mask (kLateRoot) or "the parent
+// broadcast anything" (kLatePull).
 template <int DT, class LP>
 __device__ __forceinline__ void fill_desc(const LP& P, char* const (*base)[LP::kRanks],
                                           ItemDesc& d, const Item& item, const Task& t, const BufRef* R,
                                           uint64_t half_off, int lane, uint32_t it, int* nwait_eff,
-                                          uint64_t epoch) {
+                                          uint64_t epoch, bool decided = false, uint64_t decision = 0) {
   constexpr int esize = Ops<DT>::kEsize;
   const uint64_t e0 = t.lo + (uint64_t)item.chunk * t.chunk_elems + item.off;
   // late join (phase 1) / complement (phase 2): which candidate ranks are folded
   uint64_t late = 0;
   bool dropped = (int)t.owner == P.drop_rank, force_acc = false;
   int nreg = t.nsrc, op = t.op;
+  int need_decide = 0, has_dec = 0, dec_val = 1, wait0 = 0;
   *nwait_eff = t.nwait;
-  if (P.late_mode && !dropped) {
+  if (P.late_mode && !dropped && t.lkind == kLatePush) {
+    // the late rank's own chunk goes to the root iff it is ready now (phase 1)
+    // / iff it did not go in phase 1 (phase 2)
+    int pushed = 0;
+    if (lane == 0) {
+      if (P.late_mode == 1) {
+        pushed = ld_acquire(reinterpret_cast<const uint64_t*>(base[kBufArena][t.owner] + ArenaHeader::kReady),
+                            P.ipc) >= P.late_ticket;
+        P.late_bits[it] = pushed ? 1 : 0;
+      } else {
+        pushed = P.late_bits[it] == 0;
+      }
+    }
+    pushed = __shfl_sync(0xffffffffu, pushed, 0);
+    if (!pushed) op = kOpNone;
+    has_dec = 1;
+    dec_val = pushed;
+  } else if (P.late_mode && !dropped && t.lkind == kLateRoot) {
+    if (P.late_mode == 2) {  // only the late slots' flags; recv += fold of what is left
+      nreg = 0;
+      wait0 = t.nwait - t.nlwait;
+      *nwait_eff = t.nlwait;
+      op = kOpFold;
+      force_acc = true;
+    }
+    if (!decided) {
+      need_decide = 1;
+    } else {
+      late = decision;
+      if (P.late_mode == 2) {
+        if (!late) op = kOpNone;
+        has_dec = 1;
+        dec_val = late != 0;
+      } else if (late && t.op == kOpZero) {
+        op = kOpFold;
+      }
+    }
+  } else if (P.late_mode && !dropped && t.lkind == kLatePull) {
+    if (P.late_mode == 2) {
+      if (!decided) {
+        need_decide = 1;
+      } else {  // add the parent's slot iff it broadcast anything, and forward the decision
+        if (decision) force_acc = true;
+        else op = kOpNone;
+        has_dec = 1;
+        dec_val = decision != 0;
+      }
+    }
+  } else if (P.late_mode && !dropped) {
     if (t.nlate == 0) {
       dropped = P.late_mode == 2;  // phase 2 only runs the roots' folds
     } else {
@@ -538,7 +601,8 @@ __device__ __forceinline__ void fill_desc(const LP& P, char* const (*base)[LP::k
       d.src[i] = p;
     } else {
       d.dst[i - nsrc] = p;
-      d.acc[i - nsrc] = r.accum || force_acc;
+      // (force_acc: recv += result; a STAGED broadcast slot still takes the plain result)
+      d.acc[i - nsrc] = r.accum || (force_acc && r.kind == kBufRecv);
     }
   }
   for (int i = lane; i < t.npost; i += 32) {
@@ -548,6 +612,15 @@ __device__ __forceinline__ void fill_desc(const LP& P, char* const (*base)[LP::k
   misaligned = __any_sync(0xffffffffu, misaligned);
   __syncwarp();
   if (lane == 0) {
+    d.need_decide = (uint8_t)need_decide;
+    d.wait0 = (uint16_t)wait0;
+    d.dec_val = (uint8_t)dec_val;
+    d.ndec = 0;
+    if (has_dec)  // decision words of the arena destinations (the slots this chunk lands in)
+      for (int k = 0; k < t.ndst && d.ndec < 2; ++k) {
+        const BufRef r = R[t.nsrc + k];
+        if (r.kind == kBufArena) d.dec[d.ndec++] = dec_word<DT, LP>(base, r, t, half_off, item.chunk);
+      }
     d.nsrc = (uint16_t)nsrc;
     d.ndst = t.ndst;
     d.op = (uint16_t)op;
@@ -718,13 +791,44 @@ engine_tma_kernel(const __grid_constant__ LaunchParamsT<NR> P) {
         if (!d.dropped) {
           int ok = 1;
           for (int i = lane; i < nwait; i += 32) {
-            const FlagRef f = P.flags[t.flag0 + i];
+            const FlagRef f = P.flags[t.flag0 + d.wait0 + i];
             const uint64_t* fl = reinterpret_cast<const uint64_t*>(sbase[kBufArena][f.rank] + half_off + f.off) + item.chunk;
             ok &= wait_flag(fl, epoch, P);
           }
           if (!__all_sync(0xffffffffu, ok)) {
             stop = true;
             if (lane == 0) sm.abort = 1;
+          }
+          if (!stop && d.need_decide) {
+            // STAGED late join: the decision words are readable now (their flags acquired)
+            const BufRef* R = fb ? reinterpret_cast<const BufRef*>(&sm.blob[kBlobRef0]) : P.refs + t.ref0;
+            uint64_t decision = 0;
+            if (lane == 0) {
+              if (t.lkind == kLateRoot) {
+                const uint64_t prev = P.late_mode == 2 ? P.late_bits[it] : 0;
+                for (uint32_t j = 0; j < t.nlate; ++j) {
+                  const BufRef r = R[t.nsrc + t.ndst + j];
+                  bool in;
+                  if (r.kind == kBufArena)
+                    in = *reinterpret_cast<volatile uint64_t*>(dec_word<DT, LaunchParamsT<NR>>(sbase, r, t, half_off,
+                                                                                            item.chunk)) != 0;
+                  else if (P.late_mode == 1)
+                    in = ld_acquire(reinterpret_cast<const uint64_t*>(sbase[kBufArena][r.rank] + ArenaHeader::kReady),
+                                    P.ipc) >= P.late_ticket;
+                  else
+                    in = ((prev >> j) & 1) == 0;
+                  if (in) decision |= 1ull << j;
+                }
+                if (P.late_mode == 1) P.late_bits[it] = decision;
+              } else {  // kLatePull, phase 2: did the parent broadcast anything?
+                decision = *reinterpret_cast<volatile uint64_t*>(
+                               dec_word<DT, LaunchParamsT<NR>>(sbase, R[0], t, half_off, item.chunk)) != 0;
+              }
+            }
+            decision = __shfl_sync(0xffffffffu, decision, 0);
+            int nw2 = 0;
+            fill_desc<DT>(P, sbase, d, item, t, R, half_off, lane, it, &nw2, epoch, true, decision);
+            __syncwarp();
           }
         }
       }
@@ -790,7 +894,7 @@ engine_tma_kernel(const __grid_constant__ LaunchParamsT<NR> P) {
           using E = typename Ops<DT>::E;
           for (int k = 0; k < d.ndst; ++k)
             for (uint64_t e = tid; e < d.len; e += kConsumers) reinterpret_cast<E*>(d.dst[k])[e] = E(0);
-        } else {
+        } else if (d.op != kOpNone) {
           if (!d.scalar_only) {
             const uint32_t vpt = d.tile / (16u * kConsumers);  // tile / one round of 1 vector per thread
             if (d.acc_tma) consume_acc_tma<DT>(sm, stages, d, tid, stage, sphase);
@@ -826,6 +930,8 @@ engine_tma_kernel(const __grid_constant__ LaunchParamsT<NR> P) {
         if (tid == 0 && d.npost) {
           tma_store_wait_all();  // bulk (async-proxy) stores performed ...
           fence_proxy_async();   // ... and ordered before generic-proxy accesses
+          for (int k = 0; k < d.ndec; ++k)  // STAGED late join: the decision travels with the flag
+            *reinterpret_cast<volatile uint64_t*>(d.dec[k]) = d.dec_val;
           fence(sys);      // the chunk's bytes (incl. remote NVLink stores) before its flag
           for (int i = 0; i < d.npost; ++i) st_release(d.post[i], epoch, sys);
         }

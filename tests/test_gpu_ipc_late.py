@@ -46,7 +46,8 @@ def _worker(rank, n, port, q):
         late = n - 1
         R = set(range(n)) - {late}
         msgs = []
-        for dtype in ("f32", "bf16", "i32"):
+        for engine, dtype in ((0, "f32"), (1, "f32"), (0, "bf16"), (1, "i32")):
+            comm.config("engine", engine)
             count = 300_007
             xs = rank_tensors(dtype, count, n)
             for text in (G.allreduce_stars(n, chunk=65536), G.allreduce_ring(n, chunk=32768)):
@@ -68,11 +69,11 @@ def _worker(rank, n, port, q):
                     ok2 = np.array_equal(bits(to_host(y, dtype)), bits(e2[rank]))
                     if dtype == "i32":
                         ok2 = ok2 and np.array_equal(to_host(y, "i32"), oc.allreduce_exact(xs, set(range(n)), "i32"))
-                    msgs.append((dtype, case, ok1, ok2))
+                    msgs.append((engine, dtype, case, ok1, ok2))
         err = comm.get_async_error()
         comm.finalize()
         dist.destroy_process_group()
-        q.put((rank, err == 0 and all(m[2] and m[3] for m in msgs), f"{msgs} err={err}"))
+        q.put((rank, err == 0 and all(m[3] and m[4] for m in msgs), f"{msgs} err={err}"))
     except Exception as e:  # noqa: BLE001
         import traceback
         q.put((rank, False, traceback.format_exc() + repr(e)))

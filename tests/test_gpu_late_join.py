@@ -44,8 +44,8 @@ def _comm(n, engine, mode="direct"):
 @pytest.mark.parametrize("dtype", ["f32", "bf16", "i32"])
 @pytest.mark.parametrize("case", ["all", "none", "one"])
 def test_late_join_deterministic(engine, dtype, case, mode):
-    """STAGED: late ranks push their chunks to the roots themselves (LDG
-    kernel whatever the engine setting); DIRECT: roots read them."""
+    """STAGED: late ranks push their chunks to the roots themselves;
+    DIRECT: roots read them.  Both kernels."""
     n, count = 8, 200_003
     R, late = {0, 1, 2, 4, 5, 7}, [3, 6]
     text = S.allreduce_trees([S.star(n, m) for m in range(n)] + [S.chain([0, 1, 2, 3, 4, 5, 6, 7])],
@@ -79,7 +79,7 @@ def _piece_ranges(text, count, dtype, R, grid, engine, mode="direct"):
     STAGED: the root tasks' chunks (a star root writes its recv and its
     broadcast slot)."""
     mask = sum(1 << r for r in R)
-    items, tasks = pkg.adapcc.plan_items(text, count, dtype, mask, grid, tma=engine == 1 and mode == "direct",
+    items, tasks = pkg.adapcc.plan_items(text, count, dtype, mask, grid, tma=engine == 1,
                                          late="join", mode=mode)
     if mode == "staged":
         items = items[(tasks[items["task"]]["ndst"] == 2) & (tasks[items["task"]]["nwait"] >= 1)]
@@ -88,7 +88,7 @@ def _piece_ranges(text, count, dtype, R, grid, engine, mode="direct"):
     return np.stack([a, a + items["len"]], axis=1).astype(np.int64)
 
 
-@pytest.mark.parametrize("engine,mode", [(0, "direct"), (1, "direct"), (0, "staged")])
+@pytest.mark.parametrize("engine,mode", [(0, "direct"), (1, "direct"), (0, "staged"), (1, "staged")])
 @pytest.mark.parametrize("dtype", ["f32", "i32"])
 def test_late_join_racing_signal(engine, dtype, mode):
     """Rank 3 signals from a side stream while phase 1 runs.  Per work piece
