@@ -136,7 +136,7 @@ class ClockSampler:
                                 self.reasons.add(nm)
                     except Exception:  # noqa: BLE001
                         pass
-                    time.sleep(0.01)
+                    time.sleep(0.001)
 
             self._t = threading.Thread(target=loop, daemon=True)
             self._t.start()

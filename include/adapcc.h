@@ -83,7 +83,9 @@ typedef enum { ADAPCC_MODE_DIRECT = 0, ADAPCC_MODE_STAGED = 1 } adapcc_mode_t;
  * plan kind (loopback DIRECT / STAGED, multi-process STAGED via
  * adapcc_allreduce, zero-copy via adapcc_collective_zc); not combinable with
  * ACCUMULATE.  A non-ready rank passes its (future) sendbuf: it is read only
- * after the rank signalled ready (adapcc_signal_ready).
+ * after the rank signalled ready (adapcc_signal_ready); it may not overlap
+ * that rank's recvbuf (phase 1 writes the recvbuf before phase 2 reads the
+ * chunks it missed) -- INVALID_ARGUMENT.
  *   LATE_JOIN (phase 1, mask R): every tree root also folds, per work piece
  *     (DIRECT) or per chunk (STAGED), the inputs of the non-ready ranks whose
  *     ready word already holds this call's ticket (appended after the

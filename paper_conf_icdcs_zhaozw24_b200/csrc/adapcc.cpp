@@ -803,6 +803,9 @@ adapcc_result_t adapcc_allreduce(adapcc_comm_t c, const void* sendbuf, void* rec
   const bool late = flags & (ADAPCC_FLAG_LATE_JOIN | ADAPCC_FLAG_LATE_COMPLEMENT);
   const bool ready = ((mask >> c->rank) & 1) || late;
   if (count && ready && !sendbuf) return ADAPCC_ERR_INVALID_ARGUMENT;
+  // a late rank's input is read after phase 1 wrote its recvbuf: no aliasing
+  if (late && !((mask >> c->rank) & 1) && count && overlap(sendbuf, bytes, recvbuf, bytes))
+    return ADAPCC_ERR_INVALID_ARGUMENT;
   if (misaligned(recvbuf) || (ready && misaligned(sendbuf))) return ADAPCC_ERR_INVALID_ARGUMENT;
   if (ready && sendbuf != recvbuf && overlap(sendbuf, bytes, recvbuf, bytes)) return ADAPCC_ERR_INVALID_ARGUMENT;
   const void* s[1] = {ready ? sendbuf : recvbuf};
@@ -877,6 +880,12 @@ adapcc_result_t adapcc_allreduce_lb(adapcc_comm_t c, const void* const* sendbufs
   const bool late = flags & (ADAPCC_FLAG_LATE_JOIN | ADAPCC_FLAG_LATE_COMPLEMENT);
   r = check_lb(c, sendbufs, recvbufs, bytes, bytes, late ? all : mask, 0);
   if (r != ADAPCC_SUCCESS) return r;
+  // a late rank's input is read after phase 1 wrote its recvbuf (phase 2):
+  // it may not alias it
+  if (late)
+    for (int q = 0; q < c->nranks; ++q)
+      if (((c->members >> q) & 1) && !((mask >> q) & 1) && bytes && overlap(sendbufs[q], bytes, recvbufs[q], bytes))
+        return ADAPCC_ERR_INVALID_ARGUMENT;
   return run(c, kAllReduce, sendbufs, recvbufs, count, dtype, mask, flags, stream);
 }
 
@@ -1131,6 +1140,10 @@ adapcc_result_t adapcc_collective_zc(adapcc_comm_t c, adapcc_coll_t coll, int se
       D.push_back(di->second.base[q] + recv_offset);
     }
     if (coll == ADAPCC_ALLTOALL && overlap(S[c->rank], sb, D[c->rank], rb)) return ADAPCC_ERR_INVALID_ARGUMENT;
+    // late join: a late rank's input is read after phase 1 wrote its recvbuf (same offsets on every rank)
+    if ((flags & (ADAPCC_FLAG_LATE_JOIN | ADAPCC_FLAG_LATE_COMPLEMENT)) && (mask != c->members) &&
+        overlap(S[c->rank], sb, D[c->rank], rb))
+      return ADAPCC_ERR_INVALID_ARGUMENT;
   }
   uint64_t extra = 1469598103934665603ull;
   for (uint64_t v : {(uint64_t)send_reg, (uint64_t)send_offset, (uint64_t)recv_reg, (uint64_t)recv_offset})

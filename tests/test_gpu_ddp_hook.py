@@ -5,6 +5,7 @@ equal the average of both ranks' local gradients (-m gpu)."""
 import os
 import socket
 import sys
+import time
 
 import pytest
 
@@ -22,7 +23,7 @@ def _port():
     return p
 
 
-def _worker(rank, n, port, q, auto_register=False, steps=1):
+def _worker(rank, n, port, q, auto_register=False, steps=1, coordinated=False):
     try:
         sys.path.insert(0, ROOT)
         import torch.distributed as dist
@@ -40,13 +41,24 @@ def _worker(rank, n, port, q, auto_register=False, steps=1):
         ref = [p.detach().clone() for p in model.parameters()]
         comm = pkg.Communicator.init(scratch_bytes=64 << 20, device=dev)
         ddp = DDP(model, device_ids=[dev], bucket_cap_mb=1)
-        state = AdapccHookState(comm, auto_register=auto_register)
+        coord = None
+        if coordinated:   # rank n-1 straggles: its backward starts late
+            from paper_conf_icdcs_zhaozw24_b200 import coordinator as C
+
+            def policy():
+                p = C.Coordinator(n, "allreduce", 1 << 20, 100e9, 5e-6)
+                p.buy_cost = lambda k: 200e-6
+                return p
+            coord = C.OnlineCoordinator(comm, policy, cycle=5e-6)
+        state = AdapccHookState(comm, auto_register=auto_register, coordinator=coord)
         ddp.register_comm_hook(state, adapcc_allreduce_hook)
         g = torch.Generator(device="cpu").manual_seed(100 + rank)
         ok = True
         for step in range(steps):   # parameters stay fixed: every step checks the same reduction
             ddp.zero_grad(set_to_none=False)
             x = torch.randn(32, 64, generator=g).cuda()
+            if coordinated and rank == n - 1:
+                time.sleep(0.05)
             ddp(x).square().sum().backward()
             torch.cuda.synchronize()
             # expected: average of every rank's local gradient of the same loss
@@ -63,6 +75,8 @@ def _worker(rank, n, port, q, auto_register=False, steps=1):
                 ok &= torch.allclose(p.grad.cpu(), exp, rtol=1e-5, atol=1e-6)
         if auto_register:  # every bucket went zero-copy, none through the arenas
             ok &= state.registered > 0 and state.staged_calls == 0 and state.zero_copy_calls > 0
+        if coordinated:    # the coordinator proceeded without the straggler at least once
+            ok &= any(d["action"] == "phase1" for d in state.decisions)
         err = comm.get_async_error()
         comm.finalize()
         dist.destroy_process_group()
@@ -72,19 +86,19 @@ def _worker(rank, n, port, q, auto_register=False, steps=1):
         q.put((rank, False, traceback.format_exc() + repr(e)))
 
 
-def _run(auto_register, steps):
+def _run(auto_register, steps, n=2, coordinated=False):
     if not torch.cuda.is_available():
         pytest.skip("no GPU")
     import torch.multiprocessing as mp
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _port()
-    procs = [ctx.Process(target=_worker, args=(r, 2, port, q, auto_register, steps)) for r in range(2)]
+    procs = [ctx.Process(target=_worker, args=(r, n, port, q, auto_register, steps, coordinated)) for r in range(n)]
     for p in procs:
         p.start()
     out = {}
     try:
-        for _ in range(2):
+        for _ in range(n):
             r, ok, msg = q.get(timeout=600)
             out[r] = (ok, msg)
     finally:
@@ -92,7 +106,7 @@ def _run(auto_register, steps):
             p.join(timeout=30)
             if p.is_alive():
                 p.kill()
-    for r in range(2):
+    for r in range(n):
         assert r in out and out[r][0], out.get(r)
 
 
@@ -104,3 +118,11 @@ def test_ddp_hook_auto_register_zero_copy():
     """auto_register: buckets are registered on first sight (and again after DDP's bucket rebuild)
     and every step runs the zero-copy DIRECT plan; gradients stay the cross-rank average."""
     _run(auto_register=True, steps=3)
+
+
+def test_ddp_hook_online_coordinator_with_straggler():
+    """3 processes, rank 2 starts its backward 50 ms late: the online
+    coordinator (rank 0 decides from the shared readiness board) runs phase 1
+    among the ready ranks with late join and phase 2 once rank 2 signals;
+    every gradient is still the 3-rank average."""
+    _run(auto_register=False, steps=2, n=3, coordinated=True)

@@ -224,3 +224,21 @@ def test_late_join_graph_replay(engine):
         for y, e in zip(dy, full):
             assert np.array_equal(bits(to_host(y, "i32")), bits(e))
     comm.finalize()
+
+
+def test_late_join_rejects_aliased_late_input():
+    """A late rank's input is read after phase 1 wrote its recvbuf: in-place
+    late join would fold the phase-1 result instead of the gradient."""
+    n = 4
+    comm = _comm(n, 0)
+    xs = [torch.ones(4096, device="cuda") for _ in range(n)]
+    ys = [torch.empty_like(x) for x in xs]
+    ys[3] = xs[3]                                   # rank 3 (late) in place
+    with pytest.raises(pkg.AdapccError) as e:
+        comm.allreduce_lb(xs, ys, ready={0, 1, 2}, late="join")
+    assert e.value.code == pkg.adapcc.INVALID_ARGUMENT
+    ys[3] = torch.empty_like(xs[3])
+    ys[0] = xs[0]                                   # a ready rank in place is fine
+    comm.allreduce_lb(xs, ys, ready={0, 1, 2}, late="join")
+    torch.cuda.synchronize()
+    comm.finalize()
