@@ -22,8 +22,14 @@ on the current stream) and lets the coordinator decide: everyone ready -> one
 plain AllReduce; otherwise phase 1 among the ready ranks with late join, then
 phase 2 once the late ranks signalled.  Every bucket ends with the full sum
 (the paper's model-update consistency), divided by every rank.  The
-bucket's input is staged in a per-bucket buffer, since a late rank's input is
-read after phase 1 wrote the result.
+collective runs on its own stream, NOT ordered after this rank's computation:
+a late rank still launches phase 1 right away and its chunks join as its
+ready signal lands ("asynchronously participate ... as relays"); the
+bucket is staged into a per-bucket input buffer (after the gradients, on the
+compute stream, before the signal) and the result lands in a per-bucket
+output buffer that the compute stream copies back after phase 2.  A rank is
+only in a decision's ready mask once its signal reached the board, i.e. after
+its staged input is complete.
 """
 
 import torch
@@ -39,7 +45,8 @@ class AdapccHookState:
         self.zero_copy_calls = 0
         self.staged_calls = 0
         self.decisions = []           # coordinator: one result dict per bucket
-        self._inputs = {}             # coordinator: staged input per bucket buffer
+        self._inputs = {}             # coordinator: staged input / output per bucket buffer
+        self._stream = None           # coordinator: the collective's own stream
 
     def contributors(self):
         if self.ready is None:              # every live rank (all, unless some were excluded)
@@ -52,15 +59,22 @@ class AdapccHookState:
 def _coordinated(state, buf):
     comm, coord = state.comm, state.coordinator
     key = (buf.data_ptr(), buf.numel(), buf.dtype)
-    x = state._inputs.get(key)
-    if x is None:
-        x = state._inputs[key] = torch.empty_like(buf)
-    x.copy_(buf)
-    comm.signal_ready(ticket=coord.ticket())   # after this rank's gradients on the current stream
-    res = coord.allreduce(lambda mask, late: comm.allreduce(x, buf, ready=mask, late=late))
+    xy = state._inputs.get(key)
+    if xy is None:
+        xy = state._inputs[key] = (torch.empty_like(buf), torch.empty_like(buf))
+    x, y = xy
+    if state._stream is None:
+        state._stream = torch.cuda.Stream(priority=-1)
+    cur, cs = torch.cuda.current_stream(), state._stream
+    x.copy_(buf)                                  # after this rank's gradients (compute stream)
+    comm.signal_ready(ticket=coord.ticket())      # ... then the ready signal
+    res = coord.allreduce(lambda mask, late: comm.allreduce(x, y, ready=mask, late=late, stream=cs))
+    done = torch.cuda.Event()
+    done.record(cs)
+    cur.wait_event(done)                          # the compute stream resumes after phase 2
+    buf.copy_(y).div_(len(comm.members))
     state.decisions.append(res)
     state.staged_calls += 1 + (res["phase2_after_s"] is not None)
-    buf.div_(comm.nranks if not comm.loopback else len(comm.members))
     fut = torch.futures.Future()
     fut.set_result(buf)
     return fut

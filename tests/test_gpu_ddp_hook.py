@@ -58,7 +58,7 @@ def _worker(rank, n, port, q, auto_register=False, steps=1, coordinated=False):
             ddp.zero_grad(set_to_none=False)
             x = torch.randn(32, 64, generator=g).cuda()
             if coordinated and rank == n - 1:
-                time.sleep(0.05)
+                torch.cuda._sleep(40_000_000)   # ~20 ms of "computation" on the GPU before its backward
             ddp(x).square().sum().backward()
             torch.cuda.synchronize()
             # expected: average of every rank's local gradient of the same loss
@@ -121,7 +121,7 @@ def test_ddp_hook_auto_register_zero_copy():
 
 
 def test_ddp_hook_online_coordinator_with_straggler():
-    """3 processes, rank 2 starts its backward 50 ms late: the online
+    """3 processes, rank 2's GPU starts its backward ~20 ms late: the online
     coordinator (rank 0 decides from the shared readiness board) runs phase 1
     among the ready ranks with late join and phase 2 once rank 2 signals;
     every gradient is still the 3-rank average."""
