@@ -389,6 +389,11 @@ bool overlap(const void* a, size_t an, const void* b, size_t bn) {
 // LDG fold's lower fixed cost wins (profiles/pieces_r01.json: 8 virtual ranks
 // x 4 MiB = 64 MiB of traffic, LDG 10.4 us vs TMA 13.4 us)
 constexpr uint64_t kTmaMinTraffic = uint64_t(128) << 20;
+// ACCUMULATE with bulk reduce-adds: the TMA kernel wins from ~32 MiB of traffic
+// (8 virtual ranks, 2 late: 2 MiB per rank 7.8 vs 9.0 us, 8 MiB 18.3 vs 36.2 us;
+// 1 MiB 7.1 vs 6.6 us, scripts/debug/acc_small.py): the LDG kernel pays one
+// memory latency per accumulating destination
+constexpr uint64_t kTmaMinTrafficAcc = uint64_t(32) << 20;
 
 int grid_size(const adapcc_comm_s* c, adapcc_dtype_t dtype, int kernel) {
   int grid = c->num_sms * c->occ[kernel][(int)dtype];
@@ -469,7 +474,8 @@ adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, const Strategy* strat, uin
     PlanStats st;
     for (auto& sp : segs) accumulate_stats(sp, c->loopback ? -1 : c->rank, rq.esize, &st);
     const uint64_t traffic = st.bytes_read + st.bytes_written;
-    plan->engine = c->engine != 2 ? c->engine : (traffic / std::max<size_t>(1, segs.size()) >= kTmaMinTraffic ? 1 : 0);
+    const uint64_t min_tma = rq.accumulate && c->acc_red ? kTmaMinTrafficAcc : kTmaMinTraffic;
+    plan->engine = c->engine != 2 ? c->engine : (traffic / std::max<size_t>(1, segs.size()) >= min_tma ? 1 : 0);
     // ACCUMULATE (phase 2): with bulk reduce-adds (acc_red, default) a stage
     // holds only the sources and DIRECT plans keep the 1 x 3 x 64 KiB ring
     // (profiles/acc_r02.json); the shared-memory read-modify-write (acc_red
