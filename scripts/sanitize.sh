@@ -20,11 +20,14 @@ run() {
 }
 LB=tests/test_gpu_loopback.py
 MORE="tests/test_gpu_primitives.py tests/test_gpu_late_join.py tests/test_gpu_a2a_routes.py tests/test_gpu_trace.py"
+# r02 paths: STAGED late join (both kernels), bulk reduce-add ACCUMULATE, NVLS on the emulated switch,
+# link probes, the online coordinator (loopback)
+R02="tests/test_gpu_nvls.py tests/test_gpu_link_probe.py tests/test_gpu_coordinator.py"
 # leak-check off: the only leaks reported are PyTorch caching-allocator segments alive at exit
-run memcheck "$LB $MORE" "not watchdog"
+run memcheck "$LB $MORE $R02" "not watchdog and not multiprocess and not racing and not loopback_profile and not messages_scale"
 run racecheck "$LB" "(allreduce_parity and f32 and (stars8 or dbinary)) or (alltoall and bf16) or c1_config or (tma_large_items and f32)"
-run synccheck "$LB" "(allreduce_parity and (stars8 or ring)) or allgather or c1_config"
-run initcheck "$LB" "(allreduce_parity and f32 and stars8) or c1_config or (alltoall and i32)"
+run synccheck "$LB tests/test_gpu_late_join.py tests/test_gpu_nvls.py" "(allreduce_parity and (stars8 or ring)) or allgather or c1_config or (deterministic and staged) or emulated or subnormal"
+run initcheck "$LB tests/test_gpu_late_join.py" "(allreduce_parity and f32 and stars8) or c1_config or (alltoall and i32) or (deterministic and staged and f32)"
 # racecheck's model of mbarrier handoffs (the TMA kernel's item queue): a
 # textbook correct producer/consumer handoff via mbarriers (A) vs named barriers (B)
 nvcc -gencode arch=compute_100a,code=sm_100a -o gpurun_out/rc_probe scripts/debug/racecheck_mbarrier_probe.cu \
