@@ -84,6 +84,8 @@ def main():
     ap.add_argument("--mode", default="direct")
     ap.add_argument("--engine", type=int, default=2)
     ap.add_argument("--calls", type=int, default=20)
+    ap.add_argument("--accumulate-ready", default=None,
+                    help="allreduce as phase 2: comma-separated ready ranks, recv += sum (ACCUMULATE)")
     ap.add_argument("--out", default=os.path.join(ROOT, "gpurun_out", "trace"))
     a = ap.parse_args()
     import torch
@@ -105,6 +107,10 @@ def main():
         xs = [torch.randn(count, device="cuda") for _ in range(n)]
         ys = [torch.empty_like(x) for x in xs]
     fn = getattr(comm, a.coll + "_lb")
+    if a.accumulate_ready:
+        R = {int(r) for r in a.accumulate_ready.split(",")}
+        xs = [x if r in R else None for r, x in enumerate(xs)]
+        fn = lambda x_, y_: comm.allreduce_lb(x_, y_, ready=R, accumulate=True)  # noqa: E731
     for _ in range(3):
         fn(xs, ys)
     torch.cuda.synchronize()
