@@ -56,10 +56,14 @@ def _case(seed, large=False, n=None):
     if rng.random() < 0.2:
         ready = set(range(n))
     m = int(rng.integers(1, 4))
+    # r02 knobs from their own stream: relay=store on allreduce trees, bulk reduce-add ACCUMULATE on/off
+    r3 = np.random.default_rng(seed + (8_100_000 if large else 8_000_000))
+    relay = "store" if r3.random() < 0.3 else None
+    acc_red = int(r3.integers(0, 2))
     if coll == "allreduce":
         parents = [_random_tree(rng, n) for _ in range(m)]
         noaggs = [[g for g in range(n) if p[g] != -1 and rng.random() < 0.25] for p in parents]
-        text = G.allreduce_trees(parents, [int(rng.integers(1, 5)) for _ in range(m)], chunk, noaggs)
+        text = G.allreduce_trees(parents, [int(rng.integers(1, 5)) for _ in range(m)], chunk, noaggs, relay=relay)
     elif coll == "allgather":
         text = G._header(n, "allgather")
         for s in range(n):
@@ -103,7 +107,7 @@ def _case(seed, large=False, n=None):
     knobs = dict(sched=int(r2.choice([0, 2])), pdl=int(r2.integers(0, 2)),
                  piece_kib=int(r2.choice([0, 0, 16, 48, 512])))
     return dict(n=n, coll=coll, dtype=dtype, count=count, mode=mode, engine=engine, ready=ready, text=text,
-                seed=seed, **knobs)
+                seed=seed, acc_red=acc_red, **knobs)
 
 
 def _eq(a, b):
@@ -134,7 +138,7 @@ def _run(c):
     comm = pkg.Communicator.loopback(n, device=0, scratch_bytes=scratch, mode=c["mode"])
     comm.config("timeout_ms", 20000)
     comm.config("engine", c["engine"])
-    for k in ("sched", "pdl", "piece_kib"):
+    for k in ("sched", "pdl", "piece_kib", "acc_red"):
         comm.config(k, c[k])
     comm.set_strategy(c["coll"], text)
     xs = rank_tensors(dtype, per_rank, n, base=5000 + seed)
@@ -158,4 +162,90 @@ def _run(c):
     assert comm.get_async_error() == 0, c
     for g in range(n):
         assert _eq(to_host(dy[g], dtype), exp[g]), (g, {k: v for k, v in c.items() if k != "text"}, text)
+    comm.finalize()
+
+
+# ------------------------------------------------------------- late join (NEXT-1)
+@pytest.mark.parametrize("seed", range(200))
+def test_fuzz_late_join(seed):
+    """Random trees / noagg / weights / chunks / counts / ready sets, both
+    plans and kernels: a random subset L of the late ranks signals before
+    phase 1 (so every piece includes exactly L), phase 2 adds the rest;
+    both phases bit-exact against oracle.allreduce_late (R4, R10)."""
+    rng = np.random.default_rng(9_000_000 + seed)
+    n = int(rng.integers(3, 9))
+    dtype = ["f32", "bf16", "i32"][int(rng.integers(0, 3))]
+    count = int(np.exp(rng.uniform(np.log(50), np.log(2e6))))
+    chunk = 16 * int(np.exp(rng.uniform(np.log(64), np.log((4 << 20) // 16))))
+    mode = ["direct", "staged"][int(rng.integers(0, 2))]
+    engine = int(rng.integers(0, 3))
+    m = int(rng.integers(1, 4))
+    parents = [_random_tree(rng, n) for _ in range(m)]
+    noaggs = [[g for g in range(n) if p[g] != -1 and rng.random() < 0.2] for p in parents]
+    text = G.allreduce_trees(parents, [int(rng.integers(1, 5)) for _ in range(m)], chunk, noaggs)
+    late = sorted(int(g) for g in rng.choice(n, int(rng.integers(1, n)), replace=False))
+    R = set(range(n)) - set(late)
+    L = {g for g in late if rng.random() < 0.5}
+    comm = pkg.Communicator.loopback(n, device=0, scratch_bytes=8 * count * 4 + (32 << 20), mode=mode)
+    comm.config("timeout_ms", 20000)
+    comm.config("engine", engine)
+    comm.set_strategy("allreduce", text)
+    xs = rank_tensors(dtype, count, n, base=9100 + seed)
+    dx = [to_dev(x, dtype) for x in xs]
+    dy = [empty_dev(count, dtype) for _ in range(n)]
+    t = comm.late_ticket() + 1
+    for g in L:
+        comm.signal_ready(g, ticket=t)
+    comm.allreduce_lb(dx, dy, ready=R, late="join")
+    torch.cuda.synchronize()
+    e1 = oc.allreduce_late(xs, text, R, dtype, L, phase=1)
+    case = dict(seed=seed, n=n, dtype=dtype, count=count, mode=mode, engine=engine, late=late, L=sorted(L))
+    for g in range(n):
+        assert _eq(to_host(dy[g], dtype), e1[g]), ("phase 1", g, case, text)
+    comm.allreduce_lb(dx, dy, ready=R, late="complement")
+    torch.cuda.synchronize()
+    e2 = oc.allreduce_late(xs, text, R, dtype, L, phase=2, y_prev=e1)
+    assert comm.get_async_error() == 0, case
+    for g in range(n):
+        assert _eq(to_host(dy[g], dtype), e2[g]), ("phase 2", g, case, text)
+    comm.finalize()
+
+
+# ------------------------------------------------------------- NVLS (NEXT-2)
+@pytest.mark.parametrize("seed", range(60))
+def test_fuzz_nvls_emulated(seed):
+    """Random mixtures of nvls lines and trees on the loopback-emulated switch:
+    int32 exact, fp32 / bf16 within the switch's any-order bound (R9)."""
+    from oracle import bf16 as obf
+    rng = np.random.default_rng(9_500_000 + seed)
+    n = int(rng.integers(2, 9))
+    dtype = ["f32", "bf16", "i32"][int(rng.integers(0, 3))]
+    count = int(np.exp(rng.uniform(np.log(20), np.log(2e6))))
+    chunk = 16 * int(np.exp(rng.uniform(np.log(64), np.log((2 << 20) // 16))))
+    mode = ["direct", "staged"][int(rng.integers(0, 2))]
+    lines = [f"nvls weight={int(rng.integers(1, 6))} chunk={chunk}" for _ in range(int(rng.integers(1, 3)))]
+    for _ in range(int(rng.integers(0, 3))):
+        lines.append(f"tree weight={int(rng.integers(1, 4))} chunk={chunk} parent={G._join(_random_tree(rng, n))}")
+    order = [int(i) for i in rng.permutation(len(lines))]
+    text = G._header(n, "allreduce") + "\n".join(lines[i] for i in order) + "\n"
+    comm = pkg.Communicator.loopback(n, device=0, scratch_bytes=8 * count * 4 + (32 << 20), mode=mode)
+    ok, why = comm.nvls_setup(2 * count * 4 + (1 << 20))
+    assert ok, why
+    comm.set_strategy("allreduce", text)
+    xs = rank_tensors(dtype, count, n, base=9600 + seed)
+    dy = [empty_dev(count, dtype) for _ in range(n)]
+    comm.allreduce_lb([to_dev(x, dtype) for x in xs], dy)
+    torch.cuda.synchronize()
+    assert comm.get_async_error() == 0
+    exp = oc.allreduce(xs, text, set(range(n)), dtype)
+    got = [to_host(y, dtype) for y in dy]
+    case = dict(seed=seed, n=n, dtype=dtype, count=count, mode=mode)
+    for g in range(n):
+        if dtype == "i32":
+            assert np.array_equal(got[g], exp[g]), (g, case, text)
+        else:
+            f = (lambda a: obf.to_f32(a).astype(np.float64)) if dtype == "bf16" else (lambda a: a.astype(np.float64))
+            den = np.sum(np.abs(np.stack([f(x) for x in xs])), axis=0) + 1e-30
+            # tree partitions replay bit-exactly within the same bound; nvls ones are order-free
+            assert np.max(np.abs(f(got[g]) - f(exp[g])) / den) <= 2 * oc.nvls_tolerance(dtype, n) + 1e-12, (g, case)
     comm.finalize()
