@@ -370,6 +370,8 @@ def run_single(args):
     # download overlaps step i+1's upload (PCIe is full duplex); per-step time
     # = span of all steps / steps.
     e2e_t = e2e_pipelined(comm, host_in, dx, dy, args.e2e_steps, tdt, lambda xs, ys: comm.allreduce_lb(xs, ys))
+    pcie = pcie_bidir_gbs()
+    pcie_ms = n * nbytes / (pcie * 1e9) * 1e3      # every step moves n*S each way
 
     peak, peak_src = load_peaks()
     sweep = None
@@ -410,7 +412,10 @@ def run_single(args):
                 "h2d_bytes_per_step": n * nbytes, "d2h_bytes_per_step": n * nbytes,
                 "ms_per_step": round(e2e_t, 3), "steps": args.e2e_steps,
                 "how": "pinned H2D of all inputs + allreduce_lb + D2H of all outputs per step; steps "
-                       "double-buffered with H2D and D2H on separate copy streams (full-duplex PCIe)"},
+                       "double-buffered with H2D and D2H on separate copy streams (full-duplex PCIe)",
+                "pcie_bidir_GBps_per_direction": round(pcie, 1),
+                "pcie_bound_ms_per_step": round(pcie_ms, 3),
+                "pcie_roofline_frac": round(pcie_ms / e2e_t, 4)},
         "gpu_launches": launches,
         "clocks": clk.summary(),
         "parity": parity,
@@ -427,6 +432,33 @@ def run_single(args):
         out["cpu_baseline"] = cpu_baseline_block(xs_np, text, n, args.dtype, oracle_s)
     comm.finalize()
     return out
+
+
+def pcie_bidir_gbs(nbytes=256 << 20, reps=3):
+    """Pinned host <-> device throughput with both directions busy at once
+    (the e2e steps' regime): GB/s per direction."""
+    import torch
+    h = [torch.empty(nbytes, dtype=torch.uint8).pin_memory() for _ in range(2)]
+    d = [torch.empty(nbytes, dtype=torch.uint8, device="cuda") for _ in range(2)]
+    s = [torch.cuda.Stream(), torch.cuda.Stream()]
+    cur = torch.cuda.current_stream()
+    best = 0.0
+    for _ in range(reps):
+        torch.cuda.synchronize()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(cur)
+        for x in s:
+            x.wait_stream(cur)
+        with torch.cuda.stream(s[0]):
+            d[0].copy_(h[0], non_blocking=True)
+        with torch.cuda.stream(s[1]):
+            h[1].copy_(d[1], non_blocking=True)
+        for x in s:
+            cur.wait_stream(x)
+        b.record(cur)
+        torch.cuda.synchronize()
+        best = max(best, nbytes / (a.elapsed_time(b) * 1e-3) / 1e9)
+    return best
 
 
 def e2e_pipelined(comm, host_in, dx, dy, steps, tdt, call, second=None):

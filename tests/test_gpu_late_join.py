@@ -189,8 +189,9 @@ def test_late_join_interleaved_plans(engine):
     comm.finalize()
 
 
+@pytest.mark.parametrize("mode", ["direct", "staged"])
 @pytest.mark.parametrize("engine", [0, 1])
-def test_late_join_graph_replay(engine):
+def test_late_join_graph_replay(engine, mode):
     """Phase 1 + phase 2 captured in one CUDA graph (the ticket is baked in) and replayed: every replay
     rebuilds phase 1's list of incomplete pieces from scratch (phase 2 empties its list when it ends),
     so rank 6 is added exactly once per replay (int32, exact) while rank 3 joins every piece."""
@@ -198,7 +199,7 @@ def test_late_join_graph_replay(engine):
     R, late = {0, 1, 2, 4, 5, 7}, [3, 6]
     text = G.allreduce_stars(n, chunk=65536)
     xs = rank_tensors("i32", count, n)
-    comm = _comm(n, engine)
+    comm = _comm(n, engine, mode)
     comm.set_strategy("allreduce", text)
     dx = [to_dev(x, "i32") for x in xs]
     dy = [empty_dev(count, "i32") for _ in range(n)]
