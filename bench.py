@@ -88,14 +88,19 @@ def load_peaks():
 
 
 def profile_traffic(key):
-    """dram bytes per launch from the committed ncu --set full summary, if any."""
-    path = os.path.join(ROOT, "profiles", "ncu_summary.json")
-    try:
-        with open(path) as f:
-            d = json.load(f)
-        return d.get(key, {}).get("dram_bytes_per_launch")
-    except Exception:  # noqa: BLE001
-        return None
+    """dram bytes per launch from the newest committed ncu --set full summary
+    (profiles/ncu_summary_rNN.json, else the r01 ncu_summary.json), if any."""
+    import glob
+    paths = sorted(glob.glob(os.path.join(ROOT, "profiles", "ncu_summary_r*.json")), reverse=True)
+    for path in paths + [os.path.join(ROOT, "profiles", "ncu_summary.json")]:
+        try:
+            with open(path) as f:
+                v = json.load(f).get(key, {}).get("dram_bytes_per_launch")
+            if v:
+                return v
+        except Exception:  # noqa: BLE001
+            continue
+    return None
 
 
 def traffic_key(engine, mode):
