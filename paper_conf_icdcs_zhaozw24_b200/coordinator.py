@@ -211,9 +211,12 @@ class OnlineCoordinator:
     and issues LATE_COMPLEMENT (phase 2: only the chunks phase 1 missed).
 
     issue(mask, late) enqueues this rank's collective call: late = None (a
-    plain AllReduce over everyone: the "full" decision, after which the
+    plain collective over everyone: the "full" decision, after which the
     round's ticket is retired with adapcc_late_advance), 'join' (phase 1) or
-    'complement' (phase 2).  Ranks signal readiness with comm.signal_ready(ticket=
+    'complement' (phase 2).  The callback decides what a phase is, so the
+    same coordinator drives AlltoAll / Broadcast too (phase 1 = the ready
+    sources, phase 2 = the late ones; P:L135 prices them with the policy's
+    `coll`).  Ranks signal readiness with comm.signal_ready(ticket=
     coordinator.ticket()) after their computation (the ticket of the
     collective the coordinator runs next).  policy: a Coordinator (fresh per
     call: its waited time accumulates); cycle: seconds between decisions

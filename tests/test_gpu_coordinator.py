@@ -135,3 +135,48 @@ def test_coordinator_multiprocess_shared_board():
                 p.kill()
     for r in range(n):
         assert r in out and out[r][0], out.get(r)
+
+
+def test_coordinator_alltoall_two_phases():
+    """The coordinator's issue callback is collective-agnostic: AlltoAll
+    (P:L135 prices it at N x tensor) runs phase 1 among the ready sources and
+    phase 2 for the late ones (their blocks were left untouched, reading
+    Q12); the final result is the complete block transpose."""
+    from oracle import collectives as oc2
+    n, cnt = 8, 4096
+    xs = rank_tensors("bf16", n * cnt, n)
+    comm = pkg.Communicator.loopback(n, mode="direct", scratch_bytes=64 << 20)
+    comm.set_strategy("alltoall", G.alltoall_direct(n))
+    dx = [to_dev(x, "bf16") for x in xs]
+    dy = [empty_dev(n * cnt, "bf16") for _ in range(n)]
+    side = torch.cuda.Stream()
+    all_mask = (1 << n) - 1
+
+    def policy():
+        p = C.Coordinator(n, "alltoall", n * cnt * 2, 100e9, 5e-6)
+        p.buy_cost = lambda k: 50e-6
+        return p
+
+    coord = C.OnlineCoordinator(comm, policy, cycle=2e-6)
+    t = coord.ticket()
+    for r in range(n):
+        if r not in (2, 5):
+            comm.signal_ready(r, ticket=t)
+    comm.spin(3_000_000, stream=side)
+    comm.signal_ready(2, ticket=t, stream=side)
+    comm.signal_ready(5, ticket=t, stream=side)
+
+    def issue(mask, late):
+        if late is None:
+            comm.alltoall_lb(dx, dy)
+        elif late == "join":
+            comm.alltoall_lb(dx, dy, ready=mask)
+        else:   # phase 2: the late sources' blocks
+            comm.alltoall_lb(dx, dy, ready=all_mask & ~mask)
+    res = coord.allreduce(issue)
+    torch.cuda.synchronize()
+    assert res["action"] == "phase1" and res["mask"] == all_mask & ~((1 << 2) | (1 << 5)), res
+    exp = oc2.alltoall(xs, G.alltoall_direct(n), set(range(n)), "bf16", [np.zeros(n * cnt, np.uint16)] * n)
+    for g in range(n):
+        assert np.array_equal(to_host(dy[g], "bf16"), exp[g])
+    comm.finalize()
