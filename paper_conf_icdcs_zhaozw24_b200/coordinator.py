@@ -270,6 +270,8 @@ class OnlineCoordinator:
             issue(mask, None)
         else:
             issue(mask, "join")               # phase 1
+            if self.comm.late_ticket() < t:   # (a phase 1 that is not a LATE_JOIN call, e.g. AlltoAll)
+                self.comm.late_advance()
         late = all_mask & ~mask
         t_late = None
         if late:
