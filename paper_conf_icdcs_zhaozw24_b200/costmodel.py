@@ -180,6 +180,31 @@ def chunk_from_profile(profile, S, text_for_chunk=None, candidates=(1 << 14, 1 <
     return best_chunk(fn, S, alpha, beta, candidates)
 
 
+def adapt_strategy(comm, tensor_bytes, ready=None, profile=None, engine="sm", set_default_chunk=True,
+                   **probe_kw):
+    """The paper's adaptation loop (P:L109-115 profiling -> P:L176-231 strategy
+    -> P:L341-343 swap without restart) in one call: profile the links (or use
+    `profile`), weight the n star trees by the measured per-GPU bandwidth and
+    the ready set (generator.mask_aware_star_weights, the link-load model of
+    P:L194-215), pick the chunk with the cost model (eqs. 2-6) and install
+    the result with set_strategy (stream-ordered, reading a10).  Collective in
+    multi-process mode (profiling probes every link).  Returns (text,
+    profile, chunk)."""
+    from . import generator as G
+    prof = profile or profile_links(comm, engine=engine, **probe_kw)
+    n = comm.nranks
+    R = set(range(n)) if ready is None else set(ready)
+    bw = per_gpu_bandwidth(prof)
+    ints, _, _ = G.mask_aware_star_weights(n, R, bw=bw)
+    chunk, _ = chunk_from_profile(prof, tensor_bytes,
+                                  text_for_chunk=lambda c: G.allreduce_stars(n, chunk=c, weights=ints))
+    text = G.allreduce_stars(n, chunk=chunk, weights=ints)
+    comm.set_strategy("allreduce", text)
+    if set_default_chunk:
+        comm.config("default_chunk", chunk)
+    return text, prof, chunk
+
+
 # -------------------------------------------------------------- cost model
 def _trees(text):
     n, coll, nsubs = _A.strategy_check(text)

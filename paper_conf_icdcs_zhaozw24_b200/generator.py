@@ -115,33 +115,49 @@ def mask_aware_star_weights(n, ready, bw=None, relays_as_roots=True, scale=1 << 
 
 
 def _solve_lp(n, ready, bw, relays_as_roots):
+    """Min-max weights by water-filling (no solver needed): GPU g's time
+    s_g(w) = max(egress_g(w), ingress_g(w)) / b_g is affine-increasing in its
+    own weight w (star_loads), so the lexicographic min-max allocation under
+    sum w = 1 raises a common level L until the weights w_g(L) = the largest w
+    with s_g(w) <= L (0 if g's base load already exceeds L; 0 for relays when
+    they may not root) sum to 1.  Among the min-max optima it is the one that
+    evens out every non-bottleneck GPU (an LP vertex would pile the weight
+    onto a few of them when a slow GPU's own slice sets the maximum)."""
+    ready = set(ready)
     k = len(ready)
-    try:
-        from scipy.optimize import linprog
-    except ImportError:  # symmetric two-class search (uniform links only)
-        return _two_class(n, ready, relays_as_roots)
-    # variables: w_0..w_{n-1}, t ; minimise t
-    c = [0.0] * n + [1.0]
-    A, b = [], []
+    terms = []   # per g: [(c, d)] with load = c + d w for egress and ingress
     for g in range(n):
-        a = [0.0] * (n + 1)
-        # egress: [g in R](1 - w_g) + (n-1) w_g <= t b_g
-        a[g] = (n - 1) - (1 if g in ready else 0)
-        a[n] = -bw[g]
-        A.append(a)
-        b.append(-(1.0 if g in ready else 0.0))
-        a = [0.0] * (n + 1)
-        # ingress: (k - [g in R]) w_g + 1 - w_g <= t b_g
-        a[g] = (k - (1 if g in ready else 0)) - 1
-        a[n] = -bw[g]
-        A.append(a)
-        b.append(-1.0)
-    Aeq = [[1.0] * n + [0.0]]
-    bounds = [(0, None if (g in ready or relays_as_roots) else 0) for g in range(n)] + [(0, None)]
-    res = linprog(c, A_ub=A, b_ub=b, A_eq=Aeq, b_eq=[1.0], bounds=bounds, method="highs")
-    if not res.success:
-        return _two_class(n, ready, relays_as_roots)
-    return [max(0.0, float(x)) for x in res.x[:n]]
+        r = g in ready
+        terms.append([(1.0 if r else 0.0, (n - 1) - (1.0 if r else 0.0)),      # egress
+                      (1.0, (k - (1.0 if r else 0.0)) - 1.0)])                  # ingress
+    ub = [1.0 if (g in ready or relays_as_roots) else 0.0 for g in range(n)]
+
+    def w_at(L):
+        out = []
+        for g in range(n):
+            w = ub[g]
+            for c, d in terms[g]:
+                if c > L * bw[g]:
+                    w = 0.0
+                elif d > 0:
+                    w = min(w, (L * bw[g] - c) / d)
+            out.append(max(0.0, w))
+        return out
+
+    lo, hi = 0.0, 1.0
+    while sum(w_at(hi)) < 1.0:
+        hi *= 2.0
+        if hi > 1e12:
+            return _two_class(n, ready, relays_as_roots)
+    for _ in range(200):
+        mid = 0.5 * (lo + hi)
+        if sum(w_at(mid)) < 1.0:
+            lo = mid
+        else:
+            hi = mid
+    w = w_at(hi)
+    tot = sum(w)
+    return [x / tot for x in w]
 
 
 def _two_class(n, ready, relays_as_roots):

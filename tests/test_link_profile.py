@@ -121,3 +121,37 @@ def test_multiprocess_rounds_gloo(n):
         # rank r probes (r + i) % n in round i: one partner per round, a permutation overall
         partners = [c[1] for c in calls if c[1] and len(c[1]) == 1]
         assert sorted({x[0] for x in partners}) == sorted({(r + i) % n for i in range(1, n)})
+
+
+class FakeStrategyComm(FakeComm):
+    def __init__(self, *a, **k):
+        super().__init__(*a, **k)
+        self.set_calls, self.config_calls = [], []
+
+    def set_strategy(self, coll, text):
+        self.set_calls.append((coll, text))
+
+    def config(self, key, value):
+        self.config_calls.append((key, value))
+
+
+def test_adapt_strategy_weights_follow_bandwidth():
+    """A GPU with half the link bandwidth roots a smaller partition; the
+    chunk is the cost model's choice; the strategy is installed."""
+    from paper_conf_icdcs_zhaozw24_b200 import adapcc as A
+    n = 4
+    alpha = [[2e-6] * n for _ in range(n)]
+    beta = [[1.0 / (800e9 if i != 2 else 400e9)] * n for i in range(n)]
+    c = FakeStrategyComm(n, 0, True, alpha, beta)
+    # loopback probes only rank 0's links: give every rank its own row
+    prof = CM.profile_links(c)
+    for i in range(n):
+        for j in range(n):
+            if i != j:
+                prof["beta_GBps"][i][j] = 1.0 / beta[i][j] / 1e9
+    text, _, chunk = CM.adapt_strategy(c, 64 << 20, profile=prof)
+    assert c.set_calls == [("allreduce", text)] and ("default_chunk", chunk) in c.config_calls
+    w = [A.strategy_sub(text, m)[0] for m in range(n)]
+    assert w[2] < min(w[g] for g in range(n) if g != 2)
+    assert chunk == CM.chunk_from_profile(prof, 64 << 20, text_for_chunk=lambda ch: text.replace(
+        f"chunk={chunk}", f"chunk={ch}"))[0]
