@@ -6,6 +6,7 @@ import os
 import socket
 import sys
 
+import numpy as np
 import pytest
 
 torch = pytest.importorskip("torch")
@@ -100,3 +101,24 @@ def test_multiprocess_probe_rounds():
             for j in range(n):
                 if i != j:   # every link probed by its sender (one GPU here: time-sliced, so no bound on beta)
                     assert p["alpha_us"][i][j] is not None and f"{i}->{j}" in p["samples"]
+
+
+def test_adapt_strategy_end_to_end():
+    """Profile -> bandwidth-weighted stars -> cost-model chunk -> installed
+    strategy; the next AllReduce runs on it bit-exactly (oracle replay of the
+    new text)."""
+    from oracle import collectives as oc
+    from synth import rank_tensors
+    from tests.gpu_util import bits, empty_dev, to_dev, to_host
+    n, count = 4, 1_000_003
+    comm = pkg.Communicator.loopback(n, scratch_bytes=256 << 20)
+    text, prof, chunk = CM.adapt_strategy(comm, count * 4, ready={0, 1, 3}, sizes=(1 << 16, 1 << 20),
+                                          repeats=(1, 4))
+    assert chunk % 16 == 0 and "tree" in text
+    xs = rank_tensors("f32", count, n)
+    dy = [empty_dev(count, "f32") for _ in range(n)]
+    comm.allreduce_lb([to_dev(x, "f32") for x in xs], dy, ready={0, 1, 3})
+    torch.cuda.synchronize()
+    exp = oc.allreduce(xs, text, {0, 1, 3}, "f32")
+    assert all(np.array_equal(bits(to_host(y, "f32")), bits(e)) for y, e in zip(dy, exp))
+    comm.finalize()
