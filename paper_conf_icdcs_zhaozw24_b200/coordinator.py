@@ -160,6 +160,7 @@ def exclude_faulty(comm, ready_times, phase1_end, now, factor=T_FAULT_FACTOR, st
 
 # ------------------------------------------------------- online coordinator
 BOARD_DECISION = 64      # readiness-board words: 64 sequence, 65 action, 66 mask (adapcc_ready_board)
+BOARD_PHASE2 = 68        # 68 sequence, 69 faulty mask (0: every late rank signalled, run phase 2)
 _ACTIONS = {"full": 1, "phase1": 2}
 
 
@@ -186,6 +187,20 @@ class ReadyBoard:
         w[BOARD_DECISION + 1] = _ACTIONS[action]
         w[BOARD_DECISION + 2] = mask
         w[BOARD_DECISION] = seq            # last: followers read seq first (x86 stores stay ordered)
+
+    def publish_phase2(self, seq, faulty):
+        w = self.words
+        w[BOARD_PHASE2 + 1] = faulty
+        w[BOARD_PHASE2] = seq
+
+    def wait_phase2(self, seq, timeout, clock):
+        """Follower side of the phase-2 decision; returns the faulty mask."""
+        w = self.words
+        t0 = clock()
+        while w[BOARD_PHASE2] < seq:
+            if clock() - t0 > timeout:
+                raise TimeoutError("coordinator phase-2 decision not published")
+        return int(w[BOARD_PHASE2 + 1])
 
     def wait_decision(self, seq, timeout, clock):
         w = self.words
@@ -222,8 +237,18 @@ class OnlineCoordinator:
     call: its waited time accumulates); cycle: seconds between decisions
     (the paper's 5 ms, scaled to the collective's time scale, reading R2)."""
 
-    def __init__(self, comm, policy_factory, cycle=5e-6, timeout=30.0, clock=None):
+    def __init__(self, comm, policy_factory, cycle=5e-6, timeout=30.0, clock=None, fault_factor=None,
+                 store=None, stream=None):
+        """fault_factor: apply the T_fault rule -- late ranks not
+        ready fault_factor x (phase-1 end - first ready) after phase 1 ended
+        are faulty: the survivors exclude them (adapcc_exclude; multi-process
+        through `store`) and keep the phase-1 result.  None: wait
+        for them up to `timeout`.  stream: the stream issue() enqueues phase 1
+        on (its end is T_fault's reference; default: the current stream)."""
         import time
+        self.fault_factor = fault_factor
+        self.store = store
+        self.stream = stream
         self.comm = comm
         self.board = ReadyBoard(comm)
         self.policy_factory = policy_factory
@@ -241,15 +266,21 @@ class OnlineCoordinator:
 
     def allreduce(self, issue):
         n, clock = self.comm.nranks, self.clock
-        all_mask = (1 << n) - 1
+        members = getattr(self.comm, "members", None) or set(range(n))
+        all_mask = sum(1 << r for r in members)        # excluded ranks take no part
         t = self.ticket()
         self.seq += 1
         t0 = clock()
+        t_first = None
         if self.leader:
             policy = self.policy_factory()
+            if len(members) < n and hasattr(policy, "n"):
+                policy.n = len(members)        # the policy prices the survivors' collective
             nxt = t0
             while True:
-                ready = self.board.ready(t)
+                ready = self.board.ready(t) & members
+                if ready and t_first is None:
+                    t_first = clock()          # the fastest worker became ready (T_fault's origin)
                 d = policy.step(clock() - t0, ready)
                 if d.action != "wait":
                     break
@@ -270,17 +301,62 @@ class OnlineCoordinator:
             issue(mask, None)
         else:
             issue(mask, "join")               # phase 1
+            self._p1_done = self._record()
             if self.comm.late_ticket() < t:   # (a phase 1 that is not a LATE_JOIN call, e.g. AlltoAll)
                 self.comm.late_advance()
         late = all_mask & ~mask
         t_late = None
+        faulty = 0
         if late:
-            while True:                       # phase 2 once every late rank is ready
-                if all((self.board.words[r] >= t) for r in range(n) if (late >> r) & 1):
-                    break
-                if clock() - t0 > self.timeout:
-                    raise TimeoutError("late ranks never became ready (fault: see exclude_faulty)")
-            t_late = clock()
-            issue(mask, "complement")
+            faulty = self._phase2_or_fault(t, mask, late, t0, t_first)
+            if not faulty:
+                t_late = clock()
+                issue(mask, "complement")
+            else:   # T_fault passed: the survivors keep the phase-1 result and drop the faulty ranks
+                dead = {r for r in range(n) if (faulty >> r) & 1}
+                if self.comm.loopback or self.comm.rank not in dead:
+                    self.comm.exclude(dead, store=self.store)
         return {"action": action, "mask": mask, "ticket": t, "decided_after_s": t_decide - t0,
-                "phase2_after_s": None if t_late is None else t_late - t0}
+                "phase2_after_s": None if t_late is None else t_late - t0,
+                "faulty": sorted(r for r in range(n) if (faulty >> r) & 1)}
+
+    def _phase2_or_fault(self, t, mask, late, t0, t_first):
+        """Leader: wait until every late rank signalled (-> 0) or, with a
+        fault_factor, until T_fault after phase 1 passes (-> the mask of the
+        late ranks still not ready); publish it.  Followers: read it."""
+        clock, n = self.clock, self.comm.nranks
+        self.seq2 = getattr(self, "seq2", 0) + 1
+        if not self.leader:
+            return self.board.wait_phase2(self.seq2, self.timeout, clock)
+        p1_done = self._p1_done
+        t_p1 = None
+        faulty = 0
+        while True:
+            missing = [r for r in range(n) if (late >> r) & 1 and self.board.words[r] < t]
+            if not missing:
+                break
+            now = clock()
+            if t_p1 is None and (p1_done is None or p1_done.query()):
+                t_p1 = now                     # phase 1 finished on this GPU
+            if self.fault_factor is not None and t_p1 is not None and t_first is not None and \
+                    now - t_p1 >= self.fault_factor * (t_p1 - t_first):
+                faulty = sum(1 << r for r in missing)
+                break
+            if now - t0 > self.timeout:
+                raise TimeoutError("late ranks never became ready (fault: set fault_factor or see exclude_faulty)")
+        if not self.comm.loopback:
+            self.board.publish_phase2(self.seq2, faulty)
+        return faulty
+
+    def _record(self):
+        """A CUDA event after phase 1 on the issue stream (None without a GPU:
+        host-only tests treat phase 1 as ended when issue() returns)."""
+        try:
+            import torch
+        except ImportError:
+            return None
+        if not torch.cuda.is_available():
+            return None
+        ev = torch.cuda.Event()
+        ev.record(self.stream)
+        return ev

@@ -180,3 +180,134 @@ def test_coordinator_alltoall_two_phases():
     for g in range(n):
         assert np.array_equal(to_host(dy[g], "bf16"), exp[g])
     comm.finalize()
+
+
+@pytest.mark.parametrize("mode", ["direct", "staged"])
+def test_coordinator_fault_rule_excludes_silent_rank(mode):
+    """NEXT-3 on the hot path: virtual rank 6 never signals.
+    The coordinator starts phase 1 without it, and T_fault = 5 x (phase-1 end
+    - first ready) after phase 1 marks it faulty. The survivors exclude it and
+    keep the phase-1 result (the exact survivors' sum). Later rounds, one of
+    them with a straggler among the survivors (late join + phase 2), run on
+    the survivors only: rank 6's recvbuf is no longer written."""
+    n, count, dead = 8, 1_000_003, 6
+    xs = rank_tensors("i32", count, n)
+    comm = pkg.Communicator.loopback(n, mode=mode, scratch_bytes=64 << 20)
+    comm.config("timeout_ms", 60000)
+    comm.set_strategy("allreduce", G.allreduce_stars(n, chunk=65536))
+    dx = [to_dev(x, "i32") for x in xs]
+    dy = [empty_dev(count, "i32") for _ in range(n)]
+    cs = torch.cuda.Stream(priority=-1)
+    side = torch.cuda.Stream()
+    coord = C.OnlineCoordinator(comm, lambda: _policy(n, count * 4, 50e-6), cycle=2e-6,
+                                fault_factor=5.0, stream=cs, timeout=20.0)
+    live = set(range(n)) - {dead}
+    survivors_sum = oc.allreduce_exact([xs[g] for g in sorted(live)], set(range(n - 1)), "i32")
+
+    t = coord.ticket()
+    for r in live:
+        comm.signal_ready(r, ticket=t, stream=cs)
+    res = coord.allreduce(lambda m, lt: comm.allreduce_lb(dx, dy, ready=m, late=lt, stream=cs))
+    torch.cuda.synchronize()
+    assert res["action"] == "phase1" and res["faulty"] == [dead], res
+    assert comm.members == live and comm.get_async_error() == 0
+    for g in live:
+        assert np.array_equal(to_host(dy[g], "i32"), survivors_sum), g
+    dy[dead].fill_(-7)
+    sentinel = to_host(dy[dead], "i32").copy()
+    # a full round, then a straggler (rank 2) among the survivors that signals
+    # within T_fault (phase 1 ends ~0.1-0.2 ms after the first ready rank)
+    for it, lag_us in enumerate((0, 300)):
+        for g in live:
+            dy[g].zero_()
+        t = coord.ticket()
+        for r in live - {2}:
+            comm.signal_ready(r, ticket=t, stream=cs)
+        comm.spin(lag_us * 1000, stream=side)
+        comm.signal_ready(2, ticket=t, stream=side)
+        res = coord.allreduce(lambda m, lt: comm.allreduce_lb(
+            [d if g != dead else None for g, d in enumerate(dx)], dy, ready=m, late=lt, stream=cs))
+        torch.cuda.synchronize()
+        assert comm.get_async_error() == 0
+        assert res["faulty"] == [] and res["action"] == ("full" if lag_us == 0 else "phase1"), (it, res)
+        for g in live:
+            assert np.array_equal(to_host(dy[g], "i32"), survivors_sum), (it, g)
+        assert np.array_equal(to_host(dy[dead], "i32"), sentinel)
+    comm.finalize()
+
+
+def _fault_worker(rank, n, port, q):
+    try:
+        sys.path.insert(0, ROOT)
+        import torch.distributed as dist
+        os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+        dist.init_process_group("gloo", rank=rank, world_size=n)
+        store = dist.distributed_c10d._get_default_store()
+        dev = rank % torch.cuda.device_count()
+        torch.cuda.set_device(dev)
+        comm = pkg.Communicator.init(scratch_bytes=64 << 20, device=dev)
+        comm.config("timeout_ms", 60000)
+        count = 300_007
+        xs = rank_tensors("i32", count, n)
+        x, y = to_dev(xs[rank], "i32"), empty_dev(count, "i32")
+        dead = n - 1
+        cs = torch.cuda.Stream(priority=-1)
+        coord = C.OnlineCoordinator(comm, lambda: _policy(n, count * 4, 100e-6), cycle=5e-6, fault_factor=5.0,
+                                    store=store, stream=cs, timeout=60.0)
+        t = coord.ticket()
+        dist.barrier()
+        if rank != dead:                      # the faulty rank never signals
+            comm.signal_ready(ticket=t, stream=cs)
+        res = coord.allreduce(lambda m, lt: comm.allreduce(x, y, ready=m, late=lt, stream=cs))
+        torch.cuda.synchronize()
+        live = set(range(n)) - {dead}
+        exp = oc.allreduce_exact([xs[g] for g in sorted(live)], set(range(n - 1)), "i32")
+        ok = [res["faulty"] == [dead]]
+        if rank == dead:                      # excluded: stays alive (its arena is mapped) until the survivors finish
+            store.wait(["fault-test/done"])
+        else:
+            ok.append(comm.members == live)
+            ok.append(np.array_equal(to_host(y, "i32"), exp))
+            for _ in range(2):                # the survivors carry on: a full round
+                y.zero_()
+                t = coord.ticket()
+                comm.signal_ready(ticket=t, stream=cs)
+                res = coord.allreduce(lambda m, lt: comm.allreduce(x, y, ready=m, late=lt, stream=cs))
+                torch.cuda.synchronize()
+                ok.append((res["faulty"], np.array_equal(to_host(y, "i32"), exp)))
+            if store.add("fault-test/finished", 1) == n - 1:
+                store.set("fault-test/done", b"1")
+        err = comm.get_async_error()
+        good = all(o if isinstance(o, bool) else (o[0] == [] and o[1]) for o in ok)
+        q.put((rank, err == 0 and good, f"{ok} err={err} res={res}"))
+        comm.finalize()
+    except Exception as e:  # noqa: BLE001
+        import traceback
+        q.put((rank, False, traceback.format_exc() + repr(e)))
+
+
+def test_coordinator_fault_rule_multiprocess():
+    """3 processes, rank 2 never signals: the leader applies T_fault after
+    phase 1 and publishes the faulty mask on the node-shared board; ranks 0
+    and 1 exclude rank 2 through the store (adapcc_exclude) and keep running
+    full collectives on the survivors, exact."""
+    import torch.multiprocessing as mp
+    n = 3
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _port()
+    ps = [ctx.Process(target=_fault_worker, args=(r, n, port, q)) for r in range(n)]
+    for p in ps:
+        p.start()
+    out = {}
+    try:
+        for _ in range(n):
+            r, ok, msg = q.get(timeout=300)
+            out[r] = (ok, msg)
+    finally:
+        for p in ps:
+            p.join(timeout=30)
+            if p.is_alive():
+                p.kill()
+    for r in range(n):
+        assert r in out and out[r][0], out.get(r)

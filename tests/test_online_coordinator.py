@@ -104,3 +104,84 @@ def test_follower_takes_the_leaders_decision():
     tf.join()
     assert out["l"][1] == out["f"][1] == [(0b01, "join"), (0b01, "complement")]
     assert out["f"][0]["action"] == "phase1"
+
+
+class ExcludingComm(FakeComm):
+    def __init__(self, *a, **k):
+        super().__init__(*a, **k)
+        self.members = set(range(self.nranks))
+        self.excluded = []
+
+    def exclude(self, dead, store=None):
+        self.excluded.append(set(dead))
+        self.members -= set(dead)
+
+
+def test_fault_rule_excludes_a_rank_that_never_signals():
+    """phase 1 ends, the late rank stays silent for more than
+    T_fault = factor x (phase-1 end - first ready): it is excluded, phase 2
+    is not issued; the next round prices and masks the survivors only."""
+    n, t = 4, 5
+    comm = ExcludingComm(n)
+    for r in range(3):
+        comm.board[r] = t               # rank 3 never signals
+    calls = []
+
+    def issue(m, late):
+        calls.append((m, late))
+        time.sleep(0.01)                # "phase 1" runs 10 ms after the first ready rank
+    oc = C.OnlineCoordinator(comm, lambda: _policy(n, 1e-3), cycle=1e-4, fault_factor=2.0, timeout=5.0)
+    t0 = time.perf_counter()
+    res = oc.allreduce(issue)
+    took = time.perf_counter() - t0
+    assert calls == [(0b0111, "join")] and res["faulty"] == [3] and res["phase2_after_s"] is None
+    assert comm.excluded == [{3}] and comm.members == {0, 1, 2}
+    assert 0.02 < took < 1.0            # ~ phase 1 (>= 10 ms) + 2 x that, not the timeout
+    # next round: all survivors ready -> one "full" call over the survivors' mask
+    for r in range(3):
+        comm.board[r] = t + 1
+    calls.clear()
+    res = oc.allreduce(lambda m, late: calls.append((m, late)))
+    assert res["action"] == "full" and calls == [(0b0111, None)]
+
+
+def test_late_rank_within_t_fault_is_not_excluded():
+    n, t = 4, 5
+    comm = ExcludingComm(n)
+    for r in range(3):
+        comm.board[r] = t
+    calls = []
+
+    def issue(m, late):
+        calls.append((m, late))
+        if late == "join":
+            time.sleep(0.02)
+            threading.Timer(0.01, lambda: comm.board.__setitem__(3, t)).start()   # ready 10 ms after phase 1
+    oc = C.OnlineCoordinator(comm, lambda: _policy(n, 1e-3), cycle=1e-4, fault_factor=5.0, timeout=5.0)
+    res = oc.allreduce(issue)
+    assert res["faulty"] == [] and comm.excluded == []
+    assert calls == [(0b0111, "join"), (0b0111, "complement")]
+
+
+def test_follower_takes_the_leaders_fault_decision():
+    n, t = 3, 3
+    board = (ctypes.c_uint64 * 128)()
+    board[0] = board[1] = t            # rank 2 never signals
+    lc = ExcludingComm(n, 0, False, board, t - 1)
+    fc = ExcludingComm(n, 1, False, board, t - 1)
+    leader = C.OnlineCoordinator(lc, lambda: _policy(n, 1e-3), cycle=1e-4, fault_factor=1.0, timeout=5.0)
+    follower = C.OnlineCoordinator(fc, lambda: pytest.fail("a follower must not decide"), cycle=1e-4,
+                                   timeout=5.0)
+    out = {}
+
+    def run(name, oc):
+        calls = []
+        out[name] = (oc.allreduce(lambda m, late: calls.append((m, late))), calls)
+
+    tf = threading.Thread(target=run, args=("f", follower))
+    tf.start()
+    run("l", leader)
+    tf.join()
+    assert out["l"][1] == out["f"][1] == [(0b011, "join")]
+    assert out["l"][0]["faulty"] == out["f"][0]["faulty"] == [2]
+    assert lc.excluded == fc.excluded == [{2}]
