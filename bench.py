@@ -60,6 +60,7 @@ def parse_args():
     p.add_argument("--no-nccl-legs", action="store_true",
                    help="N>1: skip the NCCL_ALGO / NVLS leg runs (separate torchrun jobs)")
     p.add_argument("--nccl-leg", default=None, help=argparse.SUPPRESS)   # internal: one NCCL variant
+    p.add_argument("--nvls-leg", action="store_true", help=argparse.SUPPRESS)   # internal: the NVLS leg
     p.add_argument("--test-same-gpu", action="store_true",
                    help="N>1 code-path check on a 1-GPU box: every rank on cuda:0, gloo, no NCCL leg "
                         "(numbers are NOT NVLink measurements)")
@@ -636,29 +637,113 @@ def run_nccl_leg(args):
     return None
 
 
+def leg_job(args, world, extra, env, name):
+    """Rank 0, after the main run: one measurement as its own torchrun job of
+    `world` ranks (fresh processes: NCCL reads its environment at start, and a
+    failing leg cannot poison this process's CUDA context).  Returns the
+    job's JSON line, or {"unavailable": why}."""
+    e = dict(os.environ)
+    for k in list(e):
+        if k in ("RANK", "WORLD_SIZE", "LOCAL_RANK", "LOCAL_WORLD_SIZE", "MASTER_ADDR", "MASTER_PORT",
+                 "GROUP_RANK", "GROUP_WORLD_SIZE", "ROLE_RANK", "ROLE_WORLD_SIZE", "ROLE_NAME") or \
+                k.startswith("TORCHELASTIC_"):
+            e.pop(k)
+    e.update(env)
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={world}",
+           "--master-addr=127.0.0.1", f"--master-port={free_port()}", os.path.abspath(__file__),
+           "--gpus", str(world), "--size-mib", str(args.size_mib), "--steps", str(args.steps),
+           "--warmup", str(args.warmup), "--chunk-kib", str(args.chunk_kib), *extra]
+    if args.test_same_gpu:
+        cmd.append("--test-same-gpu")
+    try:
+        p = subprocess.run(cmd, cwd=ROOT, capture_output=True, text=True, timeout=600, env=e)
+        lines = [ln for ln in p.stdout.splitlines() if ln.startswith("{")]
+        if p.returncode == 0 and lines:
+            return json.loads(lines[-1])
+        tail = p.stderr.strip().splitlines()[-1] if p.stderr.strip() else ""
+        return {"unavailable": f"{name}: rc={p.returncode}: {tail}"[:300]}
+    except Exception as ex:  # noqa: BLE001
+        return {"unavailable": f"{name}: {ex!r}"[:300]}
+
+
 def nccl_legs(args, world):
-    """Rank 0, after the main run: every NCCL variant as its own torchrun job
-    (NCCL reads NCCL_ALGO / NCCL_NVLS_ENABLE when it starts)."""
-    out = {}
-    for name, env in NCCL_LEGS.items():
-        e = dict(os.environ)
-        for k in list(e):
-            if k in ("RANK", "WORLD_SIZE", "LOCAL_RANK", "LOCAL_WORLD_SIZE", "MASTER_ADDR", "MASTER_PORT",
-                     "GROUP_RANK", "GROUP_WORLD_SIZE", "ROLE_RANK", "ROLE_WORLD_SIZE", "ROLE_NAME") or \
-                    k.startswith("TORCHELASTIC_"):
-                e.pop(k)
-        e.update(env)
-        cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={world}",
-               "--master-addr=127.0.0.1", f"--master-port={free_port()}", os.path.abspath(__file__),
-               "--gpus", str(world), "--nccl-leg", name, "--size-mib", str(args.size_mib)]
-        try:
-            p = subprocess.run(cmd, cwd=ROOT, capture_output=True, text=True, timeout=600, env=e)
-            lines = [ln for ln in p.stdout.splitlines() if ln.startswith("{")]
-            out[name] = json.loads(lines[-1]) if p.returncode == 0 and lines else \
-                {"unavailable": f"rc={p.returncode}: {p.stderr.strip().splitlines()[-1] if p.stderr.strip() else ''}"[:300]}
-        except Exception as ex:  # noqa: BLE001
-            out[name] = {"unavailable": repr(ex)[:300]}
-    return out
+    """Every NCCL variant as its own job (NCCL reads NCCL_ALGO / NCCL_NVLS_ENABLE when it starts)."""
+    return {name: leg_job(args, world, ["--nccl-leg", name], env, name) for name, env in NCCL_LEGS.items()}
+
+
+def run_nvls_leg(args):
+    """NEXT-2 NVLS leg (its own job): the nvls strategy line -- copy in,
+    multimem ld_reduce + st by the slice owners, copy out -- timed as the main
+    leg (max over ranks), then checked: every rank's output must be the same
+    bytes (SHA-256), and rank 0's output is within the any-order bound of the
+    exact sum (reading R9: |y - sum| <= ((n-1) + 1) 2^-24 sum |x| for fp32) on
+    a strided sample.  Rank 0 prints one JSON line; value None + reason when
+    the box cannot build a multicast team."""
+    import hashlib
+
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_icdcs_zhaozw24_b200 as pkg
+    from paper_conf_icdcs_zhaozw24_b200 import generator as G
+    from synth import rank_tensors
+    rank, world, local = dist_env()
+    dev = 0 if args.test_same_gpu else local
+    torch.cuda.set_device(dev)
+    if args.test_same_gpu:
+        dist.init_process_group("gloo")
+    else:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    nbytes = int(args.size_mib * (1 << 20)) // 16 * 16
+    count = nbytes // 4
+    comm = pkg.Communicator.init(scratch_bytes=64 << 20, device=dev)
+    comm.config("timeout_ms", 30000)
+    ok, why = comm.nvls_setup(2 * nbytes + (16 << 20))
+    out = {"nvls_leg": True, "value": None, "reason": why or None, "unit": UNIT}
+    if ok:
+        comm.set_strategy("allreduce", G.allreduce_nvls(world, chunk=args.chunk_kib * 1024))
+        xh = rank_tensors("f32", count, 1, base=1000 + rank)[0]
+        x = torch.from_numpy(xh).cuda()
+        y = torch.empty_like(x)
+        for _ in range(args.warmup):
+            comm.allreduce(x, y)
+        dist.barrier()
+        torch.cuda.synchronize()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record()
+        for _ in range(args.steps):
+            comm.allreduce(x, y)
+        b.record()
+        torch.cuda.synchronize()
+        dv = "cpu" if args.test_same_gpu else "cuda"
+        t = torch.tensor([a.elapsed_time(b) / args.steps], dtype=torch.float64, device=dv)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
+        y.fill_(float("nan"))
+        comm.allreduce(x, y)
+        torch.cuda.synchronize()
+        err = comm.get_async_error()
+        g = y.cpu().numpy()
+        hashes = [None] * world
+        dist.all_gather_object(hashes, hashlib.sha256(g.tobytes()).hexdigest())
+        out.update({"value": round(busbw(nbytes, ms / 1e3, world), 3), "ms_per_step": round(ms, 4),
+                    "async_error": err, "path": "nvls line: multimem ld_reduce + st (STAGED copy in / out)"})
+        if rank == 0:
+            idx = np.unique(np.concatenate([np.arange(0, count, 4099), np.arange(max(0, count - 4096), count)]))
+            xs = [rank_tensors("f32", count, 1, base=1000 + r)[0][idx].astype(np.float64) for r in range(world)]
+            exact = np.sum(xs, axis=0)
+            bound = world * 2.0 ** -24 * np.sum(np.abs(xs), axis=0)
+            bad = int(np.count_nonzero(~(np.abs(g[idx].astype(np.float64) - exact) <= bound)))
+            out["parity"] = {"complete": False, "sampled_elements": int(idx.size), "out_of_bound": bad,
+                             "ranks_identical": len(set(hashes)) == 1,
+                             "reference": "fp64 sum of every rank's seeded input (plain definition), "
+                                          "any-order fp32 bound n 2^-24 sum|x| (reading R9)"}
+    if rank == 0:
+        print(json.dumps(out), flush=True)
+    comm.finalize()
+    dist.destroy_process_group()
+    return None
 
 
 def run_multi(args):
@@ -782,17 +867,6 @@ def run_multi(args):
                     pt.update({"nccl_us": round(nms * 1e3, 2), "nccl_busbw": round(busbw(sb, nms / 1e3, world), 2)})
                 pts.append(pt)
             sweep[sdt] = pts
-    # NVLS switch reduction (NEXT-2): off by default, measured when the box can multicast
-    nvls = {"value": None, "reason": None}
-    ok_nv, why_nv = comm.nvls_setup(2 * nbytes + (16 << 20))
-    if ok_nv:
-        comm.set_strategy("allreduce", G.allreduce_nvls(world, chunk=args.chunk_kib * 1024))
-        ms_nv = timed(lambda: comm.allreduce(x, y), args.steps)
-        nvls.update({"value": round(busbw(nbytes, ms_nv / 1e3, world), 3), "unit": UNIT,
-                     "ms_per_step": round(ms_nv, 4), "path": "nvls line: multimem ld_reduce + st (STAGED copy in/out)"})
-        comm.set_strategy("allreduce", text)
-    else:
-        nvls["reason"] = why_nv
     parity = None if args.no_parity else multi_complete_parity(comm, x, y, text, world, rank, count, args.dtype)
     st = pkg.adapcc.plan_stats(text, count, args.dtype, (1 << world) - 1, rank=rank)
     peak_dir = probes["sm"]["one_to_one_GBps"]
@@ -828,7 +902,7 @@ def run_multi(args):
                          "zero-copy AllReduce, nccl = dist.all_reduce on the same sizes; back-to-back "
                          "enqueue (us; NCCL likewise) and, ours only, a CUDA graph (us_graph); max over ranks",
             "path": "zero-copy DIRECT plan over CUDA IPC (registered buffers)",
-            "p2p_ceiling": probes, "nvls": nvls, "paper_context": PAPER_CONTEXT,
+            "p2p_ceiling": probes, "nvls": None, "paper_context": PAPER_CONTEXT,
             "staged": {"value": round(busbw(nbytes, ms_staged / 1e3, world), 3), "unit": UNIT,
                        "ms_per_step": round(ms_staged, 4),
                        "path": "STAGED protocol (landing + broadcast slots in IPC arenas)"},
@@ -837,10 +911,14 @@ def run_multi(args):
         }
     comm.finalize()
     dist.destroy_process_group()
-    if rank == 0 and not args.test_same_gpu and not args.no_nccl_legs:
+    if rank == 0:
         del x, y, z, x2, y2
         torch.cuda.empty_cache()
-        res["nccl_legs"] = nccl_legs(args, world)
+        # NVLS (NEXT-2) in its own job: the multimem path has not run on a multicast-capable box
+        # before, so a failure there cannot take this line with it
+        res["nvls"] = leg_job(args, world, ["--nvls-leg"], {}, "nvls")
+        if not args.test_same_gpu and not args.no_nccl_legs:
+            res["nccl_legs"] = nccl_legs(args, world)
     return res
 
 
@@ -881,6 +959,8 @@ def main():
         return 2
     if args.nccl_leg:
         out = run_nccl_leg(args)
+    elif args.nvls_leg:
+        out = run_nvls_leg(args)
     elif args.impl == "reference":
         out = run_reference(args)        # CPU only: no launcher needed, rank 0 prints
     elif args.gpus > 1 and "WORLD_SIZE" not in os.environ:
