@@ -53,7 +53,9 @@ def parse_args():
     p.add_argument("--dtype", choices=["f32", "bf16"], default="f32")
     p.add_argument("--mode", choices=["direct", "staged"], default="direct")
     p.add_argument("--chunk-kib", type=int, default=256)
-    p.add_argument("--e2e-steps", type=int, default=8)
+    p.add_argument("--e2e-steps", type=int, default=16,
+                   help="e2e steps: the first upload and the last download do not overlap, so K steps "
+                        "reach at most K/(K+1) of the full-duplex PCIe bound")
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--no-parity", action="store_true")
     p.add_argument("--no-sweep", action="store_true", help="skip the busbw-vs-size sweep")
@@ -421,7 +423,8 @@ def run_single(args):
                        "double-buffered with H2D and D2H on separate copy streams (full-duplex PCIe)",
                 "pcie_bidir_GBps_per_direction": round(pcie, 1),
                 "pcie_bound_ms_per_step": round(pcie_ms, 3),
-                "pcie_roofline_frac": round(pcie_ms / e2e_t, 4)},
+                "pcie_roofline_frac": round(pcie_ms / e2e_t, 4),
+                "pipeline_bound_frac": round(args.e2e_steps / (args.e2e_steps + 1), 4)},
         "gpu_launches": launches,
         "clocks": clk.summary(),
         "parity": parity,

@@ -329,6 +329,40 @@ ADAPCC_API adapcc_result_t adapcc_ready_board(adapcc_comm_t comm, volatile uint6
  * "computation" that occupies one SM slot, not the GPU). */
 ADAPCC_API adapcc_result_t adapcc_spin(adapcc_comm_t comm, uint64_t ns, adapcc_stream_t stream);
 
+/* Online coordinator, native decision loops (NEXT-1 / NEXT-3; host only, no
+ * device work, callable without a GPU).  `board` is the page
+ * adapcc_ready_board returns (or any >= 64-word array laid out the same way:
+ * word r = the ticket rank r last signalled).  Times are CLOCK_MONOTONIC
+ * seconds (the clock of Python's time.perf_counter on Linux).  Both loops
+ * spin on plain host loads and return without touching the communicator, so
+ * a binding may call them with its interpreter lock released.
+ *
+ * adapcc_coord_decide -- the break-even (ski-rental) rule of P:L133-137 on
+ * real readiness.  Every cycle_s it reads which ranks in `members` have
+ * signalled `ticket`: all of them -> *full = 1, *ready_mask = members; else,
+ * with k >= 1 ready, if the time already waited (cycles x cycle_s) plus one
+ * more cycle exceeds buy_cost[k] (the estimated phase-1 + phase-2 time with k
+ * ready ranks; array of nranks + 1 doubles) -> *full = 0,
+ * *ready_mask = the ready ranks (phase 1); else wait one more cycle.
+ * *t_first = when the first rank was seen ready (T_fault's origin),
+ * *t_decide = when the decision was taken.  Errors: INVALID_ARGUMENT,
+ * TIMEOUT (nobody ready within timeout_s).
+ *
+ * adapcc_coord_await -- after phase 1 was enqueued: wait until every rank in
+ * late_mask has signalled `ticket` (*faulty = 0: run phase 2) or, with
+ * fault_factor > 0, until T_fault = fault_factor x (phase-1 end - t_first)
+ * has passed since phase 1 ended (*faulty = the late ranks still not ready,
+ * P:L139).  Phase 1's end is when `phase1_event` (a cudaEvent_t recorded after
+ * it; NULL = already ended) first reports complete.  Errors:
+ * INVALID_ARGUMENT, CUDA (event query failed), TIMEOUT (timeout_s passed). */
+ADAPCC_API adapcc_result_t adapcc_coord_decide(const volatile uint64_t* board, int nranks, uint64_t members,
+                                               uint64_t ticket, const double* buy_cost, double cycle_s,
+                                               double timeout_s, uint64_t* ready_mask, int* full,
+                                               double* t_first, double* t_decide);
+ADAPCC_API adapcc_result_t adapcc_coord_await(const volatile uint64_t* board, int nranks, uint64_t late_mask,
+                                              uint64_t ticket, void* phase1_event, double t_first,
+                                              double fault_factor, double timeout_s, uint64_t* faulty);
+
 /* ------------------------------------------------------------- lifecycle --- */
 
 /* Latched device error (TIMEOUT) or SUCCESS.  Does not synchronize. */

@@ -96,6 +96,11 @@ def _load():
         "adapcc_signal_ready": [vp, i32, u64, vp],
         "adapcc_ready_board": [vp, ctypes.POINTER(ctypes.c_void_p), ctypes.POINTER(i32)],
         "adapcc_spin": [vp, u64, vp],
+        "adapcc_coord_decide": [vp, i32, u64, u64, ctypes.POINTER(ctypes.c_double), ctypes.c_double,
+                                ctypes.c_double, ctypes.POINTER(u64), ctypes.POINTER(i32),
+                                ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_double)],
+        "adapcc_coord_await": [vp, i32, u64, u64, vp, ctypes.c_double, ctypes.c_double, ctypes.c_double,
+                               ctypes.POINTER(u64)],
         "adapcc_get_async_error": [vp],
         "adapcc_finalize": [vp],
         "adapcc_config": [vp, ctypes.c_char_p, i64],
@@ -320,6 +325,37 @@ def make_store_allgather(ranks, rank, store=None, tag="adapcc"):
             return 1
 
     return AG_FN(ag)
+
+
+def coord_decide(board, nranks, members, ticket, buy_cost, cycle, timeout):
+    """adapcc_coord_decide (native break-even loop; runs without
+    the GIL).  board: address of the readiness board; members: rank set;
+    buy_cost: nranks + 1 seconds.  Returns (full, ready set, t_first,
+    t_decide) on the time.perf_counter clock; TimeoutError if nobody is ready."""
+    costs = (ctypes.c_double * (nranks + 1))(*buy_cost)
+    mask, full = ctypes.c_uint64(), ctypes.c_int()
+    t_first, t_decide = ctypes.c_double(), ctypes.c_double()
+    code = _load().adapcc_coord_decide(board, nranks, _mask(members, nranks), ticket, costs, cycle, timeout,
+                                       ctypes.byref(mask), ctypes.byref(full), ctypes.byref(t_first),
+                                       ctypes.byref(t_decide))
+    if code == TIMEOUT:
+        raise TimeoutError("no worker became ready")
+    _check(code, "coord_decide")
+    return bool(full.value), {r for r in range(nranks) if (mask.value >> r) & 1}, t_first.value, t_decide.value
+
+
+def coord_await(board, nranks, late, ticket, phase1_event, t_first, fault_factor, timeout):
+    """adapcc_coord_await (native, P:L131 / P:L139): the set of late ranks
+    judged faulty (empty: all signalled, run phase 2).  phase1_event: a raw
+    cudaEvent_t handle or None."""
+    faulty = ctypes.c_uint64()
+    code = _load().adapcc_coord_await(board, nranks, _mask(late, nranks), ticket, phase1_event,
+                                      -1.0 if t_first is None else t_first, fault_factor or 0.0, timeout,
+                                      ctypes.byref(faulty))
+    if code == TIMEOUT:
+        raise TimeoutError("late ranks never became ready (fault: set fault_factor or see exclude_faulty)")
+    _check(code, "coord_await")
+    return {r for r in range(nranks) if (faulty.value >> r) & 1}
 
 
 class PreparedCall:

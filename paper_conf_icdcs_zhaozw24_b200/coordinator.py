@@ -175,6 +175,7 @@ class ReadyBoard:
     def __init__(self, comm):
         import ctypes
         addr, self.shared = comm.ready_board()
+        self.addr = addr
         self.n = comm.nranks
         self.words = (ctypes.c_uint64 * 128).from_address(addr)
 
@@ -218,7 +219,8 @@ class OnlineCoordinator:
 
     Every decision cycle the leader (rank 0, or the loopback process) reads
     the readiness board -- which ranks signalled this collective's ticket --
-    and applies the break-even rule (Coordinator.step); it publishes "full"
+    and applies the break-even rule (the native loop adapcc_coord_decide, with
+    the policy's buy_cost per ready count); it publishes "full"
     (everyone ready) or "phase1" (ready ranks aggregate, the others relay) on
     the board, and every rank issues the same LATE_JOIN call with that mask
     (late ranks' chunks still join the ongoing aggregation chunk by chunk,
@@ -233,11 +235,14 @@ class OnlineCoordinator:
     sources, phase 2 = the late ones; P:L135 prices them with the policy's
     `coll`).  Ranks signal readiness with comm.signal_ready(ticket=
     coordinator.ticket()) after their computation (the ticket of the
-    collective the coordinator runs next).  policy: a Coordinator (fresh per
-    call: its waited time accumulates); cycle: seconds between decisions
-    (the paper's 5 ms, scaled to the collective's time scale, reading R2)."""
+    collective the coordinator runs next).  policy_factory() returns a
+    Coordinator (its buy_cost(k) table drives the decision); cycle: seconds
+    between decisions (the paper's 5 ms, scaled to the collective's time
+    scale, reading R2).  The waiting loops are native (adapcc_coord_decide /
+    adapcc_coord_await: plain host loads of the board, no interpreter lock
+    held) and time with CLOCK_MONOTONIC, the clock of time.perf_counter."""
 
-    def __init__(self, comm, policy_factory, cycle=5e-6, timeout=30.0, clock=None, fault_factor=None,
+    def __init__(self, comm, policy_factory, cycle=5e-6, timeout=30.0, fault_factor=None,
                  store=None, stream=None):
         """fault_factor: apply the T_fault rule -- late ranks not
         ready fault_factor x (phase-1 end - first ready) after phase 1 ended
@@ -254,7 +259,7 @@ class OnlineCoordinator:
         self.policy_factory = policy_factory
         self.cycle = cycle
         self.timeout = timeout
-        self.clock = clock or time.perf_counter
+        self.clock = time.perf_counter
         self.seq = 0
         self.leader = comm.loopback or comm.rank == 0
         if not comm.loopback and comm.nranks > 1 and not self.board.shared:
@@ -273,26 +278,17 @@ class OnlineCoordinator:
         t0 = clock()
         t_first = None
         if self.leader:
+            from . import adapcc as A
             policy = self.policy_factory()
             if len(members) < n and hasattr(policy, "n"):
                 policy.n = len(members)        # the policy prices the survivors' collective
-            nxt = t0
-            while True:
-                ready = self.board.ready(t) & members
-                if ready and t_first is None:
-                    t_first = clock()          # the fastest worker became ready (T_fault's origin)
-                d = policy.step(clock() - t0, ready)
-                if d.action != "wait":
-                    break
-                if clock() - t0 > self.timeout:
-                    raise TimeoutError("no worker became ready")
-                nxt += self.cycle
-                while clock() < nxt:
-                    pass
-            mask = all_mask if d.action == "full" else sum(1 << r for r in d.ready)
+            costs = [float("inf")] + [policy.buy_cost(k) for k in range(1, n + 1)]
+            full, ready, t_first, _ = A.coord_decide(self.board.addr, n, members, t, costs, self.cycle,
+                                                     self.timeout)
+            action = "full" if full else "phase1"
+            mask = all_mask if full else sum(1 << r for r in ready)
             if not self.comm.loopback:
-                self.board.publish(self.seq, d.action, mask)
-            action = d.action
+                self.board.publish(self.seq, action, mask)
         else:
             action, mask = self.board.wait_decision(self.seq, self.timeout, clock)
         t_decide = clock()
@@ -324,26 +320,16 @@ class OnlineCoordinator:
         """Leader: wait until every late rank signalled (-> 0) or, with a
         fault_factor, until T_fault after phase 1 passes (-> the mask of the
         late ranks still not ready); publish it.  Followers: read it."""
-        clock, n = self.clock, self.comm.nranks
+        from . import adapcc as A
+        n = self.comm.nranks
         self.seq2 = getattr(self, "seq2", 0) + 1
         if not self.leader:
-            return self.board.wait_phase2(self.seq2, self.timeout, clock)
-        p1_done = self._p1_done
-        t_p1 = None
-        faulty = 0
-        while True:
-            missing = [r for r in range(n) if (late >> r) & 1 and self.board.words[r] < t]
-            if not missing:
-                break
-            now = clock()
-            if t_p1 is None and (p1_done is None or p1_done.query()):
-                t_p1 = now                     # phase 1 finished on this GPU
-            if self.fault_factor is not None and t_p1 is not None and t_first is not None and \
-                    now - t_p1 >= self.fault_factor * (t_p1 - t_first):
-                faulty = sum(1 << r for r in missing)
-                break
-            if now - t0 > self.timeout:
-                raise TimeoutError("late ranks never became ready (fault: set fault_factor or see exclude_faulty)")
+            return self.board.wait_phase2(self.seq2, self.timeout, self.clock)
+        ev = self._p1_done
+        dead = A.coord_await(self.board.addr, n, {r for r in range(n) if (late >> r) & 1}, t,
+                             None if ev is None else ev.cuda_event, t_first, self.fault_factor,
+                             max(self.timeout - (self.clock() - t0), 0.0))
+        faulty = sum(1 << r for r in dead)
         if not self.comm.loopback:
             self.board.publish_phase2(self.seq2, faulty)
         return faulty

@@ -20,6 +20,7 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <ctime>
 #include <list>
 #include <map>
 #include <memory>
@@ -1573,6 +1574,85 @@ adapcc_result_t adapcc_spin(adapcc_comm_t c, uint64_t ns, adapcc_stream_t stream
   CK(cudaSetDevice(c->device));
   CK(engine_spin(ns, reinterpret_cast<cudaStream_t>(stream)));
   return ADAPCC_SUCCESS;
+}
+
+// ---- online coordinator loops (host only): P:L133-137 break-even rule, P:L139 T_fault
+static double mono_now() {
+  timespec ts;
+  clock_gettime(CLOCK_MONOTONIC, &ts);
+  return (double)ts.tv_sec + 1e-9 * (double)ts.tv_nsec;
+}
+static uint64_t board_ready(const volatile uint64_t* board, int n, uint64_t among, uint64_t ticket) {
+  uint64_t m = 0;
+  for (int r = 0; r < n; ++r)
+    if (((among >> r) & 1) && board[r] >= ticket) m |= uint64_t(1) << r;
+  return m;
+}
+
+adapcc_result_t adapcc_coord_decide(const volatile uint64_t* board, int nranks, uint64_t members, uint64_t ticket,
+                                    const double* buy_cost, double cycle_s, double timeout_s, uint64_t* ready_mask,
+                                    int* full, double* t_first, double* t_decide) {
+  if (!board || !buy_cost || !ready_mask || !full || nranks < 1 || nranks > 64 || !members || cycle_s < 0)
+    return ADAPCC_ERR_INVALID_ARGUMENT;
+  const uint64_t all = nranks == 64 ? ~uint64_t(0) : ((uint64_t(1) << nranks) - 1);
+  if (members & ~all) return ADAPCC_ERR_INVALID_ARGUMENT;
+  const double t0 = mono_now();
+  double first = -1.0, waited = 0.0, next = t0;
+  for (;;) {
+    const uint64_t ready = board_ready(board, nranks, members, ticket);
+    const double now = mono_now();
+    if (ready && first < 0) first = now;
+    if (ready == members) {
+      *full = 1;
+      *ready_mask = members;
+      break;
+    }
+    if (ready && waited + cycle_s > buy_cost[__builtin_popcountll(ready)]) {  // buying beats one more cycle
+      *full = 0;
+      *ready_mask = ready;
+      break;
+    }
+    if (now - t0 > timeout_s) return ADAPCC_ERR_TIMEOUT;
+    waited += cycle_s;
+    next += cycle_s;
+    while (mono_now() < next) {
+    }
+  }
+  if (t_first) *t_first = first;
+  if (t_decide) *t_decide = mono_now();
+  return ADAPCC_SUCCESS;
+}
+
+adapcc_result_t adapcc_coord_await(const volatile uint64_t* board, int nranks, uint64_t late_mask, uint64_t ticket,
+                                   void* phase1_event, double t_first, double fault_factor, double timeout_s,
+                                   uint64_t* faulty) {
+  if (!board || !faulty || nranks < 1 || nranks > 64) return ADAPCC_ERR_INVALID_ARGUMENT;
+  const double t0 = mono_now();
+  double t_p1 = -1.0;
+  *faulty = 0;
+  for (;;) {
+    const uint64_t missing = late_mask & ~board_ready(board, nranks, late_mask, ticket);
+    if (!missing) return ADAPCC_SUCCESS;
+    const double now = mono_now();
+    if (t_p1 < 0) {
+      if (!phase1_event) {
+        t_p1 = now;
+      } else {
+        const cudaError_t q = cudaEventQuery(reinterpret_cast<cudaEvent_t>(phase1_event));
+        if (q == cudaSuccess) t_p1 = now;  // phase 1 finished on this GPU
+        else if (q != cudaErrorNotReady) {
+          g_last_cuda_error = q;
+          g_last_cuda_line = __LINE__;
+          return ADAPCC_ERR_CUDA;
+        }
+      }
+    }
+    if (fault_factor > 0 && t_p1 >= 0 && t_first >= 0 && now - t_p1 >= fault_factor * (t_p1 - t_first)) {
+      *faulty = missing;
+      return ADAPCC_SUCCESS;
+    }
+    if (now - t0 > timeout_s) return ADAPCC_ERR_TIMEOUT;
+  }
 }
 
 const char* adapcc_last_cuda_error(void) {

@@ -220,6 +220,7 @@ def test_coordinator_fault_rule_excludes_silent_rank(mode):
     for it, lag_us in enumerate((0, 300)):
         for g in live:
             dy[g].zero_()
+        torch.cuda.synchronize()            # (the collectives run on cs)
         t = coord.ticket()
         for r in live - {2}:
             comm.signal_ready(r, ticket=t, stream=cs)
@@ -270,6 +271,7 @@ def _fault_worker(rank, n, port, q):
             ok.append(np.array_equal(to_host(y, "i32"), exp))
             for _ in range(2):                # the survivors carry on: a full round
                 y.zero_()
+                torch.cuda.synchronize()      # (the collectives run on cs)
                 t = coord.ticket()
                 comm.signal_ready(ticket=t, stream=cs)
                 res = coord.allreduce(lambda m, lt: comm.allreduce(x, y, ready=m, late=lt, stream=cs))
