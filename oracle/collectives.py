@@ -351,7 +351,7 @@ def _root_terms(vals, sub, ready, dtype):
     return [value(f) for f in flows[root]]
 
 
-def allreduce_late(xs, strategy_text, ready, dtype, included, phase=1, y_prev=None):
+def allreduce_late(xs, strategy_text, ready, dtype, included, phase=1, y_prev=None, members=None):
     """Late join with a uniform inclusion set.
 
     phase 1: every tree's root folds its regular terms followed by the inputs
@@ -360,11 +360,14 @@ def allreduce_late(xs, strategy_text, ready, dtype, included, phase=1, y_prev=No
     phase 2: y_prev + fold(inputs of the late ranks NOT in ``included``,
              ascending), one rounding for the sum and one for the addition
              (the ACCUMULATE rule); nothing left -> y_prev unchanged.
-    Late ranks = ranks not in ``ready``; ``included`` must be a subset."""
+    Late ranks = ranks not in ``ready``; ``included`` must be a subset.
+    members: the live ranks after a fault exclusion (faulty
+    workers leave the group) -- excluded ranks are never late and never
+    contribute; None = every rank."""
     st = parse(strategy_text)
     n = st.nranks
     ready = set(ready)
-    late = sorted(set(range(n)) - ready)
+    late = sorted((set(range(n)) if members is None else set(members)) - ready)
     included = sorted(set(included))
     assert set(included) <= set(late)
     lens = {len(x) for x in xs if x is not None}

@@ -54,3 +54,24 @@ def test_non_kernel_root_with_late_input_is_rounded_once_bf16():
     y = oc.allreduce_late(xs, S.allreduce_trees([S.star(3, 0)], chunk=16), {1}, "bf16", {2})
     # 1 + 2^-8 is a tie in bf16 -> even -> 1.0
     assert int(y[0][0]) == 0x3f80
+
+
+def test_excluded_ranks_are_never_late_int32():
+    """members (after a fault exclusion): phase 1 + phase 2 is
+    the exact sum over the members only, for every inclusion set, and the
+    excluded rank's input (poisoned here) never enters."""
+    n, count = 6, 211
+    xs = rank_tensors("i32", count, n)
+    dead = 4
+    xs[dead] = np.full(count, 1 << 20, np.int32)
+    members = set(range(n)) - {dead}
+    R = {0, 3, 5}
+    for text in (S.allreduce_stars(n, chunk=64), S.allreduce_trees([S.star(n, 0)], chunk=32)):
+        for L in _subsets([1, 2]):
+            y1 = oc.allreduce_late(xs, text, R, "i32", L, phase=1, members=members)
+            y2 = oc.allreduce_late(xs, text, R, "i32", L, phase=2, y_prev=y1, members=members)
+            want = sum(xs[g].astype(np.int64) for g in members).astype(np.int32)
+            assert all(np.array_equal(y, want) for y in y2)
+            if L == set():
+                y2n = oc.allreduce_late(xs, text, R, "i32", L, phase=2, y_prev=y1)
+                assert not np.array_equal(y2n[0], want)     # without members the dead rank would be added
