@@ -12,7 +12,7 @@ ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 LIB = os.path.join(PKG, "libadapcc.so")
 SOURCES = ["adapcc.cpp", "strategy.cpp", "plan.cpp", "engine.cu", "engine_tma_direct.cu",
-           "engine_tma_staged.cu", "probe.cu"]
+           "engine_tma_staged.cu", "engine_flat.cu", "probe.cu"]
 HEADERS = ["engine.cuh", "engine_common.cuh", "engine_tma_impl.cuh", "launch.hpp", "plan.hpp",
            "strategy.hpp"]
 

@@ -48,6 +48,8 @@ struct DevSegment {
   FlagRef* flags = nullptr;
   Item* items = nullptr;
   uint32_t nitems = 0;
+  uint32_t ntasks = 0;
+  uint64_t flat_vecs = 0;         // flat kernel: 16-byte vectors of the tasks this rank runs
   uint64_t* late_bits = nullptr;  // per item: late ranks folded in phase 1 (late join)
   uint32_t* late_list = nullptr;  // nitems: items phase 1 left incomplete
   unsigned long long* late_count = nullptr;  // (gen << 32 | count), epoch of the last phase 1 (launch.hpp)
@@ -58,8 +60,8 @@ struct DevSegment {
 };
 
 struct DevPlan {
-  int engine = 0;      // 0: LDG fold kernel, 1: TMA pipeline
-  int kernel = 0;      // 0: LDG, 1: TMA for DIRECT plans, 2: TMA for STAGED plans
+  int engine = 0;      // 0: LDG fold kernel, 1: TMA pipeline, 3: flat (one CTA per item)
+  int kernel = 0;      // 0: LDG, 1: TMA for DIRECT plans, 2: TMA for STAGED plans, 3: flat
   std::vector<DevSegment> segs;
   bool launched = false;  // enqueued at least once: freeing the tables waits for the device
   uint64_t last_tick = 0;
@@ -182,12 +184,13 @@ struct adapcc_comm_s {
   int64_t acc_red = 1;    // TMA kernel: recv += result by bulk reduce-add in L2 (ADAPCC_ACC_RED)
   int64_t default_chunk = 262144;  // C_m of the default strategies (a link profile may set it)
   int64_t sched = 2;      // LDG kernel: 0 dynamic claims, 1 static blob schedule, 2 auto (ADAPCC_SCHED)
+  int64_t flat_ctas = 2;  // flat kernel: CTAs per SM of its grid (2 resident; more = several waves) (ADAPCC_FLAT_CTAS)
   uint64_t launches = 0;
   int num_sms = 148;
   // [kernel][dtype] resident CTAs per SM; kernels: 0 LDG fold, 1 TMA (DIRECT
   // plans), 2 TMA (STAGED plans)
   int occ[3][3] = {{1, 1, 1}, {1, 1, 1}, {1, 1, 1}};
-  int engine = 2;  // 0: LDG/STG fold, 1: TMA bulk pipeline, 2: auto by call size
+  int engine = 2;  // 0: LDG/STG fold, 1: TMA bulk pipeline, 2: auto by call size, 3: flat (flag-free plans)
   int last_engine = -1;  // kernel used by the most recent launch
   std::mutex mu;
   adapcc_bootstrap_allgather_fn ag = nullptr;  // kept for collective registration
@@ -241,7 +244,8 @@ adapcc_result_t common_init(adapcc_comm_s* c, size_t scratch) {
   c->arena_bytes = kArenaHeader + 2 * c->half_bytes;
   c->timeout_ms = env_int("ADAPCC_TIMEOUT_MS", 10000);
   c->max_ctas = env_int("ADAPCC_NCTAS", 0);
-  c->engine = (int)std::min<int64_t>(2, std::max<int64_t>(0, env_int("ADAPCC_ENGINE", 2)));
+  c->engine = (int)std::min<int64_t>(3, std::max<int64_t>(0, env_int("ADAPCC_ENGINE", 2)));
+  c->flat_ctas = std::min<int64_t>(64, std::max<int64_t>(1, env_int("ADAPCC_FLAT_CTAS", 2)));
   c->piece_kib = env_int("ADAPCC_PIECE_KIB", 0);
   c->taper = std::min<int64_t>(64, std::max<int64_t>(0, env_int("ADAPCC_TAPER", 0)));
   c->check_sig = env_int("ADAPCC_DEBUG", 0) != 0;
@@ -487,10 +491,38 @@ adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, const Strategy* strat, uin
       if (sp.nvls) plan->engine = 0;
     plan->kernel = plan->engine == 0 ? 0 : (mode == kDirect && (!rq.accumulate || c->acc_red) ? 1 : 2);
     if (plan->kernel != 0 && (c->tma_shape == 1 || c->tma_shape == 2)) plan->kernel = (int)c->tma_shape;
+    // flat kernel (engine_flat.cu): plans whose items are independent -- no
+    // flag waits or posts, no arena streams, no late join, no NVLS
+    bool flat_ok = !rq.late_join;
+    for (auto& sp : segs) {
+      if (sp.nvls) flat_ok = false;
+      for (const Task& t : sp.tasks) {
+        if (t.nwait || t.npost || t.nlate || (t.op != kOpFold && t.op != kOpZero)) flat_ok = false;
+        for (uint32_t k = 0; k < (uint32_t)t.nsrc + t.ndst; ++k)
+          if (sp.refs[t.ref0 + k].kind != kBufSend && sp.refs[t.ref0 + k].kind != kBufRecv) flat_ok = false;
+      }
+    }
+    for (auto& sp : segs) {  // the descriptor blob must fit the kernel's shared memory
+      uint32_t nt = 0, nr = 0;
+      for (const Task& t : sp.tasks)
+        if (c->loopback || t.owner == c->rank) {
+          ++nt;
+          nr += (uint32_t)t.nsrc + t.ndst;
+        }
+      if (nt > kFlatMaxTasks || nr > kFlatMaxRefs) flat_ok = false;
+    }
+    // auto: small ACCUMULATE calls (phase 2 of small buckets) take the flat
+    // kernel -- the persistent LDG kernel pays one memory round trip per
+    // accumulating destination (1 MiB per rank, 2 of 8 ready: 7.2 -> 5.8 us,
+    // profiles/flat_r02.json); everything larger stays on the TMA pipeline
+    const bool flat_auto = c->engine == 2 && rq.accumulate && plan->engine == 0;
+    if (flat_ok && (c->engine == 3 || flat_auto)) plan->engine = plan->kernel = 3;
   }
   for (auto& sp : segs) {
     DevSegment d;
-    std::vector<Item> items = order_items(sp, c->loopback ? -1 : c->rank, rq.esize, grid_size(c, dtype, plan->kernel),
+    // (the flat kernel runs tasks, not items: the items only count the work)
+    const bool flat = plan->kernel == 3;
+    std::vector<Item> items = order_items(sp, c->loopback ? -1 : c->rank, rq.esize, grid_size(c, dtype, flat ? 0 : plan->kernel),
                                           (uint64_t)c->piece_kib * 1024, (int)c->taper, plan->kernel != 0);
     d.nitems = (uint32_t)items.size();
     d.arena_free = 1;
@@ -510,7 +542,38 @@ adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, const Strategy* strat, uin
     CK(up(&d.refs, sp.refs));
     CK(up(&d.flags, sp.flags));
     CK(up(&d.items, items));
-    if (c->first_blob) {
+    if (flat) {
+      // descriptor blob (engine.cuh FlatTask): the tasks this rank runs, then their refs
+      std::vector<FlatTask> ft;
+      std::vector<BufRef> fr;
+      for (const Task& t : sp.tasks) {
+        if (!(c->loopback || t.owner == c->rank)) continue;
+        FlatTask f{};
+        f.len = t.hi - t.lo;
+        f.ref0 = (uint32_t)fr.size();
+        f.nsrc = t.nsrc;
+        f.ndst = t.ndst;
+        f.op = t.op;
+        f.owner = t.owner;
+        for (uint32_t k = 0; k < (uint32_t)t.nsrc + t.ndst; ++k) {
+          BufRef r = sp.refs[t.ref0 + k];
+          r.bias += (int64_t)(t.lo * rq.esize);
+          r.pad[0] = (uint8_t)(ft.size() & 255);
+          r.pad[1] = (uint8_t)(ft.size() >> 8);
+          if (k >= t.nsrc && r.accum) f.any_acc = 1;
+          fr.push_back(r);
+        }
+        d.flat_vecs += f.len * rq.esize / 16 + 1;
+        ft.push_back(f);
+      }
+      std::vector<uint4> blob(2 * ft.size() + fr.size());
+      if (!ft.empty()) std::memcpy(blob.data(), ft.data(), ft.size() * sizeof(FlatTask));
+      if (!fr.empty()) std::memcpy(blob.data() + 2 * ft.size(), fr.data(), fr.size() * sizeof(BufRef));
+      CK(up(&d.first, blob));
+      d.ntasks = (uint32_t)ft.size();
+      d.first_words = (uint32_t)blob.size();
+    }
+    if (c->first_blob && !flat) {
       // Item blobs (launch.hpp): item i, its task and the task's refs in one
       // run of 16-byte words.  Static schedule: every item gets one, CTA b runs
       // items b, b + grid, ... and prefetches the next blob while it folds (no
@@ -610,6 +673,7 @@ adapcc_result_t run(adapcc_comm_s* c, Coll coll, const void* const* send, void* 
     P.flags = seg.flags;
     P.items = seg.items;
     P.nitems = seg.nitems;
+    P.ntasks = seg.ntasks;
     P.first = seg.first;
     P.nfirst = seg.nfirst;
     P.first_words = seg.first_words;
@@ -657,10 +721,14 @@ adapcc_result_t run(adapcc_comm_s* c, Coll coll, const void* const* send, void* 
     // acc_red it takes the ACCUMULATE shape (2 x 3 x 32 KiB) whatever the
     // plan's kernel; item order is grid-independent, so the plan is shared
     const int kernel = (late_mode == 2 && plan->kernel == 1 && !c->acc_red && c->tma_shape != 1) ? 2 : plan->kernel;
-    const int grid = std::max(1, std::min<int>(grid_size(c, dtype, kernel), (int)std::max<uint32_t>(1, seg.nitems)));
+    // flat: flat_ctas CTAs per SM, fewer if the call has fewer vectors than the grid has threads
+    const int grid = kernel == 3 ? (int)std::max<uint64_t>(1, std::min<uint64_t>((uint64_t)c->num_sms * c->flat_ctas,
+                                                                                   (seg.flat_vecs + 255) / 256))
+                                 : std::max(1, std::min<int>(grid_size(c, dtype, kernel), (int)std::max<uint32_t>(1, seg.nitems)));
     const bool pdl = c->pdl != 0;
     CK(kernel == 1 ? tma_direct::launch(P, grid, s, pdl)
-       : kernel == 2 ? tma_staged::launch(P, grid, s, pdl) : engine_launch(P, grid, s, pdl));
+       : kernel == 2 ? tma_staged::launch(P, grid, s, pdl)
+       : kernel == 3 ? flat::launch(P, grid, s, pdl) : engine_launch(P, grid, s, pdl));
     c->last_engine = plan->engine;
     ++c->launches;
   }
@@ -1748,9 +1816,13 @@ adapcc_result_t adapcc_config(adapcc_comm_t c, const char* key, int64_t value) {
     c->max_ctas = value;
   }
   else if (!std::strcmp(key, "engine")) {
-    if (value < 0 || value > 2) return ADAPCC_ERR_INVALID_ARGUMENT;
+    if (value < 0 || value > 3) return ADAPCC_ERR_INVALID_ARGUMENT;
     if (value != c->engine) drop_plans(c);  // pieces are sized for the engine's grid
     c->engine = (int)value;
+  }
+  else if (!std::strcmp(key, "flat_ctas")) {
+    if (value < 1 || value > 64) return ADAPCC_ERR_INVALID_ARGUMENT;
+    c->flat_ctas = value;  // (launch-time: no plan depends on it)
   }
   else if (!std::strcmp(key, "piece_kib") || !std::strcmp(key, "taper")) {
     if (value < 0 || (key[0] == 't' && value > 64)) return ADAPCC_ERR_INVALID_ARGUMENT;

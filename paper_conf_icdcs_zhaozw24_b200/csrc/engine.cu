@@ -171,6 +171,57 @@ __device__ __forceinline__ void fold_vec(const Shared& sh, int nsrc, int ndst, u
   }
 }
 
+// Items with accumulating destinations (phase 2, recv += result): one vector
+// per thread per round; the sources are folded KB at a time as in fold_vec,
+// then the recv vectors of DB destinations are loaded together before their
+// adds and stores -- one memory round trip per DB destinations instead of one
+// per destination (write_dsts), 8 loads in flight per thread.  Same
+// arithmetic: fold rounded once, then recv + result rounded once.
+template <int DT, int KB, int DB>
+__device__ __forceinline__ void fold_acc_vec(const Shared& sh, int nsrc, int ndst, uint32_t nvec) {
+  using O = Ops<DT>;
+  for (uint32_t v = threadIdx.x; v < nvec; v += kThreads) {
+    const size_t off = (size_t)v * 16;
+    uint4 r;
+    if (nsrc == 1) {
+      r = ld16(sh.src[0] + off);
+    } else {
+      typename O::Acc a;
+      for (int k0 = 0; k0 < nsrc; k0 += KB) {
+        uint4 x[KB];
+#pragma unroll
+        for (int j = 0; j < KB; ++j)
+          if (k0 + j < nsrc) x[j] = ld16(sh.src[k0 + j] + off);
+#pragma unroll
+        for (int j = 0; j < KB; ++j) {
+          if (k0 + j >= nsrc) break;
+          if (k0 + j == 0) a = O::widen(x[0]);
+          else O::add(a, x[j]);
+        }
+      }
+      r = O::narrow(a);  // one rounding per task
+    }
+    for (int d0 = 0; d0 < ndst; d0 += DB) {
+      uint4 q[DB];
+#pragma unroll
+      for (int j = 0; j < DB; ++j)
+        if (d0 + j < ndst && sh.acc[d0 + j]) q[j] = ld16(sh.dst[d0 + j] + off);
+#pragma unroll
+      for (int j = 0; j < DB; ++j) {
+        if (d0 + j >= ndst) break;
+        char* p = sh.dst[d0 + j] + off;
+        if (sh.acc[d0 + j]) {
+          typename O::Acc b = O::widen(q[j]);
+          O::add(b, r);
+          st16(p, O::narrow(b));
+        } else {
+          st16(p, r);
+        }
+      }
+    }
+  }
+}
+
 // NVLS (NEXT-2 switch reduction): every 16-byte vector of the multicast
 // source is summed over all ranks' copies by the NVSwitch (multimem
 // ld_reduce; fp32 adds in the switch's order, bf16 accumulated in fp32 and
@@ -275,7 +326,8 @@ __device__ void fold_chunk(const Shared& sh, int nsrc, int ndst, uint64_t n, int
   const uint32_t nvec = (uint32_t)(n / VE);
   // bf16 accumulators are 8 floats per vector: fewer vectors per source
   // keep the kernel within 128 registers (2 CTAs/SM) without spills
-  if (nsrc == 1) copy_vec<DT, ADAPCC_COPY_UNROLL>(sh, ndst, nvec);
+  if (sh.any_acc) fold_acc_vec<DT, 4, 8>(sh, nsrc, ndst, nvec);
+  else if (nsrc == 1) copy_vec<DT, ADAPCC_COPY_UNROLL>(sh, ndst, nvec);
   else if (nsrc <= 4) fold_vec<DT, (DT == kBF16 ? 1 : 2), 4>(sh, nsrc, ndst, nvec);
   else fold_vec<DT, 1, 8>(sh, nsrc, ndst, nvec);
   if ((uint64_t)nvec * VE < n) fold_scalar<DT>(sh, nsrc, ndst, (uint64_t)nvec * VE, n);

@@ -89,6 +89,35 @@ struct Item {
 };
 static_assert(sizeof(Item) == 16, "Item layout");
 
+// Flat kernel (engine_flat.cu) descriptor blob, built at plan time: one
+// FlatTask per task, then every task's refs (sources, then destinations) with
+// the task's range start folded into BufRef::bias and the task's index in
+// BufRef::pad[0..1].
+struct FlatTask {
+  uint64_t len;      // elements of the task
+  uint64_t vstart;   // set on the device: first index of the task's vectors in the launch's vector space
+  uint32_t ref0;     // its first ref in the blob's ref array
+  uint16_t nsrc, ndst;
+  uint16_t op, owner;
+  uint8_t any_acc;   // some destination accumulates (recv += result)
+  uint8_t bad;       // set on the device: some stream is not 16-byte aligned
+  uint8_t pad[2];
+};
+static_assert(sizeof(FlatTask) == 32, "FlatTask layout");
+constexpr uint32_t kFlatMaxRefs = 1536;  // per segment (shared memory: blob + pointers + flags < 48 KiB)
+constexpr uint32_t kFlatMaxTasks = 128;
+#ifdef __CUDACC__
+__host__ __device__
+#endif
+inline uint32_t flat_nrefs(uint32_t words, uint32_t ntasks) { return words - 2 * ntasks; }
+#ifdef __CUDACC__
+__host__ __device__
+#endif
+inline size_t flat_smem_bytes(uint32_t words, uint32_t ntasks) {
+  const uint32_t nrefs = flat_nrefs(words, ntasks);
+  return ((size_t)words * 16 + (size_t)nrefs * 9 + 15) / 16 * 16;
+}
+
 // STAGED late join: per-chunk decision words (8 bytes each) sit just before
 // the slot they describe, in an array of late_dec_bytes(nchunks) bytes
 #ifdef __CUDACC__

@@ -49,6 +49,7 @@ struct LaunchCore {
   const FlagRef* flags;
   const Item* items;
   uint32_t nitems;
+  uint32_t ntasks;      // flat kernel: it strides through tasks[0 .. ntasks) (no items)
   // LDG kernel: CTA b < nfirst reads its first item (items[b]), that item's
   // task and refs as ONE blob of first_words 16-byte words at first + b *
   // first_words, loaded in a single round trip together with the epoch
@@ -156,6 +157,11 @@ int threads();
 cudaError_t occupancy(int dtype, int* blocks_per_sm);
 cudaError_t launch(const LaunchParams& p, int grid, cudaStream_t stream, bool pdl);
 }  // namespace tma_direct
+// engine_flat.cu: plans without flags or arena streams -- the whole grid
+// strides through one task after another
+namespace flat {
+cudaError_t launch(const LaunchParams& p, int grid, cudaStream_t stream, bool pdl);
+}  // namespace flat
 namespace tma_staged {
 int threads();
 cudaError_t occupancy(int dtype, int* blocks_per_sm);

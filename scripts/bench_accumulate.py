@@ -44,6 +44,18 @@ def main():
         os.environ["ADAPCC_TMA_SHAPE"] = shape
         c = pkg.Communicator.loopback(n, mode="direct", scratch_bytes=64 << 20)
         c.config("acc_red", 1 if kind == "red" else 0)
+        if kind == "ldg":
+            c.config("engine", 0)
+        if "@" in kind:                # red@96: grid capped at 96 CTAs
+            kind, cap = kind.split("@")
+            c.config("max_ctas", int(cap))
+        if kind.endswith("nopdl"):
+            c.config("pdl", 0)
+            kind = kind[:-5]
+        if kind.startswith("flat"):   # flat kernel, optional CTAs per SM: flat6 = 6 per SM
+            c.config("engine", 3)
+            if kind[4:]:
+                c.config("flat_ctas", int(kind[4:]))
         c.set_strategy("allreduce", G.allreduce_stars(n))
         comms[v] = c
     os.environ.pop("ADAPCC_TMA_SHAPE", None)

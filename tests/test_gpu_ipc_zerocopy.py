@@ -104,7 +104,7 @@ def _worker(rank, n, port, engine, q):
         q.put((rank, False, traceback.format_exc() + repr(e)))
 
 
-@pytest.mark.parametrize("engine", [0, 1])
+@pytest.mark.parametrize("engine", [0, 1, 3])
 @pytest.mark.parametrize("n", [2, 3])
 def test_zero_copy_one_gpu(n, engine):
     if not torch.cuda.is_available():
@@ -162,7 +162,7 @@ def _big_worker(rank, n, port, mib, q):
             x = to_dev(xs[rank], dtype)
             y = torch.empty_like(x)
             rx, ry = comm.register(x), comm.register(y)
-            for engine, path in ((1, "zc"), (0, "zc"), (2, "staged")):
+            for engine, path in ((1, "zc"), (0, "zc"), (3, "zc"), (2, "staged")):
                 comm.config("engine", engine)
                 y.view(torch.uint8).fill_(0x5A)
                 if path == "zc":

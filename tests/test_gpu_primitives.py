@@ -15,7 +15,7 @@ from tests.gpu_util import bits, to_dev, to_host  # noqa: E402
 
 pytestmark = pytest.mark.gpu
 MODES = ["direct", "staged"]
-ENGINES = [0, 1]
+ENGINES = [0, 1, 3]   # 0: LDG/STG fold kernel, 1: TMA bulk-copy pipeline kernel, 3: flat (flag-free plans; others fall back)
 
 
 @pytest.fixture(autouse=True)
