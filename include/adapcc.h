@@ -398,8 +398,13 @@ ADAPCC_API const char* adapcc_last_cuda_error(void);
 
 /* Runtime knobs.  key: "timeout_ms" (watchdog, default 10000; env
  * ADAPCC_TIMEOUT_MS), "max_ctas" (grid cap, 0 = #SMs x occupancy; env
- * ADAPCC_NCTAS; a change empties the plan cache, since pieces are sized for the grid), "engine" (2 = auto by call size, default; 1 = TMA bulk-copy
- * pipeline; 0 = 128-bit LDG/STG fold; env ADAPCC_ENGINE), "piece_kib" (traffic per work
+ * ADAPCC_NCTAS; a change empties the plan cache, since pieces are sized for the grid), "engine" (2 = auto by call size, default:
+ * the LDG fold below 128 MiB of traffic per launch, the TMA pipeline above, and ACCUMULATE plans
+ * without flags or arena streams under 32 MiB the flat kernel; 1 = TMA bulk-copy pipeline; 0 = 128-bit
+ * LDG/STG fold; 3 = flat kernel for every plan without flags, arena streams, late join or NVLS
+ * (others keep the auto choice): the whole grid strides through all tasks' vectors, no work items;
+ * env ADAPCC_ENGINE), "flat_ctas" (flat kernel grid: CTAs per SM, 1..64, default 2 = resident;
+ * env ADAPCC_FLAT_CTAS), "piece_kib" (traffic per work
  * piece of flag-free tasks, 0 = automatic, default; env ADAPCC_PIECE_KIB), "taper" (the last
  * ~2 x grid flag-free items are cut into this many sub-pieces, 0..64; 0 = automatic,
  * default: halve those of >= 384 KiB of traffic; 1 = off;
@@ -447,7 +452,7 @@ ADAPCC_API adapcc_result_t adapcc_trace_read(adapcc_comm_t comm, void* records, 
 
 /* Number of engine kernel launches this communicator has issued. */
 ADAPCC_API adapcc_result_t adapcc_launch_count(adapcc_comm_t comm, uint64_t* count);
-/* Kernel of the most recent launch: 0 = LDG/STG fold, 1 = TMA pipeline, -1 = none. */
+/* Kernel of the most recent launch: 0 = LDG/STG fold, 1 = TMA pipeline, 3 = flat kernel, -1 = none. */
 ADAPCC_API adapcc_result_t adapcc_last_engine(adapcc_comm_t comm, int* engine);
 
 /* ------------------------------------------------- host-only inspection ---

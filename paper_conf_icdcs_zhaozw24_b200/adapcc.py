@@ -475,7 +475,7 @@ class Communicator:
         return buf[:n.value].copy(), tot.value
 
     def last_engine(self):
-        """Kernel of the most recent launch: 0 LDG/STG fold, 1 TMA pipeline."""
+        """Kernel of the most recent launch: 0 LDG/STG fold, 1 TMA pipeline, 3 flat kernel."""
         v = ctypes.c_int()
         _check(_load().adapcc_last_engine(self._h, ctypes.byref(v)), "last_engine")
         return v.value
