@@ -181,17 +181,25 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) flat_kernel(const __grid
   __syncthreads();
   pdl_trigger();
   pdl_wait();
-  // the epoch, counters and user buffers belong to the stream order
-  if (threadIdx.x == 0) {
-    const uint64_t e = *reinterpret_cast<volatile unsigned long long*>(&P.state->epoch) + 1;
-    sh.epoch = e;
-    if (blockIdx.x == 0) {  // re-arm the other parity's counters for the next launch
-      P.state->work[(e + 1) & 1] = 0;
-      P.state->done[(e + 1) & 1] = 0;
+  // The epoch, counters and user buffers belong to the stream order.  In
+  // loopback the epoch only counts this launch done at the end, so its load
+  // stays in flight during the fold (no round trip and barrier up front);
+  // across processes the start checks below need it first.
+  uint64_t e_lazy = 0;
+  if (!P.ipc) {
+    if (threadIdx.x == 0) e_lazy = *reinterpret_cast<volatile unsigned long long*>(&P.state->epoch) + 1;
+  } else {
+    if (threadIdx.x == 0) {
+      const uint64_t e = *reinterpret_cast<volatile unsigned long long*>(&P.state->epoch) + 1;
+      sh.epoch = e;
+      if (blockIdx.x == 0) {  // re-arm the other parity's counters for the next launch
+        P.state->work[(e + 1) & 1] = 0;
+        P.state->done[(e + 1) & 1] = 0;
+      }
     }
+    __syncthreads();
   }
-  __syncthreads();
-  const uint64_t epoch = sh.epoch;
+  const uint64_t epoch = P.ipc ? sh.epoch : 0;  // (loopback: e_lazy, thread 0, at the end)
   if (P.ipc && epoch > 2) {  // peers done with the call before last (same start check as the engines)
     const int r = threadIdx.x;
     if (r < P.nranks && r != P.my_rank && ((P.members >> r) & 1))
@@ -246,9 +254,14 @@ __global__ void __launch_bounds__(kThreads, kMinBlocks) flat_kernel(const __grid
     // data; in loopback only the next launch reads anything, after this grid
     // has completed
     if (P.ipc) fence(true);
-    const unsigned done = atomicAdd(&P.state->done[epoch & 1], 1u);
+    const uint64_t ep = P.ipc ? epoch : e_lazy;
+    if (!P.ipc && blockIdx.x == 0) {  // re-arm the other parity's counters for the next launch
+      P.state->work[(ep + 1) & 1] = 0;
+      P.state->done[(ep + 1) & 1] = 0;
+    }
+    const unsigned done = atomicAdd(&P.state->done[ep & 1], 1u);
     if (done == gridDim.x - 1) {
-      *reinterpret_cast<volatile unsigned long long*>(&P.state->epoch) = epoch;
+      *reinterpret_cast<volatile unsigned long long*>(&P.state->epoch) = ep;
       if (P.ipc) {
         __threadfence_system();
         st_release(reinterpret_cast<uint64_t*>(P.hdr[P.my_rank]), epoch, true);
