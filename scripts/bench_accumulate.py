@@ -46,6 +46,9 @@ def main():
         c.config("acc_red", 1 if kind == "red" else 0)
         if kind == "ldg":
             c.config("engine", 0)
+        while "+" in kind:             # red+t4+p128: taper 4, piece_kib 128
+            kind, opt = kind.rsplit("+", 1)
+            c.config({"t": "taper", "p": "piece_kib"}[opt[0]], int(opt[1:]))
         if "@" in kind:                # red@96: grid capped at 96 CTAs
             kind, cap = kind.split("@")
             c.config("max_ctas", int(cap))

@@ -87,6 +87,7 @@ def main():
     ap.add_argument("--accumulate-ready", default=None,
                     help="allreduce as phase 2: comma-separated ready ranks, recv += sum (ACCUMULATE)")
     ap.add_argument("--out", default=os.path.join(ROOT, "gpurun_out", "trace"))
+    ap.add_argument("--raw", action="store_true", help="also save every record (<out>_raw.npy)")
     a = ap.parse_args()
     import torch
 
@@ -130,6 +131,9 @@ def main():
     os.makedirs(os.path.dirname(a.out) or ".", exist_ok=True)
     json.dump(out, open(a.out + ".json", "w"), indent=1)
     json.dump(timeline(recs, med["launch"]), open(a.out + "_timeline.json", "w"))
+    if a.raw:
+        import numpy as np
+        np.save(a.out + "_raw.npy", recs)
     print(json.dumps(out))
 
 
