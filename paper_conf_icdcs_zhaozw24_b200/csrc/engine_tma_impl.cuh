@@ -47,7 +47,7 @@ constexpr uint32_t kStageBytes = ADAPCC_TMA_STAGE_KB * 1024;
 // K = 2, 3: > 16 KiB) exist only with stages above 32 KiB.
 constexpr bool kLargeTiles = kStageBytes > 32 * 1024;
 constexpr int kMaxKS = (kStageBytes / 4096) < 8 ? (int)(kStageBytes / 4096) : 8;  // sources per stage
-constexpr int kQ = 2;           // item queue depth (4 measured: no change, r02)
+constexpr int kQ = 2;           // item queue depth
 #ifndef ADAPCC_FOLD_TMA
 #define ADAPCC_FOLD_TMA 1        // K >= 2 folds stored by TMA bulk stores from shared memory
 #endif
@@ -91,7 +91,7 @@ struct Smem {
   uint64_t qempty[kQ];
   uint64_t epoch;
   int abort;
-  int prev_stage;  // consumer tid 0: see flush_prev
+  int pad;
   ItemDesc q[kQ];
   uint4 blob[kFirstMaxWords];  // this CTA's first item: Item | Task | refs (plan-time blob)
 };
@@ -287,8 +287,9 @@ __device__ __forceinline__ void consume_copy(Smem& sm, char* stages, const ItemD
 // Other consumer threads only advance their ring position.
 template <int DT>
 __device__ __forceinline__ void copy_tma(Smem& sm, char* stages, const ItemDesc& d, int tid,
-                                         uint32_t& stage, uint32_t& sphase, int& prev) {
+                                         uint32_t& stage, uint32_t& sphase) {
   if (tid == 0) {
+    int prev = -1;
     for (uint32_t t = 0; t < d.ntiles; ++t) {
       const uint32_t tb = min(d.tile, d.vec_bytes - t * d.tile);
       mbar_wait(&sm.full[stage], sphase);
@@ -302,24 +303,14 @@ __device__ __forceinline__ void copy_tma(Smem& sm, char* stages, const ItemDesc&
       prev = (int)stage;
       if (++stage == kStages) { stage = 0; sphase ^= 1; }
     }
+    if (prev >= 0) {
+      tma_store_wait_read<0>();
+      mbar_arrive_cnt(&sm.empty[prev], kConsumerWarps);
+    }
   } else {
     const uint32_t total = stage + d.ntiles;
     sphase ^= (total / kStages) & 1;
     stage = total % kStages;
-  }
-}
-
-// The bulk-store paths (copy_tma, consume_fold_tma, consume_acc_tma) release
-// a stage once the bulk stores issued from it have read it: tid 0 keeps the
-// last such stage in `prev` ACROSS items and releases it when it commits the
-// next stage's stores, so an item boundary costs no drain (draining at every
-// item end stalled the consumers for the last tile's reads, ~1-2 us per item).
-// Paths that release stages themselves, flag posts, and the CTA's exit flush it.
-__device__ __forceinline__ void flush_prev(Smem& sm, int tid, int& prev) {
-  if (tid == 0 && prev >= 0) {
-    tma_store_wait_read<0>();
-    mbar_arrive_cnt(&sm.empty[prev], kConsumerWarps);
-    prev = -1;
   }
 }
 
@@ -331,12 +322,13 @@ __device__ __forceinline__ void flush_prev(Smem& sm, int tid, int& prev) {
 // destination's tile.  No consumer global load or store is left.
 template <int DT>
 __device__ __forceinline__ void consume_acc_tma(Smem& sm, char* stages, const ItemDesc& d, int tid,
-                                                uint32_t& stage, uint32_t& sphase, int& prev) {
+                                                uint32_t& stage, uint32_t& sphase) {
   using O = Ops<DT>;
   const uint32_t tile = d.tile;
   const int ks = d.nsrc, ndst = d.ndst;
   bool plain = false;
   for (int k = 0; k < ndst; ++k) plain |= !d.acc[k];
+  int prev = -1;  // tid 0: the stage whose bulk stores may still be reading it
   for (uint32_t t = 0; t < d.ntiles; ++t) {
     const uint32_t tb = min(tile, d.vec_bytes - t * tile);
     const uint32_t nv = tb / 16;
@@ -375,6 +367,10 @@ __device__ __forceinline__ void consume_acc_tma(Smem& sm, char* stages, const It
     }
     if (++stage == kStages) { stage = 0; sphase ^= 1; }
   }
+  if (tid == 0 && prev >= 0) {
+    tma_store_wait_read<0>();
+    mbar_arrive_cnt(&sm.empty[prev], kConsumerWarps);
+  }
 }
 
 // Fold the tiles of a K >= 2 item whose destinations are all plain stores
@@ -385,10 +381,11 @@ __device__ __forceinline__ void consume_acc_tma(Smem& sm, char* stages, const It
 // all; a stage is released once its bulk stores have read it.
 template <int DT>
 __device__ __forceinline__ void consume_fold_tma(Smem& sm, char* stages, const ItemDesc& d, int tid,
-                                                 uint32_t& stage, uint32_t& sphase, int& prev) {
+                                                 uint32_t& stage, uint32_t& sphase) {
   using O = Ops<DT>;
   const uint32_t tile = d.tile, vec_bytes = d.vec_bytes, ntiles = d.ntiles;
   const int ks = d.nsrc, ndst = d.ndst;
+  int prev = -1;  // tid 0: the stage whose bulk stores may still be reading it
   for (uint32_t t = 0; t < ntiles; ++t) {
     const uint32_t tb = min(tile, vec_bytes - t * tile);
     const uint32_t nv = tb / 16;
@@ -413,6 +410,10 @@ __device__ __forceinline__ void consume_fold_tma(Smem& sm, char* stages, const I
       prev = (int)stage;
     }
     if (++stage == kStages) { stage = 0; sphase ^= 1; }
+  }
+  if (tid == 0 && prev >= 0) {
+    tma_store_wait_read<0>();
+    mbar_arrive_cnt(&sm.empty[prev], kConsumerWarps);
   }
 }
 
@@ -884,10 +885,6 @@ engine_tma_kernel(const __grid_constant__ LaunchParamsT<NR> P) {
   } else {
     // =============================================================== consumers
     uint32_t stage = 0, sphase = 0, qi = 0, qphase = 0;
-    // tid 0: the last stage whose bulk stores may still be reading it (flush_prev); in
-    // shared memory, not a register held across the item loop
-    int& prev = sm.prev_stage;
-    if (tid == 0) prev = -1;
     for (;;) {
       mbar_wait(&sm.qfull[qi], qphase);
       const ItemDesc& d = sm.q[qi];
@@ -900,17 +897,16 @@ engine_tma_kernel(const __grid_constant__ LaunchParamsT<NR> P) {
         } else if (d.op != kOpNone) {
           if (!d.scalar_only) {
             const uint32_t vpt = d.tile / (16u * kConsumers);  // tile / one round of 1 vector per thread
-            if (d.acc_tma) consume_acc_tma<DT>(sm, stages, d, tid, stage, sphase, prev);
-            else if (d.nsrc == 1 && (!d.any_acc || d.acc_red)) copy_tma<DT>(sm, stages, d, tid, stage, sphase, prev);
-            else if (d.acc_red) consume_fold_tma<DT>(sm, stages, d, tid, stage, sphase, prev);
+            if (d.acc_tma) consume_acc_tma<DT>(sm, stages, d, tid, stage, sphase);
+            else if (d.nsrc == 1 && (!d.any_acc || d.acc_red)) copy_tma<DT>(sm, stages, d, tid, stage, sphase);
+            else if (d.acc_red) consume_fold_tma<DT>(sm, stages, d, tid, stage, sphase);
             // TMA-stored fold where per-thread stores are the cost: tiles above 16 KiB (K = 2, 3 in
             // 64 KiB stages, else fold_rounds; G1 k = 2: 0.86 -> 1.02 of the copy peak) or >= 3
             // destinations (star roots); with 1-2 destinations of small tiles the register path,
             // which frees the stage before storing, is as fast or faster (G1 k = 8: 1.08 vs 1.04)
             else if (kFoldTma && !d.any_acc && d.passes == 1 && (d.tile > 16384 || d.ndst >= 3))
-              consume_fold_tma<DT>(sm, stages, d, tid, stage, sphase, prev);
+              consume_fold_tma<DT>(sm, stages, d, tid, stage, sphase);
             else if (d.nsrc == 1) {
-              flush_prev(sm, tid, prev);  // (the register paths release their stages themselves)
               // (32 KiB stages: the 8-vector register round of consume_copy set the whole
               // kernel's register budget and made it spill at 2 CTAs/SM -- 96 registers)
               if constexpr (kLargeTiles) consume_copy<DT, 8>(sm, stages, d, tid, stage, sphase);
@@ -918,28 +914,20 @@ engine_tma_kernel(const __grid_constant__ LaunchParamsT<NR> P) {
             }
             else if (vpt >= 4) {
               if constexpr (DT == kBF16) {  // 4 x 8 fp32 accumulators per thread spill at 2 CTAs/SM
-                if (!d.any_acc) {
-                  consume_fold_tma<DT>(sm, stages, d, tid, stage, sphase, prev);
-                } else {
-                  flush_prev(sm, tid, prev);
-                  consume_fold_held<DT>(sm, stages, d, tid, stage, sphase);
-                }
+                if (!d.any_acc) consume_fold_tma<DT>(sm, stages, d, tid, stage, sphase);
+                else consume_fold_held<DT>(sm, stages, d, tid, stage, sphase);
               } else {
-                flush_prev(sm, tid, prev);
                 consume_fold<DT, 4>(sm, stages, d, tid, stage, sphase);
               }
-            } else {
-              flush_prev(sm, tid, prev);
-              if (vpt >= 2) consume_fold<DT, 2>(sm, stages, d, tid, stage, sphase);
-              else consume_fold<DT, 1>(sm, stages, d, tid, stage, sphase);
             }
+            else if (vpt >= 2) consume_fold<DT, 2>(sm, stages, d, tid, stage, sphase);
+            else consume_fold<DT, 1>(sm, stages, d, tid, stage, sphase);
           }
           constexpr int esize = Ops<DT>::kEsize;
           scalar_range<DT>(d, d.vec_bytes / esize, d.len, tid);
         }
         consumer_sync();  // every consumer's stores for this item are issued
         if (tid == 0 && d.npost) {
-          flush_prev(sm, tid, prev);
           tma_store_wait_all();  // bulk (async-proxy) stores performed ...
           fence_proxy_async();   // ... and ordered before generic-proxy accesses
           for (int k = 0; k < d.ndec; ++k)  // STAGED late join: the decision travels with the flag
@@ -954,7 +942,6 @@ engine_tma_kernel(const __grid_constant__ LaunchParamsT<NR> P) {
       if (tid == 0) mbar_arrive(&sm.qempty[qi]);
       if (++qi == kQ) { qi = 0; qphase ^= 1; }
     }
-    flush_prev(sm, tid, prev);
   }
   __syncthreads();
   if (P.trace && tid == 0) trace_put(P, kTraceCta, 0, t_entry, t_ready, globaltimer(), 0);
