@@ -34,7 +34,8 @@ METRIC = "AllReduce busbw GB/s vs size at 2/4/8 B200 (% of 900 GB/s) vs NCCL"
 UNIT = "GB/s"
 NVLINK_NOMINAL = 900.0
 ENGINE_NAMES = {0: "adapcc::engine_kernel (128-bit LDG/STG fold)",
-                1: "adapcc::{ns}::engine_tma_kernel (TMA bulk-copy pipeline)"}
+                1: "adapcc::{ns}::engine_tma_kernel (TMA bulk-copy pipeline)",
+                3: "adapcc::flat::flat_kernel (grid-stride over flag-free tasks)"}
 
 
 def engine_name(engine, mode, dtype):
@@ -401,6 +402,32 @@ def run_single(args):
                           "busbw_graph": round(busbw(sb, msg_ / 1e3, n), 2),
                           "hbm_frac_graph": round(2 * n * sb / (msg_ / 1e3) / 1e9 / peak, 4)})
         assert comm.get_async_error() == 0
+    partial = None
+    if not args.no_sweep and n == 8:
+        # C3 (BASELINE configs[2]): partial aggregation with 2 stragglers out of 8 acting as relays, at
+        # the gradient-bucket sizes -- phase 1 = the AllReduce of the 6 ready ranks (mask 0xB7, every rank
+        # receives; traffic 6 S read + 8 S written), phase 2 = ACCUMULATE of the 2 late ranks (mask 0x48,
+        # recv += sum; 2 S read + 8 S read and written).  Graph-timed on slices of the bench buffers.
+        partial = []
+        R1, R2 = {0, 1, 2, 4, 5, 7}, {3, 6}
+        for mib in (16, 25, 64, 100):
+            sb = (mib << 20) // 16 * 16
+            if sb > nbytes:
+                continue
+            c = sb // es
+            ys_ = [t[:c] for t in dy]
+            x1 = [t[:c] if r in R1 else None for r, t in enumerate(dx)]
+            x2 = [t[:c] if r in R2 else None for r, t in enumerate(dx)]
+            _, m1 = time_point(lambda: comm.allreduce_lb(x1, ys_, ready=R1))
+            e1 = comm.last_engine()
+            _, m2 = time_point(lambda: comm.allreduce_lb(x2, ys_, ready=R2, accumulate=True))
+            e2 = comm.last_engine()
+            partial.append({"mib_per_rank": mib,
+                            "phase1_us": round(m1 * 1e3, 2), "phase1_hbm_frac": round(14 * sb / (m1 / 1e3) / 1e9 / peak, 4),
+                            "phase1_kernel": engine_name(e1, args.mode, args.dtype),
+                            "phase2_us": round(m2 * 1e3, 2), "phase2_hbm_frac": round(18 * sb / (m2 / 1e3) / 1e9 / peak, 4),
+                            "phase2_kernel": engine_name(e2, args.mode, args.dtype)})
+        assert comm.get_async_error() == 0
     alg_bytes = 2 * n * nbytes   # every rank's input read once + output written once
     achieved = alg_bytes / (kern_ms / 1e3) / 1e9
     out = {
@@ -431,6 +458,11 @@ def run_single(args):
         "nccl": None,
         "paper_context": PAPER_CONTEXT,
         "sweep": sweep,
+        "partial_aggregation": partial,
+        "partial_aggregation_how": "C3 shapes on this bench's buffers, CUDA graph of back-to-back calls: phase 1 "
+                                   "= AllReduce over ready ranks {0,1,2,4,5,7} (relays 3, 6 receive), roofline "
+                                   "traffic 14 S; phase 2 = ACCUMULATE of ranks {3,6} into every recvbuf, 18 S; "
+                                   "fractions of the measured HBM copy peak (parity: tests/test_gpu_fullsize.py)",
         "sweep_how": "same call at every x4 size (slices of the bench buffers): back-to-back enqueue of a "
                      "prepared call (us: Communicator.prepare_allreduce_lb, one C call per AllReduce), of the "
                      "per-call API (us_api: allreduce_lb marshals its arguments every call), and a CUDA graph "
