@@ -104,7 +104,7 @@ def _worker(rank, n, port, engine, q):
         q.put((rank, False, traceback.format_exc() + repr(e)))
 
 
-@pytest.mark.parametrize("engine", [0, 1, 3])
+@pytest.mark.parametrize("engine", [0, 1, 2, 3])
 @pytest.mark.parametrize("n", [2, 3])
 def test_zero_copy_one_gpu(n, engine):
     if not torch.cuda.is_available():

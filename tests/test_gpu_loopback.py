@@ -120,10 +120,11 @@ def test_c1_config_bit_exact(mode, engine):
 @pytest.mark.parametrize("acc_red", [1, 0])
 @pytest.mark.parametrize("mode", MODES)
 @pytest.mark.parametrize("dtype", ["f32", "bf16", "i32"])
-@pytest.mark.parametrize("engine", ENGINES)
+@pytest.mark.parametrize("engine", ENGINES + [2])
 def test_phase1_phase2_accumulate(mode, dtype, engine, acc_red):
     """C3 shape (reduced): stragglers {3,6} relay in phase 1, join with ACCUMULATE
-    (TMA kernel: bulk reduce-add into recv, or the shared-memory read-modify-write)."""
+    (TMA kernel: bulk reduce-add into recv, or the shared-memory read-modify-write;
+    engine 2 = auto: this small DIRECT phase 2 runs on the flat kernel)."""
     n, count = 8, 65_537
     R1, R2 = {0, 1, 2, 4, 5, 7}, {3, 6}
     xs = rank_tensors(dtype, count, n)
@@ -139,6 +140,8 @@ def test_phase1_phase2_accumulate(mode, dtype, engine, acc_red):
     y2 = _run_allreduce(comm, [x if r in R2 else None for r, x in enumerate(xs)], dtype, R2,
                         accumulate=True, prev=y1)
     _assert_bits(y2, oc.allreduce(xs, t2, R2, dtype, accumulate=True, y_prev=e1), "phase2")
+    if engine == 2 and mode == "direct":
+        assert comm.last_engine() == 3   # auto: small flag-free ACCUMULATE -> flat kernel
     comm.finalize()
 
 
