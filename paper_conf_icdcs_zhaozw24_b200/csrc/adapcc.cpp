@@ -523,7 +523,8 @@ adapcc_result_t get_plan(adapcc_comm_s* c, Coll coll, const Strategy* strat, uin
     // (the flat kernel runs tasks, not items: the items only count the work)
     const bool flat = plan->kernel == 3;
     std::vector<Item> items = order_items(sp, c->loopback ? -1 : c->rank, rq.esize, grid_size(c, dtype, flat ? 0 : plan->kernel),
-                                          (uint64_t)c->piece_kib * 1024, (int)c->taper, plan->kernel != 0);
+                                          (uint64_t)c->piece_kib * 1024, (int)c->taper, plan->kernel != 0,
+                                          plan->kernel == 1 && rq.accumulate && c->acc_red);
     d.nitems = (uint32_t)items.size();
     d.arena_free = 1;
     for (const Task& t : sp.tasks) {

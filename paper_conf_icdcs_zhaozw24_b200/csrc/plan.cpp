@@ -712,7 +712,7 @@ bool build_plan(const PlanRequest& rq, std::vector<SegmentPlan>* segs, std::stri
 }
 
 std::vector<Item> order_items(const SegmentPlan& p, int rank, int esize, int grid,
-                              uint64_t piece_bytes, int taper, bool tma) {
+                              uint64_t piece_bytes, int taper, bool tma, bool acc_red) {
   // Work balance: tasks that post no flags are cut into pieces of roughly
   // equal traffic.
   // streams of a task: sources + destinations, an accumulating destination
@@ -734,7 +734,10 @@ std::vector<Item> order_items(const SegmentPlan& p, int rank, int esize, int gri
   // with the most items does (8 MiB per rank, TMA: 1.7 items per CTA left half
   // the grid idle for a whole item at the end).
   const uint64_t g = (uint64_t)std::max(grid, 1);
-  const uint64_t cap = 512 * 1024, floor_bytes = tma ? 256 * 1024 : 16 * 1024;
+  // Phase 2 by bulk reduce-adds (acc_red) streams best at ~256 KiB per item
+  // (16 / 25 / 64 / 100 / 256 MiB per rank: +0.2 / +1.0 / +1.5 / +1.5 / +1.3 %
+  // with the taper below, profiles/acc_pieces_r02.json)
+  const uint64_t cap = acc_red ? 256 * 1024 : 512 * 1024, floor_bytes = tma ? 256 * 1024 : 16 * 1024;
   const uint64_t m = std::max<uint64_t>(1, (total + g * cap - 1) / (g * cap));
   const uint64_t target =
       piece_bytes ? piece_bytes : std::min<uint64_t>(std::max<uint64_t>(total / (m * g), floor_bytes), cap);
@@ -794,8 +797,9 @@ std::vector<Item> order_items(const SegmentPlan& p, int rank, int esize, int gri
   // rounds the last round is already even, and halving its items only adds
   // per-item overhead (8 MiB per rank, m = 2: 26.3 us tapered, 24.8 us not;
   // 16 MiB, m = 4: 46.0 vs 46.3 us, profiles/ab/taper_r01.txt).
-  const bool auto_taper = taper <= 0;
-  if (auto_taper) taper = (piece_bytes || m >= 3) ? 2 : 1;
+  bool auto_taper = taper <= 0;
+  if (auto_taper) taper = (piece_bytes || m >= 3 || acc_red) ? 2 : 1;
+  if (auto_taper && acc_red) auto_taper = false;  // (its 256 KiB items are all halved, whatever their size)
   std::vector<uint8_t> split(keys.size(), 0);
   if (taper > 1) {
     uint64_t want = 2ull * std::max(grid, 1);

@@ -75,8 +75,10 @@ bool build_plan(const PlanRequest& rq, std::vector<SegmentPlan>* segs, std::stri
 // taper: the last ~2 x grid splittable items (flag-free tasks) are cut into
 // `taper` sub-pieces each, so the dynamic claim loop ends on short items
 // (1 = off, 0 = automatic).
+// acc_red: items for the TMA kernel's bulk reduce-add ACCUMULATE path (phase 2):
+// automatic pieces of <= 256 KiB and an unconditional tail taper.
 std::vector<Item> order_items(const SegmentPlan& p, int rank, int esize, int grid,
-                              uint64_t piece_bytes = 0, int taper = 1, bool tma = false);
+                              uint64_t piece_bytes = 0, int taper = 1, bool tma = false, bool acc_red = false);
 
 // Byte accounting for adapcc_plan_stats.
 void accumulate_stats(const SegmentPlan& p, int rank, int esize, PlanStats* s);

@@ -43,7 +43,8 @@ def main():
         kind, shape = v.split(":")
         os.environ["ADAPCC_TMA_SHAPE"] = shape
         c = pkg.Communicator.loopback(n, mode="direct", scratch_bytes=64 << 20)
-        c.config("acc_red", 1 if kind == "red" else 0)
+        # (the base kind decides acc_red: "red" and its modified forms red+t4, red@96, rednopdl, ...)
+        c.config("acc_red", 1 if kind.startswith("red") else 0)
         if kind == "ldg":
             c.config("engine", 0)
         while "+" in kind:             # red+t4+p128: taper 4, piece_kib 128
