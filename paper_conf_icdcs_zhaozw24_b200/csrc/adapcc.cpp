@@ -1773,6 +1773,14 @@ adapcc_result_t adapcc_exclude(adapcc_comm_t c, uint64_t dead_mask, adapcc_boots
   }
   *reinterpret_cast<volatile int*>(c->h_err) = 0;
   c->members = live;
+  // After an exclusion every launch also runs the start barrier of the debug
+  // call check (check_call_sig: every survivor's kernel of this epoch has
+  // started -- and makes the same call -- before any byte moves).  Without it
+  // a 3-process test on one GPU corrupted a tree's last chunk in ~15 % of
+  // runs after the exclusion (root cause not isolated; the barrier removes
+  // it: 0 of 16, profiles/fault_race_r02.json).  Costs one header round trip
+  // per launch, in the degraded post-fault mode only.
+  if (!c->loopback) c->check_sig = 1;
   // 4. strategies: the survivors' defaults until set_strategy names new ones
   for (int k = 0; k < kNumColl; ++k) {
     if (!parse_strategy(default_strategy((Coll)k, c->nranks, 0, live, c->default_chunk).c_str(), &c->strat[k], nullptr))

@@ -264,11 +264,18 @@ def _fault_worker(rank, n, port, q):
         live = set(range(n)) - {dead}
         exp = oc.allreduce_exact([xs[g] for g in sorted(live)], set(range(n - 1)), "i32")
         ok = [res["faulty"] == [dead]]
+        if os.environ.get("FAULT_TEST_WAIT_DEAD"):   # (diagnostic: the survivors start only once the dead rank's kernel ended)
+            if rank == dead:
+                store.set("fault-test/dead-idle", b"1")
+            else:
+                store.wait(["fault-test/dead-idle"])
         if rank == dead:                      # excluded: stays alive (its arena is mapped) until the survivors finish
             store.wait(["fault-test/done"])
         else:
             ok.append(comm.members == live)
             ok.append(np.array_equal(to_host(y, "i32"), exp))
+            if os.environ.get("FAULT_TEST_TRACE"):
+                comm.config("trace", 1 << 16)
             for _ in range(2):                # the survivors carry on: a full round
                 y.zero_()
                 torch.cuda.synchronize()      # (the collectives run on cs)
@@ -276,11 +283,29 @@ def _fault_worker(rank, n, port, q):
                 comm.signal_ready(ticket=t, stream=cs)
                 res = coord.allreduce(lambda m, lt: comm.allreduce(x, y, ready=m, late=lt, stream=cs))
                 torch.cuda.synchronize()
-                ok.append((res["faulty"], np.array_equal(to_host(y, "i32"), exp)))
+                got = to_host(y, "i32")
+                good = np.array_equal(got, exp)
+                if not good:   # diagnostics: which elements, and what they hold instead
+                    bad = np.nonzero(got != exp)[0]
+                    x0, x1 = xs[0], xs[1]
+                    kinds = {"x0": int(np.sum(got[bad] == x0[bad])), "x1": int(np.sum(got[bad] == x1[bad])),
+                             "zero": int(np.sum(got[bad] == 0)),
+                             "sum+x2": int(np.sum(got[bad] == (exp[bad] + xs[2][bad]))),
+                             "2x": int(np.sum(got[bad] == 2 * exp[bad]))}
+                    good = (False, res, int(bad.size), int(bad[0]), int(bad[-1]), kinds)
+                    os.makedirs(os.path.join(ROOT, "gpurun_out"), exist_ok=True)
+                    if os.environ.get("FAULT_TEST_TRACE"):
+                        recs, tot = comm.trace()
+                        np.save(os.path.join(ROOT, "gpurun_out", f"fault_trace_r{rank}_{os.getpid()}.npy"), recs)
+                    with open(os.path.join(ROOT, "gpurun_out", f"fault_diag_r{rank}.txt"), "a") as f:
+                        f.write(repr(good) + "\n")
+                ok.append((res["faulty"], good))
+                if os.environ.get("FAULT_TEST_TRACE") and good is True:
+                    comm.trace()   # (drain: the next round's records start empty)
             if store.add("fault-test/finished", 1) == n - 1:
                 store.set("fault-test/done", b"1")
         err = comm.get_async_error()
-        good = all(o if isinstance(o, bool) else (o[0] == [] and o[1]) for o in ok)
+        good = all(o if isinstance(o, bool) else (o[0] == [] and o[1] is True) for o in ok)
         q.put((rank, err == 0 and good, f"{ok} err={err} res={res}"))
         comm.finalize()
     except Exception as e:  # noqa: BLE001
