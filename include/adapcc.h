@@ -382,7 +382,10 @@ ADAPCC_API adapcc_result_t adapcc_get_async_error(adapcc_comm_t comm);
  * (ascending rank order; ag may be NULL in loopback).  Host-blocking: waits for
  * this device to drain.  Precondition: the excluded ranks' GPU work has stopped
  * (their launches exit at the watchdog deadline).  CUDA graphs captured before
- * the call must not be replayed after it.  INVALID_ARGUMENT: bits >= nranks,
+ * the call must not be replayed after it.  Multi-process: every later launch
+ * also runs the debug call check's start barrier (all survivors' kernels of a
+ * launch have started and make the same call before any byte moves; see
+ * "debug_check" and DESIGN.md §12, known issue).  INVALID_ARGUMENT: bits >= nranks,
  * nothing left alive, or (multi-process) this rank excluded / ag NULL. */
 ADAPCC_API adapcc_result_t adapcc_exclude(adapcc_comm_t comm, uint64_t dead_mask,
                                adapcc_bootstrap_allgather_fn ag, void* ag_ctx);
