@@ -1760,7 +1760,7 @@ adapcc_result_t adapcc_exclude(adapcc_comm_t c, uint64_t dead_mask, adapcc_boots
     if (members_allgather(c, &epoch, e.data(), sizeof(uint64_t)) != 0) return ADAPCC_ERR_BOOTSTRAP;
     for (uint64_t v : e) epoch = std::max(epoch, v);
   }
-  epoch += 2;
+  epoch += (uint64_t)std::max<int64_t>(2, env_int("ADAPCC_EXCLUDE_GAP", 2));  // (diagnostic knob: the epoch gap)
   // 3. restart the device epoch there: counters cleared, abort latch released;
   //    this rank's "done" and "entered" words say it finished `epoch`, so the
   //    next launch's start check (peers done >= epoch + 1 - 2) passes
@@ -1780,7 +1780,7 @@ adapcc_result_t adapcc_exclude(adapcc_comm_t c, uint64_t dead_mask, adapcc_boots
   // runs after the exclusion (root cause not isolated; the barrier removes
   // it: 0 of 16, profiles/fault_race_r02.json).  Costs one header round trip
   // per launch, in the degraded post-fault mode only.
-  if (!c->loopback) c->check_sig = 1;
+  if (!c->loopback && env_int("ADAPCC_EXCLUDE_BARRIER", 1) != 0) c->check_sig = 1;  // (diagnostic knob)
   // 4. strategies: the survivors' defaults until set_strategy names new ones
   for (int k = 0; k < kNumColl; ++k) {
     if (!parse_strategy(default_strategy((Coll)k, c->nranks, 0, live, c->default_chunk).c_str(), &c->strat[k], nullptr))
